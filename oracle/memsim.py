@@ -1,0 +1,292 @@
+"""ORACLE (test infrastructure only): the arena event model = definition of
+"peak live bytes" for a (input size, plan) pair.
+
+Paper basis:
+  * P:75 (§III-A): the footprint is parameters + gradients + optimizer states
+    (constant in the input size) + activations (vary with the input size).
+  * P:140 (§IV-B): a dropped block keeps only its output / input between blocks;
+    the shuttling collector's footprint equals Sublinear's.
+  * P:177 (§IV-D, Fig. 9): checkpointing the LAST encoder gives a peak close to
+    no checkpointing, because its activations are restored at once in backward
+    while the others are still alive.
+  * P:51 (§II-A): activations are released as soon as their gradients are
+    derived.
+
+The tensor list and event order are DESIGN.md "Memory model" (reading R-D);
+every size is align16(bytes).  This module is written from that spec alone;
+the GPU arena is an independent implementation of the same spec and must
+report the same integers.
+
+Pinned by: closed forms P(empty)=C+E+(L-1)a+i+Tb, LB, peak({L})=peak(empty),
+peak(first k)=P(empty)-k*i, monotonicity in x (tests/test_oracle_planning.py).
+"""
+from __future__ import annotations
+
+import dataclasses
+from typing import Dict, List, Optional, Sequence
+
+from paper_conf_ipps_liaolysshfyctzlq23_b200.workload import (
+    HEAD_QA, ModelConfig, param_spec)
+
+
+def a16(n: int) -> int:
+    return (int(n) + 15) // 16 * 16
+
+
+def ebytes(cfg: ModelConfig) -> int:
+    return 4 if cfg.dtype == "fp32" else 2
+
+
+NPART = 296   # fixed count of deterministic reduction partials (DESIGN "Memory model")
+
+
+def persistent_bytes(cfg: ModelConfig, max_seqs: int, max_seq_len: int) -> int:
+    """C: weights (e), fp32 grads, fp32 master (bf16 only), AdamW m and v, batch
+    metadata buffers, misc, and the fixed backward workspaces."""
+    e = ebytes(cfg)
+    H, F = cfg.hidden, cfg.ffn
+    npad = sum((int(_prod(s)) + 63) // 64 * 64 for _, s in param_spec(cfg))
+    c = a16(npad * e) + a16(npad * 4) + a16(npad * 4) + a16(npad * 4)   # w, grad, m, v
+    if cfg.dtype != "fp32":
+        c += a16(npad * 4)                                               # master
+    maxT = max_seqs * max_seq_len
+    c += a16(maxT * 4) * 2 + a16(max_seqs * 4) + a16(2 * max_seqs * 4)  # ids, tt, lens, labels
+    c += a16(256)                                                        # misc scalars
+    c += a16(4 * H * H * 4)                                              # wgrad split-K workspace
+    c += a16(NPART * 2 * max(3 * H, F) * 4)                              # LN / bias partials
+    return c
+
+
+def _prod(s):
+    n = 1
+    for v in s:
+        n *= v
+    return n
+
+
+@dataclasses.dataclass(frozen=True)
+class Sizes:
+    """Byte sizes of every arena object for one input shape (B, S)."""
+    C: int
+    E: List[int]          # embedding-forward objects (z0, st0, x1)
+    internals: List[int]  # one layer's saved internals
+    y: int                # layer output
+    head: List[int]       # head-forward objects
+    dy: int               # backward gradient buffer
+    head_scratch: int
+    layer_scratch: int
+    emb_scratch: int
+    n_layers: int
+
+    @property
+    def i(self) -> int:
+        return sum(self.internals)
+
+    @property
+    def a(self) -> int:
+        return self.i + self.y
+
+    @property
+    def e(self) -> int:
+        return sum(self.E)
+
+    @property
+    def hd(self) -> int:
+        return sum(self.head)
+
+
+def sizes(cfg: ModelConfig, B: int, S: int, max_seqs: Optional[int] = None,
+          max_seq_len: Optional[int] = None) -> Sizes:
+    e = ebytes(cfg)
+    H, F, h = cfg.hidden, cfg.ffn, cfg.heads
+    T = B * S
+    ms = cfg.n_seqs if max_seqs is None else max_seqs
+    mx = cfg.max_seq if max_seq_len is None else max_seq_len
+    E = [a16(T * H * e), a16(T * 8), a16(T * H * e)]                       # z0, st0, x1
+    internals = [a16(T * 3 * H * e), a16(T * H * e), a16(B * h * S * 4),   # QKV, O, LSE
+                 a16(T * H * e), a16(T * 8), a16(T * H * e),               # z1, st1, h1
+                 a16(T * F * e), a16(T * F * e),                           # u, g
+                 a16(T * H * e), a16(T * 8)]                               # z2, st2
+    y = a16(T * H * e)
+    if cfg.head == HEAD_QA:
+        head = [a16(T * 2 * 4)]
+        head_scr = a16(T * 2 * 4)
+    else:
+        head = [a16(B * H * e), a16(B * cfg.n_out * 4)]                   # pooled, logits
+        head_scr = a16(B * cfg.n_out * 4) + a16(B * H * 4) * 2
+    dy = a16(T * H * 4)
+    layer_scr = a16(T * H * 4) + a16(T * F * e) + a16(T * 3 * H * e) + a16(B * h * S * 4)
+    ntiles = (ms * mx + 1023) // 1024
+    emb_scr = a16(T * H * 4) + a16(16 * T) + a16(4 * 256 * ntiles)   # dz0, 4 int32[T] sort arrays, digit histograms
+    return Sizes(persistent_bytes(cfg, ms, mx), E, internals, y, head, dy, head_scr,
+                 layer_scr, emb_scr, cfg.n_layers)
+
+
+# --------------------------------------------------------------------------
+# event-level simulator
+# --------------------------------------------------------------------------
+
+class Arena:
+    """Two-ended accounting: a LIFO stack (activations) and a LIFO top region
+    (transients).  live = C + stack + top.  Frees must be LIFO per region."""
+
+    def __init__(self, C: int):
+        self.C = C
+        self.stack: List[int] = []
+        self.top: List[int] = []
+        self.peak = C
+        self.timeline: List[int] = [C]
+        self.top_peak_phase = 0
+
+    @property
+    def live(self) -> int:
+        return self.C + sum(self.stack) + sum(self.top)
+
+    def _tick(self):
+        v = self.live
+        self.timeline.append(v)
+        self.peak = max(self.peak, v)
+        self.top_peak_phase = max(self.top_peak_phase, sum(self.top))
+
+    def push(self, n):
+        self.stack.append(n)
+        self._tick()
+
+    def pop(self, n):
+        assert self.stack and self.stack[-1] == n, "stack free out of LIFO order"
+        self.stack.pop()
+        self.timeline.append(self.live)
+
+    def talloc(self, n):
+        self.top.append(n)
+        self._tick()
+
+    def tfree(self, n):
+        assert self.top and self.top[-1] == n, "top free out of LIFO order"
+        self.top.pop()
+        self.timeline.append(self.live)
+
+
+def simulate_step(sz: Sizes, dropped: Sequence[int]) -> Arena:
+    """One training step (forward, backward) under a plan of dropped layers
+    (0-based).  Returns the arena with its peak and timeline."""
+    L = sz.n_layers
+    drop = set(dropped)
+    A = Arena(sz.C)
+    for t in sz.E:
+        A.push(t)
+    for l in range(L):                                   # forward
+        if l in drop:                                    # no-save: internals transient
+            for t in sz.internals:
+                A.talloc(t)
+            A.push(sz.y)
+            for t in reversed(sz.internals):
+                A.tfree(t)
+        else:
+            for t in sz.internals:
+                A.push(t)
+            A.push(sz.y)
+    for t in sz.head:
+        A.push(t)
+    A.talloc(sz.dy)                                      # backward
+    A.talloc(sz.head_scratch)
+    A.tfree(sz.head_scratch)
+    for t in reversed(sz.head):
+        A.pop(t)
+    A.pop(sz.y)                                          # y_L
+    for l in reversed(range(L)):
+        if l in drop:                                    # recompute before gradients
+            for t in sz.internals:
+                A.push(t)
+        A.talloc(sz.layer_scratch)
+        A.tfree(sz.layer_scratch)
+        for t in reversed(sz.internals):
+            A.pop(t)
+        if l > 0:
+            A.pop(sz.y)                                  # y_{l-1}: input of layer l
+    A.talloc(sz.emb_scratch)
+    A.tfree(sz.emb_scratch)
+    for t in reversed(sz.E):
+        A.pop(t)
+    A.tfree(sz.dy)
+    assert A.live == sz.C
+    return A
+
+
+def peak(sz: Sizes, dropped: Sequence[int]) -> int:
+    return simulate_step(sz, dropped).peak
+
+
+def no_ckpt_peak(sz: Sizes) -> int:
+    return peak(sz, [])
+
+
+def lower_bound(sz: Sizes) -> int:
+    """LB: every layer but the last dropped (the last saves nothing at the
+    peak); equals the all-dropped peak."""
+    return peak(sz, range(sz.n_layers - 1))
+
+
+# --------------------------------------------------------------------------
+# shuttling collector (Fig. 7): what a sheltered iteration measures
+# --------------------------------------------------------------------------
+
+def collect_samples(sz: Sizes) -> Dict[str, object]:
+    """Per-layer deltas of the two forward passes (pass 1 save-mode -> a_l,
+    pass 2 no-save -> y_l), embedding / head deltas, and the backward
+    transient maxima per phase, all in arena bytes; plus the collector's own
+    peak (the sheltered iteration drops every layer)."""
+    L = sz.n_layers
+    A = Arena(sz.C)
+    base = A.live
+    for t in sz.E:
+        A.push(t)
+    E = A.live - base
+    a, y = [], []
+    for _ in range(L):
+        b0 = A.live
+        for t in sz.internals:                           # pass 1: normal forward
+            A.push(t)
+        A.push(sz.y)
+        a.append(A.live - b0)
+        A.pop(sz.y)
+        for t in reversed(sz.internals):                 # discard output + activations
+            A.pop(t)
+        for t in sz.internals:                           # pass 2: keep only the output
+            A.talloc(t)
+        A.push(sz.y)
+        for t in reversed(sz.internals):
+            A.tfree(t)
+        y.append(A.live - b0)
+    b0 = A.live
+    for t in sz.head:
+        A.push(t)
+    hd = A.live - b0
+    # backward with every layer recomputed; per-phase max of the top region
+    A.talloc(sz.dy)
+    A.top_peak_phase = sum(A.top)
+    A.talloc(sz.head_scratch)
+    A.tfree(sz.head_scratch)
+    th = A.top_peak_phase
+    for t in reversed(sz.head):
+        A.pop(t)
+    A.pop(sz.y)
+    A.top_peak_phase = sum(A.top)
+    for l in reversed(range(L)):
+        for t in sz.internals:
+            A.push(t)
+        A.talloc(sz.layer_scratch)
+        A.tfree(sz.layer_scratch)
+        for t in reversed(sz.internals):
+            A.pop(t)
+        if l > 0:
+            A.pop(sz.y)
+    tb = A.top_peak_phase
+    A.top_peak_phase = sum(A.top)
+    A.talloc(sz.emb_scratch)
+    A.tfree(sz.emb_scratch)
+    te = A.top_peak_phase
+    for t in reversed(sz.E):
+        A.pop(t)
+    A.tfree(sz.dy)
+    return dict(C=sz.C, E=E, a=a, y=y, Hd=hd, Th=th, Tb=tb, Te=te, peak=A.peak)

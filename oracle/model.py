@@ -1,0 +1,325 @@
+"""ORACLE (test infrastructure only): fp64 post-LN transformer encoder training step.
+
+What Mimose's training step computes (§II-A: forward -> loss ->
+backward -> update; §IV-C P:160 the attention structure Q x K^T -> scale ->
+softmax -> x V; P:21 checkpointing = dropping activations and "replaying the
+forward computation" in backward).  Checkpointing is exact, so the oracle's
+reference result is the PLAIN non-checkpointed step; ``plan`` only changes
+what is kept (c-C identity), never the arithmetic.
+
+Model details the paper leaves to HF transformers 4.18 follow reading
+R-A24 of DESIGN.md: post-LN BERT/RoBERTa layer, erf-GELU, biased-variance LN,
+dropout p on embeddings / attention probabilities / both residual branches /
+pooled output, pooler tanh, CE heads.
+
+Every backward formula is textbook backprop written out by hand.
+Pinned by: central finite differences (fp64), torch CPU fp64 autograd with the
+same masks injected, closed-form per-op identities (tests/test_oracle_model.py).
+"""
+from __future__ import annotations
+
+import math
+from typing import Dict, Optional, Sequence
+
+import numpy as np
+
+from paper_conf_ipps_liaolysshfyctzlq23_b200.workload import (
+    HEAD_MC, HEAD_QA, HEAD_SEQCLS, Batch, ModelConfig, param_spec)
+from . import philox as px
+
+
+# --------------------------------------------------------------------------
+# dropout masks (R-B: element order documented in DESIGN.md)
+# --------------------------------------------------------------------------
+
+class Masks:
+    """Scaled keep masks m = keep / (1-p) for one step on one rank."""
+
+    def __init__(self, cfg: ModelConfig, B: int, S: int, seed: int, step: int,
+                 rank: int = 0, p: Optional[float] = None, override=None):
+        self.cfg, self.B, self.S = cfg, B, S
+        self.seed, self.step, self.rank = seed, step, rank
+        self.p = cfg.p_drop if p is None else p
+        self.override = override or {}
+
+    def _mask(self, key, n, kind, layer, shape):
+        if key in self.override:
+            return self.override[key]
+        if self.p <= 0.0:
+            return np.ones(shape)
+        keep = px.keep_mask(n, self.p, self.seed, px.site_word(kind, layer, self.rank), self.step)
+        return keep.reshape(shape).astype(np.float64) / (1.0 - self.p)
+
+    def emb(self):
+        T, H = self.B * self.S, self.cfg.hidden
+        return self._mask(("emb",), T * H, px.KIND_EMB, px.LAYER_NONE, (T, H))
+
+    def attn_probs(self, l):
+        B, S, h = self.B, self.S, self.cfg.heads
+        return self._mask(("attn", l), B * h * S * S, px.KIND_ATTN_PROBS, l, (B, h, S, S))
+
+    def attn_out(self, l):
+        T, H = self.B * self.S, self.cfg.hidden
+        return self._mask(("ao", l), T * H, px.KIND_ATTN_OUT, l, (T, H))
+
+    def ffn_out(self, l):
+        T, H = self.B * self.S, self.cfg.hidden
+        return self._mask(("fo", l), T * H, px.KIND_FFN_OUT, l, (T, H))
+
+    def head(self):
+        B, H = self.B, self.cfg.hidden
+        return self._mask(("head",), B * H, px.KIND_HEAD, px.LAYER_NONE, (B, H))
+
+
+# --------------------------------------------------------------------------
+# elementary ops (forward, backward)
+# --------------------------------------------------------------------------
+
+def linear(x, w, b):
+    """y = x W^T + b."""
+    return x @ w.T + b
+
+
+def linear_bwd(dy, x, w):
+    """dx = dy W ; dW = dy^T x ; db = sum_rows dy."""
+    return dy @ w, dy.T @ x, dy.sum(axis=0)
+
+
+def layernorm(z, g, b, eps):
+    """(z - mu) / sqrt(var + eps) * g + b, biased variance."""
+    mu = z.mean(axis=-1, keepdims=True)
+    var = ((z - mu) ** 2).mean(axis=-1, keepdims=True)
+    rstd = 1.0 / np.sqrt(var + eps)
+    xhat = (z - mu) * rstd
+    return xhat * g + b, (xhat, rstd)
+
+
+def layernorm_bwd(dy, cache, g):
+    xhat, rstd = cache
+    dg = (dy * xhat).sum(axis=0)
+    db = dy.sum(axis=0)
+    dxhat = dy * g
+    dz = rstd * (dxhat - dxhat.mean(axis=-1, keepdims=True)
+                 - xhat * (dxhat * xhat).mean(axis=-1, keepdims=True))
+    return dz, dg, db
+
+
+_erf = np.vectorize(math.erf, otypes=[np.float64])
+
+
+def gelu(u):
+    """erf-GELU: 0.5 u (1 + erf(u / sqrt 2))."""
+    return 0.5 * u * (1.0 + _erf(u / math.sqrt(2.0)))
+
+
+def gelu_bwd(du_out, u):
+    cdf = 0.5 * (1.0 + _erf(u / math.sqrt(2.0)))
+    pdf = np.exp(-0.5 * u * u) / math.sqrt(2.0 * math.pi)
+    return du_out * (cdf + u * pdf)
+
+
+def softmax_lastdim(s):
+    m = s.max(axis=-1, keepdims=True)
+    e = np.exp(s - m)
+    z = e.sum(axis=-1, keepdims=True)
+    return e / z, (m + np.log(z))[..., 0]
+
+
+def ce_rows(logits, target):
+    """mean over rows of -log softmax(logits)[target]; returns loss, dlogits."""
+    p, lse = softmax_lastdim(logits)
+    n = logits.shape[0]
+    loss = float(np.mean(lse - logits[np.arange(n), target]))
+    d = p.copy()
+    d[np.arange(n), target] -= 1.0
+    return loss, d / n
+
+
+# --------------------------------------------------------------------------
+# attention: S = Q K^T / sqrt(d) + key-pad mask, P = softmax, O = drop(P) V
+# --------------------------------------------------------------------------
+
+def attention_fwd(qkv, lengths, B, S, h, pmask):
+    H = qkv.shape[1] // 3
+    d = H // h
+    q = qkv[:, :H].reshape(B, S, h, d).transpose(0, 2, 1, 3)
+    k = qkv[:, H:2 * H].reshape(B, S, h, d).transpose(0, 2, 1, 3)
+    v = qkv[:, 2 * H:].reshape(B, S, h, d).transpose(0, 2, 1, 3)
+    s = q @ k.transpose(0, 1, 3, 2) / math.sqrt(d)
+    keyvalid = np.arange(S)[None, :] < np.asarray(lengths)[:, None]        # [B, S]
+    s = np.where(keyvalid[:, None, None, :], s, -np.inf)
+    p, lse = softmax_lastdim(s)
+    pd = p * pmask
+    o = pd @ v                                                             # [B,h,S,d]
+    out = o.transpose(0, 2, 1, 3).reshape(B * S, H)
+    return out, (q, k, v, p, pd, lse)
+
+
+def attention_bwd(dout, cache, B, S, h, pmask):
+    q, k, v, p, pd, _ = cache
+    d = q.shape[-1]
+    H = h * d
+    do = dout.reshape(B, S, h, d).transpose(0, 2, 1, 3)
+    dv = pd.transpose(0, 1, 3, 2) @ do
+    dpd = do @ v.transpose(0, 1, 3, 2)
+    dp = dpd * pmask
+    ds = p * (dp - (dp * p).sum(axis=-1, keepdims=True))
+    dq = ds @ k / math.sqrt(d)
+    dk = ds.transpose(0, 1, 3, 2) @ q / math.sqrt(d)
+    def flat(t):
+        return t.transpose(0, 2, 1, 3).reshape(B * S, H)
+    return np.concatenate([flat(dq), flat(dk), flat(dv)], axis=1)
+
+
+# --------------------------------------------------------------------------
+# encoder layer (post-LN)
+# --------------------------------------------------------------------------
+
+def layer_fwd(cfg, W, l, x, lengths, B, S, masks: Masks):
+    p = f"layer{l}."
+    qkv = linear(x, W[p + "qkv.w"], W[p + "qkv.b"])
+    o, acache = attention_fwd(qkv, lengths, B, S, cfg.heads, masks.attn_probs(l))
+    t1 = linear(o, W[p + "o.w"], W[p + "o.b"])
+    z1 = x + t1 * masks.attn_out(l)
+    h1, ln1 = layernorm(z1, W[p + "ln1.g"], W[p + "ln1.b"], cfg.ln_eps)
+    u = linear(h1, W[p + "f1.w"], W[p + "f1.b"])
+    g = gelu(u)
+    t2 = linear(g, W[p + "f2.w"], W[p + "f2.b"])
+    z2 = h1 + t2 * masks.ffn_out(l)
+    y, ln2 = layernorm(z2, W[p + "ln2.g"], W[p + "ln2.b"], cfg.ln_eps)
+    cache = dict(x=x, qkv=qkv, o=o, acache=acache, ln1=ln1, h1=h1, u=u, g=g, ln2=ln2)
+    return y, cache
+
+
+def layer_bwd(cfg, W, l, dy, c, B, S, masks: Masks, G):
+    p = f"layer{l}."
+    dz2, G[p + "ln2.g"], G[p + "ln2.b"] = layernorm_bwd(dy, c["ln2"], W[p + "ln2.g"])
+    dt2 = dz2 * masks.ffn_out(l)
+    dg, G[p + "f2.w"], G[p + "f2.b"] = linear_bwd(dt2, c["g"], W[p + "f2.w"])
+    du = gelu_bwd(dg, c["u"])
+    dh1, G[p + "f1.w"], G[p + "f1.b"] = linear_bwd(du, c["h1"], W[p + "f1.w"])
+    dh1 = dh1 + dz2
+    dz1, G[p + "ln1.g"], G[p + "ln1.b"] = layernorm_bwd(dh1, c["ln1"], W[p + "ln1.g"])
+    dt1 = dz1 * masks.attn_out(l)
+    do, G[p + "o.w"], G[p + "o.b"] = linear_bwd(dt1, c["o"], W[p + "o.w"])
+    dqkv = attention_bwd(do, c["acache"], B, S, cfg.heads, masks.attn_probs(l))
+    dx, G[p + "qkv.w"], G[p + "qkv.b"] = linear_bwd(dqkv, c["x"], W[p + "qkv.w"])
+    return dx + dz1
+
+
+# --------------------------------------------------------------------------
+# embeddings and heads
+# --------------------------------------------------------------------------
+
+def embed_fwd(cfg, W, batch: Batch, masks: Masks):
+    B, S = batch.input_ids.shape
+    ids = batch.input_ids.reshape(-1)
+    pos = np.tile(np.arange(S) + cfg.pos_offset, B)
+    tt = batch.token_type.reshape(-1)
+    z0 = W["emb.word"][ids] + W["emb.pos"][pos] + W["emb.type"][tt]
+    ln0, cache = layernorm(z0, W["emb.ln.g"], W["emb.ln.b"], cfg.ln_eps)
+    return ln0 * masks.emb(), (ids, pos, tt, cache)
+
+
+def embed_bwd(cfg, W, dx1, ec, masks: Masks, G):
+    ids, pos, tt, cache = ec
+    dln0 = dx1 * masks.emb()
+    dz0, G["emb.ln.g"], G["emb.ln.b"] = layernorm_bwd(dln0, cache, W["emb.ln.g"])
+    for name, idx in (("emb.word", ids), ("emb.pos", pos), ("emb.type", tt)):
+        acc = np.zeros_like(W[name])
+        np.add.at(acc, idx, dz0)
+        G[name] = acc
+
+
+def head_fwd_bwd(cfg, W, y, batch: Batch, masks: Masks, G):
+    """Loss and dL/dy for the task head; fills head grads into G."""
+    B, S = batch.input_ids.shape
+    H = cfg.hidden
+    dy = np.zeros_like(y)
+    if cfg.head in (HEAD_SEQCLS, HEAD_MC):
+        rows = np.arange(B) * S                        # CLS token of every sequence
+        c = y[rows]
+        pl = np.tanh(linear(c, W["pool.w"], W["pool.b"]))
+        pd = pl * masks.head()
+        logits = linear(pd, W["cls.w"], W["cls.b"])    # [B, n_out]
+        if cfg.head == HEAD_MC:
+            logits2 = logits.reshape(B // cfg.n_choices, cfg.n_choices)
+            loss, dl2 = ce_rows(logits2, batch.labels)
+            dlogits = dl2.reshape(B, 1)
+        else:
+            loss, dlogits = ce_rows(logits, batch.labels)
+        dpd, G["cls.w"], G["cls.b"] = linear_bwd(dlogits, pd, W["cls.w"])
+        dpre = dpd * masks.head() * (1.0 - pl * pl)
+        dc, G["pool.w"], G["pool.b"] = linear_bwd(dpre, c, W["pool.w"])
+        dy[rows] = dc
+        return loss, dy
+    # QA span head: start/end logits over valid positions (pads masked, R-A26)
+    logits = linear(y, W["qa.w"], W["qa.b"]).reshape(B, S, 2)
+    valid = np.arange(S)[None, :] < batch.lengths[:, None]
+    dlog = np.zeros_like(logits)
+    loss = 0.0
+    for j in range(2):
+        lg = np.where(valid, logits[:, :, j], -np.inf)
+        lj, dj = ce_rows(lg, batch.labels[j::2])
+        loss += 0.5 * lj
+        dlog[:, :, j] = 0.5 * np.where(valid, dj, 0.0)
+    dlog = dlog.reshape(B * S, 2)
+    dy, G["qa.w"], G["qa.b"] = linear_bwd(dlog, y, W["qa.w"])
+    return loss, dy
+
+
+# --------------------------------------------------------------------------
+# the whole step
+# --------------------------------------------------------------------------
+
+def train_step_grads(cfg: ModelConfig, params: Dict[str, np.ndarray], batch: Batch,
+                     seed: int, step: int, rank: int = 0,
+                     plan: Optional[Sequence[int]] = None, p: Optional[float] = None,
+                     mask_override=None):
+    """Loss and fp64 gradients of one mini-batch.
+
+    ``plan`` = 0-based indices of dropped layers: their caches are discarded
+    after forward (only the layer input is kept) and re-created by replaying
+    the forward right before their backward."""
+    W = {k: np.asarray(v, np.float64) for k, v in params.items()}
+    B, S = batch.input_ids.shape
+    masks = Masks(cfg, B, S, seed, step, rank, p, mask_override)
+    dropped = set(plan or ())
+    G: Dict[str, np.ndarray] = {}
+    x, ec = embed_fwd(cfg, W, batch, masks)
+    caches, inputs = [], []
+    for l in range(cfg.n_layers):
+        inputs.append(x)
+        x, c = layer_fwd(cfg, W, l, x, batch.lengths, B, S, masks)
+        caches.append(None if l in dropped else c)
+    loss, dy = head_fwd_bwd(cfg, W, x, batch, masks, G)
+    for l in reversed(range(cfg.n_layers)):
+        c = caches[l]
+        if c is None:                                   # recompute (replay)
+            _, c = layer_fwd(cfg, W, l, inputs[l], batch.lengths, B, S, masks)
+        dy = layer_bwd(cfg, W, l, dy, c, B, S, masks, G)
+        caches[l] = None
+    embed_bwd(cfg, W, dy, ec, masks, G)
+    return loss, G
+
+
+def adamw(params, grads, m, v, t, lr, beta1=0.9, beta2=0.999, eps=1e-8, wd=0.0):
+    """torch.optim.AdamW semantics (R-A25), fp64, applied to every tensor.
+    Returns new (params, m, v); t is the 1-based step count."""
+    out_p, out_m, out_v = {}, {}, {}
+    bc1 = 1.0 - beta1 ** t
+    bc2 = 1.0 - beta2 ** t
+    for k in params:
+        pk = np.asarray(params[k], np.float64) * (1.0 - lr * wd)
+        mk = beta1 * m[k] + (1.0 - beta1) * grads[k]
+        vk = beta2 * v[k] + (1.0 - beta2) * grads[k] * grads[k]
+        denom = np.sqrt(vk) / math.sqrt(bc2) + eps
+        out_p[k] = pk - (lr / bc1) * mk / denom
+        out_m[k], out_v[k] = mk, vk
+    return out_p, out_m, out_v
+
+
+def dp_mean_grads(grads_per_rank):
+    """Data-parallel semantics (c-J): gradient = mean over ranks."""
+    n = len(grads_per_rank)
+    return {k: sum(g[k] for g in grads_per_rank) / n for k in grads_per_rank[0]}
