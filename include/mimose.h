@@ -1,0 +1,241 @@
+/*
+ * mimose.h — C ABI of the B200-native Mimose training-step library (libmimose.so).
+ *
+ * What it implements (PAPER.md = /root/reference/PAPER.md, "P:n" = line n):
+ *   Mimose, an input-aware activation-checkpointing planner (§IV, Fig. 6):
+ *     - shuttling online collector (§IV-B, Fig. 7)    -> mimose_collect
+ *     - lightning memory estimator  (§IV-C, §VI-E)     -> fitted inside the ctx
+ *     - responsive greedy scheduler (§IV-D, Algorithm 1) -> mimose_plan
+ *     - applying the plan on the fly (§V)             -> mimose_forward / _backward
+ *   around the checkpointed training step of a post-LN transformer encoder
+ *   (P:51 forward -> loss -> backward -> update; P:160 attention structure),
+ *   under a hard device-memory budget M (Algorithm 1 input).
+ *   Readings of silent / garbled passages: DESIGN.md "Readings" (A1..A28, R-*).
+ *
+ * Conventions
+ *   - Every call returns mimose_status; nothing throws across the ABI.
+ *   - Pointers are plain host or device pointers as documented per field; no
+ *     torch types.  The caller owns every struct it passes in.
+ *   - All device work is enqueued on cfg.stream (a cudaStream_t); calls return
+ *     before the device finishes unless an output pointer needs a host value
+ *     (loss_out), in which case only that scalar is synchronised.
+ *   - One ctx per device per host thread; no global mutable state.
+ *   - MIMOSE_E_CUDA / MIMOSE_E_NCCL are sticky: the ctx refuses further work.
+ *   - mimose_last_error() returns a human-readable message for the last failure.
+ */
+#ifndef MIMOSE_H_
+#define MIMOSE_H_
+
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+#define MIMOSE_ABI_VERSION 1
+
+typedef struct mimose_ctx mimose_ctx; /* opaque, owned by the library */
+
+typedef enum {
+  MIMOSE_OK = 0,
+  MIMOSE_E_INVALID = 1,    /* bad argument / config / size                          */
+  MIMOSE_E_STATE = 2,      /* call out of order (see "Call order")                 */
+  MIMOSE_E_NOT_READY = 3,  /* mimose_plan before the estimator is fitted           */
+  MIMOSE_E_INFEASIBLE = 4, /* even the deepest plan predicts peak > M - reserve    */
+  MIMOSE_E_BUDGET = 5,     /* an arena request would make live bytes > M: the step
+                              is abandoned before any launch, counted as a violation,
+                              and the arena is rolled back                           */
+  MIMOSE_E_CUDA = 6,       /* sticky */
+  MIMOSE_E_NCCL = 7,       /* sticky */
+  MIMOSE_E_NODEVICE = 8    /* device call on a host-only ctx (arena_base == NULL)   */
+} mimose_status;
+
+enum { MIMOSE_ARCH_POST_LN = 0 };
+enum { MIMOSE_HEAD_SEQCLS = 0, MIMOSE_HEAD_MC = 1, MIMOSE_HEAD_QA = 2 };
+enum { MIMOSE_FP32 = 0, MIMOSE_BF16 = 1 };
+enum { MIMOSE_PHASE_SHELTERED = 0, MIMOSE_PHASE_RESPONSIVE = 1 };
+
+typedef struct {
+  /* ---- model (post-LN BERT/RoBERTa encoder, P:227 models; reading A24) ---- */
+  int32_t arch;         /* MIMOSE_ARCH_POST_LN                                        */
+  int32_t head;         /* MIMOSE_HEAD_*: seq-cls, multiple-choice, QA span (Table II)  */
+  int32_t dtype;        /* MIMOSE_FP32 (toy) or MIMOSE_BF16 (bf16 storage, fp32 accum,
+                           fp32 master weights)                                          */
+  int32_t n_layers;     /* L <= 64                                                      */
+  int32_t hidden;       /* H, multiple of 64 (head dim d = H/heads must be 32 or 64)    */
+  int32_t heads;
+  int32_t ffn;          /* F, multiple of 64                                            */
+  int32_t vocab, max_pos, type_vocab, pos_offset;
+  int32_t n_choices;    /* MC: sequences per question                                   */
+  int32_t n_labels;     /* seq-cls: classes                                             */
+  float p_drop;         /* dropout probability on every site (reading A24)              */
+  float ln_eps;
+  uint64_t seed;        /* Philox4x32-10 key (reading R-B)                              */
+  /* ---- Mimose ---- */
+  int64_t budget_bytes;  /* M of Algorithm 1: hard cap on arena live bytes,
+                            persistent state included                                   */
+  int64_t reserve_bytes; /* paper's fragmentation reserve; default 0 (A22)       */
+  int32_t enforce_budget;/* 1: an allocation beyond M -> MIMOSE_E_BUDGET;
+                            0: record only (no-checkpoint baseline)                     */
+  int32_t collect_iters; /* sheltered-phase length, default 10 (A17)            */
+  int32_t bucket_num, bucket_den; /* Alg. 1 line 8 ratio, default 9/10 (A6)           */
+  int32_t degree;        /* regression degree, default 2                        */
+  int32_t max_seqs, max_seq_len; /* sizing limits of a batch                            */
+  /* ---- device plumbing (supplied by the caller, e.g. PyTorch) ---- */
+  void* arena_base;      /* device slab, >= arena_bytes, 256-B aligned, outlives ctx.
+                            NULL -> host-only ctx: collector / estimator / planner /
+                            dry-run accounting run, no kernel is launched            */
+  int64_t arena_bytes;   /* slab size; must be >= budget_bytes when enforce_budget   */
+  void* stream;          /* cudaStream_t for all compute                             */
+  int32_t rank, world;   /* data parallel (weak scaling: each rank its own batch)    */
+  const void* nccl_id;   /* 128-byte ncclUniqueId from rank 0 (broadcast by caller);
+                            NULL when world == 1                                     */
+  int32_t use_tc;        /* 1: tcgen05 GEMMs in bf16 mode (default); 0: SIMT GEMMs  */
+  int32_t reserved[7];
+} mimose_config;
+
+/* Fill defaults (collect_iters 10, ratio 9/10, degree 2, p 0.1, eps 1e-12,
+   enforce 1, world 1, use_tc 1) into *cfg; the caller then sets the model fields. */
+void mimose_default_config(mimose_config* cfg);
+
+/* One mini-batch.  All arrays are int32, row-major, caller-owned and only read
+   during the call.  on_host = 1: host pointers (pinned recommended) copied H2D
+   inside the call; 0: device pointers.
+     input_ids  [n_seqs, seq_len]   right-padded with the pad id
+     token_type [n_seqs, seq_len]
+     lengths    [n_seqs]            valid tokens per sequence, 1..seq_len
+     labels     seq-cls: [n_seqs] class; MC: [n_seqs / n_choices] choice;
+                QA: [2*n_seqs] (start, end) per sequence
+   The input size key of P:73/P:221 is x = n_seqs * seq_len. */
+typedef struct {
+  const int32_t* input_ids;
+  const int32_t* token_type;
+  const int32_t* lengths;
+  const int32_t* labels;
+  int32_t n_seqs, seq_len;
+  int32_t on_host;
+} mimose_batch;
+
+/* Algorithm 1 output L' as a bitmask over layers (bit l = layer l,
+   0-based, is dropped and recomputed in backward). */
+typedef struct {
+  uint64_t drop_mask;
+  int32_t n_dropped;
+  int32_t from_cache;      /* 1 if served by the plan cache                  */
+  int64_t input_size;      /* x                                                      */
+  int64_t predicted_peak;  /* position-aware predicted peak of L' (reading A13)     */
+  int64_t budget;          /* M - reserve                                            */
+  int32_t status;          /* MIMOSE_OK or MIMOSE_E_INFEASIBLE                       */
+  int32_t pad_;
+} mimose_plan_t;
+
+/* Collected sample of one sheltered iteration (shuttling collector):
+   arena live-byte deltas; see DESIGN.md "Memory model". */
+typedef struct {
+  int64_t x;
+  int64_t C;             /* persistent bytes at forward start                        */
+  int64_t E;             /* embedding-forward delta                                  */
+  int64_t Hd;            /* head-forward delta                                       */
+  int64_t Th, Tb, Te;    /* max top-region bytes in head / layer / embedding backward */
+  int64_t a[64];         /* pass-1 (save mode) delta per layer                       */
+  int64_t y[64];         /* pass-2 (no-save mode) delta per layer                    */
+  float   t_ms[64];      /* pass-1 forward time per layer (cudaEvent; 0 host-only)   */
+} mimose_sample;
+
+typedef struct {
+  int64_t live_bytes, peak_bytes;      /* arena now / peak of the last step           */
+  int64_t max_peak_bytes;              /* over the ctx lifetime                        */
+  int64_t persistent_bytes;            /* C                                            */
+  int64_t budget_bytes;
+  int64_t violations;                  /* MIMOSE_E_BUDGET events                       */
+  int64_t steps, collect_steps, shuttled_steps;
+  int64_t plan_calls, plan_cache_hits, plan_cache_misses;
+  int64_t n_samples;
+  int32_t phase, last_n_dropped;
+  uint64_t last_drop_mask;
+  int64_t last_predicted_peak;
+  double planner_us_total;             /* host time in estimator+planner on misses     */
+  double collector_ms_total;           /* host wall time of shuttled collect calls     */
+  int64_t kernel_launches;             /* our kernels launched since init              */
+} mimose_stats;
+
+mimose_status mimose_init(const mimose_config* cfg, mimose_ctx** out);
+void mimose_destroy(mimose_ctx* ctx);
+const char* mimose_last_error(const mimose_ctx* ctx);
+const char* mimose_status_str(mimose_status s);
+
+/* Parameters: a host fp32 blob of every parameter tensor concatenated in the
+   documented order (workload.param_spec), no
+   padding.  bf16 mode: the fp32 values become the master copy and are rounded
+   (RNE) to the bf16 working copy.  Also resets AdamW state and the step count. */
+mimose_status mimose_num_params(const mimose_ctx* ctx, int64_t* n);
+mimose_status mimose_set_params(mimose_ctx* ctx, const float* host_blob, int64_t n);
+/* Reads the working copy (bf16 mode: bf16 values widened to fp32). */
+mimose_status mimose_get_params(mimose_ctx* ctx, float* host_blob, int64_t n);
+/* fp32 gradients of the last backward (after the DP all-reduce, before the
+   1/world scale), same order.  Test hook; synchronises the stream. */
+mimose_status mimose_get_grads(mimose_ctx* ctx, float* host_blob, int64_t n);
+
+/* Sheltered phase (Fig. 7): a forward in which every layer runs twice —
+   pass 1 normal (deltas -> a_l, time -> t_l, then discarded), pass 2 keeping
+   only the layer output (delta -> y_l).  Only unseen x are shuttled;
+   seen x run the conservative all-dropped forward.  Backward then recomputes
+   every layer and measures the transients.  After collect_iters calls (at least
+   3 distinct x, at most 30 calls, reading A17) the estimator is fitted and the
+   phase becomes RESPONSIVE.  loss_out (host, may be NULL) receives the loss. */
+mimose_status mimose_collect(mimose_ctx* ctx, const mimose_batch* batch, float* loss_out);
+
+/* Algorithm 1 (our reading): (M, x, L) -> L'.  Served from the plan
+   cache when x was planned before.  Host only, no device work.
+   Returns MIMOSE_E_NOT_READY in the sheltered phase; MIMOSE_E_INFEASIBLE if even
+   the deepest plan predicts a peak above M - reserve (out->status set too). */
+mimose_status mimose_plan(mimose_ctx* ctx, int64_t input_size, mimose_plan_t* out);
+
+/* Responsive forward under plan (NULL -> no layer dropped).  Dropped layers
+   keep only their output.  The whole step's allocation sequence is
+   checked against M before any launch (MIMOSE_E_BUDGET on breach). */
+mimose_status mimose_forward(mimose_ctx* ctx, const mimose_batch* batch,
+                             const mimose_plan_t* plan, float* loss_out);
+/* Backward: recompute each dropped layer with the same kernels, launch
+   configuration and Philox sites right before its gradient kernels (P:21,
+   P:217); per-layer NCCL all-reduce overlapped with the remaining backward. */
+mimose_status mimose_backward(mimose_ctx* ctx);
+/* AdamW (torch semantics, reading A25) on the fp32 master weights. */
+mimose_status mimose_step(mimose_ctx* ctx, float lr, float beta1, float beta2, float eps, float wd);
+
+mimose_status mimose_get_stats(const mimose_ctx* ctx, mimose_stats* out);
+mimose_status mimose_phase(const mimose_ctx* ctx, int32_t* phase);
+mimose_status mimose_get_sample(const mimose_ctx* ctx, int32_t i, mimose_sample* out);
+
+/* Host-only accounting of one full step (no launch): peak arena bytes for a
+   batch shape and plan, using the same allocation sequence as the real step.
+   Used to size budgets and by tests; never consulted by the planner (c-F). */
+mimose_status mimose_dry_run(mimose_ctx* ctx, int32_t n_seqs, int32_t seq_len,
+                             uint64_t drop_mask, int64_t* peak_out);
+/* Shuttling-collector accounting alone (no launch): the sample a sheltered
+   iteration at this shape would record (t_ms = 0). */
+mimose_status mimose_dry_collect(mimose_ctx* ctx, int32_t n_seqs, int32_t seq_len,
+                                 mimose_sample* out);
+
+/* ---- stateless host helpers (tests; same code the ctx uses) ---- */
+/* Predicted series for one x: arrays a,y of n_layers entries. */
+typedef struct {
+  int64_t C, E, Hd, Th, Tb, Te;
+  const int64_t* a;
+  const int64_t* y;
+  int32_t n_layers;
+} mimose_series;
+/* Position-aware predicted peak of a plan (reading A13). */
+int64_t mimose_predicted_peak(const mimose_series* s, uint64_t drop_mask);
+/* Full planner (Alg. 1 + A12 + A13) on given predictions. */
+mimose_status mimose_plan_series(const mimose_series* s, int64_t budget, int64_t reserve,
+                                 int32_t bucket_num, int32_t bucket_den,
+                                 uint64_t* drop_mask, int64_t* predicted_peak);
+/* Quadratic least squares (reading A18): fit ys(xs), predict at x_eval[i]. */
+mimose_status mimose_fit_predict(const int64_t* xs, const int64_t* ys, int32_t n, int32_t degree,
+                                 const int64_t* x_eval, int32_t n_eval, int64_t* out);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* MIMOSE_H_ */

@@ -102,11 +102,13 @@ def sizes(cfg: ModelConfig, B: int, S: int, max_seqs: Optional[int] = None,
     T = B * S
     ms = cfg.n_seqs if max_seqs is None else max_seqs
     mx = cfg.max_seq if max_seq_len is None else max_seq_len
-    E = [a16(T * H * e), a16(T * 8), a16(T * H * e)]                       # z0, st0, x1
+    # pre-LN sums z0, z1, z2 are fp32 in every mode (reading R-P: bf16 z loses
+    # the row mean/spread balance that LayerNorm's backward needs)
+    E = [a16(T * H * 4), a16(T * 8), a16(T * H * e)]                       # z0, st0, x1
     internals = [a16(T * 3 * H * e), a16(T * H * e), a16(B * h * S * 4),   # QKV, O, LSE
-                 a16(T * H * e), a16(T * 8), a16(T * H * e),               # z1, st1, h1
+                 a16(T * H * 4), a16(T * 8), a16(T * H * e),               # z1, st1, h1
                  a16(T * F * e), a16(T * F * e),                           # u, g
-                 a16(T * H * e), a16(T * 8)]                               # z2, st2
+                 a16(T * H * 4), a16(T * 8)]                               # z2, st2
     y = a16(T * H * e)
     if cfg.head == HEAD_QA:
         head = [a16(T * 2 * 4)]

@@ -1,0 +1,1090 @@
+// libmimose host runtime: the C ABI of include/mimose.h.
+//
+//   arena      budget-enforcing two-ended LIFO arena over the caller's slab
+//              (DESIGN "Memory model"; the paper's caching allocator loses
+//              0.5-1 GB to fragmentation, P:296 — a LIFO arena cannot fragment)
+//   schedule   forward / backward / recompute / optimizer launch order of one
+//              step, run either for real or as a host-only dry run (identical
+//              allocation sequence)
+//   collector  shuttling double forward of the sheltered phase
+//   estimator  + planner + plan cache (planning.cpp)
+//   comm       per-layer NCCL gradient all-reduce overlapped with backward
+#include <cuda_runtime.h>
+#include <nccl.h>
+
+#include <algorithm>
+#include <chrono>
+#include <cmath>
+#include <cstdio>
+#include <cstring>
+#include <string>
+#include <unordered_map>
+#include <vector>
+
+#include "../../../include/mimose.h"
+#include "../kernels.h"
+#include "planning.h"
+
+using namespace mimose;
+
+namespace {
+
+inline int64_t a16(int64_t n) { return (n + 15) / 16 * 16; }
+
+struct ParamInfo {
+  int64_t numel, off;  // off in elements of the padded flat layout
+};
+
+// The documented parameter order (DESIGN "Parameter layout").
+std::vector<ParamInfo> build_layout(const mimose_config& c, int64_t* npad) {
+  std::vector<int64_t> n;
+  const int64_t H = c.hidden, F = c.ffn;
+  n.push_back((int64_t)c.vocab * H);
+  n.push_back((int64_t)c.max_pos * H);
+  n.push_back((int64_t)c.type_vocab * H);
+  n.push_back(H);
+  n.push_back(H);
+  for (int l = 0; l < c.n_layers; ++l) {
+    const int64_t v[12] = {3 * H * H, 3 * H, H * H, H, H, H, F * H, F, H * F, H, H, H};
+    for (int64_t x : v) n.push_back(x);
+  }
+  if (c.head == MIMOSE_HEAD_QA) {
+    n.push_back(2 * H);
+    n.push_back(2);
+  } else {
+    const int64_t no = c.head == MIMOSE_HEAD_MC ? 1 : c.n_labels;
+    n.push_back(H * H);
+    n.push_back(H);
+    n.push_back(no * H);
+    n.push_back(no);
+  }
+  std::vector<ParamInfo> out;
+  int64_t off = 0;
+  for (int64_t x : n) {
+    out.push_back({x, off});
+    off += (x + 63) / 64 * 64;
+  }
+  *npad = off;
+  return out;
+}
+
+enum { P_WORD = 0, P_POS, P_TYPE, P_LN0G, P_LN0B, P_LAYER0 };
+enum { L_QKVW = 0, L_QKVB, L_OW, L_OB, L_LN1G, L_LN1B, L_F1W, L_F1B, L_F2W, L_F2B, L_LN2G, L_LN2B };
+
+// ------------------------------------------------------------------ arena --
+struct Arena {
+  char* base = nullptr;
+  int64_t cap = 0, budget = 0;
+  bool enforce = true;
+  int64_t C = 0;                 // persistent bytes (bottom)
+  int64_t stack = 0;             // stack bytes above C
+  int64_t top = 0;               // top-region bytes (grow down from cap)
+  std::vector<int64_t> sstack, stop;
+  int64_t peak = 0, top_phase_peak = 0;
+  bool breach = false;
+
+  int64_t live() const { return C + stack + top; }
+  void tick() {
+    peak = std::max(peak, live());
+    top_phase_peak = std::max(top_phase_peak, top);
+    if (live() > budget && enforce) breach = true;
+    if (C + stack + top > cap) breach = true;   // physical collision: never allowed
+  }
+  char* push(int64_t n) {
+    n = a16(n);
+    char* p = base + C + stack;
+    stack += n;
+    sstack.push_back(n);
+    tick();
+    return p;
+  }
+  void pop(int64_t n) {
+    n = a16(n);
+    if (sstack.empty() || sstack.back() != n) { breach = true; return; }
+    sstack.pop_back();
+    stack -= n;
+  }
+  char* talloc(int64_t n) {
+    n = a16(n);
+    top += n;
+    stop.push_back(n);
+    tick();
+    return base + cap - top;
+  }
+  void tfree(int64_t n) {
+    n = a16(n);
+    if (stop.empty() || stop.back() != n) { breach = true; return; }
+    stop.pop_back();
+    top -= n;
+  }
+  void reset_step() {
+    stack = top = 0;
+    sstack.clear();
+    stop.clear();
+    peak = live();
+    breach = false;
+  }
+};
+
+struct LayerBufs {
+  char *qkv = nullptr, *O = nullptr, *h1 = nullptr, *u = nullptr, *g = nullptr;
+  float *z1 = nullptr, *z2 = nullptr;   // pre-LN sums, fp32 (reading R-P)
+  float *lse = nullptr;
+  float2 *st1 = nullptr, *st2 = nullptr;
+};
+
+}  // namespace
+
+struct mimose_ctx {
+  mimose_config cfg{};
+  DType dt = DT_F32;
+  int e = 4;
+  bool device = false;
+  std::string err;
+  mimose_status sticky = MIMOSE_OK;
+  cudaStream_t st = nullptr, comm_st = nullptr;
+  ncclComm_t comm = nullptr;
+  cudaEvent_t ev_comm_done = nullptr;
+  std::vector<cudaEvent_t> ev_layer;
+
+  std::vector<ParamInfo> layout;
+  int64_t npad = 0;
+  Arena ar;
+  // persistent device buffers
+  char* w = nullptr;
+  float *grad = nullptr, *master = nullptr, *m = nullptr, *v = nullptr;
+  int32_t *ids = nullptr, *tt = nullptr, *lens = nullptr, *labels = nullptr;
+  float* misc = nullptr;
+  float* ws = nullptr;        // split-K workspace (4 H H fp32)
+  float* part = nullptr;      // NPART * 2 * max(3H, F) fp32
+  int64_t ws_elems = 0;
+
+  // step state
+  int B = 0, S = 0, T = 0;
+  uint64_t drop_mask = 0;
+  bool fwd_done = false, bwd_done = false, collecting = false;
+  float* z0 = nullptr;
+  char* x1 = nullptr;
+  float2* st0 = nullptr;
+  std::vector<LayerBufs> lb;
+  std::vector<char*> y;
+  char* hp = nullptr;         // pooled (cls) or unused
+  float* logits = nullptr;
+  int64_t it = 0;             // dropout step counter (forward calls)
+  int64_t adam_t = 0;
+
+  // Mimose
+  int phase = MIMOSE_PHASE_SHELTERED;
+  std::vector<Sample> samples;
+  std::vector<int64_t> seen_x;
+  Estimator est;
+  std::unordered_map<int64_t, mimose_plan_t> cache;
+  mimose_stats stats{};
+  std::vector<cudaEvent_t> ev_t0, ev_t1;
+  bool pending_times = false;
+};
+
+namespace {
+
+mimose_status fail(mimose_ctx* c, mimose_status s, const std::string& msg) {
+  if (c) {
+    c->err = msg;
+    if (s == MIMOSE_E_CUDA || s == MIMOSE_E_NCCL) c->sticky = s;
+  }
+  return s;
+}
+
+#define CK(x)                                                                               \
+  do {                                                                                      \
+    cudaError_t e_ = (x);                                                                   \
+    if (e_ != cudaSuccess) return fail(c, MIMOSE_E_CUDA, std::string(#x ": ") + cudaGetErrorString(e_)); \
+  } while (0)
+#define NK(x)                                                                               \
+  do {                                                                                      \
+    ncclResult_t r_ = (x);                                                                  \
+    if (r_ != ncclSuccess) return fail(c, MIMOSE_E_NCCL, std::string(#x ": ") + ncclGetErrorString(r_)); \
+  } while (0)
+
+// ---------------------------------------------------------------- sizes ---
+// Exactly DESIGN "Memory model" (and oracle/memsim.py, written independently).
+struct Sz {
+  int64_t z0, st0, x1;
+  int64_t qkv, O, lse, z1, st1, h1, u, g, z2, st2;
+  int64_t y;
+  int64_t head0, head1;   // QA: head0 = logits, head1 = 0
+  int64_t dy, head_scr, layer_scr, emb_scr;
+  int64_t r_dres, r_du, r_dt;  // carve offsets inside layer scratch
+};
+
+Sz sizes(const mimose_ctx* c, int B, int S) {
+  const int64_t T = (int64_t)B * S, H = c->cfg.hidden, F = c->cfg.ffn, h = c->cfg.heads, e = c->e;
+  Sz z{};
+  z.z0 = a16(T * H * 4); z.st0 = a16(T * 8); z.x1 = a16(T * H * e);
+  z.qkv = a16(T * 3 * H * e); z.O = a16(T * H * e); z.lse = a16((int64_t)B * h * S * 4);
+  z.z1 = a16(T * H * 4); z.st1 = a16(T * 8); z.h1 = a16(T * H * e);
+  z.u = a16(T * F * e); z.g = a16(T * F * e); z.z2 = a16(T * H * 4); z.st2 = a16(T * 8);
+  z.y = a16(T * H * e);
+  if (c->cfg.head == MIMOSE_HEAD_QA) {
+    z.head0 = a16(T * 2 * 4); z.head1 = 0;
+    z.head_scr = a16(T * 2 * 4);
+  } else {
+    const int64_t no = c->cfg.head == MIMOSE_HEAD_MC ? 1 : c->cfg.n_labels;
+    z.head0 = a16((int64_t)B * H * e); z.head1 = a16((int64_t)B * no * 4);
+    z.head_scr = a16((int64_t)B * no * 4) + 2 * a16((int64_t)B * H * 4);
+  }
+  z.dy = a16(T * H * 4);
+  z.r_dres = 0;
+  z.r_du = a16(T * H * 4);
+  z.r_dt = z.r_du + a16(T * F * e);
+  z.layer_scr = z.r_dt + a16(T * 3 * H * e) + a16((int64_t)B * h * S * 4);
+  const int64_t maxT = (int64_t)c->cfg.max_seqs * c->cfg.max_seq_len;
+  const int64_t ntiles = (maxT + 1023) / 1024;
+  z.emb_scr = a16(T * H * 4) + a16(16 * T) + a16(4 * 256 * ntiles);
+  return z;
+}
+
+int64_t persistent_bytes(const mimose_ctx* c) {
+  const int64_t H = c->cfg.hidden, F = c->cfg.ffn;
+  int64_t C = a16(c->npad * c->e) + 3 * a16(c->npad * 4);     // w, grad, m, v
+  if (c->dt != DT_F32) C += a16(c->npad * 4);                  // master
+  const int64_t maxT = (int64_t)c->cfg.max_seqs * c->cfg.max_seq_len;
+  C += 2 * a16(maxT * 4) + a16((int64_t)c->cfg.max_seqs * 4) + a16(2LL * c->cfg.max_seqs * 4);
+  C += a16(256);
+  C += a16(4 * H * H * 4);
+  C += a16((int64_t)NPART * 2 * std::max(3 * H, F) * 4);
+  return C;
+}
+
+Drop make_drop(const mimose_ctx* c, uint32_t kind, uint32_t layer) {
+  Drop d{};
+  const double p = c->cfg.p_drop;
+  d.enabled = p > 0.0;
+  d.seed_lo = (uint32_t)(c->cfg.seed & 0xFFFFFFFFu);
+  d.seed_hi = (uint32_t)(c->cfg.seed >> 32);
+  d.site = site_word(kind, layer, (uint32_t)c->cfg.rank);
+  d.step = (uint32_t)c->it;
+  d.thresh = d.enabled ? (uint32_t)std::floor((1.0 - p) * 4294967296.0) : 0xFFFFFFFFu;
+  d.scale = d.enabled ? (float)(1.0 / (1.0 - p)) : 1.0f;
+  return d;
+}
+Drop no_drop() { Drop d{}; d.enabled = 0; return d; }
+
+inline char* W(mimose_ctx* c, int i) { return c->w + c->layout[i].off * c->e; }
+inline float* G(mimose_ctx* c, int i) { return c->grad + c->layout[i].off; }
+inline int LP(mimose_ctx* c, int l, int k) { (void)c; return P_LAYER0 + 12 * l + k; }
+inline int HP(mimose_ctx* c, int k) { return P_LAYER0 + 12 * c->cfg.n_layers + k; }
+
+// ------------------------------------------------------------- schedule ---
+// `real` = launch kernels; otherwise only the arena accounting runs.
+
+struct Run {
+  mimose_ctx* c;
+  bool real;
+  Sz z;
+  cudaStream_t st;
+};
+
+void layer_forward(Run& r, int l, const char* x, LayerBufs& b, char* yout) {
+  mimose_ctx* c = r.c;
+  if (!r.real) return;
+  const int T = c->T, H = c->cfg.hidden, F = c->cfg.ffn;
+  const bool tc = c->cfg.use_tc != 0;
+  GemmArgs g;
+  // QKV = x Wqkv^T + b
+  g = GemmArgs();
+  g.M = T; g.N = 3 * H; g.K = H;
+  g.A = x; g.a_sm = H; g.a_sk = 1;
+  g.B = W(c, LP(c, l, L_QKVW)); g.b_sn = H; g.b_sk = 1;
+  g.C = b.qkv; g.ldc = 3 * H; g.bias = W(c, LP(c, l, L_QKVB));
+  gemm(c->dt, EPI_BIAS, g, r.st, tc);
+  attn_fwd(c->dt, b.qkv, c->lens, b.O, b.lse, c->B, c->S, H, c->cfg.heads, make_drop(c, KIND_ATTN_PROBS, l), r.st);
+  // z1 = x + drop(O Wo^T + bo)
+  g = GemmArgs();
+  g.M = T; g.N = H; g.K = H;
+  g.A = b.O; g.a_sm = H; g.a_sk = 1;
+  g.B = W(c, LP(c, l, L_OW)); g.b_sn = H; g.b_sk = 1;
+  g.C = b.z1; g.ldc = H; g.bias = W(c, LP(c, l, L_OB)); g.res = x; g.ldr = H;
+  g.drop = make_drop(c, KIND_ATTN_OUT, l);
+  gemm(c->dt, EPI_BIAS_DROP_RES, g, r.st, tc);
+  ln_fwd(c->dt, b.z1, W(c, LP(c, l, L_LN1G)), W(c, LP(c, l, L_LN1B)), b.h1, b.st1, T, H, c->cfg.ln_eps, r.st);
+  // u = h1 W1^T + b1, g = gelu(u)
+  g = GemmArgs();
+  g.M = T; g.N = F; g.K = H;
+  g.A = b.h1; g.a_sm = H; g.a_sk = 1;
+  g.B = W(c, LP(c, l, L_F1W)); g.b_sn = H; g.b_sk = 1;
+  g.C = b.u; g.C2 = b.g; g.ldc = F; g.bias = W(c, LP(c, l, L_F1B));
+  gemm(c->dt, EPI_BIAS_GELU, g, r.st, tc);
+  // z2 = h1 + drop(g W2^T + b2)
+  g = GemmArgs();
+  g.M = T; g.N = H; g.K = F;
+  g.A = b.g; g.a_sm = F; g.a_sk = 1;
+  g.B = W(c, LP(c, l, L_F2W)); g.b_sn = F; g.b_sk = 1;
+  g.C = b.z2; g.ldc = H; g.bias = W(c, LP(c, l, L_F2B)); g.res = b.h1; g.ldr = H;
+  g.drop = make_drop(c, KIND_FFN_OUT, l);
+  gemm(c->dt, EPI_BIAS_DROP_RES, g, r.st, tc);
+  // y = LN2(z2); the store is gated off during recompute (yout == nullptr)
+  ln_fwd(c->dt, b.z2, W(c, LP(c, l, L_LN2G)), W(c, LP(c, l, L_LN2B)), yout, b.st2, T, H, c->cfg.ln_eps, r.st);
+}
+
+void alloc_internals(Run& r, LayerBufs& b, bool on_stack) {
+  Arena& a = r.c->ar;
+  auto al = [&](int64_t n) { return on_stack ? a.push(n) : a.talloc(n); };
+  b.qkv = al(r.z.qkv); b.O = al(r.z.O); b.lse = (float*)al(r.z.lse);
+  b.z1 = (float*)al(r.z.z1); b.st1 = (float2*)al(r.z.st1); b.h1 = al(r.z.h1);
+  b.u = al(r.z.u); b.g = al(r.z.g); b.z2 = (float*)al(r.z.z2); b.st2 = (float2*)al(r.z.st2);
+}
+void free_internals(Run& r, bool on_stack) {
+  Arena& a = r.c->ar;
+  const int64_t s[10] = {r.z.qkv, r.z.O, r.z.lse, r.z.z1, r.z.st1, r.z.h1, r.z.u, r.z.g, r.z.z2, r.z.st2};
+  for (int i = 9; i >= 0; --i) on_stack ? a.pop(s[i]) : a.tfree(s[i]);
+}
+
+void wgrad(Run& r, const void* dY, int N, const void* X, int K, float* out) {
+  // dW[N, K] = sum_t dY[t, n] X[t, k]; deterministic split-K over t.
+  mimose_ctx* c = r.c;
+  const int T = c->T;
+  const int tiles = ((N + 127) / 128) * ((K + 127) / 128);
+  int split = std::max(1, std::min(4, 148 / std::max(1, tiles)));
+  while (split > 1 && (int64_t)split * N * K > c->ws_elems) --split;
+  while (split > 1 && T / split < 64) --split;
+  GemmArgs g;
+  g.M = N; g.N = K; g.K = T;
+  g.A = dY; g.a_sm = 1; g.a_sk = N;
+  g.B = X; g.b_sn = 1; g.b_sk = K;
+  g.ldc = K;
+  g.split = split;
+  if (split == 1) {
+    g.C = out;
+    gemm(c->dt, EPI_F32, g, r.st, c->cfg.use_tc != 0);
+  } else {
+    g.C = c->ws; g.split_stride = (int64_t)N * K;
+    gemm(c->dt, EPI_F32, g, r.st, c->cfg.use_tc != 0);
+    splitk_reduce(c->ws, split, (int64_t)N * K, out, r.st);
+  }
+}
+
+void dgrad(Run& r, Epi epi, const void* dY, int Nout, const void* Wt, int Kin, void* out, const void* res_or_aux) {
+  mimose_ctx* c = r.c;
+  GemmArgs g;
+  g.M = c->T; g.N = Kin; g.K = Nout;
+  g.A = dY; g.a_sm = Nout; g.a_sk = 1;
+  g.B = Wt; g.b_sn = 1; g.b_sk = Kin;
+  g.C = out; g.ldc = Kin;
+  if (epi == EPI_GELU_BWD) { g.aux = res_or_aux; g.ldx = Kin; }
+  if (epi == EPI_ACC_RES_F32) { g.res = res_or_aux; g.ldr = Kin; }
+  gemm(c->dt, epi, g, r.st, c->cfg.use_tc != 0);
+}
+
+void layer_backward(Run& r, int l, const char* x, LayerBufs& b, float* dy, char* scr) {
+  mimose_ctx* c = r.c;
+  if (!r.real) return;
+  const int T = c->T, H = c->cfg.hidden, F = c->cfg.ffn, h = c->cfg.heads;
+  float* dres = (float*)(scr + r.z.r_dres);
+  char* R2 = scr + r.z.r_du;     // du, later dO
+  char* R3 = scr + r.z.r_dt;     // dt2 / dt1, later dQKV
+  float* Dbuf = (float*)(scr + r.z.r_dt + a16((int64_t)T * 3 * H * c->e));
+  float* pg = c->part;
+  float* pb = c->part + (int64_t)NPART * H;
+  float* pbias = c->part + 2LL * NPART * H;
+  // LN2 backward + dropout backward -> dz2 (dres), dt2 (R3), partials
+  ln_bwd(c->dt, dy, no_drop(), b.z2, b.st2, W(c, LP(c, l, L_LN2G)), dres, R3, make_drop(c, KIND_FFN_OUT, l),
+         pg, pb, pbias, T, H, r.st);
+  reduce_partials(pg, H, H, G(c, LP(c, l, L_LN2G)), r.st);
+  reduce_partials(pb, H, H, G(c, LP(c, l, L_LN2B)), r.st);
+  reduce_partials(pbias, H, H, G(c, LP(c, l, L_F2B)), r.st);
+  // FFN2: du = (dt2 W2) * gelu'(u); dW2 = dt2^T g
+  dgrad(r, EPI_GELU_BWD, R3, H, W(c, LP(c, l, L_F2W)), F, R2, b.u);
+  wgrad(r, R3, H, b.g, F, G(c, LP(c, l, L_F2W)));
+  // FFN1: dh1 = du W1 + dz2 (in place in dres); dW1 = du^T h1; db1 = colsum du
+  dgrad(r, EPI_ACC_RES_F32, R2, F, W(c, LP(c, l, L_F1W)), H, dres, dres);
+  wgrad(r, R2, F, b.h1, H, G(c, LP(c, l, L_F1W)));
+  colsum(c->dt, R2, T, F, c->part, r.st);
+  reduce_partials(c->part, F, F, G(c, LP(c, l, L_F1B)), r.st);
+  // LN1 backward + dropout backward -> dz1 (dres, in place), dt1 (R3)
+  ln_bwd(c->dt, dres, no_drop(), b.z1, b.st1, W(c, LP(c, l, L_LN1G)), dres, R3, make_drop(c, KIND_ATTN_OUT, l),
+         pg, pb, pbias, T, H, r.st);
+  reduce_partials(pg, H, H, G(c, LP(c, l, L_LN1G)), r.st);
+  reduce_partials(pb, H, H, G(c, LP(c, l, L_LN1B)), r.st);
+  reduce_partials(pbias, H, H, G(c, LP(c, l, L_OB)), r.st);
+  // out-proj: dO = dt1 Wo (R2); dWo = dt1^T O
+  dgrad(r, EPI_STORE, R3, H, W(c, LP(c, l, L_OW)), H, R2, nullptr);
+  wgrad(r, R3, H, b.O, H, G(c, LP(c, l, L_OW)));
+  // attention backward -> dQKV (R3)
+  attn_bwd(c->dt, b.qkv, b.O, R2, b.lse, c->lens, Dbuf, R3, c->B, c->S, H, h, make_drop(c, KIND_ATTN_PROBS, l), r.st);
+  // QKV: dx = dQKV Wqkv + dz1 -> dy buffer; dWqkv = dQKV^T x; dbqkv = colsum dQKV
+  dgrad(r, EPI_ACC_RES_F32, R3, 3 * H, W(c, LP(c, l, L_QKVW)), H, dy, dres);
+  wgrad(r, R3, 3 * H, x, H, G(c, LP(c, l, L_QKVW)));
+  colsum(c->dt, R3, T, 3 * H, c->part, r.st);
+  reduce_partials(c->part, 3 * H, 3 * H, G(c, LP(c, l, L_QKVB)), r.st);
+}
+
+int64_t bucket_begin(mimose_ctx* c, int first_param) { return c->layout[first_param].off; }
+int64_t bucket_end(mimose_ctx* c, int last_param) {
+  return c->layout[last_param].off + (c->layout[last_param].numel + 63) / 64 * 64;
+}
+
+mimose_status allreduce_bucket(mimose_ctx* c, int first, int last, int evi) {
+  if (c->cfg.world <= 1 || !c->device) return MIMOSE_OK;
+  const int64_t b0 = bucket_begin(c, first), b1 = bucket_end(c, last);
+  CK(cudaEventRecord(c->ev_layer[evi], c->st));
+  CK(cudaStreamWaitEvent(c->comm_st, c->ev_layer[evi], 0));
+  NK(ncclAllReduce(c->grad + b0, c->grad + b0, (size_t)(b1 - b0), ncclFloat, ncclSum, c->comm, c->comm_st));
+  return MIMOSE_OK;
+}
+
+mimose_status copy_batch(mimose_ctx* c, const mimose_batch* bt) {
+  const int64_t T = (int64_t)bt->n_seqs * bt->seq_len;
+  const cudaMemcpyKind k = bt->on_host ? cudaMemcpyHostToDevice : cudaMemcpyDeviceToDevice;
+  int nl;
+  if (c->cfg.head == MIMOSE_HEAD_MC) nl = bt->n_seqs / c->cfg.n_choices;
+  else if (c->cfg.head == MIMOSE_HEAD_QA) nl = 2 * bt->n_seqs;
+  else nl = bt->n_seqs;
+  CK(cudaMemcpyAsync(c->ids, bt->input_ids, T * 4, k, c->st));
+  CK(cudaMemcpyAsync(c->tt, bt->token_type, T * 4, k, c->st));
+  CK(cudaMemcpyAsync(c->lens, bt->lengths, (int64_t)bt->n_seqs * 4, k, c->st));
+  CK(cudaMemcpyAsync(c->labels, bt->labels, (int64_t)nl * 4, k, c->st));
+  return MIMOSE_OK;
+}
+
+mimose_status check_batch(mimose_ctx* c, const mimose_batch* bt) {
+  if (!bt || bt->n_seqs <= 0 || bt->seq_len <= 0 || bt->n_seqs > c->cfg.max_seqs || bt->seq_len > c->cfg.max_seq_len)
+    return fail(c, MIMOSE_E_INVALID, "batch shape outside [1, max_seqs] x [1, max_seq_len]");
+  if (c->cfg.head == MIMOSE_HEAD_MC && bt->n_seqs % c->cfg.n_choices)
+    return fail(c, MIMOSE_E_INVALID, "MC batch: n_seqs must be a multiple of n_choices");
+  if (bt->seq_len + c->cfg.pos_offset > c->cfg.max_pos)
+    return fail(c, MIMOSE_E_INVALID, "seq_len + pos_offset exceeds max_pos");
+  return MIMOSE_OK;
+}
+
+// Forward of one step.  mode 0: plan-driven; mode 1: shuttling collector.
+// When `sample` is non-null the collector deltas are recorded.
+void run_forward(Run& r, uint64_t mask, bool collect, Sample* sample) {
+  mimose_ctx* c = r.c;
+  Arena& a = c->ar;
+  const int L = c->cfg.n_layers, H = c->cfg.hidden;
+  const int64_t base = a.live();
+  c->z0 = (float*)a.push(r.z.z0);
+  c->st0 = (float2*)a.push(r.z.st0);
+  c->x1 = a.push(r.z.x1);
+  if (sample) sample->E = a.live() - base;
+  if (r.real)
+    embed_fwd(c->dt, c->ids, c->tt, W(c, P_WORD), W(c, P_POS), W(c, P_TYPE), W(c, P_LN0G), W(c, P_LN0B), c->z0,
+              c->st0, c->x1, c->B, c->S, H, c->cfg.pos_offset, c->cfg.ln_eps, make_drop(c, KIND_EMB, LAYER_NONE),
+              r.st);
+  c->lb.assign(L, LayerBufs());
+  c->y.assign(L, nullptr);
+  const char* x = c->x1;
+  for (int l = 0; l < L; ++l) {
+    const int64_t b0 = a.live();
+    if (collect && sample) {
+      // pass 1: normal forward (save mode), timed; output and activations discarded
+      LayerBufs tmp;
+      alloc_internals(r, tmp, true);
+      char* yt = a.push(r.z.y);
+      if (r.real) cudaEventRecord(c->ev_t0[l], r.st);
+      layer_forward(r, l, x, tmp, yt);
+      if (r.real) cudaEventRecord(c->ev_t1[l], r.st);
+      sample->a[l] = a.live() - b0;
+      a.pop(r.z.y);
+      free_internals(r, true);
+    }
+    const bool dropped = collect || ((mask >> l) & 1);
+    alloc_internals(r, c->lb[l], !dropped);
+    c->y[l] = a.push(r.z.y);
+    layer_forward(r, l, x, c->lb[l], c->y[l]);
+    if (dropped) free_internals(r, false);
+    if (sample) sample->y[l] = a.live() - b0;
+    x = c->y[l];
+  }
+  const int64_t h0 = a.live();
+  if (c->cfg.head == MIMOSE_HEAD_QA) {
+    c->logits = (float*)a.push(r.z.head0);
+    if (r.real)
+      head_qa_fwd(c->dt, c->y[L - 1], c->B, c->S, H, W(c, HP(c, 0)), W(c, HP(c, 1)), c->logits, c->lens,
+                  c->labels, c->misc, r.st);
+  } else {
+    c->hp = a.push(r.z.head0);
+    c->logits = (float*)a.push(r.z.head1);
+    const int no = c->cfg.head == MIMOSE_HEAD_MC ? 1 : c->cfg.n_labels;
+    if (r.real)
+      head_cls_fwd(c->dt, c->y[L - 1], c->B, c->S, H, W(c, HP(c, 0)), W(c, HP(c, 1)), W(c, HP(c, 2)),
+                   W(c, HP(c, 3)), no, c->hp, c->logits, c->labels, c->cfg.n_choices, c->cfg.head, c->misc,
+                   make_drop(c, KIND_HEAD, LAYER_NONE), r.st);
+  }
+  if (sample) sample->Hd = a.live() - h0;
+}
+
+mimose_status run_backward(Run& r, Sample* sample) {
+  mimose_ctx* c = r.c;
+  Arena& a = c->ar;
+  const int L = c->cfg.n_layers, H = c->cfg.hidden;
+  const int T = c->T;
+  float* dy = (float*)a.talloc(r.z.dy);
+  // ---- head ----
+  a.top_phase_peak = a.top;
+  char* hs = a.talloc(r.z.head_scr);
+  if (r.real) {
+    if (c->cfg.head == MIMOSE_HEAD_QA) {
+      head_qa_bwd(c->dt, c->y[L - 1], c->B, c->S, H, W(c, HP(c, 0)), c->logits, c->lens, c->labels, (float*)hs,
+                  c->part, G(c, HP(c, 0)), G(c, HP(c, 1)), dy, r.st);
+    } else {
+      CK(cudaMemsetAsync(dy, 0, (size_t)T * H * 4, r.st));
+      const int no = c->cfg.head == MIMOSE_HEAD_MC ? 1 : c->cfg.n_labels;
+      head_cls_bwd(c->dt, c->y[L - 1], c->B, c->S, H, W(c, HP(c, 0)), W(c, HP(c, 2)), no, c->hp, c->logits,
+                   c->labels, c->cfg.n_choices, c->cfg.head, (float*)hs, G(c, HP(c, 0)), G(c, HP(c, 1)),
+                   G(c, HP(c, 2)), G(c, HP(c, 3)), dy, make_drop(c, KIND_HEAD, LAYER_NONE), r.st);
+    }
+  }
+  a.tfree(r.z.head_scr);
+  if (sample) sample->Th = a.top_phase_peak;
+  if (r.real) {
+    const int nh = c->cfg.head == MIMOSE_HEAD_QA ? 2 : 4;
+    mimose_status s = allreduce_bucket(c, HP(c, 0), HP(c, nh - 1), L);
+    if (s) return s;
+  }
+  if (c->cfg.head == MIMOSE_HEAD_QA) {
+    a.pop(r.z.head0);
+  } else {
+    a.pop(r.z.head1);
+    a.pop(r.z.head0);
+  }
+  a.pop(r.z.y);                                       // y_L
+  // ---- layers ----
+  a.top_phase_peak = a.top;
+  for (int l = L - 1; l >= 0; --l) {
+    const bool dropped = (c->drop_mask >> l) & 1;
+    const char* x = l > 0 ? c->y[l - 1] : c->x1;
+    if (dropped) {                                    // recompute right before the gradients
+      alloc_internals(r, c->lb[l], true);
+      layer_forward(r, l, x, c->lb[l], nullptr);
+    }
+    char* scr = a.talloc(r.z.layer_scr);
+    layer_backward(r, l, x, c->lb[l], dy, scr);
+    a.tfree(r.z.layer_scr);
+    if (r.real) {
+      mimose_status s = allreduce_bucket(c, LP(c, l, 0), LP(c, l, 11), l);
+      if (s) return s;
+    }
+    free_internals(r, true);
+    if (l > 0) a.pop(r.z.y);                          // y_{l-1}: input of layer l
+  }
+  if (sample) sample->Tb = a.top_phase_peak;
+  // ---- embedding ----
+  a.top_phase_peak = a.top;
+  char* es = a.talloc(r.z.emb_scr);
+  if (r.real) {
+    float* dz0 = (float*)es;
+    int32_t* work = (int32_t*)(es + a16((int64_t)T * H * 4));
+    int32_t* hist = (int32_t*)(es + a16((int64_t)T * H * 4) + a16(16LL * T));
+    float* pg = c->part;
+    float* pb = c->part + (int64_t)NPART * H;
+    ln_bwd(c->dt, dy, make_drop(c, KIND_EMB, LAYER_NONE), c->z0, c->st0, W(c, P_LN0G), dz0, nullptr, no_drop(), pg,
+           pb, nullptr, T, H, r.st);
+    reduce_partials(pg, H, H, G(c, P_LN0G), r.st);
+    reduce_partials(pb, H, H, G(c, P_LN0B), r.st);
+    const int64_t e0 = c->layout[P_WORD].off, e1 = bucket_end(c, P_TYPE);
+    CK(cudaMemsetAsync(c->grad + e0, 0, (size_t)(e1 - e0) * 4, r.st));
+    pos_grad(dz0, c->B, c->S, H, c->cfg.pos_offset, G(c, P_POS), r.st);
+    type_grad(dz0, c->tt, T, H, c->cfg.type_vocab, c->part, G(c, P_TYPE), r.st);
+    const int bits = c->cfg.vocab <= 256 ? 8 : 16;
+    const int64_t maxT = (int64_t)c->cfg.max_seqs * c->cfg.max_seq_len;
+    keyed_rowsum(c->ids, bits, dz0, T, H, G(c, P_WORD), work, hist, (int)((maxT + 1023) / 1024), r.st);
+  }
+  a.tfree(r.z.emb_scr);
+  if (sample) sample->Te = a.top_phase_peak;
+  if (r.real) {
+    mimose_status s = allreduce_bucket(c, P_WORD, P_LN0B, L + 1);
+    if (s) return s;
+  }
+  a.pop(r.z.x1);
+  a.pop(r.z.st0);
+  a.pop(r.z.z0);
+  a.tfree(r.z.dy);
+  return MIMOSE_OK;
+}
+
+// Host-only accounting of a full step: peak bytes and breach flag.
+void dry_step(mimose_ctx* c, int B, int S, uint64_t mask, bool collect, int64_t* peak, bool* breach, Sample* smp) {
+  // Save the ctx step state that the dry run overwrites.
+  const int sB = c->B, sS = c->S, sT = c->T;
+  const uint64_t sm = c->drop_mask;
+  Arena saved = c->ar;
+  float* sz0 = c->z0;
+  char *sx1 = c->x1, *shp = c->hp;
+  float2* sst0 = c->st0;
+  float* slog = c->logits;
+  std::vector<LayerBufs> slb = c->lb;
+  std::vector<char*> sy = c->y;
+  c->B = B; c->S = S; c->T = B * S;
+  c->drop_mask = collect ? ~0ull : mask;
+  c->ar.reset_step();
+  c->ar.base = nullptr;
+  Run r{c, false, sizes(c, B, S), nullptr};
+  run_forward(r, mask, collect, smp);
+  run_backward(r, smp);
+  *peak = c->ar.peak;
+  *breach = c->ar.breach;
+  c->ar = saved;
+  c->B = sB; c->S = sS; c->T = sT; c->drop_mask = sm;
+  c->z0 = sz0; c->x1 = sx1; c->hp = shp; c->st0 = sst0; c->logits = slog;
+  c->lb = slb; c->y = sy;
+}
+
+mimose_status check_ready(mimose_ctx* c) {
+  if (!c) return MIMOSE_E_INVALID;
+  if (c->sticky) return c->sticky;
+  return MIMOSE_OK;
+}
+
+void resolve_times(mimose_ctx* c) {
+  if (!c->pending_times || !c->device) return;
+  cudaStreamSynchronize(c->st);
+  Sample& s = c->samples.back();
+  for (int l = 0; l < c->cfg.n_layers; ++l) {
+    float ms = 0.f;
+    cudaEventElapsedTime(&ms, c->ev_t0[l], c->ev_t1[l]);
+    s.t_ms[l] = ms;
+  }
+  c->pending_times = false;
+}
+
+mimose_status read_loss(mimose_ctx* c, float* loss_out) {
+  if (!loss_out) return MIMOSE_OK;
+  if (!c->device) { *loss_out = 0.f; return MIMOSE_OK; }
+  CK(cudaMemcpyAsync(loss_out, c->misc, 4, cudaMemcpyDeviceToHost, c->st));
+  CK(cudaStreamSynchronize(c->st));
+  return MIMOSE_OK;
+}
+
+}  // namespace
+
+// =================================================================== ABI ===
+extern "C" {
+
+void mimose_default_config(mimose_config* cfg) {
+  std::memset(cfg, 0, sizeof(*cfg));
+  cfg->arch = MIMOSE_ARCH_POST_LN;
+  cfg->head = MIMOSE_HEAD_SEQCLS;
+  cfg->dtype = MIMOSE_BF16;
+  cfg->type_vocab = 2;
+  cfg->n_choices = 4;
+  cfg->n_labels = 2;
+  cfg->p_drop = 0.1f;
+  cfg->ln_eps = 1e-12f;
+  cfg->enforce_budget = 1;
+  cfg->collect_iters = 10;
+  cfg->bucket_num = 9;
+  cfg->bucket_den = 10;
+  cfg->degree = 2;
+  cfg->world = 1;
+  cfg->use_tc = 1;
+}
+
+const char* mimose_status_str(mimose_status s) {
+  switch (s) {
+    case MIMOSE_OK: return "ok";
+    case MIMOSE_E_INVALID: return "invalid argument";
+    case MIMOSE_E_STATE: return "call out of order";
+    case MIMOSE_E_NOT_READY: return "estimator not fitted (sheltered phase)";
+    case MIMOSE_E_INFEASIBLE: return "budget infeasible";
+    case MIMOSE_E_BUDGET: return "budget violation";
+    case MIMOSE_E_CUDA: return "CUDA error";
+    case MIMOSE_E_NCCL: return "NCCL error";
+    case MIMOSE_E_NODEVICE: return "host-only context";
+  }
+  return "?";
+}
+
+const char* mimose_last_error(const mimose_ctx* c) { return c ? c->err.c_str() : "null ctx"; }
+
+mimose_status mimose_init(const mimose_config* cfgp, mimose_ctx** out) {
+  if (!cfgp || !out) return MIMOSE_E_INVALID;
+  *out = nullptr;
+  mimose_ctx* c = new mimose_ctx();
+  c->cfg = *cfgp;
+  const mimose_config& k = c->cfg;
+  auto bad = [&](const char* m) { c->err = m; return MIMOSE_E_INVALID; };
+  if (k.arch != MIMOSE_ARCH_POST_LN || k.n_layers < 1 || k.n_layers > 64 || k.hidden % 64 || k.heads < 1 ||
+      k.hidden % k.heads || (k.hidden / k.heads != 32 && k.hidden / k.heads != 64) || k.ffn % 64 ||
+      k.hidden > 1024 || k.ffn > 4096 || k.vocab < 1 || k.vocab > 65536 || k.type_vocab < 1 || k.type_vocab > 4 ||
+      k.max_seqs < 1 || k.max_seq_len < 1 || (int64_t)k.max_seqs * k.max_seq_len > 32768 || k.max_pos < 1 ||
+      k.head < 0 || k.head > 2 || (k.head == MIMOSE_HEAD_MC && k.n_choices < 1) ||
+      (k.head == MIMOSE_HEAD_SEQCLS && (k.n_labels < 1 || k.n_labels > 32)) || k.world < 1 || k.rank < 0 ||
+      k.rank >= k.world || k.bucket_den <= 0 || k.degree < 0 || k.degree > 2) {
+    mimose_status s = bad("invalid model / sizing config");
+    *out = c;   // returned so mimose_last_error works; caller destroys
+    return s;
+  }
+  if (c->cfg.collect_iters <= 0) c->cfg.collect_iters = 10;
+  c->dt = k.dtype == MIMOSE_FP32 ? DT_F32 : DT_BF16;
+  c->e = k.dtype == MIMOSE_FP32 ? 4 : 2;
+  c->layout = build_layout(k, &c->npad);
+  c->ws_elems = 4LL * k.hidden * k.hidden;
+  c->device = k.arena_base != nullptr;
+  Arena& a = c->ar;
+  a.base = (char*)k.arena_base;
+  a.cap = k.arena_base ? k.arena_bytes : (int64_t)1 << 62;
+  a.budget = k.budget_bytes > 0 ? k.budget_bytes : a.cap;
+  a.enforce = k.enforce_budget != 0;
+  if (c->device && a.enforce && a.cap < a.budget) {
+    *out = c;
+    return bad("arena_bytes < budget_bytes with enforce_budget");
+  }
+  // persistent region, in the documented order
+  int64_t off = 0;
+  auto take = [&](int64_t n) { char* p = a.base + off; off += a16(n); return p; };
+  c->w = take(c->npad * c->e);
+  c->grad = (float*)take(c->npad * 4);
+  if (c->dt != DT_F32) c->master = (float*)take(c->npad * 4);
+  c->m = (float*)take(c->npad * 4);
+  c->v = (float*)take(c->npad * 4);
+  const int64_t maxT = (int64_t)k.max_seqs * k.max_seq_len;
+  c->ids = (int32_t*)take(maxT * 4);
+  c->tt = (int32_t*)take(maxT * 4);
+  c->lens = (int32_t*)take((int64_t)k.max_seqs * 4);
+  c->labels = (int32_t*)take(2LL * k.max_seqs * 4);
+  c->misc = (float*)take(256);
+  c->ws = (float*)take(c->ws_elems * 4);
+  c->part = (float*)take((int64_t)NPART * 2 * std::max<int64_t>(3LL * k.hidden, (int64_t)k.ffn) * 4);
+  a.C = off;
+  if (a.C != persistent_bytes(c)) {
+    *out = c;
+    return bad("internal: persistent layout mismatch");
+  }
+  a.reset_step();
+  c->stats.persistent_bytes = a.C;
+  c->stats.budget_bytes = a.budget;
+  c->stats.phase = MIMOSE_PHASE_SHELTERED;
+  if (a.C > a.budget || a.C > a.cap) {
+    *out = c;
+    c->err = "persistent state alone exceeds the budget / arena";
+    return MIMOSE_E_INFEASIBLE;
+  }
+  if (c->device) {
+    c->st = (cudaStream_t)k.stream;
+    const int L = k.n_layers;
+    c->ev_t0.resize(L);
+    c->ev_t1.resize(L);
+    for (int l = 0; l < L; ++l) {
+      CK(cudaEventCreate(&c->ev_t0[l]));
+      CK(cudaEventCreate(&c->ev_t1[l]));
+    }
+    CK(cudaMemsetAsync(a.base, 0, (size_t)a.C, c->st));
+    if (k.world > 1) {
+      if (!k.nccl_id) { *out = c; return bad("world > 1 needs nccl_id"); }
+      int lo, hi;
+      CK(cudaDeviceGetStreamPriorityRange(&lo, &hi));
+      CK(cudaStreamCreateWithPriority(&c->comm_st, cudaStreamNonBlocking, hi));
+      ncclUniqueId id;
+      std::memcpy(&id, k.nccl_id, sizeof(id));
+      NK(ncclCommInitRank(&c->comm, k.world, id, k.rank));
+      c->ev_layer.resize(L + 2);
+      for (auto& e : c->ev_layer) CK(cudaEventCreateWithFlags(&e, cudaEventDisableTiming));
+      CK(cudaEventCreateWithFlags(&c->ev_comm_done, cudaEventDisableTiming));
+    }
+  }
+  *out = c;
+  return MIMOSE_OK;
+}
+
+void mimose_destroy(mimose_ctx* c) {
+  if (!c) return;
+  if (c->device) {
+    cudaStreamSynchronize(c->st);
+    for (auto e : c->ev_t0) cudaEventDestroy(e);
+    for (auto e : c->ev_t1) cudaEventDestroy(e);
+    for (auto e : c->ev_layer) cudaEventDestroy(e);
+    if (c->ev_comm_done) cudaEventDestroy(c->ev_comm_done);
+    if (c->comm) ncclCommDestroy(c->comm);
+    if (c->comm_st) cudaStreamDestroy(c->comm_st);
+  }
+  delete c;
+}
+
+mimose_status mimose_num_params(const mimose_ctx* c, int64_t* n) {
+  if (!c || !n) return MIMOSE_E_INVALID;
+  int64_t s = 0;
+  for (auto& p : c->layout) s += p.numel;
+  *n = s;
+  return MIMOSE_OK;
+}
+
+static mimose_status xfer_params(mimose_ctx* c, float* host, int64_t n, int which) {
+  if (mimose_status s = check_ready(c)) return s;
+  int64_t tot;
+  mimose_num_params(c, &tot);
+  if (n != tot || !host) return fail(c, MIMOSE_E_INVALID, "blob size mismatch");
+  if (!c->device) return fail(c, MIMOSE_E_NODEVICE, "host-only context");
+  // staging: fp32 padded image in the grad buffer's slot is not free; use a temporary device buffer
+  float* tmp = nullptr;
+  CK(cudaMallocAsync((void**)&tmp, (size_t)c->npad * 4, c->st));
+  std::vector<float> img((size_t)c->npad, 0.f);
+  if (which == 0) {  // set
+    int64_t o = 0;
+    for (auto& p : c->layout) { std::memcpy(&img[p.off], host + o, p.numel * 4); o += p.numel; }
+    CK(cudaMemcpyAsync(tmp, img.data(), (size_t)c->npad * 4, cudaMemcpyHostToDevice, c->st));
+    cast_from_f32(c->dt, tmp, c->w, c->npad, c->st);
+    if (c->master) CK(cudaMemcpyAsync(c->master, tmp, (size_t)c->npad * 4, cudaMemcpyDeviceToDevice, c->st));
+    CK(cudaMemsetAsync(c->m, 0, (size_t)c->npad * 4, c->st));
+    CK(cudaMemsetAsync(c->v, 0, (size_t)c->npad * 4, c->st));
+    c->adam_t = 0;
+  } else {
+    if (which == 1) cast_to_f32(c->dt, c->w, tmp, c->npad, c->st);
+    else CK(cudaMemcpyAsync(tmp, c->grad, (size_t)c->npad * 4, cudaMemcpyDeviceToDevice, c->st));
+    CK(cudaMemcpyAsync(img.data(), tmp, (size_t)c->npad * 4, cudaMemcpyDeviceToHost, c->st));
+  }
+  CK(cudaStreamSynchronize(c->st));
+  CK(cudaFreeAsync(tmp, c->st));
+  CK(cudaStreamSynchronize(c->st));
+  if (which != 0) {
+    int64_t o = 0;
+    for (auto& p : c->layout) { std::memcpy(host + o, &img[p.off], p.numel * 4); o += p.numel; }
+  }
+  return MIMOSE_OK;
+}
+
+mimose_status mimose_set_params(mimose_ctx* c, const float* h, int64_t n) { return xfer_params(c, (float*)h, n, 0); }
+mimose_status mimose_get_params(mimose_ctx* c, float* h, int64_t n) { return xfer_params(c, h, n, 1); }
+mimose_status mimose_get_grads(mimose_ctx* c, float* h, int64_t n) {
+  if (c && c->device && c->comm_st) cudaStreamSynchronize(c->comm_st);
+  return xfer_params(c, h, n, 2);
+}
+
+static mimose_status begin_step(mimose_ctx* c, const mimose_batch* bt, uint64_t mask, bool collect, Sample* smp) {
+  if (mimose_status s = check_batch(c, bt)) return s;
+  // whole-step accounting first: abandon before any launch on a breach
+  int64_t peak;
+  bool breach;
+  dry_step(c, bt->n_seqs, bt->seq_len, mask, collect, &peak, &breach, nullptr);
+  if (breach) {
+    c->stats.violations++;
+    return fail(c, MIMOSE_E_BUDGET, "step would exceed the budget (predicted " + std::to_string(peak) +
+                                        " B > M = " + std::to_string(c->ar.budget) + ")");
+  }
+  c->B = bt->n_seqs; c->S = bt->seq_len; c->T = c->B * c->S;
+  c->drop_mask = collect ? ~0ull : mask;
+  c->ar.reset_step();
+  c->it++;
+  if (c->device) {
+    if (mimose_status s = copy_batch(c, bt)) return s;
+  }
+  Run r{c, c->device, sizes(c, c->B, c->S), c->st};
+  run_forward(r, mask, collect, smp);
+  c->fwd_done = true;
+  c->bwd_done = false;
+  return MIMOSE_OK;
+}
+
+mimose_status mimose_collect(mimose_ctx* c, const mimose_batch* bt, float* loss_out) {
+  if (mimose_status s = check_ready(c)) return s;
+  if (c->phase != MIMOSE_PHASE_SHELTERED) return fail(c, MIMOSE_E_STATE, "collect after the sheltered phase");
+  if (c->fwd_done && !c->bwd_done) return fail(c, MIMOSE_E_STATE, "forward pending its backward");
+  resolve_times(c);
+  const int64_t x = bt ? (int64_t)bt->n_seqs * bt->seq_len : 0;
+  const bool unseen = std::find(c->seen_x.begin(), c->seen_x.end(), x) == c->seen_x.end();
+  auto t0 = std::chrono::steady_clock::now();
+  c->collecting = unseen;
+  Sample smp;
+  const int L = c->cfg.n_layers;
+  smp.a.assign(L, 0); smp.y.assign(L, 0); smp.t_ms.assign(L, 0.f);
+  mimose_status s = begin_step(c, bt, ~0ull, true, unseen ? &smp : nullptr);
+  if (s) return s;
+  if (unseen) {
+    smp.x = x;
+    smp.C = c->ar.C;
+    c->samples.push_back(smp);     // Th/Tb/Te filled by backward
+    c->seen_x.push_back(x);
+    c->pending_times = c->device;
+    c->stats.shuttled_steps++;
+  }
+  c->stats.collect_steps++;
+  if (mimose_status s2 = read_loss(c, loss_out)) return s2;
+  c->stats.collector_ms_total +=
+      std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t0).count();
+  return MIMOSE_OK;
+}
+
+mimose_status mimose_forward(mimose_ctx* c, const mimose_batch* bt, const mimose_plan_t* plan, float* loss_out) {
+  if (mimose_status s = check_ready(c)) return s;
+  if (c->fwd_done && !c->bwd_done) return fail(c, MIMOSE_E_STATE, "forward pending its backward");
+  resolve_times(c);
+  c->collecting = false;
+  const uint64_t mask = plan ? plan->drop_mask : 0;
+  if (mimose_status s = begin_step(c, bt, mask, false, nullptr)) return s;
+  return read_loss(c, loss_out);
+}
+
+mimose_status mimose_backward(mimose_ctx* c) {
+  if (mimose_status s = check_ready(c)) return s;
+  if (!c->fwd_done || c->bwd_done) return fail(c, MIMOSE_E_STATE, "backward without a pending forward");
+  Run r{c, c->device, sizes(c, c->B, c->S), c->st};
+  Sample* smp = c->collecting ? &c->samples.back() : nullptr;
+  if (mimose_status s = run_backward(r, smp)) return s;
+  c->bwd_done = true;
+  c->stats.peak_bytes = c->ar.peak;
+  c->stats.max_peak_bytes = std::max(c->stats.max_peak_bytes, c->ar.peak);
+  c->stats.steps++;
+  if (c->ar.breach) {   // cannot happen after the dry run; kept as a hard check
+    c->stats.violations++;
+    return fail(c, MIMOSE_E_BUDGET, "arena breach during backward");
+  }
+  if (c->phase == MIMOSE_PHASE_SHELTERED) {
+    std::vector<int64_t> xs;
+    for (auto& s : c->samples) xs.push_back(s.x);
+    std::sort(xs.begin(), xs.end());
+    const int distinct = (int)(std::unique(xs.begin(), xs.end()) - xs.begin());
+    const int64_t n = c->stats.collect_steps;
+    if (!c->samples.empty() && ((n >= c->cfg.collect_iters && distinct >= 3) || n >= 30)) {
+      resolve_times(c);
+      auto t0 = std::chrono::steady_clock::now();
+      c->est.fit(c->samples, c->cfg.degree);
+      c->stats.planner_us_total +=
+          std::chrono::duration<double, std::micro>(std::chrono::steady_clock::now() - t0).count();
+      c->phase = MIMOSE_PHASE_RESPONSIVE;
+      c->stats.phase = c->phase;
+    }
+  }
+  c->stats.n_samples = (int64_t)c->samples.size();
+  return MIMOSE_OK;
+}
+
+mimose_status mimose_step(mimose_ctx* c, float lr, float b1, float b2, float eps, float wd) {
+  if (mimose_status s = check_ready(c)) return s;
+  if (!c->bwd_done) return fail(c, MIMOSE_E_STATE, "step without a backward");
+  if (!c->device) return MIMOSE_OK;
+  if (c->cfg.world > 1) {
+    CK(cudaEventRecord(c->ev_comm_done, c->comm_st));
+    CK(cudaStreamWaitEvent(c->st, c->ev_comm_done, 0));
+  }
+  c->adam_t++;
+  const double bc1 = 1.0 - std::pow((double)b1, (double)c->adam_t);
+  const double bc2 = 1.0 - std::pow((double)b2, (double)c->adam_t);
+  adamw(c->dt, c->w, c->master, c->grad, c->m, c->v, c->npad, lr, b1, b2, eps, wd, (float)bc1, (float)bc2,
+        1.0f / (float)c->cfg.world, c->st);
+  CK(cudaGetLastError());
+  c->fwd_done = false;
+  return MIMOSE_OK;
+}
+
+mimose_status mimose_plan(mimose_ctx* c, int64_t x, mimose_plan_t* out) {
+  if (mimose_status s = check_ready(c)) return s;
+  if (!out || x <= 0) return fail(c, MIMOSE_E_INVALID, "bad plan arguments");
+  if (c->phase != MIMOSE_PHASE_RESPONSIVE) return fail(c, MIMOSE_E_NOT_READY, "estimator not fitted yet");
+  c->stats.plan_calls++;
+  auto it = c->cache.find(x);
+  if (it != c->cache.end()) {
+    c->stats.plan_cache_hits++;
+    *out = it->second;
+    out->from_cache = 1;
+  } else {
+    c->stats.plan_cache_misses++;
+    auto t0 = std::chrono::steady_clock::now();
+    const Series s = c->est.predict(x);
+    const PlanResult pr = plan_greedy(s, c->ar.budget, c->cfg.reserve_bytes, c->cfg.bucket_num, c->cfg.bucket_den);
+    c->stats.planner_us_total +=
+        std::chrono::duration<double, std::micro>(std::chrono::steady_clock::now() - t0).count();
+    mimose_plan_t p{};
+    p.drop_mask = pr.drop_mask;
+    p.n_dropped = __builtin_popcountll(pr.drop_mask);
+    p.from_cache = 0;
+    p.input_size = x;
+    p.predicted_peak = pr.peak;
+    p.budget = c->ar.budget - c->cfg.reserve_bytes;
+    p.status = pr.feasible ? MIMOSE_OK : MIMOSE_E_INFEASIBLE;
+    c->cache[x] = p;
+    *out = p;
+  }
+  c->stats.last_drop_mask = out->drop_mask;
+  c->stats.last_n_dropped = out->n_dropped;
+  c->stats.last_predicted_peak = out->predicted_peak;
+  if (out->status != MIMOSE_OK) return fail(c, MIMOSE_E_INFEASIBLE, "no plan fits the budget");
+  return MIMOSE_OK;
+}
+
+mimose_status mimose_get_stats(const mimose_ctx* c, mimose_stats* out) {
+  if (!c || !out) return MIMOSE_E_INVALID;
+  *out = c->stats;
+  out->live_bytes = c->ar.live();
+  out->phase = c->phase;
+  out->kernel_launches = kernel_launch_count();
+  return MIMOSE_OK;
+}
+
+mimose_status mimose_phase(const mimose_ctx* c, int32_t* p) {
+  if (!c || !p) return MIMOSE_E_INVALID;
+  *p = c->phase;
+  return MIMOSE_OK;
+}
+
+mimose_status mimose_get_sample(const mimose_ctx* c, int32_t i, mimose_sample* out) {
+  if (!c || !out || i < 0 || i >= (int)c->samples.size()) return MIMOSE_E_INVALID;
+  const_cast<mimose_ctx*>(c)->err.clear();
+  resolve_times(const_cast<mimose_ctx*>(c));
+  const Sample& s = c->samples[i];
+  std::memset(out, 0, sizeof(*out));
+  out->x = s.x; out->C = s.C; out->E = s.E; out->Hd = s.Hd; out->Th = s.Th; out->Tb = s.Tb; out->Te = s.Te;
+  for (size_t l = 0; l < s.a.size(); ++l) { out->a[l] = s.a[l]; out->y[l] = s.y[l]; out->t_ms[l] = s.t_ms[l]; }
+  return MIMOSE_OK;
+}
+
+mimose_status mimose_dry_run(mimose_ctx* c, int32_t n_seqs, int32_t seq_len, uint64_t mask, int64_t* peak) {
+  if (!c || !peak) return MIMOSE_E_INVALID;
+  mimose_batch bt{nullptr, nullptr, nullptr, nullptr, n_seqs, seq_len, 1};
+  if (mimose_status s = check_batch(c, &bt)) return s;
+  bool breach;
+  const bool enf = c->ar.enforce;
+  c->ar.enforce = false;
+  dry_step(c, n_seqs, seq_len, mask, false, peak, &breach, nullptr);
+  c->ar.enforce = enf;
+  return MIMOSE_OK;
+}
+
+mimose_status mimose_dry_collect(mimose_ctx* c, int32_t n_seqs, int32_t seq_len, mimose_sample* out) {
+  if (!c || !out) return MIMOSE_E_INVALID;
+  mimose_batch bt{nullptr, nullptr, nullptr, nullptr, n_seqs, seq_len, 1};
+  if (mimose_status s = check_batch(c, &bt)) return s;
+  const int L = c->cfg.n_layers;
+  Sample smp;
+  smp.a.assign(L, 0); smp.y.assign(L, 0); smp.t_ms.assign(L, 0.f);
+  int64_t peak;
+  bool breach;
+  const bool enf = c->ar.enforce;
+  c->ar.enforce = false;
+  dry_step(c, n_seqs, seq_len, ~0ull, true, &peak, &breach, &smp);
+  c->ar.enforce = enf;
+  std::memset(out, 0, sizeof(*out));
+  out->x = (int64_t)n_seqs * seq_len; out->C = c->ar.C;
+  out->E = smp.E; out->Hd = smp.Hd; out->Th = smp.Th; out->Tb = smp.Tb; out->Te = smp.Te;
+  for (int l = 0; l < L; ++l) { out->a[l] = smp.a[l]; out->y[l] = smp.y[l]; }
+  return MIMOSE_OK;
+}
+
+static Series to_series(const mimose_series* s) {
+  Series r;
+  r.C = s->C; r.E = s->E; r.Hd = s->Hd; r.Th = s->Th; r.Tb = s->Tb; r.Te = s->Te;
+  r.a.assign(s->a, s->a + s->n_layers);
+  r.y.assign(s->y, s->y + s->n_layers);
+  return r;
+}
+
+int64_t mimose_predicted_peak(const mimose_series* s, uint64_t mask) { return predicted_peak(to_series(s), mask); }
+
+mimose_status mimose_plan_series(const mimose_series* s, int64_t budget, int64_t reserve, int32_t bn, int32_t bd,
+                                 uint64_t* mask, int64_t* peak) {
+  if (!s || !mask || !peak || s->n_layers < 1 || s->n_layers > 64 || bd <= 0) return MIMOSE_E_INVALID;
+  const PlanResult r = plan_greedy(to_series(s), budget, reserve, bn, bd);
+  *mask = r.drop_mask;
+  *peak = r.peak;
+  return r.feasible ? MIMOSE_OK : MIMOSE_E_INFEASIBLE;
+}
+
+mimose_status mimose_fit_predict(const int64_t* xs, const int64_t* ys, int32_t n, int32_t degree,
+                                 const int64_t* xe, int32_t ne, int64_t* out) {
+  if (!xs || !ys || n < 1 || !xe || !out || degree < 0 || degree > 2) return MIMOSE_E_INVALID;
+  Poly p;
+  p.fit(std::vector<int64_t>(xs, xs + n), std::vector<int64_t>(ys, ys + n), degree);
+  for (int i = 0; i < ne; ++i) out[i] = p.predict(xe[i]);
+  return MIMOSE_OK;
+}
+
+}  // extern "C"

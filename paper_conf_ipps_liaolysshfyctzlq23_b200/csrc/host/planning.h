@@ -1,0 +1,57 @@
+// Host-side Mimose planning: lightning memory estimator (§IV-C,
+// P:144-164; §VI-E) and the greedy scheduler (§IV-D, Algorithm 1
+// P:186-213) with the readings of DESIGN.md (A1-A13, A18).  Pure C++, no CUDA.
+#pragma once
+#include <cstdint>
+#include <unordered_map>
+#include <vector>
+
+namespace mimose {
+
+// Quadratic least squares in t = x / x_ref (reading A18): normal equations,
+// Gaussian elimination with partial pivoting, Horner evaluation, integer
+// predictions rounded half-to-even plus a non-negative residual margin.
+struct Poly {
+  int degree = 0;
+  double x_ref = 1.0;
+  double coef[3] = {0, 0, 0};
+  int64_t margin = 0;
+  void fit(const std::vector<int64_t>& xs, const std::vector<int64_t>& ys, int max_degree);
+  double eval(int64_t x) const;
+  int64_t predict(int64_t x) const;
+};
+
+// Per-series sizes for one input size x (what the planner reasons about).
+struct Series {
+  int64_t C = 0, E = 0, Hd = 0, Th = 0, Tb = 0, Te = 0;
+  std::vector<int64_t> a, y;   // per layer
+};
+
+// Position-aware peak of the arena event model (reading A13).
+int64_t predicted_peak(const Series& s, uint64_t drop_mask);
+
+struct PlanResult {
+  bool feasible = false;
+  uint64_t drop_mask = 0;
+  int64_t peak = 0;
+};
+// Algorithm 1 (A1-A11) + last-layer exclusion (A12) + verify (A13).
+PlanResult plan_greedy(const Series& s, int64_t budget, int64_t reserve, int bucket_num, int bucket_den);
+
+// One collected sheltered-iteration sample (arena deltas).
+struct Sample {
+  int64_t x = 0, C = 0, E = 0, Hd = 0, Th = 0, Tb = 0, Te = 0;
+  std::vector<int64_t> a, y;
+  std::vector<float> t_ms;
+};
+
+struct Estimator {
+  bool fitted = false;
+  int64_t C = 0;
+  std::vector<Poly> fa, fy;
+  Poly fE, fHd, fTh, fTb, fTe;
+  void fit(const std::vector<Sample>& samples, int degree);
+  Series predict(int64_t x) const;
+};
+
+}  // namespace mimose

@@ -1,0 +1,741 @@
+// HBM-bound kernels of the Mimose step on sm_100a: embedding, LayerNorm
+// forward/backward (fused with dropout and bias-gradient partials), column
+// sums, deterministic keyed row sums (embedding gradient), task heads, AdamW.
+//
+// Determinism: no floating-point atomics anywhere;
+// every reduction has a fixed assignment of rows to partials and a fixed
+// summation order, so recompute and plan changes cannot change a
+// single bit of the gradients.
+#include "kernels.h"
+
+#include <atomic>
+#include <cmath>
+
+namespace mimose {
+
+static std::atomic<long long> g_launches{0};
+void note_launch(int n) { g_launches.fetch_add(n, std::memory_order_relaxed); }
+int64_t kernel_launch_count() { return g_launches.load(); }
+
+template <typename F>
+static void dispatch(DType dt, F f) {
+  if (dt == DT_F32) f((float*)nullptr); else f((__nv_bfloat16*)nullptr);
+}
+
+static inline int cdiv(int64_t a, int64_t b) { return (int)((a + b - 1) / b); }
+
+// ===================================================================== LN ===
+
+template <typename E>
+__global__ void __launch_bounds__(256) k_ln_fwd(const float* __restrict__ z, const E* __restrict__ g,
+                                                const E* __restrict__ b, E* __restrict__ y,
+                                                float2* __restrict__ st, int T, int H, float eps) {
+  const int row = (blockIdx.x * blockDim.x + threadIdx.x) >> 5, lane = threadIdx.x & 31;
+  if (row >= T) return;
+  const int nv = H >> 5;
+  const float* zr = z + (int64_t)row * H;
+  float v[32];
+  float s = 0.f;
+#pragma unroll
+  for (int k = 0; k < 32; ++k)
+    if (k < nv) { v[k] = ldf(zr + lane + 32 * k); s += v[k]; }
+  const float mu = warp_sum(s) / (float)H;
+  float q = 0.f;
+#pragma unroll
+  for (int k = 0; k < 32; ++k)
+    if (k < nv) { const float d = v[k] - mu; q += d * d; }
+  const float rstd = rsqrtf(warp_sum(q) / (float)H + eps);
+  if (lane == 0) st[row] = make_float2(mu, rstd);
+  if (y) {
+    E* yr = y + (int64_t)row * H;
+#pragma unroll
+    for (int k = 0; k < 32; ++k)
+      if (k < nv) {
+        const int c = lane + 32 * k;
+        stf(yr + c, (v[k] - mu) * rstd * ldf(g + c) + ldf(b + c));
+      }
+  }
+}
+
+void ln_fwd(DType dt, const float* z, const void* g, const void* b, void* y, float2* st, int T,
+            int H, float eps, cudaStream_t s) {
+  note_launch(1);
+  dispatch(dt, [&](auto* tag) {
+    using E = std::remove_pointer_t<decltype(tag)>;
+    k_ln_fwd<E><<<cdiv(T, 8), 256, 0, s>>>(z, (const E*)g, (const E*)b, (E*)y, st, T, H, eps);
+  });
+}
+
+// 8 warps per CTA, NPART CTAs; warp w of CTA p owns rows r = p*8 + w + k*NPART*8.
+template <typename E>
+__global__ void __launch_bounds__(256) k_ln_bwd(const float* dy, Drop premask, const float* __restrict__ z,
+                                                const float2* __restrict__ st, const E* __restrict__ g,
+                                                float* dz, E* __restrict__ dtout, Drop mask,
+                                                float* __restrict__ pg, float* __restrict__ pb,
+                                                float* __restrict__ pbias, int T, int H) {
+  extern __shared__ float sm[];
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  float* ag = sm + (size_t)warp * 3 * H;
+  float* ab = ag + H;
+  float* at = ab + H;
+  for (int c = lane; c < H; c += 32) { ag[c] = 0.f; ab[c] = 0.f; at[c] = 0.f; }
+  const int nv = H >> 5;
+  const float invH = 1.0f / (float)H;
+  for (int row = blockIdx.x * 8 + warp; row < T; row += NPART * 8) {
+    const float* dyr = dy + (int64_t)row * H;
+    const float* zr = z + (int64_t)row * H;
+    const float2 ms = st[row];
+    float xh[32], dyv[32];
+    float s1 = 0.f, s2 = 0.f;
+#pragma unroll
+    for (int k = 0; k < 32; ++k)
+      if (k < nv) {
+        const int c = lane + 32 * k;
+        float d = dyr[c];
+        if (premask.enabled) d *= drop_factor(premask, (uint64_t)row * H + c);
+        dyv[k] = d;
+        xh[k] = (ldf(zr + c) - ms.x) * ms.y;
+        const float dxh = d * ldf(g + c);
+        s1 += dxh;
+        s2 += dxh * xh[k];
+      }
+    s1 = warp_sum(s1) * invH;
+    s2 = warp_sum(s2) * invH;
+    float* dzr = dz + (int64_t)row * H;
+#pragma unroll
+    for (int k = 0; k < 32; ++k)
+      if (k < nv) {
+        const int c = lane + 32 * k;
+        const float dxh = dyv[k] * ldf(g + c);
+        const float v = ms.y * (dxh - s1 - xh[k] * s2);
+        ag[c] += dyv[k] * xh[k];
+        ab[c] += dyv[k];
+        dzr[c] = v;
+        if (dtout) {
+          E* p = dtout + (int64_t)row * H + c;
+          stf(p, v * drop_factor(mask, (uint64_t)row * H + c));
+          at[c] += ldf(p);
+        }
+      }
+  }
+  __syncthreads();
+  for (int c = threadIdx.x; c < H; c += blockDim.x) {
+    float sg = 0.f, sb = 0.f, sbias = 0.f;
+    for (int w = 0; w < 8; ++w) {
+      const float* base = sm + (size_t)w * 3 * H;
+      sg += base[c]; sb += base[H + c]; sbias += base[2 * H + c];
+    }
+    pg[(size_t)blockIdx.x * H + c] = sg;
+    pb[(size_t)blockIdx.x * H + c] = sb;
+    if (pbias) pbias[(size_t)blockIdx.x * H + c] = sbias;
+  }
+}
+
+void ln_bwd(DType dt, const float* dy, Drop premask, const float* z, const float2* st, const void* g,
+            float* dz, void* dtout, Drop mask, float* pg, float* pb, float* pbias, int T, int H,
+            cudaStream_t s) {
+  const size_t smem = (size_t)8 * 3 * H * sizeof(float);
+  note_launch(1);
+  dispatch(dt, [&](auto* tag) {
+    using E = std::remove_pointer_t<decltype(tag)>;
+    static bool attr = false;
+    if (!attr) {
+      cudaFuncSetAttribute(k_ln_bwd<E>, cudaFuncAttributeMaxDynamicSharedMemorySize, 8 * 3 * 1024 * 4);
+      attr = true;
+    }
+    k_ln_bwd<E><<<NPART, 256, smem, s>>>(dy, premask, z, st, (const E*)g, dz, (E*)dtout,
+                                         mask, pg, pb, pbias, T, H);
+  });
+}
+
+__global__ void k_reduce_partials(const float* __restrict__ part, int64_t ld, int n, float* __restrict__ out) {
+  const int c = blockIdx.x * blockDim.x + threadIdx.x;
+  if (c >= n) return;
+  float s = 0.f;
+  for (int p = 0; p < NPART; ++p) s += part[(int64_t)p * ld + c];
+  out[c] = s;
+}
+void reduce_partials(const float* part, int64_t ld, int n, float* out, cudaStream_t s) {
+  note_launch(1);
+  k_reduce_partials<<<cdiv(n, 256), 256, 0, s>>>(part, ld, n, out);
+}
+
+__global__ void k_splitk_reduce(const float* __restrict__ part, int splits, int64_t n, float* __restrict__ out) {
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
+    float s = 0.f;
+    for (int k = 0; k < splits; ++k) s += part[k * n + i];
+    out[i] = s;
+  }
+}
+void splitk_reduce(const float* part, int splits, int64_t n, float* out, cudaStream_t s) {
+  note_launch(1);
+  k_splitk_reduce<<<592, 256, 0, s>>>(part, splits, n, out);
+}
+
+// column sums of X [T, N]: CTA p owns rows p, p+NPART, ...; thread owns columns tid + 256 j.
+template <typename E>
+__global__ void __launch_bounds__(256) k_colsum(const E* __restrict__ X, int T, int N, float* __restrict__ part) {
+  float acc[16];
+#pragma unroll
+  for (int j = 0; j < 16; ++j) acc[j] = 0.f;
+  for (int r = blockIdx.x; r < T; r += NPART) {
+    const E* xr = X + (int64_t)r * N;
+#pragma unroll
+    for (int j = 0; j < 16; ++j) {
+      const int c = threadIdx.x + 256 * j;
+      if (c < N) acc[j] += ldf(xr + c);
+    }
+  }
+#pragma unroll
+  for (int j = 0; j < 16; ++j) {
+    const int c = threadIdx.x + 256 * j;
+    if (c < N) part[(int64_t)blockIdx.x * N + c] = acc[j];
+  }
+}
+void colsum(DType dt, const void* X, int T, int N, float* part, cudaStream_t s) {
+  note_launch(1);
+  dispatch(dt, [&](auto* tag) {
+    using E = std::remove_pointer_t<decltype(tag)>;
+    k_colsum<E><<<NPART, 256, 0, s>>>((const E*)X, T, N, part);
+  });
+}
+
+// ============================================================== embedding ===
+
+template <typename E>
+__global__ void __launch_bounds__(256) k_embed_fwd(const int32_t* __restrict__ ids, const int32_t* __restrict__ tt,
+                                                   const E* __restrict__ Ww, const E* __restrict__ Wp,
+                                                   const E* __restrict__ Wt, const E* __restrict__ g,
+                                                   const E* __restrict__ b, float* __restrict__ z0,
+                                                   float2* __restrict__ st0, E* __restrict__ x1, int T,
+                                                   int S, int H, int pos_offset, float eps, Drop drop) {
+  const int t = (blockIdx.x * blockDim.x + threadIdx.x) >> 5, lane = threadIdx.x & 31;
+  if (t >= T) return;
+  const int s = t % S;
+  const E* w = Ww + (int64_t)ids[t] * H;
+  const E* p = Wp + (int64_t)(pos_offset + s) * H;
+  const E* ty = Wt + (int64_t)tt[t] * H;
+  const int nv = H >> 5;
+  float v[32];
+  float sum = 0.f;
+#pragma unroll
+  for (int k = 0; k < 32; ++k)
+    if (k < nv) {
+      const int c = lane + 32 * k;
+      v[k] = ldf(w + c) + ldf(p + c) + ldf(ty + c);
+      z0[(int64_t)t * H + c] = v[k];
+      sum += v[k];
+    }
+  const float mu = warp_sum(sum) / (float)H;
+  float q = 0.f;
+#pragma unroll
+  for (int k = 0; k < 32; ++k)
+    if (k < nv) { const float d = v[k] - mu; q += d * d; }
+  const float rstd = rsqrtf(warp_sum(q) / (float)H + eps);
+  if (lane == 0) st0[t] = make_float2(mu, rstd);
+#pragma unroll
+  for (int k = 0; k < 32; ++k)
+    if (k < nv) {
+      const int c = lane + 32 * k;
+      const float o = ((v[k] - mu) * rstd * ldf(g + c) + ldf(b + c)) *
+                      drop_factor(drop, (uint64_t)t * H + c);
+      stf(x1 + (int64_t)t * H + c, o);
+    }
+}
+
+void embed_fwd(DType dt, const int32_t* ids, const int32_t* tt, const void* Ww, const void* Wp,
+               const void* Wt, const void* g, const void* b, float* z0, float2* st0, void* x1, int B,
+               int S, int H, int pos_offset, float eps, Drop drop, cudaStream_t s) {
+  const int T = B * S;
+  note_launch(1);
+  dispatch(dt, [&](auto* tag) {
+    using E = std::remove_pointer_t<decltype(tag)>;
+    k_embed_fwd<E><<<cdiv(T, 8), 256, 0, s>>>(ids, tt, (const E*)Ww, (const E*)Wp, (const E*)Wt,
+                                              (const E*)g, (const E*)b, z0, st0, (E*)x1, T, S, H,
+                                              pos_offset, eps, drop);
+  });
+}
+
+// partials [NPART][TV*H]; CTA p owns rows p, p+NPART, ...
+__global__ void __launch_bounds__(256) k_type_part(const float* __restrict__ dz0, const int32_t* __restrict__ tt,
+                                                   int T, int H, int TV, float* __restrict__ part) {
+  float acc[4][4];
+#pragma unroll
+  for (int k = 0; k < 4; ++k)
+#pragma unroll
+    for (int j = 0; j < 4; ++j) acc[k][j] = 0.f;
+  for (int r = blockIdx.x; r < T; r += NPART) {
+    const int key = tt[r];
+#pragma unroll
+    for (int j = 0; j < 4; ++j) {
+      const int c = threadIdx.x + 256 * j;
+      if (c < H) {
+        const float v = dz0[(int64_t)r * H + c];
+#pragma unroll
+        for (int k = 0; k < 4; ++k) acc[k][j] += (k == key) ? v : 0.f;
+      }
+    }
+  }
+  for (int k = 0; k < TV; ++k)
+#pragma unroll
+    for (int j = 0; j < 4; ++j) {
+      const int c = threadIdx.x + 256 * j;
+      if (c < H) part[(int64_t)blockIdx.x * TV * H + (int64_t)k * H + c] = acc[k][j];
+    }
+}
+void type_grad(const float* dz0, const int32_t* tt, int T, int H, int TV, float* part, float* dWt, cudaStream_t s) {
+  note_launch(1);
+  k_type_part<<<NPART, 256, 0, s>>>(dz0, tt, T, H, TV, part);
+  reduce_partials(part, (int64_t)TV * H, TV * H, dWt, s);
+}
+
+__global__ void k_pos_grad(const float* __restrict__ dz0, int B, int S, int H, int pos_offset,
+                           float* __restrict__ dWp) {
+  const int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
+  if (i >= (int64_t)S * H) return;
+  const int s = (int)(i / H), c = (int)(i % H);
+  float acc = 0.f;
+  for (int b = 0; b < B; ++b) acc += dz0[((int64_t)b * S + s) * H + c];
+  dWp[(int64_t)(pos_offset + s) * H + c] = acc;
+}
+void pos_grad(const float* dz0, int B, int S, int H, int pos_offset, float* dWp, cudaStream_t s) {
+  note_launch(1);
+  k_pos_grad<<<cdiv((int64_t)S * H, 256), 256, 0, s>>>(dz0, B, S, H, pos_offset, dWp);
+}
+
+// ---- stable LSD radix sort of (key, token) pairs, 8-bit digits, 1024-key tiles ----
+__global__ void __launch_bounds__(1024) k_rs_hist(const int32_t* __restrict__ keys, int T, int shift,
+                                                  int ntiles, int32_t* __restrict__ hist) {
+  __shared__ int h[256];
+  if (threadIdx.x < 256) h[threadIdx.x] = 0;
+  __syncthreads();
+  const int i = blockIdx.x * 1024 + threadIdx.x;
+  if (i < T) atomicAdd(&h[(keys[i] >> shift) & 0xFF], 1);   // integer counts: order-free
+  __syncthreads();
+  if (threadIdx.x < 256) hist[threadIdx.x * ntiles + blockIdx.x] = h[threadIdx.x];
+}
+
+// exclusive scan of n <= 8192 ints, one CTA of 1024 threads, 8 per thread
+__global__ void __launch_bounds__(1024) k_rs_scan(int32_t* __restrict__ a, int n) {
+  __shared__ int ws[32];
+  int v[8], s = 0;
+  const int base = threadIdx.x * 8;
+#pragma unroll
+  for (int j = 0; j < 8; ++j) { v[j] = base + j < n ? a[base + j] : 0; s += v[j]; }
+  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+  int inc = s;
+#pragma unroll
+  for (int o = 1; o < 32; o <<= 1) { const int t = __shfl_up_sync(0xffffffffu, inc, o); if (lane >= o) inc += t; }
+  if (lane == 31) ws[warp] = inc;
+  __syncthreads();
+  if (warp == 0) {
+    int w = ws[lane], wi = w;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) { const int t = __shfl_up_sync(0xffffffffu, wi, o); if (lane >= o) wi += t; }
+    ws[lane] = wi - w;
+  }
+  __syncthreads();
+  int run = ws[warp] + inc - s;
+#pragma unroll
+  for (int j = 0; j < 8; ++j) {
+    if (base + j < n) a[base + j] = run;
+    run += v[j];
+  }
+}
+
+__global__ void __launch_bounds__(1024) k_rs_scatter(const int32_t* __restrict__ kin, const int32_t* __restrict__ vin,
+                                                     int T, int shift, int ntiles, const int32_t* __restrict__ off,
+                                                     int32_t* __restrict__ kout, int32_t* __restrict__ vout) {
+  __shared__ int wc[32][257];
+  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+  for (int i = threadIdx.x; i < 32 * 257; i += 1024) (&wc[0][0])[i] = 0;
+  __syncthreads();
+  const int i = blockIdx.x * 1024 + threadIdx.x;
+  const bool valid = i < T;
+  const int key = valid ? kin[i] : 0;
+  const int val = valid ? (vin ? vin[i] : i) : 0;
+  const int d = valid ? (key >> shift) & 0xFF : 256 + lane;
+  const unsigned peers = __match_any_sync(0xffffffffu, d);
+  const int rank = __popc(peers & ((1u << lane) - 1u));
+  if (valid && rank == 0) wc[warp][d] = __popc(peers);
+  __syncthreads();
+  if (threadIdx.x < 256) {
+    int run = 0;
+    for (int w = 0; w < 32; ++w) { const int c = wc[w][threadIdx.x]; wc[w][threadIdx.x] = run; run += c; }
+  }
+  __syncthreads();
+  if (valid) {
+    const int pos = off[d * ntiles + blockIdx.x] + wc[warp][d] + rank;
+    kout[pos] = key;
+    vout[pos] = val;
+  }
+}
+
+// piece sums: warp per 32 sorted positions; a piece = a run of equal keys inside the chunk.
+// The piece sum overwrites the X row of the piece's first token (read-before-write, same warp).
+__global__ void __launch_bounds__(256) k_piece_sum(const int32_t* __restrict__ keys, const int32_t* __restrict__ tok,
+                                                   float* X, int T, int H) {
+  const int chunk = (blockIdx.x * blockDim.x + threadIdx.x) >> 5, lane = threadIdx.x & 31;
+  const int r0 = chunk * 32;
+  if (r0 >= T) return;
+  const int r1 = min(r0 + 32, T);
+  for (int c0 = 0; c0 < H; c0 += 32 * 8) {
+    float acc[8];
+    int start = r0;
+#pragma unroll
+    for (int j = 0; j < 8; ++j) acc[j] = 0.f;
+    for (int r = r0; r < r1; ++r) {
+      const float* xr = X + (int64_t)tok[r] * H;
+#pragma unroll
+      for (int j = 0; j < 8; ++j) {
+        const int c = c0 + lane + 32 * j;
+        if (c < H) acc[j] += xr[c];
+      }
+      if (r + 1 == r1 || keys[r + 1] != keys[r]) {
+        float* dst = X + (int64_t)tok[start] * H;
+#pragma unroll
+        for (int j = 0; j < 8; ++j) {
+          const int c = c0 + lane + 32 * j;
+          if (c < H) dst[c] = acc[j];
+          acc[j] = 0.f;
+        }
+        start = r + 1;
+      }
+    }
+  }
+}
+
+// segment sums: warp per sorted position that starts a run of equal keys.
+__global__ void __launch_bounds__(256) k_segment_sum(const int32_t* __restrict__ keys, const int32_t* __restrict__ tok,
+                                                     const float* __restrict__ X, int T, int H, float* __restrict__ out) {
+  const int r = (blockIdx.x * blockDim.x + threadIdx.x) >> 5, lane = threadIdx.x & 31;
+  if (r >= T) return;
+  const int key = keys[r];
+  if (r > 0 && keys[r - 1] == key) return;
+  int end = r + 1;
+  while (end < T && keys[end] == key) ++end;
+  for (int c = lane; c < H; c += 32) {
+    float acc = X[(int64_t)tok[r] * H + c];
+    for (int q = (r / 32 + 1) * 32; q < end; q += 32) acc += X[(int64_t)tok[q] * H + c];
+    out[(int64_t)key * H + c] = acc;
+  }
+}
+
+void keyed_rowsum(const int32_t* keys, int key_bits, float* X, int T, int H, float* out,
+                  int32_t* work, int32_t* hist, int max_tiles, cudaStream_t s) {
+  const int ntiles = cdiv(T, 1024);
+  int32_t *kA = work, *vA = work + T, *kB = work + 2 * T, *vB = work + 3 * T;
+  const int passes = key_bits <= 8 ? 1 : 2;
+  const int32_t* kin = keys;
+  const int32_t* vin = nullptr;
+  for (int p = 0; p < passes; ++p) {
+    int32_t* ko = (p == 0) ? kB : kA;
+    int32_t* vo = (p == 0) ? vB : vA;
+    k_rs_hist<<<ntiles, 1024, 0, s>>>(kin, T, 8 * p, ntiles, hist);
+    k_rs_scan<<<1, 1024, 0, s>>>(hist, 256 * ntiles);
+    k_rs_scatter<<<ntiles, 1024, 0, s>>>(kin, vin, T, 8 * p, ntiles, hist, ko, vo);
+    kin = ko;
+    vin = vo;
+  }
+  (void)max_tiles;
+  note_launch(3 * passes + 2);
+  k_piece_sum<<<cdiv(cdiv(T, 32), 8), 256, 0, s>>>(kin, vin, X, T, H);
+  k_segment_sum<<<cdiv(T, 8), 256, 0, s>>>(kin, vin, X, T, H, out);
+}
+
+// ================================================================== heads ===
+
+template <typename E>
+__global__ void k_pool_fwd(const E* __restrict__ y, int B, int S, int H, const E* __restrict__ Wp,
+                           const E* __restrict__ bp, E* __restrict__ p) {
+  const int w = (blockIdx.x * blockDim.x + threadIdx.x) >> 5, lane = threadIdx.x & 31;
+  if (w >= B * H) return;
+  const int b = w / H, j = w % H;
+  const E* yr = y + (int64_t)b * S * H;
+  const E* wr = Wp + (int64_t)j * H;
+  float acc = 0.f;
+  for (int k = lane; k < H; k += 32) acc += ldf(yr + k) * ldf(wr + k);
+  acc = warp_sum(acc);
+  if (lane == 0) stf(p + (int64_t)b * H + j, tanhf(acc + ldf(bp + j)));
+}
+
+template <typename E>
+__global__ void k_cls_fwd(const E* __restrict__ p, int B, int H, const E* __restrict__ Wc,
+                          const E* __restrict__ bc, int n_out, float* __restrict__ logits, Drop drop) {
+  const int w = (blockIdx.x * blockDim.x + threadIdx.x) >> 5, lane = threadIdx.x & 31;
+  if (w >= B * n_out) return;
+  const int b = w / n_out, o = w % n_out;
+  float acc = 0.f;
+  for (int j = lane; j < H; j += 32)
+    acc += ldf(p + (int64_t)b * H + j) * drop_factor(drop, (uint64_t)b * H + j) * ldf(Wc + (int64_t)o * H + j);
+  acc = warp_sum(acc);
+  if (lane == 0) logits[b * n_out + o] = acc + ldf(bc + o);
+}
+
+// rows x cols view of the logits for the CE: MC [B/C, C], seq-cls [B, n_out]
+__device__ void ce_view(int head_kind, int B, int n_out, int n_choices, int& rows, int& cols) {
+  if (head_kind == 1) { rows = B / n_choices; cols = n_choices; } else { rows = B; cols = n_out; }
+}
+
+// loss (fwd) or dlogits (bwd): one warp, rows processed in order.
+__global__ void k_cls_ce(const float* __restrict__ logits, const int32_t* __restrict__ labels, int B,
+                         int n_out, int n_choices, int head_kind, float* __restrict__ loss,
+                         float* __restrict__ dlog) {
+  int rows, cols;
+  ce_view(head_kind, B, n_out, n_choices, rows, cols);
+  const int lane = threadIdx.x;
+  float total = 0.f;
+  for (int r = 0; r < rows; ++r) {
+    const float* lr = logits + (int64_t)r * cols;
+    float m = -INFINITY;
+    for (int c = lane; c < cols; c += 32) m = fmaxf(m, lr[c]);
+    m = warp_max(m);
+    float z = 0.f;
+    for (int c = lane; c < cols; c += 32) z += expf(lr[c] - m);
+    z = warp_sum(z);
+    const float lse = m + logf(z);
+    total += lse - lr[labels[r]];
+    if (dlog)
+      for (int c = lane; c < cols; c += 32)
+        dlog[(int64_t)r * cols + c] = (expf(lr[c] - lse) - (c == labels[r] ? 1.f : 0.f)) / (float)rows;
+  }
+  if (loss && lane == 0) *loss = total / (float)rows;
+}
+
+void head_cls_fwd(DType dt, const void* y, int B, int S, int H, const void* Wp, const void* bp,
+                  const void* Wc, const void* bc, int n_out, void* p, float* logits,
+                  const int32_t* labels, int n_choices, int head_kind, float* loss, Drop drop,
+                  cudaStream_t s) {
+  note_launch(3);
+  dispatch(dt, [&](auto* tag) {
+    using E = std::remove_pointer_t<decltype(tag)>;
+    k_pool_fwd<E><<<cdiv((int64_t)B * H, 8), 256, 0, s>>>((const E*)y, B, S, H, (const E*)Wp, (const E*)bp, (E*)p);
+    k_cls_fwd<E><<<cdiv((int64_t)B * n_out, 8), 256, 0, s>>>((const E*)p, B, H, (const E*)Wc, (const E*)bc, n_out, logits, drop);
+  });
+  k_cls_ce<<<1, 32, 0, s>>>(logits, labels, B, n_out, n_choices, head_kind, loss, nullptr);
+}
+
+template <typename E>
+__global__ void k_cls_wgrad(const float* __restrict__ dlog, const E* __restrict__ p, int B, int H, int n_out,
+                            float* __restrict__ dWc, float* __restrict__ dbc, Drop drop) {
+  const int i = blockIdx.x * blockDim.x + threadIdx.x;
+  if (i < n_out * H) {
+    const int o = i / H, j = i % H;
+    float acc = 0.f;
+    for (int b = 0; b < B; ++b)
+      acc += dlog[b * n_out + o] * ldf(p + (int64_t)b * H + j) * drop_factor(drop, (uint64_t)b * H + j);
+    dWc[i] = acc;
+  }
+  if (i < n_out) {
+    float acc = 0.f;
+    for (int b = 0; b < B; ++b) acc += dlog[b * n_out + i];
+    dbc[i] = acc;
+  }
+}
+
+template <typename E>
+__global__ void k_pool_dpre(const float* __restrict__ dlog, const E* __restrict__ p, const E* __restrict__ Wc,
+                            int B, int H, int n_out, float* __restrict__ dpre, Drop drop) {
+  const int i = blockIdx.x * blockDim.x + threadIdx.x;
+  if (i >= B * H) return;
+  const int b = i / H, j = i % H;
+  float acc = 0.f;
+  for (int o = 0; o < n_out; ++o) acc += dlog[b * n_out + o] * ldf(Wc + (int64_t)o * H + j);
+  const float pv = ldf(p + i);
+  dpre[i] = acc * drop_factor(drop, (uint64_t)b * H + j) * (1.f - pv * pv);
+}
+
+template <typename E>
+__global__ void k_pool_wgrad(const float* __restrict__ dpre, const E* __restrict__ y, int B, int S, int H,
+                             float* __restrict__ dWp, float* __restrict__ dbp) {
+  const int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
+  if (i < (int64_t)H * H) {
+    const int j = (int)(i / H), k = (int)(i % H);
+    float acc = 0.f;
+    for (int b = 0; b < B; ++b) acc += dpre[b * H + j] * ldf(y + (int64_t)b * S * H + k);
+    dWp[i] = acc;
+  }
+  if (i < H) {
+    float acc = 0.f;
+    for (int b = 0; b < B; ++b) acc += dpre[b * H + i];
+    dbp[i] = acc;
+  }
+}
+
+template <typename E>
+__global__ void k_pool_dx(const float* __restrict__ dpre, const E* __restrict__ Wp, int B, int S, int H,
+                          float* __restrict__ dy) {
+  const int i = blockIdx.x * blockDim.x + threadIdx.x;
+  if (i >= B * H) return;
+  const int b = i / H, k = i % H;
+  float acc = 0.f;
+  for (int j = 0; j < H; ++j) acc += dpre[b * H + j] * ldf(Wp + (int64_t)j * H + k);
+  dy[(int64_t)b * S * H + k] = acc;
+}
+
+void head_cls_bwd(DType dt, const void* y, int B, int S, int H, const void* Wp, const void* Wc, int n_out,
+                  const void* p, const float* logits, const int32_t* labels, int n_choices, int head_kind,
+                  float* scratch, float* dWp, float* dbp, float* dWc, float* dbc, float* dy, Drop drop,
+                  cudaStream_t s) {
+  float* dlog = scratch;
+  note_launch(5);
+  float* dpre = scratch + ((B * n_out + 3) / 4 * 4) + (int64_t)B * H;
+  k_cls_ce<<<1, 32, 0, s>>>(logits, labels, B, n_out, n_choices, head_kind, nullptr, dlog);
+  dispatch(dt, [&](auto* tag) {
+    using E = std::remove_pointer_t<decltype(tag)>;
+    k_cls_wgrad<E><<<cdiv(n_out * H, 256), 256, 0, s>>>(dlog, (const E*)p, B, H, n_out, dWc, dbc, drop);
+    k_pool_dpre<E><<<cdiv(B * H, 256), 256, 0, s>>>(dlog, (const E*)p, (const E*)Wc, B, H, n_out, dpre, drop);
+    k_pool_wgrad<E><<<cdiv((int64_t)H * H, 256), 256, 0, s>>>(dpre, (const E*)y, B, S, H, dWp, dbp);
+    k_pool_dx<E><<<cdiv(B * H, 256), 256, 0, s>>>(dpre, (const E*)Wp, B, S, H, dy);
+  });
+}
+
+// ---- QA span head ----
+template <typename E>
+__global__ void k_qa_logits(const E* __restrict__ y, int T, int H, const E* __restrict__ Wq,
+                            const E* __restrict__ bq, float* __restrict__ logits) {
+  const int t = (blockIdx.x * blockDim.x + threadIdx.x) >> 5, lane = threadIdx.x & 31;
+  if (t >= T) return;
+  float a0 = 0.f, a1 = 0.f;
+  for (int c = lane; c < H; c += 32) {
+    const float v = ldf(y + (int64_t)t * H + c);
+    a0 += v * ldf(Wq + c);
+    a1 += v * ldf(Wq + H + c);
+  }
+  a0 = warp_sum(a0);
+  a1 = warp_sum(a1);
+  if (lane == 0) { logits[2 * t] = a0 + ldf(bq); logits[2 * t + 1] = a1 + ldf(bq + 1); }
+}
+
+// one warp; per sequence b and side j: masked softmax CE over s < len
+__global__ void k_qa_ce(const float* __restrict__ logits, const int32_t* __restrict__ lengths,
+                        const int32_t* __restrict__ labels, int B, int S, float* __restrict__ loss,
+                        float* __restrict__ dlog) {
+  const int lane = threadIdx.x;
+  float tot[2] = {0.f, 0.f};
+  for (int b = 0; b < B; ++b) {
+    const int len = lengths[b];
+    for (int j = 0; j < 2; ++j) {
+      float m = -INFINITY;
+      for (int s = lane; s < len; s += 32) m = fmaxf(m, logits[2 * (b * S + s) + j]);
+      m = warp_max(m);
+      float z = 0.f;
+      for (int s = lane; s < len; s += 32) z += expf(logits[2 * (b * S + s) + j] - m);
+      z = warp_sum(z);
+      const float lse = m + logf(z);
+      const int lab = labels[2 * b + j];
+      tot[j] += lse - logits[2 * (b * S + lab) + j];
+      if (dlog)
+        for (int s = lane; s < S; s += 32)
+          dlog[2 * (b * S + s) + j] =
+              s < len ? 0.5f * (expf(logits[2 * (b * S + s) + j] - lse) - (s == lab ? 1.f : 0.f)) / (float)B : 0.f;
+    }
+  }
+  if (loss && lane == 0) *loss = 0.5f * (tot[0] / (float)B + tot[1] / (float)B);
+}
+
+void head_qa_fwd(DType dt, const void* y, int B, int S, int H, const void* Wq, const void* bq, float* logits,
+                 const int32_t* lengths, const int32_t* labels, float* loss, cudaStream_t s) {
+  const int T = B * S;
+  note_launch(2);
+  dispatch(dt, [&](auto* tag) {
+    using E = std::remove_pointer_t<decltype(tag)>;
+    k_qa_logits<E><<<cdiv(T, 8), 256, 0, s>>>((const E*)y, T, H, (const E*)Wq, (const E*)bq, logits);
+  });
+  k_qa_ce<<<1, 32, 0, s>>>(logits, lengths, labels, B, S, loss, nullptr);
+}
+
+template <typename E>
+__global__ void k_qa_dx(const float* __restrict__ dlog, const E* __restrict__ Wq, int T, int H, float* __restrict__ dy) {
+  const int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
+  if (i >= (int64_t)T * H) return;
+  const int t = (int)(i / H), c = (int)(i % H);
+  dy[i] = dlog[2 * t] * ldf(Wq + c) + dlog[2 * t + 1] * ldf(Wq + H + c);
+}
+
+// partials [NPART][2H + 2]: dWq rows then dbq
+template <typename E>
+__global__ void k_qa_wgrad_part(const float* __restrict__ dlog, const E* __restrict__ y, int T, int H,
+                                float* __restrict__ part) {
+  const int ld = 2 * H + 2;
+  for (int c = threadIdx.x; c < ld; c += blockDim.x) {
+    float acc = 0.f;
+    for (int t = blockIdx.x; t < T; t += NPART) {
+      if (c < 2 * H) acc += dlog[2 * t + c / H] * ldf(y + (int64_t)t * H + c % H);
+      else acc += dlog[2 * t + (c - 2 * H)];
+    }
+    part[(int64_t)blockIdx.x * ld + c] = acc;
+  }
+}
+
+void head_qa_bwd(DType dt, const void* y, int B, int S, int H, const void* Wq, const float* logits,
+                 const int32_t* lengths, const int32_t* labels, float* dlog, float* part, float* dWq,
+                 float* dbq, float* dy, cudaStream_t s) {
+  const int T = B * S;
+  note_launch(3);
+  k_qa_ce<<<1, 32, 0, s>>>(logits, lengths, labels, B, S, nullptr, dlog);
+  dispatch(dt, [&](auto* tag) {
+    using E = std::remove_pointer_t<decltype(tag)>;
+    k_qa_dx<E><<<cdiv((int64_t)T * H, 256), 256, 0, s>>>(dlog, (const E*)Wq, T, H, dy);
+    k_qa_wgrad_part<E><<<NPART, 256, 0, s>>>(dlog, (const E*)y, T, H, part);
+  });
+  reduce_partials(part, 2 * H + 2, 2 * H, dWq, s);
+  reduce_partials(part + 2 * H, 2 * H + 2, 2, dbq, s);
+}
+
+// ============================================================== optimizer ===
+
+template <typename E>
+__global__ void k_adamw(E* __restrict__ w, float* __restrict__ master, const float* __restrict__ g,
+                        float* __restrict__ m, float* __restrict__ v, int64_t n, float lr, float b1,
+                        float b2, float eps, float wd, float bc1, float bc2, float gs) {
+  const float step = lr / bc1, rb2 = 1.0f / sqrtf(bc2), decay = 1.0f - lr * wd;
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
+    const float gi = g[i] * gs;
+    float p = master ? master[i] : ldf(w + i);
+    p *= decay;
+    const float mi = b1 * m[i] + (1.f - b1) * gi;
+    const float vi = b2 * v[i] + (1.f - b2) * gi * gi;
+    p -= step * mi / (sqrtf(vi) * rb2 + eps);
+    m[i] = mi;
+    v[i] = vi;
+    if (master) master[i] = p;
+    stf(w + i, p);
+  }
+}
+
+void adamw(DType dt, void* w, float* master, const float* g, float* m, float* v, int64_t n, float lr,
+           float b1, float b2, float eps, float wd, float bc1, float bc2, float gs, cudaStream_t s) {
+  note_launch(1);
+  dispatch(dt, [&](auto* tag) {
+    using E = std::remove_pointer_t<decltype(tag)>;
+    k_adamw<E><<<148 * 8, 256, 0, s>>>((E*)w, master, g, m, v, n, lr, b1, b2, eps, wd, bc1, bc2, gs);
+  });
+}
+
+template <typename E>
+__global__ void k_cast_from(const float* __restrict__ src, E* __restrict__ dst, int64_t n) {
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x)
+    stf(dst + i, src[i]);
+}
+template <typename E>
+__global__ void k_cast_to(const E* __restrict__ src, float* __restrict__ dst, int64_t n) {
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x)
+    dst[i] = ldf(src + i);
+}
+void cast_from_f32(DType dt, const float* src, void* dst, int64_t n, cudaStream_t s) {
+  note_launch(1);
+  dispatch(dt, [&](auto* tag) {
+    using E = std::remove_pointer_t<decltype(tag)>;
+    k_cast_from<E><<<592, 256, 0, s>>>(src, (E*)dst, n);
+  });
+}
+void cast_to_f32(DType dt, const void* src, float* dst, int64_t n, cudaStream_t s) {
+  note_launch(1);
+  dispatch(dt, [&](auto* tag) {
+    using E = std::remove_pointer_t<decltype(tag)>;
+    k_cast_to<E><<<592, 256, 0, s>>>((const E*)src, dst, n);
+  });
+}
+
+}  // namespace mimose

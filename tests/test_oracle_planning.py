@@ -107,11 +107,12 @@ def test_collected_series_and_predicted_peak_formula(name):
 
 
 def test_bert_base_saved_bytes_per_token():
-    """(8H+2F)e + 4h + 16 bytes per token per kept layer."""
+    """SURVEY §8(a) a7 layout with the pre-LN sums z1, z2 in fp32 (reading R-P):
+    (6H + 2F) e + 2*4H + 4h + 16 bytes per token per kept layer."""
     cfg = wl.CONFIGS["bert-base"]
     sz = om.sizes(cfg, 64, 128)
     T = 64 * 128
-    assert sz.a == T * ((8 * 768 + 2 * 3072) * 2 + 4 * 12 + 16)
+    assert sz.a == T * ((6 * 768 + 2 * 3072) * 2 + 2 * 4 * 768 + 4 * 12 + 16)
 
 
 # ---------------------------------------------------------- estimator -----
