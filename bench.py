@@ -1,0 +1,395 @@
+#!/usr/bin/env python
+"""Throughput of the Mimose checkpointed training step under a fixed memory
+budget with a dynamic sequence length (BASELINE.json metric), on N GPUs.
+
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--config bert-base]
+    python bench.py --impl reference ...      # the fp64 CPU oracle arm
+
+One step = Mimose plan lookup (estimator + Algorithm 1 on a cache miss)
++ forward + backward with recompute + AdamW, on one synthetic SWAG-like batch
+(DESIGN "Input recipe").  The sheltered phase (collect_iters shuttled
+iterations) runs before the warm-up and is reported separately.
+Multi-GPU: one process per GPU (torchrun), weak scaling, the same S_t on every
+rank, per-layer NCCL gradient all-reduce overlapped with backward.
+Prints ONE JSON line on rank 0.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import subprocess
+import sys
+import threading
+import time
+
+import numpy as np
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+from paper_conf_ipps_liaolysshfyctzlq23_b200 import workload as wl  # noqa: E402
+
+METRIC = "samples/sec under fixed memory budget, dynamic seq len, 1/2/4/8 B200"
+
+
+def parse():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=30)
+    ap.add_argument("--warmup", type=int, default=5)
+    ap.add_argument("--impl", default="mimose", choices=["mimose", "reference"])
+    ap.add_argument("--config", default="bert-base", choices=sorted(wl.CONFIGS))
+    ap.add_argument("--no-baselines", action="store_true", help="skip static-plan / no-ckpt arms")
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--simt", action="store_true", help="SIMT GEMMs instead of tcgen05")
+    return ap.parse_args()
+
+
+def peaks():
+    p = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    if os.path.exists(p):
+        d = json.load(open(p))
+        return d, "measured"
+    return {"hbm_gbs": 6650.0, "bf16_tflops": 1590.0, "bf16_tflops_sustained": 1400.0,
+            "sm_max_mhz": 1965.0}, "fallback"
+
+
+class Clocks:
+    """nvidia-smi sampler for the timed region (B200_PROFILING.md clocks line)."""
+    Q = ("index,clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,"
+         "clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
+         "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, dev: int):
+        self.dev, self.rows, self.stop = dev, [], threading.Event()
+
+    def _run(self):
+        while not self.stop.is_set():
+            try:
+                out = subprocess.run(["nvidia-smi", "-i", str(self.dev), "--query-gpu=" + self.Q,
+                                      "--format=csv,noheader,nounits"], capture_output=True,
+                                     text=True, timeout=5).stdout.strip()
+                if out:
+                    self.rows.append([t.strip() for t in out.split(",")])
+            except Exception:
+                pass
+            self.stop.wait(0.2)
+
+    def __enter__(self):
+        self.t = threading.Thread(target=self._run, daemon=True)
+        self.t.start()
+        return self
+
+    def __exit__(self, *a):
+        self.stop.set()
+        self.t.join(10)
+
+    def summary(self):
+        if not self.rows:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["no samples"]}
+        sm = [float(r[1]) for r in self.rows if r[1].replace(".", "").isdigit()]
+        mx = [float(r[2]) for r in self.rows if r[2].replace(".", "").isdigit()]
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        reasons = sorted({n for r in self.rows for n, v in zip(names, r[5:9]) if v.lower() == "active"})
+        return {"sm_mhz": float(np.median(sm)) if sm else None, "sm_max_mhz": max(mx) if mx else None,
+                "reasons": reasons, "samples": len(self.rows)}
+
+
+def dist_env():
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    return world, rank, local
+
+
+# ---------------------------------------------------------------------------
+# reference arm: the fp64 CPU oracle (DESIGN "Measurement")
+# ---------------------------------------------------------------------------
+
+def oracle_sample_step(cfg, S_longest, n_q, step):
+    """One oracle training step on a bounded sample: n_q questions of the workload."""
+    from oracle import model as om
+    sub = wl.small_config(cfg.name, n_seqs=n_q * (cfg.n_choices if cfg.head == wl.HEAD_MC else 1))
+    params = ORACLE_PARAMS.setdefault(cfg.name, wl.init_params(cfg))
+    b = wl.make_batch(sub, S_longest, seed=wl.batch_seed(cfg, step))
+    t0 = time.perf_counter()
+    loss, G = om.train_step_grads(sub, params, b, wl.dropout_seed(cfg), step + 1)
+    zeros = {k: np.zeros_like(v, np.float64) for k, v in G.items()}
+    om.adamw(params, G, zeros, dict(zeros), 1, 1e-4)
+    return time.perf_counter() - t0, n_q if cfg.head == wl.HEAD_MC else b.n_seqs
+
+
+ORACLE_PARAMS: dict = {}
+
+
+def cpu_baseline(cfg, n_steps=1, n_q=2):
+    S = wl.roundup((cfg.seq_lo + cfg.seq_hi) // 2, cfg.pad)
+    tot_t, tot_s = 0.0, 0
+    for i in range(n_steps):
+        t, s = oracle_sample_step(cfg, S, n_q, i)
+        tot_t += t
+        tot_s += s
+    unit = "questions" if cfg.head == wl.HEAD_MC else "sequences"
+    return {"value": tot_s / tot_t, "unit": "samples/s", "cores": len(os.sched_getaffinity(0)),
+            "kind": "oracle",
+            "sample": f"{n_steps} fp64 numpy training step(s) of {n_q} {unit} at S_pad={S} "
+                      f"({cfg.name}, full width/depth), {tot_t:.1f} s"}
+
+
+def run_reference(args):
+    world, rank, _ = dist_env()
+    if rank != 0:
+        return
+    cfg = wl.CONFIGS[args.config]
+    sched = wl.length_schedule(cfg, args.warmup + args.steps)
+    n_q = 1
+    for i in range(args.warmup):
+        oracle_sample_step(cfg, sched[i], n_q, i)
+    tot_t, tot_s = 0.0, 0
+    for i in range(args.steps):
+        t, s = oracle_sample_step(cfg, sched[args.warmup + i], n_q, args.warmup + i)
+        tot_t += t
+        tot_s += s
+    v = tot_s / tot_t
+    sample = f"per step {n_q} questions of the {cfg.name} workload at the schedule's S_t (fp64 numpy)"
+    line = {"impl": "reference", "metric": METRIC, "value": v, "unit": "samples/s", "n_gpus": args.gpus,
+            "steps": args.steps, "warmup": args.warmup, "ms_per_step": 1000 * tot_t / args.steps,
+            "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "f64",
+            "data": "synthetic", "config": {"workload": cfg.name},
+            "cpu_baseline": {"value": v, "unit": "samples/s", "cores": len(os.sched_getaffinity(0)),
+                             "kind": "oracle", "sample": sample},
+            "e2e": {"value": v, "unit": "samples/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+    print(json.dumps(line), flush=True)
+
+
+# ---------------------------------------------------------------------------
+# Mimose arm
+# ---------------------------------------------------------------------------
+
+def main():
+    args = parse()
+    if args.impl == "reference":
+        return run_reference(args)
+    import torch
+    import torch.distributed as dist
+    from paper_conf_ipps_liaolysshfyctzlq23_b200 import binding as mb
+
+    world, rank, local = dist_env()
+    torch.cuda.set_device(local)
+    if world > 1:
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+    cfg = wl.CONFIGS[args.config]
+    stream = torch.cuda.current_stream()
+    use_tc = 0 if args.simt else 1
+
+    # ---- budget (D2 / reading A21) from the library's own allocation sequence ----
+    probe_ctx = mb.Mimose(cfg, 0)
+    C0 = probe_ctx.stats()["persistent_bytes"]
+    P0 = probe_ctx.dry_run(cfg.n_seqs, cfg.max_seq, [])
+    LB = probe_ctx.dry_run(cfg.n_seqs, cfg.max_seq, range(cfg.n_layers))
+    M = max(C0 + int(cfg.budget_frac * (P0 - C0)), LB)
+    probe_ctx.close()
+
+    nccl_id = None
+    if world > 1:
+        t = torch.zeros(128, dtype=torch.uint8, device="cuda")
+        if rank == 0:
+            t.copy_(torch.frombuffer(bytearray(mb.nccl_unique_id()), dtype=torch.uint8))
+        dist.broadcast(t, 0)
+        nccl_id = bytes(t.cpu().numpy().tolist())
+
+    def new_ctx(budget, slab_bytes, enforce=1):
+        slab = torch.empty(slab_bytes, dtype=torch.uint8, device="cuda")
+        ctx = mb.Mimose(cfg, budget, slab=slab, stream=stream, rank=rank, world=world,
+                        nccl_id=nccl_id, enforce_budget=enforce, use_tc=use_tc)
+        ctx.set_params(wl.pack_params(cfg, wl.init_params(cfg)))
+        return ctx
+
+    n_total = args.warmup + args.steps
+    sched = wl.length_schedule(cfg, 10 + n_total)      # shared by every rank (same S_t)
+
+    def host_batches(offset):
+        return [wl.make_batch(cfg, sched[offset + i], seed=wl.batch_seed(cfg, offset + i, rank))
+                for i in range(n_total)]
+
+    def to_dev(b):
+        return [torch.tensor(np.ascontiguousarray(x, np.int32)).cuda() for x in
+                (b.input_ids, b.token_type, b.lengths, b.labels)]
+
+    def barrier():
+        torch.cuda.synchronize()
+        if world > 1:
+            dist.barrier()
+
+    def timed(ctx, batches, mode, plan_fixed=None, host=False, clocks=None, probe=False):
+        """Runs warm-up then the timed steps; returns device ms (max over ranks)."""
+        dev = None if host else [to_dev(b) for b in batches]
+        pinned = None
+        if host:
+            pinned = []
+            for b in batches:
+                ts = [torch.from_numpy(np.ascontiguousarray(x, np.int32)).pin_memory() for x in
+                      (b.input_ids, b.token_type, b.lengths, b.labels)]
+                pinned.append(ts)
+
+        def one(i):
+            b = batches[i]
+            bs = (mb.Mimose.batch_struct(*pinned[i], b.n_seqs, b.seq_len, True) if host else
+                  mb.Mimose.batch_struct(*dev[i], b.n_seqs, b.seq_len, False))
+            if mode == "mimose":
+                p = ctx.plan(b.input_size)
+            elif mode == "static":
+                p = plan_fixed
+            else:
+                p = None
+            ctx.forward(bs, p, want_loss=host)
+            ctx.backward()
+            ctx.step(1e-5)
+
+        for i in range(args.warmup):
+            one(i)
+        barrier()
+        if probe:
+            ctx.probe(1)
+        launches0 = ctx.stats()["kernel_launches"]
+        ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        ev0.record(stream)
+        if clocks:
+            clocks.__enter__()
+        for i in range(args.warmup, n_total):
+            one(i)
+        ev1.record(stream)
+        barrier()
+        if clocks:
+            clocks.__exit__()
+        ms = ev0.elapsed_time(ev1)
+        launches = ctx.stats()["kernel_launches"] - launches0
+        pr = ctx.probe_read() if probe else None
+        if probe:
+            ctx.probe(0)
+        if world > 1:
+            t = torch.tensor([ms], device="cuda")
+            dist.all_reduce(t, op=dist.ReduceOp.MAX)
+            ms = float(t.item())
+        return ms, launches, pr
+
+    samples_per_step = cfg.samples_per_step * world
+
+    # ---- Mimose: sheltered phase, then the timed responsive steps ----
+    ctx = new_ctx(M, M)
+    t0 = time.perf_counter()
+    i = 0
+    while ctx.phase == mb.PHASE_SHELTERED:
+        b = wl.make_batch(cfg, sched[i % len(sched)], seed=wl.batch_seed(cfg, 10**6 + i, rank))
+        ctx.collect(ctx.host_batch(b), want_loss=False)
+        ctx.backward()
+        ctx.step(1e-5)
+        i += 1
+    torch.cuda.synchronize()
+    sheltered_s = time.perf_counter() - t0
+    batches = host_batches(10)
+    clocks = Clocks(local)
+    ms, launches, pr = timed(ctx, batches, "mimose", clocks=clocks, probe=True)
+    st = ctx.stats()
+    value = samples_per_step * args.steps / (ms / 1000.0)
+    # e2e: host buffers through the public API; H2D + loss D2H inside the timed region
+    ms_e2e, _, _ = timed(ctx, batches, "mimose", host=True)
+    e2e = samples_per_step * args.steps / (ms_e2e / 1000.0)
+    per_step_h2d = int(np.mean([(b.input_ids.size * 2 + b.lengths.size + b.labels.size) * 4 for b in batches]))
+    st2 = ctx.stats()
+    dropped = []
+    for b in batches[args.warmup:]:
+        dropped.append(ctx.plan(b.input_size).n_dropped)
+    samples = [ctx.sample(j) for j in range(st["n_samples"])]
+    t_ms = [np.mean(s["t_ms"]) for s in samples]
+
+    pk, kind = peaks()
+    gemm_ms, gemm_flops, gemm_n = pr
+    tc = use_tc == 1 and mb.tc_gemm_available()
+    if tc:
+        bound, peak, unit = "tensor", float(pk.get("bf16_tflops_sustained", pk["bf16_tflops"])), "TFLOP/s"
+        peak_note = f"bf16_tflops_sustained ({kind})"
+    else:
+        # SIMT fp32 FMA: 148 SMs x 128 lanes x 2 FLOP x sm_max clock
+        peak = 148 * 128 * 2 * float(pk.get("sm_max_mhz", 1965.0)) * 1e6 / 1e12
+        bound, unit = "alu", "TFLOP/s"
+        peak_note = f"FP32 FMA: 148 SM x 128 lanes x 2 x {pk.get('sm_max_mhz', 1965.0)} MHz ({kind} clock)"
+    achieved = gemm_flops / (gemm_ms / 1000.0) / 1e12 if gemm_ms > 0 else 0.0
+    roofline = {"bound": bound, "achieved": achieved, "peak": peak, "unit": unit,
+                "frac": achieved / peak if peak else None, "traffic": None,
+                "kernel": "GEMM (all linear layers: fwd, dgrad, wgrad)",
+                "peak_source": peak_note, "launches": gemm_n,
+                "share_of_step": gemm_ms / ms if ms else None,
+                "flops_per_launch": gemm_flops / max(gemm_n, 1)}
+
+    result = {
+        "metric": METRIC, "value": value, "unit": "samples/s", "n_gpus": world, "steps": args.steps,
+        "warmup": args.warmup, "ms_per_step": ms / args.steps, "higher_is_better": True,
+        "scaling": "weak", "vs_baseline": None, "dtype": "bf16" if cfg.dtype == "bf16" else "f32",
+        "data": "synthetic",
+        "config": {"workload": cfg.name, "task": "SWAG-like multiple choice" if cfg.head == wl.HEAD_MC else "span QA",
+                   "batch_per_gpu": cfg.n_seqs, "samples_per_gpu_step": cfg.samples_per_step,
+                   "seq_len": f"U[{cfg.seq_lo},{cfg.seq_hi}] pad {cfg.pad}", "budget_frac": cfg.budget_frac,
+                   "budget_bytes": M, "persistent_bytes": C0, "no_ckpt_peak_at_max": P0,
+                   "lower_bound_at_max": LB, "parallelism": f"dp{world}",
+                   "l2": "no flush: per-step working set (weights+grads+optimizer >= 1.9 GB, activations) >> 126 MB L2",
+                   "gemm": "tcgen05" if tc else "simt"},
+        "roofline": roofline,
+        "e2e": {"value": e2e, "unit": "samples/s", "h2d_bytes_per_step": per_step_h2d, "d2h_bytes_per_step": 4},
+        "gpu_launches": launches,
+        "clocks": clocks.summary(),
+        "mimose": {"violations": st2["violations"], "peak_bytes_max": st2["max_peak_bytes"],
+                   "budget_bytes": M, "mean_layers_dropped": float(np.mean(dropped)),
+                   "plan_cache_hits": st2["plan_cache_hits"], "plan_cache_misses": st2["plan_cache_misses"],
+                   "planner_us_total": st2["planner_us_total"], "sheltered_iters": st2["collect_steps"],
+                   "shuttled_iters": st2["shuttled_steps"], "sheltered_s": sheltered_s,
+                   "collector_layer_fwd_ms_mean": float(np.mean(t_ms)) if t_ms else None},
+    }
+    ctx.close()
+    del ctx
+    torch.cuda.empty_cache()
+
+    if not args.no_baselines:
+        # static largest-input plan (Sublinear-style conservatism)
+        ctx = new_ctx(M, M)
+        while ctx.phase == mb.PHASE_SHELTERED:
+            b = wl.make_batch(cfg, sched[ctx.stats()["collect_steps"] % len(sched)], seed=5)
+            ctx.collect(ctx.host_batch(b), want_loss=False)
+            ctx.backward()
+            ctx.step(1e-5)
+        pstatic = ctx.plan(cfg.n_seqs * cfg.max_seq)
+        ms_s, _, _ = timed(ctx, batches, "static", plan_fixed=pstatic)
+        ctx.close()
+        del ctx
+        torch.cuda.empty_cache()
+        # no checkpointing, budget not enforced (reports the peak it needs)
+        ctx = new_ctx(M, P0 + (1 << 20), enforce=0)
+        ms_n, _, _ = timed(ctx, batches, "none")
+        peak_n = ctx.stats()["max_peak_bytes"]
+        ctx.close()
+        del ctx
+        result["static_plan"] = {"value": samples_per_step * args.steps / (ms_s / 1000.0),
+                                 "ms_per_step": ms_s / args.steps, "layers_dropped": pstatic.n_dropped}
+        result["no_ckpt"] = {"value": samples_per_step * args.steps / (ms_n / 1000.0),
+                             "ms_per_step": ms_n / args.steps, "peak_bytes": peak_n,
+                             "over_budget": peak_n > M}
+        result["recompute_ratio"] = ms / ms_n
+        result["speedup_vs_static"] = ms_s / ms
+        result["paper_context"] = ("V100 (P:227): Mimose ~18.0% faster than Sublinear, ~15.0% than DTR "
+                                   "(P:252-254); 2.6% slower than no-checkpoint at 8 GB (P:258)")
+
+    if rank == 0 and world == 1 and not args.no_cpu_baseline:
+        try:
+            result["cpu_baseline"] = cpu_baseline(cfg)
+        except Exception as e:  # never let the reported baseline kill the line
+            result["cpu_baseline"] = {"value": None, "error": str(e)[:200], "kind": "oracle"}
+    if rank == 0:
+        print(json.dumps(result), flush=True)
+    if world > 1:
+        dist.barrier()
+        dist.destroy_process_group()
+
+
+if __name__ == "__main__":
+    main()

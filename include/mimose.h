@@ -217,6 +217,21 @@ mimose_status mimose_dry_run(mimose_ctx* ctx, int32_t n_seqs, int32_t seq_len,
 mimose_status mimose_dry_collect(mimose_ctx* ctx, int32_t n_seqs, int32_t seq_len,
                                  mimose_sample* out);
 
+/* Writes a fresh 128-byte ncclUniqueId (rank 0 calls it and broadcasts the
+   bytes through the caller's process group before mimose_init on every rank). */
+mimose_status mimose_nccl_unique_id(void* out128);
+
+/* Kernel probe for the roofline report: when enabled (kind = 1: every GEMM
+   launch of the step) the library records a cudaEvent pair around each probed
+   launch on cfg.stream and accumulates the algorithmic FLOPs (2 M N K).
+   mimose_probe_read synchronises, returns the summed device time (ms), FLOPs
+   and launch count since the last enable, and keeps the probe running. */
+mimose_status mimose_probe(mimose_ctx* ctx, int32_t kind);
+mimose_status mimose_probe_read(mimose_ctx* ctx, double* total_ms, double* total_flops, int64_t* launches);
+
+/* 1 if this build routes bf16 GEMMs to the tcgen05/TMEM/TMA kernels. */
+int32_t mimose_tc_available(void);
+
 /* ---- stateless host helpers (tests; same code the ctx uses) ---- */
 /* Predicted series for one x: arrays a,y of n_layers entries. */
 typedef struct {

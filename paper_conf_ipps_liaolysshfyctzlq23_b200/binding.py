@@ -115,11 +115,32 @@ _lib.mimose_plan_series.argtypes = [C.POINTER(Series), C.c_int64, C.c_int64, C.c
 _lib.mimose_fit_predict.argtypes = [C.POINTER(C.c_int64), C.POINTER(C.c_int64), C.c_int32, C.c_int32,
                                     C.POINTER(C.c_int64), C.c_int32, C.POINTER(C.c_int64)]
 
+_lib.mimose_nccl_unique_id.argtypes = [_P]
+_lib.mimose_probe.argtypes = [_P, C.c_int32]
+_lib.mimose_probe_read.argtypes = [_P, C.POINTER(C.c_double), C.POINTER(C.c_double), C.POINTER(C.c_int64)]
+
 EXPORTED = ["mimose_default_config", "mimose_init", "mimose_destroy", "mimose_last_error",
             "mimose_status_str", "mimose_num_params", "mimose_set_params", "mimose_get_params",
             "mimose_get_grads", "mimose_collect", "mimose_plan", "mimose_forward", "mimose_backward",
             "mimose_step", "mimose_get_stats", "mimose_phase", "mimose_get_sample", "mimose_dry_run",
-            "mimose_dry_collect", "mimose_predicted_peak", "mimose_plan_series", "mimose_fit_predict"]
+            "mimose_dry_collect", "mimose_predicted_peak", "mimose_plan_series", "mimose_fit_predict",
+            "mimose_nccl_unique_id", "mimose_probe", "mimose_probe_read"]
+
+
+_lib.mimose_tc_available.restype = C.c_int32
+EXPORTED.append("mimose_tc_available")
+
+
+def tc_gemm_available() -> bool:
+    return bool(_lib.mimose_tc_available())
+
+
+def nccl_unique_id() -> bytes:
+    buf = C.create_string_buffer(128)
+    st = _lib.mimose_nccl_unique_id(buf)
+    if st != OK:
+        raise MimoseError(st, "ncclGetUniqueId failed")
+    return buf.raw
 
 
 def make_config(cfg: wl.ModelConfig, **kw) -> Config:
@@ -262,6 +283,14 @@ class Mimose:
         pk = C.c_int64()
         self._chk(_lib.mimose_dry_run(self.h, n_seqs, seq_len, C.c_uint64(mask), C.byref(pk)))
         return pk.value
+
+    def probe(self, kind: int = 1):
+        self._chk(_lib.mimose_probe(self.h, kind))
+
+    def probe_read(self):
+        ms, fl, n = C.c_double(), C.c_double(), C.c_int64()
+        self._chk(_lib.mimose_probe_read(self.h, C.byref(ms), C.byref(fl), C.byref(n)))
+        return ms.value, fl.value, n.value
 
     def dry_collect(self, n_seqs: int, seq_len: int) -> Dict:
         s = SampleS()

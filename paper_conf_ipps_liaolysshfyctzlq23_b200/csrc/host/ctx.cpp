@@ -182,6 +182,11 @@ struct mimose_ctx {
   mimose_stats stats{};
   std::vector<cudaEvent_t> ev_t0, ev_t1;
   bool pending_times = false;
+  // GEMM probe (roofline): event pairs around probed launches
+  int probe = 0;
+  std::vector<cudaEvent_t> probe_ev;
+  size_t probe_used = 0;
+  double probe_flops = 0.0;
 };
 
 namespace {
@@ -274,6 +279,27 @@ inline float* G(mimose_ctx* c, int i) { return c->grad + c->layout[i].off; }
 inline int LP(mimose_ctx* c, int l, int k) { (void)c; return P_LAYER0 + 12 * l + k; }
 inline int HP(mimose_ctx* c, int k) { return P_LAYER0 + 12 * c->cfg.n_layers + k; }
 
+// ------------------------------------------------------------- probe ------
+void pgemm(mimose_ctx* c, Epi epi, const GemmArgs& g, cudaStream_t st) {
+  const bool on = c->probe == 1 && st != nullptr;
+  if (on) {
+    if (c->probe_used + 2 > c->probe_ev.size()) {
+      for (int i = 0; i < 256; ++i) {
+        cudaEvent_t e;
+        cudaEventCreate(&e);
+        c->probe_ev.push_back(e);
+      }
+    }
+    cudaEventRecord(c->probe_ev[c->probe_used], st);
+  }
+  gemm(c->dt, epi, g, st, c->cfg.use_tc != 0);
+  if (on) {
+    cudaEventRecord(c->probe_ev[c->probe_used + 1], st);
+    c->probe_used += 2;
+    c->probe_flops += 2.0 * g.M * (double)g.N * g.K;
+  }
+}
+
 // ------------------------------------------------------------- schedule ---
 // `real` = launch kernels; otherwise only the arena accounting runs.
 
@@ -288,7 +314,6 @@ void layer_forward(Run& r, int l, const char* x, LayerBufs& b, char* yout) {
   mimose_ctx* c = r.c;
   if (!r.real) return;
   const int T = c->T, H = c->cfg.hidden, F = c->cfg.ffn;
-  const bool tc = c->cfg.use_tc != 0;
   GemmArgs g;
   // QKV = x Wqkv^T + b
   g = GemmArgs();
@@ -296,7 +321,7 @@ void layer_forward(Run& r, int l, const char* x, LayerBufs& b, char* yout) {
   g.A = x; g.a_sm = H; g.a_sk = 1;
   g.B = W(c, LP(c, l, L_QKVW)); g.b_sn = H; g.b_sk = 1;
   g.C = b.qkv; g.ldc = 3 * H; g.bias = W(c, LP(c, l, L_QKVB));
-  gemm(c->dt, EPI_BIAS, g, r.st, tc);
+  pgemm(c, EPI_BIAS, g, r.st);
   attn_fwd(c->dt, b.qkv, c->lens, b.O, b.lse, c->B, c->S, H, c->cfg.heads, make_drop(c, KIND_ATTN_PROBS, l), r.st);
   // z1 = x + drop(O Wo^T + bo)
   g = GemmArgs();
@@ -305,7 +330,7 @@ void layer_forward(Run& r, int l, const char* x, LayerBufs& b, char* yout) {
   g.B = W(c, LP(c, l, L_OW)); g.b_sn = H; g.b_sk = 1;
   g.C = b.z1; g.ldc = H; g.bias = W(c, LP(c, l, L_OB)); g.res = x; g.ldr = H;
   g.drop = make_drop(c, KIND_ATTN_OUT, l);
-  gemm(c->dt, EPI_BIAS_DROP_RES, g, r.st, tc);
+  pgemm(c, EPI_BIAS_DROP_RES, g, r.st);
   ln_fwd(c->dt, b.z1, W(c, LP(c, l, L_LN1G)), W(c, LP(c, l, L_LN1B)), b.h1, b.st1, T, H, c->cfg.ln_eps, r.st);
   // u = h1 W1^T + b1, g = gelu(u)
   g = GemmArgs();
@@ -313,7 +338,7 @@ void layer_forward(Run& r, int l, const char* x, LayerBufs& b, char* yout) {
   g.A = b.h1; g.a_sm = H; g.a_sk = 1;
   g.B = W(c, LP(c, l, L_F1W)); g.b_sn = H; g.b_sk = 1;
   g.C = b.u; g.C2 = b.g; g.ldc = F; g.bias = W(c, LP(c, l, L_F1B));
-  gemm(c->dt, EPI_BIAS_GELU, g, r.st, tc);
+  pgemm(c, EPI_BIAS_GELU, g, r.st);
   // z2 = h1 + drop(g W2^T + b2)
   g = GemmArgs();
   g.M = T; g.N = H; g.K = F;
@@ -321,7 +346,7 @@ void layer_forward(Run& r, int l, const char* x, LayerBufs& b, char* yout) {
   g.B = W(c, LP(c, l, L_F2W)); g.b_sn = F; g.b_sk = 1;
   g.C = b.z2; g.ldc = H; g.bias = W(c, LP(c, l, L_F2B)); g.res = b.h1; g.ldr = H;
   g.drop = make_drop(c, KIND_FFN_OUT, l);
-  gemm(c->dt, EPI_BIAS_DROP_RES, g, r.st, tc);
+  pgemm(c, EPI_BIAS_DROP_RES, g, r.st);
   // y = LN2(z2); the store is gated off during recompute (yout == nullptr)
   ln_fwd(c->dt, b.z2, W(c, LP(c, l, L_LN2G)), W(c, LP(c, l, L_LN2B)), yout, b.st2, T, H, c->cfg.ln_eps, r.st);
 }
@@ -355,10 +380,10 @@ void wgrad(Run& r, const void* dY, int N, const void* X, int K, float* out) {
   g.split = split;
   if (split == 1) {
     g.C = out;
-    gemm(c->dt, EPI_F32, g, r.st, c->cfg.use_tc != 0);
+    pgemm(c, EPI_F32, g, r.st);
   } else {
     g.C = c->ws; g.split_stride = (int64_t)N * K;
-    gemm(c->dt, EPI_F32, g, r.st, c->cfg.use_tc != 0);
+    pgemm(c, EPI_F32, g, r.st);
     splitk_reduce(c->ws, split, (int64_t)N * K, out, r.st);
   }
 }
@@ -372,7 +397,7 @@ void dgrad(Run& r, Epi epi, const void* dY, int Nout, const void* Wt, int Kin, v
   g.C = out; g.ldc = Kin;
   if (epi == EPI_GELU_BWD) { g.aux = res_or_aux; g.ldx = Kin; }
   if (epi == EPI_ACC_RES_F32) { g.res = res_or_aux; g.ldr = Kin; }
-  gemm(c->dt, epi, g, r.st, c->cfg.use_tc != 0);
+  pgemm(c, epi, g, r.st);
 }
 
 void layer_backward(Run& r, int l, const char* x, LayerBufs& b, float* dy, char* scr) {
@@ -794,6 +819,7 @@ void mimose_destroy(mimose_ctx* c) {
     for (auto e : c->ev_t0) cudaEventDestroy(e);
     for (auto e : c->ev_t1) cudaEventDestroy(e);
     for (auto e : c->ev_layer) cudaEventDestroy(e);
+    for (auto e : c->probe_ev) cudaEventDestroy(e);
     if (c->ev_comm_done) cudaEventDestroy(c->ev_comm_done);
     if (c->comm) ncclCommDestroy(c->comm);
     if (c->comm_st) cudaStreamDestroy(c->comm_st);
@@ -998,6 +1024,41 @@ mimose_status mimose_plan(mimose_ctx* c, int64_t x, mimose_plan_t* out) {
   c->stats.last_n_dropped = out->n_dropped;
   c->stats.last_predicted_peak = out->predicted_peak;
   if (out->status != MIMOSE_OK) return fail(c, MIMOSE_E_INFEASIBLE, "no plan fits the budget");
+  return MIMOSE_OK;
+}
+
+int32_t mimose_tc_available(void) { return tc_available() ? 1 : 0; }
+
+mimose_status mimose_nccl_unique_id(void* out128) {
+  if (!out128) return MIMOSE_E_INVALID;
+  ncclUniqueId id;
+  if (ncclGetUniqueId(&id) != ncclSuccess) return MIMOSE_E_NCCL;
+  std::memcpy(out128, &id, sizeof(id));
+  return MIMOSE_OK;
+}
+
+mimose_status mimose_probe(mimose_ctx* c, int32_t kind) {
+  if (!c) return MIMOSE_E_INVALID;
+  c->probe = kind;
+  c->probe_used = 0;
+  c->probe_flops = 0.0;
+  return MIMOSE_OK;
+}
+
+mimose_status mimose_probe_read(mimose_ctx* c, double* ms, double* flops, int64_t* launches) {
+  if (!c || !ms || !flops || !launches) return MIMOSE_E_INVALID;
+  double tot = 0.0;
+  if (c->device && c->probe_used) {
+    CK(cudaStreamSynchronize(c->st));
+    for (size_t i = 0; i + 1 < c->probe_used; i += 2) {
+      float t = 0.f;
+      CK(cudaEventElapsedTime(&t, c->probe_ev[i], c->probe_ev[i + 1]));
+      tot += t;
+    }
+  }
+  *ms = tot;
+  *flops = c->probe_flops;
+  *launches = (int64_t)(c->probe_used / 2);
   return MIMOSE_OK;
 }
 

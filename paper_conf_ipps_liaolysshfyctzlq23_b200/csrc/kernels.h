@@ -36,6 +36,7 @@ struct GemmArgs {
   int split = 1; int64_t split_stride = 0;
 };
 void gemm(DType dt, Epi epi, const GemmArgs& g, cudaStream_t st, bool use_tc);
+bool tc_available();
 // Deterministic split-K reduction: out[i] = sum_s part[s*n + i] (fixed order).
 void splitk_reduce(const float* part, int splits, int64_t n, float* out, cudaStream_t st);
 

@@ -3,4 +3,5 @@
 #include "kernels.h"
 namespace mimose {
 bool gemm_tc(Epi, const GemmArgs&, cudaStream_t) { return false; }
+bool tc_available() { return false; }
 }  // namespace mimose
