@@ -281,7 +281,7 @@ inline int HP(mimose_ctx* c, int k) { return P_LAYER0 + 12 * c->cfg.n_layers + k
 
 // ------------------------------------------------------------- probe ------
 void pgemm(mimose_ctx* c, Epi epi, const GemmArgs& g, cudaStream_t st) {
-  const bool on = c->probe == 1 && st != nullptr;
+  const bool on = c->probe == 1 && c->device;
   if (on) {
     if (c->probe_used + 2 > c->probe_ev.size()) {
       for (int i = 0; i < 256; ++i) {
@@ -748,10 +748,12 @@ mimose_status mimose_init(const mimose_config* cfgp, mimose_ctx** out) {
   c->device = k.arena_base != nullptr;
   Arena& a = c->ar;
   a.base = (char*)k.arena_base;
-  a.cap = k.arena_base ? k.arena_bytes : (int64_t)1 << 62;
+  // every allocation is a multiple of 16 B, so live <= M  <=>  live <= floor16(M):
+  // flooring the slab end keeps top-region addresses 16-B aligned at no cost
+  a.cap = k.arena_base ? (k.arena_bytes & ~(int64_t)15) : (int64_t)1 << 62;
   a.budget = k.budget_bytes > 0 ? k.budget_bytes : a.cap;
   a.enforce = k.enforce_budget != 0;
-  if (c->device && a.enforce && a.cap < a.budget) {
+  if (c->device && a.enforce && a.cap < (a.budget & ~(int64_t)15)) {
     *out = c;
     return bad("arena_bytes < budget_bytes with enforce_budget");
   }
