@@ -229,6 +229,15 @@ mimose_status mimose_nccl_unique_id(void* out128);
 mimose_status mimose_probe(mimose_ctx* ctx, int32_t kind);
 mimose_status mimose_probe_read(mimose_ctx* ctx, double* total_ms, double* total_flops, int64_t* launches);
 
+/* Test hook: one bf16 GEMM of the library, C[m,n] = sum_k A(m,k) B(n,k) with
+   A(m,k) = A[m*a_sm + k*a_sk], B(n,k) = B[n*b_sn + k*b_sk] (element strides),
+   epilogue `epi` (0 store bf16, 1 +bias bf16, 6 fp32; split-K writes `split`
+   fp32 partials at C + z*M*ldc), tensor-core path if use_tc.  Device pointers;
+   enqueued on `stream`. */
+mimose_status mimose_debug_gemm(int32_t epi, int32_t M, int32_t N, int32_t K, const void* A, int64_t a_sm,
+                                int64_t a_sk, const void* B, int64_t b_sn, int64_t b_sk, void* C, int64_t ldc,
+                                const void* bias, int32_t split, int32_t use_tc, void* stream);
+
 /* 1 if this build routes bf16 GEMMs to the tcgen05/TMEM/TMA kernels. */
 int32_t mimose_tc_available(void);
 

@@ -131,6 +131,20 @@ _lib.mimose_tc_available.restype = C.c_int32
 EXPORTED.append("mimose_tc_available")
 
 
+_lib.mimose_debug_gemm.argtypes = [C.c_int32, C.c_int32, C.c_int32, C.c_int32, _P, C.c_int64, C.c_int64,
+                                   _P, C.c_int64, C.c_int64, _P, C.c_int64, _P, C.c_int32, C.c_int32, _P]
+EXPORTED.append("mimose_debug_gemm")
+
+
+def debug_gemm(epi, M, N, K, A, a_sm, a_sk, B, b_sn, b_sk, Cm, ldc, bias=None, split=1, use_tc=True, stream=0):
+    """Test hook over one library GEMM (torch tensors in, device pointers out)."""
+    st = _lib.mimose_debug_gemm(epi, M, N, K, A.data_ptr(), a_sm, a_sk, B.data_ptr(), b_sn, b_sk, Cm.data_ptr(),
+                                ldc, bias.data_ptr() if bias is not None else None, split, 1 if use_tc else 0,
+                                stream)
+    if st != OK:
+        raise MimoseError(st, "debug_gemm")
+
+
 def tc_gemm_available() -> bool:
     return bool(_lib.mimose_tc_available())
 

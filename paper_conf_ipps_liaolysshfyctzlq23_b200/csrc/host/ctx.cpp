@@ -1031,6 +1031,21 @@ mimose_status mimose_plan(mimose_ctx* c, int64_t x, mimose_plan_t* out) {
 
 int32_t mimose_tc_available(void) { return tc_available() ? 1 : 0; }
 
+mimose_status mimose_debug_gemm(int32_t epi, int32_t M, int32_t N, int32_t K, const void* A, int64_t a_sm,
+                                int64_t a_sk, const void* B, int64_t b_sn, int64_t b_sk, void* Cp, int64_t ldc,
+                                const void* bias, int32_t split, int32_t use_tc, void* stream) {
+  if (epi != EPI_STORE && epi != EPI_BIAS && epi != EPI_F32) return MIMOSE_E_INVALID;
+  GemmArgs g;
+  g.M = M; g.N = N; g.K = K;
+  g.A = A; g.a_sm = a_sm; g.a_sk = a_sk;
+  g.B = B; g.b_sn = b_sn; g.b_sk = b_sk;
+  g.C = Cp; g.ldc = ldc; g.bias = bias;
+  g.split = split < 1 ? 1 : split;
+  g.split_stride = (int64_t)M * ldc;
+  gemm(DT_BF16, (Epi)epi, g, (cudaStream_t)stream, use_tc != 0);
+  return cudaGetLastError() == cudaSuccess ? MIMOSE_OK : MIMOSE_E_CUDA;
+}
+
 mimose_status mimose_nccl_unique_id(void* out128) {
   if (!out128) return MIMOSE_E_INVALID;
   ncclUniqueId id;

@@ -1,7 +1,400 @@
-// tcgen05 / TMEM / TMA GEMM for bf16 mode (sm_100a).  Placeholder until the
-// tensor-core path lands: returning false routes to the SIMT GEMM.
+// tcgen05 / TMEM / TMA GEMM for bf16 mode on sm_100a.
+//
+//   C[m, n] = sum_k A(m, k) B(n, k)  (+ the fused epilogues of gemm_epi.cuh)
+//
+// One CTA computes a 128 x BN tile with fp32 accumulators in TMEM:
+//   warp 0      TMA producer: 128B-swizzled A/B k-blocks (64 wide) into a
+//               STAGES-deep smem ring, mbarrier complete_tx
+//   warp 1      TMEM allocation + the single-thread tcgen05.mma issuer
+//               (kind::f16, M=128, N=BN, K=16 per instruction); tcgen05.commit
+//               frees smem stages and finally signals the epilogue
+//   warps 2..5  epilogue: tcgen05.ld 32x32b.x32 (warp w reads TMEM lanes
+//               32*(w%4)..), fused bias / GELU / dropout+residual / GELU' /
+//               residual-add / split-K fp32, vectorised global stores
+// Operands may be K-major (forward: X, W; dgrad: dY) or MN-major (dgrad: W;
+// wgrad: dY^T, X^T) — the UMMA descriptors encode both, so no transposes are
+// materialised.  Split-K over blockIdx.z writes fp32 partials that a fixed-order
+// kernel reduces (deterministic wgrad).
+#include <cuda.h>
+
+#include <cstdio>
+#include <mutex>
+#include <unordered_map>
+
+#include "gemm_epi.cuh"
 #include "kernels.h"
+
 namespace mimose {
-bool gemm_tc(Epi, const GemmArgs&, cudaStream_t) { return false; }
-bool tc_available() { return false; }
+
+constexpr int TBM = 128, TBK = 64;
+constexpr int TC_THREADS = 192;
+
+template <int BN>
+struct TcCfg {
+  static constexpr int STAGES = BN >= 256 ? 4 : 6;
+  static constexpr int A_BYTES = TBM * TBK * 2;
+  static constexpr int B_BYTES = BN * TBK * 2;
+  static constexpr int STAGE_BYTES = A_BYTES + B_BYTES;
+  static constexpr int SMEM = STAGES * STAGE_BYTES + 1024 /*align*/ + 256 /*barriers*/;
+};
+
+struct TcArgs {
+  GemmArgs g;
+  int a_mn, b_mn;           // 1: operand is MN-major (MN contiguous)
+  int kb_per_split;         // k-blocks per blockIdx.z
+  int kb_total;
+};
+
+// ------------------------------------------------------------ PTX helpers --
+MDEV uint32_t smem_u32(const void* p) { return (uint32_t)__cvta_generic_to_shared(p); }
+
+MDEV void mbar_init(uint64_t* b, uint32_t count) {
+  asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(smem_u32(b)), "r"(count));
+}
+MDEV void mbar_expect_tx(uint64_t* b, uint32_t bytes) {
+  asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(b)), "r"(bytes) : "memory");
+}
+MDEV void mbar_wait(uint64_t* b, uint32_t parity) {
+  asm volatile(
+      "{\n\t.reg .pred P1;\n\tLAB_WAIT:\n\t"
+      "mbarrier.try_wait.parity.shared::cta.b64 P1, [%0], %1, %2;\n\t"
+      "@P1 bra DONE;\n\tbra LAB_WAIT;\n\tDONE:\n\t}" ::"r"(smem_u32(b)), "r"(parity), "r"(0x989680)
+      : "memory");
+}
+MDEV void tma_load_2d(const CUtensorMap* map, uint64_t* bar, void* dst, int c0, int c1) {
+  asm volatile(
+      "cp.async.bulk.tensor.2d.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1, {%3, %4}], [%2];"
+      ::"r"(smem_u32(dst)), "l"(map), "r"(smem_u32(bar)), "r"(c0), "r"(c1) : "memory");
+}
+MDEV uint64_t make_desc(uint32_t saddr, uint32_t lbo, uint32_t sbo) {
+  uint64_t d = 0;
+  d |= (uint64_t)((saddr >> 4) & 0x3FFF);
+  d |= (uint64_t)((lbo >> 4) & 0x3FFF) << 16;
+  d |= (uint64_t)((sbo >> 4) & 0x3FFF) << 32;
+  d |= (uint64_t)1 << 46;              // descriptor version (sm100)
+  d |= (uint64_t)2 << 61;              // SWIZZLE_128B
+  return d;
+}
+MDEV void mma_bf16(uint32_t tmem_d, uint64_t da, uint64_t db, uint32_t idesc, uint32_t acc) {
+  asm volatile(
+      "{\n\t.reg .pred p;\n\tsetp.ne.b32 p, %4, 0;\n\t"
+      "tcgen05.mma.cta_group::1.kind::f16 [%0], %1, %2, %3, p;\n\t}"
+      ::"r"(tmem_d), "l"(da), "l"(db), "r"(idesc), "r"(acc));
+}
+MDEV void mma_commit(uint64_t* bar) {
+  asm volatile("tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%0];" ::"r"(smem_u32(bar))
+               : "memory");
+}
+MDEV void tmem_ld32(uint32_t taddr, float (&v)[32]) {
+  uint32_t r[32];
+  asm volatile(
+      "tcgen05.ld.sync.aligned.32x32b.x32.b32 {%0,%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15,"
+      "%16,%17,%18,%19,%20,%21,%22,%23,%24,%25,%26,%27,%28,%29,%30,%31}, [%32];"
+      : "=r"(r[0]), "=r"(r[1]), "=r"(r[2]), "=r"(r[3]), "=r"(r[4]), "=r"(r[5]), "=r"(r[6]), "=r"(r[7]),
+        "=r"(r[8]), "=r"(r[9]), "=r"(r[10]), "=r"(r[11]), "=r"(r[12]), "=r"(r[13]), "=r"(r[14]), "=r"(r[15]),
+        "=r"(r[16]), "=r"(r[17]), "=r"(r[18]), "=r"(r[19]), "=r"(r[20]), "=r"(r[21]), "=r"(r[22]), "=r"(r[23]),
+        "=r"(r[24]), "=r"(r[25]), "=r"(r[26]), "=r"(r[27]), "=r"(r[28]), "=r"(r[29]), "=r"(r[30]), "=r"(r[31])
+      : "r"(taddr));
+  asm volatile("tcgen05.wait::ld.sync.aligned;" ::: "memory");
+#pragma unroll
+  for (int i = 0; i < 32; ++i) v[i] = __uint_as_float(r[i]);
+}
+
+MDEV uint4 pack8(const float* v) {
+  uint4 o;
+  __nv_bfloat162 t;
+  t = __floats2bfloat162_rn(v[0], v[1]); o.x = *(uint32_t*)&t;
+  t = __floats2bfloat162_rn(v[2], v[3]); o.y = *(uint32_t*)&t;
+  t = __floats2bfloat162_rn(v[4], v[5]); o.z = *(uint32_t*)&t;
+  t = __floats2bfloat162_rn(v[6], v[7]); o.w = *(uint32_t*)&t;
+  return o;
+}
+MDEV void unpack8(uint4 u, float* v) {
+  const __nv_bfloat162* p = (const __nv_bfloat162*)&u;
+#pragma unroll
+  for (int i = 0; i < 4; ++i) { float2 f = __bfloat1622float2(p[i]); v[2 * i] = f.x; v[2 * i + 1] = f.y; }
+}
+MDEV void ld_bf16x32(const __nv_bfloat16* p, float* v) {
+#pragma unroll
+  for (int i = 0; i < 4; ++i) unpack8(((const uint4*)p)[i], v + 8 * i);
+}
+MDEV void st_bf16x32(__nv_bfloat16* p, const float* v) {
+#pragma unroll
+  for (int i = 0; i < 4; ++i) ((uint4*)p)[i] = pack8(v + 8 * i);
+}
+
+// Vectorised epilogue of 32 consecutive columns [n, n+32) of row m (all in range).
+template <int EPI>
+MDEV void epi_row32(const GemmArgs& g, int m, int n, float (&v)[32]) {
+  using E = __nv_bfloat16;
+  const int64_t o = (int64_t)m * g.ldc + n;
+  if constexpr (EPI == EPI_STORE) {
+    st_bf16x32((E*)g.C + o, v);
+  } else if constexpr (EPI == EPI_BIAS || EPI == EPI_BIAS_GELU || EPI == EPI_BIAS_DROP_RES) {
+    float b[32];
+    ld_bf16x32((const E*)g.bias + n, b);
+#pragma unroll
+    for (int i = 0; i < 32; ++i) v[i] += b[i];
+    if constexpr (EPI == EPI_BIAS) {
+      st_bf16x32((E*)g.C + o, v);
+    } else if constexpr (EPI == EPI_BIAS_GELU) {
+      st_bf16x32((E*)g.C + o, v);
+#pragma unroll
+      for (int i = 0; i < 32; ++i) v[i] = gelu_f(__bfloat162float(__float2bfloat16_rn(v[i])));
+      st_bf16x32((E*)g.C2 + o, v);
+    } else {
+      float r[32];
+      ld_bf16x32((const E*)g.res + (int64_t)m * g.ldr + n, r);
+      float* out = (float*)g.C + o;
+#pragma unroll
+      for (int q = 0; q < 8; ++q) {
+        const float4 f = drop_factor4(g.drop, (uint64_t)(o + 4 * q) >> 2);
+        float4 w;
+        w.x = r[4 * q + 0] + v[4 * q + 0] * f.x;
+        w.y = r[4 * q + 1] + v[4 * q + 1] * f.y;
+        w.z = r[4 * q + 2] + v[4 * q + 2] * f.z;
+        w.w = r[4 * q + 3] + v[4 * q + 3] * f.w;
+        ((float4*)out)[q] = w;
+      }
+    }
+  } else if constexpr (EPI == EPI_GELU_BWD) {
+    float u[32];
+    ld_bf16x32((const E*)g.aux + (int64_t)m * g.ldx + n, u);
+#pragma unroll
+    for (int i = 0; i < 32; ++i) v[i] *= gelu_grad_f(u[i]);
+    st_bf16x32((E*)g.C + o, v);
+  } else if constexpr (EPI == EPI_ACC_RES_F32) {
+    const float4* r = (const float4*)((const float*)g.res + (int64_t)m * g.ldr + n);
+    float4* out = (float4*)((float*)g.C + o);
+#pragma unroll
+    for (int q = 0; q < 8; ++q) {
+      const float4 a = r[q];
+      out[q] = make_float4(v[4 * q] + a.x, v[4 * q + 1] + a.y, v[4 * q + 2] + a.z, v[4 * q + 3] + a.w);
+    }
+  } else {
+    float4* out = (float4*)((float*)g.C + (int64_t)blockIdx.z * g.split_stride + o);
+#pragma unroll
+    for (int q = 0; q < 8; ++q) out[q] = make_float4(v[4 * q], v[4 * q + 1], v[4 * q + 2], v[4 * q + 3]);
+  }
+}
+
+template <int BN, int EPI>
+__global__ void __launch_bounds__(TC_THREADS, 1)
+    k_gemm_tc(const __grid_constant__ CUtensorMap tma_a, const __grid_constant__ CUtensorMap tma_b, const TcArgs args) {
+  using Cf = TcCfg<BN>;
+  extern __shared__ uint8_t smem_raw[];
+  uint8_t* smem = (uint8_t*)(((uintptr_t)smem_raw + 1023) & ~(uintptr_t)1023);
+  uint64_t* full = (uint64_t*)(smem + Cf::STAGES * Cf::STAGE_BYTES);
+  uint64_t* empty = full + Cf::STAGES;
+  uint64_t* tfull = empty + Cf::STAGES;
+  uint32_t* tmem_slot = (uint32_t*)(tfull + 1);
+
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const int n0 = blockIdx.x * BN, m0 = blockIdx.y * TBM;
+  const int kb0 = blockIdx.z * args.kb_per_split;
+  const int kb1 = min(args.kb_total, kb0 + args.kb_per_split);
+  const int nkb = kb1 - kb0;
+
+  if (warp == 0 && lane == 0) {
+    for (int s = 0; s < Cf::STAGES; ++s) { mbar_init(&full[s], 1); mbar_init(&empty[s], 1); }
+    mbar_init(tfull, 1);
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+    asm volatile("prefetch.tensormap [%0];" ::"l"(&tma_a) : "memory");
+    asm volatile("prefetch.tensormap [%0];" ::"l"(&tma_b) : "memory");
+  }
+  if (warp == 1) {
+    asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(smem_u32(tmem_slot)),
+                 "r"(BN));
+    asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;");
+  }
+  asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
+  __syncthreads();
+  asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
+  const uint32_t tmem = *tmem_slot;
+
+  if (warp == 0) {
+    if (lane == 0) {                                   // ---------------- TMA producer
+      for (int i = 0; i < nkb; ++i) {
+        const int s = i % Cf::STAGES;
+        if (i >= Cf::STAGES) mbar_wait(&empty[s], ((i / Cf::STAGES) - 1) & 1);
+        uint8_t* sa = smem + s * Cf::STAGE_BYTES;
+        uint8_t* sb = sa + Cf::A_BYTES;
+        const int k = (kb0 + i) * TBK;
+        mbar_expect_tx(&full[s], Cf::STAGE_BYTES);
+        if (args.a_mn) {
+          tma_load_2d(&tma_a, &full[s], sa, m0, k);
+          tma_load_2d(&tma_a, &full[s], sa + 8192, m0 + 64, k);
+        } else {
+          tma_load_2d(&tma_a, &full[s], sa, k, m0);
+        }
+        if (args.b_mn) {
+#pragma unroll
+          for (int j = 0; j < BN / 64; ++j) tma_load_2d(&tma_b, &full[s], sb + 8192 * j, n0 + 64 * j, k);
+        } else {
+          tma_load_2d(&tma_b, &full[s], sb, k, n0);
+        }
+      }
+    }
+  } else if (warp == 1) {
+    if (lane == 0) {                                   // ---------------- MMA issuer
+      const uint32_t idesc = (1u << 4) | (1u << 7) | (1u << 10) | ((uint32_t)args.a_mn << 15) |
+                             ((uint32_t)args.b_mn << 16) | ((uint32_t)(BN >> 3) << 17) | ((uint32_t)(TBM >> 4) << 24);
+      for (int i = 0; i < nkb; ++i) {
+        const int s = i % Cf::STAGES;
+        mbar_wait(&full[s], (i / Cf::STAGES) & 1);
+        asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
+        const uint32_t sa = smem_u32(smem + s * Cf::STAGE_BYTES);
+        const uint32_t sb = sa + Cf::A_BYTES;
+#pragma unroll
+        for (int kk = 0; kk < TBK / 16; ++kk) {
+          const uint64_t da = args.a_mn ? make_desc(sa + kk * 2048, 8192, 1024) : make_desc(sa + kk * 32, 16, 1024);
+          const uint64_t db = args.b_mn ? make_desc(sb + kk * 2048, 8192, 1024) : make_desc(sb + kk * 32, 16, 1024);
+          mma_bf16(tmem, da, db, idesc, (i > 0 || kk > 0) ? 1u : 0u);
+        }
+        mma_commit(&empty[s]);
+      }
+      mma_commit(tfull);
+    }
+  } else {                                             // ---------------- epilogue warps 2..5
+    const int q = warp & 3;
+    const int m = m0 + 32 * q + lane;
+    mbar_wait(tfull, 0);
+    asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
+    const GemmArgs& g = args.g;
+#pragma unroll 1
+    for (int c = 0; c < BN / 32; ++c) {
+      float v[32];
+      tmem_ld32(tmem + ((uint32_t)(32 * q) << 16) + 32 * c, v);
+      if (nkb <= 0) {                                  // empty split-K slice: exact zeros
+#pragma unroll
+        for (int i = 0; i < 32; ++i) v[i] = 0.f;
+      }
+      const int n = n0 + 32 * c;
+      if (m < g.M) {
+        if (n + 32 <= g.N) {
+          epi_row32<EPI>(g, m, n, v);
+        } else {
+          for (int i = 0; i < 32 && n + i < g.N; ++i) epilogue<__nv_bfloat16, EPI>(g, m, n + i, v[i]);
+        }
+      }
+    }
+  }
+  asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
+  __syncthreads();
+  if (warp == 1) {
+    asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
+    asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(tmem), "r"(BN));
+  }
+}
+
+// ------------------------------------------------------------------ host --
+typedef CUresult (*EncodeFn)(CUtensorMap*, CUtensorMapDataType, cuuint32_t, void*, const cuuint64_t*,
+                             const cuuint64_t*, const cuuint32_t*, const cuuint32_t*, CUtensorMapInterleave,
+                             CUtensorMapSwizzle, CUtensorMapL2promotion, CUtensorMapFloatOOBfill);
+
+static EncodeFn encode_fn() {
+  static EncodeFn fn = nullptr;
+  static std::once_flag once;
+  std::call_once(once, [] {
+    void* p = nullptr;
+    cudaDriverEntryPointQueryResult q;
+    if (cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &p, cudaEnableDefault, &q) == cudaSuccess &&
+        q == cudaDriverEntryPointSuccess)
+      fn = (EncodeFn)p;
+  });
+  return fn;
+}
+
+struct MapKey {
+  const void* ptr;
+  uint64_t inner, outer, stride;
+  uint32_t box_inner, box_outer;
+  bool operator==(const MapKey& o) const {
+    return ptr == o.ptr && inner == o.inner && outer == o.outer && stride == o.stride &&
+           box_inner == o.box_inner && box_outer == o.box_outer;
+  }
+};
+struct MapKeyHash {
+  size_t operator()(const MapKey& k) const {
+    size_t h = std::hash<const void*>()(k.ptr);
+    for (uint64_t v : {k.inner, k.outer, k.stride, (uint64_t)k.box_inner << 32 | k.box_outer})
+      h ^= std::hash<uint64_t>()(v) + 0x9e3779b97f4a7c15ull + (h << 6) + (h >> 2);
+    return h;
+  }
+};
+
+// 2D bf16 tensor [outer][inner] (inner contiguous), row stride in elements.
+static bool make_map(CUtensorMap* out, const void* ptr, uint64_t inner, uint64_t outer, uint64_t stride_elems,
+                     uint32_t box_inner, uint32_t box_outer) {
+  static std::unordered_map<MapKey, CUtensorMap, MapKeyHash> cache;
+  static std::mutex mu;
+  MapKey key{ptr, inner, outer, stride_elems, box_inner, box_outer};
+  std::lock_guard<std::mutex> lk(mu);
+  auto it = cache.find(key);
+  if (it != cache.end()) { *out = it->second; return true; }
+  EncodeFn fn = encode_fn();
+  if (!fn) return false;
+  cuuint64_t dims[2] = {inner, outer};
+  cuuint64_t strides[1] = {stride_elems * 2};
+  cuuint32_t box[2] = {box_inner, box_outer};
+  cuuint32_t es[2] = {1, 1};
+  CUresult r = fn(out, CU_TENSOR_MAP_DATA_TYPE_BFLOAT16, 2, const_cast<void*>(ptr), dims, strides, box, es,
+                  CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+                  CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+  if (r != CUDA_SUCCESS) return false;
+  if (cache.size() > 8192) cache.clear();
+  cache.emplace(key, *out);
+  return true;
+}
+
+template <int BN, int EPI>
+static void launch_tc(const CUtensorMap& ma, const CUtensorMap& mb, const TcArgs& a, dim3 grid, cudaStream_t st) {
+  static bool attr = false;
+  if (!attr) {
+    cudaFuncSetAttribute(k_gemm_tc<BN, EPI>, cudaFuncAttributeMaxDynamicSharedMemorySize, TcCfg<BN>::SMEM);
+    attr = true;
+  }
+  k_gemm_tc<BN, EPI><<<grid, TC_THREADS, TcCfg<BN>::SMEM, st>>>(ma, mb, a);
+}
+
+bool tc_available() { return encode_fn() != nullptr; }
+
+bool gemm_tc(Epi epi, const GemmArgs& g, cudaStream_t st) {
+  constexpr int BN = 128;
+  TcArgs a;
+  a.g = g;
+  // operand majors from the strides; the contiguous stride must be 1 and the
+  // row stride 16-B aligned (multiple of 8 bf16)
+  if (g.a_sk == 1 && g.a_sm % 8 == 0) a.a_mn = 0;
+  else if (g.a_sm == 1 && g.a_sk % 8 == 0) a.a_mn = 1;
+  else return false;
+  if (g.b_sk == 1 && g.b_sn % 8 == 0) a.b_mn = 0;
+  else if (g.b_sn == 1 && g.b_sk % 8 == 0) a.b_mn = 1;
+  else return false;
+  if (((uintptr_t)g.A | (uintptr_t)g.B) & 15) return false;
+  // vectorised epilogue needs 16-B aligned rows of every epilogue tensor
+  if (g.ldc % 8 || (g.res && g.ldr % 8) || (g.aux && g.ldx % 8)) return false;
+  CUtensorMap ma, mb;
+  bool ok;
+  if (a.a_mn) ok = make_map(&ma, g.A, g.M, g.K, g.a_sk, 64, 64);
+  else ok = make_map(&ma, g.A, g.K, g.M, g.a_sm, 64, TBM);
+  if (!ok) return false;
+  if (a.b_mn) ok = make_map(&mb, g.B, g.N, g.K, g.b_sk, 64, 64);
+  else ok = make_map(&mb, g.B, g.K, g.N, g.b_sn, 64, BN);
+  if (!ok) return false;
+  a.kb_total = (g.K + TBK - 1) / TBK;
+  a.kb_per_split = (a.kb_total + g.split - 1) / g.split;
+  dim3 grid((g.N + BN - 1) / BN, (g.M + TBM - 1) / TBM, g.split);
+  switch (epi) {
+    case EPI_STORE: launch_tc<BN, EPI_STORE>(ma, mb, a, grid, st); break;
+    case EPI_BIAS: launch_tc<BN, EPI_BIAS>(ma, mb, a, grid, st); break;
+    case EPI_BIAS_GELU: launch_tc<BN, EPI_BIAS_GELU>(ma, mb, a, grid, st); break;
+    case EPI_BIAS_DROP_RES: launch_tc<BN, EPI_BIAS_DROP_RES>(ma, mb, a, grid, st); break;
+    case EPI_GELU_BWD: launch_tc<BN, EPI_GELU_BWD>(ma, mb, a, grid, st); break;
+    case EPI_ACC_RES_F32: launch_tc<BN, EPI_ACC_RES_F32>(ma, mb, a, grid, st); break;
+    default: launch_tc<BN, EPI_F32>(ma, mb, a, grid, st); break;
+  }
+  return true;
+}
+
 }  // namespace mimose

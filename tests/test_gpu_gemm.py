@@ -1,0 +1,66 @@
+"""The library's bf16 GEMMs (tcgen05/TMEM/TMA and SIMT) against a plain PyTorch
+fp32 reference of the same op: every operand-major combination the step uses
+(forward NT, dgrad NN, wgrad TN), ragged M/N/K tails, bias epilogue, split-K."""
+import pytest
+
+torch = pytest.importorskip("torch")
+pytestmark = pytest.mark.gpu
+
+
+def mb():
+    from paper_conf_ipps_liaolysshfyctzlq23_b200 import binding
+    return binding
+
+
+SHAPES = [(256, 256, 128), (300, 200, 136), (2048, 768, 768), (1000, 2304, 768), (768, 3072, 520), (128, 128, 64)]
+
+
+def operands(M, N, K, a_mn, b_mn, seed=0):
+    g = torch.Generator(device="cuda").manual_seed(seed)
+    A = torch.randn(M, K, device="cuda", generator=g).bfloat16()
+    B = torch.randn(N, K, device="cuda", generator=g).bfloat16()
+    # storage: K-major = [rows, K] row-major; MN-major = [K, rows] row-major
+    As = A.t().contiguous() if a_mn else A.contiguous()
+    Bs = B.t().contiguous() if b_mn else B.contiguous()
+    a_sm, a_sk = (1, M) if a_mn else (K, 1)
+    b_sn, b_sk = (1, N) if b_mn else (K, 1)
+    return A, B, As, Bs, a_sm, a_sk, b_sn, b_sk
+
+
+@pytest.mark.parametrize("use_tc", [True, False])
+@pytest.mark.parametrize("a_mn,b_mn", [(0, 0), (0, 1), (1, 1)])
+@pytest.mark.parametrize("shape", SHAPES)
+def test_gemm_f32_out(shape, a_mn, b_mn, use_tc):
+    M, N, K = shape
+    A, B, As, Bs, a_sm, a_sk, b_sn, b_sk = operands(M, N, K, a_mn, b_mn)
+    C = torch.full((M, N), float("nan"), device="cuda")
+    mb().debug_gemm(6, M, N, K, As, a_sm, a_sk, Bs, b_sn, b_sk, C, N, use_tc=use_tc)
+    torch.cuda.synchronize()
+    ref = A.float() @ B.float().t()
+    err = (C - ref).abs().max().item() / ref.abs().max().item()
+    assert err < 1e-5, err
+
+
+@pytest.mark.parametrize("shape", [(300, 200, 136), (2048, 768, 768)])
+def test_gemm_bias_bf16_out(shape):
+    M, N, K = shape
+    A, B, As, Bs, a_sm, a_sk, b_sn, b_sk = operands(M, N, K, 0, 0, seed=1)
+    bias = torch.randn(N, device="cuda").bfloat16()
+    C = torch.zeros(M, N, device="cuda", dtype=torch.bfloat16)
+    mb().debug_gemm(1, M, N, K, As, a_sm, a_sk, Bs, b_sn, b_sk, C, N, bias=bias)
+    torch.cuda.synchronize()
+    ref = A.float() @ B.float().t() + bias.float()
+    err = (C.float() - ref).abs().max().item() / ref.abs().max().item()
+    assert err < 1e-2, err
+
+
+@pytest.mark.parametrize("split", [2, 3, 4])
+def test_gemm_split_k(split):
+    M, N, K = 768, 768, 1000            # wgrad-like: TN, K = tokens
+    A, B, As, Bs, a_sm, a_sk, b_sn, b_sk = operands(M, N, K, 1, 1, seed=2)
+    C = torch.zeros(split, M, N, device="cuda")
+    mb().debug_gemm(6, M, N, K, As, a_sm, a_sk, Bs, b_sn, b_sk, C, N, split=split)
+    torch.cuda.synchronize()
+    ref = A.float() @ B.float().t()
+    err = (C.sum(0) - ref).abs().max().item() / ref.abs().max().item()
+    assert err < 1e-5, err
