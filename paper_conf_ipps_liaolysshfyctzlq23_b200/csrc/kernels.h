@@ -44,6 +44,9 @@ void splitk_reduce(const float* part, int splits, int64_t n, float* out, cudaStr
 // qkv [B*S, 3H] (q | k | v, head-major columns), O [B*S, H], lse [B, h, S].
 void attn_fwd(DType dt, const void* qkv, const int32_t* lengths, void* O, float* lse,
               int B, int S, int H, int h, Drop drop, cudaStream_t st);
+// bf16 with head dim 64 and S <= 128 runs on tcgen05 unless disabled (tests).
+void set_attn_tc(bool on);
+bool attn_tc_enabled();
 // D [B,h,S] = rowsum(dO * O); dqkv [B*S, 3H].
 void attn_bwd(DType dt, const void* qkv, const void* O, const void* dO, const float* lse,
               const int32_t* lengths, float* Dbuf, void* dqkv, int B, int S, int H, int h,

@@ -17,6 +17,16 @@ namespace mimose {
 
 static inline int cdiv(int64_t a, int64_t b) { return (int)((a + b - 1) / b); }
 
+// tcgen05 versions (kernels_attn_tc.cu): bf16, head dim 64, S <= 128
+bool attn_fwd_tc(const void* qkv, const int32_t* lengths, void* O, float* lse, int B, int S, int H, int h,
+                 Drop drop, cudaStream_t st);
+bool attn_bwd_tc(const void* qkv, const void* O, const void* dO, const float* lse, const int32_t* lengths,
+                 void* dqkv, int B, int S, int H, int h, Drop drop, cudaStream_t st);
+
+static bool g_attn_tc = true;
+void set_attn_tc(bool on) { g_attn_tc = on; }
+bool attn_tc_enabled() { return g_attn_tc; }
+
 constexpr int AT = 64;  // forward: rows per CTA / keys per tile
 constexpr int BT = 32;  // backward tile (4 fp32 tiles must fit the 48 KB static smem)
 
@@ -88,10 +98,11 @@ __global__ void __launch_bounds__(AT) k_attn_fwd(const E* __restrict__ qkv, cons
 
 void attn_fwd(DType dt, const void* qkv, const int32_t* lengths, void* O, float* lse, int B, int S, int H,
               int h, Drop drop, cudaStream_t st) {
+  note_launch(1);
+  if (dt == DT_BF16 && attn_tc_enabled() && attn_fwd_tc(qkv, lengths, O, lse, B, S, H, h, drop, st)) return;
   const int D = H / h;
   const float scale = 1.0f / sqrtf((float)D);
   dim3 grid(cdiv(S, AT), B * h);
-  note_launch(1);
   auto go = [&](auto* tag, auto dconst) {
     using E = std::remove_pointer_t<decltype(tag)>;
     constexpr int DD = decltype(dconst)::value;
@@ -245,6 +256,11 @@ __global__ void __launch_bounds__(BT) k_attn_bwd_q(const E* __restrict__ qkv, co
 void attn_bwd(DType dt, const void* qkv, const void* O, const void* dO, const float* lse,
               const int32_t* lengths, float* Dbuf, void* dqkv, int B, int S, int H, int h, Drop drop,
               cudaStream_t st) {
+  if (dt == DT_BF16 && attn_tc_enabled() &&
+      attn_bwd_tc(qkv, O, dO, lse, lengths, dqkv, B, S, H, h, drop, st)) {
+    note_launch(1);
+    return;
+  }
   const int D = H / h;
   const float scale = 1.0f / sqrtf((float)D);
   dim3 grid(cdiv(S, BT), B * h);

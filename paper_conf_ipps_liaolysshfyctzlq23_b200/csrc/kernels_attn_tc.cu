@@ -1,0 +1,344 @@
+// Attention on the 5th-gen tensor cores (tcgen05 / TMEM / TMA), head dim 64,
+// whole sequence in one 128-row tile (S <= 128: the BERT-base workload range).
+// PAPER.md P:160 / Fig. 8: S = Q K^T -> scale -> softmax -> x V.
+//
+// One CTA (4 warps) per (sequence b, head h); thread t owns TMEM lane t, i.e.
+// query row t (S, dP, O, dQ) or key row t (dV, dK).
+//
+// forward:  TMA Q,K,V tiles -> S = Q K^T (TMEM) -> row softmax + Philox dropout
+//           in registers -> P~ (bf16, 128B-swizzled smem) -> O = P~ V (TMEM)
+//           -> O (bf16) and LSE (fp32) to global.
+// backward: TMA Q,K,V,dO -> S = Q K^T, dP~ = dO V^T (TMEM) -> P = exp(S - LSE),
+//           dS = P (dP~ f - D), D = rowsum(dO * O) -> P~, dS tiles (smem) ->
+//           dV = P~^T dO, dK = dS^T Q, dQ = dS K (the same smem tile read as an
+//           MN-major or a K-major operand) -> dQKV (bf16).  No atomics.
+// Dropout element e = ((b*h + head)*S + q)*S + k, site (KIND_ATTN_PROBS, layer),
+// identical to the SIMT kernels and the oracle.
+#include <cuda.h>
+
+#include <mutex>
+
+#include "kernels.h"
+#include "tc_common.cuh"
+
+namespace mimose {
+
+constexpr int AQ = 128;                  // rows of the tile (queries / keys)
+constexpr int AD = 64;                   // head dim
+constexpr int TILE = AQ * AD * 2;        // 16 KB: one [128 x 64] bf16 SW128 tile
+constexpr int PT = AQ * AQ * 2;          // 32 KB: one [128 x 128] bf16 tile (2 atoms)
+
+struct AttnArgs {
+  int S, H, h, B;
+  float scale;
+  Drop drop;
+  const int32_t* lengths;
+  const __nv_bfloat16* O;      // fwd output / bwd input
+  __nv_bfloat16* Oout;
+  float* lse;
+  const float* lse_in;
+  __nv_bfloat16* dqkv;
+  const __nv_bfloat16* dO;
+};
+
+// Write 32 consecutive bf16 values (keys [32c, 32c+32)) of row r into a
+// [128 x 128] K-major SW128 tile made of two 64-wide atoms.
+MDEV void st_tile_row32(uint8_t* tile, int r, int c, const float* v) {
+  const int atom = c >> 1, cb = (c & 1) * 4;
+  uint8_t* base = tile + atom * (AQ * 128);
+#pragma unroll
+  for (int j = 0; j < 4; ++j) *(uint4*)(base + sw128(r, cb + j)) = pack8(v + 8 * j);
+}
+
+MDEV float4 drop4_or(const Drop& d, uint64_t e) {
+  if (!d.enabled) return make_float4(1.f, 1.f, 1.f, 1.f);
+  if ((e & 3) == 0) return drop_factor4(d, e >> 2);
+  return make_float4(drop_factor(d, e), drop_factor(d, e + 1), drop_factor(d, e + 2), drop_factor(d, e + 3));
+}
+
+__global__ void __launch_bounds__(128) k_attn_fwd_tc(const __grid_constant__ CUtensorMap tq, const AttnArgs a) {
+  extern __shared__ uint8_t smem_raw[];
+  uint8_t* sm = (uint8_t*)(((uintptr_t)smem_raw + 1023) & ~(uintptr_t)1023);
+  uint8_t* sQ = sm;
+  uint8_t* sK = sm + TILE;
+  uint8_t* sV = sm + 2 * TILE;
+  uint8_t* sP = sm + 3 * TILE;
+  uint64_t* bar = (uint64_t*)(sP + PT);   // [0] tma, [1] mma S, [2] mma O
+  uint32_t* tslot = (uint32_t*)(bar + 4);
+  const int t = threadIdx.x, warp = t >> 5;
+  const int bh = blockIdx.x, b = bh / a.h, hd = bh % a.h;
+  const int S = a.S, len = a.lengths[b];
+  if (t == 0) {
+    for (int i = 0; i < 3; ++i) mbar_init(&bar[i], 1);
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+  }
+  if (warp == 0) {
+    asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(smem_u32(tslot)), "r"(256));
+    asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;");
+  }
+  tc_fence_before();
+  __syncthreads();
+  tc_fence_after();
+  const uint32_t tmem = *tslot;
+  const int row0 = b * S;
+  if (t == 0) {
+    mbar_expect_tx(&bar[0], 3 * TILE);
+    tma_load_2d(&tq, &bar[0], sQ, hd * AD, row0);
+    tma_load_2d(&tq, &bar[0], sK, a.H + hd * AD, row0);
+    tma_load_2d(&tq, &bar[0], sV, 2 * a.H + hd * AD, row0);
+    mbar_wait(&bar[0], 0);
+    tc_fence_after();
+    const uint32_t id = idesc_bf16(AQ, AQ, 0, 0);
+    const uint32_t q0 = smem_u32(sQ), k0 = smem_u32(sK);
+#pragma unroll
+    for (int kk = 0; kk < AD / 16; ++kk)
+      mma_bf16(tmem, make_desc(q0 + 32 * kk, 16, 1024), make_desc(k0 + 32 * kk, 16, 1024), id, kk > 0);
+    mma_commit(&bar[1]);
+  }
+  mbar_wait(&bar[1], 0);
+  __syncwarp();
+  tc_fence_after();
+  // ---- softmax of row t over keys [0, len) ----
+  const uint32_t trow = tmem + ((uint32_t)(32 * warp) << 16);
+  float m = -INFINITY, l = 0.f;
+#pragma unroll 1
+  for (int c = 0; c < 4; ++c) {
+    float v[32];
+    tmem_ld32(trow + 32 * c, v);
+#pragma unroll
+    for (int i = 0; i < 32; ++i) {
+      const float s = (32 * c + i < len) ? v[i] * a.scale : -INFINITY;
+      if (s > m) { l = l * __expf(m - s) + 1.f; m = s; } else { l += __expf(s - m); }
+    }
+  }
+  const float L = m + __logf(l);
+  const uint64_t ebase = (((uint64_t)b * a.h + hd) * S + (uint64_t)t) * S;
+#pragma unroll 1
+  for (int c = 0; c < 4; ++c) {
+    float v[32];
+    tmem_ld32(trow + 32 * c, v);
+#pragma unroll
+    for (int j = 0; j < 8; ++j) {
+      const int k = 32 * c + 4 * j;
+      const float4 f = (t < S && k < len) ? drop4_or(a.drop, ebase + k) : make_float4(0.f, 0.f, 0.f, 0.f);
+      const float ff[4] = {f.x, f.y, f.z, f.w};
+#pragma unroll
+      for (int i = 0; i < 4; ++i)
+        v[4 * j + i] = (k + i < len) ? __expf(v[4 * j + i] * a.scale - L) * ff[i] : 0.f;
+    }
+    st_tile_row32(sP, t, c, v);
+  }
+  fence_async_smem();
+  tc_fence_before();
+  __syncthreads();
+  tc_fence_after();
+  if (t == 0) {
+    const uint32_t id = idesc_bf16(AQ, AD, 0, 1);
+    const uint32_t p0 = smem_u32(sP), v0 = smem_u32(sV);
+#pragma unroll
+    for (int kk = 0; kk < AQ / 16; ++kk) {
+      const uint64_t da = make_desc(p0 + (kk >> 2) * (AQ * 128) + 32 * (kk & 3), 16, 1024);
+      const uint64_t db = make_desc(v0 + 2048 * kk, 16384, 1024);
+      mma_bf16(tmem + 128, da, db, id, kk > 0);
+    }
+    mma_commit(&bar[2]);
+  }
+  mbar_wait(&bar[2], 0);
+  __syncwarp();
+  tc_fence_after();
+  {  // tcgen05.ld is .sync.aligned: every lane loads, only rows t < S store
+    __nv_bfloat16* orow = a.Oout + ((int64_t)row0 + t) * a.H + hd * AD;
+#pragma unroll
+    for (int c = 0; c < 2; ++c) {
+      float v[32];
+      tmem_ld32(trow + 128 + 32 * c, v);
+      if (t < S) st_bf16x32(orow + 32 * c, v);
+    }
+    if (t < S) a.lse[((int64_t)b * a.h + hd) * S + t] = L;
+  }
+  tc_fence_before();
+  __syncthreads();
+  if (warp == 0) {
+    tc_fence_after();
+    asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(tmem), "r"(256));
+  }
+}
+
+__global__ void __launch_bounds__(128) k_attn_bwd_tc(const __grid_constant__ CUtensorMap tq,
+                                                     const __grid_constant__ CUtensorMap tdo, const AttnArgs a) {
+  extern __shared__ uint8_t smem_raw[];
+  uint8_t* sm = (uint8_t*)(((uintptr_t)smem_raw + 1023) & ~(uintptr_t)1023);
+  uint8_t* sQ = sm;
+  uint8_t* sK = sm + TILE;
+  uint8_t* sV = sm + 2 * TILE;
+  uint8_t* sdO = sm + 3 * TILE;
+  uint8_t* sP = sm + 4 * TILE;
+  uint8_t* sdS = sP + PT;
+  uint64_t* bar = (uint64_t*)(sdS + PT);  // [0] tma, [1] mma S/dP, [2] mma grads
+  uint32_t* tslot = (uint32_t*)(bar + 4);
+  const int t = threadIdx.x, warp = t >> 5;
+  const int bh = blockIdx.x, b = bh / a.h, hd = bh % a.h;
+  const int S = a.S, len = a.lengths[b];
+  if (t == 0) {
+    for (int i = 0; i < 3; ++i) mbar_init(&bar[i], 1);
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+  }
+  if (warp == 0) {
+    asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(smem_u32(tslot)), "r"(256));
+    asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;");
+  }
+  tc_fence_before();
+  __syncthreads();
+  tc_fence_after();
+  const uint32_t tmem = *tslot;
+  const int row0 = b * S;
+  if (t == 0) {
+    mbar_expect_tx(&bar[0], 4 * TILE);
+    tma_load_2d(&tq, &bar[0], sQ, hd * AD, row0);
+    tma_load_2d(&tq, &bar[0], sK, a.H + hd * AD, row0);
+    tma_load_2d(&tq, &bar[0], sV, 2 * a.H + hd * AD, row0);
+    tma_load_2d(&tdo, &bar[0], sdO, hd * AD, row0);
+    mbar_wait(&bar[0], 0);
+    tc_fence_after();
+    const uint32_t id = idesc_bf16(AQ, AQ, 0, 0);
+    const uint32_t q0 = smem_u32(sQ), k0 = smem_u32(sK), v0 = smem_u32(sV), o0 = smem_u32(sdO);
+#pragma unroll
+    for (int kk = 0; kk < AD / 16; ++kk)
+      mma_bf16(tmem, make_desc(q0 + 32 * kk, 16, 1024), make_desc(k0 + 32 * kk, 16, 1024), id, kk > 0);
+#pragma unroll
+    for (int kk = 0; kk < AD / 16; ++kk)
+      mma_bf16(tmem + 128, make_desc(o0 + 32 * kk, 16, 1024), make_desc(v0 + 32 * kk, 16, 1024), id, kk > 0);
+    mma_commit(&bar[1]);
+  }
+  // D_t = rowsum(dO * O) for query row t (global reads overlap the MMAs)
+  float Dt = 0.f, Lt = 0.f;
+  if (t < len) {
+    const __nv_bfloat16* orow = a.O + ((int64_t)row0 + t) * a.H + hd * AD;
+    const __nv_bfloat16* drow = a.dO + ((int64_t)row0 + t) * a.H + hd * AD;
+    float ov[32], dv[32];
+#pragma unroll
+    for (int c = 0; c < 2; ++c) {
+      ld_bf16x32(orow + 32 * c, ov);
+      ld_bf16x32(drow + 32 * c, dv);
+#pragma unroll
+      for (int i = 0; i < 32; ++i) Dt += ov[i] * dv[i];
+    }
+    Lt = a.lse_in[((int64_t)b * a.h + hd) * S + t];
+  }
+  mbar_wait(&bar[1], 0);
+  __syncwarp();
+  tc_fence_after();
+  const uint32_t trow = tmem + ((uint32_t)(32 * warp) << 16);
+  const uint64_t ebase = (((uint64_t)b * a.h + hd) * S + (uint64_t)t) * S;
+#pragma unroll 1
+  for (int c = 0; c < 4; ++c) {
+    float sv[32], dp[32];
+    tmem_ld32(trow + 32 * c, sv);
+    tmem_ld32(trow + 128 + 32 * c, dp);
+#pragma unroll
+    for (int j = 0; j < 8; ++j) {
+      const int k = 32 * c + 4 * j;
+      const bool live = t < len;                // padded / foreign query rows contribute 0
+      const float4 f = (live && k < len) ? drop4_or(a.drop, ebase + k) : make_float4(0.f, 0.f, 0.f, 0.f);
+      const float ff[4] = {f.x, f.y, f.z, f.w};
+#pragma unroll
+      for (int i = 0; i < 4; ++i) {
+        const int kk = k + i;
+        const float p = (live && kk < len) ? __expf(sv[4 * j + i] * a.scale - Lt) : 0.f;
+        sv[4 * j + i] = p * ff[i];                                  // P~
+        dp[4 * j + i] = p * (dp[4 * j + i] * ff[i] - Dt) * a.scale; // dS (scale folded)
+      }
+    }
+    st_tile_row32(sP, t, c, sv);
+    st_tile_row32(sdS, t, c, dp);
+  }
+  fence_async_smem();
+  tc_fence_before();
+  __syncthreads();
+  tc_fence_after();
+  if (t == 0) {
+    const uint32_t id_t = idesc_bf16(AQ, AD, 1, 1);   // A MN-major (keys), B MN-major (d)
+    const uint32_t id_q = idesc_bf16(AQ, AD, 0, 1);   // A K-major (queries), B MN-major (d)
+    const uint32_t p0 = smem_u32(sP), s0 = smem_u32(sdS);
+    const uint32_t q0 = smem_u32(sQ), k0 = smem_u32(sK), o0 = smem_u32(sdO);
+#pragma unroll
+    for (int kk = 0; kk < AQ / 16; ++kk) {      // contraction over queries (dV, dK) / keys (dQ)
+      const uint64_t at_p = make_desc(p0 + 2048 * kk, 16384, 1024);
+      const uint64_t at_s = make_desc(s0 + 2048 * kk, 16384, 1024);
+      const uint64_t bq_do = make_desc(o0 + 2048 * kk, 16384, 1024);
+      const uint64_t bq_q = make_desc(q0 + 2048 * kk, 16384, 1024);
+      mma_bf16(tmem + 0, at_p, bq_do, id_t, kk > 0);          // dV = P~^T dO
+      mma_bf16(tmem + 64, at_s, bq_q, id_t, kk > 0);          // dK = dS^T Q
+      const uint64_t ak_s = make_desc(s0 + (kk >> 2) * (AQ * 128) + 32 * (kk & 3), 16, 1024);
+      const uint64_t bk_k = make_desc(k0 + 2048 * kk, 16384, 1024);
+      mma_bf16(tmem + 128, ak_s, bk_k, id_q, kk > 0);         // dQ = dS K
+    }
+    mma_commit(&bar[2]);
+  }
+  mbar_wait(&bar[2], 0);
+  __syncwarp();
+  tc_fence_after();
+  {  // every lane loads (.sync.aligned); rows t < S store
+    __nv_bfloat16* row = a.dqkv + ((int64_t)row0 + t) * 3 * a.H + hd * AD;
+    const bool st = t < S;
+#pragma unroll
+    for (int c = 0; c < 2; ++c) {
+      float v[32];
+      tmem_ld32(trow + 128 + 32 * c, v);
+      if (st) st_bf16x32(row + 32 * c, v);                     // dQ
+      tmem_ld32(trow + 64 + 32 * c, v);
+      if (st) st_bf16x32(row + a.H + 32 * c, v);               // dK
+      tmem_ld32(trow + 32 * c, v);
+      if (st) st_bf16x32(row + 2 * a.H + 32 * c, v);           // dV
+    }
+  }
+  tc_fence_before();
+  __syncthreads();
+  if (warp == 0) {
+    tc_fence_after();
+    asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(tmem), "r"(256));
+  }
+}
+
+// ------------------------------------------------------------------ host --
+bool tc_map_bf16(CUtensorMap* out, const void* ptr, uint64_t inner, uint64_t outer, uint64_t stride_elems,
+                 uint32_t box_inner, uint32_t box_outer);   // kernels_gemm_tc.cu
+
+constexpr int FWD_SMEM = 3 * TILE + PT + 1024 + 128;
+constexpr int BWD_SMEM = 4 * TILE + 2 * PT + 1024 + 128;
+
+bool attn_tc_ok(int S, int H, int h) { return S <= AQ && H / h == AD && H % 64 == 0; }
+
+bool attn_fwd_tc(const void* qkv, const int32_t* lengths, void* O, float* lse, int B, int S, int H, int h,
+                 Drop drop, cudaStream_t st) {
+  if (!attn_tc_ok(S, H, h)) return false;
+  CUtensorMap tq;
+  if (!tc_map_bf16(&tq, qkv, 3ull * H, (uint64_t)B * S, 3ull * H, 64, AQ)) return false;
+  static std::once_flag once;
+  std::call_once(once, [] { cudaFuncSetAttribute(k_attn_fwd_tc, cudaFuncAttributeMaxDynamicSharedMemorySize, FWD_SMEM); });
+  AttnArgs a{};
+  a.S = S; a.H = H; a.h = h; a.B = B;
+  a.scale = 1.0f / sqrtf((float)AD);
+  a.drop = drop; a.lengths = lengths; a.Oout = (__nv_bfloat16*)O; a.lse = lse;
+  k_attn_fwd_tc<<<B * h, 128, FWD_SMEM, st>>>(tq, a);
+  return true;
+}
+
+bool attn_bwd_tc(const void* qkv, const void* O, const void* dO, const float* lse, const int32_t* lengths,
+                 void* dqkv, int B, int S, int H, int h, Drop drop, cudaStream_t st) {
+  if (!attn_tc_ok(S, H, h)) return false;
+  CUtensorMap tq, tdo;
+  if (!tc_map_bf16(&tq, qkv, 3ull * H, (uint64_t)B * S, 3ull * H, 64, AQ)) return false;
+  if (!tc_map_bf16(&tdo, dO, (uint64_t)H, (uint64_t)B * S, (uint64_t)H, 64, AQ)) return false;
+  static std::once_flag once;
+  std::call_once(once, [] { cudaFuncSetAttribute(k_attn_bwd_tc, cudaFuncAttributeMaxDynamicSharedMemorySize, BWD_SMEM); });
+  AttnArgs a{};
+  a.S = S; a.H = H; a.h = h; a.B = B;
+  a.scale = 1.0f / sqrtf((float)AD);
+  a.drop = drop; a.lengths = lengths; a.O = (const __nv_bfloat16*)O; a.dO = (const __nv_bfloat16*)dO;
+  a.lse_in = lse; a.dqkv = (__nv_bfloat16*)dqkv;
+  k_attn_bwd_tc<<<B * h, 128, BWD_SMEM, st>>>(tq, tdo, a);
+  return true;
+}
+
+}  // namespace mimose

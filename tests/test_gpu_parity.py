@@ -88,6 +88,9 @@ CASES = {
                                max_pos=64, n_seqs=8, seq_lo=8, seq_hi=40, pad=8),
     "qa-bf16": wl.small_config("bert-large", n_layers=2, hidden=128, heads=2, ffn=512, vocab=300,
                                max_pos=80, n_seqs=3, seq_lo=20, seq_hi=72, pad=8),
+    # S > 128: the bf16 attention takes the SIMT path (tcgen05 tile covers S <= 128)
+    "qa-bf16-long": wl.small_config("bert-large", n_layers=2, hidden=128, heads=2, ffn=256, vocab=300,
+                                    max_pos=200, n_seqs=2, seq_lo=130, seq_hi=190, pad=8),
     "qa-fp32": wl.small_config("bert-large", n_layers=2, hidden=64, heads=2, ffn=128, vocab=300,
                                max_pos=80, n_seqs=3, seq_lo=20, seq_hi=70, pad=1, dtype="fp32"),
     "mc-roberta-bf16": wl.small_config("roberta-large", n_layers=2, hidden=128, heads=2, ffn=256,
