@@ -238,6 +238,11 @@ mimose_status mimose_debug_gemm(int32_t epi, int32_t M, int32_t N, int32_t K, co
                                 int64_t a_sk, const void* B, int64_t b_sn, int64_t b_sk, void* C, int64_t ldc,
                                 const void* bias, int32_t split, int32_t use_tc, void* stream);
 
+/* Test hook: process-wide kernel options. gemm_mode 0 = one 128x128 tile per CTA,
+   1 = persistent double-buffered tcgen05 GEMM (default); attn_tc 0/1 routes bf16
+   attention with S <= 128 to the SIMT / tcgen05 kernels.  Negative = unchanged. */
+void mimose_debug_options(int32_t gemm_mode, int32_t attn_tc);
+
 /* 1 if this build routes bf16 GEMMs to the tcgen05/TMEM/TMA kernels. */
 int32_t mimose_tc_available(void);
 

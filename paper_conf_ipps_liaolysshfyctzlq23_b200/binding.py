@@ -145,6 +145,15 @@ def debug_gemm(epi, M, N, K, A, a_sm, a_sk, B, b_sn, b_sk, Cm, ldc, bias=None, s
         raise MimoseError(st, "debug_gemm")
 
 
+_lib.mimose_debug_options.argtypes = [C.c_int32, C.c_int32]
+_lib.mimose_debug_options.restype = None
+EXPORTED.append("mimose_debug_options")
+
+
+def debug_options(gemm_mode: int = -1, attn_tc: int = -1):
+    _lib.mimose_debug_options(gemm_mode, attn_tc)
+
+
 def tc_gemm_available() -> bool:
     return bool(_lib.mimose_tc_available())
 

@@ -11,7 +11,8 @@ MDEV float gelu_grad_f(float u) {
 
 // Epilogue of one output element.
 template <typename E, int EPI>
-MDEV void epilogue(const GemmArgs& g, int m, int n, float acc) {
+MDEV void epilogue(const GemmArgs& g, int m, int n, float acc, int z = -1) {
+  if (z < 0) z = blockIdx.z;
   const int64_t o = (int64_t)m * g.ldc + n;
   if constexpr (EPI == EPI_STORE) {
     stf((E*)g.C + o, acc);
@@ -29,7 +30,7 @@ MDEV void epilogue(const GemmArgs& g, int m, int n, float acc) {
   } else if constexpr (EPI == EPI_ACC_RES_F32) {
     ((float*)g.C)[o] = acc + ((const float*)g.res)[(int64_t)m * g.ldr + n];
   } else {
-    ((float*)g.C)[(int64_t)blockIdx.z * g.split_stride + o] = acc;
+    ((float*)g.C)[(int64_t)z * g.split_stride + o] = acc;
   }
 }
 

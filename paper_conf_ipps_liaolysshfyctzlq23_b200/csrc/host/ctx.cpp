@@ -414,9 +414,8 @@ void layer_backward(Run& r, int l, const char* x, LayerBufs& b, float* dy, char*
   // LN2 backward + dropout backward -> dz2 (dres), dt2 (R3), partials
   ln_bwd(c->dt, dy, no_drop(), b.z2, b.st2, W(c, LP(c, l, L_LN2G)), dres, R3, make_drop(c, KIND_FFN_OUT, l),
          pg, pb, pbias, T, H, r.st);
-  reduce_partials(pg, H, H, G(c, LP(c, l, L_LN2G)), r.st);
-  reduce_partials(pb, H, H, G(c, LP(c, l, L_LN2B)), r.st);
-  reduce_partials(pbias, H, H, G(c, LP(c, l, L_F2B)), r.st);
+  reduce_rows3(pg, G(c, LP(c, l, L_LN2G)), pb, G(c, LP(c, l, L_LN2B)), pbias, G(c, LP(c, l, L_F2B)), NPART, H, H,
+               r.st);
   // FFN2: du = (dt2 W2) * gelu'(u); dW2 = dt2^T g
   dgrad(r, EPI_GELU_BWD, R3, H, W(c, LP(c, l, L_F2W)), F, R2, b.u);
   wgrad(r, R3, H, b.g, F, G(c, LP(c, l, L_F2W)));
@@ -428,9 +427,8 @@ void layer_backward(Run& r, int l, const char* x, LayerBufs& b, float* dy, char*
   // LN1 backward + dropout backward -> dz1 (dres, in place), dt1 (R3)
   ln_bwd(c->dt, dres, no_drop(), b.z1, b.st1, W(c, LP(c, l, L_LN1G)), dres, R3, make_drop(c, KIND_ATTN_OUT, l),
          pg, pb, pbias, T, H, r.st);
-  reduce_partials(pg, H, H, G(c, LP(c, l, L_LN1G)), r.st);
-  reduce_partials(pb, H, H, G(c, LP(c, l, L_LN1B)), r.st);
-  reduce_partials(pbias, H, H, G(c, LP(c, l, L_OB)), r.st);
+  reduce_rows3(pg, G(c, LP(c, l, L_LN1G)), pb, G(c, LP(c, l, L_LN1B)), pbias, G(c, LP(c, l, L_OB)), NPART, H, H,
+               r.st);
   // out-proj: dO = dt1 Wo (R2); dWo = dt1^T O
   dgrad(r, EPI_STORE, R3, H, W(c, LP(c, l, L_OW)), H, R2, nullptr);
   wgrad(r, R3, H, b.O, H, G(c, LP(c, l, L_OW)));
@@ -605,8 +603,7 @@ mimose_status run_backward(Run& r, Sample* sample) {
     float* pb = c->part + (int64_t)NPART * H;
     ln_bwd(c->dt, dy, make_drop(c, KIND_EMB, LAYER_NONE), c->z0, c->st0, W(c, P_LN0G), dz0, nullptr, no_drop(), pg,
            pb, nullptr, T, H, r.st);
-    reduce_partials(pg, H, H, G(c, P_LN0G), r.st);
-    reduce_partials(pb, H, H, G(c, P_LN0B), r.st);
+    reduce_rows3(pg, G(c, P_LN0G), pb, G(c, P_LN0B), nullptr, nullptr, NPART, H, H, r.st);
     const int64_t e0 = c->layout[P_WORD].off, e1 = bucket_end(c, P_TYPE);
     CK(cudaMemsetAsync(c->grad + e0, 0, (size_t)(e1 - e0) * 4, r.st));
     pos_grad(dz0, c->B, c->S, H, c->cfg.pos_offset, G(c, P_POS), r.st);
@@ -1030,6 +1027,11 @@ mimose_status mimose_plan(mimose_ctx* c, int64_t x, mimose_plan_t* out) {
 }
 
 int32_t mimose_tc_available(void) { return tc_available() ? 1 : 0; }
+
+void mimose_debug_options(int32_t gemm_mode, int32_t attn_tc) {
+  if (gemm_mode >= 0) set_gemm_mode(gemm_mode);
+  if (attn_tc >= 0) set_attn_tc(attn_tc != 0);
+}
 
 mimose_status mimose_debug_gemm(int32_t epi, int32_t M, int32_t N, int32_t K, const void* A, int64_t a_sm,
                                 int64_t a_sk, const void* B, int64_t b_sn, int64_t b_sk, void* Cp, int64_t ldc,

@@ -37,6 +37,8 @@ struct GemmArgs {
 };
 void gemm(DType dt, Epi epi, const GemmArgs& g, cudaStream_t st, bool use_tc);
 bool tc_available();
+// 0: one tile per CTA; 1: persistent double-buffered (default).
+void set_gemm_mode(int m);
 // Deterministic split-K reduction: out[i] = sum_s part[s*n + i] (fixed order).
 void splitk_reduce(const float* part, int splits, int64_t n, float* out, cudaStream_t st);
 
@@ -64,6 +66,9 @@ void ln_bwd(DType dt, const float* dy, Drop premask, const float* z, const float
             float* pbias, int T, int H, cudaStream_t st_);
 // out[c] = sum_p part[p*ld + c], p = 0..NPART-1 (fixed order)
 void reduce_partials(const float* part, int64_t ld, int n, float* out, cudaStream_t st);
+// Up to three such reductions in one launch (p1/p2 may be null), `rows` partial rows.
+void reduce_rows3(const float* p0, float* o0, const float* p1, float* o1, const float* p2, float* o2, int rows,
+                  int64_t ld, int n, cudaStream_t st);
 // partials [NPART][N] of column sums of X [T, N] (E)
 void colsum(DType dt, const void* X, int T, int N, float* part, cudaStream_t st);
 

@@ -25,35 +25,75 @@ static void dispatch(DType dt, F f) {
 static inline int cdiv(int64_t a, int64_t b) { return (int)((a + b - 1) / b); }
 
 // ===================================================================== LN ===
+// Vector helpers: 8 consecutive elements (16 B of bf16 / 32 B of fp32).
+MDEV void ld8(const float* p, float* v) {
+  const float4 a = ((const float4*)p)[0], b = ((const float4*)p)[1];
+  v[0] = a.x; v[1] = a.y; v[2] = a.z; v[3] = a.w; v[4] = b.x; v[5] = b.y; v[6] = b.z; v[7] = b.w;
+}
+MDEV void ld8(const __nv_bfloat16* p, float* v) {
+  const uint4 u = *(const uint4*)p;
+  const __nv_bfloat162* h = (const __nv_bfloat162*)&u;
+#pragma unroll
+  for (int i = 0; i < 4; ++i) { const float2 f = __bfloat1622float2(h[i]); v[2 * i] = f.x; v[2 * i + 1] = f.y; }
+}
+MDEV void st8(float* p, const float* v) {
+  ((float4*)p)[0] = make_float4(v[0], v[1], v[2], v[3]);
+  ((float4*)p)[1] = make_float4(v[4], v[5], v[6], v[7]);
+}
+MDEV void st8(__nv_bfloat16* p, const float* v) {
+  uint4 u;
+  __nv_bfloat162* h = (__nv_bfloat162*)&u;
+#pragma unroll
+  for (int i = 0; i < 4; ++i) h[i] = __floats2bfloat162_rn(v[2 * i], v[2 * i + 1]);
+  *(uint4*)p = u;
+}
+MDEV void drop8(const Drop& d, uint64_t e, float* f) {   // e multiple of 8
+  const float4 a = drop_factor4(d, e >> 2), b = drop_factor4(d, (e >> 2) + 1);
+  f[0] = a.x; f[1] = a.y; f[2] = a.z; f[3] = a.w; f[4] = b.x; f[5] = b.y; f[6] = b.z; f[7] = b.w;
+}
 
+// warp per row; lane owns 8-column chunks j = lane + 32 k (H % 8 == 0, H <= 1024)
 template <typename E>
 __global__ void __launch_bounds__(256) k_ln_fwd(const float* __restrict__ z, const E* __restrict__ g,
                                                 const E* __restrict__ b, E* __restrict__ y,
                                                 float2* __restrict__ st, int T, int H, float eps) {
   const int row = (blockIdx.x * blockDim.x + threadIdx.x) >> 5, lane = threadIdx.x & 31;
   if (row >= T) return;
-  const int nv = H >> 5;
+  const int nch = H >> 3;
   const float* zr = z + (int64_t)row * H;
-  float v[32];
+  float v[4][8];
   float s = 0.f;
 #pragma unroll
-  for (int k = 0; k < 32; ++k)
-    if (k < nv) { v[k] = ldf(zr + lane + 32 * k); s += v[k]; }
+  for (int k = 0; k < 4; ++k) {
+    const int j = lane + 32 * k;
+    if (j < nch) {
+      ld8(zr + 8 * j, v[k]);
+#pragma unroll
+      for (int i = 0; i < 8; ++i) s += v[k][i];
+    }
+  }
   const float mu = warp_sum(s) / (float)H;
   float q = 0.f;
 #pragma unroll
-  for (int k = 0; k < 32; ++k)
-    if (k < nv) { const float d = v[k] - mu; q += d * d; }
+  for (int k = 0; k < 4; ++k)
+    if (lane + 32 * k < nch)
+#pragma unroll
+      for (int i = 0; i < 8; ++i) { const float d = v[k][i] - mu; q += d * d; }
   const float rstd = rsqrtf(warp_sum(q) / (float)H + eps);
   if (lane == 0) st[row] = make_float2(mu, rstd);
   if (y) {
-    E* yr = y + (int64_t)row * H;
 #pragma unroll
-    for (int k = 0; k < 32; ++k)
-      if (k < nv) {
-        const int c = lane + 32 * k;
-        stf(yr + c, (v[k] - mu) * rstd * ldf(g + c) + ldf(b + c));
+    for (int k = 0; k < 4; ++k) {
+      const int j = lane + 32 * k;
+      if (j < nch) {
+        float gv[8], bv[8], o[8];
+        ld8(g + 8 * j, gv);
+        ld8(b + 8 * j, bv);
+#pragma unroll
+        for (int i = 0; i < 8; ++i) o[i] = (v[k][i] - mu) * rstd * gv[i] + bv[i];
+        st8(y + (int64_t)row * H + 8 * j, o);
       }
+    }
   }
 }
 
@@ -66,7 +106,9 @@ void ln_fwd(DType dt, const float* z, const void* g, const void* b, void* y, flo
   });
 }
 
-// 8 warps per CTA, NPART CTAs; warp w of CTA p owns rows r = p*8 + w + k*NPART*8.
+// NPART CTAs x 8 warps; warp w of CTA p owns rows r = p*8 + w + k*NPART*8 (fixed).
+// Per-lane register partials of dgamma, dbeta, dbias over the warp's rows, then a
+// fixed-order reduction over the 8 warps through shared memory.
 template <typename E>
 __global__ void __launch_bounds__(256) k_ln_bwd(const float* dy, Drop premask, const float* __restrict__ z,
                                                 const float2* __restrict__ st, const E* __restrict__ g,
@@ -75,48 +117,77 @@ __global__ void __launch_bounds__(256) k_ln_bwd(const float* dy, Drop premask, c
                                                 float* __restrict__ pbias, int T, int H) {
   extern __shared__ float sm[];
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
-  float* ag = sm + (size_t)warp * 3 * H;
-  float* ab = ag + H;
-  float* at = ab + H;
-  for (int c = lane; c < H; c += 32) { ag[c] = 0.f; ab[c] = 0.f; at[c] = 0.f; }
-  const int nv = H >> 5;
+  const int nch = H >> 3;
   const float invH = 1.0f / (float)H;
+  float ag[4][8], ab[4][8], at[4][8], gv[4][8];
+#pragma unroll
+  for (int k = 0; k < 4; ++k) {
+    const int j = lane + 32 * k;
+#pragma unroll
+    for (int i = 0; i < 8; ++i) { ag[k][i] = 0.f; ab[k][i] = 0.f; at[k][i] = 0.f; gv[k][i] = 0.f; }
+    if (j < nch) ld8(g + 8 * j, gv[k]);
+  }
   for (int row = blockIdx.x * 8 + warp; row < T; row += NPART * 8) {
-    const float* dyr = dy + (int64_t)row * H;
-    const float* zr = z + (int64_t)row * H;
     const float2 ms = st[row];
-    float xh[32], dyv[32];
+    float dyv[4][8], xh[4][8];
     float s1 = 0.f, s2 = 0.f;
 #pragma unroll
-    for (int k = 0; k < 32; ++k)
-      if (k < nv) {
-        const int c = lane + 32 * k;
-        float d = dyr[c];
-        if (premask.enabled) d *= drop_factor(premask, (uint64_t)row * H + c);
-        dyv[k] = d;
-        xh[k] = (ldf(zr + c) - ms.x) * ms.y;
-        const float dxh = d * ldf(g + c);
-        s1 += dxh;
-        s2 += dxh * xh[k];
-      }
-    s1 = warp_sum(s1) * invH;
-    s2 = warp_sum(s2) * invH;
-    float* dzr = dz + (int64_t)row * H;
+    for (int k = 0; k < 4; ++k) {
+      const int j = lane + 32 * k;
+      if (j < nch) {
+        ld8(dy + (int64_t)row * H + 8 * j, dyv[k]);
+        ld8(z + (int64_t)row * H + 8 * j, xh[k]);
+        if (premask.enabled) {
+          float f[8];
+          drop8(premask, (uint64_t)row * H + 8 * j, f);
 #pragma unroll
-    for (int k = 0; k < 32; ++k)
-      if (k < nv) {
-        const int c = lane + 32 * k;
-        const float dxh = dyv[k] * ldf(g + c);
-        const float v = ms.y * (dxh - s1 - xh[k] * s2);
-        ag[c] += dyv[k] * xh[k];
-        ab[c] += dyv[k];
-        dzr[c] = v;
-        if (dtout) {
-          E* p = dtout + (int64_t)row * H + c;
-          stf(p, v * drop_factor(mask, (uint64_t)row * H + c));
-          at[c] += ldf(p);
+          for (int i = 0; i < 8; ++i) dyv[k][i] *= f[i];
+        }
+#pragma unroll
+        for (int i = 0; i < 8; ++i) {
+          xh[k][i] = (xh[k][i] - ms.x) * ms.y;
+          const float dxh = dyv[k][i] * gv[k][i];
+          s1 += dxh;
+          s2 += dxh * xh[k][i];
         }
       }
+    }
+    s1 = warp_sum(s1) * invH;
+    s2 = warp_sum(s2) * invH;
+#pragma unroll
+    for (int k = 0; k < 4; ++k) {
+      const int j = lane + 32 * k;
+      if (j < nch) {
+        float o[8];
+#pragma unroll
+        for (int i = 0; i < 8; ++i) {
+          o[i] = ms.y * (dyv[k][i] * gv[k][i] - s1 - xh[k][i] * s2);
+          ag[k][i] += dyv[k][i] * xh[k][i];
+          ab[k][i] += dyv[k][i];
+        }
+        st8(dz + (int64_t)row * H + 8 * j, o);
+        if (dtout) {
+          float f[8];
+          drop8(mask, (uint64_t)row * H + 8 * j, f);
+#pragma unroll
+          for (int i = 0; i < 8; ++i) o[i] = rnd(o[i] * f[i], dtout);   // the stored value
+          st8(dtout + (int64_t)row * H + 8 * j, o);
+#pragma unroll
+          for (int i = 0; i < 8; ++i) at[k][i] += o[i];
+        }
+      }
+    }
+  }
+  // fixed-order cross-warp reduction: smem [8 warps][3][H]
+#pragma unroll
+  for (int k = 0; k < 4; ++k) {
+    const int j = lane + 32 * k;
+    if (j < nch) {
+      float* base = sm + (size_t)warp * 3 * H + 8 * j;
+      st8(base, ag[k]);
+      st8(base + H, ab[k]);
+      st8(base + 2 * H, at[k]);
+    }
   }
   __syncthreads();
   for (int c = threadIdx.x; c < H; c += blockDim.x) {
@@ -148,23 +219,47 @@ void ln_bwd(DType dt, const float* dy, Drop premask, const float* z, const float
   });
 }
 
-__global__ void k_reduce_partials(const float* __restrict__ part, int64_t ld, int n, float* __restrict__ out) {
-  const int c = blockIdx.x * blockDim.x + threadIdx.x;
-  if (c >= n) return;
-  float s = 0.f;
-  for (int p = 0; p < NPART; ++p) s += part[(int64_t)p * ld + c];
-  out[c] = s;
+// out[c] = sum_{p < rows} part[p*ld + c] in a fixed order: warp w sums rows
+// p = w, w+8, ... ascending; warp 0 then adds the 8 warp sums in order w = 0..7.
+// blockIdx.y selects one of up to 3 (part, out) pairs.
+struct RedJob { const float* part; float* out; };
+struct RedJobs { RedJob j[3]; };
+__global__ void __launch_bounds__(256) k_reduce_rows(RedJobs jobs, int rows, int64_t ld, int n) {
+  __shared__ float sw[8][33];
+  const RedJob jb = jobs.j[blockIdx.y];
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const int c = blockIdx.x * 32 + lane;
+  float acc = 0.f;
+  if (c < n)
+    for (int p = warp; p < rows; p += 8) acc += jb.part[(int64_t)p * ld + c];
+  sw[warp][lane] = acc;
+  __syncthreads();
+  if (warp == 0 && c < n) {
+    float t = 0.f;
+#pragma unroll
+    for (int w = 0; w < 8; ++w) t += sw[w][lane];
+    jb.out[c] = t;
+  }
+}
+void reduce_rows3(const float* p0, float* o0, const float* p1, float* o1, const float* p2, float* o2, int rows,
+                  int64_t ld, int n, cudaStream_t s) {
+  note_launch(1);
+  RedJobs jobs{{{p0, o0}, {p1, o1}, {p2, o2}}};
+  const int nj = p2 ? 3 : p1 ? 2 : 1;
+  k_reduce_rows<<<dim3(cdiv(n, 32), nj), 256, 0, s>>>(jobs, rows, ld, n);
 }
 void reduce_partials(const float* part, int64_t ld, int n, float* out, cudaStream_t s) {
-  note_launch(1);
-  k_reduce_partials<<<cdiv(n, 256), 256, 0, s>>>(part, ld, n, out);
+  reduce_rows3(part, out, nullptr, nullptr, nullptr, nullptr, NPART, ld, n, s);
 }
 
 __global__ void k_splitk_reduce(const float* __restrict__ part, int splits, int64_t n, float* __restrict__ out) {
-  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
-    float s = 0.f;
-    for (int k = 0; k < splits; ++k) s += part[k * n + i];
-    out[i] = s;
+  for (int64_t i = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) * 4; i < n; i += (int64_t)gridDim.x * blockDim.x * 4) {
+    float4 s = ((const float4*)(part + i))[0];
+    for (int k = 1; k < splits; ++k) {
+      const float4 v = ((const float4*)(part + k * n + i))[0];
+      s.x += v.x; s.y += v.y; s.z += v.z; s.w += v.w;
+    }
+    *(float4*)(out + i) = s;
   }
 }
 void splitk_reduce(const float* part, int splits, int64_t n, float* out, cudaStream_t s) {
@@ -172,31 +267,26 @@ void splitk_reduce(const float* part, int splits, int64_t n, float* out, cudaStr
   k_splitk_reduce<<<592, 256, 0, s>>>(part, splits, n, out);
 }
 
-// column sums of X [T, N]: CTA p owns rows p, p+NPART, ...; thread owns columns tid + 256 j.
+// column sums of X [T, N] (E): CTA (cx, p) owns rows p, p+NPART, ... and columns
+// [2048 cx, 2048 cx + 2048); a thread owns 8 consecutive columns.
 template <typename E>
 __global__ void __launch_bounds__(256) k_colsum(const E* __restrict__ X, int T, int N, float* __restrict__ part) {
-  float acc[16];
+  const int c = blockIdx.x * 2048 + threadIdx.x * 8;
+  if (c >= N) return;
+  float acc[8] = {0.f, 0.f, 0.f, 0.f, 0.f, 0.f, 0.f, 0.f};
+  for (int r = blockIdx.y; r < T; r += NPART) {
+    float v[8];
+    ld8(X + (int64_t)r * N + c, v);
 #pragma unroll
-  for (int j = 0; j < 16; ++j) acc[j] = 0.f;
-  for (int r = blockIdx.x; r < T; r += NPART) {
-    const E* xr = X + (int64_t)r * N;
-#pragma unroll
-    for (int j = 0; j < 16; ++j) {
-      const int c = threadIdx.x + 256 * j;
-      if (c < N) acc[j] += ldf(xr + c);
-    }
+    for (int i = 0; i < 8; ++i) acc[i] += v[i];
   }
-#pragma unroll
-  for (int j = 0; j < 16; ++j) {
-    const int c = threadIdx.x + 256 * j;
-    if (c < N) part[(int64_t)blockIdx.x * N + c] = acc[j];
-  }
+  st8(part + (int64_t)blockIdx.y * N + c, acc);
 }
 void colsum(DType dt, const void* X, int T, int N, float* part, cudaStream_t s) {
   note_launch(1);
   dispatch(dt, [&](auto* tag) {
     using E = std::remove_pointer_t<decltype(tag)>;
-    k_colsum<E><<<NPART, 256, 0, s>>>((const E*)X, T, N, part);
+    k_colsum<E><<<dim3(cdiv(N, 2048), NPART), 256, 0, s>>>((const E*)X, T, N, part);
   });
 }
 
@@ -686,21 +776,36 @@ void head_qa_bwd(DType dt, const void* y, int B, int S, int H, const void* Wq, c
 // ============================================================== optimizer ===
 
 template <typename E>
-__global__ void k_adamw(E* __restrict__ w, float* __restrict__ master, const float* __restrict__ g,
-                        float* __restrict__ m, float* __restrict__ v, int64_t n, float lr, float b1,
-                        float b2, float eps, float wd, float bc1, float bc2, float gs) {
+__global__ void __launch_bounds__(256) k_adamw(E* __restrict__ w, float* __restrict__ master, const float* __restrict__ g,
+                                               float* __restrict__ m, float* __restrict__ v, int64_t n, float lr, float b1,
+                                               float b2, float eps, float wd, float bc1, float bc2, float gs) {
   const float step = lr / bc1, rb2 = 1.0f / sqrtf(bc2), decay = 1.0f - lr * wd;
-  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
-    const float gi = g[i] * gs;
-    float p = master ? master[i] : ldf(w + i);
-    p *= decay;
-    const float mi = b1 * m[i] + (1.f - b1) * gi;
-    const float vi = b2 * v[i] + (1.f - b2) * gi * gi;
-    p -= step * mi / (sqrtf(vi) * rb2 + eps);
-    m[i] = mi;
-    v[i] = vi;
-    if (master) master[i] = p;
-    stf(w + i, p);
+  for (int64_t i = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) * 4; i < n;
+       i += (int64_t)gridDim.x * blockDim.x * 4) {
+    const float4 g4 = *(const float4*)(g + i);
+    float4 m4 = *(const float4*)(m + i), v4 = *(const float4*)(v + i);
+    float p[4];
+    if (master) {
+      const float4 p4 = *(const float4*)(master + i);
+      p[0] = p4.x; p[1] = p4.y; p[2] = p4.z; p[3] = p4.w;
+    } else {
+#pragma unroll
+      for (int k = 0; k < 4; ++k) p[k] = ldf(w + i + k);
+    }
+    float gg[4] = {g4.x * gs, g4.y * gs, g4.z * gs, g4.w * gs};
+    float mm[4] = {m4.x, m4.y, m4.z, m4.w}, vv[4] = {v4.x, v4.y, v4.z, v4.w};
+#pragma unroll
+    for (int k = 0; k < 4; ++k) {
+      p[k] *= decay;
+      mm[k] = b1 * mm[k] + (1.f - b1) * gg[k];
+      vv[k] = b2 * vv[k] + (1.f - b2) * gg[k] * gg[k];
+      p[k] -= step * mm[k] / (sqrtf(vv[k]) * rb2 + eps);
+    }
+    *(float4*)(m + i) = make_float4(mm[0], mm[1], mm[2], mm[3]);
+    *(float4*)(v + i) = make_float4(vv[0], vv[1], vv[2], vv[3]);
+    if (master) *(float4*)(master + i) = make_float4(p[0], p[1], p[2], p[3]);
+#pragma unroll
+    for (int k = 0; k < 4; ++k) stf(w + i + k, p[k]);
   }
 }
 

@@ -27,10 +27,22 @@ def operands(M, N, K, a_mn, b_mn, seed=0):
     return A, B, As, Bs, a_sm, a_sk, b_sn, b_sk
 
 
+SHAPES += [(2048, 3072, 768), (512, 768, 3072), (4096, 2304, 768)]   # BN=256 persistent tiles
+
+
+@pytest.fixture(params=[1, 0], ids=["persistent", "tile-per-cta"])
+def gemm_mode(request):
+    mb().debug_options(gemm_mode=request.param)
+    yield request.param
+    mb().debug_options(gemm_mode=1)
+
+
 @pytest.mark.parametrize("use_tc", [True, False])
 @pytest.mark.parametrize("a_mn,b_mn", [(0, 0), (0, 1), (1, 1)])
 @pytest.mark.parametrize("shape", SHAPES)
-def test_gemm_f32_out(shape, a_mn, b_mn, use_tc):
+def test_gemm_f32_out(shape, a_mn, b_mn, use_tc, gemm_mode):
+    if not use_tc and gemm_mode == 0:
+        pytest.skip("SIMT path does not depend on the tcgen05 mode")
     M, N, K = shape
     A, B, As, Bs, a_sm, a_sk, b_sn, b_sk = operands(M, N, K, a_mn, b_mn)
     C = torch.full((M, N), float("nan"), device="cuda")
@@ -41,8 +53,8 @@ def test_gemm_f32_out(shape, a_mn, b_mn, use_tc):
     assert err < 1e-5, err
 
 
-@pytest.mark.parametrize("shape", [(300, 200, 136), (2048, 768, 768)])
-def test_gemm_bias_bf16_out(shape):
+@pytest.mark.parametrize("shape", [(300, 200, 136), (2048, 768, 768), (2048, 3072, 768)])
+def test_gemm_bias_bf16_out(shape, gemm_mode):
     M, N, K = shape
     A, B, As, Bs, a_sm, a_sk, b_sn, b_sk = operands(M, N, K, 0, 0, seed=1)
     bias = torch.randn(N, device="cuda").bfloat16()
@@ -55,7 +67,7 @@ def test_gemm_bias_bf16_out(shape):
 
 
 @pytest.mark.parametrize("split", [2, 3, 4])
-def test_gemm_split_k(split):
+def test_gemm_split_k(split, gemm_mode):
     M, N, K = 768, 768, 1000            # wgrad-like: TN, K = tokens
     A, B, As, Bs, a_sm, a_sk, b_sn, b_sk = operands(M, N, K, 1, 1, seed=2)
     C = torch.zeros(split, M, N, device="cuda")
