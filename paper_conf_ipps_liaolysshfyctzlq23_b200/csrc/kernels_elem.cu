@@ -230,8 +230,15 @@ __global__ void __launch_bounds__(256) k_reduce_rows(RedJobs jobs, int rows, int
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const int c = blockIdx.x * 32 + lane;
   float acc = 0.f;
-  if (c < n)
-    for (int p = warp; p < rows; p += 8) acc += jb.part[(int64_t)p * ld + c];
+  if (c < n) {
+    int p = warp;
+    for (; p + 24 < rows; p += 32) {      // 4 independent loads in flight, added in row order
+      const float v0 = jb.part[(int64_t)p * ld + c], v1 = jb.part[(int64_t)(p + 8) * ld + c];
+      const float v2 = jb.part[(int64_t)(p + 16) * ld + c], v3 = jb.part[(int64_t)(p + 24) * ld + c];
+      acc += v0; acc += v1; acc += v2; acc += v3;
+    }
+    for (; p < rows; p += 8) acc += jb.part[(int64_t)p * ld + c];
+  }
   sw[warp][lane] = acc;
   __syncthreads();
   if (warp == 0 && c < n) {
@@ -502,8 +509,12 @@ __global__ void __launch_bounds__(256) k_segment_sum(const int32_t* __restrict__
   if (r >= T) return;
   const int key = keys[r];
   if (r > 0 && keys[r - 1] == key) return;
-  int end = r + 1;
-  while (end < T && keys[end] == key) ++end;
+  int end = T;                                        // warp-parallel search for the run end
+  for (int base = r + 1; base < T; base += 32) {
+    const int i = base + lane;
+    const unsigned diff = __ballot_sync(0xffffffffu, i < T && keys[i] != key);
+    if (diff) { end = base + __ffs(diff) - 1; break; }
+  }
   for (int c = lane; c < H; c += 32) {
     float acc = X[(int64_t)tok[r] * H + c];
     for (int q = (r / 32 + 1) * 32; q < end; q += 32) acc += X[(int64_t)tok[q] * H + c];

@@ -200,7 +200,9 @@ __global__ void __launch_bounds__(TC_THREADS, 2)
         if (n + 32 <= g.N) {
           epi_row32<EPI>(g, m, n, v);
         } else {
-          for (int i = 0; i < 32 && n + i < g.N; ++i) epilogue<__nv_bfloat16, EPI>(g, m, n + i, v[i]);
+#pragma unroll
+          for (int i = 0; i < 32; ++i)
+            if (n + i < g.N) epilogue<__nv_bfloat16, EPI>(g, m, n + i, v[i]);
         }
       }
     }
@@ -340,10 +342,21 @@ __global__ void __launch_bounds__(TP_THREADS, 1)
       const int m0 = (r / args.n_blocks) * TBM, n0 = (r % args.n_blocks) * BN;
       const int kb0 = z * ta.kb_per_split, kb1 = min(ta.kb_total, kb0 + ta.kb_per_split);
       const int acc = local & 1;
+      const int m = m0 + 32 * q + lane;
+      {  // pull this tile's epilogue inputs into L2 while the MMAs run
+        const int nb = n0 + half * (BN / 2);
+        if (m < g.M && nb < g.N) {
+          const char* pa = nullptr;
+          int bytes = 0;
+          if constexpr (EPI == EPI_GELU_BWD) { pa = (const char*)((const __nv_bfloat16*)g.aux + (int64_t)m * g.ldx + nb); bytes = BN; }
+          if constexpr (EPI == EPI_BIAS_DROP_RES) { pa = (const char*)((const __nv_bfloat16*)g.res + (int64_t)m * g.ldr + nb); bytes = BN; }
+          if constexpr (EPI == EPI_ACC_RES_F32) { pa = (const char*)((const float*)g.res + (int64_t)m * g.ldr + nb); bytes = 2 * BN; }
+          for (int o = 0; o < bytes; o += 128) asm volatile("prefetch.global.L2 [%0];" ::"l"(pa + o));
+        }
+      }
       mbar_wait(&tfull[acc], (local >> 1) & 1);
       __syncwarp();
       tc_fence_after();
-      const int m = m0 + 32 * q + lane;
 #pragma unroll 1
       for (int c = half * (BN / 64); c < (half + 1) * (BN / 64); ++c) {
         float v[32];
@@ -357,7 +370,9 @@ __global__ void __launch_bounds__(TP_THREADS, 1)
           if (n + 32 <= g.N) {
             epi_row32<EPI>(g, m, n, v, z);
           } else {
-            for (int i = 0; i < 32 && n + i < g.N; ++i) epilogue<__nv_bfloat16, EPI>(g, m, n + i, v[i], z);
+  #pragma unroll
+          for (int i = 0; i < 32; ++i)
+            if (n + i < g.N) epilogue<__nv_bfloat16, EPI>(g, m, n + i, v[i], z);
           }
         }
       }
