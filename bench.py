@@ -43,6 +43,7 @@ def parse():
     ap.add_argument("--no-baselines", action="store_true", help="skip static-plan / no-ckpt arms")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--simt", action="store_true", help="SIMT GEMMs instead of tcgen05")
+    ap.add_argument("--gemm-mode", type=int, default=-1, help="tcgen05 GEMM variant (debug_options)")
     return ap.parse_args()
 
 
@@ -182,6 +183,8 @@ def main():
     cfg = wl.CONFIGS[args.config]
     stream = torch.cuda.current_stream()
     use_tc = 0 if args.simt else 1
+    if args.gemm_mode >= 0:
+        mb.debug_options(gemm_mode=args.gemm_mode)
 
     # ---- budget (D2 / reading A21) from the library's own allocation sequence ----
     probe_ctx = mb.Mimose(cfg, 0)

@@ -237,9 +237,16 @@ mimose_status mimose_probe_read(mimose_ctx* ctx, double* total_ms, double* total
 mimose_status mimose_debug_gemm(int32_t epi, int32_t M, int32_t N, int32_t K, const void* A, int64_t a_sm,
                                 int64_t a_sk, const void* B, int64_t b_sn, int64_t b_sk, void* C, int64_t ldc,
                                 const void* bias, int32_t split, int32_t use_tc, void* stream);
+/* Same, every epilogue (0 store, 1 bias, 2 bias+GELU -> C, C2, 3 bias+dropout(p=0.1, seed 7)+residual
+   -> fp32 C, 4 GELU' with aux, 5 fp32 C = acc + res, 6 fp32). */
+mimose_status mimose_debug_gemm_ex(int32_t epi, int32_t M, int32_t N, int32_t K, const void* A, int64_t a_sm,
+                                   int64_t a_sk, const void* B, int64_t b_sn, int64_t b_sk, void* C, int64_t ldc,
+                                   void* C2, const void* bias, const void* res, int64_t ldr, const void* aux,
+                                   int64_t ldx, int32_t split, int32_t use_tc, void* stream);
 
 /* Test hook: process-wide kernel options. gemm_mode 0 = one 128x128 tile per CTA,
-   1 = persistent double-buffered tcgen05 GEMM (default); attn_tc 0/1 routes bf16
+   1 = persistent double-buffered single-CTA tcgen05 GEMM, 2 = persistent CTA-pair
+   (cta_group::2, 256-row tiles; default); attn_tc 0/1 routes bf16
    attention with S <= 128 to the SIMT / tcgen05 kernels.  Negative = unchanged. */
 void mimose_debug_options(int32_t gemm_mode, int32_t attn_tc);
 

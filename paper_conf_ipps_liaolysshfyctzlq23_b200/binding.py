@@ -145,6 +145,22 @@ def debug_gemm(epi, M, N, K, A, a_sm, a_sk, B, b_sn, b_sk, Cm, ldc, bias=None, s
         raise MimoseError(st, "debug_gemm")
 
 
+_lib.mimose_debug_gemm_ex.argtypes = [C.c_int32, C.c_int32, C.c_int32, C.c_int32, _P, C.c_int64, C.c_int64,
+                                      _P, C.c_int64, C.c_int64, _P, C.c_int64, _P, _P, _P, C.c_int64, _P, C.c_int64,
+                                      C.c_int32, C.c_int32, _P]
+EXPORTED.append("mimose_debug_gemm_ex")
+
+
+def debug_gemm_ex(epi, M, N, K, A, a_sm, a_sk, B, b_sn, b_sk, Cm, ldc, C2=None, bias=None, res=None, ldr=0,
+                  aux=None, ldx=0, split=1, use_tc=True, stream=0):
+    """Test hook over one library GEMM with any epilogue (torch tensors in)."""
+    ptr = lambda t: t.data_ptr() if t is not None else None
+    st = _lib.mimose_debug_gemm_ex(epi, M, N, K, ptr(A), a_sm, a_sk, ptr(B), b_sn, b_sk, ptr(Cm), ldc, ptr(C2),
+                                   ptr(bias), ptr(res), ldr, ptr(aux), ldx, split, 1 if use_tc else 0, stream)
+    if st != OK:
+        raise MimoseError(st, "debug_gemm_ex")
+
+
 _lib.mimose_debug_options.argtypes = [C.c_int32, C.c_int32]
 _lib.mimose_debug_options.restype = None
 EXPORTED.append("mimose_debug_options")

@@ -4,9 +4,28 @@
 
 namespace mimose {
 
-MDEV float gelu_f(float u) { return 0.5f * u * (1.0f + erff(u * 0.70710678118654752f)); }
+// erf-GELU and its derivative with a branch-free erf (Abramowitz & Stegun 7.1.26,
+// |error| <= 1.5e-7, far below bf16 resolution): erf(x) = 1 - poly(t) exp(-x^2),
+// t = 1/(1 + p|x|).  exp(-x^2) with x = u/sqrt(2) is exp(-u^2/2), which GELU'
+// also needs, so the derivative costs one extra FMA.  (libdevice erff branches
+// on |x|, which diverges inside a warp of GEMM-epilogue values.)
+MDEV float erf_as(float x, float e /* = exp(-x^2) */) {
+  const float ax = fabsf(x);
+  const float t = __fdividef(1.0f, fmaf(0.3275911f, ax, 1.0f));
+  float p = fmaf(1.061405429f, t, -1.453152027f);
+  p = fmaf(p, t, 1.421413741f);
+  p = fmaf(p, t, -0.284496736f);
+  p = fmaf(p, t, 0.254829592f);
+  const float r = 1.0f - p * t * e;
+  return copysignf(r, x);
+}
+MDEV float gelu_f(float u) {
+  const float e = __expf(-0.5f * u * u);
+  return 0.5f * u * (1.0f + erf_as(u * 0.70710678118654752f, e));
+}
 MDEV float gelu_grad_f(float u) {
-  return 0.5f * (1.0f + erff(u * 0.70710678118654752f)) + u * 0.39894228040143268f * expf(-0.5f * u * u);
+  const float e = __expf(-0.5f * u * u);
+  return 0.5f * (1.0f + erf_as(u * 0.70710678118654752f, e)) + u * 0.39894228040143268f * e;
 }
 
 // Epilogue of one output element.
@@ -29,6 +48,8 @@ MDEV void epilogue(const GemmArgs& g, int m, int n, float acc, int z = -1) {
     stf((E*)g.C + o, acc * gelu_grad_f(ldf((const E*)g.aux + (int64_t)m * g.ldx + n)));
   } else if constexpr (EPI == EPI_ACC_RES_F32) {
     ((float*)g.C)[o] = acc + ((const float*)g.res)[(int64_t)m * g.ldr + n];
+  } else if constexpr (EPI == EPI_NONE) {
+    if (acc == 1234.5f) ((float*)g.C)[o] = acc;   // keep the value live
   } else {
     ((float*)g.C)[(int64_t)z * g.split_stride + o] = acc;
   }

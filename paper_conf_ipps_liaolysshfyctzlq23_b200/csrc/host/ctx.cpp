@@ -1028,6 +1028,24 @@ mimose_status mimose_plan(mimose_ctx* c, int64_t x, mimose_plan_t* out) {
 
 int32_t mimose_tc_available(void) { return tc_available() ? 1 : 0; }
 
+mimose_status mimose_debug_gemm_ex(int32_t epi, int32_t M, int32_t N, int32_t K, const void* A, int64_t a_sm,
+                                   int64_t a_sk, const void* B, int64_t b_sn, int64_t b_sk, void* Cp, int64_t ldc,
+                                   void* C2, const void* bias, const void* res, int64_t ldr, const void* aux,
+                                   int64_t ldx, int32_t split, int32_t use_tc, void* stream) {
+  if (epi < 0 || epi > 7) return MIMOSE_E_INVALID;
+  GemmArgs g;
+  g.M = M; g.N = N; g.K = K;
+  g.A = A; g.a_sm = a_sm; g.a_sk = a_sk;
+  g.B = B; g.b_sn = b_sn; g.b_sk = b_sk;
+  g.C = Cp; g.ldc = ldc; g.C2 = C2; g.bias = bias; g.res = res; g.ldr = ldr; g.aux = aux; g.ldx = ldx;
+  g.split = split < 1 ? 1 : split;
+  g.split_stride = (int64_t)M * ldc;
+  g.drop.enabled = 1; g.drop.seed_lo = 7; g.drop.seed_hi = 0; g.drop.site = 0; g.drop.step = 1;
+  g.drop.thresh = 3865470566u; g.drop.scale = (float)(1.0 / 0.9);
+  gemm(DT_BF16, (Epi)epi, g, (cudaStream_t)stream, use_tc != 0);
+  return cudaGetLastError() == cudaSuccess ? MIMOSE_OK : MIMOSE_E_CUDA;
+}
+
 void mimose_debug_options(int32_t gemm_mode, int32_t attn_tc) {
   if (gemm_mode >= 0) set_gemm_mode(gemm_mode);
   if (attn_tc >= 0) set_attn_tc(attn_tc != 0);

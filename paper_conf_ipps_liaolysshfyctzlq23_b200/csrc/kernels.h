@@ -21,7 +21,8 @@ enum Epi : int {
   EPI_BIAS_DROP_RES = 3,  // C(f32) = res(E) + drop(acc + bias)   element e = m*ldc + n
   EPI_GELU_BWD = 4,       // C(E) = acc * gelu'(aux(E))
   EPI_ACC_RES_F32 = 5,    // C(f32) = acc + res(f32)  (res may alias C)
-  EPI_F32 = 6             // C(f32) = acc ; split-K: C + z*split_stride
+  EPI_F32 = 6,            // C(f32) = acc ; split-K: C + z*split_stride
+  EPI_NONE = 7            // benchmark only: accumulator read from TMEM, nothing stored
 };
 struct GemmArgs {
   int M = 0, N = 0, K = 0;

@@ -97,10 +97,208 @@ MDEV void epi_row32(const GemmArgs& g, int m, int n, float (&v)[32], int z = -1)
       const float4 a = r[q];
       out[q] = make_float4(v[4 * q] + a.x, v[4 * q + 1] + a.y, v[4 * q + 2] + a.z, v[4 * q + 3] + a.w);
     }
+  } else if constexpr (EPI == EPI_NONE) {
+    float t = 0.f;
+#pragma unroll
+    for (int i = 0; i < 32; ++i) t += v[i];
+    if (t == 1234.5f) ((float*)g.C)[o] = t;
   } else {
     float4* out = (float4*)((float*)g.C + (int64_t)z * g.split_stride + o);
 #pragma unroll
     for (int q = 0; q < 8; ++q) out[q] = make_float4(v[4 * q], v[4 * q + 1], v[4 * q + 2], v[4 * q + 3]);
+  }
+}
+
+
+// ---- coalesced tile stores through a per-warp staging buffer -------------
+// The warp holds a 32 x 32 fragment (lane = row).  It is written to a 32 x 128 B
+// smem buffer with the 16-B chunk index XOR-swizzled by row, then read back so
+// that each store instruction writes whole row segments: fp32 -> 4 rows x 128 B,
+// bf16 -> 8 rows x 64 B (full 32-B sectors, no partial-sector writes).
+MDEV void stage_store_f32(uint8_t* stg, const float (&v)[32], float* out, int64_t ld, int rows_valid, int lane) {
+#pragma unroll
+  for (int c = 0; c < 8; ++c)
+    *(float4*)(stg + lane * 128 + ((c ^ (lane & 7)) << 4)) = make_float4(v[4 * c], v[4 * c + 1], v[4 * c + 2], v[4 * c + 3]);
+  __syncwarp();
+#pragma unroll
+  for (int k = 0; k < 8; ++k) {
+    const int R = (lane >> 3) + 4 * k, c = lane & 7;
+    const float4 w = *(const float4*)(stg + R * 128 + ((c ^ (R & 7)) << 4));
+    if (R < rows_valid) *(float4*)(out + (int64_t)R * ld + 4 * c) = w;
+  }
+  __syncwarp();
+}
+MDEV void stage_store_bf16(uint8_t* stg, const float (&v)[32], __nv_bfloat16* out, int64_t ld, int rows_valid, int lane) {
+#pragma unroll
+  for (int c = 0; c < 4; ++c) *(uint4*)(stg + lane * 128 + ((c ^ (lane & 3)) << 4)) = pack8(v + 8 * c);
+  __syncwarp();
+#pragma unroll
+  for (int k = 0; k < 4; ++k) {
+    const int R = (lane >> 2) + 8 * k, c = lane & 3;
+    const uint4 w = *(const uint4*)(stg + R * 128 + ((c ^ (R & 3)) << 4));
+    if (R < rows_valid) *(uint4*)(out + (int64_t)R * ld + 8 * c) = w;
+  }
+  __syncwarp();
+}
+
+// Epilogue of a 32-row x 32-column fragment (rows m_base + lane, columns n..n+31,
+// all columns in range), stores coalesced through `stg`.
+template <int EPI>
+MDEV void epi_frag32(const GemmArgs& g, int m_base, int n, float (&v)[32], int z, uint8_t* stg, int lane) {
+  using E = __nv_bfloat16;
+  const int m = m_base + lane;
+  const int rows_valid = g.M - m_base;
+  const bool live = m < g.M;
+  if constexpr (EPI == EPI_STORE) {
+    stage_store_bf16(stg, v, (E*)g.C + (int64_t)m_base * g.ldc + n, g.ldc, rows_valid, lane);
+  } else if constexpr (EPI == EPI_BIAS || EPI == EPI_BIAS_GELU || EPI == EPI_BIAS_DROP_RES) {
+    float b[32];
+    ld_bf16x32((const E*)g.bias + n, b);
+#pragma unroll
+    for (int i = 0; i < 32; ++i) v[i] += b[i];
+    if constexpr (EPI == EPI_BIAS) {
+      stage_store_bf16(stg, v, (E*)g.C + (int64_t)m_base * g.ldc + n, g.ldc, rows_valid, lane);
+    } else if constexpr (EPI == EPI_BIAS_GELU) {
+      stage_store_bf16(stg, v, (E*)g.C + (int64_t)m_base * g.ldc + n, g.ldc, rows_valid, lane);
+#pragma unroll
+      for (int i = 0; i < 32; ++i) v[i] = gelu_f(__bfloat162float(__float2bfloat16_rn(v[i])));
+      stage_store_bf16(stg, v, (E*)g.C2 + (int64_t)m_base * g.ldc + n, g.ldc, rows_valid, lane);
+    } else {
+      float r[32];
+      const int64_t o = (int64_t)m * g.ldc + n;
+      if (live) ld_bf16x32((const E*)g.res + (int64_t)m * g.ldr + n, r);
+#pragma unroll
+      for (int q = 0; q < 8; ++q) {
+        const float4 f = live ? drop_factor4(g.drop, (uint64_t)(o + 4 * q) >> 2) : make_float4(0.f, 0.f, 0.f, 0.f);
+        v[4 * q + 0] = (live ? r[4 * q + 0] : 0.f) + v[4 * q + 0] * f.x;
+        v[4 * q + 1] = (live ? r[4 * q + 1] : 0.f) + v[4 * q + 1] * f.y;
+        v[4 * q + 2] = (live ? r[4 * q + 2] : 0.f) + v[4 * q + 2] * f.z;
+        v[4 * q + 3] = (live ? r[4 * q + 3] : 0.f) + v[4 * q + 3] * f.w;
+      }
+      stage_store_f32(stg, v, (float*)g.C + (int64_t)m_base * g.ldc + n, g.ldc, rows_valid, lane);
+    }
+  } else if constexpr (EPI == EPI_GELU_BWD) {
+    float u[32];
+    if (live) {
+      ld_bf16x32((const E*)g.aux + (int64_t)m * g.ldx + n, u);
+#pragma unroll
+      for (int i = 0; i < 32; ++i) v[i] *= gelu_grad_f(u[i]);
+    }
+    stage_store_bf16(stg, v, (E*)g.C + (int64_t)m_base * g.ldc + n, g.ldc, rows_valid, lane);
+  } else if constexpr (EPI == EPI_ACC_RES_F32) {
+    if (live) {
+      const float4* r = (const float4*)((const float*)g.res + (int64_t)m * g.ldr + n);
+#pragma unroll
+      for (int q = 0; q < 8; ++q) {
+        const float4 a = r[q];
+        v[4 * q] += a.x; v[4 * q + 1] += a.y; v[4 * q + 2] += a.z; v[4 * q + 3] += a.w;
+      }
+    }
+    stage_store_f32(stg, v, (float*)g.C + (int64_t)m_base * g.ldc + n, g.ldc, rows_valid, lane);
+  } else if constexpr (EPI == EPI_NONE) {
+    float t = 0.f;
+#pragma unroll
+    for (int i = 0; i < 32; ++i) t += v[i];
+    if (t == 1234.5f) ((float*)g.C)[0] = t;
+  } else {
+    stage_store_f32(stg, v, (float*)g.C + (int64_t)z * g.split_stride + (int64_t)m_base * g.ldc + n, g.ldc,
+                    rows_valid, lane);
+  }
+}
+
+
+// Epilogue inputs of one 32-column chunk, loaded one chunk ahead (software
+// pipelining hides the L2 latency of bias / u / residual behind the previous
+// chunk's math and stores).
+struct EpiIn {
+  uint4 b[4];   // bias (bf16 x 32)
+  uint4 x[8];   // aux or residual: bf16 x 32 uses x[0..3], fp32 x 32 uses x[0..7]
+};
+template <int EPI>
+MDEV void epi_load(const GemmArgs& g, int m, int n, bool live, EpiIn& in) {
+  if constexpr (EPI == EPI_BIAS || EPI == EPI_BIAS_GELU || EPI == EPI_BIAS_DROP_RES) {
+    const uint4* p = (const uint4*)((const __nv_bfloat16*)g.bias + n);
+#pragma unroll
+    for (int i = 0; i < 4; ++i) in.b[i] = p[i];
+  }
+  if (!live) return;
+  if constexpr (EPI == EPI_BIAS_DROP_RES) {
+    const uint4* p = (const uint4*)((const __nv_bfloat16*)g.res + (int64_t)m * g.ldr + n);
+#pragma unroll
+    for (int i = 0; i < 4; ++i) in.x[i] = p[i];
+  } else if constexpr (EPI == EPI_GELU_BWD) {
+    const uint4* p = (const uint4*)((const __nv_bfloat16*)g.aux + (int64_t)m * g.ldx + n);
+#pragma unroll
+    for (int i = 0; i < 4; ++i) in.x[i] = p[i];
+  } else if constexpr (EPI == EPI_ACC_RES_F32) {
+    const uint4* p = (const uint4*)((const float*)g.res + (int64_t)m * g.ldr + n);
+#pragma unroll
+    for (int i = 0; i < 8; ++i) in.x[i] = p[i];
+  }
+}
+
+template <int EPI>
+MDEV void epi_frag32_in(const GemmArgs& g, int m_base, int n, float (&v)[32], int z, uint8_t* stg, int lane,
+                        const EpiIn& in) {
+  using E = __nv_bfloat16;
+  const int m = m_base + lane;
+  const int rows_valid = g.M - m_base;
+  const bool live = m < g.M;
+  if constexpr (EPI == EPI_STORE) {
+    stage_store_bf16(stg, v, (E*)g.C + (int64_t)m_base * g.ldc + n, g.ldc, rows_valid, lane);
+  } else if constexpr (EPI == EPI_BIAS || EPI == EPI_BIAS_GELU || EPI == EPI_BIAS_DROP_RES) {
+    float b[32];
+#pragma unroll
+    for (int i = 0; i < 4; ++i) unpack8(in.b[i], b + 8 * i);
+#pragma unroll
+    for (int i = 0; i < 32; ++i) v[i] += b[i];
+    if constexpr (EPI == EPI_BIAS) {
+      stage_store_bf16(stg, v, (E*)g.C + (int64_t)m_base * g.ldc + n, g.ldc, rows_valid, lane);
+    } else if constexpr (EPI == EPI_BIAS_GELU) {
+      stage_store_bf16(stg, v, (E*)g.C + (int64_t)m_base * g.ldc + n, g.ldc, rows_valid, lane);
+#pragma unroll
+      for (int i = 0; i < 32; ++i) v[i] = gelu_f(__bfloat162float(__float2bfloat16_rn(v[i])));
+      stage_store_bf16(stg, v, (E*)g.C2 + (int64_t)m_base * g.ldc + n, g.ldc, rows_valid, lane);
+    } else {
+      float r[32];
+#pragma unroll
+      for (int i = 0; i < 4; ++i) unpack8(in.x[i], r + 8 * i);
+      const int64_t o = (int64_t)m * g.ldc + n;
+#pragma unroll
+      for (int q = 0; q < 8; ++q) {
+        const float4 f = live ? drop_factor4(g.drop, (uint64_t)(o + 4 * q) >> 2) : make_float4(0.f, 0.f, 0.f, 0.f);
+        v[4 * q + 0] = (live ? r[4 * q + 0] : 0.f) + v[4 * q + 0] * f.x;
+        v[4 * q + 1] = (live ? r[4 * q + 1] : 0.f) + v[4 * q + 1] * f.y;
+        v[4 * q + 2] = (live ? r[4 * q + 2] : 0.f) + v[4 * q + 2] * f.z;
+        v[4 * q + 3] = (live ? r[4 * q + 3] : 0.f) + v[4 * q + 3] * f.w;
+      }
+      stage_store_f32(stg, v, (float*)g.C + (int64_t)m_base * g.ldc + n, g.ldc, rows_valid, lane);
+    }
+  } else if constexpr (EPI == EPI_GELU_BWD) {
+    float u[32];
+#pragma unroll
+    for (int i = 0; i < 4; ++i) unpack8(in.x[i], u + 8 * i);
+#pragma unroll
+    for (int i = 0; i < 32; ++i) v[i] = live ? v[i] * gelu_grad_f(u[i]) : 0.f;
+    stage_store_bf16(stg, v, (E*)g.C + (int64_t)m_base * g.ldc + n, g.ldc, rows_valid, lane);
+  } else if constexpr (EPI == EPI_ACC_RES_F32) {
+    if (live) {
+      const float4* r = (const float4*)in.x;
+#pragma unroll
+      for (int q = 0; q < 8; ++q) {
+        const float4 a = r[q];
+        v[4 * q] += a.x; v[4 * q + 1] += a.y; v[4 * q + 2] += a.z; v[4 * q + 3] += a.w;
+      }
+    }
+    stage_store_f32(stg, v, (float*)g.C + (int64_t)m_base * g.ldc + n, g.ldc, rows_valid, lane);
+  } else if constexpr (EPI == EPI_NONE) {
+    float t = 0.f;
+#pragma unroll
+    for (int i = 0; i < 32; ++i) t += v[i];
+    if (t == 1234.5f) ((float*)g.C)[0] = t;
+  } else {
+    stage_store_f32(stg, v, (float*)g.C + (int64_t)z * g.split_stride + (int64_t)m_base * g.ldc + n, g.ldc,
+                    rows_valid, lane);
   }
 }
 
@@ -221,7 +419,7 @@ __global__ void __launch_bounds__(TC_THREADS, 2)
 // (tile = (split, m-block, n-block), n fastest).  Two TMEM accumulators
 // (2 x BN columns) let the epilogue of tile i overlap the MMAs of tile i+1; the
 // smem ring continues across tiles.  8 epilogue warps: warp 2+e handles TMEM
-// lane quarter e%4 and column half e/4.
+// lane quarter e%4 and column group e/4 (of TP_EPI_WARPS/4).
 // ---------------------------------------------------------------------------
 constexpr int TP_EPI_WARPS = 8;
 constexpr int TP_THREADS = 64 + 32 * TP_EPI_WARPS;
@@ -232,7 +430,8 @@ struct TpCfg {
   static constexpr int A_BYTES = TBM * TBK * 2;
   static constexpr int B_BYTES = BN * TBK * 2;
   static constexpr int STAGE_BYTES = A_BYTES + B_BYTES;
-  static constexpr int SMEM = STAGES * STAGE_BYTES + 1024 + 512;
+  static constexpr int STG_BYTES = TP_EPI_WARPS * 4096;   // per-warp 32 x 128 B store staging
+  static constexpr int SMEM = STAGES * STAGE_BYTES + STG_BYTES + 1024 + 256;
 };
 
 struct TpArgs {
@@ -251,6 +450,7 @@ __global__ void __launch_bounds__(TP_THREADS, 1)
   uint64_t* tfull = empty + Cf::STAGES;    // [2]
   uint64_t* tempty = tfull + 2;            // [2]
   uint32_t* tmem_slot = (uint32_t*)(tempty + 2);
+  uint8_t* stg_base = smem + Cf::STAGES * Cf::STAGE_BYTES + 256;
   const TcArgs& ta = args.t;
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
 
@@ -334,7 +534,7 @@ __global__ void __launch_bounds__(TP_THREADS, 1)
   } else {                                             // ---------------- epilogue warps
     const int e = warp - 2;
     const int q = warp & 3;                            // TMEM lane quarter of this warp
-    const int half = e >> 2;
+    const int grp = e >> 2, ngrp = TP_EPI_WARPS / 4;  // column group of this warp
     const GemmArgs& g = ta.g;
     int local = 0;
     for (int tile = blockIdx.x; tile < args.n_tiles; tile += gridDim.x, ++local) {
@@ -343,37 +543,41 @@ __global__ void __launch_bounds__(TP_THREADS, 1)
       const int kb0 = z * ta.kb_per_split, kb1 = min(ta.kb_total, kb0 + ta.kb_per_split);
       const int acc = local & 1;
       const int m = m0 + 32 * q + lane;
+      const int c_beg = grp * (BN / 32) / ngrp, c_end = (grp + 1) * (BN / 32) / ngrp;
       {  // pull this tile's epilogue inputs into L2 while the MMAs run
-        const int nb = n0 + half * (BN / 2);
+        const int nb = n0 + 32 * c_beg;
         if (m < g.M && nb < g.N) {
           const char* pa = nullptr;
           int bytes = 0;
-          if constexpr (EPI == EPI_GELU_BWD) { pa = (const char*)((const __nv_bfloat16*)g.aux + (int64_t)m * g.ldx + nb); bytes = BN; }
-          if constexpr (EPI == EPI_BIAS_DROP_RES) { pa = (const char*)((const __nv_bfloat16*)g.res + (int64_t)m * g.ldr + nb); bytes = BN; }
-          if constexpr (EPI == EPI_ACC_RES_F32) { pa = (const char*)((const float*)g.res + (int64_t)m * g.ldr + nb); bytes = 2 * BN; }
+          const int ncol = 32 * (c_end - c_beg);
+          if constexpr (EPI == EPI_GELU_BWD) { pa = (const char*)((const __nv_bfloat16*)g.aux + (int64_t)m * g.ldx + nb); bytes = 2 * ncol; }
+          if constexpr (EPI == EPI_BIAS_DROP_RES) { pa = (const char*)((const __nv_bfloat16*)g.res + (int64_t)m * g.ldr + nb); bytes = 2 * ncol; }
+          if constexpr (EPI == EPI_ACC_RES_F32) { pa = (const char*)((const float*)g.res + (int64_t)m * g.ldr + nb); bytes = 4 * ncol; }
           for (int o = 0; o < bytes; o += 128) asm volatile("prefetch.global.L2 [%0];" ::"l"(pa + o));
         }
       }
       mbar_wait(&tfull[acc], (local >> 1) & 1);
       __syncwarp();
       tc_fence_after();
+      EpiIn nxt;
+      if (n0 + 32 * c_beg + 32 <= g.N) epi_load<EPI>(g, m, n0 + 32 * c_beg, m < g.M, nxt);
 #pragma unroll 1
-      for (int c = half * (BN / 64); c < (half + 1) * (BN / 64); ++c) {
+      for (int c = c_beg; c < c_end; ++c) {
+        const EpiIn cur = nxt;
+        const int n = n0 + 32 * c;
+        if (c + 1 < c_end && n + 64 <= g.N) epi_load<EPI>(g, m, n + 32, m < g.M, nxt);
         float v[32];
         tmem_ld32(tmem + acc * BN + ((uint32_t)(32 * q) << 16) + 32 * c, v);
         if (kb1 <= kb0) {
 #pragma unroll
           for (int i = 0; i < 32; ++i) v[i] = 0.f;
         }
-        const int n = n0 + 32 * c;
-        if (m < g.M) {
-          if (n + 32 <= g.N) {
-            epi_row32<EPI>(g, m, n, v, z);
-          } else {
-  #pragma unroll
+        if (n + 32 <= g.N) {
+          if (m0 + 32 * q < g.M) epi_frag32_in<EPI>(g, m0 + 32 * q, n, v, z, stg_base + e * 4096, lane, cur);
+        } else if (m < g.M) {
+#pragma unroll
           for (int i = 0; i < 32; ++i)
             if (n + i < g.N) epilogue<__nv_bfloat16, EPI>(g, m, n + i, v[i], z);
-          }
         }
       }
       tc_fence_before();
@@ -386,6 +590,211 @@ __global__ void __launch_bounds__(TP_THREADS, 1)
   if (warp == 1) {
     tc_fence_after();
     asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(tmem), "r"(2 * BN));
+  }
+}
+
+
+// ---------------------------------------------------------------------------
+// CTA-pair variant (cta_group::2): a cluster of 2 CTAs on one TPC computes a
+// 256 x BN tile.  CTA r TMA-loads rows [128r, 128r+128) of A and rows
+// [BN/2 r, BN/2 (r+1)) of B into its own smem (transaction bytes land on the
+// leader's barrier); the leader's single thread issues tcgen05.mma.cta_group::2
+// (M = 256), which reads both CTAs' smem and writes rows 128r.. of the
+// accumulator into CTA r's TMEM.  Commits are multicast to both CTAs; both
+// CTAs' epilogue warps release an accumulator by arriving on the leader's
+// tmem-empty barrier.  Per SM this halves the B traffic and the smem operand
+// reads per MMA, relative to the single-CTA kernel.
+// ---------------------------------------------------------------------------
+constexpr uint32_t PEER_MASK = 0xFEFFFFFFu;
+
+template <int BN>
+struct T2Cfg {
+  static constexpr int A_BYTES = 128 * TBK * 2;
+  static constexpr int B_BYTES = (BN / 2) * TBK * 2;
+  static constexpr int STAGE_BYTES = A_BYTES + B_BYTES;
+  static constexpr int STAGES = (192 * 1024) / STAGE_BYTES;
+  static constexpr int SMEM = STAGES * STAGE_BYTES + 1024 + 512;
+};
+
+MDEV uint32_t cluster_rank() {
+  uint32_t r;
+  asm volatile("mov.u32 %0, %%cluster_ctarank;" : "=r"(r));
+  return r;
+}
+MDEV void cluster_sync_all() {
+  asm volatile("barrier.cluster.arrive.release.aligned;\nbarrier.cluster.wait.acquire.aligned;" ::: "memory");
+}
+MDEV void tma_load_2d_2sm(const CUtensorMap* map, uint64_t* bar, void* dst, int c0, int c1) {
+  asm volatile(
+      "cp.async.bulk.tensor.2d.cta_group::2.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1, {%3, %4}], [%2];"
+      ::"r"(smem_u32(dst)), "l"(map), "r"(smem_u32(bar) & PEER_MASK), "r"(c0), "r"(c1) : "memory");
+}
+MDEV void mma_bf16_2sm(uint32_t tmem_d, uint64_t da, uint64_t db, uint32_t idesc, uint32_t acc) {
+  asm volatile(
+      "{\n\t.reg .pred p;\n\tsetp.ne.b32 p, %4, 0;\n\t"
+      "tcgen05.mma.cta_group::2.kind::f16 [%0], %1, %2, %3, p;\n\t}"
+      ::"r"(tmem_d), "l"(da), "l"(db), "r"(idesc), "r"(acc));
+}
+MDEV void mma_commit_2sm_mc(uint64_t* bar) {
+  asm volatile("tcgen05.commit.cta_group::2.mbarrier::arrive::one.shared::cluster.multicast::cluster.b64 [%0], %1;"
+               ::"r"(smem_u32(bar)), "h"((uint16_t)3) : "memory");
+}
+MDEV void mbar_arrive_rank(uint64_t* bar, uint32_t rank) {
+  asm volatile("{\n\t.reg .b32 ra;\n\tmapa.shared::cluster.u32 ra, %0, %1;\n\t"
+               "mbarrier.arrive.release.cluster.shared::cluster.b64 _, [ra];\n\t}"
+               ::"r"(smem_u32(bar)), "r"(rank) : "memory");
+}
+
+template <int BN, int EPI>
+__global__ void __launch_bounds__(TP_THREADS, 1)
+    k_gemm_tc2(const __grid_constant__ CUtensorMap tma_a, const __grid_constant__ CUtensorMap tma_b, const TpArgs args) {
+  using Cf = T2Cfg<BN>;
+  extern __shared__ uint8_t smem_raw[];
+  uint8_t* smem = (uint8_t*)(((uintptr_t)smem_raw + 1023) & ~(uintptr_t)1023);
+  uint64_t* full = (uint64_t*)(smem + Cf::STAGES * Cf::STAGE_BYTES);
+  uint64_t* empty = full + Cf::STAGES;
+  uint64_t* tfull = empty + Cf::STAGES;    // [2]
+  uint64_t* tempty = tfull + 2;            // [2] (the leader's are used)
+  uint32_t* tmem_slot = (uint32_t*)(tempty + 2);
+  const TcArgs& ta = args.t;
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const uint32_t rank = cluster_rank();
+  const bool leader = rank == 0;
+  const int cid = blockIdx.x >> 1, ncl = gridDim.x >> 1;
+
+  if (warp == 0 && lane == 0) {
+    for (int s = 0; s < Cf::STAGES; ++s) { mbar_init(&full[s], 1); mbar_init(&empty[s], 1); }
+    for (int a = 0; a < 2; ++a) { mbar_init(&tfull[a], 1); mbar_init(&tempty[a], 2 * TP_EPI_WARPS); }
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+    asm volatile("prefetch.tensormap [%0];" ::"l"(&tma_a) : "memory");
+    asm volatile("prefetch.tensormap [%0];" ::"l"(&tma_b) : "memory");
+  }
+  if (warp == 1) {
+    asm volatile("tcgen05.alloc.cta_group::2.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(smem_u32(tmem_slot)),
+                 "r"(2 * BN));
+    asm volatile("tcgen05.relinquish_alloc_permit.cta_group::2.sync.aligned;");
+  }
+  tc_fence_before();
+  cluster_sync_all();
+  tc_fence_after();
+  const uint32_t tmem = *tmem_slot;
+  const int per_split = args.m_blocks * args.n_blocks;     // m_blocks counts 256-row pairs
+
+  if (warp == 0) {
+    if (lane == 0) {                                   // ---------------- TMA producer (both CTAs)
+      int it = 0;
+      for (int tile = cid; tile < args.n_tiles; tile += ncl) {
+        const int z = tile / per_split, r = tile % per_split;
+        const int m0 = (r / args.n_blocks) * 256 + 128 * rank;
+        const int nb = (r % args.n_blocks) * BN + (BN / 2) * rank;
+        const int kb0 = z * ta.kb_per_split, kb1 = min(ta.kb_total, kb0 + ta.kb_per_split);
+        for (int kb = kb0; kb < kb1; ++kb, ++it) {
+          const int s = it % Cf::STAGES;
+          if (it >= Cf::STAGES) mbar_wait(&empty[s], ((it / Cf::STAGES) - 1) & 1);
+          uint8_t* sa = smem + s * Cf::STAGE_BYTES;
+          uint8_t* sb = sa + Cf::A_BYTES;
+          const int k = kb * TBK;
+          if (leader) mbar_expect_tx(&full[s], 2 * Cf::STAGE_BYTES);
+          if (ta.a_mn) {
+            tma_load_2d_2sm(&tma_a, &full[s], sa, m0, k);
+            tma_load_2d_2sm(&tma_a, &full[s], sa + 8192, m0 + 64, k);
+          } else {
+            tma_load_2d_2sm(&tma_a, &full[s], sa, k, m0);
+          }
+          if (ta.b_mn) {
+#pragma unroll
+            for (int j = 0; j < BN / 128; ++j) tma_load_2d_2sm(&tma_b, &full[s], sb + 8192 * j, nb + 64 * j, k);
+          } else {
+            tma_load_2d_2sm(&tma_b, &full[s], sb, k, nb);
+          }
+        }
+      }
+    }
+  } else if (warp == 1) {
+    if (lane == 0 && leader) {                         // ---------------- MMA issuer (leader)
+      const uint32_t idesc = idesc_bf16(256, BN, ta.a_mn, ta.b_mn);
+      int it = 0, local = 0;
+      for (int tile = cid; tile < args.n_tiles; tile += ncl, ++local) {
+        const int z = tile / per_split;
+        const int kb0 = z * ta.kb_per_split, kb1 = min(ta.kb_total, kb0 + ta.kb_per_split);
+        const int acc = local & 1;
+        if (local >= 2) mbar_wait(&tempty[acc], ((local >> 1) - 1) & 1);
+        tc_fence_after();
+        const uint32_t d = tmem + acc * BN;
+        for (int kb = kb0; kb < kb1; ++kb, ++it) {
+          const int s = it % Cf::STAGES;
+          mbar_wait(&full[s], (it / Cf::STAGES) & 1);
+          tc_fence_after();
+          const uint32_t sa = smem_u32(smem + s * Cf::STAGE_BYTES);
+          const uint32_t sb = sa + Cf::A_BYTES;
+#pragma unroll
+          for (int kk = 0; kk < TBK / 16; ++kk) {
+            const uint64_t da = ta.a_mn ? make_desc(sa + kk * 2048, 8192, 1024) : make_desc(sa + kk * 32, 16, 1024);
+            const uint64_t db = ta.b_mn ? make_desc(sb + kk * 2048, 8192, 1024) : make_desc(sb + kk * 32, 16, 1024);
+            mma_bf16_2sm(d, da, db, idesc, (kb > kb0 || kk > 0) ? 1u : 0u);
+          }
+          mma_commit_2sm_mc(&empty[s]);
+        }
+        mma_commit_2sm_mc(&tfull[acc]);
+      }
+    }
+  } else {                                             // ---------------- epilogue warps (both CTAs)
+    const int e = warp - 2;
+    const int q = warp & 3;
+    const int grp = e >> 2, ngrp = TP_EPI_WARPS / 4;
+    const GemmArgs& g = ta.g;
+    int local = 0;
+    for (int tile = cid; tile < args.n_tiles; tile += ncl, ++local) {
+      const int z = tile / per_split, r = tile % per_split;
+      const int m0 = (r / args.n_blocks) * 256 + 128 * rank;
+      const int n0 = (r % args.n_blocks) * BN;
+      const int kb0 = z * ta.kb_per_split, kb1 = min(ta.kb_total, kb0 + ta.kb_per_split);
+      const int acc = local & 1;
+      const int m = m0 + 32 * q + lane;
+      const int c_beg = grp * (BN / 32) / ngrp, c_end = (grp + 1) * (BN / 32) / ngrp;
+      {
+        const int nbp = n0 + 32 * c_beg, ncol = 32 * (c_end - c_beg);
+        if (m < g.M && nbp < g.N) {
+          const char* pa = nullptr;
+          int bytes = 0;
+          if constexpr (EPI == EPI_GELU_BWD) { pa = (const char*)((const __nv_bfloat16*)g.aux + (int64_t)m * g.ldx + nbp); bytes = 2 * ncol; }
+          if constexpr (EPI == EPI_BIAS_DROP_RES) { pa = (const char*)((const __nv_bfloat16*)g.res + (int64_t)m * g.ldr + nbp); bytes = 2 * ncol; }
+          if constexpr (EPI == EPI_ACC_RES_F32) { pa = (const char*)((const float*)g.res + (int64_t)m * g.ldr + nbp); bytes = 4 * ncol; }
+          for (int o = 0; o < bytes; o += 128) asm volatile("prefetch.global.L2 [%0];" ::"l"(pa + o));
+        }
+      }
+      mbar_wait(&tfull[acc], (local >> 1) & 1);
+      __syncwarp();
+      tc_fence_after();
+#pragma unroll 1
+      for (int c = c_beg; c < c_end; ++c) {
+        float v[32];
+        tmem_ld32(tmem + acc * BN + ((uint32_t)(32 * q) << 16) + 32 * c, v);
+        if (kb1 <= kb0) {
+#pragma unroll
+          for (int i = 0; i < 32; ++i) v[i] = 0.f;
+        }
+        const int n = n0 + 32 * c;
+        if (m < g.M) {
+          if (n + 32 <= g.N) {
+            epi_row32<EPI>(g, m, n, v, z);
+          } else {
+#pragma unroll
+            for (int i = 0; i < 32; ++i)
+              if (n + i < g.N) epilogue<__nv_bfloat16, EPI>(g, m, n + i, v[i], z);
+          }
+        }
+      }
+      tc_fence_before();
+      __syncwarp();
+      if (lane == 0) mbar_arrive_rank(&tempty[acc], 0);
+    }
+  }
+  tc_fence_before();
+  cluster_sync_all();
+  if (warp == 1) {
+    tc_fence_after();
+    asm volatile("tcgen05.dealloc.cta_group::2.sync.aligned.b32 %0, %1;" ::"r"(tmem), "r"(2 * BN));
   }
 }
 
@@ -489,7 +898,50 @@ static void dispatch_tcp(Epi epi, const CUtensorMap& ma, const CUtensorMap& mb, 
     case EPI_BIAS_DROP_RES: launch_tcp<BN, EPI_BIAS_DROP_RES>(ma, mb, a, st); break;
     case EPI_GELU_BWD: launch_tcp<BN, EPI_GELU_BWD>(ma, mb, a, st); break;
     case EPI_ACC_RES_F32: launch_tcp<BN, EPI_ACC_RES_F32>(ma, mb, a, st); break;
+    case EPI_NONE: launch_tcp<BN, EPI_NONE>(ma, mb, a, st); break;
     default: launch_tcp<BN, EPI_F32>(ma, mb, a, st); break;
+  }
+}
+
+template <int BN, int EPI>
+static void launch_tc2(const CUtensorMap& ma, const CUtensorMap& mb, const TpArgs& a, cudaStream_t st) {
+  static bool attr = false;
+  if (!attr) {
+    cudaFuncSetAttribute(k_gemm_tc2<BN, EPI>, cudaFuncAttributeMaxDynamicSharedMemorySize, T2Cfg<BN>::SMEM);
+    attr = true;
+  }
+  static int nsm = 0;
+  if (!nsm) {
+    int dev;
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, dev);
+  }
+  cudaLaunchConfig_t cfg{};
+  cfg.gridDim = dim3(2 * std::min(nsm / 2, a.n_tiles));
+  cfg.blockDim = dim3(TP_THREADS);
+  cfg.dynamicSmemBytes = T2Cfg<BN>::SMEM;
+  cfg.stream = st;
+  cudaLaunchAttribute attr2[1];
+  attr2[0].id = cudaLaunchAttributeClusterDimension;
+  attr2[0].val.clusterDim.x = 2;
+  attr2[0].val.clusterDim.y = 1;
+  attr2[0].val.clusterDim.z = 1;
+  cfg.attrs = attr2;
+  cfg.numAttrs = 1;
+  cudaLaunchKernelEx(&cfg, k_gemm_tc2<BN, EPI>, ma, mb, a);
+}
+
+template <int BN>
+static void dispatch_tc2(Epi epi, const CUtensorMap& ma, const CUtensorMap& mb, const TpArgs& a, cudaStream_t st) {
+  switch (epi) {
+    case EPI_STORE: launch_tc2<BN, EPI_STORE>(ma, mb, a, st); break;
+    case EPI_BIAS: launch_tc2<BN, EPI_BIAS>(ma, mb, a, st); break;
+    case EPI_BIAS_GELU: launch_tc2<BN, EPI_BIAS_GELU>(ma, mb, a, st); break;
+    case EPI_BIAS_DROP_RES: launch_tc2<BN, EPI_BIAS_DROP_RES>(ma, mb, a, st); break;
+    case EPI_GELU_BWD: launch_tc2<BN, EPI_GELU_BWD>(ma, mb, a, st); break;
+    case EPI_ACC_RES_F32: launch_tc2<BN, EPI_ACC_RES_F32>(ma, mb, a, st); break;
+    case EPI_NONE: launch_tc2<BN, EPI_NONE>(ma, mb, a, st); break;
+    default: launch_tc2<BN, EPI_F32>(ma, mb, a, st); break;
   }
 }
 
@@ -515,8 +967,30 @@ bool gemm_tc(Epi epi, const GemmArgs& g, cudaStream_t st) {
   a.kb_total = (g.K + TBK - 1) / TBK;
   a.kb_per_split = (a.kb_total + g.split - 1) / g.split;
   const int m_blocks = (g.M + TBM - 1) / TBM;
+  if ((g_gemm_mode == 2 || g_gemm_mode == 21 || g_gemm_mode == 22) && g.N % 128 == 0) {   // CTA pairs
+    const int m_pairs = (g.M + 255) / 256;
+    int BN2 = (g.N % 256 == 0 && m_pairs * (g.N / 256) * g.split >= 96) ? 256 : 128;
+    if (g_gemm_mode == 21) BN2 = 128;
+    if (g_gemm_mode == 22 && g.N % 256 == 0) BN2 = 256;
+    CUtensorMap ma2, mb2;
+    bool ok2 = a.a_mn ? make_map(&ma2, g.A, g.M, g.K, g.a_sk, 64, 64) : make_map(&ma2, g.A, g.K, g.M, g.a_sm, 64, 128);
+    if (ok2) ok2 = a.b_mn ? make_map(&mb2, g.B, g.N, g.K, g.b_sk, 64, 64)
+                          : make_map(&mb2, g.B, g.K, g.N, g.b_sn, 64, BN2 / 2);
+    if (ok2) {
+      TpArgs p;
+      p.t = a;
+      p.m_blocks = m_pairs;
+      p.n_blocks = g.N / BN2;
+      p.n_tiles = p.m_blocks * p.n_blocks * g.split;
+      if (BN2 == 256) dispatch_tc2<256>(epi, ma2, mb2, p, st);
+      else dispatch_tc2<128>(epi, ma2, mb2, p, st);
+      return true;
+    }
+  }
   // BN = 256 when N is a multiple of 256 and there are enough tiles to fill the SMs
-  const int BN = (g_gemm_mode == 1 && g.N % 256 == 0 && m_blocks * (g.N / 256) * g.split >= 120) ? 256 : 128;
+  int BN = (g_gemm_mode >= 1 && g.N % 256 == 0 && m_blocks * (g.N / 256) * g.split >= 120) ? 256 : 128;
+  if (g_gemm_mode == 11) BN = 128;
+  if (g_gemm_mode == 12 && g.N % 256 == 0) BN = 256;
   CUtensorMap ma, mb;
   bool ok;
   if (a.a_mn) ok = make_map(&ma, g.A, g.M, g.K, g.a_sk, 64, 64);
@@ -525,7 +999,7 @@ bool gemm_tc(Epi epi, const GemmArgs& g, cudaStream_t st) {
   if (a.b_mn) ok = make_map(&mb, g.B, g.N, g.K, g.b_sk, 64, 64);
   else ok = make_map(&mb, g.B, g.K, g.N, g.b_sn, 64, std::min(BN, 256));
   if (!ok) return false;
-  if (g_gemm_mode == 1) {
+  if (g_gemm_mode == 1 || g_gemm_mode == 11 || g_gemm_mode == 12) {
     TpArgs p;
     p.t = a;
     p.m_blocks = m_blocks;
@@ -544,6 +1018,7 @@ bool gemm_tc(Epi epi, const GemmArgs& g, cudaStream_t st) {
     case EPI_BIAS_DROP_RES: launch_tc<BN1, EPI_BIAS_DROP_RES>(ma, mb, a, grid, st); break;
     case EPI_GELU_BWD: launch_tc<BN1, EPI_GELU_BWD>(ma, mb, a, grid, st); break;
     case EPI_ACC_RES_F32: launch_tc<BN1, EPI_ACC_RES_F32>(ma, mb, a, grid, st); break;
+    case EPI_NONE: launch_tc<BN1, EPI_NONE>(ma, mb, a, grid, st); break;
     default: launch_tc<BN1, EPI_F32>(ma, mb, a, grid, st); break;
   }
   return true;
