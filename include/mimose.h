@@ -91,7 +91,9 @@ typedef struct {
   const void* nccl_id;   /* 128-byte ncclUniqueId from rank 0 (broadcast by caller);
                             NULL when world == 1                                     */
   int32_t use_tc;        /* 1: tcgen05 GEMMs in bf16 mode (default); 0: SIMT GEMMs  */
-  int32_t reserved[7];
+  int32_t pad_id;        /* padding token id: its embedding row gets no gradient (HF
+                            padding_idx semantics, reading A24); -1 = none           */
+  int32_t reserved[6];
 } mimose_config;
 
 /* Fill defaults (collect_iters 10, ratio 9/10, degree 2, p 0.1, eps 1e-12,

@@ -229,6 +229,10 @@ def embed_bwd(cfg, W, dx1, ec, masks: Masks, G):
         acc = np.zeros_like(W[name])
         np.add.at(acc, idx, dz0)
         G[name] = acc
+    # HF padding_idx semantics (reading A24): the pad token's embedding row gets
+    # no gradient.  (Its accumulated value is 0 anyway: padded rows carry zero
+    # gradient because no loss term reads them, A26.)
+    G["emb.word"][cfg.pad_id] = 0.0
 
 
 def head_fwd_bwd(cfg, W, y, batch: Batch, masks: Masks, G):

@@ -44,7 +44,7 @@ class Config(C.Structure):
                 ("max_seqs", C.c_int32), ("max_seq_len", C.c_int32),
                 ("arena_base", C.c_void_p), ("arena_bytes", C.c_int64), ("stream", C.c_void_p),
                 ("rank", C.c_int32), ("world", C.c_int32), ("nccl_id", C.c_void_p),
-                ("use_tc", C.c_int32), ("reserved", C.c_int32 * 7)]
+                ("use_tc", C.c_int32), ("pad_id", C.c_int32), ("reserved", C.c_int32 * 6)]
 
 
 class BatchS(C.Structure):
@@ -194,6 +194,7 @@ def make_config(cfg: wl.ModelConfig, **kw) -> Config:
     c.p_drop, c.ln_eps = cfg.p_drop, cfg.ln_eps
     c.seed = wl.dropout_seed(cfg)
     c.max_seqs, c.max_seq_len = cfg.n_seqs, cfg.max_seq
+    c.pad_id = cfg.pad_id
     for k, v in kw.items():
         setattr(c, k, v)
     return c

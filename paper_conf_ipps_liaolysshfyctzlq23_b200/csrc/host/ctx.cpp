@@ -610,7 +610,8 @@ mimose_status run_backward(Run& r, Sample* sample) {
     type_grad(dz0, c->tt, T, H, c->cfg.type_vocab, c->part, G(c, P_TYPE), r.st);
     const int bits = c->cfg.vocab <= 256 ? 8 : 16;
     const int64_t maxT = (int64_t)c->cfg.max_seqs * c->cfg.max_seq_len;
-    keyed_rowsum(c->ids, bits, dz0, T, H, G(c, P_WORD), work, hist, (int)((maxT + 1023) / 1024), r.st);
+    keyed_rowsum(c->ids, bits, dz0, T, H, G(c, P_WORD), work, hist, (int)((maxT + 1023) / 1024), c->cfg.pad_id,
+                 r.st);
   }
   a.tfree(r.z.emb_scr);
   if (sample) sample->Te = a.top_phase_peak;
@@ -700,6 +701,7 @@ void mimose_default_config(mimose_config* cfg) {
   cfg->degree = 2;
   cfg->world = 1;
   cfg->use_tc = 1;
+  cfg->pad_id = -1;
 }
 
 const char* mimose_status_str(mimose_status s) {

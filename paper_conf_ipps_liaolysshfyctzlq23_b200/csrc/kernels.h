@@ -78,10 +78,11 @@ void embed_fwd(DType dt, const int32_t* ids, const int32_t* tt, const void* Ww, 
                const void* Wt, const void* g, const void* b, float* z0, float2* st0, void* x1,
                int B, int S, int H, int pos_offset, float eps, Drop drop, cudaStream_t st);
 // Deterministic keyed row-sum: out[key[t]] = sum over tokens with that key, in
-// token order, of rows of X [T, H] (fp32).  out rows not present are untouched.
+// token order, of rows of X [T, H] (fp32).  out rows not present, and the row of
+// key `skip` (the padding id: HF padding_idx semantics), are untouched.
 // X is clobbered (piece sums are written in place).  work: 4*T int32 + hist.
 void keyed_rowsum(const int32_t* keys, int key_bits, float* X, int T, int H, float* out,
-                  int32_t* work, int32_t* hist, int max_tiles, cudaStream_t st);
+                  int32_t* work, int32_t* hist, int max_tiles, int skip, cudaStream_t st);
 // dWt[k] = sum over tokens with token_type k of dz0 rows (fixed-order partials)
 void type_grad(const float* dz0, const int32_t* tt, int T, int H, int TV, float* part, float* dWt, cudaStream_t st);
 // dWp[pos_offset + s] = sum_b dz0[b*S + s]

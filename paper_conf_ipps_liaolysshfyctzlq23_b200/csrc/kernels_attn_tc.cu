@@ -56,24 +56,25 @@ MDEV float4 drop4_or(const Drop& d, uint64_t e) {
   return make_float4(drop_factor(d, e), drop_factor(d, e + 1), drop_factor(d, e + 2), drop_factor(d, e + 3));
 }
 
+// kmax = roundup(S, 32): the key range every MMA and every softmax pass covers.
 __global__ void __launch_bounds__(128) k_attn_fwd_tc(const __grid_constant__ CUtensorMap tq, const AttnArgs a) {
-  extern __shared__ uint8_t smem_raw[];
-  uint8_t* sm = (uint8_t*)(((uintptr_t)smem_raw + 1023) & ~(uintptr_t)1023);
+  extern __shared__ __align__(1024) uint8_t sm[];
   uint8_t* sQ = sm;
   uint8_t* sK = sm + TILE;
   uint8_t* sV = sm + 2 * TILE;
-  uint8_t* sP = sm + 3 * TILE;
-  uint64_t* bar = (uint64_t*)(sP + PT);   // [0] tma, [1] mma S, [2] mma O
+  uint8_t* sP = sm;                       // reuses Q and K (dead after S = Q K^T)
+  uint64_t* bar = (uint64_t*)(sm + 3 * TILE);   // [0] tma, [1] mma S, [2] mma O
   uint32_t* tslot = (uint32_t*)(bar + 4);
   const int t = threadIdx.x, warp = t >> 5;
   const int bh = blockIdx.x, b = bh / a.h, hd = bh % a.h;
   const int S = a.S, len = a.lengths[b];
+  const int kmax = (S + 31) & ~31, nch = kmax >> 5;
   if (t == 0) {
     for (int i = 0; i < 3; ++i) mbar_init(&bar[i], 1);
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
   }
   if (warp == 0) {
-    asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(smem_u32(tslot)), "r"(256));
+    asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(smem_u32(tslot)), "r"(128));
     asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;");
   }
   tc_fence_before();
@@ -88,7 +89,7 @@ __global__ void __launch_bounds__(128) k_attn_fwd_tc(const __grid_constant__ CUt
     tma_load_2d(&tq, &bar[0], sV, 2 * a.H + hd * AD, row0);
     mbar_wait(&bar[0], 0);
     tc_fence_after();
-    const uint32_t id = idesc_bf16(AQ, AQ, 0, 0);
+    const uint32_t id = idesc_bf16(AQ, kmax, 0, 0);
     const uint32_t q0 = smem_u32(sQ), k0 = smem_u32(sK);
 #pragma unroll
     for (int kk = 0; kk < AD / 16; ++kk)
@@ -101,30 +102,37 @@ __global__ void __launch_bounds__(128) k_attn_fwd_tc(const __grid_constant__ CUt
   // ---- softmax of row t over keys [0, len) ----
   const uint32_t trow = tmem + ((uint32_t)(32 * warp) << 16);
   float m = -INFINITY, l = 0.f;
-#pragma unroll 1
-  for (int c = 0; c < 4; ++c) {
+  for (int c = 0; c < nch; ++c) {
     float v[32];
-    tmem_ld32(trow + 32 * c, v);
+    tmem_ld32(trow + 32 * c, v);                // every lane loads (.sync.aligned)
+    if (32 * c < len) {
 #pragma unroll
-    for (int i = 0; i < 32; ++i) {
-      const float s = (32 * c + i < len) ? v[i] * a.scale : -INFINITY;
-      if (s > m) { l = l * __expf(m - s) + 1.f; m = s; } else { l += __expf(s - m); }
+      for (int i = 0; i < 32; ++i) {
+        const float s = (32 * c + i < len) ? v[i] * a.scale : -INFINITY;
+        if (s > m) { l = l * __expf(m - s) + 1.f; m = s; } else { l += __expf(s - m); }
+      }
     }
   }
   const float L = m + __logf(l);
   const uint64_t ebase = (((uint64_t)b * a.h + hd) * S + (uint64_t)t) * S;
-#pragma unroll 1
-  for (int c = 0; c < 4; ++c) {
+  // The S MMA has completed (bar[1]), so Q and K are dead: each thread writes its
+  // P~ row straight into their space.
+  for (int c = 0; c < nch; ++c) {
     float v[32];
     tmem_ld32(trow + 32 * c, v);
+    if (32 * c < len && t < S) {
 #pragma unroll
-    for (int j = 0; j < 8; ++j) {
-      const int k = 32 * c + 4 * j;
-      const float4 f = (t < S && k < len) ? drop4_or(a.drop, ebase + k) : make_float4(0.f, 0.f, 0.f, 0.f);
-      const float ff[4] = {f.x, f.y, f.z, f.w};
+      for (int j = 0; j < 8; ++j) {
+        const int k = 32 * c + 4 * j;
+        const float4 f = (k < len) ? drop4_or(a.drop, ebase + k) : make_float4(0.f, 0.f, 0.f, 0.f);
+        const float ff[4] = {f.x, f.y, f.z, f.w};
 #pragma unroll
-      for (int i = 0; i < 4; ++i)
-        v[4 * j + i] = (k + i < len) ? __expf(v[4 * j + i] * a.scale - L) * ff[i] : 0.f;
+        for (int i = 0; i < 4; ++i)
+          v[4 * j + i] = (k + i < len) ? __expf(v[4 * j + i] * a.scale - L) * ff[i] : 0.f;
+      }
+    } else {
+#pragma unroll
+      for (int i = 0; i < 32; ++i) v[i] = 0.f;
     }
     st_tile_row32(sP, t, c, v);
   }
@@ -135,11 +143,10 @@ __global__ void __launch_bounds__(128) k_attn_fwd_tc(const __grid_constant__ CUt
   if (t == 0) {
     const uint32_t id = idesc_bf16(AQ, AD, 0, 1);
     const uint32_t p0 = smem_u32(sP), v0 = smem_u32(sV);
-#pragma unroll
-    for (int kk = 0; kk < AQ / 16; ++kk) {
+    for (int kk = 0; kk < kmax / 16; ++kk) {
       const uint64_t da = make_desc(p0 + (kk >> 2) * (AQ * 128) + 32 * (kk & 3), 16, 1024);
       const uint64_t db = make_desc(v0 + 2048 * kk, 16384, 1024);
-      mma_bf16(tmem + 128, da, db, id, kk > 0);
+      mma_bf16(tmem, da, db, id, kk > 0);                   // O over S's dead columns
     }
     mma_commit(&bar[2]);
   }
@@ -151,7 +158,7 @@ __global__ void __launch_bounds__(128) k_attn_fwd_tc(const __grid_constant__ CUt
 #pragma unroll
     for (int c = 0; c < 2; ++c) {
       float v[32];
-      tmem_ld32(trow + 128 + 32 * c, v);
+      tmem_ld32(trow + 32 * c, v);
       if (t < S) st_bf16x32(orow + 32 * c, v);
     }
     if (t < S) a.lse[((int64_t)b * a.h + hd) * S + t] = L;
@@ -160,25 +167,25 @@ __global__ void __launch_bounds__(128) k_attn_fwd_tc(const __grid_constant__ CUt
   __syncthreads();
   if (warp == 0) {
     tc_fence_after();
-    asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(tmem), "r"(256));
+    asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(tmem), "r"(128));
   }
 }
 
 __global__ void __launch_bounds__(128) k_attn_bwd_tc(const __grid_constant__ CUtensorMap tq,
                                                      const __grid_constant__ CUtensorMap tdo, const AttnArgs a) {
-  extern __shared__ uint8_t smem_raw[];
-  uint8_t* sm = (uint8_t*)(((uintptr_t)smem_raw + 1023) & ~(uintptr_t)1023);
+  extern __shared__ __align__(1024) uint8_t sm[];
   uint8_t* sQ = sm;
   uint8_t* sK = sm + TILE;
-  uint8_t* sV = sm + 2 * TILE;
-  uint8_t* sdO = sm + 3 * TILE;
-  uint8_t* sP = sm + 4 * TILE;
-  uint8_t* sdS = sP + PT;
+  uint8_t* sdO = sm + 2 * TILE;
+  uint8_t* sV = sm + 3 * TILE;
+  uint8_t* sP = sV;                        // P~ (32 KB) reuses V (dead after dP) + 16 KB
+  uint8_t* sdS = sm + 5 * TILE;
   uint64_t* bar = (uint64_t*)(sdS + PT);  // [0] tma, [1] mma S/dP, [2] mma grads
   uint32_t* tslot = (uint32_t*)(bar + 4);
   const int t = threadIdx.x, warp = t >> 5;
   const int bh = blockIdx.x, b = bh / a.h, hd = bh % a.h;
   const int S = a.S, len = a.lengths[b];
+  const int kmax = (S + 31) & ~31, nch = kmax >> 5;
   if (t == 0) {
     for (int i = 0; i < 3; ++i) mbar_init(&bar[i], 1);
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
@@ -200,7 +207,7 @@ __global__ void __launch_bounds__(128) k_attn_bwd_tc(const __grid_constant__ CUt
     tma_load_2d(&tdo, &bar[0], sdO, hd * AD, row0);
     mbar_wait(&bar[0], 0);
     tc_fence_after();
-    const uint32_t id = idesc_bf16(AQ, AQ, 0, 0);
+    const uint32_t id = idesc_bf16(AQ, kmax, 0, 0);
     const uint32_t q0 = smem_u32(sQ), k0 = smem_u32(sK), v0 = smem_u32(sV), o0 = smem_u32(sdO);
 #pragma unroll
     for (int kk = 0; kk < AD / 16; ++kk)
@@ -230,24 +237,29 @@ __global__ void __launch_bounds__(128) k_attn_bwd_tc(const __grid_constant__ CUt
   tc_fence_after();
   const uint32_t trow = tmem + ((uint32_t)(32 * warp) << 16);
   const uint64_t ebase = (((uint64_t)b * a.h + hd) * S + (uint64_t)t) * S;
-#pragma unroll 1
-  for (int c = 0; c < 4; ++c) {
+  // P~ overwrites V: wait until every thread is past the MMA (V is dead)
+  for (int c = 0; c < nch; ++c) {
     float sv[32], dp[32];
     tmem_ld32(trow + 32 * c, sv);
     tmem_ld32(trow + 128 + 32 * c, dp);
+    const bool live = t < len && 32 * c < len;   // padded / foreign query rows contribute 0
+    if (live) {
 #pragma unroll
-    for (int j = 0; j < 8; ++j) {
-      const int k = 32 * c + 4 * j;
-      const bool live = t < len;                // padded / foreign query rows contribute 0
-      const float4 f = (live && k < len) ? drop4_or(a.drop, ebase + k) : make_float4(0.f, 0.f, 0.f, 0.f);
-      const float ff[4] = {f.x, f.y, f.z, f.w};
+      for (int j = 0; j < 8; ++j) {
+        const int k = 32 * c + 4 * j;
+        const float4 f = (k < len) ? drop4_or(a.drop, ebase + k) : make_float4(0.f, 0.f, 0.f, 0.f);
+        const float ff[4] = {f.x, f.y, f.z, f.w};
 #pragma unroll
-      for (int i = 0; i < 4; ++i) {
-        const int kk = k + i;
-        const float p = (live && kk < len) ? __expf(sv[4 * j + i] * a.scale - Lt) : 0.f;
-        sv[4 * j + i] = p * ff[i];                                  // P~
-        dp[4 * j + i] = p * (dp[4 * j + i] * ff[i] - Dt) * a.scale; // dS (scale folded)
+        for (int i = 0; i < 4; ++i) {
+          const int kk = k + i;
+          const float p = (kk < len) ? __expf(sv[4 * j + i] * a.scale - Lt) : 0.f;
+          sv[4 * j + i] = p * ff[i];                                  // P~
+          dp[4 * j + i] = p * (dp[4 * j + i] * ff[i] - Dt) * a.scale; // dS (scale folded)
+        }
       }
+    } else {
+#pragma unroll
+      for (int i = 0; i < 32; ++i) { sv[i] = 0.f; dp[i] = 0.f; }
     }
     st_tile_row32(sP, t, c, sv);
     st_tile_row32(sdS, t, c, dp);
@@ -261,8 +273,7 @@ __global__ void __launch_bounds__(128) k_attn_bwd_tc(const __grid_constant__ CUt
     const uint32_t id_q = idesc_bf16(AQ, AD, 0, 1);   // A K-major (queries), B MN-major (d)
     const uint32_t p0 = smem_u32(sP), s0 = smem_u32(sdS);
     const uint32_t q0 = smem_u32(sQ), k0 = smem_u32(sK), o0 = smem_u32(sdO);
-#pragma unroll
-    for (int kk = 0; kk < AQ / 16; ++kk) {      // contraction over queries (dV, dK) / keys (dQ)
+    for (int kk = 0; kk < kmax / 16; ++kk) {    // contraction over queries (dV, dK) / keys (dQ)
       const uint64_t at_p = make_desc(p0 + 2048 * kk, 16384, 1024);
       const uint64_t at_s = make_desc(s0 + 2048 * kk, 16384, 1024);
       const uint64_t bq_do = make_desc(o0 + 2048 * kk, 16384, 1024);
@@ -304,8 +315,8 @@ __global__ void __launch_bounds__(128) k_attn_bwd_tc(const __grid_constant__ CUt
 bool tc_map_bf16(CUtensorMap* out, const void* ptr, uint64_t inner, uint64_t outer, uint64_t stride_elems,
                  uint32_t box_inner, uint32_t box_outer);   // kernels_gemm_tc.cu
 
-constexpr int FWD_SMEM = 3 * TILE + PT + 1024 + 128;
-constexpr int BWD_SMEM = 4 * TILE + 2 * PT + 1024 + 128;
+constexpr int FWD_SMEM = 3 * TILE + 128;                  // P~ reuses Q/K
+constexpr int BWD_SMEM = 5 * TILE + PT + 128;             // P~ reuses V
 
 bool attn_tc_ok(int S, int H, int h) { return S <= AQ && H / h == AD && H % 64 == 0; }
 

@@ -224,27 +224,27 @@ void ln_bwd(DType dt, const float* dy, Drop premask, const float* z, const float
 // blockIdx.y selects one of up to 3 (part, out) pairs.
 struct RedJob { const float* part; float* out; };
 struct RedJobs { RedJob j[3]; };
-__global__ void __launch_bounds__(256) k_reduce_rows(RedJobs jobs, int rows, int64_t ld, int n) {
-  __shared__ float sw[8][33];
+__global__ void __launch_bounds__(1024) k_reduce_rows(RedJobs jobs, int rows, int64_t ld, int n) {
+  __shared__ float sw[32][33];
   const RedJob jb = jobs.j[blockIdx.y];
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const int c = blockIdx.x * 32 + lane;
   float acc = 0.f;
   if (c < n) {
     int p = warp;
-    for (; p + 24 < rows; p += 32) {      // 4 independent loads in flight, added in row order
-      const float v0 = jb.part[(int64_t)p * ld + c], v1 = jb.part[(int64_t)(p + 8) * ld + c];
-      const float v2 = jb.part[(int64_t)(p + 16) * ld + c], v3 = jb.part[(int64_t)(p + 24) * ld + c];
+    for (; p + 96 < rows; p += 128) {     // 4 independent loads in flight, added in row order
+      const float v0 = jb.part[(int64_t)p * ld + c], v1 = jb.part[(int64_t)(p + 32) * ld + c];
+      const float v2 = jb.part[(int64_t)(p + 64) * ld + c], v3 = jb.part[(int64_t)(p + 96) * ld + c];
       acc += v0; acc += v1; acc += v2; acc += v3;
     }
-    for (; p < rows; p += 8) acc += jb.part[(int64_t)p * ld + c];
+    for (; p < rows; p += 32) acc += jb.part[(int64_t)p * ld + c];
   }
   sw[warp][lane] = acc;
   __syncthreads();
   if (warp == 0 && c < n) {
     float t = 0.f;
 #pragma unroll
-    for (int w = 0; w < 8; ++w) t += sw[w][lane];
+    for (int w = 0; w < 32; ++w) t += sw[w][lane];
     jb.out[c] = t;
   }
 }
@@ -253,7 +253,7 @@ void reduce_rows3(const float* p0, float* o0, const float* p1, float* o1, const 
   note_launch(1);
   RedJobs jobs{{{p0, o0}, {p1, o1}, {p2, o2}}};
   const int nj = p2 ? 3 : p1 ? 2 : 1;
-  k_reduce_rows<<<dim3(cdiv(n, 32), nj), 256, 0, s>>>(jobs, rows, ld, n);
+  k_reduce_rows<<<dim3(cdiv(n, 32), nj), 1024, 0, s>>>(jobs, rows, ld, n);
 }
 void reduce_partials(const float* part, int64_t ld, int n, float* out, cudaStream_t s) {
   reduce_rows3(part, out, nullptr, nullptr, nullptr, nullptr, NPART, ld, n, s);
@@ -470,60 +470,76 @@ __global__ void __launch_bounds__(1024) k_rs_scatter(const int32_t* __restrict__
 
 // piece sums: warp per 32 sorted positions; a piece = a run of equal keys inside the chunk.
 // The piece sum overwrites the X row of the piece's first token (read-before-write, same warp).
+// Keys equal to `skip` (the pad id) are ignored.
 __global__ void __launch_bounds__(256) k_piece_sum(const int32_t* __restrict__ keys, const int32_t* __restrict__ tok,
-                                                   float* X, int T, int H) {
+                                                   float* X, int T, int H, int skip) {
   const int chunk = (blockIdx.x * blockDim.x + threadIdx.x) >> 5, lane = threadIdx.x & 31;
   const int r0 = chunk * 32;
   if (r0 >= T) return;
   const int r1 = min(r0 + 32, T);
-  for (int c0 = 0; c0 < H; c0 += 32 * 8) {
-    float acc[8];
-    int start = r0;
+  const int nv = H >> 5;
+  float acc[32];
 #pragma unroll
-    for (int j = 0; j < 8; ++j) acc[j] = 0.f;
-    for (int r = r0; r < r1; ++r) {
+  for (int j = 0; j < 32; ++j) acc[j] = 0.f;
+  int start = r0;
+  for (int r = r0; r < r1; ++r) {
+    const int key = keys[r];
+    if (key != skip) {
       const float* xr = X + (int64_t)tok[r] * H;
+      float v[32];
 #pragma unroll
-      for (int j = 0; j < 8; ++j) {
-        const int c = c0 + lane + 32 * j;
-        if (c < H) acc[j] += xr[c];
-      }
-      if (r + 1 == r1 || keys[r + 1] != keys[r]) {
+      for (int j = 0; j < 32; ++j) v[j] = j < nv ? xr[lane + 32 * j] : 0.f;
+#pragma unroll
+      for (int j = 0; j < 32; ++j) acc[j] += v[j];
+    }
+    if (r + 1 == r1 || keys[r + 1] != key) {
+      if (key != skip) {
         float* dst = X + (int64_t)tok[start] * H;
 #pragma unroll
-        for (int j = 0; j < 8; ++j) {
-          const int c = c0 + lane + 32 * j;
-          if (c < H) dst[c] = acc[j];
-          acc[j] = 0.f;
-        }
-        start = r + 1;
+        for (int j = 0; j < 32; ++j)
+          if (j < nv) dst[lane + 32 * j] = acc[j];
       }
+#pragma unroll
+      for (int j = 0; j < 32; ++j) acc[j] = 0.f;
+      start = r + 1;
     }
   }
 }
 
 // segment sums: warp per sorted position that starts a run of equal keys.
 __global__ void __launch_bounds__(256) k_segment_sum(const int32_t* __restrict__ keys, const int32_t* __restrict__ tok,
-                                                     const float* __restrict__ X, int T, int H, float* __restrict__ out) {
+                                                     const float* __restrict__ X, int T, int H, float* __restrict__ out,
+                                                     int skip) {
   const int r = (blockIdx.x * blockDim.x + threadIdx.x) >> 5, lane = threadIdx.x & 31;
   if (r >= T) return;
   const int key = keys[r];
-  if (r > 0 && keys[r - 1] == key) return;
+  if (key == skip || (r > 0 && keys[r - 1] == key)) return;
   int end = T;                                        // warp-parallel search for the run end
   for (int base = r + 1; base < T; base += 32) {
     const int i = base + lane;
     const unsigned diff = __ballot_sync(0xffffffffu, i < T && keys[i] != key);
     if (diff) { end = base + __ffs(diff) - 1; break; }
   }
-  for (int c = lane; c < H; c += 32) {
-    float acc = X[(int64_t)tok[r] * H + c];
-    for (int q = (r / 32 + 1) * 32; q < end; q += 32) acc += X[(int64_t)tok[q] * H + c];
-    out[(int64_t)key * H + c] = acc;
+  const int nv = H >> 5;
+  float acc[32];
+  const float* x0 = X + (int64_t)tok[r] * H;
+#pragma unroll
+  for (int j = 0; j < 32; ++j) acc[j] = j < nv ? x0[lane + 32 * j] : 0.f;
+  for (int q = (r / 32 + 1) * 32; q < end; q += 32) {
+    const float* xq = X + (int64_t)tok[q] * H;
+    float v[32];
+#pragma unroll
+    for (int j = 0; j < 32; ++j) v[j] = j < nv ? xq[lane + 32 * j] : 0.f;
+#pragma unroll
+    for (int j = 0; j < 32; ++j) acc[j] += v[j];
   }
+#pragma unroll
+  for (int j = 0; j < 32; ++j)
+    if (j < nv) out[(int64_t)key * H + lane + 32 * j] = acc[j];
 }
 
 void keyed_rowsum(const int32_t* keys, int key_bits, float* X, int T, int H, float* out,
-                  int32_t* work, int32_t* hist, int max_tiles, cudaStream_t s) {
+                  int32_t* work, int32_t* hist, int max_tiles, int skip, cudaStream_t s) {
   const int ntiles = cdiv(T, 1024);
   int32_t *kA = work, *vA = work + T, *kB = work + 2 * T, *vB = work + 3 * T;
   const int passes = key_bits <= 8 ? 1 : 2;
@@ -540,8 +556,8 @@ void keyed_rowsum(const int32_t* keys, int key_bits, float* X, int T, int H, flo
   }
   (void)max_tiles;
   note_launch(3 * passes + 2);
-  k_piece_sum<<<cdiv(cdiv(T, 32), 8), 256, 0, s>>>(kin, vin, X, T, H);
-  k_segment_sum<<<cdiv(T, 8), 256, 0, s>>>(kin, vin, X, T, H, out);
+  k_piece_sum<<<cdiv(cdiv(T, 32), 8), 256, 0, s>>>(kin, vin, X, T, H, skip);
+  k_segment_sum<<<cdiv(T, 8), 256, 0, s>>>(kin, vin, X, T, H, out, skip);
 }
 
 // ================================================================== heads ===
