@@ -104,7 +104,7 @@ def layernorm_bwd(dy, cache, g):
     return dz, dg, db
 
 
-_erf = np.vectorize(math.erf, otypes=[np.float64])
+from scipy.special import erf as _erf   # library primitive (fp64 erf)
 
 
 def gelu(u):
