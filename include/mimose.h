@@ -50,15 +50,17 @@ typedef enum {
   MIMOSE_E_NODEVICE = 8    /* device call on a host-only ctx (arena_base == NULL)   */
 } mimose_status;
 
-enum { MIMOSE_ARCH_POST_LN = 0 };
-enum { MIMOSE_HEAD_SEQCLS = 0, MIMOSE_HEAD_MC = 1, MIMOSE_HEAD_QA = 2 };
+enum { MIMOSE_ARCH_POST_LN = 0, MIMOSE_ARCH_PRE_LN = 1 };
+enum { MIMOSE_HEAD_SEQCLS = 0, MIMOSE_HEAD_MC = 1, MIMOSE_HEAD_QA = 2, MIMOSE_HEAD_LM = 3 };
 enum { MIMOSE_FP32 = 0, MIMOSE_BF16 = 1 };
 enum { MIMOSE_PHASE_SHELTERED = 0, MIMOSE_PHASE_RESPONSIVE = 1 };
 
 typedef struct {
   /* ---- model (post-LN BERT/RoBERTa encoder, P:227 models; reading A24) ---- */
-  int32_t arch;         /* MIMOSE_ARCH_POST_LN                                        */
-  int32_t head;         /* MIMOSE_HEAD_*: seq-cls, multiple-choice, QA span (Table II)  */
+  int32_t arch;         /* MIMOSE_ARCH_POST_LN (BERT/RoBERTa) or MIMOSE_ARCH_PRE_LN (GPT-2:
+                           causal, fp32 residual stream, tied wte, final LN)             */
+  int32_t head;         /* MIMOSE_HEAD_*: seq-cls, multiple-choice, QA span (Table II);
+                           MIMOSE_HEAD_LM (pre-LN only): chunked next-token CE          */
   int32_t dtype;        /* MIMOSE_FP32 (toy) or MIMOSE_BF16 (bf16 storage, fp32 accum,
                            fp32 master weights)                                          */
   int32_t n_layers;     /* L <= 64                                                      */
@@ -107,7 +109,8 @@ void mimose_default_config(mimose_config* cfg);
      token_type [n_seqs, seq_len]
      lengths    [n_seqs]            valid tokens per sequence, 1..seq_len
      labels     seq-cls: [n_seqs] class; MC: [n_seqs / n_choices] choice;
-                QA: [2*n_seqs] (start, end) per sequence
+                QA: [2*n_seqs] (start, end) per sequence; LM: unused (targets are
+                input_ids shifted by one inside each sequence, s < len - 1)
    The input size key of P:73/P:221 is x = n_seqs * seq_len. */
 typedef struct {
   const int32_t* input_ids;

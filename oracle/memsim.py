@@ -26,7 +26,13 @@ import dataclasses
 from typing import Dict, List, Optional, Sequence
 
 from paper_conf_ipps_liaolysshfyctzlq23_b200.workload import (
-    HEAD_QA, ModelConfig, param_spec)
+    ARCH_PRE_LN, HEAD_LM, HEAD_QA, ModelConfig, param_spec)
+
+LM_CHUNK = 512     # tokens per LM-head chunk (logits never exceed LM_CHUNK x Vpad)
+
+
+def vpad(v: int) -> int:
+    return (v + 7) // 8 * 8
 
 
 def a16(n: int) -> int:
@@ -77,6 +83,7 @@ class Sizes:
     layer_scratch: int
     emb_scratch: int
     n_layers: int
+    head_fwd_scratch: int = 0   # transient during the head forward (LM logits chunk)
 
     @property
     def i(self) -> int:
@@ -104,24 +111,42 @@ def sizes(cfg: ModelConfig, B: int, S: int, max_seqs: Optional[int] = None,
     mx = cfg.max_seq if max_seq_len is None else max_seq_len
     # pre-LN sums z0, z1, z2 are fp32 in every mode (reading R-P: bf16 z loses
     # the row mean/spread balance that LayerNorm's backward needs)
-    E = [a16(T * H * 4), a16(T * 8), a16(T * H * e)]                       # z0, st0, x1
-    internals = [a16(T * 3 * H * e), a16(T * H * e), a16(B * h * S * 4),   # QKV, O, LSE
-                 a16(T * H * 4), a16(T * 8), a16(T * H * e),               # z1, st1, h1
-                 a16(T * F * e), a16(T * F * e),                           # u, g
-                 a16(T * H * 4), a16(T * 8)]                               # z2, st2
-    y = a16(T * H * e)
-    if cfg.head == HEAD_QA:
+    pre = cfg.arch == ARCH_PRE_LN
+    if pre:
+        # GPT-2: the residual stream (x1, r1, y) is fp32; LN outputs a, m are the GEMM operands
+        E = [a16(T * H * 4)]                                                   # x1
+        internals = [a16(T * H * e), a16(T * 8), a16(T * 3 * H * e),          # a, st1, QKV
+                     a16(T * H * e), a16(B * h * S * 4),                       # O, LSE
+                     a16(T * H * 4), a16(T * 8), a16(T * H * e),               # r1, st2, m
+                     a16(T * F * e), a16(T * F * e)]                           # u, g
+        y = a16(T * H * 4)
+    else:
+        # pre-LN sums z0, z1, z2 are fp32 in every mode (reading R-P: bf16 z loses
+        # the row mean/spread balance that LayerNorm's backward needs)
+        E = [a16(T * H * 4), a16(T * 8), a16(T * H * e)]                       # z0, st0, x1
+        internals = [a16(T * 3 * H * e), a16(T * H * e), a16(B * h * S * 4),   # QKV, O, LSE
+                     a16(T * H * 4), a16(T * 8), a16(T * H * e),               # z1, st1, h1
+                     a16(T * F * e), a16(T * F * e),                           # u, g
+                     a16(T * H * 4), a16(T * 8)]                               # z2, st2
+        y = a16(T * H * e)
+    head_fwd = 0
+    if cfg.head == HEAD_LM:
+        VP = vpad(cfg.vocab)
+        head = [a16(T * H * e), a16(T * 8), a16(T * 8)]                       # hf, stf, (lse, nll)
+        head_fwd = a16(LM_CHUNK * VP * 4)                                      # fp32 logits chunk
+        head_scr = a16(LM_CHUNK * VP * 4) + a16(LM_CHUNK * VP * e)             # logits, dlogits
+    elif cfg.head == HEAD_QA:
         head = [a16(T * 2 * 4)]
         head_scr = a16(T * 2 * 4)
     else:
-        head = [a16(B * H * e), a16(B * cfg.n_out * 4)]                   # pooled, logits
+        head = [a16(B * H * e), a16(B * cfg.n_out * 4)]                       # pooled, logits
         head_scr = a16(B * cfg.n_out * 4) + a16(B * H * 4) * 2
     dy = a16(T * H * 4)
     layer_scr = a16(T * H * 4) + a16(T * F * e) + a16(T * 3 * H * e) + a16(B * h * S * 4)
     ntiles = (ms * mx + 1023) // 1024
     emb_scr = a16(T * H * 4) + a16(16 * T) + a16(4 * 256 * ntiles)   # dz0, 4 int32[T] sort arrays, digit histograms
     return Sizes(persistent_bytes(cfg, ms, mx), E, internals, y, head, dy, head_scr,
-                 layer_scr, emb_scr, cfg.n_layers)
+                 layer_scr, emb_scr, cfg.n_layers, head_fwd)
 
 
 # --------------------------------------------------------------------------
@@ -190,6 +215,9 @@ def simulate_step(sz: Sizes, dropped: Sequence[int]) -> Arena:
             A.push(sz.y)
     for t in sz.head:
         A.push(t)
+    if sz.head_fwd_scratch:                              # LM logits chunk (head forward)
+        A.talloc(sz.head_fwd_scratch)
+        A.tfree(sz.head_fwd_scratch)
     A.talloc(sz.dy)                                      # backward
     A.talloc(sz.head_scratch)
     A.tfree(sz.head_scratch)
@@ -224,9 +252,11 @@ def no_ckpt_peak(sz: Sizes) -> int:
 
 
 def lower_bound(sz: Sizes) -> int:
-    """LB: every layer but the last dropped (the last saves nothing at the
-    peak); equals the all-dropped peak."""
-    return peak(sz, range(sz.n_layers - 1))
+    """LB: every layer dropped.  For post-LN stacks this equals dropping all but
+    the last (the last saves nothing at the layer-backward peak); when the
+    head-backward event dominates (GPT-2's LM head) dropping the last layer too
+    lowers it (reading A12's last resort)."""
+    return peak(sz, range(sz.n_layers))
 
 
 # --------------------------------------------------------------------------
@@ -264,6 +294,9 @@ def collect_samples(sz: Sizes) -> Dict[str, object]:
     for t in sz.head:
         A.push(t)
     hd = A.live - b0
+    if sz.head_fwd_scratch:
+        A.talloc(sz.head_fwd_scratch)
+        A.tfree(sz.head_fwd_scratch)
     # backward with every layer recomputed; per-phase max of the top region
     A.talloc(sz.dy)
     A.top_peak_phase = sum(A.top)

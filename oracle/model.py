@@ -24,7 +24,7 @@ from typing import Dict, Optional, Sequence
 import numpy as np
 
 from paper_conf_ipps_liaolysshfyctzlq23_b200.workload import (
-    HEAD_MC, HEAD_QA, HEAD_SEQCLS, Batch, ModelConfig, param_spec)
+    ARCH_PRE_LN, HEAD_LM, HEAD_MC, HEAD_QA, HEAD_SEQCLS, Batch, ModelConfig, param_spec)
 from . import philox as px
 
 
@@ -118,6 +118,19 @@ def gelu_bwd(du_out, u):
     return du_out * (cdf + u * pdf)
 
 
+_K0 = math.sqrt(2.0 / math.pi)
+
+
+def gelu_tanh(u):
+    """GPT-2 "gelu_new": 0.5 u (1 + tanh(sqrt(2/pi) (u + 0.044715 u^3)))."""
+    return 0.5 * u * (1.0 + np.tanh(_K0 * (u + 0.044715 * u ** 3)))
+
+
+def gelu_tanh_bwd(du_out, u):
+    th = np.tanh(_K0 * (u + 0.044715 * u ** 3))
+    return du_out * (0.5 * (1.0 + th) + 0.5 * u * (1.0 - th * th) * _K0 * (1.0 + 3 * 0.044715 * u * u))
+
+
 def softmax_lastdim(s):
     m = s.max(axis=-1, keepdims=True)
     e = np.exp(s - m)
@@ -139,7 +152,7 @@ def ce_rows(logits, target):
 # attention: S = Q K^T / sqrt(d) + key-pad mask, P = softmax, O = drop(P) V
 # --------------------------------------------------------------------------
 
-def attention_fwd(qkv, lengths, B, S, h, pmask):
+def attention_fwd(qkv, lengths, B, S, h, pmask, causal=False):
     H = qkv.shape[1] // 3
     d = H // h
     q = qkv[:, :H].reshape(B, S, h, d).transpose(0, 2, 1, 3)
@@ -147,7 +160,10 @@ def attention_fwd(qkv, lengths, B, S, h, pmask):
     v = qkv[:, 2 * H:].reshape(B, S, h, d).transpose(0, 2, 1, 3)
     s = q @ k.transpose(0, 1, 3, 2) / math.sqrt(d)
     keyvalid = np.arange(S)[None, :] < np.asarray(lengths)[:, None]        # [B, S]
-    s = np.where(keyvalid[:, None, None, :], s, -np.inf)
+    allowed = np.broadcast_to(keyvalid[:, None, None, :], s.shape)
+    if causal:                                                             # key k <= query q
+        allowed = allowed & (np.arange(S)[None, :] <= np.arange(S)[:, None])[None, None]
+    s = np.where(allowed, s, -np.inf)
     p, lse = softmax_lastdim(s)
     pd = p * pmask
     o = pd @ v                                                             # [B,h,S,d]
@@ -192,6 +208,7 @@ def layer_fwd(cfg, W, l, x, lengths, B, S, masks: Masks):
 
 
 def layer_bwd(cfg, W, l, dy, c, B, S, masks: Masks, G):
+    """post-LN layer backward."""
     p = f"layer{l}."
     dz2, G[p + "ln2.g"], G[p + "ln2.b"] = layernorm_bwd(dy, c["ln2"], W[p + "ln2.g"])
     dt2 = dz2 * masks.ffn_out(l)
@@ -208,10 +225,49 @@ def layer_bwd(cfg, W, l, dy, c, B, S, masks: Masks, G):
 
 
 # --------------------------------------------------------------------------
+# GPT-2 pre-LN layer (causal): a = LN1(x); r1 = x + drop(Attn(a) Wo + bo);
+# m = LN2(r1); y = r1 + drop(gelu_tanh(m W1 + b1) W2 + b2)
+# --------------------------------------------------------------------------
+
+def layer_fwd_pre(cfg, W, l, x, lengths, B, S, masks: Masks):
+    p = f"layer{l}."
+    a, ln1 = layernorm(x, W[p + "ln1.g"], W[p + "ln1.b"], cfg.ln_eps)
+    qkv = linear(a, W[p + "qkv.w"], W[p + "qkv.b"])
+    o, acache = attention_fwd(qkv, lengths, B, S, cfg.heads, masks.attn_probs(l), causal=True)
+    r1 = x + linear(o, W[p + "o.w"], W[p + "o.b"]) * masks.attn_out(l)
+    m, ln2 = layernorm(r1, W[p + "ln2.g"], W[p + "ln2.b"], cfg.ln_eps)
+    u = linear(m, W[p + "f1.w"], W[p + "f1.b"])
+    g = gelu_tanh(u)
+    y = r1 + linear(g, W[p + "f2.w"], W[p + "f2.b"]) * masks.ffn_out(l)
+    return y, dict(a=a, ln1=ln1, qkv=qkv, o=o, acache=acache, m=m, ln2=ln2, u=u, g=g)
+
+
+def layer_bwd_pre(cfg, W, l, dy, c, B, S, masks: Masks, G):
+    p = f"layer{l}."
+    dt2 = dy * masks.ffn_out(l)
+    dg, G[p + "f2.w"], G[p + "f2.b"] = linear_bwd(dt2, c["g"], W[p + "f2.w"])
+    du = gelu_tanh_bwd(dg, c["u"])
+    dm, G[p + "f1.w"], G[p + "f1.b"] = linear_bwd(du, c["m"], W[p + "f1.w"])
+    dr1_ln, G[p + "ln2.g"], G[p + "ln2.b"] = layernorm_bwd(dm, c["ln2"], W[p + "ln2.g"])
+    dr1 = dy + dr1_ln
+    dt1 = dr1 * masks.attn_out(l)
+    do, G[p + "o.w"], G[p + "o.b"] = linear_bwd(dt1, c["o"], W[p + "o.w"])
+    dqkv = attention_bwd(do, c["acache"], B, S, cfg.heads, masks.attn_probs(l))
+    da, G[p + "qkv.w"], G[p + "qkv.b"] = linear_bwd(dqkv, c["a"], W[p + "qkv.w"])
+    dx_ln, G[p + "ln1.g"], G[p + "ln1.b"] = layernorm_bwd(da, c["ln1"], W[p + "ln1.g"])
+    return dr1 + dx_ln
+
+
+# --------------------------------------------------------------------------
 # embeddings and heads
 # --------------------------------------------------------------------------
 
 def embed_fwd(cfg, W, batch: Batch, masks: Masks):
+    if cfg.arch == ARCH_PRE_LN:                   # GPT-2: drop(wte[ids] + wpe[pos]), no LN
+        B, S = batch.input_ids.shape
+        ids = batch.input_ids.reshape(-1)
+        pos = np.tile(np.arange(S) + cfg.pos_offset, B)
+        return (W["emb.word"][ids] + W["emb.pos"][pos]) * masks.emb(), (ids, pos, None, None)
     B, S = batch.input_ids.shape
     ids = batch.input_ids.reshape(-1)
     pos = np.tile(np.arange(S) + cfg.pos_offset, B)
@@ -223,15 +279,22 @@ def embed_fwd(cfg, W, batch: Batch, masks: Masks):
 
 def embed_bwd(cfg, W, dx1, ec, masks: Masks, G):
     ids, pos, tt, cache = ec
+    if cfg.arch == ARCH_PRE_LN:                   # tied wte: add to the LM-head gradient
+        dz0 = dx1 * masks.emb()
+        np.add.at(G["emb.word"], ids, dz0)
+        acc = np.zeros_like(W["emb.pos"])
+        np.add.at(acc, pos, dz0)
+        G["emb.pos"] = acc
+        return
     dln0 = dx1 * masks.emb()
     dz0, G["emb.ln.g"], G["emb.ln.b"] = layernorm_bwd(dln0, cache, W["emb.ln.g"])
     for name, idx in (("emb.word", ids), ("emb.pos", pos), ("emb.type", tt)):
         acc = np.zeros_like(W[name])
         np.add.at(acc, idx, dz0)
         G[name] = acc
-    # HF padding_idx semantics (reading A24): the pad token's embedding row gets
-    # no gradient.  (Its accumulated value is 0 anyway: padded rows carry zero
-    # gradient because no loss term reads them, A26.)
+    # HF padding_idx semantics (reading A24, BERT/RoBERTa): the pad token's
+    # embedding row gets no gradient.  (Its accumulated value is 0 anyway: padded
+    # rows carry zero gradient because no loss term reads them, A26.)
     G["emb.word"][cfg.pad_id] = 0.0
 
 
@@ -256,6 +319,25 @@ def head_fwd_bwd(cfg, W, y, batch: Batch, masks: Masks, G):
         dpre = dpd * masks.head() * (1.0 - pl * pl)
         dc, G["pool.w"], G["pool.b"] = linear_bwd(dpre, c, W["pool.w"])
         dy[rows] = dc
+        return loss, dy
+    if cfg.head == HEAD_LM:
+        # final LN -> tied vocabulary projection -> next-token CE over s < len-1 (pads ignored)
+        hf, lnf = layernorm(y, W["lnf.g"], W["lnf.b"], cfg.ln_eps)
+        logits = hf @ W["emb.word"].T                                   # [T, V]
+        ids = batch.input_ids
+        valid = np.zeros((B, S), bool)
+        tgt = np.zeros((B, S), np.int64)
+        for b in range(B):
+            n = int(batch.lengths[b])
+            valid[b, :max(n - 1, 0)] = True
+            tgt[b, :max(n - 1, 0)] = ids[b, 1:n]
+        rows = np.nonzero(valid.reshape(-1))[0]
+        loss, dl = ce_rows(logits[rows], tgt.reshape(-1)[rows])
+        dlog = np.zeros_like(logits)
+        dlog[rows] = dl
+        dhf = dlog @ W["emb.word"]
+        G["emb.word"] = dlog.T @ hf
+        dy, G["lnf.g"], G["lnf.b"] = layernorm_bwd(dhf, lnf, W["lnf.g"])
         return loss, dy
     # QA span head: start/end logits over valid positions (pads masked, R-A26)
     logits = linear(y, W["qa.w"], W["qa.b"]).reshape(B, S, 2)
@@ -292,16 +374,18 @@ def train_step_grads(cfg: ModelConfig, params: Dict[str, np.ndarray], batch: Bat
     G: Dict[str, np.ndarray] = {}
     x, ec = embed_fwd(cfg, W, batch, masks)
     caches, inputs = [], []
+    fwd = layer_fwd_pre if cfg.arch == ARCH_PRE_LN else layer_fwd
+    bwd = layer_bwd_pre if cfg.arch == ARCH_PRE_LN else layer_bwd
     for l in range(cfg.n_layers):
         inputs.append(x)
-        x, c = layer_fwd(cfg, W, l, x, batch.lengths, B, S, masks)
+        x, c = fwd(cfg, W, l, x, batch.lengths, B, S, masks)
         caches.append(None if l in dropped else c)
     loss, dy = head_fwd_bwd(cfg, W, x, batch, masks, G)
     for l in reversed(range(cfg.n_layers)):
         c = caches[l]
         if c is None:                                   # recompute (replay)
-            _, c = layer_fwd(cfg, W, l, inputs[l], batch.lengths, B, S, masks)
-        dy = layer_bwd(cfg, W, l, dy, c, B, S, masks, G)
+            _, c = fwd(cfg, W, l, inputs[l], batch.lengths, B, S, masks)
+        dy = bwd(cfg, W, l, dy, c, B, S, masks, G)
         caches[l] = None
     embed_bwd(cfg, W, dy, ec, masks, G)
     return loss, G

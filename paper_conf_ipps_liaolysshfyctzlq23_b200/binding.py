@@ -185,7 +185,7 @@ def nccl_unique_id() -> bytes:
 def make_config(cfg: wl.ModelConfig, **kw) -> Config:
     c = Config()
     _lib.mimose_default_config(C.byref(c))
-    c.arch = 0
+    c.arch = cfg.arch
     c.head = cfg.head
     c.dtype = 0 if cfg.dtype == "fp32" else 1
     c.n_layers, c.hidden, c.heads, c.ffn = cfg.n_layers, cfg.hidden, cfg.heads, cfg.ffn

@@ -28,6 +28,18 @@ MDEV float gelu_grad_f(float u) {
   return 0.5f * (1.0f + erf_as(u * 0.70710678118654752f, e)) + u * 0.39894228040143268f * e;
 }
 
+// GPT-2 "gelu_new": 0.5 u (1 + tanh(k0 (u + 0.044715 u^3))), tanh via one exp.
+MDEV float tanh_fast(float z) { return 1.0f - __fdividef(2.0f, __expf(2.0f * z) + 1.0f); }
+MDEV float gelu_tanh_f(float u) {
+  const float z = 0.7978845608028654f * fmaf(0.044715f * u, u * u, u);
+  return 0.5f * u * (1.0f + tanh_fast(z));
+}
+MDEV float gelu_tanh_grad_f(float u) {
+  const float z = 0.7978845608028654f * fmaf(0.044715f * u, u * u, u);
+  const float th = tanh_fast(z);
+  return 0.5f * (1.0f + th) + 0.5f * u * (1.0f - th * th) * 0.7978845608028654f * fmaf(0.134145f, u * u, 1.0f);
+}
+
 // Epilogue of one output element.
 template <typename E, int EPI>
 MDEV void epilogue(const GemmArgs& g, int m, int n, float acc, int z = -1) {
@@ -48,6 +60,17 @@ MDEV void epilogue(const GemmArgs& g, int m, int n, float acc, int z = -1) {
     stf((E*)g.C + o, acc * gelu_grad_f(ldf((const E*)g.aux + (int64_t)m * g.ldx + n)));
   } else if constexpr (EPI == EPI_ACC_RES_F32) {
     ((float*)g.C)[o] = acc + ((const float*)g.res)[(int64_t)m * g.ldr + n];
+  } else if constexpr (EPI == EPI_BIAS_GELUT) {
+    E* up = (E*)g.C + o;
+    stf(up, acc + ldf((const E*)g.bias + n));
+    stf((E*)g.C2 + o, gelu_tanh_f(ldf(up)));
+  } else if constexpr (EPI == EPI_GELUT_BWD) {
+    stf((E*)g.C + o, acc * gelu_tanh_grad_f(ldf((const E*)g.aux + (int64_t)m * g.ldx + n)));
+  } else if constexpr (EPI == EPI_BIAS_DROP_RESF32) {
+    const float t = acc + ldf((const E*)g.bias + n);
+    ((float*)g.C)[o] = ((const float*)g.res)[(int64_t)m * g.ldr + n] + t * drop_factor(g.drop, (uint64_t)o);
+  } else if constexpr (EPI == EPI_ACC_F32) {
+    ((float*)g.C)[o] += acc;
   } else if constexpr (EPI == EPI_NONE) {
     if (acc == 1234.5f) ((float*)g.C)[o] = acc;   // keep the value live
   } else {

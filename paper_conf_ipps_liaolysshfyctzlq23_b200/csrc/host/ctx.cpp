@@ -36,9 +36,27 @@ struct ParamInfo {
 };
 
 // The documented parameter order (DESIGN "Parameter layout").
+constexpr int LM_CHUNK = 512;   // tokens per LM-head chunk (DESIGN "Memory model")
+inline int64_t vpad(int64_t v) { return (v + 7) / 8 * 8; }
+
 std::vector<ParamInfo> build_layout(const mimose_config& c, int64_t* npad) {
   std::vector<int64_t> n;
   const int64_t H = c.hidden, F = c.ffn;
+  if (c.arch == 1) {             // GPT-2: wte, wpe, pre-LN layers, lnf
+    n.push_back((int64_t)c.vocab * H);
+    n.push_back((int64_t)c.max_pos * H);
+    for (int l = 0; l < c.n_layers; ++l) {
+      const int64_t v[12] = {H, H, 3 * H * H, 3 * H, H * H, H, H, H, F * H, F, H * F, H};
+      for (int64_t x : v) n.push_back(x);
+    }
+    n.push_back(H);
+    n.push_back(H);
+    std::vector<ParamInfo> out;
+    int64_t off = 0;
+    for (int64_t x : n) { out.push_back({x, off}); off += (x + 63) / 64 * 64; }
+    *npad = off;
+    return out;
+  }
   n.push_back((int64_t)c.vocab * H);
   n.push_back((int64_t)c.max_pos * H);
   n.push_back((int64_t)c.type_vocab * H);
@@ -129,6 +147,8 @@ struct Arena {
 struct LayerBufs {
   char *qkv = nullptr, *O = nullptr, *h1 = nullptr, *u = nullptr, *g = nullptr;
   float *z1 = nullptr, *z2 = nullptr;   // pre-LN sums, fp32 (reading R-P)
+  char *a = nullptr, *m = nullptr;      // GPT-2: LN1 / LN2 outputs (GEMM operands)
+  float* r1 = nullptr;                  // GPT-2: mid-layer residual stream (fp32)
   float *lse = nullptr;
   float2 *st1 = nullptr, *st2 = nullptr;
 };
@@ -168,8 +188,9 @@ struct mimose_ctx {
   float2* st0 = nullptr;
   std::vector<LayerBufs> lb;
   std::vector<char*> y;
-  char* hp = nullptr;         // pooled (cls) or unused
+  char* hp = nullptr;         // pooled (cls) or LM: LNf output hf
   float* logits = nullptr;
+  float2 *lm_stf = nullptr, *lm_tok = nullptr;   // LM head: LNf stats, per-token (lse, nll)
   int64_t it = 0;             // dropout step counter (forward calls)
   int64_t adam_t = 0;
 
@@ -216,20 +237,32 @@ struct Sz {
   int64_t z0, st0, x1;
   int64_t qkv, O, lse, z1, st1, h1, u, g, z2, st2;
   int64_t y;
-  int64_t head0, head1;   // QA: head0 = logits, head1 = 0
+  int64_t head0, head1, head2;   // QA: logits; cls: pooled, logits; LM: hf, stf, tokstat
+  int64_t head_fwd;               // LM: fp32 logits chunk during the head forward
   int64_t dy, head_scr, layer_scr, emb_scr;
+  // pre-LN (GPT-2) internals
+  int64_t a, r1, m;
   int64_t r_dres, r_du, r_dt;  // carve offsets inside layer scratch
 };
 
 Sz sizes(const mimose_ctx* c, int B, int S) {
   const int64_t T = (int64_t)B * S, H = c->cfg.hidden, F = c->cfg.ffn, h = c->cfg.heads, e = c->e;
   Sz z{};
-  z.z0 = a16(T * H * 4); z.st0 = a16(T * 8); z.x1 = a16(T * H * e);
+  const bool pre = c->cfg.arch == 1;
+  z.z0 = a16(T * H * 4); z.st0 = a16(T * 8); z.x1 = pre ? a16(T * H * 4) : a16(T * H * e);
+  z.a = a16(T * H * e); z.r1 = a16(T * H * 4); z.m = a16(T * H * e);
   z.qkv = a16(T * 3 * H * e); z.O = a16(T * H * e); z.lse = a16((int64_t)B * h * S * 4);
   z.z1 = a16(T * H * 4); z.st1 = a16(T * 8); z.h1 = a16(T * H * e);
   z.u = a16(T * F * e); z.g = a16(T * F * e); z.z2 = a16(T * H * 4); z.st2 = a16(T * 8);
-  z.y = a16(T * H * e);
-  if (c->cfg.head == MIMOSE_HEAD_QA) {
+  z.y = pre ? a16(T * H * 4) : a16(T * H * e);
+  z.head2 = 0;
+  z.head_fwd = 0;
+  if (c->cfg.head == 3) {                     // LM head (GPT-2)
+    const int64_t VP = vpad(c->cfg.vocab);
+    z.head0 = a16(T * H * e); z.head1 = a16(T * 8); z.head2 = a16(T * 8);
+    z.head_fwd = a16((int64_t)LM_CHUNK * VP * 4);
+    z.head_scr = a16((int64_t)LM_CHUNK * VP * 4) + a16((int64_t)LM_CHUNK * VP * e);
+  } else if (c->cfg.head == MIMOSE_HEAD_QA) {
     z.head0 = a16(T * 2 * 4); z.head1 = 0;
     z.head_scr = a16(T * 2 * 4);
   } else {
@@ -276,8 +309,14 @@ Drop no_drop() { Drop d{}; d.enabled = 0; return d; }
 
 inline char* W(mimose_ctx* c, int i) { return c->w + c->layout[i].off * c->e; }
 inline float* G(mimose_ctx* c, int i) { return c->grad + c->layout[i].off; }
-inline int LP(mimose_ctx* c, int l, int k) { (void)c; return P_LAYER0 + 12 * l + k; }
-inline int HP(mimose_ctx* c, int k) { return P_LAYER0 + 12 * c->cfg.n_layers + k; }
+// Parameter index of semantic slot k (L_*) of layer l.  Post-LN order is the
+// L_* enum order; GPT-2 (pre-LN) stores [ln1, qkv, o, ln2, f1, f2].
+inline int layer_base(const mimose_ctx* c) { return c->cfg.arch == 1 ? 2 : P_LAYER0; }
+inline int LP(mimose_ctx* c, int l, int k) {
+  static const int pre_pos[12] = {2, 3, 4, 5, 0, 1, 8, 9, 10, 11, 6, 7};
+  return layer_base(c) + 12 * l + (c->cfg.arch == 1 ? pre_pos[k] : k);
+}
+inline int HP(mimose_ctx* c, int k) { return layer_base(c) + 12 * c->cfg.n_layers + k; }
 
 // ------------------------------------------------------------- probe ------
 void pgemm(mimose_ctx* c, Epi epi, const GemmArgs& g, cudaStream_t st) {
@@ -354,13 +393,21 @@ void layer_forward(Run& r, int l, const char* x, LayerBufs& b, char* yout) {
 void alloc_internals(Run& r, LayerBufs& b, bool on_stack) {
   Arena& a = r.c->ar;
   auto al = [&](int64_t n) { return on_stack ? a.push(n) : a.talloc(n); };
+  if (r.c->cfg.arch == 1) {   // [a, st1, QKV, O, LSE, r1, st2, m, u, g]
+    b.a = al(r.z.a); b.st1 = (float2*)al(r.z.st1); b.qkv = al(r.z.qkv); b.O = al(r.z.O);
+    b.lse = (float*)al(r.z.lse); b.r1 = (float*)al(r.z.r1); b.st2 = (float2*)al(r.z.st2); b.m = al(r.z.m);
+    b.u = al(r.z.u); b.g = al(r.z.g);
+    return;
+  }
   b.qkv = al(r.z.qkv); b.O = al(r.z.O); b.lse = (float*)al(r.z.lse);
   b.z1 = (float*)al(r.z.z1); b.st1 = (float2*)al(r.z.st1); b.h1 = al(r.z.h1);
   b.u = al(r.z.u); b.g = al(r.z.g); b.z2 = (float*)al(r.z.z2); b.st2 = (float2*)al(r.z.st2);
 }
 void free_internals(Run& r, bool on_stack) {
   Arena& a = r.c->ar;
-  const int64_t s[10] = {r.z.qkv, r.z.O, r.z.lse, r.z.z1, r.z.st1, r.z.h1, r.z.u, r.z.g, r.z.z2, r.z.st2};
+  const int64_t s0[10] = {r.z.qkv, r.z.O, r.z.lse, r.z.z1, r.z.st1, r.z.h1, r.z.u, r.z.g, r.z.z2, r.z.st2};
+  const int64_t s1[10] = {r.z.a, r.z.st1, r.z.qkv, r.z.O, r.z.lse, r.z.r1, r.z.st2, r.z.m, r.z.u, r.z.g};
+  const int64_t* s = r.c->cfg.arch == 1 ? s1 : s0;
   for (int i = 9; i >= 0; --i) on_stack ? a.pop(s[i]) : a.tfree(s[i]);
 }
 
@@ -441,6 +488,153 @@ void layer_backward(Run& r, int l, const char* x, LayerBufs& b, float* dy, char*
   reduce_partials(c->part, 3 * H, 3 * H, G(c, LP(c, l, L_QKVB)), r.st);
 }
 
+// ---------------------------------------------------------------------------
+// GPT-2 pre-LN layer (causal): a = LN1(x); r1 = x + drop(Attn(a) Wo + bo);
+// m = LN2(r1); y = r1 + drop(gelu_tanh(m W1 + b1) W2 + b2).  x, r1, y fp32.
+// In recompute (yout == nullptr) the FFN2 GEMM is skipped: y is not needed.
+// ---------------------------------------------------------------------------
+void layer_forward_pre(Run& r, int l, const float* x, LayerBufs& b, float* yout) {
+  mimose_ctx* c = r.c;
+  if (!r.real) return;
+  const int T = c->T, H = c->cfg.hidden, F = c->cfg.ffn;
+  ln_fwd(c->dt, x, W(c, LP(c, l, L_LN1G)), W(c, LP(c, l, L_LN1B)), b.a, b.st1, T, H, c->cfg.ln_eps, r.st);
+  GemmArgs g;
+  g.M = T; g.N = 3 * H; g.K = H;
+  g.A = b.a; g.a_sm = H; g.a_sk = 1;
+  g.B = W(c, LP(c, l, L_QKVW)); g.b_sn = H; g.b_sk = 1;
+  g.C = b.qkv; g.ldc = 3 * H; g.bias = W(c, LP(c, l, L_QKVB));
+  pgemm(c, EPI_BIAS, g, r.st);
+  attn_fwd(c->dt, b.qkv, c->lens, b.O, b.lse, c->B, c->S, H, c->cfg.heads, make_drop(c, KIND_ATTN_PROBS, l), r.st,
+           true);
+  g = GemmArgs();
+  g.M = T; g.N = H; g.K = H;
+  g.A = b.O; g.a_sm = H; g.a_sk = 1;
+  g.B = W(c, LP(c, l, L_OW)); g.b_sn = H; g.b_sk = 1;
+  g.C = b.r1; g.ldc = H; g.bias = W(c, LP(c, l, L_OB)); g.res = x; g.ldr = H;
+  g.drop = make_drop(c, KIND_ATTN_OUT, l);
+  pgemm(c, EPI_BIAS_DROP_RESF32, g, r.st);
+  ln_fwd(c->dt, b.r1, W(c, LP(c, l, L_LN2G)), W(c, LP(c, l, L_LN2B)), b.m, b.st2, T, H, c->cfg.ln_eps, r.st);
+  g = GemmArgs();
+  g.M = T; g.N = F; g.K = H;
+  g.A = b.m; g.a_sm = H; g.a_sk = 1;
+  g.B = W(c, LP(c, l, L_F1W)); g.b_sn = H; g.b_sk = 1;
+  g.C = b.u; g.C2 = b.g; g.ldc = F; g.bias = W(c, LP(c, l, L_F1B));
+  pgemm(c, EPI_BIAS_GELUT, g, r.st);
+  if (!yout) return;
+  g = GemmArgs();
+  g.M = T; g.N = H; g.K = F;
+  g.A = b.g; g.a_sm = F; g.a_sk = 1;
+  g.B = W(c, LP(c, l, L_F2W)); g.b_sn = F; g.b_sk = 1;
+  g.C = yout; g.ldc = H; g.bias = W(c, LP(c, l, L_F2B)); g.res = b.r1; g.ldr = H;
+  g.drop = make_drop(c, KIND_FFN_OUT, l);
+  pgemm(c, EPI_BIAS_DROP_RESF32, g, r.st);
+}
+
+void layer_backward_pre(Run& r, int l, const float* x, LayerBufs& b, float* dy, char* scr) {
+  mimose_ctx* c = r.c;
+  if (!r.real) return;
+  const int T = c->T, H = c->cfg.hidden, F = c->cfg.ffn, h = c->cfg.heads;
+  float* dres = (float*)(scr + r.z.r_dres);
+  char* R2 = scr + r.z.r_du;     // du, later dO
+  char* R3 = scr + r.z.r_dt;     // dt2 / dt1, later dQKV
+  float* Dbuf = (float*)(scr + r.z.r_dt + a16((int64_t)T * 3 * H * c->e));
+  float* pg = c->part;
+  float* pb = c->part + (int64_t)NPART * H;
+  float* pbias = c->part + 2LL * NPART * H;
+  // dt2 = dy * mask (bf16), db2 = colsum dt2
+  drop_cast_colsum(c->dt, dy, make_drop(c, KIND_FFN_OUT, l), R3, T, H, pbias, r.st);
+  reduce_partials(pbias, H, H, G(c, LP(c, l, L_F2B)), r.st);
+  // FFN2: du = (dt2 W2) * gelu_tanh'(u); dW2 = dt2^T g
+  {
+    GemmArgs g;
+    g.M = T; g.N = F; g.K = H;
+    g.A = R3; g.a_sm = H; g.a_sk = 1;
+    g.B = W(c, LP(c, l, L_F2W)); g.b_sn = 1; g.b_sk = F;
+    g.C = R2; g.ldc = F; g.aux = b.u; g.ldx = F;
+    pgemm(c, EPI_GELUT_BWD, g, r.st);
+  }
+  wgrad(r, R3, H, b.g, F, G(c, LP(c, l, L_F2W)));
+  // FFN1: dm = du W1 (fp32, dres); dW1 = du^T m; db1
+  dgrad(r, EPI_F32, R2, F, W(c, LP(c, l, L_F1W)), H, dres, nullptr);
+  wgrad(r, R2, F, b.m, H, G(c, LP(c, l, L_F1W)));
+  colsum(c->dt, R2, T, F, c->part, r.st);
+  reduce_partials(c->part, F, F, G(c, LP(c, l, L_F1B)), r.st);
+  // LN2 backward + residual: dr1 = dy + LN2'(dm) (in place in dy); dt1 = dr1 * mask (R3)
+  ln_bwd(c->dt, dres, no_drop(), b.r1, b.st2, W(c, LP(c, l, L_LN2G)), dy, R3, make_drop(c, KIND_ATTN_OUT, l),
+         pg, pb, pbias, T, H, r.st, dy);
+  reduce_rows3(pg, G(c, LP(c, l, L_LN2G)), pb, G(c, LP(c, l, L_LN2B)), pbias, G(c, LP(c, l, L_OB)), NPART, H, H,
+               r.st);
+  // out-proj: dO = dt1 Wo (R2); dWo = dt1^T O
+  dgrad(r, EPI_STORE, R3, H, W(c, LP(c, l, L_OW)), H, R2, nullptr);
+  wgrad(r, R3, H, b.O, H, G(c, LP(c, l, L_OW)));
+  attn_bwd(c->dt, b.qkv, b.O, R2, b.lse, c->lens, Dbuf, R3, c->B, c->S, H, h, make_drop(c, KIND_ATTN_PROBS, l),
+           r.st, true);
+  // QKV: da = dQKV Wqkv (fp32, dres); dWqkv = dQKV^T a; dbqkv
+  dgrad(r, EPI_F32, R3, 3 * H, W(c, LP(c, l, L_QKVW)), H, dres, nullptr);
+  wgrad(r, R3, 3 * H, b.a, H, G(c, LP(c, l, L_QKVW)));
+  colsum(c->dt, R3, T, 3 * H, c->part, r.st);
+  reduce_partials(c->part, 3 * H, 3 * H, G(c, LP(c, l, L_QKVB)), r.st);
+  // LN1 backward + residual: dx = dr1 + LN1'(da) (in place in dy)
+  ln_bwd(c->dt, dres, no_drop(), x, b.st1, W(c, LP(c, l, L_LN1G)), dy, nullptr, no_drop(), pg, pb, nullptr, T, H,
+         r.st, dy);
+  reduce_rows3(pg, G(c, LP(c, l, L_LN1G)), pb, G(c, LP(c, l, L_LN1B)), nullptr, nullptr, NPART, H, H, r.st);
+}
+
+// LM head (GPT-2): hf = LNf(y); chunks of LM_CHUNK tokens: logits = hf W_e^T (fp32),
+// per-token (lse, nll); loss = sum nll / #targets.
+void lm_head_forward(Run& r, float* yL, char* hf, float2* stf, float2* tok, float* logits) {
+  mimose_ctx* c = r.c;
+  const int T = c->T, H = c->cfg.hidden, V = c->cfg.vocab;
+  const int64_t VP = vpad(V);
+  ln_fwd(c->dt, yL, W(c, HP(c, 0)), W(c, HP(c, 1)), hf, stf, T, H, c->cfg.ln_eps, r.st);
+  for (int r0 = 0; r0 < T; r0 += LM_CHUNK) {
+    const int nc = std::min(LM_CHUNK, T - r0);
+    GemmArgs g;
+    g.M = nc; g.N = V; g.K = H;
+    g.A = hf + (int64_t)r0 * H * c->e; g.a_sm = H; g.a_sk = 1;
+    g.B = W(c, P_WORD); g.b_sn = H; g.b_sk = 1;
+    g.C = logits; g.ldc = VP;
+    pgemm(c, EPI_F32, g, r.st);
+    lm_ce_fwd(logits, VP, V, r0, nc, c->ids, c->lens, c->S, tok, r.st);
+  }
+  lm_loss(tok, T, c->lens, c->B, c->S, c->misc, r.st);
+}
+
+// Backward of the LM head into dy (fp32 [T, H]); dW_e accumulates chunk by chunk.
+void lm_head_backward(Run& r, float* yL, char* hf, float2* stf, float2* tok, char* scr, float* dy) {
+  mimose_ctx* c = r.c;
+  const int T = c->T, H = c->cfg.hidden, V = c->cfg.vocab;
+  const int64_t VP = vpad(V);
+  float* logits = (float*)scr;
+  char* dlog = scr + a16((int64_t)LM_CHUNK * VP * 4);
+  for (int r0 = 0; r0 < T; r0 += LM_CHUNK) {
+    const int nc = std::min(LM_CHUNK, T - r0);
+    GemmArgs g;
+    g.M = nc; g.N = V; g.K = H;
+    g.A = hf + (int64_t)r0 * H * c->e; g.a_sm = H; g.a_sk = 1;
+    g.B = W(c, P_WORD); g.b_sn = H; g.b_sk = 1;
+    g.C = logits; g.ldc = VP;
+    pgemm(c, EPI_F32, g, r.st);                                  // recompute the chunk's logits
+    lm_ce_bwd(c->dt, logits, VP, V, r0, nc, c->ids, c->lens, c->B, c->S, tok, dlog, r.st);
+    g = GemmArgs();                                               // dh = dlog W_e
+    g.M = nc; g.N = H; g.K = V;
+    g.A = dlog; g.a_sm = VP; g.a_sk = 1;
+    g.B = W(c, P_WORD); g.b_sn = 1; g.b_sk = H;
+    g.C = dy + (int64_t)r0 * H; g.ldc = H;
+    pgemm(c, EPI_F32, g, r.st);
+    g = GemmArgs();                                               // dW_e += dlog^T hf
+    g.M = V; g.N = H; g.K = nc;
+    g.A = dlog; g.a_sm = 1; g.a_sk = VP;
+    g.B = hf + (int64_t)r0 * H * c->e; g.b_sn = 1; g.b_sk = H;
+    g.C = G(c, P_WORD); g.ldc = H;
+    pgemm(c, EPI_ACC_F32, g, r.st);
+  }
+  float* pg = c->part;
+  float* pb = c->part + (int64_t)NPART * H;
+  ln_bwd(c->dt, dy, no_drop(), yL, stf, W(c, HP(c, 0)), dy, nullptr, no_drop(), pg, pb, nullptr, T, H, r.st);
+  reduce_rows3(pg, G(c, HP(c, 0)), pb, G(c, HP(c, 1)), nullptr, nullptr, NPART, H, H, r.st);
+}
+
 int64_t bucket_begin(mimose_ctx* c, int first_param) { return c->layout[first_param].off; }
 int64_t bucket_end(mimose_ctx* c, int last_param) {
   return c->layout[last_param].off + (c->layout[last_param].numel + 63) / 64 * 64;
@@ -461,11 +655,12 @@ mimose_status copy_batch(mimose_ctx* c, const mimose_batch* bt) {
   int nl;
   if (c->cfg.head == MIMOSE_HEAD_MC) nl = bt->n_seqs / c->cfg.n_choices;
   else if (c->cfg.head == MIMOSE_HEAD_QA) nl = 2 * bt->n_seqs;
+  else if (c->cfg.head == 3) nl = 0;            // LM targets are the next input tokens
   else nl = bt->n_seqs;
   CK(cudaMemcpyAsync(c->ids, bt->input_ids, T * 4, k, c->st));
   CK(cudaMemcpyAsync(c->tt, bt->token_type, T * 4, k, c->st));
   CK(cudaMemcpyAsync(c->lens, bt->lengths, (int64_t)bt->n_seqs * 4, k, c->st));
-  CK(cudaMemcpyAsync(c->labels, bt->labels, (int64_t)nl * 4, k, c->st));
+  if (nl) CK(cudaMemcpyAsync(c->labels, bt->labels, (int64_t)nl * 4, k, c->st));
   return MIMOSE_OK;
 }
 
@@ -479,6 +674,15 @@ mimose_status check_batch(mimose_ctx* c, const mimose_batch* bt) {
   return MIMOSE_OK;
 }
 
+void layer_fwd_any(Run& r, int l, const char* x, LayerBufs& b, char* yout) {
+  if (r.c->cfg.arch == 1) layer_forward_pre(r, l, (const float*)x, b, (float*)yout);
+  else layer_forward(r, l, x, b, yout);
+}
+void layer_bwd_any(Run& r, int l, const char* x, LayerBufs& b, float* dy, char* scr) {
+  if (r.c->cfg.arch == 1) layer_backward_pre(r, l, (const float*)x, b, dy, scr);
+  else layer_backward(r, l, x, b, dy, scr);
+}
+
 // Forward of one step.  mode 0: plan-driven; mode 1: shuttling collector.
 // When `sample` is non-null the collector deltas are recorded.
 void run_forward(Run& r, uint64_t mask, bool collect, Sample* sample) {
@@ -486,14 +690,24 @@ void run_forward(Run& r, uint64_t mask, bool collect, Sample* sample) {
   Arena& a = c->ar;
   const int L = c->cfg.n_layers, H = c->cfg.hidden;
   const int64_t base = a.live();
-  c->z0 = (float*)a.push(r.z.z0);
-  c->st0 = (float2*)a.push(r.z.st0);
-  c->x1 = a.push(r.z.x1);
-  if (sample) sample->E = a.live() - base;
-  if (r.real)
-    embed_fwd(c->dt, c->ids, c->tt, W(c, P_WORD), W(c, P_POS), W(c, P_TYPE), W(c, P_LN0G), W(c, P_LN0B), c->z0,
-              c->st0, c->x1, c->B, c->S, H, c->cfg.pos_offset, c->cfg.ln_eps, make_drop(c, KIND_EMB, LAYER_NONE),
-              r.st);
+  if (c->cfg.arch == 1) {                       // GPT-2: x1 = drop(wte[ids] + wpe[pos]) (fp32)
+    c->z0 = nullptr;
+    c->st0 = nullptr;
+    c->x1 = a.push(r.z.x1);
+    if (sample) sample->E = a.live() - base;
+    if (r.real)
+      embed_fwd_pre(c->dt, c->ids, W(c, P_WORD), W(c, P_POS), (float*)c->x1, c->B, c->S, H, c->cfg.pos_offset,
+                    make_drop(c, KIND_EMB, LAYER_NONE), r.st);
+  } else {
+    c->z0 = (float*)a.push(r.z.z0);
+    c->st0 = (float2*)a.push(r.z.st0);
+    c->x1 = a.push(r.z.x1);
+    if (sample) sample->E = a.live() - base;
+    if (r.real)
+      embed_fwd(c->dt, c->ids, c->tt, W(c, P_WORD), W(c, P_POS), W(c, P_TYPE), W(c, P_LN0G), W(c, P_LN0B), c->z0,
+                c->st0, c->x1, c->B, c->S, H, c->cfg.pos_offset, c->cfg.ln_eps, make_drop(c, KIND_EMB, LAYER_NONE),
+                r.st);
+  }
   c->lb.assign(L, LayerBufs());
   c->y.assign(L, nullptr);
   const char* x = c->x1;
@@ -505,7 +719,7 @@ void run_forward(Run& r, uint64_t mask, bool collect, Sample* sample) {
       alloc_internals(r, tmp, true);
       char* yt = a.push(r.z.y);
       if (r.real) cudaEventRecord(c->ev_t0[l], r.st);
-      layer_forward(r, l, x, tmp, yt);
+      layer_fwd_any(r, l, x, tmp, yt);
       if (r.real) cudaEventRecord(c->ev_t1[l], r.st);
       sample->a[l] = a.live() - b0;
       a.pop(r.z.y);
@@ -514,13 +728,22 @@ void run_forward(Run& r, uint64_t mask, bool collect, Sample* sample) {
     const bool dropped = collect || ((mask >> l) & 1);
     alloc_internals(r, c->lb[l], !dropped);
     c->y[l] = a.push(r.z.y);
-    layer_forward(r, l, x, c->lb[l], c->y[l]);
+    layer_fwd_any(r, l, x, c->lb[l], c->y[l]);
     if (dropped) free_internals(r, false);
     if (sample) sample->y[l] = a.live() - b0;
     x = c->y[l];
   }
   const int64_t h0 = a.live();
-  if (c->cfg.head == MIMOSE_HEAD_QA) {
+  if (c->cfg.head == 3) {                       // LM head: hf, stf, tokstat; fp32 logits chunk transient
+    c->hp = a.push(r.z.head0);
+    c->lm_stf = (float2*)a.push(r.z.head1);
+    c->lm_tok = (float2*)a.push(r.z.head2);
+    if (sample) sample->Hd = a.live() - h0;
+    float* lg = (float*)a.talloc(r.z.head_fwd);
+    if (r.real) lm_head_forward(r, (float*)c->y[L - 1], c->hp, c->lm_stf, c->lm_tok, lg);
+    a.tfree(r.z.head_fwd);
+    return;
+  } else if (c->cfg.head == MIMOSE_HEAD_QA) {
     c->logits = (float*)a.push(r.z.head0);
     if (r.real)
       head_qa_fwd(c->dt, c->y[L - 1], c->B, c->S, H, W(c, HP(c, 0)), W(c, HP(c, 1)), c->logits, c->lens,
@@ -547,7 +770,11 @@ mimose_status run_backward(Run& r, Sample* sample) {
   a.top_phase_peak = a.top;
   char* hs = a.talloc(r.z.head_scr);
   if (r.real) {
-    if (c->cfg.head == MIMOSE_HEAD_QA) {
+    if (c->cfg.head == 3) {
+      // the tied wte gradient accumulates: LM head chunks now, the embedding lookup later
+      CK(cudaMemsetAsync(G(c, P_WORD), 0, (size_t)c->layout[P_WORD].numel * 4, r.st));
+      lm_head_backward(r, (float*)c->y[L - 1], c->hp, c->lm_stf, c->lm_tok, hs, dy);
+    } else if (c->cfg.head == MIMOSE_HEAD_QA) {
       head_qa_bwd(c->dt, c->y[L - 1], c->B, c->S, H, W(c, HP(c, 0)), c->logits, c->lens, c->labels, (float*)hs,
                   c->part, G(c, HP(c, 0)), G(c, HP(c, 1)), dy, r.st);
     } else {
@@ -561,11 +788,15 @@ mimose_status run_backward(Run& r, Sample* sample) {
   a.tfree(r.z.head_scr);
   if (sample) sample->Th = a.top_phase_peak;
   if (r.real) {
-    const int nh = c->cfg.head == MIMOSE_HEAD_QA ? 2 : 4;
+    const int nh = (c->cfg.head == MIMOSE_HEAD_QA || c->cfg.head == 3) ? 2 : 4;
     mimose_status s = allreduce_bucket(c, HP(c, 0), HP(c, nh - 1), L);
     if (s) return s;
   }
-  if (c->cfg.head == MIMOSE_HEAD_QA) {
+  if (c->cfg.head == 3) {
+    a.pop(r.z.head2);
+    a.pop(r.z.head1);
+    a.pop(r.z.head0);
+  } else if (c->cfg.head == MIMOSE_HEAD_QA) {
     a.pop(r.z.head0);
   } else {
     a.pop(r.z.head1);
@@ -579,13 +810,13 @@ mimose_status run_backward(Run& r, Sample* sample) {
     const char* x = l > 0 ? c->y[l - 1] : c->x1;
     if (dropped) {                                    // recompute right before the gradients
       alloc_internals(r, c->lb[l], true);
-      layer_forward(r, l, x, c->lb[l], nullptr);
+      layer_fwd_any(r, l, x, c->lb[l], nullptr);
     }
     char* scr = a.talloc(r.z.layer_scr);
-    layer_backward(r, l, x, c->lb[l], dy, scr);
+    layer_bwd_any(r, l, x, c->lb[l], dy, scr);
     a.tfree(r.z.layer_scr);
     if (r.real) {
-      mimose_status s = allreduce_bucket(c, LP(c, l, 0), LP(c, l, 11), l);
+      mimose_status s = allreduce_bucket(c, layer_base(c) + 12 * l, layer_base(c) + 12 * l + 11, l);
       if (s) return s;
     }
     free_internals(r, true);
@@ -595,7 +826,17 @@ mimose_status run_backward(Run& r, Sample* sample) {
   // ---- embedding ----
   a.top_phase_peak = a.top;
   char* es = a.talloc(r.z.emb_scr);
-  if (r.real) {
+  if (r.real && c->cfg.arch == 1) {
+    float* dz0 = (float*)es;
+    int32_t* work = (int32_t*)(es + a16((int64_t)T * H * 4));
+    int32_t* hist = (int32_t*)(es + a16((int64_t)T * H * 4) + a16(16LL * T));
+    drop_f32(dy, make_drop(c, KIND_EMB, LAYER_NONE), dz0, (int64_t)T * H, r.st);
+    CK(cudaMemsetAsync(G(c, P_POS), 0, (size_t)c->layout[P_POS].numel * 4, r.st));
+    pos_grad(dz0, c->B, c->S, H, c->cfg.pos_offset, G(c, P_POS), r.st);
+    const int64_t maxT = (int64_t)c->cfg.max_seqs * c->cfg.max_seq_len;
+    keyed_rowsum(c->ids, c->cfg.vocab <= 256 ? 8 : 16, dz0, T, H, G(c, P_WORD), work, hist,
+                 (int)((maxT + 1023) / 1024), c->cfg.pad_id, r.st, /*accumulate=*/true);
+  } else if (r.real) {
     float* dz0 = (float*)es;
     int32_t* work = (int32_t*)(es + a16((int64_t)T * H * 4));
     int32_t* hist = (int32_t*)(es + a16((int64_t)T * H * 4) + a16(16LL * T));
@@ -616,12 +857,14 @@ mimose_status run_backward(Run& r, Sample* sample) {
   a.tfree(r.z.emb_scr);
   if (sample) sample->Te = a.top_phase_peak;
   if (r.real) {
-    mimose_status s = allreduce_bucket(c, P_WORD, P_LN0B, L + 1);
+    mimose_status s = allreduce_bucket(c, P_WORD, c->cfg.arch == 1 ? P_POS : P_LN0B, L + 1);
     if (s) return s;
   }
   a.pop(r.z.x1);
-  a.pop(r.z.st0);
-  a.pop(r.z.z0);
+  if (c->cfg.arch != 1) {
+    a.pop(r.z.st0);
+    a.pop(r.z.z0);
+  }
   a.tfree(r.z.dy);
   return MIMOSE_OK;
 }
@@ -728,11 +971,12 @@ mimose_status mimose_init(const mimose_config* cfgp, mimose_ctx** out) {
   c->cfg = *cfgp;
   const mimose_config& k = c->cfg;
   auto bad = [&](const char* m) { c->err = m; return MIMOSE_E_INVALID; };
-  if (k.arch != MIMOSE_ARCH_POST_LN || k.n_layers < 1 || k.n_layers > 64 || k.hidden % 64 || k.heads < 1 ||
+  const bool arch_ok = (k.arch == MIMOSE_ARCH_POST_LN && k.head >= 0 && k.head <= 2) || (k.arch == 1 && k.head == 3);
+  if (!arch_ok || k.n_layers < 1 || k.n_layers > 64 || k.hidden % 64 || k.heads < 1 ||
       k.hidden % k.heads || (k.hidden / k.heads != 32 && k.hidden / k.heads != 64) || k.ffn % 64 ||
-      k.hidden > 1024 || k.ffn > 4096 || k.vocab < 1 || k.vocab > 65536 || k.type_vocab < 1 || k.type_vocab > 4 ||
+      k.hidden > 1024 || k.ffn > 4096 || k.vocab < 1 || k.vocab > 65536 || (k.arch == 0 && (k.type_vocab < 1 || k.type_vocab > 4)) ||
       k.max_seqs < 1 || k.max_seq_len < 1 || (int64_t)k.max_seqs * k.max_seq_len > 32768 || k.max_pos < 1 ||
-      k.head < 0 || k.head > 2 || (k.head == MIMOSE_HEAD_MC && k.n_choices < 1) ||
+      (k.head == MIMOSE_HEAD_MC && k.n_choices < 1) ||
       (k.head == MIMOSE_HEAD_SEQCLS && (k.n_labels < 1 || k.n_labels > 32)) || k.world < 1 || k.rank < 0 ||
       k.rank >= k.world || k.bucket_den <= 0 || k.degree < 0 || k.degree > 2) {
     mimose_status s = bad("invalid model / sizing config");

@@ -22,7 +22,11 @@ enum Epi : int {
   EPI_GELU_BWD = 4,       // C(E) = acc * gelu'(aux(E))
   EPI_ACC_RES_F32 = 5,    // C(f32) = acc + res(f32)  (res may alias C)
   EPI_F32 = 6,            // C(f32) = acc ; split-K: C + z*split_stride
-  EPI_NONE = 7            // benchmark only: accumulator read from TMEM, nothing stored
+  EPI_NONE = 7,           // benchmark only: accumulator read from TMEM, nothing stored
+  EPI_BIAS_GELUT = 8,     // C(E) = u = acc + bias ; C2(E) = gelu_tanh(u)        (GPT-2)
+  EPI_GELUT_BWD = 9,      // C(E) = acc * gelu_tanh'(aux(E))
+  EPI_BIAS_DROP_RESF32 = 10,  // C(f32) = res(f32) + drop(acc + bias)  (pre-LN residual stream)
+  EPI_ACC_F32 = 11        // C(f32) += acc  (fixed-order accumulation across launches)
 };
 struct GemmArgs {
   int M = 0, N = 0, K = 0;
@@ -46,14 +50,14 @@ void splitk_reduce(const float* part, int splits, int64_t n, float* out, cudaStr
 // ----------------------------------------------------------- attention ----
 // qkv [B*S, 3H] (q | k | v, head-major columns), O [B*S, H], lse [B, h, S].
 void attn_fwd(DType dt, const void* qkv, const int32_t* lengths, void* O, float* lse,
-              int B, int S, int H, int h, Drop drop, cudaStream_t st);
+              int B, int S, int H, int h, Drop drop, cudaStream_t st, bool causal = false);
 // bf16 with head dim 64 and S <= 128 runs on tcgen05 unless disabled (tests).
 void set_attn_tc(bool on);
 bool attn_tc_enabled();
 // D [B,h,S] = rowsum(dO * O); dqkv [B*S, 3H].
 void attn_bwd(DType dt, const void* qkv, const void* O, const void* dO, const float* lse,
               const int32_t* lengths, float* Dbuf, void* dqkv, int B, int S, int H, int h,
-              Drop drop, cudaStream_t st);
+              Drop drop, cudaStream_t st, bool causal = false);
 
 // ----------------------------------------------------------- layernorm ----
 // y = LN(z) (y may be null: recompute with the output store gated off); st = (mu, rstd).
@@ -62,9 +66,12 @@ void ln_fwd(DType dt, const float* z, const void* g, const void* b, void* y, flo
             int T, int H, float eps, cudaStream_t st_);
 // dz = LN'(dy [* premask]); dt = dz * mask (if dt != null);
 // partials: pg, pb (dgamma, dbeta) and pbias (= colsum dt, if non-null), [NPART][H].
+// res (nullable, may alias dz): dz = LN'(dy) + res before the dropout/bias step.
 void ln_bwd(DType dt, const float* dy, Drop premask, const float* z, const float2* st,
             const void* g, float* dz, void* dtout, Drop mask, float* pg, float* pb,
-            float* pbias, int T, int H, cudaStream_t st_);
+            float* pbias, int T, int H, cudaStream_t st_, const float* res = nullptr);
+// out(E) = in(f32) * mask ; part [NPART][N] = column sums of the stored out
+void drop_cast_colsum(DType dt, const float* in, Drop mask, void* out, int T, int N, float* part, cudaStream_t st);
 // out[c] = sum_p part[p*ld + c], p = 0..NPART-1 (fixed order)
 void reduce_partials(const float* part, int64_t ld, int n, float* out, cudaStream_t st);
 // Up to three such reductions in one launch (p1/p2 may be null), `rows` partial rows.
@@ -82,7 +89,13 @@ void embed_fwd(DType dt, const int32_t* ids, const int32_t* tt, const void* Ww, 
 // key `skip` (the padding id: HF padding_idx semantics), are untouched.
 // X is clobbered (piece sums are written in place).  work: 4*T int32 + hist.
 void keyed_rowsum(const int32_t* keys, int key_bits, float* X, int T, int H, float* out,
-                  int32_t* work, int32_t* hist, int max_tiles, int skip, cudaStream_t st);
+                  int32_t* work, int32_t* hist, int max_tiles, int skip, cudaStream_t st,
+                  bool accumulate = false);
+// GPT-2 embedding: x1(f32) = drop(wte[ids] + wpe[pos_offset + s])
+void embed_fwd_pre(DType dt, const int32_t* ids, const void* Ww, const void* Wp, float* x1, int B, int S, int H,
+                   int pos_offset, Drop drop, cudaStream_t st);
+// dz0(f32) = dy * mask
+void drop_f32(const float* dy, Drop mask, float* out, int64_t n, cudaStream_t st);
 // dWt[k] = sum over tokens with token_type k of dz0 rows (fixed-order partials)
 void type_grad(const float* dz0, const int32_t* tt, int T, int H, int TV, float* part, float* dWt, cudaStream_t st);
 // dWp[pos_offset + s] = sum_b dz0[b*S + s]
@@ -105,6 +118,15 @@ void head_qa_fwd(DType dt, const void* y, int B, int S, int H, const void* Wq, c
 void head_qa_bwd(DType dt, const void* y, int B, int S, int H, const void* Wq, const float* logits,
                  const int32_t* lengths, const int32_t* labels, float* dlog, float* part,
                  float* dWq, float* dbq, float* dy, cudaStream_t st);
+
+// LM head (next-token CE over s < len-1).  logits: fp32 [nrows, ldv] of tokens
+// row0..row0+nrows; tokstat[t] = (lse, nll).
+void lm_ce_fwd(const float* logits, int64_t ldv, int V, int row0, int nrows, const int32_t* ids,
+               const int32_t* lengths, int S, float2* tokstat, cudaStream_t st);
+void lm_loss(const float2* tokstat, int T, const int32_t* lengths, int B, int S, float* loss, cudaStream_t st);
+// dlog(E) = valid ? (softmax - onehot) / n_valid : 0
+void lm_ce_bwd(DType dt, const float* logits, int64_t ldv, int V, int row0, int nrows, const int32_t* ids,
+               const int32_t* lengths, int B, int S, const float2* tokstat, void* dlog, cudaStream_t st);
 
 // ----------------------------------------------------------- optimizer ----
 // AdamW (torch semantics).  master == nullptr: fp32 mode, w is the master.

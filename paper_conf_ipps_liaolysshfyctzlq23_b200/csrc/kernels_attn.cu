@@ -19,9 +19,9 @@ static inline int cdiv(int64_t a, int64_t b) { return (int)((a + b - 1) / b); }
 
 // tcgen05 versions (kernels_attn_tc.cu): bf16, head dim 64, S <= 128
 bool attn_fwd_tc(const void* qkv, const int32_t* lengths, void* O, float* lse, int B, int S, int H, int h,
-                 Drop drop, cudaStream_t st);
+                 Drop drop, cudaStream_t st, bool causal);
 bool attn_bwd_tc(const void* qkv, const void* O, const void* dO, const float* lse, const int32_t* lengths,
-                 void* dqkv, int B, int S, int H, int h, Drop drop, cudaStream_t st);
+                 void* dqkv, int B, int S, int H, int h, Drop drop, cudaStream_t st, bool causal);
 
 static bool g_attn_tc = true;
 void set_attn_tc(bool on) { g_attn_tc = on; }
@@ -33,7 +33,7 @@ constexpr int BT = 32;  // backward tile (4 fp32 tiles must fit the 48 KB static
 template <typename E, int D>
 __global__ void __launch_bounds__(AT) k_attn_fwd(const E* __restrict__ qkv, const int32_t* __restrict__ lengths,
                                                  E* __restrict__ O, float* __restrict__ lse, int S, int H,
-                                                 int h, float scale, Drop drop) {
+                                                 int h, float scale, Drop drop, int causal) {
   __shared__ float Ks[AT][D + 1];
   __shared__ float Vs[AT][D + 1];
   const int bh = blockIdx.y, b = bh / h, hd = bh % h;
@@ -41,6 +41,7 @@ __global__ void __launch_bounds__(AT) k_attn_fwd(const E* __restrict__ qkv, cons
   const int len = lengths[b];
   const int64_t ld = 3 * (int64_t)H;
   const bool active = q < S;
+  const int kl = causal ? min(len, q + 1) : len;      // keys visible to this query
   float qv[D];
   const E* qrow = qkv + ((int64_t)b * S + (active ? q : 0)) * ld + hd * D;
 #pragma unroll
@@ -55,7 +56,7 @@ __global__ void __launch_bounds__(AT) k_attn_fwd(const E* __restrict__ qkv, cons
       Ks[r][c] = kk < len ? ldf(qkv + ((int64_t)b * S + kk) * ld + H + hd * D + c) : 0.f;
     }
     __syncthreads();
-    const int kend = min(AT, len - k0);
+    const int kend = min(AT, kl - k0);
     for (int j = 0; j < kend; ++j) {
       float s = 0.f;
 #pragma unroll
@@ -79,7 +80,7 @@ __global__ void __launch_bounds__(AT) k_attn_fwd(const E* __restrict__ qkv, cons
       Vs[r][c] = kk < len ? ldf(base + 2 * H) : 0.f;
     }
     __syncthreads();
-    const int kend = min(AT, len - k0);
+    const int kend = min(AT, kl - k0);
     for (int j = 0; j < kend; ++j) {
       float s = 0.f;
 #pragma unroll
@@ -97,16 +98,16 @@ __global__ void __launch_bounds__(AT) k_attn_fwd(const E* __restrict__ qkv, cons
 }
 
 void attn_fwd(DType dt, const void* qkv, const int32_t* lengths, void* O, float* lse, int B, int S, int H,
-              int h, Drop drop, cudaStream_t st) {
+              int h, Drop drop, cudaStream_t st, bool causal) {
   note_launch(1);
-  if (dt == DT_BF16 && attn_tc_enabled() && attn_fwd_tc(qkv, lengths, O, lse, B, S, H, h, drop, st)) return;
+  if (dt == DT_BF16 && attn_tc_enabled() && attn_fwd_tc(qkv, lengths, O, lse, B, S, H, h, drop, st, causal)) return;
   const int D = H / h;
   const float scale = 1.0f / sqrtf((float)D);
   dim3 grid(cdiv(S, AT), B * h);
   auto go = [&](auto* tag, auto dconst) {
     using E = std::remove_pointer_t<decltype(tag)>;
     constexpr int DD = decltype(dconst)::value;
-    k_attn_fwd<E, DD><<<grid, AT, 0, st>>>((const E*)qkv, lengths, (E*)O, lse, S, H, h, scale, drop);
+    k_attn_fwd<E, DD><<<grid, AT, 0, st>>>((const E*)qkv, lengths, (E*)O, lse, S, H, h, scale, drop, causal ? 1 : 0);
   };
   if (dt == DT_F32) {
     if (D == 32) go((float*)nullptr, std::integral_constant<int, 32>{});
@@ -137,7 +138,7 @@ template <typename E, int D>
 __global__ void __launch_bounds__(BT) k_attn_bwd_kv(const E* __restrict__ qkv, const E* __restrict__ dO,
                                                     const float* __restrict__ lse, const float* __restrict__ Dbuf,
                                                     const int32_t* __restrict__ lengths, E* __restrict__ dqkv,
-                                                    int S, int H, int h, float scale, Drop drop) {
+                                                    int S, int H, int h, float scale, Drop drop, int causal) {
   __shared__ float Qs[BT][D + 1];
   __shared__ float dOs[BT][D + 1];
   __shared__ float Kt[D][BT + 1];
@@ -177,6 +178,7 @@ __global__ void __launch_bounds__(BT) k_attn_bwd_kv(const E* __restrict__ qkv, c
     if (!keyvalid) continue;
     const int qend = min(BT, len - q0);
     for (int i = 0; i < qend; ++i) {
+      if (causal && q0 + i < j) continue;           // key j invisible to earlier queries
       float s = 0.f, dp = 0.f;
 #pragma unroll
       for (int c = 0; c < D; ++c) { s += Qs[i][c] * Kt[c][threadIdx.x]; dp += dOs[i][c] * Vt[c][threadIdx.x]; }
@@ -200,7 +202,7 @@ template <typename E, int D>
 __global__ void __launch_bounds__(BT) k_attn_bwd_q(const E* __restrict__ qkv, const E* __restrict__ dO,
                                                    const float* __restrict__ lse, const float* __restrict__ Dbuf,
                                                    const int32_t* __restrict__ lengths, E* __restrict__ dqkv,
-                                                   int S, int H, int h, float scale, Drop drop) {
+                                                   int S, int H, int h, float scale, Drop drop, int causal) {
   __shared__ float Qt[D][BT + 1];
   __shared__ float dOt[D][BT + 1];
   __shared__ float Ks[BT][D + 1];
@@ -234,7 +236,7 @@ __global__ void __launch_bounds__(BT) k_attn_bwd_q(const E* __restrict__ qkv, co
     }
     __syncthreads();
     if (!valid) continue;
-    const int kend = min(BT, len - k0);
+    const int kend = min(BT, (causal ? min(len, i + 1) : len) - k0);
     for (int jj = 0; jj < kend; ++jj) {
       float s = 0.f, dp = 0.f;
 #pragma unroll
@@ -255,9 +257,9 @@ __global__ void __launch_bounds__(BT) k_attn_bwd_q(const E* __restrict__ qkv, co
 
 void attn_bwd(DType dt, const void* qkv, const void* O, const void* dO, const float* lse,
               const int32_t* lengths, float* Dbuf, void* dqkv, int B, int S, int H, int h, Drop drop,
-              cudaStream_t st) {
+              cudaStream_t st, bool causal) {
   if (dt == DT_BF16 && attn_tc_enabled() &&
-      attn_bwd_tc(qkv, O, dO, lse, lengths, dqkv, B, S, H, h, drop, st)) {
+      attn_bwd_tc(qkv, O, dO, lse, lengths, dqkv, B, S, H, h, drop, st, causal)) {
     note_launch(1);
     return;
   }
@@ -270,9 +272,9 @@ void attn_bwd(DType dt, const void* qkv, const void* O, const void* dO, const fl
     constexpr int DD = decltype(dconst)::value;
     k_attn_dot<E><<<cdiv((int64_t)B * h * S, 8), 256, 0, st>>>((const E*)O, (const E*)dO, Dbuf, B, S, H, h);
     k_attn_bwd_kv<E, DD><<<grid, BT, 0, st>>>((const E*)qkv, (const E*)dO, lse, Dbuf, lengths, (E*)dqkv, S, H, h,
-                                             scale, drop);
+                                             scale, drop, causal ? 1 : 0);
     k_attn_bwd_q<E, DD><<<grid, BT, 0, st>>>((const E*)qkv, (const E*)dO, lse, Dbuf, lengths, (E*)dqkv, S, H, h,
-                                            scale, drop);
+                                            scale, drop, causal ? 1 : 0);
   };
   if (dt == DT_F32) {
     if (D == 32) go((float*)nullptr, std::integral_constant<int, 32>{});

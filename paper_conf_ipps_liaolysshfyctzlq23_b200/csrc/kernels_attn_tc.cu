@@ -30,6 +30,7 @@ constexpr int PT = AQ * AQ * 2;          // 32 KB: one [128 x 128] bf16 tile (2 
 
 struct AttnArgs {
   int S, H, h, B;
+  int causal;                  // GPT-2: key k visible to query q iff k <= q
   float scale;
   Drop drop;
   const int32_t* lengths;
@@ -99,16 +100,17 @@ __global__ void __launch_bounds__(128) k_attn_fwd_tc(const __grid_constant__ CUt
   mbar_wait(&bar[1], 0);
   __syncwarp();
   tc_fence_after();
-  // ---- softmax of row t over keys [0, len) ----
+  // ---- softmax of row t over keys [0, kl), kl = len (or min(len, t+1) causal) ----
   const uint32_t trow = tmem + ((uint32_t)(32 * warp) << 16);
+  const int kl = a.causal ? min(len, t + 1) : len;
   float m = -INFINITY, l = 0.f;
   for (int c = 0; c < nch; ++c) {
     float v[32];
     tmem_ld32(trow + 32 * c, v);                // every lane loads (.sync.aligned)
-    if (32 * c < len) {
+    if (32 * c < kl) {
 #pragma unroll
       for (int i = 0; i < 32; ++i) {
-        const float s = (32 * c + i < len) ? v[i] * a.scale : -INFINITY;
+        const float s = (32 * c + i < kl) ? v[i] * a.scale : -INFINITY;
         if (s > m) { l = l * __expf(m - s) + 1.f; m = s; } else { l += __expf(s - m); }
       }
     }
@@ -120,15 +122,15 @@ __global__ void __launch_bounds__(128) k_attn_fwd_tc(const __grid_constant__ CUt
   for (int c = 0; c < nch; ++c) {
     float v[32];
     tmem_ld32(trow + 32 * c, v);
-    if (32 * c < len && t < S) {
+    if (32 * c < kl && t < S) {
 #pragma unroll
       for (int j = 0; j < 8; ++j) {
         const int k = 32 * c + 4 * j;
-        const float4 f = (k < len) ? drop4_or(a.drop, ebase + k) : make_float4(0.f, 0.f, 0.f, 0.f);
+        const float4 f = (k < kl) ? drop4_or(a.drop, ebase + k) : make_float4(0.f, 0.f, 0.f, 0.f);
         const float ff[4] = {f.x, f.y, f.z, f.w};
 #pragma unroll
         for (int i = 0; i < 4; ++i)
-          v[4 * j + i] = (k + i < len) ? __expf(v[4 * j + i] * a.scale - L) * ff[i] : 0.f;
+          v[4 * j + i] = (k + i < kl) ? __expf(v[4 * j + i] * a.scale - L) * ff[i] : 0.f;
       }
     } else {
 #pragma unroll
@@ -237,22 +239,23 @@ __global__ void __launch_bounds__(128) k_attn_bwd_tc(const __grid_constant__ CUt
   tc_fence_after();
   const uint32_t trow = tmem + ((uint32_t)(32 * warp) << 16);
   const uint64_t ebase = (((uint64_t)b * a.h + hd) * S + (uint64_t)t) * S;
+  const int kl = a.causal ? min(len, t + 1) : len;
   // P~ overwrites V: wait until every thread is past the MMA (V is dead)
   for (int c = 0; c < nch; ++c) {
     float sv[32], dp[32];
     tmem_ld32(trow + 32 * c, sv);
     tmem_ld32(trow + 128 + 32 * c, dp);
-    const bool live = t < len && 32 * c < len;   // padded / foreign query rows contribute 0
+    const bool live = t < len && 32 * c < kl;    // padded / foreign query rows contribute 0
     if (live) {
 #pragma unroll
       for (int j = 0; j < 8; ++j) {
         const int k = 32 * c + 4 * j;
-        const float4 f = (k < len) ? drop4_or(a.drop, ebase + k) : make_float4(0.f, 0.f, 0.f, 0.f);
+        const float4 f = (k < kl) ? drop4_or(a.drop, ebase + k) : make_float4(0.f, 0.f, 0.f, 0.f);
         const float ff[4] = {f.x, f.y, f.z, f.w};
 #pragma unroll
         for (int i = 0; i < 4; ++i) {
           const int kk = k + i;
-          const float p = (kk < len) ? __expf(sv[4 * j + i] * a.scale - Lt) : 0.f;
+          const float p = (kk < kl) ? __expf(sv[4 * j + i] * a.scale - Lt) : 0.f;
           sv[4 * j + i] = p * ff[i];                                  // P~
           dp[4 * j + i] = p * (dp[4 * j + i] * ff[i] - Dt) * a.scale; // dS (scale folded)
         }
@@ -321,7 +324,7 @@ constexpr int BWD_SMEM = 5 * TILE + PT + 128;             // P~ reuses V
 bool attn_tc_ok(int S, int H, int h) { return S <= AQ && H / h == AD && H % 64 == 0; }
 
 bool attn_fwd_tc(const void* qkv, const int32_t* lengths, void* O, float* lse, int B, int S, int H, int h,
-                 Drop drop, cudaStream_t st) {
+                 Drop drop, cudaStream_t st, bool causal) {
   if (!attn_tc_ok(S, H, h)) return false;
   CUtensorMap tq;
   if (!tc_map_bf16(&tq, qkv, 3ull * H, (uint64_t)B * S, 3ull * H, 64, AQ)) return false;
@@ -330,13 +333,13 @@ bool attn_fwd_tc(const void* qkv, const int32_t* lengths, void* O, float* lse, i
   AttnArgs a{};
   a.S = S; a.H = H; a.h = h; a.B = B;
   a.scale = 1.0f / sqrtf((float)AD);
-  a.drop = drop; a.lengths = lengths; a.Oout = (__nv_bfloat16*)O; a.lse = lse;
+  a.drop = drop; a.lengths = lengths; a.Oout = (__nv_bfloat16*)O; a.lse = lse; a.causal = causal;
   k_attn_fwd_tc<<<B * h, 128, FWD_SMEM, st>>>(tq, a);
   return true;
 }
 
 bool attn_bwd_tc(const void* qkv, const void* O, const void* dO, const float* lse, const int32_t* lengths,
-                 void* dqkv, int B, int S, int H, int h, Drop drop, cudaStream_t st) {
+                 void* dqkv, int B, int S, int H, int h, Drop drop, cudaStream_t st, bool causal) {
   if (!attn_tc_ok(S, H, h)) return false;
   CUtensorMap tq, tdo;
   if (!tc_map_bf16(&tq, qkv, 3ull * H, (uint64_t)B * S, 3ull * H, 64, AQ)) return false;
@@ -347,7 +350,7 @@ bool attn_bwd_tc(const void* qkv, const void* O, const void* dO, const float* ls
   a.S = S; a.H = H; a.h = h; a.B = B;
   a.scale = 1.0f / sqrtf((float)AD);
   a.drop = drop; a.lengths = lengths; a.O = (const __nv_bfloat16*)O; a.dO = (const __nv_bfloat16*)dO;
-  a.lse_in = lse; a.dqkv = (__nv_bfloat16*)dqkv;
+  a.lse_in = lse; a.dqkv = (__nv_bfloat16*)dqkv; a.causal = causal;
   k_attn_bwd_tc<<<B * h, 128, BWD_SMEM, st>>>(tq, tdo, a);
   return true;
 }

@@ -114,7 +114,7 @@ __global__ void __launch_bounds__(256) k_ln_bwd(const float* dy, Drop premask, c
                                                 const float2* __restrict__ st, const E* __restrict__ g,
                                                 float* dz, E* __restrict__ dtout, Drop mask,
                                                 float* __restrict__ pg, float* __restrict__ pb,
-                                                float* __restrict__ pbias, int T, int H) {
+                                                float* __restrict__ pbias, int T, int H, const float* res) {
   extern __shared__ float sm[];
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const int nch = H >> 3;
@@ -165,6 +165,12 @@ __global__ void __launch_bounds__(256) k_ln_bwd(const float* dy, Drop premask, c
           ag[k][i] += dyv[k][i] * xh[k][i];
           ab[k][i] += dyv[k][i];
         }
+        if (res) {                                    // pre-LN: residual gradient joins here
+          float rv[8];
+          ld8(res + (int64_t)row * H + 8 * j, rv);
+#pragma unroll
+          for (int i = 0; i < 8; ++i) o[i] += rv[i];
+        }
         st8(dz + (int64_t)row * H + 8 * j, o);
         if (dtout) {
           float f[8];
@@ -204,7 +210,7 @@ __global__ void __launch_bounds__(256) k_ln_bwd(const float* dy, Drop premask, c
 
 void ln_bwd(DType dt, const float* dy, Drop premask, const float* z, const float2* st, const void* g,
             float* dz, void* dtout, Drop mask, float* pg, float* pb, float* pbias, int T, int H,
-            cudaStream_t s) {
+            cudaStream_t s, const float* res) {
   const size_t smem = (size_t)8 * 3 * H * sizeof(float);
   note_launch(1);
   dispatch(dt, [&](auto* tag) {
@@ -215,7 +221,7 @@ void ln_bwd(DType dt, const float* dy, Drop premask, const float* z, const float
       attr = true;
     }
     k_ln_bwd<E><<<NPART, 256, smem, s>>>(dy, premask, z, st, (const E*)g, dz, (E*)dtout,
-                                         mask, pg, pb, pbias, T, H);
+                                         mask, pg, pb, pbias, T, H, res);
   });
 }
 
@@ -295,6 +301,48 @@ void colsum(DType dt, const void* X, int T, int N, float* part, cudaStream_t s) 
     using E = std::remove_pointer_t<decltype(tag)>;
     k_colsum<E><<<dim3(cdiv(N, 2048), NPART), 256, 0, s>>>((const E*)X, T, N, part);
   });
+}
+
+// out(E) = in(f32) * mask, with column-sum partials of the stored values.
+template <typename E>
+__global__ void __launch_bounds__(256) k_drop_cast_colsum(const float* __restrict__ in, Drop mask, E* __restrict__ out,
+                                                          int T, int N, float* __restrict__ part) {
+  const int c = blockIdx.x * 2048 + threadIdx.x * 8;
+  if (c >= N) return;
+  float acc[8] = {0.f, 0.f, 0.f, 0.f, 0.f, 0.f, 0.f, 0.f};
+  for (int r = blockIdx.y; r < T; r += NPART) {
+    float v[8], f[8];
+    ld8(in + (int64_t)r * N + c, v);
+    drop8(mask, (uint64_t)r * N + c, f);
+#pragma unroll
+    for (int i = 0; i < 8; ++i) v[i] = rnd(v[i] * f[i], out);
+    st8(out + (int64_t)r * N + c, v);
+#pragma unroll
+    for (int i = 0; i < 8; ++i) acc[i] += v[i];
+  }
+  st8(part + (int64_t)blockIdx.y * N + c, acc);
+}
+void drop_cast_colsum(DType dt, const float* in, Drop mask, void* out, int T, int N, float* part, cudaStream_t s) {
+  note_launch(1);
+  dispatch(dt, [&](auto* tag) {
+    using E = std::remove_pointer_t<decltype(tag)>;
+    k_drop_cast_colsum<E><<<dim3(cdiv(N, 2048), NPART), 256, 0, s>>>(in, mask, (E*)out, T, N, part);
+  });
+}
+
+__global__ void k_drop_f32(const float* __restrict__ in, Drop mask, float* __restrict__ out, int64_t n) {
+  for (int64_t i = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) * 8; i < n; i += (int64_t)gridDim.x * blockDim.x * 8) {
+    float v[8], f[8];
+    ld8(in + i, v);
+    drop8(mask, (uint64_t)i, f);
+#pragma unroll
+    for (int k = 0; k < 8; ++k) v[k] *= f[k];
+    st8(out + i, v);
+  }
+}
+void drop_f32(const float* in, Drop mask, float* out, int64_t n, cudaStream_t s) {
+  note_launch(1);
+  k_drop_f32<<<592, 256, 0, s>>>(in, mask, out, n);
 }
 
 // ============================================================== embedding ===
@@ -384,6 +432,31 @@ void type_grad(const float* dz0, const int32_t* tt, int T, int H, int TV, float*
   note_launch(1);
   k_type_part<<<NPART, 256, 0, s>>>(dz0, tt, T, H, TV, part);
   reduce_partials(part, (int64_t)TV * H, TV * H, dWt, s);
+}
+
+template <typename E>
+__global__ void k_embed_fwd_pre(const int32_t* __restrict__ ids, const E* __restrict__ Ww, const E* __restrict__ Wp,
+                                float* __restrict__ x1, int T, int S, int H, int pos_offset, Drop drop) {
+  const int64_t i = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) * 8;
+  if (i >= (int64_t)T * H) return;
+  const int t = (int)(i / H), c = (int)(i % H);
+  float w[8], p[8], f[8];
+  ld8(Ww + (int64_t)ids[t] * H + c, w);
+  ld8(Wp + (int64_t)(pos_offset + t % S) * H + c, p);
+  drop8(drop, (uint64_t)i, f);
+#pragma unroll
+  for (int k = 0; k < 8; ++k) w[k] = (w[k] + p[k]) * f[k];
+  st8(x1 + i, w);
+}
+void embed_fwd_pre(DType dt, const int32_t* ids, const void* Ww, const void* Wp, float* x1, int B, int S, int H,
+                   int pos_offset, Drop drop, cudaStream_t s) {
+  note_launch(1);
+  const int T = B * S;
+  dispatch(dt, [&](auto* tag) {
+    using E = std::remove_pointer_t<decltype(tag)>;
+    k_embed_fwd_pre<E><<<cdiv((int64_t)T * H / 8, 256), 256, 0, s>>>(ids, (const E*)Ww, (const E*)Wp, x1, T, S, H,
+                                                                     pos_offset, drop);
+  });
 }
 
 __global__ void k_pos_grad(const float* __restrict__ dz0, int B, int S, int H, int pos_offset,
@@ -509,7 +582,7 @@ __global__ void __launch_bounds__(256) k_piece_sum(const int32_t* __restrict__ k
 // segment sums: warp per sorted position that starts a run of equal keys.
 __global__ void __launch_bounds__(256) k_segment_sum(const int32_t* __restrict__ keys, const int32_t* __restrict__ tok,
                                                      const float* __restrict__ X, int T, int H, float* __restrict__ out,
-                                                     int skip) {
+                                                     int skip, int accumulate) {
   const int r = (blockIdx.x * blockDim.x + threadIdx.x) >> 5, lane = threadIdx.x & 31;
   if (r >= T) return;
   const int key = keys[r];
@@ -535,11 +608,14 @@ __global__ void __launch_bounds__(256) k_segment_sum(const int32_t* __restrict__
   }
 #pragma unroll
   for (int j = 0; j < 32; ++j)
-    if (j < nv) out[(int64_t)key * H + lane + 32 * j] = acc[j];
+    if (j < nv) {
+      float* o = out + (int64_t)key * H + lane + 32 * j;
+      *o = accumulate ? *o + acc[j] : acc[j];     // one writer per key: deterministic
+    }
 }
 
 void keyed_rowsum(const int32_t* keys, int key_bits, float* X, int T, int H, float* out,
-                  int32_t* work, int32_t* hist, int max_tiles, int skip, cudaStream_t s) {
+                  int32_t* work, int32_t* hist, int max_tiles, int skip, cudaStream_t s, bool accumulate) {
   const int ntiles = cdiv(T, 1024);
   int32_t *kA = work, *vA = work + T, *kB = work + 2 * T, *vB = work + 3 * T;
   const int passes = key_bits <= 8 ? 1 : 2;
@@ -557,7 +633,7 @@ void keyed_rowsum(const int32_t* keys, int key_bits, float* X, int T, int H, flo
   (void)max_tiles;
   note_launch(3 * passes + 2);
   k_piece_sum<<<cdiv(cdiv(T, 32), 8), 256, 0, s>>>(kin, vin, X, T, H, skip);
-  k_segment_sum<<<cdiv(T, 8), 256, 0, s>>>(kin, vin, X, T, H, out, skip);
+  k_segment_sum<<<cdiv(T, 8), 256, 0, s>>>(kin, vin, X, T, H, out, skip, accumulate ? 1 : 0);
 }
 
 // ================================================================== heads ===
@@ -798,6 +874,102 @@ void head_qa_bwd(DType dt, const void* y, int B, int S, int H, const void* Wq, c
   });
   reduce_partials(part, 2 * H + 2, 2 * H, dWq, s);
   reduce_partials(part + 2 * H, 2 * H + 2, 2, dbq, s);
+}
+
+// ================================================================ LM head ===
+// Block (1024 threads) per token row of the chunk; fixed-order block reductions.
+MDEV float block_reduce(float v, bool is_max, float* sh) {
+  v = is_max ? warp_max(v) : warp_sum(v);
+  const int w = threadIdx.x >> 5, l = threadIdx.x & 31;
+  __syncthreads();
+  if (l == 0) sh[w] = v;
+  __syncthreads();
+  float r = is_max ? -INFINITY : 0.f;
+  if (threadIdx.x < 32) {
+    r = threadIdx.x < (int)(blockDim.x >> 5) ? sh[threadIdx.x] : (is_max ? -INFINITY : 0.f);
+    r = is_max ? warp_max(r) : warp_sum(r);
+    if (threadIdx.x == 0) sh[32] = r;
+  }
+  __syncthreads();
+  return sh[32];
+}
+
+MDEV bool lm_target(const int32_t* ids, const int32_t* lengths, int S, int t, int& tgt) {
+  const int b = t / S, s = t % S;
+  if (s + 1 >= lengths[b]) return false;
+  tgt = ids[t + 1];
+  return true;
+}
+
+__global__ void __launch_bounds__(1024) k_lm_ce_fwd(const float* __restrict__ logits, int64_t ldv, int V, int row0,
+                                                    const int32_t* __restrict__ ids, const int32_t* __restrict__ lengths,
+                                                    int S, float2* __restrict__ tokstat) {
+  __shared__ float sh[33];
+  const int r = blockIdx.x, t = row0 + r;
+  const float* lr = logits + (int64_t)r * ldv;
+  float m = -INFINITY;
+  for (int v = threadIdx.x; v < V; v += blockDim.x) m = fmaxf(m, lr[v]);
+  m = block_reduce(m, true, sh);
+  float z = 0.f;
+  for (int v = threadIdx.x; v < V; v += blockDim.x) z += __expf(lr[v] - m);
+  z = block_reduce(z, false, sh);
+  if (threadIdx.x == 0) {
+    const float lse = m + __logf(z);
+    int tgt;
+    const float nll = lm_target(ids, lengths, S, t, tgt) ? lse - lr[tgt] : 0.f;
+    tokstat[t] = make_float2(lse, nll);
+  }
+}
+void lm_ce_fwd(const float* logits, int64_t ldv, int V, int row0, int nrows, const int32_t* ids,
+               const int32_t* lengths, int S, float2* tokstat, cudaStream_t s) {
+  note_launch(1);
+  k_lm_ce_fwd<<<nrows, 1024, 0, s>>>(logits, ldv, V, row0, ids, lengths, S, tokstat);
+}
+
+__global__ void __launch_bounds__(1024) k_lm_loss(const float2* __restrict__ tokstat, int T,
+                                                  const int32_t* __restrict__ lengths, int B, float* __restrict__ loss) {
+  __shared__ float sh[33];
+  float a = 0.f;
+  for (int t = threadIdx.x; t < T; t += blockDim.x) a += tokstat[t].y;
+  a = block_reduce(a, false, sh);
+  float nv = 0.f;
+  for (int b = threadIdx.x; b < B; b += blockDim.x) nv += (float)max(lengths[b] - 1, 0);
+  nv = block_reduce(nv, false, sh);
+  if (threadIdx.x == 0) *loss = a / fmaxf(nv, 1.f);
+}
+void lm_loss(const float2* tokstat, int T, const int32_t* lengths, int B, int S, float* loss, cudaStream_t s) {
+  (void)S;
+  note_launch(1);
+  k_lm_loss<<<1, 1024, 0, s>>>(tokstat, T, lengths, B, loss);
+}
+
+template <typename E>
+__global__ void __launch_bounds__(256) k_lm_ce_bwd(const float* __restrict__ logits, int64_t ldv, int V, int row0,
+                                                   const int32_t* __restrict__ ids, const int32_t* __restrict__ lengths,
+                                                   int B, int S, const float2* __restrict__ tokstat, E* __restrict__ dlog) {
+  __shared__ float inv_n;
+  if (threadIdx.x == 0) {
+    int nv = 0;
+    for (int b = 0; b < B; ++b) nv += max(lengths[b] - 1, 0);
+    inv_n = 1.0f / (float)max(nv, 1);
+  }
+  __syncthreads();
+  const int r = blockIdx.x, t = row0 + r;
+  int tgt = -1;
+  const bool valid = lm_target(ids, lengths, S, t, tgt);
+  const float lse = tokstat[t].x;
+  const float* lr = logits + (int64_t)r * ldv;
+  E* dr = dlog + (int64_t)r * ldv;
+  for (int v = threadIdx.x; v < V; v += blockDim.x)
+    stf(dr + v, valid ? (__expf(lr[v] - lse) - (v == tgt ? 1.f : 0.f)) * inv_n : 0.f);
+}
+void lm_ce_bwd(DType dt, const float* logits, int64_t ldv, int V, int row0, int nrows, const int32_t* ids,
+               const int32_t* lengths, int B, int S, const float2* tokstat, void* dlog, cudaStream_t s) {
+  note_launch(1);
+  dispatch(dt, [&](auto* tag) {
+    using E = std::remove_pointer_t<decltype(tag)>;
+    k_lm_ce_bwd<E><<<nrows, 256, 0, s>>>(logits, ldv, V, row0, ids, lengths, B, S, tokstat, (E*)dlog);
+  });
 }
 
 // ============================================================== optimizer ===

@@ -75,6 +75,10 @@ static void launch_simt(Epi epi, const GemmArgs& g, cudaStream_t st) {
     case EPI_BIAS_DROP_RES: k_gemm_simt<E, EPI_BIAS_DROP_RES><<<grid, 256, 0, st>>>(g); break;
     case EPI_GELU_BWD: k_gemm_simt<E, EPI_GELU_BWD><<<grid, 256, 0, st>>>(g); break;
     case EPI_ACC_RES_F32: k_gemm_simt<E, EPI_ACC_RES_F32><<<grid, 256, 0, st>>>(g); break;
+    case EPI_BIAS_GELUT: k_gemm_simt<E, EPI_BIAS_GELUT><<<grid, 256, 0, st>>>(g); break;
+    case EPI_GELUT_BWD: k_gemm_simt<E, EPI_GELUT_BWD><<<grid, 256, 0, st>>>(g); break;
+    case EPI_BIAS_DROP_RESF32: k_gemm_simt<E, EPI_BIAS_DROP_RESF32><<<grid, 256, 0, st>>>(g); break;
+    case EPI_ACC_F32: k_gemm_simt<E, EPI_ACC_F32><<<grid, 256, 0, st>>>(g); break;
     default: k_gemm_simt<E, EPI_F32><<<grid, 256, 0, st>>>(g); break;
   }
 }

@@ -102,6 +102,10 @@ MDEV void epi_row32(const GemmArgs& g, int m, int n, float (&v)[32], int z = -1)
 #pragma unroll
     for (int i = 0; i < 32; ++i) t += v[i];
     if (t == 1234.5f) ((float*)g.C)[o] = t;
+  } else if constexpr (EPI == EPI_BIAS_GELUT || EPI == EPI_GELUT_BWD || EPI == EPI_BIAS_DROP_RESF32 ||
+                       EPI == EPI_ACC_F32) {
+#pragma unroll
+    for (int i = 0; i < 32; ++i) epilogue<__nv_bfloat16, EPI>(g, m, n + i, v[i], z);
   } else {
     float4* out = (float4*)((float*)g.C + (int64_t)z * g.split_stride + o);
 #pragma unroll
@@ -216,7 +220,8 @@ struct EpiIn {
 };
 template <int EPI>
 MDEV void epi_load(const GemmArgs& g, int m, int n, bool live, EpiIn& in) {
-  if constexpr (EPI == EPI_BIAS || EPI == EPI_BIAS_GELU || EPI == EPI_BIAS_DROP_RES) {
+  if constexpr (EPI == EPI_BIAS || EPI == EPI_BIAS_GELU || EPI == EPI_BIAS_DROP_RES || EPI == EPI_BIAS_GELUT ||
+                EPI == EPI_BIAS_DROP_RESF32) {
     const uint4* p = (const uint4*)((const __nv_bfloat16*)g.bias + n);
 #pragma unroll
     for (int i = 0; i < 4; ++i) in.b[i] = p[i];
@@ -226,11 +231,11 @@ MDEV void epi_load(const GemmArgs& g, int m, int n, bool live, EpiIn& in) {
     const uint4* p = (const uint4*)((const __nv_bfloat16*)g.res + (int64_t)m * g.ldr + n);
 #pragma unroll
     for (int i = 0; i < 4; ++i) in.x[i] = p[i];
-  } else if constexpr (EPI == EPI_GELU_BWD) {
+  } else if constexpr (EPI == EPI_GELU_BWD || EPI == EPI_GELUT_BWD) {
     const uint4* p = (const uint4*)((const __nv_bfloat16*)g.aux + (int64_t)m * g.ldx + n);
 #pragma unroll
     for (int i = 0; i < 4; ++i) in.x[i] = p[i];
-  } else if constexpr (EPI == EPI_ACC_RES_F32) {
+  } else if constexpr (EPI == EPI_ACC_RES_F32 || EPI == EPI_BIAS_DROP_RESF32) {
     const uint4* p = (const uint4*)((const float*)g.res + (int64_t)m * g.ldr + n);
 #pragma unroll
     for (int i = 0; i < 8; ++i) in.x[i] = p[i];
@@ -291,6 +296,47 @@ MDEV void epi_frag32_in(const GemmArgs& g, int m_base, int n, float (&v)[32], in
       }
     }
     stage_store_f32(stg, v, (float*)g.C + (int64_t)m_base * g.ldc + n, g.ldc, rows_valid, lane);
+  } else if constexpr (EPI == EPI_BIAS_GELUT || EPI == EPI_BIAS_DROP_RESF32) {
+    float b[32];
+#pragma unroll
+    for (int i = 0; i < 4; ++i) unpack8(in.b[i], b + 8 * i);
+#pragma unroll
+    for (int i = 0; i < 32; ++i) v[i] += b[i];
+    if constexpr (EPI == EPI_BIAS_GELUT) {
+      stage_store_bf16(stg, v, (E*)g.C + (int64_t)m_base * g.ldc + n, g.ldc, rows_valid, lane);
+#pragma unroll
+      for (int i = 0; i < 32; ++i) v[i] = gelu_tanh_f(__bfloat162float(__float2bfloat16_rn(v[i])));
+      stage_store_bf16(stg, v, (E*)g.C2 + (int64_t)m_base * g.ldc + n, g.ldc, rows_valid, lane);
+    } else {
+      const float* r = (const float*)in.x;
+      const int64_t o = (int64_t)m * g.ldc + n;
+#pragma unroll
+      for (int q = 0; q < 8; ++q) {
+        const float4 f = live ? drop_factor4(g.drop, (uint64_t)(o + 4 * q) >> 2) : make_float4(0.f, 0.f, 0.f, 0.f);
+        v[4 * q + 0] = (live ? r[4 * q + 0] : 0.f) + v[4 * q + 0] * f.x;
+        v[4 * q + 1] = (live ? r[4 * q + 1] : 0.f) + v[4 * q + 1] * f.y;
+        v[4 * q + 2] = (live ? r[4 * q + 2] : 0.f) + v[4 * q + 2] * f.z;
+        v[4 * q + 3] = (live ? r[4 * q + 3] : 0.f) + v[4 * q + 3] * f.w;
+      }
+      stage_store_f32(stg, v, (float*)g.C + (int64_t)m_base * g.ldc + n, g.ldc, rows_valid, lane);
+    }
+  } else if constexpr (EPI == EPI_GELUT_BWD) {
+    float u[32];
+#pragma unroll
+    for (int i = 0; i < 4; ++i) unpack8(in.x[i], u + 8 * i);
+#pragma unroll
+    for (int i = 0; i < 32; ++i) v[i] = live ? v[i] * gelu_tanh_grad_f(u[i]) : 0.f;
+    stage_store_bf16(stg, v, (E*)g.C + (int64_t)m_base * g.ldc + n, g.ldc, rows_valid, lane);
+  } else if constexpr (EPI == EPI_ACC_F32) {
+    if (live) {
+      float* out = (float*)g.C + (int64_t)m * g.ldc + n;
+#pragma unroll
+      for (int q = 0; q < 8; ++q) {
+        float4 a = ((float4*)out)[q];
+        a.x += v[4 * q]; a.y += v[4 * q + 1]; a.z += v[4 * q + 2]; a.w += v[4 * q + 3];
+        ((float4*)out)[q] = a;
+      }
+    }
   } else if constexpr (EPI == EPI_NONE) {
     float t = 0.f;
 #pragma unroll
@@ -550,7 +596,8 @@ __global__ void __launch_bounds__(TP_THREADS, 1)
           const char* pa = nullptr;
           int bytes = 0;
           const int ncol = 32 * (c_end - c_beg);
-          if constexpr (EPI == EPI_GELU_BWD) { pa = (const char*)((const __nv_bfloat16*)g.aux + (int64_t)m * g.ldx + nb); bytes = 2 * ncol; }
+          if constexpr (EPI == EPI_GELU_BWD || EPI == EPI_GELUT_BWD) { pa = (const char*)((const __nv_bfloat16*)g.aux + (int64_t)m * g.ldx + nb); bytes = 2 * ncol; }
+          if constexpr (EPI == EPI_BIAS_DROP_RESF32) { pa = (const char*)((const float*)g.res + (int64_t)m * g.ldr + nb); bytes = 4 * ncol; }
           if constexpr (EPI == EPI_BIAS_DROP_RES) { pa = (const char*)((const __nv_bfloat16*)g.res + (int64_t)m * g.ldr + nb); bytes = 2 * ncol; }
           if constexpr (EPI == EPI_ACC_RES_F32) { pa = (const char*)((const float*)g.res + (int64_t)m * g.ldr + nb); bytes = 4 * ncol; }
           for (int o = 0; o < bytes; o += 128) asm volatile("prefetch.global.L2 [%0];" ::"l"(pa + o));
@@ -899,6 +946,10 @@ static void dispatch_tcp(Epi epi, const CUtensorMap& ma, const CUtensorMap& mb, 
     case EPI_GELU_BWD: launch_tcp<BN, EPI_GELU_BWD>(ma, mb, a, st); break;
     case EPI_ACC_RES_F32: launch_tcp<BN, EPI_ACC_RES_F32>(ma, mb, a, st); break;
     case EPI_NONE: launch_tcp<BN, EPI_NONE>(ma, mb, a, st); break;
+    case EPI_BIAS_GELUT: launch_tcp<BN, EPI_BIAS_GELUT>(ma, mb, a, st); break;
+    case EPI_GELUT_BWD: launch_tcp<BN, EPI_GELUT_BWD>(ma, mb, a, st); break;
+    case EPI_BIAS_DROP_RESF32: launch_tcp<BN, EPI_BIAS_DROP_RESF32>(ma, mb, a, st); break;
+    case EPI_ACC_F32: launch_tcp<BN, EPI_ACC_F32>(ma, mb, a, st); break;
     default: launch_tcp<BN, EPI_F32>(ma, mb, a, st); break;
   }
 }
@@ -941,6 +992,10 @@ static void dispatch_tc2(Epi epi, const CUtensorMap& ma, const CUtensorMap& mb, 
     case EPI_GELU_BWD: launch_tc2<BN, EPI_GELU_BWD>(ma, mb, a, st); break;
     case EPI_ACC_RES_F32: launch_tc2<BN, EPI_ACC_RES_F32>(ma, mb, a, st); break;
     case EPI_NONE: launch_tc2<BN, EPI_NONE>(ma, mb, a, st); break;
+    case EPI_BIAS_GELUT: launch_tc2<BN, EPI_BIAS_GELUT>(ma, mb, a, st); break;
+    case EPI_GELUT_BWD: launch_tc2<BN, EPI_GELUT_BWD>(ma, mb, a, st); break;
+    case EPI_BIAS_DROP_RESF32: launch_tc2<BN, EPI_BIAS_DROP_RESF32>(ma, mb, a, st); break;
+    case EPI_ACC_F32: launch_tc2<BN, EPI_ACC_F32>(ma, mb, a, st); break;
     default: launch_tc2<BN, EPI_F32>(ma, mb, a, st); break;
   }
 }
@@ -1019,6 +1074,10 @@ bool gemm_tc(Epi epi, const GemmArgs& g, cudaStream_t st) {
     case EPI_GELU_BWD: launch_tc<BN1, EPI_GELU_BWD>(ma, mb, a, grid, st); break;
     case EPI_ACC_RES_F32: launch_tc<BN1, EPI_ACC_RES_F32>(ma, mb, a, grid, st); break;
     case EPI_NONE: launch_tc<BN1, EPI_NONE>(ma, mb, a, grid, st); break;
+    case EPI_BIAS_GELUT: launch_tc<BN1, EPI_BIAS_GELUT>(ma, mb, a, grid, st); break;
+    case EPI_GELUT_BWD: launch_tc<BN1, EPI_GELUT_BWD>(ma, mb, a, grid, st); break;
+    case EPI_BIAS_DROP_RESF32: launch_tc<BN1, EPI_BIAS_DROP_RESF32>(ma, mb, a, grid, st); break;
+    case EPI_ACC_F32: launch_tc<BN1, EPI_ACC_F32>(ma, mb, a, grid, st); break;
     default: launch_tc<BN1, EPI_F32>(ma, mb, a, grid, st); break;
   }
   return true;

@@ -21,9 +21,11 @@ from typing import Dict, List, Tuple
 import numpy as np
 
 ARCH_POST_LN = 0     # BERT / RoBERTa post-LN encoder
+ARCH_PRE_LN = 1      # GPT-2 pre-LN causal decoder stack
 HEAD_SEQCLS = 0      # pooler -> dropout -> linear(n_labels) -> CE
 HEAD_MC = 1          # pooler -> dropout -> linear(1) -> [B_q, n_choices] -> CE
 HEAD_QA = 2          # linear(2) on every token -> start/end CE
+HEAD_LM = 3          # final LN -> tied vocabulary projection -> next-token CE
 
 
 @dataclasses.dataclass(frozen=True)
@@ -54,6 +56,11 @@ class ModelConfig:
     sep_id: int
     pad_id: int
     first_tok: int
+    arch: int = ARCH_POST_LN
+
+    @property
+    def causal(self) -> bool:
+        return self.arch == ARCH_PRE_LN
 
     @property
     def head_dim(self) -> int:
@@ -65,6 +72,8 @@ class ModelConfig:
             return self.n_labels
         if self.head == HEAD_MC:
             return 1
+        if self.head == HEAD_LM:
+            return self.vocab
         return 2
 
     @property
@@ -81,6 +90,8 @@ class ModelConfig:
             return self.n_seqs // self.n_choices
         if self.head == HEAD_QA:
             return 2 * self.n_seqs
+        if self.head == HEAD_LM:
+            return 0                      # targets are the next input tokens
         return self.n_seqs
 
     @property
@@ -105,6 +116,12 @@ CONFIGS: Dict[str, ModelConfig] = {
     "roberta-large": ModelConfig("roberta-large", 3, 24, 1024, 16, 4096, 50265, 514, 1, 2,
                                  HEAD_MC, 4, 2, "bf16", 1e-5, 0.1, 64, 64, 512, 8, 0.5,
                                  0, 2, 1, 3),
+    # configs[4]: GPT-2 medium, causal pre-LN, seq 256-1024, budget 40%, 8 sequences
+    # per GPU (batch not given in BASELINE; chosen).  No special tokens but the
+    # end-of-text id 50256, used as the pad id.
+    "gpt2-medium": ModelConfig("gpt2-medium", 4, 24, 1024, 16, 4096, 50257, 1024, 0, 0,
+                               HEAD_LM, 1, 2, "bf16", 1e-5, 0.1, 8, 256, 1024, 8, 0.4,
+                               50256, 50256, 50256, 0, ARCH_PRE_LN),
 }
 
 
@@ -120,6 +137,21 @@ def small_config(base: str, **over) -> ModelConfig:
 def param_spec(cfg: ModelConfig) -> List[Tuple[str, Tuple[int, ...]]]:
     H, F, V = cfg.hidden, cfg.ffn, cfg.vocab
     P = cfg.max_pos
+    if cfg.arch == ARCH_PRE_LN:
+        # GPT-2: wte (tied with the LM head), wpe; pre-LN layers; final LN
+        spec = [("emb.word", (V, H)), ("emb.pos", (P, H))]
+        for l in range(cfg.n_layers):
+            p = f"layer{l}."
+            spec += [
+                (p + "ln1.g", (H,)), (p + "ln1.b", (H,)),
+                (p + "qkv.w", (3 * H, H)), (p + "qkv.b", (3 * H,)),
+                (p + "o.w", (H, H)), (p + "o.b", (H,)),
+                (p + "ln2.g", (H,)), (p + "ln2.b", (H,)),
+                (p + "f1.w", (F, H)), (p + "f1.b", (F,)),
+                (p + "f2.w", (H, F)), (p + "f2.b", (H,)),
+            ]
+        spec += [("lnf.g", (H,)), ("lnf.b", (H,))]
+        return spec
     spec: List[Tuple[str, Tuple[int, ...]]] = [
         ("emb.word", (V, H)), ("emb.pos", (P, H)), ("emb.type", (cfg.type_vocab, H)),
         ("emb.ln.g", (H,)), ("emb.ln.b", (H,)),
@@ -155,7 +187,7 @@ def init_params(cfg: ModelConfig, parity: bool = False, seed: int | None = None)
         leaf = name.rsplit(".", 1)[-1]
         if leaf == "g":
             v = rng.uniform(0.5, 1.5, shape) if parity else np.ones(shape)
-        elif leaf == "b" and ".ln" in name:
+        elif leaf == "b" and name.split(".")[-2].startswith("ln"):
             v = rng.normal(0.0, 0.1, shape) if parity else np.zeros(shape)
         elif leaf == "b":
             v = rng.normal(0.0, 0.02, shape) if parity else np.zeros(shape)
@@ -242,12 +274,17 @@ def make_batch(cfg: ModelConfig, longest: int, seed: int, n_seqs: int | None = N
     tt = np.zeros((B, S), np.int32)
     for b in range(B):
         n = int(lens[b])
+        if cfg.arch == ARCH_PRE_LN:                 # GPT-2: plain text tokens
+            ids[b, :n] = rng.integers(cfg.first_tok, cfg.vocab - 1, size=n)
+            continue
         ids[b, :n] = rng.integers(cfg.first_tok, cfg.vocab, size=n)
         ids[b, 0] = cfg.cls_id
         ids[b, n - 1] = cfg.sep_id
         if cfg.type_vocab > 1:
             tt[b, n // 2:n] = 1
-    if cfg.head == HEAD_SEQCLS:
+    if cfg.head == HEAD_LM:
+        labels = np.zeros(0, np.int32)
+    elif cfg.head == HEAD_SEQCLS:
         labels = rng.integers(0, cfg.n_labels, size=B).astype(np.int32)
     elif cfg.head == HEAD_MC:
         labels = rng.integers(0, cfg.n_choices, size=B // cfg.n_choices).astype(np.int32)

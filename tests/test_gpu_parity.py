@@ -95,6 +95,17 @@ CASES = {
                                max_pos=80, n_seqs=3, seq_lo=20, seq_hi=70, pad=1, dtype="fp32"),
     "mc-roberta-bf16": wl.small_config("roberta-large", n_layers=2, hidden=128, heads=2, ffn=256,
                                        vocab=700, max_pos=66, n_seqs=8, seq_lo=10, seq_hi=64, pad=8),
+    # GPT-2 (pre-LN, causal, tied LM head, chunked CE): tcgen05 attention (S <= 128),
+    # SIMT causal attention (S > 128), fp32
+    "lm-gpt2-bf16": wl.small_config("gpt2-medium", n_layers=2, hidden=128, heads=2, ffn=256, vocab=600,
+                                    max_pos=128, n_seqs=3, seq_lo=40, seq_hi=120, pad=8, pad_id=599,
+                                    cls_id=599, sep_id=599),
+    "lm-gpt2-bf16-long": wl.small_config("gpt2-medium", n_layers=2, hidden=128, heads=2, ffn=256, vocab=600,
+                                         max_pos=256, n_seqs=2, seq_lo=130, seq_hi=200, pad=8, pad_id=599,
+                                         cls_id=599, sep_id=599),
+    "lm-gpt2-fp32": wl.small_config("gpt2-medium", n_layers=2, hidden=64, heads=2, ffn=128, vocab=300,
+                                    max_pos=64, n_seqs=3, seq_lo=10, seq_hi=50, pad=1, pad_id=299,
+                                    cls_id=299, sep_id=299, dtype="fp32"),
 }
 
 
@@ -122,7 +133,7 @@ def test_step_parity_against_oracle(case):
             assert normwise(gd[k], G[k], floor) <= tolinf, (case, k, normwise(gd[k], G[k], floor))
 
 
-@pytest.mark.parametrize("case", ["toy-fp32", "mc-bf16", "qa-bf16"])
+@pytest.mark.parametrize("case", ["toy-fp32", "mc-bf16", "qa-bf16", "lm-gpt2-bf16", "lm-gpt2-bf16-long"])
 def test_recompute_replay_bitwise(case):
     cfg = CASES[case]
     params = wl.init_params(cfg, parity=True, seed=3)

@@ -21,7 +21,8 @@ from paper_conf_ipps_liaolysshfyctzlq23_b200 import binding as mb
 from paper_conf_ipps_liaolysshfyctzlq23_b200 import workload as wl
 
 ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
-CFGS = ["toy", "bert-base", "bert-large", "roberta-large"]
+CFGS = ["toy", "bert-base", "bert-large", "roberta-large", "gpt2-medium"]
+POST_LN = ["toy", "bert-base", "bert-large", "roberta-large"]
 
 
 def test_exports_every_header_symbol():

@@ -210,3 +210,79 @@ def test_adamw_against_torch():
         P, m, v = om.adamw(P, G, m, v, t, 1e-2, wd=0.01)
         for k in P:
             assert np.allclose(P[k], tp[k].detach().numpy(), rtol=0, atol=1e-14)
+
+
+# ------------------------------------------------------------ GPT-2 (pre-LN) --
+
+def tiny_gpt2(**kw):
+    base = dict(n_layers=2, hidden=16, heads=2, ffn=32, vocab=50, max_pos=16, pad_id=49, cls_id=49,
+                sep_id=49, first_tok=0, n_seqs=3, seq_lo=3, seq_hi=9, pad=1)
+    base.update(kw)
+    return wl.small_config("gpt2-medium", **base)
+
+
+def torch_step_gpt2(cfg, params, batch, masks):
+    """Independent GPT-2 (pre-LN, causal, tied LM head, tanh-GELU) in torch fp64."""
+    W = {k: torch.tensor(v, dtype=torch.float64, requires_grad=True) for k, v in params.items()}
+    B, S = batch.input_ids.shape
+    H, h = cfg.hidden, cfg.heads
+    d = H // h
+    F_ = torch.nn.functional
+    ids = torch.tensor(batch.input_ids, dtype=torch.long)
+    x = (W["emb.word"][ids] + W["emb.pos"][torch.arange(S)][None]).reshape(B * S, H) * torch.tensor(masks.emb())
+    valid = torch.arange(S)[None, :] < torch.tensor(batch.lengths)[:, None]
+    causal = torch.arange(S)[None, :] <= torch.arange(S)[:, None]
+    allowed = valid[:, None, None, :] & causal[None, None]
+    for l in range(cfg.n_layers):
+        p = f"layer{l}."
+        a = F_.layer_norm(x, (H,), W[p + "ln1.g"], W[p + "ln1.b"], cfg.ln_eps)
+        qkv = F_.linear(a, W[p + "qkv.w"], W[p + "qkv.b"]).reshape(B, S, 3, h, d)
+        q, k, v = (qkv[:, :, i].permute(0, 2, 1, 3) for i in range(3))
+        sc = (q @ k.transpose(-1, -2) / math.sqrt(d)).masked_fill(~allowed, float("-inf"))
+        pr = torch.softmax(sc, dim=-1) * torch.tensor(masks.attn_probs(l))
+        o = (pr @ v).permute(0, 2, 1, 3).reshape(B * S, H)
+        r1 = x + F_.linear(o, W[p + "o.w"], W[p + "o.b"]) * torch.tensor(masks.attn_out(l))
+        m = F_.layer_norm(r1, (H,), W[p + "ln2.g"], W[p + "ln2.b"], cfg.ln_eps)
+        g = F_.gelu(F_.linear(m, W[p + "f1.w"], W[p + "f1.b"]), approximate="tanh")
+        x = r1 + F_.linear(g, W[p + "f2.w"], W[p + "f2.b"]) * torch.tensor(masks.ffn_out(l))
+    hf = F_.layer_norm(x, (H,), W["lnf.g"], W["lnf.b"], cfg.ln_eps)
+    logits = (hf @ W["emb.word"].t()).reshape(B, S, -1)
+    labels = ids.clone()
+    labels[~valid] = -100
+    loss = F_.cross_entropy(logits[:, :-1].reshape(-1, cfg.vocab), labels[:, 1:].reshape(-1), ignore_index=-100)
+    loss.backward()
+    return float(loss), {k: t.grad.numpy() for k, t in W.items()}
+
+
+@pytest.mark.parametrize("p", [0.0, 0.1])
+def test_gpt2_against_torch_autograd(p):
+    cfg = tiny_gpt2()
+    params = wl.init_params(cfg, parity=True, seed=4)
+    batch = wl.make_batch(cfg, 8, seed=6)
+    loss, G = om.train_step_grads(cfg, params, batch, 13, 2, p=p)
+    masks = om.Masks(cfg, *batch.input_ids.shape, 13, 2, 0, p)
+    tloss, TG = torch_step_gpt2(cfg, params, batch, masks)
+    assert abs(loss - tloss) <= 1e-12 * max(1.0, abs(tloss))
+    for k in TG:
+        assert normwise(G[k], TG[k]) <= 1e-10, k
+
+
+def test_gpt2_finite_differences_and_replay():
+    cfg = tiny_gpt2()
+    params = {k: v.astype(np.float64) for k, v in wl.init_params(cfg, parity=True, seed=8).items()}
+    batch = wl.make_batch(cfg, 7, seed=2)
+    loss, G = om.train_step_grads(cfg, params, batch, 3, 1)
+    rng = np.random.default_rng(1)
+    for name in ("emb.word", "layer0.qkv.w", "layer1.f2.w", "layer1.ln1.g", "lnf.b", "emb.pos"):
+        flat = params[name].reshape(-1)
+        for i in rng.choice(flat.size, 4, replace=False):
+            old = flat[i]
+            flat[i] = old + 1e-6
+            lp, _ = om.train_step_grads(cfg, params, batch, 3, 1)
+            flat[i] = old - 1e-6
+            lm, _ = om.train_step_grads(cfg, params, batch, 3, 1)
+            flat[i] = old
+            assert abs((lp - lm) / 2e-6 - G[name].reshape(-1)[i]) <= 1e-6 * np.abs(G[name]).max() + 2e-9, name
+    for plan in ([0], [0, 1]):
+        l2, G2 = om.train_step_grads(cfg, params, batch, 3, 1, plan=plan)
+        assert l2 == loss and all(np.array_equal(G[k], G2[k]) for k in G)
