@@ -207,6 +207,8 @@ def main():
         ctx = mb.Mimose(cfg, budget, slab=slab, stream=stream, rank=rank, world=world,
                         nccl_id=nccl_id, enforce_budget=enforce, use_tc=use_tc)
         ctx.set_params(wl.pack_params(cfg, wl.init_params(cfg)))
+        # AdamW per gradient bucket on a side stream, overlapping the backward
+        ctx.set_optimizer(1e-5, fused=True)
         return ctx
 
     n_total = args.warmup + args.steps

@@ -207,6 +207,14 @@ mimose_status mimose_forward(mimose_ctx* ctx, const mimose_batch* batch,
 mimose_status mimose_backward(mimose_ctx* ctx);
 /* AdamW (torch semantics, reading A25) on the fp32 master weights. */
 mimose_status mimose_step(mimose_ctx* ctx, float lr, float beta1, float beta2, float eps, float wd);
+/* Register the optimizer.  fused = 1: mimose_backward launches AdamW for every
+   gradient bucket (encoder layer, head, embeddings) on a separate stream as
+   soon as that bucket is final (after its all-reduce under DP), overlapping the
+   rest of the backward; mimose_step then only orders the next forward after the
+   updates and must be called with the same arguments.  Same arithmetic as the
+   unfused step. */
+mimose_status mimose_set_optimizer(mimose_ctx* ctx, float lr, float beta1, float beta2, float eps, float wd,
+                                   int32_t fused);
 
 mimose_status mimose_get_stats(const mimose_ctx* ctx, mimose_stats* out);
 mimose_status mimose_phase(const mimose_ctx* ctx, int32_t* phase);

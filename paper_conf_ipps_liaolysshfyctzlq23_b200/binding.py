@@ -116,6 +116,7 @@ _lib.mimose_fit_predict.argtypes = [C.POINTER(C.c_int64), C.POINTER(C.c_int64), 
                                     C.POINTER(C.c_int64), C.c_int32, C.POINTER(C.c_int64)]
 
 _lib.mimose_nccl_unique_id.argtypes = [_P]
+_lib.mimose_set_optimizer.argtypes = [_P, C.c_float, C.c_float, C.c_float, C.c_float, C.c_float, C.c_int32]
 _lib.mimose_probe.argtypes = [_P, C.c_int32]
 _lib.mimose_probe_read.argtypes = [_P, C.POINTER(C.c_double), C.POINTER(C.c_double), C.POINTER(C.c_int64)]
 
@@ -124,7 +125,7 @@ EXPORTED = ["mimose_default_config", "mimose_init", "mimose_destroy", "mimose_la
             "mimose_get_grads", "mimose_collect", "mimose_plan", "mimose_forward", "mimose_backward",
             "mimose_step", "mimose_get_stats", "mimose_phase", "mimose_get_sample", "mimose_dry_run",
             "mimose_dry_collect", "mimose_predicted_peak", "mimose_plan_series", "mimose_fit_predict",
-            "mimose_nccl_unique_id", "mimose_probe", "mimose_probe_read"]
+            "mimose_nccl_unique_id", "mimose_probe", "mimose_probe_read", "mimose_set_optimizer"]
 
 
 _lib.mimose_tc_available.restype = C.c_int32
@@ -295,6 +296,9 @@ class Mimose:
 
     def backward(self):
         self._chk(_lib.mimose_backward(self.h))
+
+    def set_optimizer(self, lr=1e-4, beta1=0.9, beta2=0.999, eps=1e-8, wd=0.0, fused=True):
+        self._chk(_lib.mimose_set_optimizer(self.h, lr, beta1, beta2, eps, wd, 1 if fused else 0))
 
     def step(self, lr=1e-4, beta1=0.9, beta2=0.999, eps=1e-8, wd=0.0):
         self._chk(_lib.mimose_step(self.h, lr, beta1, beta2, eps, wd))

@@ -162,10 +162,13 @@ struct mimose_ctx {
   bool device = false;
   std::string err;
   mimose_status sticky = MIMOSE_OK;
-  cudaStream_t st = nullptr, comm_st = nullptr;
+  cudaStream_t st = nullptr, comm_st = nullptr, opt_st = nullptr;
   ncclComm_t comm = nullptr;
-  cudaEvent_t ev_comm_done = nullptr;
-  std::vector<cudaEvent_t> ev_layer;
+  cudaEvent_t ev_comm_done = nullptr, ev_opt_done = nullptr;
+  std::vector<cudaEvent_t> ev_layer, ev_ar;
+  // fused optimizer: per-bucket AdamW on opt_st as soon as the bucket's gradients are final
+  bool opt_fused = false;
+  float opt_lr = 0.f, opt_b1 = 0.9f, opt_b2 = 0.999f, opt_eps = 1e-8f, opt_wd = 0.f;
 
   std::vector<ParamInfo> layout;
   int64_t npad = 0;
@@ -640,12 +643,28 @@ int64_t bucket_end(mimose_ctx* c, int last_param) {
   return c->layout[last_param].off + (c->layout[last_param].numel + 63) / 64 * 64;
 }
 
+// A gradient bucket (params first..last) is final: all-reduce it (DP) on the
+// comm stream and, with the fused optimizer, update it on the optimizer stream,
+// both overlapping the rest of the backward.
 mimose_status allreduce_bucket(mimose_ctx* c, int first, int last, int evi) {
-  if (c->cfg.world <= 1 || !c->device) return MIMOSE_OK;
+  if (!c->device || (c->cfg.world <= 1 && !c->opt_fused)) return MIMOSE_OK;
   const int64_t b0 = bucket_begin(c, first), b1 = bucket_end(c, last);
   CK(cudaEventRecord(c->ev_layer[evi], c->st));
-  CK(cudaStreamWaitEvent(c->comm_st, c->ev_layer[evi], 0));
-  NK(ncclAllReduce(c->grad + b0, c->grad + b0, (size_t)(b1 - b0), ncclFloat, ncclSum, c->comm, c->comm_st));
+  cudaEvent_t ready = c->ev_layer[evi];
+  if (c->cfg.world > 1) {
+    CK(cudaStreamWaitEvent(c->comm_st, c->ev_layer[evi], 0));
+    NK(ncclAllReduce(c->grad + b0, c->grad + b0, (size_t)(b1 - b0), ncclFloat, ncclSum, c->comm, c->comm_st));
+    CK(cudaEventRecord(c->ev_ar[evi], c->comm_st));
+    ready = c->ev_ar[evi];
+  }
+  if (c->opt_fused) {
+    CK(cudaStreamWaitEvent(c->opt_st, ready, 0));
+    const double t = (double)(c->adam_t + 1);
+    const double bc1 = 1.0 - std::pow((double)c->opt_b1, t), bc2 = 1.0 - std::pow((double)c->opt_b2, t);
+    adamw(c->dt, c->w + b0 * c->e, c->master ? c->master + b0 : nullptr, c->grad + b0, c->m + b0, c->v + b0, b1 - b0,
+          c->opt_lr, c->opt_b1, c->opt_b2, c->opt_eps, c->opt_wd, (float)bc1, (float)bc2, 1.0f / (float)c->cfg.world,
+          c->opt_st);
+  }
   return MIMOSE_OK;
 }
 
@@ -1040,6 +1059,12 @@ mimose_status mimose_init(const mimose_config* cfgp, mimose_ctx** out) {
       CK(cudaEventCreate(&c->ev_t1[l]));
     }
     CK(cudaMemsetAsync(a.base, 0, (size_t)a.C, c->st));
+    c->ev_layer.resize(L + 2);
+    c->ev_ar.resize(L + 2);
+    for (auto& e : c->ev_layer) CK(cudaEventCreateWithFlags(&e, cudaEventDisableTiming));
+    for (auto& e : c->ev_ar) CK(cudaEventCreateWithFlags(&e, cudaEventDisableTiming));
+    CK(cudaStreamCreateWithFlags(&c->opt_st, cudaStreamNonBlocking));
+    CK(cudaEventCreateWithFlags(&c->ev_opt_done, cudaEventDisableTiming));
     if (k.world > 1) {
       if (!k.nccl_id) { *out = c; return bad("world > 1 needs nccl_id"); }
       int lo, hi;
@@ -1048,8 +1073,6 @@ mimose_status mimose_init(const mimose_config* cfgp, mimose_ctx** out) {
       ncclUniqueId id;
       std::memcpy(&id, k.nccl_id, sizeof(id));
       NK(ncclCommInitRank(&c->comm, k.world, id, k.rank));
-      c->ev_layer.resize(L + 2);
-      for (auto& e : c->ev_layer) CK(cudaEventCreateWithFlags(&e, cudaEventDisableTiming));
       CK(cudaEventCreateWithFlags(&c->ev_comm_done, cudaEventDisableTiming));
     }
   }
@@ -1063,8 +1086,12 @@ void mimose_destroy(mimose_ctx* c) {
     cudaStreamSynchronize(c->st);
     for (auto e : c->ev_t0) cudaEventDestroy(e);
     for (auto e : c->ev_t1) cudaEventDestroy(e);
+    if (c->opt_st) cudaStreamSynchronize(c->opt_st);
     for (auto e : c->ev_layer) cudaEventDestroy(e);
+    for (auto e : c->ev_ar) cudaEventDestroy(e);
     for (auto e : c->probe_ev) cudaEventDestroy(e);
+    if (c->ev_opt_done) cudaEventDestroy(c->ev_opt_done);
+    if (c->opt_st) cudaStreamDestroy(c->opt_st);
     if (c->ev_comm_done) cudaEventDestroy(c->ev_comm_done);
     if (c->comm) ncclCommDestroy(c->comm);
     if (c->comm_st) cudaStreamDestroy(c->comm_st);
@@ -1086,7 +1113,7 @@ static mimose_status xfer_params(mimose_ctx* c, float* host, int64_t n, int whic
   mimose_num_params(c, &tot);
   if (n != tot || !host) return fail(c, MIMOSE_E_INVALID, "blob size mismatch");
   if (!c->device) return fail(c, MIMOSE_E_NODEVICE, "host-only context");
-  // staging: fp32 padded image in the grad buffer's slot is not free; use a temporary device buffer
+  if (c->opt_st) CK(cudaStreamSynchronize(c->opt_st));
   float* tmp = nullptr;
   CK(cudaMallocAsync((void**)&tmp, (size_t)c->npad * 4, c->st));
   std::vector<float> img((size_t)c->npad, 0.f);
@@ -1223,6 +1250,15 @@ mimose_status mimose_step(mimose_ctx* c, float lr, float b1, float b2, float eps
   if (mimose_status s = check_ready(c)) return s;
   if (!c->bwd_done) return fail(c, MIMOSE_E_STATE, "step without a backward");
   if (!c->device) return MIMOSE_OK;
+  if (c->opt_fused) {   // the per-bucket updates were launched during backward
+    if (lr != c->opt_lr || b1 != c->opt_b1 || b2 != c->opt_b2 || eps != c->opt_eps || wd != c->opt_wd)
+      return fail(c, MIMOSE_E_INVALID, "fused optimizer: step arguments differ from mimose_set_optimizer");
+    CK(cudaEventRecord(c->ev_opt_done, c->opt_st));
+    CK(cudaStreamWaitEvent(c->st, c->ev_opt_done, 0));
+    c->adam_t++;
+    c->fwd_done = false;
+    return MIMOSE_OK;
+  }
   if (c->cfg.world > 1) {
     CK(cudaEventRecord(c->ev_comm_done, c->comm_st));
     CK(cudaStreamWaitEvent(c->st, c->ev_comm_done, 0));
@@ -1234,6 +1270,14 @@ mimose_status mimose_step(mimose_ctx* c, float lr, float b1, float b2, float eps
         1.0f / (float)c->cfg.world, c->st);
   CK(cudaGetLastError());
   c->fwd_done = false;
+  return MIMOSE_OK;
+}
+
+mimose_status mimose_set_optimizer(mimose_ctx* c, float lr, float b1, float b2, float eps, float wd, int32_t fused) {
+  if (mimose_status s = check_ready(c)) return s;
+  if (c->fwd_done && !c->bwd_done) return fail(c, MIMOSE_E_STATE, "set_optimizer inside a step");
+  c->opt_fused = fused != 0;
+  c->opt_lr = lr; c->opt_b1 = b1; c->opt_b2 = b2; c->opt_eps = eps; c->opt_wd = wd;
   return MIMOSE_OK;
 }
 

@@ -203,3 +203,25 @@ def test_adamw_step_against_oracle():
     newP, _, _ = omodel.adamw(P, G, zeros, dict(zeros), 1, 1e-3, wd=0.01)
     for k in P:
         assert np.abs(got[k] - newP[k]).max() <= 1e-6, k
+
+
+@pytest.mark.parametrize("case", ["mc-bf16", "lm-gpt2-bf16"])
+def test_fused_optimizer_bitwise_equal(case):
+    """Per-bucket AdamW on the side stream during backward == one AdamW after it."""
+    cfg = CASES[case]
+    params = wl.init_params(cfg, parity=True, seed=8)
+    out = []
+    for fused in (False, True):
+        ctx = make_ctx(cfg)
+        ctx.set_params(wl.pack_params(cfg, params))
+        if fused:
+            ctx.set_optimizer(lr=1e-3, wd=0.01, fused=True)
+        for step, L in enumerate([cfg.seq_hi - 2, cfg.seq_lo + 5]):
+            b = wl.make_batch(cfg, L, seed=50 + step)
+            ctx.forward(device_batch(ctx, b), None, False)
+            ctx.backward()
+            ctx.step(lr=1e-3, wd=0.01)
+        torch.cuda.synchronize()
+        out.append(ctx.get_params())
+        ctx.close()
+    assert np.array_equal(out[0], out[1])
