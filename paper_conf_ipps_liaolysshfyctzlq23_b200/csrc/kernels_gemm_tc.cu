@@ -119,27 +119,39 @@ MDEV void epi_row32(const GemmArgs& g, int m, int n, float (&v)[32], int z = -1)
 // smem buffer with the 16-B chunk index XOR-swizzled by row, then read back so
 // that each store instruction writes whole row segments: fp32 -> 4 rows x 128 B,
 // bf16 -> 8 rows x 64 B (full 32-B sectors, no partial-sector writes).
-MDEV void stage_store_f32(uint8_t* stg, const float (&v)[32], float* out, int64_t ld, int rows_valid, int lane) {
+MDEV void sts128(uint32_t a, uint4 w) {
+  asm volatile("st.shared.v4.b32 [%0], {%1, %2, %3, %4};" ::"r"(a), "r"(w.x), "r"(w.y), "r"(w.z), "r"(w.w) : "memory");
+}
+MDEV uint4 lds128(uint32_t a) {
+  uint4 w;
+  asm volatile("ld.shared.v4.b32 {%0, %1, %2, %3}, [%4];" : "=r"(w.x), "=r"(w.y), "=r"(w.z), "=r"(w.w) : "r"(a) : "memory");
+  return w;
+}
+MDEV void stage_store_f32(uint8_t* stg_p, const float (&v)[32], float* out, int64_t ld, int rows_valid, int lane) {
+  const uint32_t stg = (uint32_t)__cvta_generic_to_shared(stg_p);
 #pragma unroll
   for (int c = 0; c < 8; ++c)
-    *(float4*)(stg + lane * 128 + ((c ^ (lane & 7)) << 4)) = make_float4(v[4 * c], v[4 * c + 1], v[4 * c + 2], v[4 * c + 3]);
+    sts128(stg + lane * 128 + ((c ^ (lane & 7)) << 4),
+           make_uint4(__float_as_uint(v[4 * c]), __float_as_uint(v[4 * c + 1]), __float_as_uint(v[4 * c + 2]),
+                      __float_as_uint(v[4 * c + 3])));
   __syncwarp();
 #pragma unroll
   for (int k = 0; k < 8; ++k) {
     const int R = (lane >> 3) + 4 * k, c = lane & 7;
-    const float4 w = *(const float4*)(stg + R * 128 + ((c ^ (R & 7)) << 4));
-    if (R < rows_valid) *(float4*)(out + (int64_t)R * ld + 4 * c) = w;
+    const uint4 w = lds128(stg + R * 128 + ((c ^ (R & 7)) << 4));
+    if (R < rows_valid) *(uint4*)(out + (int64_t)R * ld + 4 * c) = w;
   }
   __syncwarp();
 }
-MDEV void stage_store_bf16(uint8_t* stg, const float (&v)[32], __nv_bfloat16* out, int64_t ld, int rows_valid, int lane) {
+MDEV void stage_store_bf16(uint8_t* stg_p, const float (&v)[32], __nv_bfloat16* out, int64_t ld, int rows_valid, int lane) {
+  const uint32_t stg = (uint32_t)__cvta_generic_to_shared(stg_p);
 #pragma unroll
-  for (int c = 0; c < 4; ++c) *(uint4*)(stg + lane * 128 + ((c ^ (lane & 3)) << 4)) = pack8(v + 8 * c);
+  for (int c = 0; c < 4; ++c) sts128(stg + lane * 128 + ((c ^ (lane & 3)) << 4), pack8(v + 8 * c));
   __syncwarp();
 #pragma unroll
   for (int k = 0; k < 4; ++k) {
     const int R = (lane >> 2) + 8 * k, c = lane & 3;
-    const uint4 w = *(const uint4*)(stg + R * 128 + ((c ^ (R & 3)) << 4));
+    const uint4 w = lds128(stg + R * 128 + ((c ^ (R & 3)) << 4));
     if (R < rows_valid) *(uint4*)(out + (int64_t)R * ld + 8 * c) = w;
   }
   __syncwarp();
@@ -226,7 +238,11 @@ MDEV void epi_load(const GemmArgs& g, int m, int n, bool live, EpiIn& in) {
 #pragma unroll
     for (int i = 0; i < 4; ++i) in.b[i] = p[i];
   }
-  if (!live) return;
+  if (!live) {   // rows >= M: defined (zero) inputs, results never stored
+#pragma unroll
+    for (int i = 0; i < 8; ++i) in.x[i] = make_uint4(0u, 0u, 0u, 0u);
+    return;
+  }
   if constexpr (EPI == EPI_BIAS_DROP_RES) {
     const uint4* p = (const uint4*)((const __nv_bfloat16*)g.res + (int64_t)m * g.ldr + n);
 #pragma unroll
@@ -256,13 +272,22 @@ MDEV void epi_frag32_in(const GemmArgs& g, int m_base, int n, float (&v)[32], in
 #pragma unroll
     for (int i = 0; i < 4; ++i) unpack8(in.b[i], b + 8 * i);
 #pragma unroll
-    for (int i = 0; i < 32; ++i) v[i] += b[i];
+    for (int i = 0; i < 32; i += 2) {
+      const float2 r = fadd2(make_float2(v[i], v[i + 1]), make_float2(b[i], b[i + 1]));
+      v[i] = r.x;
+      v[i + 1] = r.y;
+    }
     if constexpr (EPI == EPI_BIAS) {
       stage_store_bf16(stg, v, (E*)g.C + (int64_t)m_base * g.ldc + n, g.ldc, rows_valid, lane);
     } else if constexpr (EPI == EPI_BIAS_GELU) {
       stage_store_bf16(stg, v, (E*)g.C + (int64_t)m_base * g.ldc + n, g.ldc, rows_valid, lane);
 #pragma unroll
-      for (int i = 0; i < 32; ++i) v[i] = gelu_f(__bfloat162float(__float2bfloat16_rn(v[i])));
+      for (int i = 0; i < 32; i += 2) {
+        const float2 r = gelu_x2(make_float2(__bfloat162float(__float2bfloat16_rn(v[i])),
+                                             __bfloat162float(__float2bfloat16_rn(v[i + 1]))));
+        v[i] = r.x;
+        v[i + 1] = r.y;
+      }
       stage_store_bf16(stg, v, (E*)g.C2 + (int64_t)m_base * g.ldc + n, g.ldc, rows_valid, lane);
     } else {
       float r[32];
@@ -284,7 +309,11 @@ MDEV void epi_frag32_in(const GemmArgs& g, int m_base, int n, float (&v)[32], in
 #pragma unroll
     for (int i = 0; i < 4; ++i) unpack8(in.x[i], u + 8 * i);
 #pragma unroll
-    for (int i = 0; i < 32; ++i) v[i] = live ? v[i] * gelu_grad_f(u[i]) : 0.f;
+    for (int i = 0; i < 32; i += 2) {   // rows >= M are never stored
+      const float2 r = fmul2(make_float2(v[i], v[i + 1]), gelu_grad_x2(make_float2(u[i], u[i + 1])));
+      v[i] = r.x;
+      v[i + 1] = r.y;
+    }
     stage_store_bf16(stg, v, (E*)g.C + (int64_t)m_base * g.ldc + n, g.ldc, rows_valid, lane);
   } else if constexpr (EPI == EPI_ACC_RES_F32) {
     if (live) {
@@ -325,7 +354,7 @@ MDEV void epi_frag32_in(const GemmArgs& g, int m_base, int n, float (&v)[32], in
 #pragma unroll
     for (int i = 0; i < 4; ++i) unpack8(in.x[i], u + 8 * i);
 #pragma unroll
-    for (int i = 0; i < 32; ++i) v[i] = live ? v[i] * gelu_tanh_grad_f(u[i]) : 0.f;
+    for (int i = 0; i < 32; ++i) v[i] *= gelu_tanh_grad_f(u[i]);
     stage_store_bf16(stg, v, (E*)g.C + (int64_t)m_base * g.ldc + n, g.ldc, rows_valid, lane);
   } else if constexpr (EPI == EPI_ACC_F32) {
     if (live) {
@@ -472,7 +501,7 @@ constexpr int TP_THREADS = 64 + 32 * TP_EPI_WARPS;
 
 template <int BN>
 struct TpCfg {
-  static constexpr int STAGES = BN >= 256 ? 4 : 6;
+  static constexpr int STAGES = BN >= 256 ? 4 : (BN >= 128 ? 6 : 8);
   static constexpr int A_BYTES = TBM * TBK * 2;
   static constexpr int B_BYTES = BN * TBK * 2;
   static constexpr int STAGE_BYTES = A_BYTES + B_BYTES;
@@ -1042,10 +1071,19 @@ bool gemm_tc(Epi epi, const GemmArgs& g, cudaStream_t st) {
       return true;
     }
   }
-  // BN = 256 when N is a multiple of 256 and there are enough tiles to fill the SMs
-  int BN = (g_gemm_mode >= 1 && g.N % 256 == 0 && m_blocks * (g.N / 256) * g.split >= 120) ? 256 : 128;
+  // BN = 256 when N is a multiple of 256 and the 128x256 tiles still fill most
+  // of the 148 SMs; BN = 128 otherwise (measured per shape, tools/bench_gemm.py:
+  // BN = 64 loses on every step shape -- the per-tile fixed cost dominates).
+  auto tiles = [&](int bn) { return m_blocks * ((g.N + bn - 1) / bn) * g.split; };
+  int BN = (g.N % 256 == 0 && tiles(256) >= 100) ? 256 : 128;
   if (g_gemm_mode == 11) BN = 128;
   if (g_gemm_mode == 12 && g.N % 256 == 0) BN = 256;
+  if (g_gemm_mode == 13) BN = 64;
+  // Modes 0 (and the CTA-pair fallback when N % 128 != 0) run the one-tile-per-CTA
+  // kernel, whose B tile is 128 rows: the tensor-map box must match the kernel.
+  const bool persistent = g_gemm_mode == 1 || g_gemm_mode == 11 || g_gemm_mode == 12 || g_gemm_mode == 13 ||
+                          g_gemm_mode == 2 || g_gemm_mode == 21 || g_gemm_mode == 22;
+  if (!persistent) BN = 128;
   CUtensorMap ma, mb;
   bool ok;
   if (a.a_mn) ok = make_map(&ma, g.A, g.M, g.K, g.a_sk, 64, 64);
@@ -1054,14 +1092,15 @@ bool gemm_tc(Epi epi, const GemmArgs& g, cudaStream_t st) {
   if (a.b_mn) ok = make_map(&mb, g.B, g.N, g.K, g.b_sk, 64, 64);
   else ok = make_map(&mb, g.B, g.K, g.N, g.b_sn, 64, std::min(BN, 256));
   if (!ok) return false;
-  if (g_gemm_mode == 1 || g_gemm_mode == 11 || g_gemm_mode == 12) {
+  if (persistent) {
     TpArgs p;
     p.t = a;
     p.m_blocks = m_blocks;
     p.n_blocks = (g.N + BN - 1) / BN;
     p.n_tiles = p.m_blocks * p.n_blocks * g.split;
     if (BN == 256) dispatch_tcp<256>(epi, ma, mb, p, st);
-    else dispatch_tcp<128>(epi, ma, mb, p, st);
+    else if (BN == 128) dispatch_tcp<128>(epi, ma, mb, p, st);
+    else dispatch_tcp<64>(epi, ma, mb, p, st);
     return true;
   }
   constexpr int BN1 = 128;

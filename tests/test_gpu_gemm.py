@@ -30,18 +30,18 @@ def operands(M, N, K, a_mn, b_mn, seed=0):
 SHAPES += [(2048, 3072, 768), (512, 768, 3072), (4096, 2304, 768)]   # BN=256 persistent tiles
 
 
-@pytest.fixture(params=[2, 1, 0], ids=["cta-pair", "persistent", "tile-per-cta"])
+@pytest.fixture(params=[1, 13, 2, 0], ids=["persistent", "persistent-bn64", "cta-pair", "tile-per-cta"])
 def gemm_mode(request):
     mb().debug_options(gemm_mode=request.param)
     yield request.param
-    mb().debug_options(gemm_mode=2)
+    mb().debug_options(gemm_mode=1)
 
 
 @pytest.mark.parametrize("use_tc", [True, False])
 @pytest.mark.parametrize("a_mn,b_mn", [(0, 0), (0, 1), (1, 1)])
 @pytest.mark.parametrize("shape", SHAPES)
 def test_gemm_f32_out(shape, a_mn, b_mn, use_tc, gemm_mode):
-    if not use_tc and gemm_mode != 2:
+    if not use_tc and gemm_mode != 1:
         pytest.skip("SIMT path does not depend on the tcgen05 mode")
     M, N, K = shape
     A, B, As, Bs, a_sm, a_sk, b_sn, b_sk = operands(M, N, K, a_mn, b_mn)

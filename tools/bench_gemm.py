@@ -25,6 +25,8 @@ def timeit(fn, reps=20):
 
 def main():
     T = int(sys.argv[1]) if len(sys.argv) > 1 else 5120
+    only = sys.argv[2] if len(sys.argv) > 2 else ""          # substring filter on the case name
+    modes = [int(m) for m in sys.argv[3].split(",")] if len(sys.argv) > 3 else [1, 11, 12, 13]
     H, F = 768, 3072
     dev = "cuda"
     bf = torch.bfloat16
@@ -60,11 +62,13 @@ def main():
         ("wgr out  (H,H,T) s4", 6, H, H, T, dyH, 1, H, x, 1, H, dict(split=4)),
     ]
     for name, epi, M, N, K, A, asm, ask, B, bsn, bsk, ex in cases:
+        if only and only not in name:
+            continue
         fl = 2.0 * M * N * K
         split = ex.pop("split", 1)
         C = (outf if epi in (3, 5, 6) else outb)
         C_ = ws if split > 1 else C
-        for mode in (2, 1, 0):
+        for mode in modes:
             mb.debug_options(gemm_mode=mode)
             us = timeit(lambda: mb.debug_gemm_ex(epi, M, N, K, A, asm, ask, B, bsn, bsk, C_, N, bias=bias,
                                                  split=split, **ex))
@@ -75,7 +79,7 @@ def main():
         Bm = B if bsk == 1 else B.t()
         us = timeit(lambda: torch.matmul(Am, Bm.t() if bsk == 1 else B))
         print(f"{name:22s} T={T:5d} cuBLAS  {us:8.1f} us  {fl / us / 1e6:7.1f} TFLOP/s", flush=True)
-    mb.debug_options(gemm_mode=2)
+    mb.debug_options(gemm_mode=1)
 
 
 if __name__ == "__main__":
