@@ -36,7 +36,7 @@ METRIC = "samples/sec under fixed memory budget, dynamic seq len, 1/2/4/8 B200"
 def parse():
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
-    ap.add_argument("--steps", type=int, default=30)
+    ap.add_argument("--steps", type=int, default=200)
     ap.add_argument("--warmup", type=int, default=5)
     ap.add_argument("--impl", default="mimose", choices=["mimose", "reference"])
     ap.add_argument("--config", default="bert-base", choices=sorted(wl.CONFIGS))
@@ -56,6 +56,17 @@ def peaks():
             "sm_max_mhz": 1965.0}, "fallback"
 
 
+def gemm_traffic():
+    """DRAM bytes (read + write) per GEMM launch, from the committed ncu pass
+    over this bench (tools/gemm_traffic.py -> profiles/<round>/gemm_traffic.json)."""
+    import glob
+    fs = sorted(glob.glob(os.path.join(ROOT, "profiles", "*", "gemm_traffic.json")))
+    if not fs:
+        return None, None
+    d = json.load(open(fs[-1]))
+    return d["dram_bytes_per_launch"], os.path.relpath(fs[-1], ROOT) + ": " + d["how"]
+
+
 class Clocks:
     """nvidia-smi sampler for the timed region (B200_PROFILING.md clocks line)."""
     Q = ("index,clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,"
@@ -65,17 +76,39 @@ class Clocks:
     def __init__(self, dev: int):
         self.dev, self.rows, self.stop = dev, [], threading.Event()
 
+    def _nvml_row(self, nv, h):
+        r = nv.nvmlDeviceGetCurrentClocksEventReasons(h)
+        bits = [nv.nvmlClocksEventReasonHwSlowdown, nv.nvmlClocksEventReasonHwThermalSlowdown,
+                nv.nvmlClocksEventReasonSwThermalSlowdown, nv.nvmlClocksEventReasonSwPowerCap]
+        return [str(self.dev), str(nv.nvmlDeviceGetClockInfo(h, nv.NVML_CLOCK_SM)),
+                str(nv.nvmlDeviceGetMaxClockInfo(h, nv.NVML_CLOCK_SM)),
+                str(nv.nvmlDeviceGetPowerUsage(h) / 1000.0), hex(r)] + \
+               ["Active" if r & b else "Not Active" for b in bits]
+
     def _run(self):
+        # NVML in-process (a sample every ~20 ms, so a sub-second timed region
+        # still gets many samples); nvidia-smi subprocess as the fallback
+        nv = h = None
+        try:
+            import pynvml as nv
+            nv.nvmlInit()
+            h = nv.nvmlDeviceGetHandleByIndex(self.dev)
+        except Exception:
+            nv = None
         while not self.stop.is_set():
             try:
-                out = subprocess.run(["nvidia-smi", "-i", str(self.dev), "--query-gpu=" + self.Q,
-                                      "--format=csv,noheader,nounits"], capture_output=True,
-                                     text=True, timeout=5).stdout.strip()
-                if out:
-                    self.rows.append([t.strip() for t in out.split(",")])
+                if nv is not None:
+                    self.rows.append(self._nvml_row(nv, h))
+                else:
+                    out = subprocess.run(["nvidia-smi", "-i", str(self.dev), "--query-gpu=" + self.Q,
+                                          "--format=csv,noheader,nounits"], capture_output=True,
+                                         text=True, timeout=5).stdout.strip()
+                    if out:
+                        self.rows.append([t.strip() for t in out.split(",")])
             except Exception:
                 pass
-            self.stop.wait(0.2)
+            self.stop.wait(0.02 if nv is not None else 0.2)
+        self.source = "nvml" if nv is not None else "nvidia-smi"
 
     def __enter__(self):
         self.t = threading.Thread(target=self._run, daemon=True)
@@ -94,7 +127,19 @@ class Clocks:
         names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
         reasons = sorted({n for r in self.rows for n, v in zip(names, r[5:9]) if v.lower() == "active"})
         return {"sm_mhz": float(np.median(sm)) if sm else None, "sm_max_mhz": max(mx) if mx else None,
-                "reasons": reasons, "samples": len(self.rows)}
+                "reasons": reasons, "samples": len(self.rows), "source": getattr(self, "source", None)}
+
+
+def step_flops(cfg, n_seqs, S):
+    """Algorithmic FLOPs of one step: model = 3 x forward
+    (+ the LM head), and the forward FLOPs of one layer (added per dropped layer)."""
+    H, F, T = cfg.hidden, cfg.ffn, n_seqs * S
+    attn = 4.0 * n_seqs * S * S * H * (0.5 if cfg.arch == wl.ARCH_PRE_LN else 1.0)
+    layer = 2.0 * T * (4 * H * H + 2 * H * F) + attn
+    model = 3.0 * layer * cfg.n_layers
+    if cfg.head == wl.HEAD_LM:
+        model += 3.0 * 2.0 * T * H * cfg.vocab
+    return model, layer
 
 
 def dist_env():
@@ -124,7 +169,7 @@ def oracle_sample_step(cfg, S_longest, n_q, step):
 ORACLE_PARAMS: dict = {}
 
 
-def cpu_baseline(cfg, n_steps=1, n_q=2):
+def cpu_baseline(cfg, n_steps=2, n_q=2):
     S = wl.roundup((cfg.seq_lo + cfg.seq_hi) // 2, cfg.pad)
     tot_t, tot_s = 0.0, 0
     for i in range(n_steps):
@@ -305,9 +350,17 @@ def main():
     e2e = samples_per_step * args.steps / (ms_e2e / 1000.0)
     per_step_h2d = int(np.mean([(b.input_ids.size * 2 + b.lengths.size + b.labels.size) * 4 for b in batches]))
     st2 = ctx.stats()
-    dropped = []
+    dropped, pred_err, flops_model, flops_hw = [], [], 0.0, 0.0
     for b in batches[args.warmup:]:
-        dropped.append(ctx.plan(b.input_size).n_dropped)
+        p = ctx.plan(b.input_size)
+        dropped.append(p.n_dropped)
+        # prediction error as the paper defines it, on the whole-step peak:
+        # the estimator's predicted peak for the plan vs the arena's exact peak
+        actual = ctx.dry_run(b.n_seqs, b.seq_len, p.dropped)
+        pred_err.append(abs(p.predicted_peak - actual) / actual)
+        fm, fr = step_flops(cfg, b.n_seqs, b.seq_len)
+        flops_model += fm
+        flops_hw += fm + fr * p.n_dropped
     samples = [ctx.sample(j) for j in range(st["n_samples"])]
     t_ms = [np.mean(s["t_ms"]) for s in samples]
 
@@ -323,8 +376,9 @@ def main():
         bound, unit = "alu", "TFLOP/s"
         peak_note = f"FP32 FMA: 148 SM x 128 lanes x 2 x {pk.get('sm_max_mhz', 1965.0)} MHz ({kind} clock)"
     achieved = gemm_flops / (gemm_ms / 1000.0) / 1e12 if gemm_ms > 0 else 0.0
+    traffic, traffic_src = gemm_traffic()
     roofline = {"bound": bound, "achieved": achieved, "peak": peak, "unit": unit,
-                "frac": achieved / peak if peak else None, "traffic": None,
+                "frac": achieved / peak if peak else None, "traffic": traffic, "traffic_source": traffic_src,
                 "kernel": "GEMM (all linear layers: fwd, dgrad, wgrad)",
                 "peak_source": peak_note, "launches": gemm_n,
                 "share_of_step": gemm_ms / ms_probe if ms_probe else None,
@@ -352,7 +406,11 @@ def main():
                    "plan_cache_hits": st2["plan_cache_hits"], "plan_cache_misses": st2["plan_cache_misses"],
                    "planner_us_total": st2["planner_us_total"], "sheltered_iters": st2["collect_steps"],
                    "shuttled_iters": st2["shuttled_steps"], "sheltered_s": sheltered_s,
-                   "collector_layer_fwd_ms_mean": float(np.mean(t_ms)) if t_ms else None},
+                   "collector_layer_fwd_ms_mean": float(np.mean(t_ms)) if t_ms else None,
+                   "prediction_error_mean": float(np.mean(pred_err)), "prediction_error_max": float(np.max(pred_err))},
+        "mfu": flops_model * world / (ms / 1000.0) / 1e12 / peak if tc else None,
+        "hfu": flops_hw * world / (ms / 1000.0) / 1e12 / peak if tc else None,
+        "tflops_model": flops_model * world / (ms / 1000.0) / 1e12,
     }
     ctx.close()
     del ctx

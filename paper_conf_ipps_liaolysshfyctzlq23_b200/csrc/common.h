@@ -4,6 +4,8 @@
 #include <cstdint>
 #include <cuda_runtime.h>
 #include <cuda_bf16.h>
+#include <cstdlib>
+#include <utility>
 
 namespace mimose {
 
@@ -26,10 +28,49 @@ struct Drop {
   int enabled;       // p > 0
 };
 
+// Programmatic dependent launch (PDL).  Every kernel of the library is launched
+// with cudaLaunchAttributeProgrammaticStreamSerialization, so the next kernel in
+// the stream is scheduled as soon as every CTA of the running one has started;
+// it runs its prologue (barrier init, TMEM alloc, tensor-map prefetch) and then
+// blocks in griddepcontrol.wait until the previous grid has completed and its
+// memory is visible.  Every kernel calls pdl_enter() (or pdl_trigger() +
+// pdl_wait() around a prologue that touches no global memory) before its first
+// global access, so the stream order of all reads and writes is unchanged: the
+// results are bitwise those of plain launches.  MIMOSE_PDL=0 disables it.
+inline bool pdl_enabled() {
+  static const int v = [] {
+    const char* e = std::getenv("MIMOSE_PDL");
+    return e ? std::atoi(e) : 1;
+  }();
+  return v != 0;
+}
+template <typename... KArgs, typename... Args>
+inline cudaError_t launch_k(void (*k)(KArgs...), dim3 grid, dim3 block, size_t smem, cudaStream_t s,
+                            Args&&... args) {
+  cudaLaunchConfig_t cfg = {};
+  cfg.gridDim = grid;
+  cfg.blockDim = block;
+  cfg.dynamicSmemBytes = smem;
+  cfg.stream = s;
+  cudaLaunchAttribute at[1];
+  at[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+  at[0].val.programmaticStreamSerializationAllowed = 1;
+  cfg.attrs = at;
+  cfg.numAttrs = pdl_enabled() ? 1 : 0;
+  return cudaLaunchKernelEx(&cfg, k, std::forward<Args>(args)...);
+}
+
 constexpr int NPART = 296;   // fixed reduction-partial count (DESIGN "Memory model")
 
 #if defined(__CUDACC__)
 #define MDEV __device__ __forceinline__
+
+MDEV void pdl_trigger() { asm volatile("griddepcontrol.launch_dependents;" ::: "memory"); }
+MDEV void pdl_wait() { asm volatile("griddepcontrol.wait;" ::: "memory"); }
+MDEV void pdl_enter() {
+  pdl_trigger();
+  pdl_wait();
+}
 
 // Philox4x32-10, Salmon et al. SC'11 (same constants as Random123).
 MDEV uint4 philox4x32_10(uint4 c, uint32_t k0, uint32_t k1) {

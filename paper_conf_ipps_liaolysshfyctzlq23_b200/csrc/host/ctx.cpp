@@ -16,6 +16,7 @@
 #include <chrono>
 #include <cmath>
 #include <cstdio>
+#include <cstdlib>
 #include <cstring>
 #include <string>
 #include <unordered_map>
@@ -414,10 +415,51 @@ void free_internals(Run& r, bool on_stack) {
   for (int i = 9; i >= 0; --i) on_stack ? a.pop(s[i]) : a.tfree(s[i]);
 }
 
+// MIMOSE_WGRAD_FUSED=1 enables (default off until it wins; see DESIGN) instead of the 128 x 128 / separate-reduction wgrad (A/B).
+static bool wgrad_fused(const mimose_ctx*) {
+  static const int v = [] {
+    const char* e = std::getenv("MIMOSE_WGRAD_FUSED");
+    return e ? std::atoi(e) : 0;
+  }();
+  return v != 0;
+}
+
 void wgrad(Run& r, const void* dY, int N, const void* X, int K, float* out) {
   // dW[N, K] = sum_t dY[t, n] X[t, k]; deterministic split-K over t.
   mimose_ctx* c = r.c;
   const int T = c->T;
+  if (c->dt == DT_BF16 && c->cfg.use_tc && K % 256 == 0 && N % 128 == 0 && wgrad_fused(c)) {
+    // 128 x 256 tiles (N = 256 MMAs; 128 x 128 ones are smem-bound at half
+    // rate) with an in-kernel fused split-K: pick the split s minimising
+    // rounds(s) / s, with the s-1 fp32 partials fitting the workspace; the
+    // 128 x 128 path below is modelled at 0.85 of a 128 x 256 tile-time.
+    const int t256 = (N / 128) * (K / 256);
+    double best = 1e30;
+    int bs = 1;
+    for (int s = 1; s <= 8; ++s) {
+      if ((int64_t)(s - 1) * N * K > c->ws_elems || T / s < 256) break;
+      const double v = (double)((t256 * s + 147) / 148) / s;
+      if (v < best - 1e-9) { best = v; bs = s; }
+    }
+    const int t128 = ((N + 127) / 128) * ((K + 127) / 128);
+    int s_old = std::max(1, std::min(4, 148 / std::max(1, t128)));
+    while (s_old > 1 && (int64_t)s_old * N * K > c->ws_elems) --s_old;
+    const double v_old = 0.85 * (double)((t128 * s_old + 147) / 148) / s_old;
+    if (best <= v_old) {
+      GemmArgs g;
+      g.M = N; g.N = K; g.K = T;
+      g.A = dY; g.a_sm = 1; g.a_sk = N;
+      g.B = X; g.b_sn = 1; g.b_sk = K;
+      g.C = out; g.ldc = K;
+      g.bn = 256;
+      g.split = bs;
+      g.fused_split = bs > 1;
+      g.ws = c->ws;
+      g.split_stride = (int64_t)N * K;
+      pgemm(c, EPI_F32, g, r.st);
+      return;
+    }
+  }
   const int tiles = ((N + 127) / 128) * ((K + 127) / 128);
   int split = std::max(1, std::min(4, 148 / std::max(1, tiles)));
   while (split > 1 && (int64_t)split * N * K > c->ws_elems) --split;
@@ -1330,6 +1372,14 @@ mimose_status mimose_debug_gemm_ex(int32_t epi, int32_t M, int32_t N, int32_t K,
   g.C = Cp; g.ldc = ldc; g.C2 = C2; g.bias = bias; g.res = res; g.ldr = ldr; g.aux = aux; g.ldx = ldx;
   g.split = split < 1 ? 1 : split;
   g.split_stride = (int64_t)M * ldc;
+  if (split < 0) {          // fused split-K (EPI_F32, tile width 256): C2 is the partial workspace
+    if (epi != EPI_F32) return MIMOSE_E_INVALID;
+    g.split = -split;
+    g.fused_split = 1;
+    g.bn = 256;
+    g.ws = (float*)C2;
+    g.C2 = nullptr;
+  }
   g.drop.enabled = 1; g.drop.seed_lo = 7; g.drop.seed_hi = 0; g.drop.site = 0; g.drop.step = 1;
   g.drop.thresh = 3865470566u; g.drop.scale = (float)(1.0 / 0.9);
   gemm(DT_BF16, (Epi)epi, g, (cudaStream_t)stream, use_tc != 0);

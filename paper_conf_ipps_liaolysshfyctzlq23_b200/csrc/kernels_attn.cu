@@ -34,6 +34,7 @@ template <typename E, int D>
 __global__ void __launch_bounds__(AT) k_attn_fwd(const E* __restrict__ qkv, const int32_t* __restrict__ lengths,
                                                  E* __restrict__ O, float* __restrict__ lse, int S, int H,
                                                  int h, float scale, Drop drop, int causal) {
+  pdl_enter();
   __shared__ float Ks[AT][D + 1];
   __shared__ float Vs[AT][D + 1];
   const int bh = blockIdx.y, b = bh / h, hd = bh % h;
@@ -107,7 +108,7 @@ void attn_fwd(DType dt, const void* qkv, const int32_t* lengths, void* O, float*
   auto go = [&](auto* tag, auto dconst) {
     using E = std::remove_pointer_t<decltype(tag)>;
     constexpr int DD = decltype(dconst)::value;
-    k_attn_fwd<E, DD><<<grid, AT, 0, st>>>((const E*)qkv, lengths, (E*)O, lse, S, H, h, scale, drop, causal ? 1 : 0);
+    launch_k(k_attn_fwd<E, DD>, grid, AT, 0, st, (const E*)qkv, lengths, (E*)O, lse, S, H, h, scale, drop, causal ? 1 : 0);
   };
   if (dt == DT_F32) {
     if (D == 32) go((float*)nullptr, std::integral_constant<int, 32>{});
@@ -122,6 +123,7 @@ void attn_fwd(DType dt, const void* qkv, const int32_t* lengths, void* O, float*
 template <typename E>
 __global__ void k_attn_dot(const E* __restrict__ O, const E* __restrict__ dO, float* __restrict__ Dbuf,
                            int B, int S, int H, int h) {
+  pdl_enter();
   const int w = (blockIdx.x * blockDim.x + threadIdx.x) >> 5, lane = threadIdx.x & 31;
   if (w >= B * h * S) return;
   const int q = w % S, bh = w / S, b = bh / h, hd = bh % h;
@@ -139,6 +141,7 @@ __global__ void __launch_bounds__(BT) k_attn_bwd_kv(const E* __restrict__ qkv, c
                                                     const float* __restrict__ lse, const float* __restrict__ Dbuf,
                                                     const int32_t* __restrict__ lengths, E* __restrict__ dqkv,
                                                     int S, int H, int h, float scale, Drop drop, int causal) {
+  pdl_enter();
   __shared__ float Qs[BT][D + 1];
   __shared__ float dOs[BT][D + 1];
   __shared__ float Kt[D][BT + 1];
@@ -203,6 +206,7 @@ __global__ void __launch_bounds__(BT) k_attn_bwd_q(const E* __restrict__ qkv, co
                                                    const float* __restrict__ lse, const float* __restrict__ Dbuf,
                                                    const int32_t* __restrict__ lengths, E* __restrict__ dqkv,
                                                    int S, int H, int h, float scale, Drop drop, int causal) {
+  pdl_enter();
   __shared__ float Qt[D][BT + 1];
   __shared__ float dOt[D][BT + 1];
   __shared__ float Ks[BT][D + 1];
@@ -270,10 +274,10 @@ void attn_bwd(DType dt, const void* qkv, const void* O, const void* dO, const fl
   auto go = [&](auto* tag, auto dconst) {
     using E = std::remove_pointer_t<decltype(tag)>;
     constexpr int DD = decltype(dconst)::value;
-    k_attn_dot<E><<<cdiv((int64_t)B * h * S, 8), 256, 0, st>>>((const E*)O, (const E*)dO, Dbuf, B, S, H, h);
-    k_attn_bwd_kv<E, DD><<<grid, BT, 0, st>>>((const E*)qkv, (const E*)dO, lse, Dbuf, lengths, (E*)dqkv, S, H, h,
+    launch_k(k_attn_dot<E>, cdiv((int64_t)B * h * S, 8), 256, 0, st, (const E*)O, (const E*)dO, Dbuf, B, S, H, h);
+    launch_k(k_attn_bwd_kv<E, DD>, grid, BT, 0, st, (const E*)qkv, (const E*)dO, lse, Dbuf, lengths, (E*)dqkv, S, H, h,
                                              scale, drop, causal ? 1 : 0);
-    k_attn_bwd_q<E, DD><<<grid, BT, 0, st>>>((const E*)qkv, (const E*)dO, lse, Dbuf, lengths, (E*)dqkv, S, H, h,
+    launch_k(k_attn_bwd_q<E, DD>, grid, BT, 0, st, (const E*)qkv, (const E*)dO, lse, Dbuf, lengths, (E*)dqkv, S, H, h,
                                             scale, drop, causal ? 1 : 0);
   };
   if (dt == DT_F32) {

@@ -51,14 +51,38 @@ MDEV void st_tile_row32(uint8_t* tile, int r, int c, const float* v) {
   for (int j = 0; j < 4; ++j) *(uint4*)(base + sw128(r, cb + j)) = pack8(v + 8 * j);
 }
 
+// Same, for the 16 keys [32c + 16hh, 32c + 16hh + 16).
+MDEV void st_tile_row16(uint8_t* tile, int r, int c, int hh, const float* v) {
+  const int atom = c >> 1, cb = (c & 1) * 4 + 2 * hh;
+  uint8_t* base = tile + atom * (AQ * 128);
+#pragma unroll
+  for (int j = 0; j < 2; ++j) *(uint4*)(base + sw128(r, cb + j)) = pack8(v + 8 * j);
+}
+
 MDEV float4 drop4_or(const Drop& d, uint64_t e) {
   if (!d.enabled) return make_float4(1.f, 1.f, 1.f, 1.f);
   if ((e & 3) == 0) return drop_factor4(d, e >> 2);
   return make_float4(drop_factor(d, e), drop_factor(d, e + 1), drop_factor(d, e + 2), drop_factor(d, e + 3));
 }
 
+// 8 warps: warp w reads TMEM lane quarter w % 4 (rows 32(w%4)..+31) and
+// handles column half w / 4 of every row: key chunks [0, cmid) or [cmid, nch).
+// The two halves of a row combine their max / sum / dot partials through
+// shared memory in a fixed order (half 0 + half 1), so results are
+// deterministic.
+constexpr int ATT = 256;
+MDEV float ex2f(float x) {
+  float y;
+  asm("ex2.approx.ftz.f32 %0, %1;" : "=f"(y) : "f"(x));
+  return y;
+}
+
 // kmax = roundup(S, 32): the key range every MMA and every softmax pass covers.
-__global__ void __launch_bounds__(128) k_attn_fwd_tc(const __grid_constant__ CUtensorMap tq, const AttnArgs a) {
+// Softmax: pass 1 takes the row max, pass 2 writes the unnormalised
+// P~ = exp(s - max) * dropout (bf16) and the row sum l; O = (P~ V) / l in the
+// epilogue, LSE = max + log l (what the backward recomputes P from).
+__global__ void __launch_bounds__(ATT, 3) k_attn_fwd_tc(const __grid_constant__ CUtensorMap tq, const AttnArgs a) {
+  pdl_enter();
   extern __shared__ __align__(1024) uint8_t sm[];
   uint8_t* sQ = sm;
   uint8_t* sK = sm + TILE;
@@ -66,11 +90,14 @@ __global__ void __launch_bounds__(128) k_attn_fwd_tc(const __grid_constant__ CUt
   uint8_t* sP = sm;                       // reuses Q and K (dead after S = Q K^T)
   uint64_t* bar = (uint64_t*)(sm + 3 * TILE);   // [0] tma, [1] mma S, [2] mma O
   uint32_t* tslot = (uint32_t*)(bar + 4);
-  const int t = threadIdx.x, warp = t >> 5;
+  float* red = (float*)(sm + 3 * TILE + 64);     // [2][128] per-half row partials
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const int hf = warp >> 2, t = 32 * (warp & 3) + lane;
   const int bh = blockIdx.x, b = bh / a.h, hd = bh % a.h;
   const int S = a.S, len = a.lengths[b];
-  const int kmax = (S + 31) & ~31, nch = kmax >> 5;
-  if (t == 0) {
+  const int kmax = (S + 31) & ~31, nch = kmax >> 5, cmid = (nch + 1) >> 1;
+  const int c0 = hf ? cmid : 0, c1 = hf ? nch : cmid;
+  if (threadIdx.x == 0) {
     for (int i = 0; i < 3; ++i) mbar_init(&bar[i], 1);
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
   }
@@ -83,7 +110,7 @@ __global__ void __launch_bounds__(128) k_attn_fwd_tc(const __grid_constant__ CUt
   tc_fence_after();
   const uint32_t tmem = *tslot;
   const int row0 = b * S;
-  if (t == 0) {
+  if (threadIdx.x == 0) {
     mbar_expect_tx(&bar[0], 3 * TILE);
     tma_load_2d(&tq, &bar[0], sQ, hd * AD, row0);
     tma_load_2d(&tq, &bar[0], sK, a.H + hd * AD, row0);
@@ -101,48 +128,60 @@ __global__ void __launch_bounds__(128) k_attn_fwd_tc(const __grid_constant__ CUt
   __syncwarp();
   tc_fence_after();
   // ---- softmax of row t over keys [0, kl), kl = len (or min(len, t+1) causal) ----
-  const uint32_t trow = tmem + ((uint32_t)(32 * warp) << 16);
+  const uint32_t trow = tmem + ((uint32_t)(32 * (warp & 3)) << 16);
   const int kl = a.causal ? min(len, t + 1) : len;
-  float m = -INFINITY, l = 0.f;
-  for (int c = 0; c < nch; ++c) {
+  float mx = -INFINITY;
+  for (int c = c0; c < c1; ++c) {
     float v[32];
     tmem_ld32(trow + 32 * c, v);                // every lane loads (.sync.aligned)
     if (32 * c < kl) {
 #pragma unroll
-      for (int i = 0; i < 32; ++i) {
-        const float s = (32 * c + i < kl) ? v[i] * a.scale : -INFINITY;
-        if (s > m) { l = l * __expf(m - s) + 1.f; m = s; } else { l += __expf(s - m); }
-      }
+      for (int i = 0; i < 32; ++i)
+        if (32 * c + i < kl) mx = fmaxf(mx, v[i]);
     }
   }
-  const float L = m + __logf(l);
+  red[hf * 128 + t] = mx;
+  __syncthreads();
+  const float sl2 = a.scale * 1.4426950408889634f;               // scale * log2(e)
+  const float mrow = fmaxf(red[t], red[128 + t]) * sl2;          // row max of s * scale * log2(e)
   const uint64_t ebase = (((uint64_t)b * a.h + hd) * S + (uint64_t)t) * S;
   // The S MMA has completed (bar[1]), so Q and K are dead: each thread writes its
   // P~ row straight into their space.
-  for (int c = 0; c < nch; ++c) {
-    float v[32];
-    tmem_ld32(trow + 32 * c, v);
-    if (32 * c < kl && t < S) {
+  float l = 0.f;
+  for (int c = c0; c < c1; ++c) {
 #pragma unroll
-      for (int j = 0; j < 8; ++j) {
-        const int k = 32 * c + 4 * j;
-        const float4 f = (k < kl) ? drop4_or(a.drop, ebase + k) : make_float4(0.f, 0.f, 0.f, 0.f);
-        const float ff[4] = {f.x, f.y, f.z, f.w};
+    for (int hh = 0; hh < 2; ++hh) {
+      float v[16];
+      tmem_ld16(trow + 32 * c + 16 * hh, v);
+      const int kb = 32 * c + 16 * hh;
+      if (kb < kl && t < S) {
 #pragma unroll
-        for (int i = 0; i < 4; ++i)
-          v[4 * j + i] = (k + i < kl) ? __expf(v[4 * j + i] * a.scale - L) * ff[i] : 0.f;
+        for (int j = 0; j < 4; ++j) {
+          const int k = kb + 4 * j;
+          const float4 f = (k < kl) ? drop4_or(a.drop, ebase + k) : make_float4(0.f, 0.f, 0.f, 0.f);
+          const float ff[4] = {f.x, f.y, f.z, f.w};
+#pragma unroll
+          for (int i = 0; i < 4; ++i) {
+            const float p = (k + i < kl) ? ex2f(fmaf(v[4 * j + i], sl2, -mrow)) : 0.f;
+            l += p;
+            v[4 * j + i] = p * ff[i];
+          }
+        }
+      } else {
+#pragma unroll
+        for (int i = 0; i < 16; ++i) v[i] = 0.f;
       }
-    } else {
-#pragma unroll
-      for (int i = 0; i < 32; ++i) v[i] = 0.f;
+      st_tile_row16(sP, t, c, hh, v);
     }
-    st_tile_row32(sP, t, c, v);
   }
+  __syncthreads();                              // red[] (max) reads done before reuse
+  red[hf * 128 + t] = l;
   fence_async_smem();
   tc_fence_before();
   __syncthreads();
   tc_fence_after();
-  if (t == 0) {
+  const float lsum = red[t] + red[128 + t];
+  if (threadIdx.x == 0) {
     const uint32_t id = idesc_bf16(AQ, AD, 0, 1);
     const uint32_t p0 = smem_u32(sP), v0 = smem_u32(sV);
     for (int kk = 0; kk < kmax / 16; ++kk) {
@@ -155,15 +194,15 @@ __global__ void __launch_bounds__(128) k_attn_fwd_tc(const __grid_constant__ CUt
   mbar_wait(&bar[2], 0);
   __syncwarp();
   tc_fence_after();
-  {  // tcgen05.ld is .sync.aligned: every lane loads, only rows t < S store
+  {  // tcgen05.ld is .sync.aligned: every lane loads, only rows t < S store; half hf stores dims 32hf..
     __nv_bfloat16* orow = a.Oout + ((int64_t)row0 + t) * a.H + hd * AD;
+    const float inv = lsum > 0.f ? 1.0f / lsum : 0.f;
+    float v[32];
+    tmem_ld32(trow + 32 * hf, v);
 #pragma unroll
-    for (int c = 0; c < 2; ++c) {
-      float v[32];
-      tmem_ld32(trow + 32 * c, v);
-      if (t < S) st_bf16x32(orow + 32 * c, v);
-    }
-    if (t < S) a.lse[((int64_t)b * a.h + hd) * S + t] = L;
+    for (int i = 0; i < 32; ++i) v[i] *= inv;
+    if (t < S) st_bf16x32(orow + 32 * hf, v);
+    if (t < S && hf == 0) a.lse[((int64_t)b * a.h + hd) * S + t] = (mrow + __log2f(lsum)) * 0.69314718055994531f;
   }
   tc_fence_before();
   __syncthreads();
@@ -173,8 +212,9 @@ __global__ void __launch_bounds__(128) k_attn_fwd_tc(const __grid_constant__ CUt
   }
 }
 
-__global__ void __launch_bounds__(128) k_attn_bwd_tc(const __grid_constant__ CUtensorMap tq,
+__global__ void __launch_bounds__(ATT, 2) k_attn_bwd_tc(const __grid_constant__ CUtensorMap tq,
                                                      const __grid_constant__ CUtensorMap tdo, const AttnArgs a) {
+  pdl_enter();
   extern __shared__ __align__(1024) uint8_t sm[];
   uint8_t* sQ = sm;
   uint8_t* sK = sm + TILE;
@@ -184,11 +224,14 @@ __global__ void __launch_bounds__(128) k_attn_bwd_tc(const __grid_constant__ CUt
   uint8_t* sdS = sm + 5 * TILE;
   uint64_t* bar = (uint64_t*)(sdS + PT);  // [0] tma, [1] mma S/dP, [2] mma grads
   uint32_t* tslot = (uint32_t*)(bar + 4);
-  const int t = threadIdx.x, warp = t >> 5;
+  float* red = (float*)sdS;               // [2][128] per-half partial of D (dS is written only after D is read)
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const int hf = warp >> 2, t = 32 * (warp & 3) + lane;
   const int bh = blockIdx.x, b = bh / a.h, hd = bh % a.h;
   const int S = a.S, len = a.lengths[b];
-  const int kmax = (S + 31) & ~31, nch = kmax >> 5;
-  if (t == 0) {
+  const int kmax = (S + 31) & ~31, nch = kmax >> 5, cmid = (nch + 1) >> 1;
+  const int c0 = hf ? cmid : 0, c1 = hf ? nch : cmid;
+  if (threadIdx.x == 0) {
     for (int i = 0; i < 3; ++i) mbar_init(&bar[i], 1);
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
   }
@@ -201,7 +244,7 @@ __global__ void __launch_bounds__(128) k_attn_bwd_tc(const __grid_constant__ CUt
   tc_fence_after();
   const uint32_t tmem = *tslot;
   const int row0 = b * S;
-  if (t == 0) {
+  if (threadIdx.x == 0) {
     mbar_expect_tx(&bar[0], 4 * TILE);
     tma_load_2d(&tq, &bar[0], sQ, hd * AD, row0);
     tma_load_2d(&tq, &bar[0], sK, a.H + hd * AD, row0);
@@ -219,59 +262,63 @@ __global__ void __launch_bounds__(128) k_attn_bwd_tc(const __grid_constant__ CUt
       mma_bf16(tmem + 128, make_desc(o0 + 32 * kk, 16, 1024), make_desc(v0 + 32 * kk, 16, 1024), id, kk > 0);
     mma_commit(&bar[1]);
   }
-  // D_t = rowsum(dO * O) for query row t (global reads overlap the MMAs)
-  float Dt = 0.f, Lt = 0.f;
+  // D_t = rowsum(dO * O) for query row t: half hf sums dims [32hf, 32hf+32)
+  // (global reads overlap the MMAs); D = half 0 + half 1
+  float Dh = 0.f, Lt = 0.f;
   if (t < len) {
-    const __nv_bfloat16* orow = a.O + ((int64_t)row0 + t) * a.H + hd * AD;
-    const __nv_bfloat16* drow = a.dO + ((int64_t)row0 + t) * a.H + hd * AD;
+    const __nv_bfloat16* orow = a.O + ((int64_t)row0 + t) * a.H + hd * AD + 32 * hf;
+    const __nv_bfloat16* drow = a.dO + ((int64_t)row0 + t) * a.H + hd * AD + 32 * hf;
     float ov[32], dv[32];
+    ld_bf16x32(orow, ov);
+    ld_bf16x32(drow, dv);
 #pragma unroll
-    for (int c = 0; c < 2; ++c) {
-      ld_bf16x32(orow + 32 * c, ov);
-      ld_bf16x32(drow + 32 * c, dv);
-#pragma unroll
-      for (int i = 0; i < 32; ++i) Dt += ov[i] * dv[i];
-    }
+    for (int i = 0; i < 32; ++i) Dh += ov[i] * dv[i];
     Lt = a.lse_in[((int64_t)b * a.h + hd) * S + t];
   }
+  red[hf * 128 + t] = Dh;
   mbar_wait(&bar[1], 0);
-  __syncwarp();
+  __syncthreads();                        // red[] complete; every thread is past the MMAs (V dead)
   tc_fence_after();
-  const uint32_t trow = tmem + ((uint32_t)(32 * warp) << 16);
+  const float Dt = red[t] + red[128 + t];
+  __syncthreads();                        // every D read before dS overwrites red[]
+  const uint32_t trow = tmem + ((uint32_t)(32 * (warp & 3)) << 16);
   const uint64_t ebase = (((uint64_t)b * a.h + hd) * S + (uint64_t)t) * S;
   const int kl = a.causal ? min(len, t + 1) : len;
-  // P~ overwrites V: wait until every thread is past the MMA (V is dead)
-  for (int c = 0; c < nch; ++c) {
-    float sv[32], dp[32];
-    tmem_ld32(trow + 32 * c, sv);
-    tmem_ld32(trow + 128 + 32 * c, dp);
-    const bool live = t < len && 32 * c < kl;    // padded / foreign query rows contribute 0
+  const float sl2 = a.scale * 1.4426950408889634f, Ll2 = Lt * 1.4426950408889634f;
+  for (int c = c0; c < c1; ++c)
+#pragma unroll
+  for (int hh = 0; hh < 2; ++hh) {
+    float sv[16], dp[16];
+    tmem_ld16(trow + 32 * c + 16 * hh, sv);
+    tmem_ld16(trow + 128 + 32 * c + 16 * hh, dp);
+    const int kb = 32 * c + 16 * hh;
+    const bool live = t < len && kb < kl;        // padded / foreign query rows contribute 0
     if (live) {
 #pragma unroll
-      for (int j = 0; j < 8; ++j) {
-        const int k = 32 * c + 4 * j;
+      for (int j = 0; j < 4; ++j) {
+        const int k = kb + 4 * j;
         const float4 f = (k < kl) ? drop4_or(a.drop, ebase + k) : make_float4(0.f, 0.f, 0.f, 0.f);
         const float ff[4] = {f.x, f.y, f.z, f.w};
 #pragma unroll
         for (int i = 0; i < 4; ++i) {
           const int kk = k + i;
-          const float p = (kk < kl) ? __expf(sv[4 * j + i] * a.scale - Lt) : 0.f;
+          const float p = (kk < kl) ? ex2f(fmaf(sv[4 * j + i], sl2, -Ll2)) : 0.f;
           sv[4 * j + i] = p * ff[i];                                  // P~
           dp[4 * j + i] = p * (dp[4 * j + i] * ff[i] - Dt) * a.scale; // dS (scale folded)
         }
       }
     } else {
 #pragma unroll
-      for (int i = 0; i < 32; ++i) { sv[i] = 0.f; dp[i] = 0.f; }
+      for (int i = 0; i < 16; ++i) { sv[i] = 0.f; dp[i] = 0.f; }
     }
-    st_tile_row32(sP, t, c, sv);
-    st_tile_row32(sdS, t, c, dp);
+    st_tile_row16(sP, t, c, hh, sv);
+    st_tile_row16(sdS, t, c, hh, dp);
   }
   fence_async_smem();
   tc_fence_before();
   __syncthreads();
   tc_fence_after();
-  if (t == 0) {
+  if (threadIdx.x == 0) {
     const uint32_t id_t = idesc_bf16(AQ, AD, 1, 1);   // A MN-major (keys), B MN-major (d)
     const uint32_t id_q = idesc_bf16(AQ, AD, 0, 1);   // A K-major (queries), B MN-major (d)
     const uint32_t p0 = smem_u32(sP), s0 = smem_u32(sdS);
@@ -292,19 +339,16 @@ __global__ void __launch_bounds__(128) k_attn_bwd_tc(const __grid_constant__ CUt
   mbar_wait(&bar[2], 0);
   __syncwarp();
   tc_fence_after();
-  {  // every lane loads (.sync.aligned); rows t < S store
-    __nv_bfloat16* row = a.dqkv + ((int64_t)row0 + t) * 3 * a.H + hd * AD;
+  {  // every lane loads (.sync.aligned); rows t < S store; half hf stores dims [32hf, 32hf+32)
+    __nv_bfloat16* row = a.dqkv + ((int64_t)row0 + t) * 3 * a.H + hd * AD + 32 * hf;
     const bool st = t < S;
-#pragma unroll
-    for (int c = 0; c < 2; ++c) {
-      float v[32];
-      tmem_ld32(trow + 128 + 32 * c, v);
-      if (st) st_bf16x32(row + 32 * c, v);                     // dQ
-      tmem_ld32(trow + 64 + 32 * c, v);
-      if (st) st_bf16x32(row + a.H + 32 * c, v);               // dK
-      tmem_ld32(trow + 32 * c, v);
-      if (st) st_bf16x32(row + 2 * a.H + 32 * c, v);           // dV
-    }
+    float v[32];
+    tmem_ld32(trow + 128 + 32 * hf, v);
+    if (st) st_bf16x32(row, v);                              // dQ
+    tmem_ld32(trow + 64 + 32 * hf, v);
+    if (st) st_bf16x32(row + a.H, v);                        // dK
+    tmem_ld32(trow + 32 * hf, v);
+    if (st) st_bf16x32(row + 2 * a.H, v);                    // dV
   }
   tc_fence_before();
   __syncthreads();
@@ -318,8 +362,8 @@ __global__ void __launch_bounds__(128) k_attn_bwd_tc(const __grid_constant__ CUt
 bool tc_map_bf16(CUtensorMap* out, const void* ptr, uint64_t inner, uint64_t outer, uint64_t stride_elems,
                  uint32_t box_inner, uint32_t box_outer);   // kernels_gemm_tc.cu
 
-constexpr int FWD_SMEM = 3 * TILE + 128;                  // P~ reuses Q/K
-constexpr int BWD_SMEM = 5 * TILE + PT + 128;             // P~ reuses V
+constexpr int FWD_SMEM = 3 * TILE + 64 + 1024 + 128;      // P~ reuses Q/K; + barriers, row partials
+constexpr int BWD_SMEM = 5 * TILE + PT + 128;             // P~ reuses V; D partials live in dS (2 CTAs / SM)
 
 bool attn_tc_ok(int S, int H, int h) { return S <= AQ && H / h == AD && H % 64 == 0; }
 
@@ -334,7 +378,7 @@ bool attn_fwd_tc(const void* qkv, const int32_t* lengths, void* O, float* lse, i
   a.S = S; a.H = H; a.h = h; a.B = B;
   a.scale = 1.0f / sqrtf((float)AD);
   a.drop = drop; a.lengths = lengths; a.Oout = (__nv_bfloat16*)O; a.lse = lse; a.causal = causal;
-  k_attn_fwd_tc<<<B * h, 128, FWD_SMEM, st>>>(tq, a);
+  launch_k(k_attn_fwd_tc, B * h, ATT, FWD_SMEM, st, tq, a);
   return true;
 }
 
@@ -351,7 +395,7 @@ bool attn_bwd_tc(const void* qkv, const void* O, const void* dO, const float* ls
   a.scale = 1.0f / sqrtf((float)AD);
   a.drop = drop; a.lengths = lengths; a.O = (const __nv_bfloat16*)O; a.dO = (const __nv_bfloat16*)dO;
   a.lse_in = lse; a.dqkv = (__nv_bfloat16*)dqkv; a.causal = causal;
-  k_attn_bwd_tc<<<B * h, 128, BWD_SMEM, st>>>(tq, tdo, a);
+  launch_k(k_attn_bwd_tc, B * h, ATT, BWD_SMEM, st, tq, tdo, a);
   return true;
 }
 

@@ -57,6 +57,7 @@ template <typename E>
 __global__ void __launch_bounds__(256) k_ln_fwd(const float* __restrict__ z, const E* __restrict__ g,
                                                 const E* __restrict__ b, E* __restrict__ y,
                                                 float2* __restrict__ st, int T, int H, float eps) {
+  pdl_enter();
   const int row = (blockIdx.x * blockDim.x + threadIdx.x) >> 5, lane = threadIdx.x & 31;
   if (row >= T) return;
   const int nch = H >> 3;
@@ -102,7 +103,7 @@ void ln_fwd(DType dt, const float* z, const void* g, const void* b, void* y, flo
   note_launch(1);
   dispatch(dt, [&](auto* tag) {
     using E = std::remove_pointer_t<decltype(tag)>;
-    k_ln_fwd<E><<<cdiv(T, 8), 256, 0, s>>>(z, (const E*)g, (const E*)b, (E*)y, st, T, H, eps);
+    launch_k(k_ln_fwd<E>, cdiv(T, 8), 256, 0, s, z, (const E*)g, (const E*)b, (E*)y, st, T, H, eps);
   });
 }
 
@@ -115,6 +116,7 @@ __global__ void __launch_bounds__(256) k_ln_bwd(const float* dy, Drop premask, c
                                                 float* dz, E* __restrict__ dtout, Drop mask,
                                                 float* __restrict__ pg, float* __restrict__ pb,
                                                 float* __restrict__ pbias, int T, int H, const float* res) {
+  pdl_enter();
   extern __shared__ float sm[];
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const int nch = H >> 3;
@@ -220,7 +222,7 @@ void ln_bwd(DType dt, const float* dy, Drop premask, const float* z, const float
       cudaFuncSetAttribute(k_ln_bwd<E>, cudaFuncAttributeMaxDynamicSharedMemorySize, 8 * 3 * 1024 * 4);
       attr = true;
     }
-    k_ln_bwd<E><<<NPART, 256, smem, s>>>(dy, premask, z, st, (const E*)g, dz, (E*)dtout,
+    launch_k(k_ln_bwd<E>, NPART, 256, smem, s, dy, premask, z, st, (const E*)g, dz, (E*)dtout,
                                          mask, pg, pb, pbias, T, H, res);
   });
 }
@@ -231,6 +233,7 @@ void ln_bwd(DType dt, const float* dy, Drop premask, const float* z, const float
 struct RedJob { const float* part; float* out; };
 struct RedJobs { RedJob j[3]; };
 __global__ void __launch_bounds__(1024) k_reduce_rows(RedJobs jobs, int rows, int64_t ld, int n) {
+  pdl_enter();
   __shared__ float sw[32][33];
   const RedJob jb = jobs.j[blockIdx.y];
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
@@ -259,13 +262,14 @@ void reduce_rows3(const float* p0, float* o0, const float* p1, float* o1, const 
   note_launch(1);
   RedJobs jobs{{{p0, o0}, {p1, o1}, {p2, o2}}};
   const int nj = p2 ? 3 : p1 ? 2 : 1;
-  k_reduce_rows<<<dim3(cdiv(n, 32), nj), 1024, 0, s>>>(jobs, rows, ld, n);
+  launch_k(k_reduce_rows, dim3(cdiv(n, 32), nj), 1024, 0, s, jobs, rows, ld, n);
 }
 void reduce_partials(const float* part, int64_t ld, int n, float* out, cudaStream_t s) {
   reduce_rows3(part, out, nullptr, nullptr, nullptr, nullptr, NPART, ld, n, s);
 }
 
 __global__ void k_splitk_reduce(const float* __restrict__ part, int splits, int64_t n, float* __restrict__ out) {
+  pdl_enter();
   for (int64_t i = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) * 4; i < n; i += (int64_t)gridDim.x * blockDim.x * 4) {
     float4 s = ((const float4*)(part + i))[0];
     for (int k = 1; k < splits; ++k) {
@@ -277,13 +281,14 @@ __global__ void k_splitk_reduce(const float* __restrict__ part, int splits, int6
 }
 void splitk_reduce(const float* part, int splits, int64_t n, float* out, cudaStream_t s) {
   note_launch(1);
-  k_splitk_reduce<<<592, 256, 0, s>>>(part, splits, n, out);
+  launch_k(k_splitk_reduce, 592, 256, 0, s, part, splits, n, out);
 }
 
 // column sums of X [T, N] (E): CTA (cx, p) owns rows p, p+NPART, ... and columns
 // [2048 cx, 2048 cx + 2048); a thread owns 8 consecutive columns.
 template <typename E>
 __global__ void __launch_bounds__(256) k_colsum(const E* __restrict__ X, int T, int N, float* __restrict__ part) {
+  pdl_enter();
   const int c = blockIdx.x * 2048 + threadIdx.x * 8;
   if (c >= N) return;
   float acc[8] = {0.f, 0.f, 0.f, 0.f, 0.f, 0.f, 0.f, 0.f};
@@ -299,7 +304,7 @@ void colsum(DType dt, const void* X, int T, int N, float* part, cudaStream_t s) 
   note_launch(1);
   dispatch(dt, [&](auto* tag) {
     using E = std::remove_pointer_t<decltype(tag)>;
-    k_colsum<E><<<dim3(cdiv(N, 2048), NPART), 256, 0, s>>>((const E*)X, T, N, part);
+    launch_k(k_colsum<E>, dim3(cdiv(N, 2048), NPART), 256, 0, s, (const E*)X, T, N, part);
   });
 }
 
@@ -307,6 +312,7 @@ void colsum(DType dt, const void* X, int T, int N, float* part, cudaStream_t s) 
 template <typename E>
 __global__ void __launch_bounds__(256) k_drop_cast_colsum(const float* __restrict__ in, Drop mask, E* __restrict__ out,
                                                           int T, int N, float* __restrict__ part) {
+  pdl_enter();
   const int c = blockIdx.x * 2048 + threadIdx.x * 8;
   if (c >= N) return;
   float acc[8] = {0.f, 0.f, 0.f, 0.f, 0.f, 0.f, 0.f, 0.f};
@@ -326,11 +332,12 @@ void drop_cast_colsum(DType dt, const float* in, Drop mask, void* out, int T, in
   note_launch(1);
   dispatch(dt, [&](auto* tag) {
     using E = std::remove_pointer_t<decltype(tag)>;
-    k_drop_cast_colsum<E><<<dim3(cdiv(N, 2048), NPART), 256, 0, s>>>(in, mask, (E*)out, T, N, part);
+    launch_k(k_drop_cast_colsum<E>, dim3(cdiv(N, 2048), NPART), 256, 0, s, in, mask, (E*)out, T, N, part);
   });
 }
 
 __global__ void k_drop_f32(const float* __restrict__ in, Drop mask, float* __restrict__ out, int64_t n) {
+  pdl_enter();
   for (int64_t i = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) * 8; i < n; i += (int64_t)gridDim.x * blockDim.x * 8) {
     float v[8], f[8];
     ld8(in + i, v);
@@ -342,7 +349,7 @@ __global__ void k_drop_f32(const float* __restrict__ in, Drop mask, float* __res
 }
 void drop_f32(const float* in, Drop mask, float* out, int64_t n, cudaStream_t s) {
   note_launch(1);
-  k_drop_f32<<<592, 256, 0, s>>>(in, mask, out, n);
+  launch_k(k_drop_f32, 592, 256, 0, s, in, mask, out, n);
 }
 
 // ============================================================== embedding ===
@@ -354,6 +361,7 @@ __global__ void __launch_bounds__(256) k_embed_fwd(const int32_t* __restrict__ i
                                                    const E* __restrict__ b, float* __restrict__ z0,
                                                    float2* __restrict__ st0, E* __restrict__ x1, int T,
                                                    int S, int H, int pos_offset, float eps, Drop drop) {
+  pdl_enter();
   const int t = (blockIdx.x * blockDim.x + threadIdx.x) >> 5, lane = threadIdx.x & 31;
   if (t >= T) return;
   const int s = t % S;
@@ -395,7 +403,7 @@ void embed_fwd(DType dt, const int32_t* ids, const int32_t* tt, const void* Ww, 
   note_launch(1);
   dispatch(dt, [&](auto* tag) {
     using E = std::remove_pointer_t<decltype(tag)>;
-    k_embed_fwd<E><<<cdiv(T, 8), 256, 0, s>>>(ids, tt, (const E*)Ww, (const E*)Wp, (const E*)Wt,
+    launch_k(k_embed_fwd<E>, cdiv(T, 8), 256, 0, s, ids, tt, (const E*)Ww, (const E*)Wp, (const E*)Wt,
                                               (const E*)g, (const E*)b, z0, st0, (E*)x1, T, S, H,
                                               pos_offset, eps, drop);
   });
@@ -404,6 +412,7 @@ void embed_fwd(DType dt, const int32_t* ids, const int32_t* tt, const void* Ww, 
 // partials [NPART][TV*H]; CTA p owns rows p, p+NPART, ...
 __global__ void __launch_bounds__(256) k_type_part(const float* __restrict__ dz0, const int32_t* __restrict__ tt,
                                                    int T, int H, int TV, float* __restrict__ part) {
+  pdl_enter();
   float acc[4][4];
 #pragma unroll
   for (int k = 0; k < 4; ++k)
@@ -430,13 +439,14 @@ __global__ void __launch_bounds__(256) k_type_part(const float* __restrict__ dz0
 }
 void type_grad(const float* dz0, const int32_t* tt, int T, int H, int TV, float* part, float* dWt, cudaStream_t s) {
   note_launch(1);
-  k_type_part<<<NPART, 256, 0, s>>>(dz0, tt, T, H, TV, part);
+  launch_k(k_type_part, NPART, 256, 0, s, dz0, tt, T, H, TV, part);
   reduce_partials(part, (int64_t)TV * H, TV * H, dWt, s);
 }
 
 template <typename E>
 __global__ void k_embed_fwd_pre(const int32_t* __restrict__ ids, const E* __restrict__ Ww, const E* __restrict__ Wp,
                                 float* __restrict__ x1, int T, int S, int H, int pos_offset, Drop drop) {
+  pdl_enter();
   const int64_t i = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) * 8;
   if (i >= (int64_t)T * H) return;
   const int t = (int)(i / H), c = (int)(i % H);
@@ -454,13 +464,14 @@ void embed_fwd_pre(DType dt, const int32_t* ids, const void* Ww, const void* Wp,
   const int T = B * S;
   dispatch(dt, [&](auto* tag) {
     using E = std::remove_pointer_t<decltype(tag)>;
-    k_embed_fwd_pre<E><<<cdiv((int64_t)T * H / 8, 256), 256, 0, s>>>(ids, (const E*)Ww, (const E*)Wp, x1, T, S, H,
+    launch_k(k_embed_fwd_pre<E>, cdiv((int64_t)T * H / 8, 256), 256, 0, s, ids, (const E*)Ww, (const E*)Wp, x1, T, S, H,
                                                                      pos_offset, drop);
   });
 }
 
 __global__ void k_pos_grad(const float* __restrict__ dz0, int B, int S, int H, int pos_offset,
                            float* __restrict__ dWp) {
+  pdl_enter();
   const int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
   if (i >= (int64_t)S * H) return;
   const int s = (int)(i / H), c = (int)(i % H);
@@ -470,12 +481,13 @@ __global__ void k_pos_grad(const float* __restrict__ dz0, int B, int S, int H, i
 }
 void pos_grad(const float* dz0, int B, int S, int H, int pos_offset, float* dWp, cudaStream_t s) {
   note_launch(1);
-  k_pos_grad<<<cdiv((int64_t)S * H, 256), 256, 0, s>>>(dz0, B, S, H, pos_offset, dWp);
+  launch_k(k_pos_grad, cdiv((int64_t)S * H, 256), 256, 0, s, dz0, B, S, H, pos_offset, dWp);
 }
 
 // ---- stable LSD radix sort of (key, token) pairs, 8-bit digits, 1024-key tiles ----
 __global__ void __launch_bounds__(1024) k_rs_hist(const int32_t* __restrict__ keys, int T, int shift,
                                                   int ntiles, int32_t* __restrict__ hist) {
+  pdl_enter();
   __shared__ int h[256];
   if (threadIdx.x < 256) h[threadIdx.x] = 0;
   __syncthreads();
@@ -487,6 +499,7 @@ __global__ void __launch_bounds__(1024) k_rs_hist(const int32_t* __restrict__ ke
 
 // exclusive scan of n <= 8192 ints, one CTA of 1024 threads, 8 per thread
 __global__ void __launch_bounds__(1024) k_rs_scan(int32_t* __restrict__ a, int n) {
+  pdl_enter();
   __shared__ int ws[32];
   int v[8], s = 0;
   const int base = threadIdx.x * 8;
@@ -516,6 +529,7 @@ __global__ void __launch_bounds__(1024) k_rs_scan(int32_t* __restrict__ a, int n
 __global__ void __launch_bounds__(1024) k_rs_scatter(const int32_t* __restrict__ kin, const int32_t* __restrict__ vin,
                                                      int T, int shift, int ntiles, const int32_t* __restrict__ off,
                                                      int32_t* __restrict__ kout, int32_t* __restrict__ vout) {
+  pdl_enter();
   __shared__ int wc[32][257];
   const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
   for (int i = threadIdx.x; i < 32 * 257; i += 1024) (&wc[0][0])[i] = 0;
@@ -546,6 +560,7 @@ __global__ void __launch_bounds__(1024) k_rs_scatter(const int32_t* __restrict__
 // Keys equal to `skip` (the pad id) are ignored.
 __global__ void __launch_bounds__(256) k_piece_sum(const int32_t* __restrict__ keys, const int32_t* __restrict__ tok,
                                                    float* X, int T, int H, int skip) {
+  pdl_enter();
   const int chunk = (blockIdx.x * blockDim.x + threadIdx.x) >> 5, lane = threadIdx.x & 31;
   const int r0 = chunk * 32;
   if (r0 >= T) return;
@@ -583,6 +598,7 @@ __global__ void __launch_bounds__(256) k_piece_sum(const int32_t* __restrict__ k
 __global__ void __launch_bounds__(256) k_segment_sum(const int32_t* __restrict__ keys, const int32_t* __restrict__ tok,
                                                      const float* __restrict__ X, int T, int H, float* __restrict__ out,
                                                      int skip, int accumulate) {
+  pdl_enter();
   const int r = (blockIdx.x * blockDim.x + threadIdx.x) >> 5, lane = threadIdx.x & 31;
   if (r >= T) return;
   const int key = keys[r];
@@ -624,16 +640,16 @@ void keyed_rowsum(const int32_t* keys, int key_bits, float* X, int T, int H, flo
   for (int p = 0; p < passes; ++p) {
     int32_t* ko = (p == 0) ? kB : kA;
     int32_t* vo = (p == 0) ? vB : vA;
-    k_rs_hist<<<ntiles, 1024, 0, s>>>(kin, T, 8 * p, ntiles, hist);
-    k_rs_scan<<<1, 1024, 0, s>>>(hist, 256 * ntiles);
-    k_rs_scatter<<<ntiles, 1024, 0, s>>>(kin, vin, T, 8 * p, ntiles, hist, ko, vo);
+    launch_k(k_rs_hist, ntiles, 1024, 0, s, kin, T, 8 * p, ntiles, hist);
+    launch_k(k_rs_scan, 1, 1024, 0, s, hist, 256 * ntiles);
+    launch_k(k_rs_scatter, ntiles, 1024, 0, s, kin, vin, T, 8 * p, ntiles, hist, ko, vo);
     kin = ko;
     vin = vo;
   }
   (void)max_tiles;
   note_launch(3 * passes + 2);
-  k_piece_sum<<<cdiv(cdiv(T, 32), 8), 256, 0, s>>>(kin, vin, X, T, H, skip);
-  k_segment_sum<<<cdiv(T, 8), 256, 0, s>>>(kin, vin, X, T, H, out, skip, accumulate ? 1 : 0);
+  launch_k(k_piece_sum, cdiv(cdiv(T, 32), 8), 256, 0, s, kin, vin, X, T, H, skip);
+  launch_k(k_segment_sum, cdiv(T, 8), 256, 0, s, kin, vin, X, T, H, out, skip, accumulate ? 1 : 0);
 }
 
 // ================================================================== heads ===
@@ -641,6 +657,7 @@ void keyed_rowsum(const int32_t* keys, int key_bits, float* X, int T, int H, flo
 template <typename E>
 __global__ void k_pool_fwd(const E* __restrict__ y, int B, int S, int H, const E* __restrict__ Wp,
                            const E* __restrict__ bp, E* __restrict__ p) {
+  pdl_enter();
   const int w = (blockIdx.x * blockDim.x + threadIdx.x) >> 5, lane = threadIdx.x & 31;
   if (w >= B * H) return;
   const int b = w / H, j = w % H;
@@ -655,6 +672,7 @@ __global__ void k_pool_fwd(const E* __restrict__ y, int B, int S, int H, const E
 template <typename E>
 __global__ void k_cls_fwd(const E* __restrict__ p, int B, int H, const E* __restrict__ Wc,
                           const E* __restrict__ bc, int n_out, float* __restrict__ logits, Drop drop) {
+  pdl_enter();
   const int w = (blockIdx.x * blockDim.x + threadIdx.x) >> 5, lane = threadIdx.x & 31;
   if (w >= B * n_out) return;
   const int b = w / n_out, o = w % n_out;
@@ -674,6 +692,7 @@ __device__ void ce_view(int head_kind, int B, int n_out, int n_choices, int& row
 __global__ void k_cls_ce(const float* __restrict__ logits, const int32_t* __restrict__ labels, int B,
                          int n_out, int n_choices, int head_kind, float* __restrict__ loss,
                          float* __restrict__ dlog) {
+  pdl_enter();
   int rows, cols;
   ce_view(head_kind, B, n_out, n_choices, rows, cols);
   const int lane = threadIdx.x;
@@ -702,33 +721,56 @@ void head_cls_fwd(DType dt, const void* y, int B, int S, int H, const void* Wp, 
   note_launch(3);
   dispatch(dt, [&](auto* tag) {
     using E = std::remove_pointer_t<decltype(tag)>;
-    k_pool_fwd<E><<<cdiv((int64_t)B * H, 8), 256, 0, s>>>((const E*)y, B, S, H, (const E*)Wp, (const E*)bp, (E*)p);
-    k_cls_fwd<E><<<cdiv((int64_t)B * n_out, 8), 256, 0, s>>>((const E*)p, B, H, (const E*)Wc, (const E*)bc, n_out, logits, drop);
+    launch_k(k_pool_fwd<E>, cdiv((int64_t)B * H, 8), 256, 0, s, (const E*)y, B, S, H, (const E*)Wp, (const E*)bp, (E*)p);
+    launch_k(k_cls_fwd<E>, cdiv((int64_t)B * n_out, 8), 256, 0, s, (const E*)p, B, H, (const E*)Wc, (const E*)bc, n_out, logits, drop);
   });
-  k_cls_ce<<<1, 32, 0, s>>>(logits, labels, B, n_out, n_choices, head_kind, loss, nullptr);
+  launch_k(k_cls_ce, 1, 32, 0, s, logits, labels, B, n_out, n_choices, head_kind, loss, nullptr);
 }
 
+// dWc[o, j] = sum_b dlog[b, o] * drop(p)[b, j], dbc[o] = sum_b dlog[b, o].
+// Block: 128 columns (lane owns 4 consecutive j, one Philox call per 4), warp w
+// sums b = w, w+8, ... ascending; the 8 warp sums are added in warp order.
 template <typename E>
-__global__ void k_cls_wgrad(const float* __restrict__ dlog, const E* __restrict__ p, int B, int H, int n_out,
-                            float* __restrict__ dWc, float* __restrict__ dbc, Drop drop) {
-  const int i = blockIdx.x * blockDim.x + threadIdx.x;
-  if (i < n_out * H) {
-    const int o = i / H, j = i % H;
-    float acc = 0.f;
-    for (int b = 0; b < B; ++b)
-      acc += dlog[b * n_out + o] * ldf(p + (int64_t)b * H + j) * drop_factor(drop, (uint64_t)b * H + j);
-    dWc[i] = acc;
+__global__ void __launch_bounds__(256) k_cls_wgrad(const float* __restrict__ dlog, const E* __restrict__ p, int B,
+                                                   int H, int n_out, float* __restrict__ dWc, float* __restrict__ dbc,
+                                                   Drop drop) {
+  pdl_enter();
+  __shared__ float4 red[8][32];
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const int nblk = (H + 127) / 128;
+  const int o = blockIdx.x / nblk, j = (blockIdx.x % nblk) * 128 + 4 * lane;
+  float4 acc = make_float4(0.f, 0.f, 0.f, 0.f);
+  if (j < H)
+    for (int b = warp; b < B; b += 8) {
+      const float d = dlog[b * n_out + o];
+      const float4 f = drop_factor4(drop, ((uint64_t)b * H + j) >> 2);
+      acc.x += d * ldf(p + (int64_t)b * H + j) * f.x;
+      acc.y += d * ldf(p + (int64_t)b * H + j + 1) * f.y;
+      acc.z += d * ldf(p + (int64_t)b * H + j + 2) * f.z;
+      acc.w += d * ldf(p + (int64_t)b * H + j + 3) * f.w;
+    }
+  red[warp][lane] = acc;
+  __syncthreads();
+  if (warp == 0 && j < H) {
+    float4 t = red[0][lane];
+    for (int w = 1; w < 8; ++w) {
+      const float4 v = red[w][lane];
+      t.x += v.x; t.y += v.y; t.z += v.z; t.w += v.w;
+    }
+    float* out = dWc + (int64_t)o * H + j;
+    out[0] = t.x; out[1] = t.y; out[2] = t.z; out[3] = t.w;
   }
-  if (i < n_out) {
-    float acc = 0.f;
-    for (int b = 0; b < B; ++b) acc += dlog[b * n_out + i];
-    dbc[i] = acc;
+  if (blockIdx.x % nblk == 0 && threadIdx.x == 0) {
+    float t = 0.f;
+    for (int b = 0; b < B; ++b) t += dlog[b * n_out + o];
+    dbc[o] = t;
   }
 }
 
 template <typename E>
 __global__ void k_pool_dpre(const float* __restrict__ dlog, const E* __restrict__ p, const E* __restrict__ Wc,
                             int B, int H, int n_out, float* __restrict__ dpre, Drop drop) {
+  pdl_enter();
   const int i = blockIdx.x * blockDim.x + threadIdx.x;
   if (i >= B * H) return;
   const int b = i / H, j = i % H;
@@ -738,32 +780,80 @@ __global__ void k_pool_dpre(const float* __restrict__ dlog, const E* __restrict_
   dpre[i] = acc * drop_factor(drop, (uint64_t)b * H + j) * (1.f - pv * pv);
 }
 
+// dWp[j, k] = sum_b dpre[b, j] y[b, 0, k] (b ascending); dbp[j] = sum_b dpre[b, j].
+// Block: 32 columns k (lane) x 64 rows j (warp w owns j0 + 8w .. +7); dpre's
+// [B x 64] slab is staged in shared memory.
 template <typename E>
-__global__ void k_pool_wgrad(const float* __restrict__ dpre, const E* __restrict__ y, int B, int S, int H,
-                             float* __restrict__ dWp, float* __restrict__ dbp) {
-  const int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
-  if (i < (int64_t)H * H) {
-    const int j = (int)(i / H), k = (int)(i % H);
-    float acc = 0.f;
-    for (int b = 0; b < B; ++b) acc += dpre[b * H + j] * ldf(y + (int64_t)b * S * H + k);
-    dWp[i] = acc;
+__global__ void __launch_bounds__(256) k_pool_wgrad(const float* __restrict__ dpre, const E* __restrict__ y, int B,
+                                                    int S, int H, float* __restrict__ dWp, float* __restrict__ dbp) {
+  pdl_enter();
+  extern __shared__ float sdp[];          // [B][64]
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const int k = blockIdx.x * 32 + lane, j0 = blockIdx.y * 64;
+  for (int i = threadIdx.x; i < B * 64; i += 256) {
+    const int b = i >> 6, jj = j0 + (i & 63);
+    sdp[i] = jj < H ? dpre[(int64_t)b * H + jj] : 0.f;
   }
-  if (i < H) {
-    float acc = 0.f;
-    for (int b = 0; b < B; ++b) acc += dpre[b * H + i];
-    dbp[i] = acc;
+  __syncthreads();
+  float acc[8];
+#pragma unroll
+  for (int r = 0; r < 8; ++r) acc[r] = 0.f;
+  if (k < H)
+    for (int b = 0; b < B; ++b) {
+      const float yv = ldf(y + (int64_t)b * S * H + k);
+      const float* d = sdp + b * 64 + 8 * warp;
+#pragma unroll
+      for (int r = 0; r < 8; ++r) acc[r] += d[r] * yv;
+    }
+#pragma unroll
+  for (int r = 0; r < 8; ++r) {
+    const int j = j0 + 8 * warp + r;
+    if (j < H && k < H) dWp[(int64_t)j * H + k] = acc[r];
+  }
+  if (blockIdx.x == 0) {
+    const int jj = threadIdx.x;
+    if (jj < 64 && j0 + jj < H) {
+      float t = 0.f;
+      for (int b = 0; b < B; ++b) t += sdp[b * 64 + jj];
+      dbp[j0 + jj] = t;
+    }
   }
 }
 
+// dy[b, 0, k] = sum_j dpre[b, j] Wp[j, k].  Block: 32 columns k (lane) x 8
+// sequences; warp w sums j in [w H/8, (w+1) H/8) ascending, and the 8 warp
+// partials are added in warp order.
 template <typename E>
-__global__ void k_pool_dx(const float* __restrict__ dpre, const E* __restrict__ Wp, int B, int S, int H,
-                          float* __restrict__ dy) {
-  const int i = blockIdx.x * blockDim.x + threadIdx.x;
-  if (i >= B * H) return;
-  const int b = i / H, k = i % H;
-  float acc = 0.f;
-  for (int j = 0; j < H; ++j) acc += dpre[b * H + j] * ldf(Wp + (int64_t)j * H + k);
-  dy[(int64_t)b * S * H + k] = acc;
+__global__ void __launch_bounds__(256) k_pool_dx(const float* __restrict__ dpre, const E* __restrict__ Wp, int B,
+                                                 int S, int H, float* __restrict__ dy) {
+  pdl_enter();
+  __shared__ float red[8][8][33];
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const int k = blockIdx.x * 32 + lane, b0 = blockIdx.y * 8;
+  const int jb = warp * H / 8, je = (warp + 1) * H / 8;
+  float acc[8];
+#pragma unroll
+  for (int r = 0; r < 8; ++r) acc[r] = 0.f;
+  if (k < H) {
+#pragma unroll 4
+    for (int j = jb; j < je; ++j) {
+      const float w = ldf(Wp + (int64_t)j * H + k);
+#pragma unroll
+      for (int r = 0; r < 8; ++r)
+        if (b0 + r < B) acc[r] += dpre[(int64_t)(b0 + r) * H + j] * w;
+    }
+  }
+#pragma unroll
+  for (int r = 0; r < 8; ++r) red[warp][r][lane] = acc[r];
+  __syncthreads();
+  if (warp == 0 && k < H) {
+    for (int r = 0; r < 8; ++r) {
+      if (b0 + r >= B) break;
+      float t = red[0][r][lane];
+      for (int w = 1; w < 8; ++w) t += red[w][r][lane];
+      dy[(int64_t)(b0 + r) * S * H + k] = t;
+    }
+  }
 }
 
 void head_cls_bwd(DType dt, const void* y, int B, int S, int H, const void* Wp, const void* Wc, int n_out,
@@ -773,13 +863,14 @@ void head_cls_bwd(DType dt, const void* y, int B, int S, int H, const void* Wp, 
   float* dlog = scratch;
   note_launch(5);
   float* dpre = scratch + ((B * n_out + 3) / 4 * 4) + (int64_t)B * H;
-  k_cls_ce<<<1, 32, 0, s>>>(logits, labels, B, n_out, n_choices, head_kind, nullptr, dlog);
+  launch_k(k_cls_ce, 1, 32, 0, s, logits, labels, B, n_out, n_choices, head_kind, nullptr, dlog);
   dispatch(dt, [&](auto* tag) {
     using E = std::remove_pointer_t<decltype(tag)>;
-    k_cls_wgrad<E><<<cdiv(n_out * H, 256), 256, 0, s>>>(dlog, (const E*)p, B, H, n_out, dWc, dbc, drop);
-    k_pool_dpre<E><<<cdiv(B * H, 256), 256, 0, s>>>(dlog, (const E*)p, (const E*)Wc, B, H, n_out, dpre, drop);
-    k_pool_wgrad<E><<<cdiv((int64_t)H * H, 256), 256, 0, s>>>(dpre, (const E*)y, B, S, H, dWp, dbp);
-    k_pool_dx<E><<<cdiv(B * H, 256), 256, 0, s>>>(dpre, (const E*)Wp, B, S, H, dy);
+    launch_k(k_cls_wgrad<E>, n_out * cdiv(H, 128), 256, 0, s, dlog, (const E*)p, B, H, n_out, dWc, dbc, drop);
+    launch_k(k_pool_dpre<E>, cdiv(B * H, 256), 256, 0, s, dlog, (const E*)p, (const E*)Wc, B, H, n_out, dpre, drop);
+    launch_k(k_pool_wgrad<E>, dim3(cdiv(H, 32), cdiv(H, 64)), 256, (size_t)B * 64 * 4, s, dpre, (const E*)y, B, S,
+             H, dWp, dbp);
+    launch_k(k_pool_dx<E>, dim3(cdiv(H, 32), cdiv(B, 8)), 256, 0, s, dpre, (const E*)Wp, B, S, H, dy);
   });
 }
 
@@ -787,6 +878,7 @@ void head_cls_bwd(DType dt, const void* y, int B, int S, int H, const void* Wp, 
 template <typename E>
 __global__ void k_qa_logits(const E* __restrict__ y, int T, int H, const E* __restrict__ Wq,
                             const E* __restrict__ bq, float* __restrict__ logits) {
+  pdl_enter();
   const int t = (blockIdx.x * blockDim.x + threadIdx.x) >> 5, lane = threadIdx.x & 31;
   if (t >= T) return;
   float a0 = 0.f, a1 = 0.f;
@@ -804,6 +896,7 @@ __global__ void k_qa_logits(const E* __restrict__ y, int T, int H, const E* __re
 __global__ void k_qa_ce(const float* __restrict__ logits, const int32_t* __restrict__ lengths,
                         const int32_t* __restrict__ labels, int B, int S, float* __restrict__ loss,
                         float* __restrict__ dlog) {
+  pdl_enter();
   const int lane = threadIdx.x;
   float tot[2] = {0.f, 0.f};
   for (int b = 0; b < B; ++b) {
@@ -833,13 +926,14 @@ void head_qa_fwd(DType dt, const void* y, int B, int S, int H, const void* Wq, c
   note_launch(2);
   dispatch(dt, [&](auto* tag) {
     using E = std::remove_pointer_t<decltype(tag)>;
-    k_qa_logits<E><<<cdiv(T, 8), 256, 0, s>>>((const E*)y, T, H, (const E*)Wq, (const E*)bq, logits);
+    launch_k(k_qa_logits<E>, cdiv(T, 8), 256, 0, s, (const E*)y, T, H, (const E*)Wq, (const E*)bq, logits);
   });
-  k_qa_ce<<<1, 32, 0, s>>>(logits, lengths, labels, B, S, loss, nullptr);
+  launch_k(k_qa_ce, 1, 32, 0, s, logits, lengths, labels, B, S, loss, nullptr);
 }
 
 template <typename E>
 __global__ void k_qa_dx(const float* __restrict__ dlog, const E* __restrict__ Wq, int T, int H, float* __restrict__ dy) {
+  pdl_enter();
   const int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
   if (i >= (int64_t)T * H) return;
   const int t = (int)(i / H), c = (int)(i % H);
@@ -850,6 +944,7 @@ __global__ void k_qa_dx(const float* __restrict__ dlog, const E* __restrict__ Wq
 template <typename E>
 __global__ void k_qa_wgrad_part(const float* __restrict__ dlog, const E* __restrict__ y, int T, int H,
                                 float* __restrict__ part) {
+  pdl_enter();
   const int ld = 2 * H + 2;
   for (int c = threadIdx.x; c < ld; c += blockDim.x) {
     float acc = 0.f;
@@ -866,11 +961,11 @@ void head_qa_bwd(DType dt, const void* y, int B, int S, int H, const void* Wq, c
                  float* dbq, float* dy, cudaStream_t s) {
   const int T = B * S;
   note_launch(3);
-  k_qa_ce<<<1, 32, 0, s>>>(logits, lengths, labels, B, S, nullptr, dlog);
+  launch_k(k_qa_ce, 1, 32, 0, s, logits, lengths, labels, B, S, nullptr, dlog);
   dispatch(dt, [&](auto* tag) {
     using E = std::remove_pointer_t<decltype(tag)>;
-    k_qa_dx<E><<<cdiv((int64_t)T * H, 256), 256, 0, s>>>(dlog, (const E*)Wq, T, H, dy);
-    k_qa_wgrad_part<E><<<NPART, 256, 0, s>>>(dlog, (const E*)y, T, H, part);
+    launch_k(k_qa_dx<E>, cdiv((int64_t)T * H, 256), 256, 0, s, dlog, (const E*)Wq, T, H, dy);
+    launch_k(k_qa_wgrad_part<E>, NPART, 256, 0, s, dlog, (const E*)y, T, H, part);
   });
   reduce_partials(part, 2 * H + 2, 2 * H, dWq, s);
   reduce_partials(part + 2 * H, 2 * H + 2, 2, dbq, s);
@@ -904,6 +999,7 @@ MDEV bool lm_target(const int32_t* ids, const int32_t* lengths, int S, int t, in
 __global__ void __launch_bounds__(1024) k_lm_ce_fwd(const float* __restrict__ logits, int64_t ldv, int V, int row0,
                                                     const int32_t* __restrict__ ids, const int32_t* __restrict__ lengths,
                                                     int S, float2* __restrict__ tokstat) {
+  pdl_enter();
   __shared__ float sh[33];
   const int r = blockIdx.x, t = row0 + r;
   const float* lr = logits + (int64_t)r * ldv;
@@ -923,11 +1019,12 @@ __global__ void __launch_bounds__(1024) k_lm_ce_fwd(const float* __restrict__ lo
 void lm_ce_fwd(const float* logits, int64_t ldv, int V, int row0, int nrows, const int32_t* ids,
                const int32_t* lengths, int S, float2* tokstat, cudaStream_t s) {
   note_launch(1);
-  k_lm_ce_fwd<<<nrows, 1024, 0, s>>>(logits, ldv, V, row0, ids, lengths, S, tokstat);
+  launch_k(k_lm_ce_fwd, nrows, 1024, 0, s, logits, ldv, V, row0, ids, lengths, S, tokstat);
 }
 
 __global__ void __launch_bounds__(1024) k_lm_loss(const float2* __restrict__ tokstat, int T,
                                                   const int32_t* __restrict__ lengths, int B, float* __restrict__ loss) {
+  pdl_enter();
   __shared__ float sh[33];
   float a = 0.f;
   for (int t = threadIdx.x; t < T; t += blockDim.x) a += tokstat[t].y;
@@ -940,13 +1037,14 @@ __global__ void __launch_bounds__(1024) k_lm_loss(const float2* __restrict__ tok
 void lm_loss(const float2* tokstat, int T, const int32_t* lengths, int B, int S, float* loss, cudaStream_t s) {
   (void)S;
   note_launch(1);
-  k_lm_loss<<<1, 1024, 0, s>>>(tokstat, T, lengths, B, loss);
+  launch_k(k_lm_loss, 1, 1024, 0, s, tokstat, T, lengths, B, loss);
 }
 
 template <typename E>
 __global__ void __launch_bounds__(256) k_lm_ce_bwd(const float* __restrict__ logits, int64_t ldv, int V, int row0,
                                                    const int32_t* __restrict__ ids, const int32_t* __restrict__ lengths,
                                                    int B, int S, const float2* __restrict__ tokstat, E* __restrict__ dlog) {
+  pdl_enter();
   __shared__ float inv_n;
   if (threadIdx.x == 0) {
     int nv = 0;
@@ -968,7 +1066,7 @@ void lm_ce_bwd(DType dt, const float* logits, int64_t ldv, int V, int row0, int 
   note_launch(1);
   dispatch(dt, [&](auto* tag) {
     using E = std::remove_pointer_t<decltype(tag)>;
-    k_lm_ce_bwd<E><<<nrows, 256, 0, s>>>(logits, ldv, V, row0, ids, lengths, B, S, tokstat, (E*)dlog);
+    launch_k(k_lm_ce_bwd<E>, nrows, 256, 0, s, logits, ldv, V, row0, ids, lengths, B, S, tokstat, (E*)dlog);
   });
 }
 
@@ -978,6 +1076,7 @@ template <typename E>
 __global__ void __launch_bounds__(256) k_adamw(E* __restrict__ w, float* __restrict__ master, const float* __restrict__ g,
                                                float* __restrict__ m, float* __restrict__ v, int64_t n, float lr, float b1,
                                                float b2, float eps, float wd, float bc1, float bc2, float gs) {
+  pdl_enter();
   const float step = lr / bc1, rb2 = 1.0f / sqrtf(bc2), decay = 1.0f - lr * wd;
   for (int64_t i = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) * 4; i < n;
        i += (int64_t)gridDim.x * blockDim.x * 4) {
@@ -1013,17 +1112,19 @@ void adamw(DType dt, void* w, float* master, const float* g, float* m, float* v,
   note_launch(1);
   dispatch(dt, [&](auto* tag) {
     using E = std::remove_pointer_t<decltype(tag)>;
-    k_adamw<E><<<148 * 8, 256, 0, s>>>((E*)w, master, g, m, v, n, lr, b1, b2, eps, wd, bc1, bc2, gs);
+    launch_k(k_adamw<E>, 148 * 8, 256, 0, s, (E*)w, master, g, m, v, n, lr, b1, b2, eps, wd, bc1, bc2, gs);
   });
 }
 
 template <typename E>
 __global__ void k_cast_from(const float* __restrict__ src, E* __restrict__ dst, int64_t n) {
+  pdl_enter();
   for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x)
     stf(dst + i, src[i]);
 }
 template <typename E>
 __global__ void k_cast_to(const E* __restrict__ src, float* __restrict__ dst, int64_t n) {
+  pdl_enter();
   for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x)
     dst[i] = ldf(src + i);
 }
@@ -1031,14 +1132,14 @@ void cast_from_f32(DType dt, const float* src, void* dst, int64_t n, cudaStream_
   note_launch(1);
   dispatch(dt, [&](auto* tag) {
     using E = std::remove_pointer_t<decltype(tag)>;
-    k_cast_from<E><<<592, 256, 0, s>>>(src, (E*)dst, n);
+    launch_k(k_cast_from<E>, 592, 256, 0, s, src, (E*)dst, n);
   });
 }
 void cast_to_f32(DType dt, const void* src, float* dst, int64_t n, cudaStream_t s) {
   note_launch(1);
   dispatch(dt, [&](auto* tag) {
     using E = std::remove_pointer_t<decltype(tag)>;
-    k_cast_to<E><<<592, 256, 0, s>>>((const E*)src, dst, n);
+    launch_k(k_cast_to<E>, 592, 256, 0, s, (const E*)src, dst, n);
   });
 }
 

@@ -22,6 +22,7 @@ constexpr int SBM = 64, SBN = 64, SBK = 16;
 
 template <typename E, int EPI>
 __global__ void __launch_bounds__(256) k_gemm_simt(const GemmArgs g) {
+  pdl_enter();
   __shared__ float As[SBK][SBM + 4];
   __shared__ float Bs[SBK][SBN + 4];
   const int tid = threadIdx.x, tx = tid % 16, ty = tid / 16;
@@ -69,17 +70,17 @@ template <typename E>
 static void launch_simt(Epi epi, const GemmArgs& g, cudaStream_t st) {
   dim3 grid(cdiv(g.N, SBN), cdiv(g.M, SBM), g.split);
   switch (epi) {
-    case EPI_STORE: k_gemm_simt<E, EPI_STORE><<<grid, 256, 0, st>>>(g); break;
-    case EPI_BIAS: k_gemm_simt<E, EPI_BIAS><<<grid, 256, 0, st>>>(g); break;
-    case EPI_BIAS_GELU: k_gemm_simt<E, EPI_BIAS_GELU><<<grid, 256, 0, st>>>(g); break;
-    case EPI_BIAS_DROP_RES: k_gemm_simt<E, EPI_BIAS_DROP_RES><<<grid, 256, 0, st>>>(g); break;
-    case EPI_GELU_BWD: k_gemm_simt<E, EPI_GELU_BWD><<<grid, 256, 0, st>>>(g); break;
-    case EPI_ACC_RES_F32: k_gemm_simt<E, EPI_ACC_RES_F32><<<grid, 256, 0, st>>>(g); break;
-    case EPI_BIAS_GELUT: k_gemm_simt<E, EPI_BIAS_GELUT><<<grid, 256, 0, st>>>(g); break;
-    case EPI_GELUT_BWD: k_gemm_simt<E, EPI_GELUT_BWD><<<grid, 256, 0, st>>>(g); break;
-    case EPI_BIAS_DROP_RESF32: k_gemm_simt<E, EPI_BIAS_DROP_RESF32><<<grid, 256, 0, st>>>(g); break;
-    case EPI_ACC_F32: k_gemm_simt<E, EPI_ACC_F32><<<grid, 256, 0, st>>>(g); break;
-    default: k_gemm_simt<E, EPI_F32><<<grid, 256, 0, st>>>(g); break;
+    case EPI_STORE: launch_k(k_gemm_simt<E, EPI_STORE>, grid, 256, 0, st, g); break;
+    case EPI_BIAS: launch_k(k_gemm_simt<E, EPI_BIAS>, grid, 256, 0, st, g); break;
+    case EPI_BIAS_GELU: launch_k(k_gemm_simt<E, EPI_BIAS_GELU>, grid, 256, 0, st, g); break;
+    case EPI_BIAS_DROP_RES: launch_k(k_gemm_simt<E, EPI_BIAS_DROP_RES>, grid, 256, 0, st, g); break;
+    case EPI_GELU_BWD: launch_k(k_gemm_simt<E, EPI_GELU_BWD>, grid, 256, 0, st, g); break;
+    case EPI_ACC_RES_F32: launch_k(k_gemm_simt<E, EPI_ACC_RES_F32>, grid, 256, 0, st, g); break;
+    case EPI_BIAS_GELUT: launch_k(k_gemm_simt<E, EPI_BIAS_GELUT>, grid, 256, 0, st, g); break;
+    case EPI_GELUT_BWD: launch_k(k_gemm_simt<E, EPI_GELUT_BWD>, grid, 256, 0, st, g); break;
+    case EPI_BIAS_DROP_RESF32: launch_k(k_gemm_simt<E, EPI_BIAS_DROP_RESF32>, grid, 256, 0, st, g); break;
+    case EPI_ACC_F32: launch_k(k_gemm_simt<E, EPI_ACC_F32>, grid, 256, 0, st, g); break;
+    default: launch_k(k_gemm_simt<E, EPI_F32>, grid, 256, 0, st, g); break;
   }
 }
 
@@ -87,6 +88,14 @@ void gemm(DType dt, Epi epi, const GemmArgs& g, cudaStream_t st, bool use_tc) {
   if (g.M <= 0 || g.N <= 0) return;
   note_launch(1);
   if (use_tc && dt == DT_BF16 && gemm_tc(epi, g, st)) return;
+  if (g.fused_split) {          // SIMT: one pass over all of K straight into C
+    GemmArgs g1 = g;
+    g1.fused_split = 0;
+    g1.split = 1;
+    if (dt == DT_F32) launch_simt<float>(epi, g1, st);
+    else launch_simt<__nv_bfloat16>(epi, g1, st);
+    return;
+  }
   if (dt == DT_F32) launch_simt<float>(epi, g, st);
   else launch_simt<__nv_bfloat16>(epi, g, st);
 }

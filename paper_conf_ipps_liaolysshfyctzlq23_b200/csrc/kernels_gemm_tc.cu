@@ -18,6 +18,7 @@
 #include <cuda.h>
 
 #include <cstdio>
+#include <atomic>
 #include <mutex>
 #include <unordered_map>
 
@@ -380,6 +381,7 @@ MDEV void epi_frag32_in(const GemmArgs& g, int m_base, int n, float (&v)[32], in
 template <int BN, int EPI>
 __global__ void __launch_bounds__(TC_THREADS, 2)
     k_gemm_tc(const __grid_constant__ CUtensorMap tma_a, const __grid_constant__ CUtensorMap tma_b, const TcArgs args) {
+  pdl_enter();
   using Cf = TcCfg<BN>;
   extern __shared__ uint8_t smem_raw[];
   uint8_t* smem = (uint8_t*)(((uintptr_t)smem_raw + 1023) & ~(uintptr_t)1023);
@@ -512,11 +514,35 @@ struct TpCfg {
 struct TpArgs {
   TcArgs t;
   int m_blocks, n_blocks, n_tiles;
+  uint32_t* flags;     // fused split-K: [split-1][per_split][TP_EPI_WARPS] release flags
+  uint32_t epoch;      // this launch's flag value (never reused within a process)
 };
+
+// Split index of persistent unit `tile`.  Fused split-K orders the units
+// z = split-1 first and z = 0 last, so a split-0 unit (which waits for its
+// partials) is never scheduled in an earlier round than the units it waits on.
+MDEV int unit_z(const TcArgs& ta, int tile, int per_split) {
+  const int q = tile / per_split;
+  return ta.g.fused_split ? ta.g.split - 1 - q : q;
+}
+MDEV uint32_t ld_acquire_u32(const uint32_t* p) {
+  uint32_t v;
+  asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
+  return v;
+}
+MDEV void st_release_u32(uint32_t* p, uint32_t v) {
+  asm volatile("st.release.gpu.global.u32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
+}
+MDEV float4 ld_cg_f4(const float* p) {
+  float4 v;
+  asm volatile("ld.global.cg.v4.f32 {%0, %1, %2, %3}, [%4];" : "=f"(v.x), "=f"(v.y), "=f"(v.z), "=f"(v.w) : "l"(p));
+  return v;
+}
 
 template <int BN, int EPI>
 __global__ void __launch_bounds__(TP_THREADS, 1)
     k_gemm_tcp(const __grid_constant__ CUtensorMap tma_a, const __grid_constant__ CUtensorMap tma_b, const TpArgs args) {
+  pdl_trigger();
   using Cf = TpCfg<BN>;
   extern __shared__ uint8_t smem_raw[];
   uint8_t* smem = (uint8_t*)(((uintptr_t)smem_raw + 1023) & ~(uintptr_t)1023);
@@ -545,13 +571,14 @@ __global__ void __launch_bounds__(TP_THREADS, 1)
   __syncthreads();
   tc_fence_after();
   const uint32_t tmem = *tmem_slot;
+  pdl_wait();                                       // prologue above overlaps the previous kernel
   const int per_split = args.m_blocks * args.n_blocks;
 
   if (warp == 0) {
     if (lane == 0) {                                   // ---------------- TMA producer
       int it = 0;
       for (int tile = blockIdx.x; tile < args.n_tiles; tile += gridDim.x) {
-        const int z = tile / per_split, r = tile % per_split;
+        const int z = unit_z(ta, tile, per_split), r = tile % per_split;
         const int m0 = (r / args.n_blocks) * TBM, n0 = (r % args.n_blocks) * BN;
         const int kb0 = z * ta.kb_per_split, kb1 = min(ta.kb_total, kb0 + ta.kb_per_split);
         for (int kb = kb0; kb < kb1; ++kb, ++it) {
@@ -583,7 +610,7 @@ __global__ void __launch_bounds__(TP_THREADS, 1)
       const uint32_t idesc = idesc_bf16(TBM, BN, ta.a_mn, ta.b_mn);
       int it = 0, local = 0;
       for (int tile = blockIdx.x; tile < args.n_tiles; tile += gridDim.x, ++local) {
-        const int z = tile / per_split;
+        const int z = unit_z(ta, tile, per_split);
         const int kb0 = z * ta.kb_per_split, kb1 = min(ta.kb_total, kb0 + ta.kb_per_split);
         const int acc = local & 1;
         if (local >= 2) mbar_wait(&tempty[acc], ((local >> 1) - 1) & 1);
@@ -613,7 +640,7 @@ __global__ void __launch_bounds__(TP_THREADS, 1)
     const GemmArgs& g = ta.g;
     int local = 0;
     for (int tile = blockIdx.x; tile < args.n_tiles; tile += gridDim.x, ++local) {
-      const int z = tile / per_split, r = tile % per_split;
+      const int z = unit_z(ta, tile, per_split), r = tile % per_split;
       const int m0 = (r / args.n_blocks) * TBM, n0 = (r % args.n_blocks) * BN;
       const int kb0 = z * ta.kb_per_split, kb1 = min(ta.kb_total, kb0 + ta.kb_per_split);
       const int acc = local & 1;
@@ -632,6 +659,16 @@ __global__ void __launch_bounds__(TP_THREADS, 1)
           for (int o = 0; o < bytes; o += 128) asm volatile("prefetch.global.L2 [%0];" ::"l"(pa + o));
         }
       }
+      if constexpr (EPI == EPI_F32) {
+        if (g.fused_split && z == 0) {   // wait for this warp's partials of splits 1..split-1
+          if (lane == 0)
+            for (int zz = 1; zz < g.split; ++zz) {
+              const uint32_t* f = args.flags + ((size_t)(zz - 1) * per_split + r) * TP_EPI_WARPS + e;
+              while (ld_acquire_u32(f) != args.epoch) __nanosleep(64);
+            }
+          __syncwarp();
+        }
+      }
       mbar_wait(&tfull[acc], (local >> 1) & 1);
       __syncwarp();
       tc_fence_after();
@@ -648,12 +685,39 @@ __global__ void __launch_bounds__(TP_THREADS, 1)
 #pragma unroll
           for (int i = 0; i < 32; ++i) v[i] = 0.f;
         }
-        if (n + 32 <= g.N) {
+        if (EPI == EPI_F32 && g.fused_split && n + 32 <= g.N) {
+          const int mb = m0 + 32 * q;
+          if (mb < g.M) {
+            float* dst;
+            if (z > 0) {
+              dst = g.ws + (int64_t)(z - 1) * g.split_stride;
+            } else {
+              dst = (float*)g.C;
+              if (m < g.M)
+                for (int zz = 1; zz < g.split; ++zz) {
+                  const float* p = g.ws + (int64_t)(zz - 1) * g.split_stride + (int64_t)m * g.ldc + n;
+#pragma unroll
+                  for (int j = 0; j < 8; ++j) {
+                    const float4 w = ld_cg_f4(p + 4 * j);
+                    v[4 * j] += w.x; v[4 * j + 1] += w.y; v[4 * j + 2] += w.z; v[4 * j + 3] += w.w;
+                  }
+                }
+            }
+            stage_store_f32(stg_base + e * 4096, v, dst + (int64_t)mb * g.ldc + n, g.ldc, g.M - mb, lane);
+          }
+        } else if (n + 32 <= g.N) {
           if (m0 + 32 * q < g.M) epi_frag32_in<EPI>(g, m0 + 32 * q, n, v, z, stg_base + e * 4096, lane, cur);
         } else if (m < g.M) {
 #pragma unroll
           for (int i = 0; i < 32; ++i)
             if (n + i < g.N) epilogue<__nv_bfloat16, EPI>(g, m, n + i, v[i], z);
+        }
+      }
+      if constexpr (EPI == EPI_F32) {
+        if (g.fused_split && z > 0) {    // publish this warp's partial rows/columns
+          __threadfence();
+          __syncwarp();
+          if (lane == 0) st_release_u32(args.flags + ((size_t)(z - 1) * per_split + r) * TP_EPI_WARPS + e, args.epoch);
         }
       }
       tc_fence_before();
@@ -724,6 +788,7 @@ MDEV void mbar_arrive_rank(uint64_t* bar, uint32_t rank) {
 template <int BN, int EPI>
 __global__ void __launch_bounds__(TP_THREADS, 1)
     k_gemm_tc2(const __grid_constant__ CUtensorMap tma_a, const __grid_constant__ CUtensorMap tma_b, const TpArgs args) {
+  pdl_enter();
   using Cf = T2Cfg<BN>;
   extern __shared__ uint8_t smem_raw[];
   uint8_t* smem = (uint8_t*)(((uintptr_t)smem_raw + 1023) & ~(uintptr_t)1023);
@@ -946,7 +1011,7 @@ static void launch_tc(const CUtensorMap& ma, const CUtensorMap& mb, const TcArgs
     cudaFuncSetAttribute(k_gemm_tc<BN, EPI>, cudaFuncAttributeMaxDynamicSharedMemorySize, TcCfg<BN>::SMEM);
     attr = true;
   }
-  k_gemm_tc<BN, EPI><<<grid, TC_THREADS, TcCfg<BN>::SMEM, st>>>(ma, mb, a);
+  launch_k(k_gemm_tc<BN, EPI>, grid, TC_THREADS, TcCfg<BN>::SMEM, st, ma, mb, a);
 }
 
 template <int BN, int EPI>
@@ -962,7 +1027,7 @@ static void launch_tcp(const CUtensorMap& ma, const CUtensorMap& mb, const TpArg
     cudaGetDevice(&dev);
     cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, dev);
   }
-  k_gemm_tcp<BN, EPI><<<std::min(nsm, a.n_tiles), TP_THREADS, TpCfg<BN>::SMEM, st>>>(ma, mb, a);
+  launch_k(k_gemm_tcp<BN, EPI>, std::min(nsm, a.n_tiles), TP_THREADS, TpCfg<BN>::SMEM, st, ma, mb, a);
 }
 
 template <int BN>
@@ -1029,6 +1094,33 @@ static void dispatch_tc2(Epi epi, const CUtensorMap& ma, const CUtensorMap& mb, 
   }
 }
 
+// Release flags of the fused split-K GEMMs: one zero-initialised buffer per
+// device (outside the arena, like NCCL's buffers: 256 KB), and a process-wide
+// launch epoch, so flags never need resetting.  Fused split-K GEMMs of one
+// device are issued on one stream (the compute stream), never concurrently.
+constexpr size_t kFlagWords = 1 << 16;
+static uint32_t* splitk_flags() {
+  static std::mutex mu;
+  static std::unordered_map<int, uint32_t*> bufs;
+  int dev = 0;
+  cudaGetDevice(&dev);
+  std::lock_guard<std::mutex> lk(mu);
+  auto it = bufs.find(dev);
+  if (it != bufs.end()) return it->second;
+  uint32_t* p = nullptr;
+  if (cudaMalloc(&p, kFlagWords * 4) != cudaSuccess) return nullptr;
+  if (cudaMemset(p, 0, kFlagWords * 4) != cudaSuccess) return nullptr;
+  cudaDeviceSynchronize();
+  bufs[dev] = p;
+  return p;
+}
+static uint32_t next_epoch() {
+  static std::atomic<uint32_t> e{0};
+  uint32_t v = ++e;
+  if (v == 0) v = ++e;
+  return v;
+}
+
 static int g_gemm_mode = 1;   // 0: one tile per CTA (k_gemm_tc); 1: persistent (k_gemm_tcp)
 void set_gemm_mode(int m) { g_gemm_mode = m; }
 
@@ -1076,6 +1168,8 @@ bool gemm_tc(Epi epi, const GemmArgs& g, cudaStream_t st) {
   // BN = 64 loses on every step shape -- the per-tile fixed cost dominates).
   auto tiles = [&](int bn) { return m_blocks * ((g.N + bn - 1) / bn) * g.split; };
   int BN = (g.N % 256 == 0 && tiles(256) >= 100) ? 256 : 128;
+  if (g.bn == 256 && g.N % 256 == 0) BN = 256;
+  if (g.bn == 128) BN = 128;
   if (g_gemm_mode == 11) BN = 128;
   if (g_gemm_mode == 12 && g.N % 256 == 0) BN = 256;
   if (g_gemm_mode == 13) BN = 64;
@@ -1084,6 +1178,7 @@ bool gemm_tc(Epi epi, const GemmArgs& g, cudaStream_t st) {
   const bool persistent = g_gemm_mode == 1 || g_gemm_mode == 11 || g_gemm_mode == 12 || g_gemm_mode == 13 ||
                           g_gemm_mode == 2 || g_gemm_mode == 21 || g_gemm_mode == 22;
   if (!persistent) BN = 128;
+  if (g.fused_split && (!persistent || epi != EPI_F32 || BN == 64)) return false;
   CUtensorMap ma, mb;
   bool ok;
   if (a.a_mn) ok = make_map(&ma, g.A, g.M, g.K, g.a_sk, 64, 64);
@@ -1098,6 +1193,14 @@ bool gemm_tc(Epi epi, const GemmArgs& g, cudaStream_t st) {
     p.m_blocks = m_blocks;
     p.n_blocks = (g.N + BN - 1) / BN;
     p.n_tiles = p.m_blocks * p.n_blocks * g.split;
+    p.flags = nullptr;
+    p.epoch = 0;
+    if (g.fused_split) {
+      if ((size_t)(g.split - 1) * p.m_blocks * p.n_blocks * TP_EPI_WARPS > kFlagWords) return false;
+      p.flags = splitk_flags();
+      if (!p.flags) return false;
+      p.epoch = next_epoch();
+    }
     if (BN == 256) dispatch_tcp<256>(epi, ma, mb, p, st);
     else if (BN == 128) dispatch_tcp<128>(epi, ma, mb, p, st);
     else dispatch_tcp<64>(epi, ma, mb, p, st);

@@ -76,3 +76,23 @@ def test_gemm_split_k(split, gemm_mode):
     ref = A.float() @ B.float().t()
     err = (C.sum(0) - ref).abs().max().item() / ref.abs().max().item()
     assert err < 1e-5, err
+
+
+@pytest.mark.parametrize("shape,split", [((768, 3072, 5120), 2), ((3072, 768, 4096), 2), ((2304, 768, 2048), 3),
+                                         ((768, 768, 5120), 5), ((1024, 1024, 1536), 4), ((640, 512, 777), 2)])
+def test_gemm_fused_splitk(shape, split):
+    """wgrad-shaped TN GEMM with the in-kernel fused split-K: matches the fp32
+    reference, and two launches are bitwise identical (fixed reduction order)."""
+    M, N, K = shape
+    A, B, As, Bs, a_sm, a_sk, b_sn, b_sk = operands(M, N, K, 1, 1, seed=3)
+    ws = torch.full(((split - 1) * M * N,), float("nan"), device="cuda")
+    outs = []
+    for _ in range(2):
+        C = torch.full((M, N), float("nan"), device="cuda")
+        mb().debug_gemm_ex(6, M, N, K, As, a_sm, a_sk, Bs, b_sn, b_sk, C, N, C2=ws, split=-split)
+        torch.cuda.synchronize()
+        outs.append(C)
+    ref = A.float() @ B.float().t()
+    err = (outs[0] - ref).abs().max().item() / ref.abs().max().item()
+    assert err < 1e-5, err
+    assert torch.equal(outs[0], outs[1])
