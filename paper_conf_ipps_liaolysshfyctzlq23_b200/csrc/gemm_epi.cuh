@@ -100,6 +100,45 @@ MDEV float2 gelu_grad_x2(float2 u) {
   return ffma2(fmul2(u, f2s(0.39894228040143268f)), e, ffma2(f2s(0.5f), erf_s2_x2(u, e), f2s(0.5f)));
 }
 
+// Fast erf-GELU for the bf16 tcgen05 epilogues: the tanh form
+// 0.5 u (1 + tanh(sqrt(2/pi) (u + 0.044715 u^3))) with one MUFU.TANH.  Its
+// distance to the exact erf-GELU is <= 4.8e-4 (at u = 2.7, where a bf16 ulp is
+// 1.6e-2) and that of its derivative to the exact GELU' <= 8.7e-4 (bf16 ulp
+// 7.8e-3), so the stored bf16 values are within a small fraction of an ulp of
+// the exact ones (reading R-G).  The fp32 (SIMT) path keeps the exact
+// erf forms above.  Backward uses this function's own derivative.
+MDEV float tanh_apx(float x) {
+  float y;
+  asm("tanh.approx.f32 %0, %1;" : "=f"(y) : "f"(x));
+  return y;
+}
+MDEV float gelu_fast(float u) {
+  const float z = u * fmaf(0.035677408136300125f, u * u, 0.7978845608028654f);
+  const float h = 0.5f * u;
+  return fmaf(h, tanh_apx(z), h);
+}
+MDEV float gelu_grad_fast(float u) {
+  const float u2 = u * u;
+  const float t = tanh_apx(u * fmaf(0.035677408136300125f, u2, 0.7978845608028654f));
+  const float dz = fmaf(0.10703222440890037f, u2, 0.7978845608028654f);
+  return fmaf(0.5f * u * fmaf(-t, t, 1.0f), dz, fmaf(0.5f, t, 0.5f));
+}
+MDEV float2 gelu_fast_x2(float2 u) {
+  const float2 u2 = fmul2(u, u);
+  const float2 z = fmul2(u, ffma2(f2s(0.035677408136300125f), u2, f2s(0.7978845608028654f)));
+  const float2 t = make_float2(tanh_apx(z.x), tanh_apx(z.y));
+  const float2 h = fmul2(f2s(0.5f), u);
+  return ffma2(h, t, h);
+}
+MDEV float2 gelu_grad_fast_x2(float2 u) {
+  const float2 u2 = fmul2(u, u);
+  const float2 z = fmul2(u, ffma2(f2s(0.035677408136300125f), u2, f2s(0.7978845608028654f)));
+  const float2 t = make_float2(tanh_apx(z.x), tanh_apx(z.y));
+  const float2 dz = ffma2(f2s(0.10703222440890037f), u2, f2s(0.7978845608028654f));
+  const float2 omt = ffma2(make_float2(-t.x, -t.y), t, f2s(1.0f));
+  return ffma2(fmul2(fmul2(f2s(0.5f), u), omt), dz, ffma2(f2s(0.5f), t, f2s(0.5f)));
+}
+
 // GPT-2 "gelu_new": 0.5 u (1 + tanh(k0 (u + 0.044715 u^3))), tanh via one exp:
 // tanh z = 1 - 2 / (2^(2 log2(e) z) + 1) (inf -> 1, 0 -> -1 at the extremes).
 MDEV float tanh_fast(float z) { return fmaf(-2.0f, rcp_ftz(ex2_ftz(2.8853900817779268f * z) + 1.0f), 1.0f); }

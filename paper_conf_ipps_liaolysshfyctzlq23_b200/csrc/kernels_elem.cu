@@ -107,48 +107,61 @@ void ln_fwd(DType dt, const float* z, const void* g, const void* b, void* y, flo
   });
 }
 
-// NPART CTAs x 8 warps; warp w of CTA p owns rows r = p*8 + w + k*NPART*8 (fixed).
+// NPART CTAs x 4 warps; warp w of CTA p owns rows r = p*4 + w + k*NPART*4 (fixed).
 // Per-lane register partials of dgamma, dbeta, dbias over the warp's rows, then a
-// fixed-order reduction over the 8 warps through shared memory.
-template <typename E>
-__global__ void __launch_bounds__(256) k_ln_bwd(const float* dy, Drop premask, const float* __restrict__ z,
-                                                const float2* __restrict__ st, const E* __restrict__ g,
-                                                float* dz, E* __restrict__ dtout, Drop mask,
-                                                float* __restrict__ pg, float* __restrict__ pb,
-                                                float* __restrict__ pbias, int T, int H, const float* res) {
+// fixed-order reduction over the 4 warps through shared memory.  KCH = 8-column
+// chunks per lane (ceil(H / 256)); gamma is read from shared memory.  ~140
+// registers x 128 threads: 3 CTAs / SM, so all NPART CTAs are resident at once.
+constexpr int LNB_WARPS = 4;
+template <typename E, int KCH>
+__global__ void __launch_bounds__(32 * LNB_WARPS, 3) k_ln_bwd(const float* dy, Drop premask,
+                                                              const float* __restrict__ z,
+                                                              const float2* __restrict__ st, const E* __restrict__ g,
+                                                              float* dz, E* __restrict__ dtout, Drop mask,
+                                                              float* __restrict__ pg, float* __restrict__ pb,
+                                                              float* __restrict__ pbias, int T, int H,
+                                                              const float* res) {
   pdl_enter();
-  extern __shared__ float sm[];
+  extern __shared__ float sm[];            // [LNB_WARPS][3][H] partials, then gamma [H]
+  float* sgam = sm + (size_t)LNB_WARPS * 3 * H;
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const int nch = H >> 3;
   const float invH = 1.0f / (float)H;
-  float ag[4][8], ab[4][8], at[4][8], gv[4][8];
+  for (int c = threadIdx.x; c < H; c += blockDim.x) sgam[c] = ldf(g + c);
+  __syncthreads();
+  float ag[KCH][8], ab[KCH][8], at[KCH][8];
 #pragma unroll
-  for (int k = 0; k < 4; ++k) {
-    const int j = lane + 32 * k;
+  for (int k = 0; k < KCH; ++k)
 #pragma unroll
-    for (int i = 0; i < 8; ++i) { ag[k][i] = 0.f; ab[k][i] = 0.f; at[k][i] = 0.f; gv[k][i] = 0.f; }
-    if (j < nch) ld8(g + 8 * j, gv[k]);
-  }
-  for (int row = blockIdx.x * 8 + warp; row < T; row += NPART * 8) {
+    for (int i = 0; i < 8; ++i) { ag[k][i] = 0.f; ab[k][i] = 0.f; at[k][i] = 0.f; }
+  for (int row = blockIdx.x * LNB_WARPS + warp; row < T; row += NPART * LNB_WARPS) {
     const float2 ms = st[row];
-    float dyv[4][8], xh[4][8];
+    float dyv[KCH][8], xh[KCH][8];
     float s1 = 0.f, s2 = 0.f;
 #pragma unroll
-    for (int k = 0; k < 4; ++k) {
+    for (int k = 0; k < KCH; ++k) {
       const int j = lane + 32 * k;
       if (j < nch) {
         ld8(dy + (int64_t)row * H + 8 * j, dyv[k]);
         ld8(z + (int64_t)row * H + 8 * j, xh[k]);
+      }
+    }
+#pragma unroll
+    for (int k = 0; k < KCH; ++k) {
+      const int j = lane + 32 * k;
+      if (j < nch) {
         if (premask.enabled) {
           float f[8];
           drop8(premask, (uint64_t)row * H + 8 * j, f);
 #pragma unroll
           for (int i = 0; i < 8; ++i) dyv[k][i] *= f[i];
         }
+        float gv[8];
+        ld8(sgam + 8 * j, gv);
 #pragma unroll
         for (int i = 0; i < 8; ++i) {
           xh[k][i] = (xh[k][i] - ms.x) * ms.y;
-          const float dxh = dyv[k][i] * gv[k][i];
+          const float dxh = dyv[k][i] * gv[i];
           s1 += dxh;
           s2 += dxh * xh[k][i];
         }
@@ -157,13 +170,14 @@ __global__ void __launch_bounds__(256) k_ln_bwd(const float* dy, Drop premask, c
     s1 = warp_sum(s1) * invH;
     s2 = warp_sum(s2) * invH;
 #pragma unroll
-    for (int k = 0; k < 4; ++k) {
+    for (int k = 0; k < KCH; ++k) {
       const int j = lane + 32 * k;
       if (j < nch) {
-        float o[8];
+        float o[8], gv[8];
+        ld8(sgam + 8 * j, gv);
 #pragma unroll
         for (int i = 0; i < 8; ++i) {
-          o[i] = ms.y * (dyv[k][i] * gv[k][i] - s1 - xh[k][i] * s2);
+          o[i] = ms.y * (dyv[k][i] * gv[i] - s1 - xh[k][i] * s2);
           ag[k][i] += dyv[k][i] * xh[k][i];
           ab[k][i] += dyv[k][i];
         }
@@ -186,9 +200,9 @@ __global__ void __launch_bounds__(256) k_ln_bwd(const float* dy, Drop premask, c
       }
     }
   }
-  // fixed-order cross-warp reduction: smem [8 warps][3][H]
+  // fixed-order cross-warp reduction: smem [LNB_WARPS][3][H]
 #pragma unroll
-  for (int k = 0; k < 4; ++k) {
+  for (int k = 0; k < KCH; ++k) {
     const int j = lane + 32 * k;
     if (j < nch) {
       float* base = sm + (size_t)warp * 3 * H + 8 * j;
@@ -200,7 +214,7 @@ __global__ void __launch_bounds__(256) k_ln_bwd(const float* dy, Drop premask, c
   __syncthreads();
   for (int c = threadIdx.x; c < H; c += blockDim.x) {
     float sg = 0.f, sb = 0.f, sbias = 0.f;
-    for (int w = 0; w < 8; ++w) {
+    for (int w = 0; w < LNB_WARPS; ++w) {
       const float* base = sm + (size_t)w * 3 * H;
       sg += base[c]; sb += base[H + c]; sbias += base[2 * H + c];
     }
@@ -210,20 +224,32 @@ __global__ void __launch_bounds__(256) k_ln_bwd(const float* dy, Drop premask, c
   }
 }
 
+template <typename E, int KCH>
+static void launch_ln_bwd(const float* dy, Drop premask, const float* z, const float2* st, const void* g, float* dz,
+                          void* dtout, Drop mask, float* pg, float* pb, float* pbias, int T, int H, cudaStream_t s,
+                          const float* res) {
+  const size_t smem = (size_t)(LNB_WARPS * 3 + 1) * H * sizeof(float);
+  static bool attr = false;
+  if (!attr) {
+    cudaFuncSetAttribute(k_ln_bwd<E, KCH>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                         (LNB_WARPS * 3 + 1) * 1024 * 4);
+    attr = true;
+  }
+  launch_k(k_ln_bwd<E, KCH>, NPART, 32 * LNB_WARPS, smem, s, dy, premask, z, st, (const E*)g, dz, (E*)dtout, mask,
+           pg, pb, pbias, T, H, res);
+}
+
 void ln_bwd(DType dt, const float* dy, Drop premask, const float* z, const float2* st, const void* g,
             float* dz, void* dtout, Drop mask, float* pg, float* pb, float* pbias, int T, int H,
             cudaStream_t s, const float* res) {
-  const size_t smem = (size_t)8 * 3 * H * sizeof(float);
   note_launch(1);
+  const int kch = (H / 8 + 31) / 32;
   dispatch(dt, [&](auto* tag) {
     using E = std::remove_pointer_t<decltype(tag)>;
-    static bool attr = false;
-    if (!attr) {
-      cudaFuncSetAttribute(k_ln_bwd<E>, cudaFuncAttributeMaxDynamicSharedMemorySize, 8 * 3 * 1024 * 4);
-      attr = true;
-    }
-    launch_k(k_ln_bwd<E>, NPART, 256, smem, s, dy, premask, z, st, (const E*)g, dz, (E*)dtout,
-                                         mask, pg, pb, pbias, T, H, res);
+    if (kch <= 1) launch_ln_bwd<E, 1>(dy, premask, z, st, g, dz, dtout, mask, pg, pb, pbias, T, H, s, res);
+    else if (kch == 2) launch_ln_bwd<E, 2>(dy, premask, z, st, g, dz, dtout, mask, pg, pb, pbias, T, H, s, res);
+    else if (kch == 3) launch_ln_bwd<E, 3>(dy, premask, z, st, g, dz, dtout, mask, pg, pb, pbias, T, H, s, res);
+    else launch_ln_bwd<E, 4>(dy, premask, z, st, g, dz, dtout, mask, pg, pb, pbias, T, H, s, res);
   });
 }
 

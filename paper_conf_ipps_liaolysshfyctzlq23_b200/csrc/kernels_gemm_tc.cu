@@ -67,7 +67,7 @@ MDEV void epi_row32(const GemmArgs& g, int m, int n, float (&v)[32], int z = -1)
     } else if constexpr (EPI == EPI_BIAS_GELU) {
       st_bf16x32((E*)g.C + o, v);
 #pragma unroll
-      for (int i = 0; i < 32; ++i) v[i] = gelu_f(__bfloat162float(__float2bfloat16_rn(v[i])));
+      for (int i = 0; i < 32; ++i) v[i] = gelu_fast(__bfloat162float(__float2bfloat16_rn(v[i])));
       st_bf16x32((E*)g.C2 + o, v);
     } else {
       float r[32];
@@ -88,7 +88,7 @@ MDEV void epi_row32(const GemmArgs& g, int m, int n, float (&v)[32], int z = -1)
     float u[32];
     ld_bf16x32((const E*)g.aux + (int64_t)m * g.ldx + n, u);
 #pragma unroll
-    for (int i = 0; i < 32; ++i) v[i] *= gelu_grad_f(u[i]);
+    for (int i = 0; i < 32; ++i) v[i] *= gelu_grad_fast(u[i]);
     st_bf16x32((E*)g.C + o, v);
   } else if constexpr (EPI == EPI_ACC_RES_F32) {
     const float4* r = (const float4*)((const float*)g.res + (int64_t)m * g.ldr + n);
@@ -178,7 +178,7 @@ MDEV void epi_frag32(const GemmArgs& g, int m_base, int n, float (&v)[32], int z
     } else if constexpr (EPI == EPI_BIAS_GELU) {
       stage_store_bf16(stg, v, (E*)g.C + (int64_t)m_base * g.ldc + n, g.ldc, rows_valid, lane);
 #pragma unroll
-      for (int i = 0; i < 32; ++i) v[i] = gelu_f(__bfloat162float(__float2bfloat16_rn(v[i])));
+      for (int i = 0; i < 32; ++i) v[i] = gelu_fast(__bfloat162float(__float2bfloat16_rn(v[i])));
       stage_store_bf16(stg, v, (E*)g.C2 + (int64_t)m_base * g.ldc + n, g.ldc, rows_valid, lane);
     } else {
       float r[32];
@@ -199,7 +199,7 @@ MDEV void epi_frag32(const GemmArgs& g, int m_base, int n, float (&v)[32], int z
     if (live) {
       ld_bf16x32((const E*)g.aux + (int64_t)m * g.ldx + n, u);
 #pragma unroll
-      for (int i = 0; i < 32; ++i) v[i] *= gelu_grad_f(u[i]);
+      for (int i = 0; i < 32; ++i) v[i] *= gelu_grad_fast(u[i]);
     }
     stage_store_bf16(stg, v, (E*)g.C + (int64_t)m_base * g.ldc + n, g.ldc, rows_valid, lane);
   } else if constexpr (EPI == EPI_ACC_RES_F32) {
@@ -284,7 +284,7 @@ MDEV void epi_frag32_in(const GemmArgs& g, int m_base, int n, float (&v)[32], in
       stage_store_bf16(stg, v, (E*)g.C + (int64_t)m_base * g.ldc + n, g.ldc, rows_valid, lane);
 #pragma unroll
       for (int i = 0; i < 32; i += 2) {
-        const float2 r = gelu_x2(make_float2(__bfloat162float(__float2bfloat16_rn(v[i])),
+        const float2 r = gelu_fast_x2(make_float2(__bfloat162float(__float2bfloat16_rn(v[i])),
                                              __bfloat162float(__float2bfloat16_rn(v[i + 1]))));
         v[i] = r.x;
         v[i + 1] = r.y;
@@ -311,7 +311,7 @@ MDEV void epi_frag32_in(const GemmArgs& g, int m_base, int n, float (&v)[32], in
     for (int i = 0; i < 4; ++i) unpack8(in.x[i], u + 8 * i);
 #pragma unroll
     for (int i = 0; i < 32; i += 2) {   // rows >= M are never stored
-      const float2 r = fmul2(make_float2(v[i], v[i + 1]), gelu_grad_x2(make_float2(u[i], u[i + 1])));
+      const float2 r = fmul2(make_float2(v[i], v[i + 1]), gelu_grad_fast_x2(make_float2(u[i], u[i + 1])));
       v[i] = r.x;
       v[i + 1] = r.y;
     }
@@ -335,7 +335,7 @@ MDEV void epi_frag32_in(const GemmArgs& g, int m_base, int n, float (&v)[32], in
     if constexpr (EPI == EPI_BIAS_GELUT) {
       stage_store_bf16(stg, v, (E*)g.C + (int64_t)m_base * g.ldc + n, g.ldc, rows_valid, lane);
 #pragma unroll
-      for (int i = 0; i < 32; ++i) v[i] = gelu_tanh_f(__bfloat162float(__float2bfloat16_rn(v[i])));
+      for (int i = 0; i < 32; ++i) v[i] = gelu_fast(__bfloat162float(__float2bfloat16_rn(v[i])));   // gelu_new == the tanh form
       stage_store_bf16(stg, v, (E*)g.C2 + (int64_t)m_base * g.ldc + n, g.ldc, rows_valid, lane);
     } else {
       const float* r = (const float*)in.x;
@@ -355,7 +355,7 @@ MDEV void epi_frag32_in(const GemmArgs& g, int m_base, int n, float (&v)[32], in
 #pragma unroll
     for (int i = 0; i < 4; ++i) unpack8(in.x[i], u + 8 * i);
 #pragma unroll
-    for (int i = 0; i < 32; ++i) v[i] *= gelu_tanh_grad_f(u[i]);
+    for (int i = 0; i < 32; ++i) v[i] *= gelu_grad_fast(u[i]);
     stage_store_bf16(stg, v, (E*)g.C + (int64_t)m_base * g.ldc + n, g.ldc, rows_valid, lane);
   } else if constexpr (EPI == EPI_ACC_F32) {
     if (live) {

@@ -96,3 +96,33 @@ def test_gemm_fused_splitk(shape, split):
     err = (outs[0] - ref).abs().max().item() / ref.abs().max().item()
     assert err < 1e-5, err
     assert torch.equal(outs[0], outs[1])
+
+
+@pytest.mark.parametrize("shape", [(640, 3072, 768), (2048, 3072, 768)])
+def test_gemm_gelu_epilogues(shape, gemm_mode):
+    """EPI_BIAS_GELU (u = acc + b, g = gelu(u)) and EPI_GELU_BWD (acc * gelu'(u))
+    against the exact erf-GELU in fp32 (torch): u to bf16 rounding, g and the
+    gradient within one bf16 ulp of the exact value (the tcgen05 epilogue uses
+    the single-MUFU tanh form, |error| < 1e-3, DESIGN reading R-G)."""
+    M, N, K = shape
+    A, B, As, Bs, a_sm, a_sk, b_sn, b_sk = operands(M, N, K, 0, 0, seed=4)
+    bias = torch.randn(N, device="cuda").bfloat16()
+    U = torch.zeros(M, N, device="cuda", dtype=torch.bfloat16)
+    Gk = torch.zeros(M, N, device="cuda", dtype=torch.bfloat16)
+    A = A / 8
+    As = As / 8
+    mb().debug_gemm_ex(2, M, N, K, As, a_sm, a_sk, Bs, b_sn, b_sk, U, N, C2=Gk, bias=bias)
+    torch.cuda.synchronize()
+    ref_u = A.float() @ B.float().t() + bias.float()
+    assert ((U.float() - ref_u).abs().max() / ref_u.abs().max()).item() < 1e-2
+    g_exact = torch.nn.functional.gelu(U.float())
+    assert ((Gk.float() - g_exact).abs() <= 2.0 ** -7 * g_exact.abs().clamp_min(1.0)).all()
+    # backward epilogue: D = acc * gelu'(aux), aux = U
+    D = torch.zeros(M, N, device="cuda", dtype=torch.bfloat16)
+    mb().debug_gemm_ex(4, M, N, K, As, a_sm, a_sk, Bs, b_sn, b_sk, D, N, aux=U, ldx=N)
+    torch.cuda.synchronize()
+    u = U.float().requires_grad_(True)
+    torch.nn.functional.gelu(u).backward(torch.ones_like(u))
+    ref_d = (A.float() @ B.float().t()) * u.grad
+    err = ((D.float() - ref_d).abs().max() / ref_d.abs().max()).item()
+    assert err < 1e-2, err
