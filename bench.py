@@ -44,6 +44,8 @@ def parse():
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--simt", action="store_true", help="SIMT GEMMs instead of tcgen05")
     ap.add_argument("--gemm-mode", type=int, default=-1, help="tcgen05 GEMM variant (debug_options)")
+    ap.add_argument("--planner", default="greedy", choices=["greedy", "exact"],
+                    help="Algorithm 1 (default) or the exact fewest-recompute planner (reading A29)")
     return ap.parse_args()
 
 
@@ -254,6 +256,8 @@ def main():
         ctx.set_params(wl.pack_params(cfg, wl.init_params(cfg)))
         # AdamW per gradient bucket on a side stream, overlapping the backward
         ctx.set_optimizer(1e-5, fused=True)
+        if args.planner == "exact":
+            ctx.set_planner(mb.PLANNER_EXACT)
         return ctx
 
     n_total = args.warmup + args.steps
@@ -401,7 +405,7 @@ def main():
         "e2e": {"value": e2e, "unit": "samples/s", "h2d_bytes_per_step": per_step_h2d, "d2h_bytes_per_step": 4},
         "gpu_launches": launches,
         "clocks": clocks.summary(),
-        "mimose": {"violations": st2["violations"], "peak_bytes_max": st2["max_peak_bytes"],
+        "mimose": {"planner": args.planner, "violations": st2["violations"], "peak_bytes_max": st2["max_peak_bytes"],
                    "budget_bytes": M, "mean_layers_dropped": float(np.mean(dropped)),
                    "plan_cache_hits": st2["plan_cache_hits"], "plan_cache_misses": st2["plan_cache_misses"],
                    "planner_us_total": st2["planner_us_total"], "sheltered_iters": st2["collect_steps"],

@@ -17,6 +17,11 @@ Readings (DESIGN.md register, numbered as SURVEY §8(c)-R):
          last resort before INFEASIBLE
   A13    when the linear accounting says excess <= 0, re-check with the
          position-aware predicted peak P(L',x) and continue if still over
+  A29    the exact alternative planner ("a flexible interface for ...
+         other scheduling algorithms, such as the Knapsack optimization"):
+         fewest recomputed layers (unit cost: homogeneous encoder layers)
+         with predicted_peak <= M - reserve, then the lowest peak, then the
+         lexicographically smallest sorted layer list = brute_force(cost=1)
 All byte arithmetic is in Python integers.
 
 Pinned by: hand traces (tests/golden/alg1_traces.txt), brute force over all
@@ -156,3 +161,14 @@ def brute_force(p: Dict, budget: int, cost: Sequence[float], reserve: int = 0):
     if best is None:
         return INFEASIBLE, None, None
     return OK, list(best[2]), best[1]
+
+
+def plan_exact(p: Dict, budget: int, reserve: int = 0):
+    """Reading A29: the exact planner is, by definition, the brute-force
+    minimum over all 2^L drop sets with unit recompute cost (small L only).
+    An infeasible budget returns (INFEASIBLE, all layers, their peak)."""
+    L = len(p["a"])
+    st, dropped, pk = brute_force(p, budget, [1] * L, reserve)
+    if st != OK:
+        return INFEASIBLE, list(range(L)), predicted_peak(p, range(L))
+    return OK, dropped, pk

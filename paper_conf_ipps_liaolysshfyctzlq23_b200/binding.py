@@ -119,13 +119,15 @@ _lib.mimose_nccl_unique_id.argtypes = [_P]
 _lib.mimose_set_optimizer.argtypes = [_P, C.c_float, C.c_float, C.c_float, C.c_float, C.c_float, C.c_int32]
 _lib.mimose_probe.argtypes = [_P, C.c_int32]
 _lib.mimose_probe_read.argtypes = [_P, C.POINTER(C.c_double), C.POINTER(C.c_double), C.POINTER(C.c_int64)]
+_lib.mimose_set_planner.argtypes = [_P, C.c_int32]
 
 EXPORTED = ["mimose_default_config", "mimose_init", "mimose_destroy", "mimose_last_error",
             "mimose_status_str", "mimose_num_params", "mimose_set_params", "mimose_get_params",
             "mimose_get_grads", "mimose_collect", "mimose_plan", "mimose_forward", "mimose_backward",
             "mimose_step", "mimose_get_stats", "mimose_phase", "mimose_get_sample", "mimose_dry_run",
             "mimose_dry_collect", "mimose_predicted_peak", "mimose_plan_series", "mimose_fit_predict",
-            "mimose_nccl_unique_id", "mimose_probe", "mimose_probe_read", "mimose_set_optimizer"]
+            "mimose_nccl_unique_id", "mimose_probe", "mimose_probe_read", "mimose_set_optimizer",
+            "mimose_set_planner"]
 
 
 _lib.mimose_tc_available.restype = C.c_int32
@@ -288,6 +290,10 @@ class Mimose:
         self._chk(_lib.mimose_plan(self.h, int(x), C.byref(p)), allow=(E_INFEASIBLE,))
         return p
 
+    def set_planner(self, kind: int):
+        """0 = Algorithm 1 greedy (default), 1 = exact fewest-recompute planner."""
+        self._chk(_lib.mimose_set_planner(self.h, int(kind)))
+
     def forward(self, batch: BatchS, plan: Optional[Plan] = None, want_loss: bool = True) -> Optional[float]:
         loss = C.c_float()
         self._chk(_lib.mimose_forward(self.h, C.byref(batch), C.byref(plan) if plan is not None else None,
@@ -360,7 +366,13 @@ def predicted_peak(p: Dict, dropped=()) -> int:
     return _lib.mimose_predicted_peak(C.byref(s), C.c_uint64(mask))
 
 
-def plan_series(p: Dict, budget: int, reserve: int = 0, num: int = 9, den: int = 10):
+PLANNER_GREEDY, PLANNER_EXACT = 0, 1
+
+
+def plan_series(p: Dict, budget: int, reserve: int = 0, num: int = 9, den: int = 10, planner: int = PLANNER_GREEDY):
+    """The library's planner on explicit per-series sizes (test hook)."""
+    if planner == PLANNER_EXACT:
+        num = 0
     s, keep = _series(p)
     mask = C.c_uint64()
     pk = C.c_int64()

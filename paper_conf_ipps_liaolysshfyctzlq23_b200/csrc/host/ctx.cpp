@@ -182,6 +182,7 @@ struct mimose_ctx {
   float* ws = nullptr;        // split-K workspace (4 H H fp32)
   float* part = nullptr;      // NPART * 2 * max(3H, F) fp32
   int64_t ws_elems = 0;
+  int planner = PLANNER_GREEDY;   // mimose_set_planner
 
   // step state
   int B = 0, S = 0, T = 0;
@@ -1323,6 +1324,14 @@ mimose_status mimose_set_optimizer(mimose_ctx* c, float lr, float b1, float b2, 
   return MIMOSE_OK;
 }
 
+mimose_status mimose_set_planner(mimose_ctx* c, int32_t kind) {
+  if (mimose_status s = check_ready(c)) return s;
+  if (kind != PLANNER_GREEDY && kind != PLANNER_EXACT) return fail(c, MIMOSE_E_INVALID, "unknown planner");
+  if (kind != c->planner) c->cache.clear();      // cached plans belong to the previous planner
+  c->planner = kind;
+  return MIMOSE_OK;
+}
+
 mimose_status mimose_plan(mimose_ctx* c, int64_t x, mimose_plan_t* out) {
   if (mimose_status s = check_ready(c)) return s;
   if (!out || x <= 0) return fail(c, MIMOSE_E_INVALID, "bad plan arguments");
@@ -1337,7 +1346,9 @@ mimose_status mimose_plan(mimose_ctx* c, int64_t x, mimose_plan_t* out) {
     c->stats.plan_cache_misses++;
     auto t0 = std::chrono::steady_clock::now();
     const Series s = c->est.predict(x);
-    const PlanResult pr = plan_greedy(s, c->ar.budget, c->cfg.reserve_bytes, c->cfg.bucket_num, c->cfg.bucket_den);
+    const PlanResult pr = c->planner == PLANNER_EXACT
+                              ? plan_exact(s, c->ar.budget, c->cfg.reserve_bytes)
+                              : plan_greedy(s, c->ar.budget, c->cfg.reserve_bytes, c->cfg.bucket_num, c->cfg.bucket_den);
     c->stats.planner_us_total +=
         std::chrono::duration<double, std::micro>(std::chrono::steady_clock::now() - t0).count();
     mimose_plan_t p{};
@@ -1510,7 +1521,7 @@ int64_t mimose_predicted_peak(const mimose_series* s, uint64_t mask) { return pr
 mimose_status mimose_plan_series(const mimose_series* s, int64_t budget, int64_t reserve, int32_t bn, int32_t bd,
                                  uint64_t* mask, int64_t* peak) {
   if (!s || !mask || !peak || s->n_layers < 1 || s->n_layers > 64 || bd <= 0) return MIMOSE_E_INVALID;
-  const PlanResult r = plan_greedy(to_series(s), budget, reserve, bn, bd);
+  const PlanResult r = bn == 0 ? plan_exact(to_series(s), budget, reserve) : plan_greedy(to_series(s), budget, reserve, bn, bd);
   *mask = r.drop_mask;
   *peak = r.peak;
   return r.feasible ? MIMOSE_OK : MIMOSE_E_INFEASIBLE;

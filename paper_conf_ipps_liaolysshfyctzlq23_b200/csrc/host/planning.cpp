@@ -129,6 +129,65 @@ PlanResult plan_greedy(const Series& s, int64_t budget, int64_t reserve, int bnu
   return {false, mask, predicted_peak(s, mask)};
 }
 
+namespace {
+struct ExactSearch {
+  const Series& s;
+  int L;
+  int64_t R;           // limit - (C + E): room for stack + transients
+  int k;               // drops to place
+  std::vector<int64_t> need;   // per-layer transient on top of its prefix
+  std::vector<int64_t> suf_a, suf_dmax;   // sum a_j and max (a_j - y_j) over j >= l
+  bool found = false;
+  int64_t best_pk = 0;
+  uint64_t best_mask = 0;
+  // Layers [l, L) remain; `left` drops still to place; prefix = stack bytes
+  // below layer l; runmax = max over the constraints of layers < l.
+  void dfs(int l, int left, int64_t prefix, int64_t runmax, uint64_t mask) {
+    if (found && runmax >= best_pk) return;             // cannot beat the best peak
+    if (l == L) {
+      if (left) return;
+      const int64_t pk = std::max(runmax, prefix + s.Hd + s.Th);
+      if (pk > R) return;
+      if (!found || pk < best_pk) { found = true; best_pk = pk; best_mask = mask; }
+      return;
+    }
+    if (L - l < left) return;
+    // even the `left` largest savings below cannot bring the head event under R
+    if (prefix + suf_a[l] - (int64_t)left * suf_dmax[l] + s.Hd + s.Th > R) return;
+    const int64_t here = prefix + need[l];              // layer l's forward / backward events
+    if (here > R) return;                               // fixed by the choices below l
+    const int64_t rm = std::max(runmax, here);
+    if (left > 0) dfs(l + 1, left - 1, prefix + s.y[l], rm, mask | (1ull << l));   // drop first: lex order
+    dfs(l + 1, left, prefix + s.a[l], rm, mask);
+  }
+};
+}  // namespace
+
+PlanResult plan_exact(const Series& s, int64_t budget, int64_t reserve) {
+  const int L = (int)s.a.size();
+  const int64_t base = s.C + s.E;
+  ExactSearch x{s, L, budget - reserve - base, 0, {}};
+  x.need.resize(L);
+  for (int l = 0; l < L; ++l) x.need[l] = std::max(s.a[l], s.a[l] - s.y[l] + s.Tb);
+  x.suf_a.assign(L + 1, 0);
+  x.suf_dmax.assign(L + 1, 0);
+  for (int l = L - 1; l >= 0; --l) {
+    x.suf_a[l] = x.suf_a[l + 1] + s.a[l];
+    x.suf_dmax[l] = std::max(x.suf_dmax[l + 1], s.a[l] - s.y[l]);
+  }
+  if (s.Te <= x.R) {
+    for (int k = 0; k <= L && !x.found; ++k) {
+      x.k = k;
+      x.dfs(0, k, 0, s.Te, 0);
+    }
+  }
+  if (!x.found) {
+    const uint64_t all = L >= 64 ? ~0ull : ((1ull << L) - 1);
+    return {false, all, predicted_peak(s, all)};
+  }
+  return {true, x.best_mask, base + x.best_pk};
+}
+
 void Estimator::fit(const std::vector<Sample>& smp, int degree) {
   const int L = (int)smp.front().a.size();
   std::vector<int64_t> xs;

@@ -38,6 +38,16 @@ struct PlanResult {
 // Algorithm 1 (A1-A11) + last-layer exclusion (A12) + verify (A13).
 PlanResult plan_greedy(const Series& s, int64_t budget, int64_t reserve, int bucket_num, int bucket_den);
 
+// The exact alternative behind the same (M, x, L) -> L' interface ("a
+// flexible interface ... such as the Knapsack optimization"): among all drop
+// sets whose position-aware predicted peak is <= budget - reserve, the one with
+// the fewest recomputed layers (unit recompute cost: the encoder layers are
+// homogeneous), then the lowest peak, then the lexicographically smallest
+// sorted layer list.  Depth-first over layers in order with the exact prefix
+// constraints of predicted_peak as pruning (reading A29).
+PlanResult plan_exact(const Series& s, int64_t budget, int64_t reserve);
+enum PlannerKind : int { PLANNER_GREEDY = 0, PLANNER_EXACT = 1 };
+
 // One collected sheltered-iteration sample (arena deltas).
 struct Sample {
   int64_t x = 0, C = 0, E = 0, Hd = 0, Th = 0, Tb = 0, Te = 0;

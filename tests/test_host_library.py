@@ -170,3 +170,56 @@ def test_call_order_and_budget_errors():
     with pytest.raises(mb.MimoseError) as e:
         mb.Mimose(cfg, om.sizes(cfg, 2, 32).C - 1)
     assert e.value.status == mb.E_INFEASIBLE
+
+
+def _random_series(rng, L, hom):
+    ys = [rng.randint(1, 50)] * L if hom else [rng.randint(1, 50) for _ in range(L)]
+    a = [ys[0] + rng.randint(1, 200)] * L if hom else [ys[l] + rng.randint(1, 200) for l in range(L)]
+    return dict(C=rng.randint(0, 1000), E=rng.randint(1, 100), a=a, y=ys, Hd=rng.randint(0, 20),
+                Th=rng.randint(1, 100), Tb=rng.randint(50, 400), Te=rng.randint(1, 300))
+
+
+def test_exact_planner_matches_brute_force():
+    """Reading A29: the library's exact planner (mimose_set_planner kind 1) equals
+    the oracle's brute force over all drop sets (fewest layers, then lowest
+    peak, then lexicographically smallest), and never recomputes more layers
+    than Algorithm 1; on homogeneous stacks the two coincide."""
+    rng = random.Random(29)
+    fewer = 0
+    for it in range(800):
+        L = rng.randint(1, 11)
+        hom = it % 2 == 0
+        p = _random_series(rng, L, hom)
+        lo, hi = op.predicted_peak(p, range(L)), op.predicted_peak(p, [])
+        M = rng.randint(lo - 5, hi + 5)
+        st, dropped, pk = mb.plan_series(p, M, planner=mb.PLANNER_EXACT)
+        ost, odropped, opk = op.plan_exact(p, M)
+        assert (st == mb.OK) == (ost == op.OK)
+        if ost == op.OK:
+            assert dropped == odropped and pk == opk <= M
+            gst, gdropped, gpk = mb.plan_series(p, M)
+            assert gst == mb.OK and len(dropped) <= len(gdropped)
+            if hom:
+                assert dropped == gdropped and pk == gpk
+            fewer += len(dropped) < len(gdropped)
+    assert fewer > 0        # heterogeneous stacks where the exact plan recomputes less
+
+
+@pytest.mark.parametrize("name", CFGS)
+def test_exact_planner_on_config_series(name):
+    """24-layer series of the real configs: feasible whenever greedy is, never
+    more layers, within the budget, and fast enough for a cache miss."""
+    import time
+    cfg = wl.CONFIGS[name]
+    M = budget_for(cfg)
+    worst = 0.0
+    for S in range(cfg.pad, cfg.max_seq + 1, max(cfg.pad, cfg.max_seq // 8)):
+        p = om.collect_samples(om.sizes(cfg, cfg.n_seqs, S))
+        t0 = time.perf_counter()
+        st, dropped, pk = mb.plan_series(p, M, planner=mb.PLANNER_EXACT)
+        worst = max(worst, time.perf_counter() - t0)
+        gst, gdropped, gpk = mb.plan_series(p, M)
+        assert (st == mb.OK) == (gst == mb.OK)
+        if st == mb.OK:
+            assert pk <= M and pk == op.predicted_peak(p, dropped) and len(dropped) <= len(gdropped)
+    assert worst < 0.5, worst
