@@ -23,6 +23,12 @@ bool attn_fwd_tc(const void* qkv, const int32_t* lengths, void* O, float* lse, i
 bool attn_bwd_tc(const void* qkv, const void* O, const void* dO, const float* lse, const int32_t* lengths,
                  void* dqkv, int B, int S, int H, int h, Drop drop, cudaStream_t st, bool causal);
 
+// tcgen05 versions for 128 < S <= 1024 (kernels_attn_tcl.cu)
+bool attn_fwd_tcl(const void* qkv, const int32_t* lengths, void* O, float* lse, int B, int S, int H, int h,
+                  Drop drop, cudaStream_t st, bool causal);
+bool attn_bwd_tcl(const void* qkv, const void* O, const void* dO, const float* lse, const int32_t* lengths,
+                  float* Dbuf, void* dqkv, int B, int S, int H, int h, Drop drop, cudaStream_t st, bool causal);
+
 static bool g_attn_tc = true;
 void set_attn_tc(bool on) { g_attn_tc = on; }
 bool attn_tc_enabled() { return g_attn_tc; }
@@ -101,7 +107,10 @@ __global__ void __launch_bounds__(AT) k_attn_fwd(const E* __restrict__ qkv, cons
 void attn_fwd(DType dt, const void* qkv, const int32_t* lengths, void* O, float* lse, int B, int S, int H,
               int h, Drop drop, cudaStream_t st, bool causal) {
   note_launch(1);
-  if (dt == DT_BF16 && attn_tc_enabled() && attn_fwd_tc(qkv, lengths, O, lse, B, S, H, h, drop, st, causal)) return;
+  if (dt == DT_BF16 && attn_tc_enabled() &&
+      (attn_fwd_tc(qkv, lengths, O, lse, B, S, H, h, drop, st, causal) ||
+       attn_fwd_tcl(qkv, lengths, O, lse, B, S, H, h, drop, st, causal)))
+    return;
   const int D = H / h;
   const float scale = 1.0f / sqrtf((float)D);
   dim3 grid(cdiv(S, AT), B * h);
@@ -265,6 +274,11 @@ void attn_bwd(DType dt, const void* qkv, const void* O, const void* dO, const fl
   if (dt == DT_BF16 && attn_tc_enabled() &&
       attn_bwd_tc(qkv, O, dO, lse, lengths, dqkv, B, S, H, h, drop, st, causal)) {
     note_launch(1);
+    return;
+  }
+  if (dt == DT_BF16 && attn_tc_enabled() &&
+      attn_bwd_tcl(qkv, O, dO, lse, lengths, Dbuf, dqkv, B, S, H, h, drop, st, causal)) {
+    note_launch(2);
     return;
   }
   const int D = H / h;

@@ -88,21 +88,27 @@ CASES = {
                                max_pos=64, n_seqs=8, seq_lo=8, seq_hi=40, pad=8),
     "qa-bf16": wl.small_config("bert-large", n_layers=2, hidden=128, heads=2, ffn=512, vocab=300,
                                max_pos=80, n_seqs=3, seq_lo=20, seq_hi=72, pad=8),
-    # S > 128: the bf16 attention takes the SIMT path (tcgen05 tile covers S <= 128)
+    # S > 128: the bf16 attention takes the tiled tcgen05 kernels (kernels_attn_tcl.cu):
+    # 2 tiles with a ragged tail, and 4-5 tiles up to S = 520
     "qa-bf16-long": wl.small_config("bert-large", n_layers=2, hidden=128, heads=2, ffn=256, vocab=300,
                                     max_pos=200, n_seqs=2, seq_lo=130, seq_hi=190, pad=8),
+    "qa-bf16-xlong": wl.small_config("bert-large", n_layers=2, hidden=128, heads=2, ffn=256, vocab=300,
+                                     max_pos=520, n_seqs=2, seq_lo=390, seq_hi=520, pad=8),
     "qa-fp32": wl.small_config("bert-large", n_layers=2, hidden=64, heads=2, ffn=128, vocab=300,
                                max_pos=80, n_seqs=3, seq_lo=20, seq_hi=70, pad=1, dtype="fp32"),
     "mc-roberta-bf16": wl.small_config("roberta-large", n_layers=2, hidden=128, heads=2, ffn=256,
                                        vocab=700, max_pos=66, n_seqs=8, seq_lo=10, seq_hi=64, pad=8),
-    # GPT-2 (pre-LN, causal, tied LM head, chunked CE): tcgen05 attention (S <= 128),
-    # SIMT causal attention (S > 128), fp32
+    # GPT-2 (pre-LN, causal, tied LM head, chunked CE): tcgen05 attention (S <= 128
+    # one tile; S > 128 tiled, causal tile skipping), fp32 (SIMT)
     "lm-gpt2-bf16": wl.small_config("gpt2-medium", n_layers=2, hidden=128, heads=2, ffn=256, vocab=600,
                                     max_pos=128, n_seqs=3, seq_lo=40, seq_hi=120, pad=8, pad_id=599,
                                     cls_id=599, sep_id=599),
     "lm-gpt2-bf16-long": wl.small_config("gpt2-medium", n_layers=2, hidden=128, heads=2, ffn=256, vocab=600,
                                          max_pos=256, n_seqs=2, seq_lo=130, seq_hi=200, pad=8, pad_id=599,
                                          cls_id=599, sep_id=599),
+    "lm-gpt2-bf16-xlong": wl.small_config("gpt2-medium", n_layers=2, hidden=128, heads=2, ffn=256, vocab=600,
+                                          max_pos=640, n_seqs=1, seq_lo=500, seq_hi=632, pad=8, pad_id=599,
+                                          cls_id=599, sep_id=599),
     "lm-gpt2-fp32": wl.small_config("gpt2-medium", n_layers=2, hidden=64, heads=2, ffn=128, vocab=300,
                                     max_pos=64, n_seqs=3, seq_lo=10, seq_hi=50, pad=1, pad_id=299,
                                     cls_id=299, sep_id=299, dtype="fp32"),
