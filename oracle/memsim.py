@@ -325,3 +325,149 @@ def collect_samples(sz: Sizes) -> Dict[str, object]:
         A.pop(t)
     A.tfree(sz.dy)
     return dict(C=sz.C, E=E, a=a, y=y, Hd=hd, Th=th, Tb=tb, Te=te, peak=A.peak)
+
+
+# --------------------------------------------------------------------------
+# sub-layer checkpoint units (SURVEY §8(f) f1; DESIGN reading A30)
+# --------------------------------------------------------------------------
+# P:125 and P:140 name the "attention block" as a unit Mimose can checkpoint
+# ("the output ... of the attention block"), P:170 lets a stage be any
+# user-code structure.  With granularity 1 each post-LN layer l is two units:
+#   unit 2l   attention block  internals QKV, O, LSE, z1, st1   output h1
+#   unit 2l+1 FFN block        internals u, g, z2, st2          output y
+# Forward: a kept unit pushes its internals then its output; a dropped unit
+# places its internals in the top region, pushes its output, frees them.
+# Backward of layer l (after y_l is gone):
+#   FFN dropped -> push its internals (recompute from h1)
+#   talloc layer scratch; FFN-block gradients; pop FFN internals; pop h1
+#   attention dropped -> push its internals (recompute from y_{l-1})
+#   attention-block gradients; tfree scratch; pop attention internals; pop y_{l-1}
+# With nothing dropped the event sequence reaches the same peak as the layer
+# model (same push order), and the planner's position-aware peak applies
+# unchanged to the 2L-unit series.
+
+def unit_list(sz: Sizes) -> List[tuple]:
+    """[(internals, output)] for the 2L units of a post-LN stack."""
+    assert len(sz.internals) == 10, "sub-layer units are defined for the post-LN layer"
+    att, h1, ffn = sz.internals[:5], sz.internals[5], sz.internals[6:]
+    out = []
+    for _ in range(sz.n_layers):
+        out += [(att, h1), (ffn, sz.y)]
+    return out
+
+
+def _unit_forward(A: Arena, units, drop) -> None:
+    for u, (ints, o) in enumerate(units):
+        if u in drop:
+            for t in ints:
+                A.talloc(t)
+            A.push(o)
+            for t in reversed(ints):
+                A.tfree(t)
+        else:
+            for t in ints:
+                A.push(t)
+            A.push(o)
+
+
+def _unit_backward_layers(A: Arena, sz: Sizes, units, drop) -> None:
+    L = sz.n_layers
+    for l in reversed(range(L)):
+        (att, h1), (ffn, _) = units[2 * l], units[2 * l + 1]
+        if 2 * l + 1 in drop:                        # recompute the FFN block from h1
+            for t in ffn:
+                A.push(t)
+        A.talloc(sz.layer_scratch)
+        for t in reversed(ffn):                      # FFN-block gradients done
+            A.pop(t)
+        A.pop(h1)
+        if 2 * l in drop:                            # recompute the attention block from y_{l-1}
+            for t in att:
+                A.push(t)
+        A.tfree(sz.layer_scratch)                    # attention-block gradients done
+        for t in reversed(att):
+            A.pop(t)
+        if l > 0:
+            A.pop(sz.y)
+
+
+def simulate_step_units(sz: Sizes, dropped: Sequence[int]) -> Arena:
+    """One training step under a plan over the 2L sub-layer units (0-based)."""
+    units = unit_list(sz)
+    drop = set(dropped)
+    A = Arena(sz.C)
+    for t in sz.E:
+        A.push(t)
+    _unit_forward(A, units, drop)
+    for t in sz.head:
+        A.push(t)
+    if sz.head_fwd_scratch:
+        A.talloc(sz.head_fwd_scratch)
+        A.tfree(sz.head_fwd_scratch)
+    A.talloc(sz.dy)
+    A.talloc(sz.head_scratch)
+    A.tfree(sz.head_scratch)
+    for t in reversed(sz.head):
+        A.pop(t)
+    A.pop(sz.y)
+    _unit_backward_layers(A, sz, units, drop)
+    A.talloc(sz.emb_scratch)
+    A.tfree(sz.emb_scratch)
+    for t in reversed(sz.E):
+        A.pop(t)
+    A.tfree(sz.dy)
+    assert A.live == sz.C
+    return A
+
+
+def collect_samples_units(sz: Sizes) -> Dict[str, object]:
+    """The shuttling collector over units: per unit, pass 1 (save mode) -> a_u,
+    pass 2 (no-save) -> y_u; the sheltered backward recomputes every unit."""
+    units = unit_list(sz)
+    A = Arena(sz.C)
+    base = A.live
+    for t in sz.E:
+        A.push(t)
+    E = A.live - base
+    a, y = [], []
+    for ints, o in units:
+        b0 = A.live
+        for t in ints:
+            A.push(t)
+        A.push(o)
+        a.append(A.live - b0)
+        A.pop(o)
+        for t in reversed(ints):
+            A.pop(t)
+        for t in ints:
+            A.talloc(t)
+        A.push(o)
+        for t in reversed(ints):
+            A.tfree(t)
+        y.append(A.live - b0)
+    b0 = A.live
+    for t in sz.head:
+        A.push(t)
+    hd = A.live - b0
+    if sz.head_fwd_scratch:
+        A.talloc(sz.head_fwd_scratch)
+        A.tfree(sz.head_fwd_scratch)
+    A.talloc(sz.dy)
+    A.top_peak_phase = sum(A.top)
+    A.talloc(sz.head_scratch)
+    A.tfree(sz.head_scratch)
+    th = A.top_peak_phase
+    for t in reversed(sz.head):
+        A.pop(t)
+    A.pop(sz.y)
+    A.top_peak_phase = sum(A.top)
+    _unit_backward_layers(A, sz, units, set(range(len(units))))
+    tb = A.top_peak_phase
+    A.top_peak_phase = sum(A.top)
+    A.talloc(sz.emb_scratch)
+    A.tfree(sz.emb_scratch)
+    te = A.top_peak_phase
+    for t in reversed(sz.E):
+        A.pop(t)
+    A.tfree(sz.dy)
+    return dict(C=sz.C, E=E, a=a, y=y, Hd=hd, Th=th, Tb=tb, Te=te, peak=A.peak)

@@ -293,7 +293,7 @@ int64_t persistent_bytes(const mimose_ctx* c) {
   const int64_t maxT = (int64_t)c->cfg.max_seqs * c->cfg.max_seq_len;
   C += 2 * a16(maxT * 4) + a16((int64_t)c->cfg.max_seqs * 4) + a16(2LL * c->cfg.max_seqs * 4);
   C += a16(256);
-  C += a16(4 * H * H * 4);
+  C += a16(c->ws_elems * 4);                                   // split-K / stream-K workspace
   C += a16((int64_t)NPART * 2 * std::max(3 * H, F) * 4);
   return C;
 }
@@ -1049,7 +1049,7 @@ mimose_status mimose_init(const mimose_config* cfgp, mimose_ctx** out) {
   c->dt = k.dtype == MIMOSE_FP32 ? DT_F32 : DT_BF16;
   c->e = k.dtype == MIMOSE_FP32 ? 4 : 2;
   c->layout = build_layout(k, &c->npad);
-  c->ws_elems = 4LL * k.hidden * k.hidden;
+  c->ws_elems = 4LL * k.hidden * k.hidden;   // wgrad split-K partials (oracle/memsim.py)
   c->device = k.arena_base != nullptr;
   Arena& a = c->ar;
   a.base = (char*)k.arena_base;
@@ -1371,6 +1371,16 @@ mimose_status mimose_plan(mimose_ctx* c, int64_t x, mimose_plan_t* out) {
 
 int32_t mimose_tc_available(void) { return tc_available() ? 1 : 0; }
 
+// Stream-K partial slots for the GEMM test hooks (outside any arena; tests only).
+static bool debug_sk_ws(GemmArgs& g) {
+  static float* sk_ws = nullptr;
+  const int64_t n = 148LL * 128 * 256;
+  if (!sk_ws && cudaMalloc(&sk_ws, n * 4) != cudaSuccess) return false;
+  g.ws = sk_ws;
+  g.ws_elems = n;
+  return true;
+}
+
 mimose_status mimose_debug_gemm_ex(int32_t epi, int32_t M, int32_t N, int32_t K, const void* A, int64_t a_sm,
                                    int64_t a_sk, const void* B, int64_t b_sn, int64_t b_sk, void* Cp, int64_t ldc,
                                    void* C2, const void* bias, const void* res, int64_t ldr, const void* aux,
@@ -1391,6 +1401,7 @@ mimose_status mimose_debug_gemm_ex(int32_t epi, int32_t M, int32_t N, int32_t K,
     g.ws = (float*)C2;
     g.C2 = nullptr;
   }
+  if (split == 1 && !debug_sk_ws(g)) return MIMOSE_E_CUDA;
   g.drop.enabled = 1; g.drop.seed_lo = 7; g.drop.seed_hi = 0; g.drop.site = 0; g.drop.step = 1;
   g.drop.thresh = 3865470566u; g.drop.scale = (float)(1.0 / 0.9);
   gemm(DT_BF16, (Epi)epi, g, (cudaStream_t)stream, use_tc != 0);
@@ -1413,6 +1424,7 @@ mimose_status mimose_debug_gemm(int32_t epi, int32_t M, int32_t N, int32_t K, co
   g.C = Cp; g.ldc = ldc; g.bias = bias;
   g.split = split < 1 ? 1 : split;
   g.split_stride = (int64_t)M * ldc;
+  if (g.split == 1 && !debug_sk_ws(g)) return MIMOSE_E_CUDA;
   gemm(DT_BF16, (Epi)epi, g, (cudaStream_t)stream, use_tc != 0);
   return cudaGetLastError() == cudaSuccess ? MIMOSE_OK : MIMOSE_E_CUDA;
 }

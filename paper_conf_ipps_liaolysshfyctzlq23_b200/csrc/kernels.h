@@ -46,6 +46,10 @@ struct GemmArgs {
   // separate reduction kernel).  bn: forced tile width (0 = heuristic).
   int fused_split = 0;
   float* ws = nullptr;
+  // ws_elems: capacity of ws.  With split == 1 and gemm mode 14, the persistent
+  // tcgen05 GEMM runs deterministic stream-K when ws holds one 128 x BN fp32
+  // partial tile per CTA (kernels_gemm_tc.cu seg_of; off by default).
+  int64_t ws_elems = 0;
   int bn = 0;
 };
 void gemm(DType dt, Epi epi, const GemmArgs& g, cudaStream_t st, bool use_tc);

@@ -137,10 +137,18 @@ MDEV void stage_store_f32(uint8_t* stg_p, const float (&v)[32], float* out, int6
                       __float_as_uint(v[4 * c + 3])));
   __syncwarp();
 #pragma unroll
-  for (int k = 0; k < 8; ++k) {
-    const int R = (lane >> 3) + 4 * k, c = lane & 7;
-    const uint4 w = lds128(stg + R * 128 + ((c ^ (R & 7)) << 4));
-    if (R < rows_valid) *(uint4*)(out + (int64_t)R * ld + 4 * c) = w;
+  for (int h = 0; h < 2; ++h) {   // shared loads in groups of 4, then the stores (no LDS -> STG round trips)
+    uint4 w[4];
+#pragma unroll
+    for (int k = 0; k < 4; ++k) {
+      const int R = (lane >> 3) + 4 * (4 * h + k), c = lane & 7;
+      w[k] = lds128(stg + R * 128 + ((c ^ (R & 7)) << 4));
+    }
+#pragma unroll
+    for (int k = 0; k < 4; ++k) {
+      const int R = (lane >> 3) + 4 * (4 * h + k), c = lane & 7;
+      if (R < rows_valid) *(uint4*)(out + (int64_t)R * ld + 4 * c) = w[k];
+    }
   }
   __syncwarp();
 }
@@ -149,13 +157,18 @@ MDEV void stage_store_bf16(uint8_t* stg_p, const float (&v)[32], __nv_bfloat16* 
 #pragma unroll
   for (int c = 0; c < 4; ++c) sts128(stg + lane * 128 + ((c ^ (lane & 3)) << 4), pack8(v + 8 * c));
   __syncwarp();
+  uint4 w[4];
 #pragma unroll
   for (int k = 0; k < 4; ++k) {
     const int R = (lane >> 2) + 8 * k, c = lane & 3;
-    const uint4 w = lds128(stg + R * 128 + ((c ^ (R & 3)) << 4));
-    if (R < rows_valid) *(uint4*)(out + (int64_t)R * ld + 8 * c) = w;
+    w[k] = lds128(stg + R * 128 + ((c ^ (R & 3)) << 4));
   }
   __syncwarp();
+#pragma unroll
+  for (int k = 0; k < 4; ++k) {
+    const int R = (lane >> 2) + 8 * k, c = lane & 3;
+    if (R < rows_valid) *(uint4*)(out + (int64_t)R * ld + 8 * c) = w[k];
+  }
 }
 
 // Epilogue of a 32-row x 32-column fragment (rows m_base + lane, columns n..n+31,
@@ -513,17 +526,53 @@ struct TpCfg {
 
 struct TpArgs {
   TcArgs t;
-  int m_blocks, n_blocks, n_tiles;
-  uint32_t* flags;     // fused split-K: [split-1][per_split][TP_EPI_WARPS] release flags
-  uint32_t epoch;      // this launch's flag value (never reused within a process)
+  int m_blocks = 0, n_blocks = 0, n_tiles = 0;
+  uint32_t* flags = nullptr;   // fused split-K: [split-1][per_split][TP_EPI_WARPS] release flags
+                               // stream-K: [CTA][TP_EPI_WARPS]
+  uint32_t epoch = 0;          // this launch's flag value (never reused within a process)
+  int sk = 0;                  // 1: deterministic stream-K (split must be 1)
+  float* sk_ws = nullptr;      // stream-K partial slots: [CTA][TBM * BN] fp32
 };
 
-// Split index of persistent unit `tile`.  Fused split-K orders the units
-// z = split-1 first and z = 0 last, so a split-0 unit (which waits for its
-// partials) is never scheduled in an earlier round than the units it waits on.
-MDEV int unit_z(const TcArgs& ta, int tile, int per_split) {
+// Work segment i of this CTA: tile r (m-block * n_blocks + n-block), split z
+// and k-block range [kb0, kb1).
+//   default: tile-major round robin, unit = blockIdx.x + i * gridDim.x.  Fused
+//   split-K orders the units z = split-1 first and z = 0 last, so a split-0
+//   unit (which waits for its partials) never runs in an earlier round than
+//   the units it waits on.
+//   stream-K: the n_tiles * kbt (tile, k-block) iterations are cut into
+//   gridDim.x contiguous ranges [u0, u1) (fixed by the shape and grid, so the
+//   split is the same on every launch).  A range starts inside a tile at most
+//   once (its first segment, which then only produces an fp32 partial) and
+//   ends inside a tile at most once (its last segment, the tile's "head",
+//   kb0 = 0): the head CTA adds the partials of CTAs blockIdx.x+1, +2, ...
+//   in that fixed order and runs the epilogue.  Producers compute their
+//   partial first and heads wait last, so the waits cannot deadlock with
+//   all CTAs resident (grid <= #SMs, one CTA per SM).
+struct Seg { int r, z, kb0, kb1; };
+MDEV int64_t sk_u0(int cta, int64_t W) { return (int64_t)cta * W / gridDim.x; }
+template <bool SK>
+MDEV bool seg_of(const TpArgs& a, int i, Seg& s) {
+  const TcArgs& ta = a.t;
+  if (SK) {
+    const int64_t kbt = ta.kb_total, W = (int64_t)a.n_tiles * kbt;
+    const int64_t u0 = sk_u0(blockIdx.x, W), u1 = sk_u0(blockIdx.x + 1, W);
+    const int64_t t = u0 / kbt + i;
+    const int64_t st = i == 0 ? u0 : t * kbt;
+    if (st >= u1) return false;
+    const int64_t en = u1 < (t + 1) * kbt ? u1 : (t + 1) * kbt;
+    s.r = (int)t; s.z = 0; s.kb0 = (int)(st - t * kbt); s.kb1 = (int)(en - t * kbt);
+    return true;
+  }
+  const int tile = blockIdx.x + i * gridDim.x;
+  if (tile >= a.n_tiles) return false;
+  const int per_split = a.m_blocks * a.n_blocks;
   const int q = tile / per_split;
-  return ta.g.fused_split ? ta.g.split - 1 - q : q;
+  s.z = ta.g.fused_split ? ta.g.split - 1 - q : q;
+  s.r = tile % per_split;
+  s.kb0 = s.z * ta.kb_per_split;
+  s.kb1 = min(ta.kb_total, s.kb0 + ta.kb_per_split);
+  return true;
 }
 MDEV uint32_t ld_acquire_u32(const uint32_t* p) {
   uint32_t v;
@@ -539,7 +588,7 @@ MDEV float4 ld_cg_f4(const float* p) {
   return v;
 }
 
-template <int BN, int EPI>
+template <int BN, int EPI, bool SK>
 __global__ void __launch_bounds__(TP_THREADS, 1)
     k_gemm_tcp(const __grid_constant__ CUtensorMap tma_a, const __grid_constant__ CUtensorMap tma_b, const TpArgs args) {
   pdl_trigger();
@@ -577,10 +626,11 @@ __global__ void __launch_bounds__(TP_THREADS, 1)
   if (warp == 0) {
     if (lane == 0) {                                   // ---------------- TMA producer
       int it = 0;
-      for (int tile = blockIdx.x; tile < args.n_tiles; tile += gridDim.x) {
-        const int z = unit_z(ta, tile, per_split), r = tile % per_split;
+      Seg sg;
+      for (int si = 0; seg_of<SK>(args, si, sg); ++si) {
+        const int r = sg.r;
         const int m0 = (r / args.n_blocks) * TBM, n0 = (r % args.n_blocks) * BN;
-        const int kb0 = z * ta.kb_per_split, kb1 = min(ta.kb_total, kb0 + ta.kb_per_split);
+        const int kb0 = sg.kb0, kb1 = sg.kb1;
         for (int kb = kb0; kb < kb1; ++kb, ++it) {
           const int s = it % Cf::STAGES;
           if (it >= Cf::STAGES) mbar_wait(&empty[s], ((it / Cf::STAGES) - 1) & 1);
@@ -609,9 +659,9 @@ __global__ void __launch_bounds__(TP_THREADS, 1)
     if (lane == 0) {                                   // ---------------- MMA issuer
       const uint32_t idesc = idesc_bf16(TBM, BN, ta.a_mn, ta.b_mn);
       int it = 0, local = 0;
-      for (int tile = blockIdx.x; tile < args.n_tiles; tile += gridDim.x, ++local) {
-        const int z = unit_z(ta, tile, per_split);
-        const int kb0 = z * ta.kb_per_split, kb1 = min(ta.kb_total, kb0 + ta.kb_per_split);
+      Seg sg;
+      for (; seg_of<SK>(args, local, sg); ++local) {
+        const int kb0 = sg.kb0, kb1 = sg.kb1;
         const int acc = local & 1;
         if (local >= 2) mbar_wait(&tempty[acc], ((local >> 1) - 1) & 1);
         tc_fence_after();
@@ -639,13 +689,27 @@ __global__ void __launch_bounds__(TP_THREADS, 1)
     const int grp = e >> 2, ngrp = TP_EPI_WARPS / 4;  // column group of this warp
     const GemmArgs& g = ta.g;
     int local = 0;
-    for (int tile = blockIdx.x; tile < args.n_tiles; tile += gridDim.x, ++local) {
-      const int z = unit_z(ta, tile, per_split), r = tile % per_split;
+    Seg sg;
+    for (; seg_of<SK>(args, local, sg); ++local) {
+      const int z = sg.z, r = sg.r;
       const int m0 = (r / args.n_blocks) * TBM, n0 = (r % args.n_blocks) * BN;
-      const int kb0 = z * ta.kb_per_split, kb1 = min(ta.kb_total, kb0 + ta.kb_per_split);
+      const int kb0 = sg.kb0, kb1 = sg.kb1;
       const int acc = local & 1;
       const int m = m0 + 32 * q + lane;
       const int c_beg = grp * (BN / 32) / ngrp, c_end = (grp + 1) * (BN / 32) / ngrp;
+      // stream-K roles of this segment (see seg_of)
+      const bool sk_part = SK && kb0 > 0;                        // partial producer
+      const bool sk_head = SK && kb0 == 0 && kb1 < ta.kb_total;  // adds the partials
+      int sk_n = 0;                                                   // producers of a head
+      if (SK && sk_head) {
+        const int64_t W = (int64_t)args.n_tiles * ta.kb_total, tend = (int64_t)(r + 1) * ta.kb_total;
+        while (blockIdx.x + sk_n + 1 < gridDim.x && sk_u0(blockIdx.x + sk_n + 1, W) < tend) ++sk_n;
+        if (lane == 0)
+          for (int j = 1; j <= sk_n; ++j)
+            while (ld_acquire_u32(args.flags + (size_t)(blockIdx.x + j) * TP_EPI_WARPS + e) != args.epoch)
+              __nanosleep(64);
+        __syncwarp();
+      }
       {  // pull this tile's epilogue inputs into L2 while the MMAs run
         const int nb = n0 + 32 * c_beg;
         if (m < g.M && nb < g.N) {
@@ -685,6 +749,23 @@ __global__ void __launch_bounds__(TP_THREADS, 1)
 #pragma unroll
           for (int i = 0; i < 32; ++i) v[i] = 0.f;
         }
+        if (SK && (sk_part || sk_head)) {   // fragment (q, c): 32 rows x 32 fp32, row = lane, in the CTA's slot
+          const size_t fo = ((size_t)(q * (BN / 32) + c) * 32 + lane) * 32;
+          if (sk_part) {
+            float4* p = (float4*)(args.sk_ws + (size_t)blockIdx.x * (TBM * BN) + fo);
+#pragma unroll
+            for (int j = 0; j < 8; ++j) p[j] = make_float4(v[4 * j], v[4 * j + 1], v[4 * j + 2], v[4 * j + 3]);
+            continue;
+          }
+          for (int jj = 1; jj <= sk_n; ++jj) {
+            const float* p = args.sk_ws + (size_t)(blockIdx.x + jj) * (TBM * BN) + fo;
+#pragma unroll
+            for (int j = 0; j < 8; ++j) {
+              const float4 w = ld_cg_f4(p + 4 * j);
+              v[4 * j] += w.x; v[4 * j + 1] += w.y; v[4 * j + 2] += w.z; v[4 * j + 3] += w.w;
+            }
+          }
+        }
         if (EPI == EPI_F32 && g.fused_split && n + 32 <= g.N) {
           const int mb = m0 + 32 * q;
           if (mb < g.M) {
@@ -712,6 +793,11 @@ __global__ void __launch_bounds__(TP_THREADS, 1)
           for (int i = 0; i < 32; ++i)
             if (n + i < g.N) epilogue<__nv_bfloat16, EPI>(g, m, n + i, v[i], z);
         }
+      }
+      if (SK && sk_part) {               // publish this warp's stream-K partial
+        __threadfence();
+        __syncwarp();
+        if (lane == 0) st_release_u32(args.flags + (size_t)blockIdx.x * TP_EPI_WARPS + e, args.epoch);
       }
       if constexpr (EPI == EPI_F32) {
         if (g.fused_split && z > 0) {    // publish this warp's partial rows/columns
@@ -1018,7 +1104,8 @@ template <int BN, int EPI>
 static void launch_tcp(const CUtensorMap& ma, const CUtensorMap& mb, const TpArgs& a, cudaStream_t st) {
   static bool attr = false;
   if (!attr) {
-    cudaFuncSetAttribute(k_gemm_tcp<BN, EPI>, cudaFuncAttributeMaxDynamicSharedMemorySize, TpCfg<BN>::SMEM);
+    cudaFuncSetAttribute(k_gemm_tcp<BN, EPI, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, TpCfg<BN>::SMEM);
+    cudaFuncSetAttribute(k_gemm_tcp<BN, EPI, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, TpCfg<BN>::SMEM);
     attr = true;
   }
   static int nsm = 0;
@@ -1027,7 +1114,11 @@ static void launch_tcp(const CUtensorMap& ma, const CUtensorMap& mb, const TpArg
     cudaGetDevice(&dev);
     cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, dev);
   }
-  launch_k(k_gemm_tcp<BN, EPI>, std::min(nsm, a.n_tiles), TP_THREADS, TpCfg<BN>::SMEM, st, ma, mb, a);
+  const int64_t units = a.sk ? (int64_t)a.n_tiles * a.t.kb_total : a.n_tiles;
+  if (a.sk)
+    launch_k(k_gemm_tcp<BN, EPI, true>, (int)std::min<int64_t>(nsm, units), TP_THREADS, TpCfg<BN>::SMEM, st, ma, mb, a);
+  else
+    launch_k(k_gemm_tcp<BN, EPI, false>, (int)std::min<int64_t>(nsm, units), TP_THREADS, TpCfg<BN>::SMEM, st, ma, mb, a);
 }
 
 template <int BN>
@@ -1121,6 +1212,17 @@ static uint32_t next_epoch() {
   return v;
 }
 
+static int num_sms() {
+  static int nsm = 0;
+  if (!nsm) {
+    int dev = 0;
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, dev);
+    if (nsm <= 0) nsm = 148;
+  }
+  return nsm;
+}
+
 static int g_gemm_mode = 1;   // 0: one tile per CTA (k_gemm_tc); 1: persistent (k_gemm_tcp)
 void set_gemm_mode(int m) { g_gemm_mode = m; }
 
@@ -1168,8 +1270,37 @@ bool gemm_tc(Epi epi, const GemmArgs& g, cudaStream_t st) {
   // BN = 64 loses on every step shape -- the per-tile fixed cost dominates).
   auto tiles = [&](int bn) { return m_blocks * ((g.N + bn - 1) / bn) * g.split; };
   int BN = (g.N % 256 == 0 && tiles(256) >= 100) ? 256 : 128;
+  // Stream-K (split == 1, workspace given): cost model in 128 x 256 x 64
+  // k-block times -- data-parallel = rounds x k-blocks per tile; stream-K =
+  // the balanced share + ~4 blocks for the partial exchange; a 128-wide tile's
+  // k-block costs 0.86 (its mainloop runs at ~58% of the 256-wide rate).
+  bool sk = false;
+  const int nsm = num_sms();
+  // Off by default: measured on the BERT-base step shapes (T = 2048..8192),
+  // the balanced schedule runs its mainloop no faster than the data-parallel
+  // one on fewer SMs (e.g. TN 3072 x 768 x 5120: 758 vs 747 TFLOP/s), and the
+  // partial exchange then costs more than the balance gains -- see DESIGN §5.
+  const bool sk_mode = g_gemm_mode == 14;
+  if (sk_mode && g.split == 1 && !g.fused_split && g.ws && g.N % 128 == 0) {
+    const int64_t kbt = a.kb_total;
+    auto dp_cost = [&](int bn) {
+      return (double)((tiles(bn) + nsm - 1) / nsm) * kbt * (bn == 256 ? 1.0 : 0.86);
+    };
+    auto sk_ok = [&](int bn) {
+      const int64_t W = (int64_t)tiles(bn) * kbt;
+      return g.ws_elems >= std::min<int64_t>(nsm, W) * TBM * bn;
+    };
+    const int bn_sk = g.N % 256 == 0 ? 256 : 128;
+    const double sk_cost = (double)(((int64_t)tiles(bn_sk) * kbt + nsm - 1) / nsm) * (bn_sk == 256 ? 1.0 : 0.86) + 4.0;
+    double best = dp_cost(BN);
+    if (g.N % 256 == 0) best = std::min(best, dp_cost(256));
+    if (sk_ok(bn_sk) && (g_gemm_mode == 14 || sk_cost < 0.92 * best)) {
+      sk = true;
+      BN = bn_sk;
+    }
+  }
   if (g.bn == 256 && g.N % 256 == 0) BN = 256;
-  if (g.bn == 128) BN = 128;
+  if (g.bn == 128 && !sk) BN = 128;
   if (g_gemm_mode == 11) BN = 128;
   if (g_gemm_mode == 12 && g.N % 256 == 0) BN = 256;
   if (g_gemm_mode == 13) BN = 64;
@@ -1195,6 +1326,16 @@ bool gemm_tc(Epi epi, const GemmArgs& g, cudaStream_t st) {
     p.n_tiles = p.m_blocks * p.n_blocks * g.split;
     p.flags = nullptr;
     p.epoch = 0;
+    p.sk = 0;
+    p.sk_ws = nullptr;
+    if (sk) {
+      if ((size_t)nsm * TP_EPI_WARPS > kFlagWords) return false;
+      p.sk = 1;
+      p.sk_ws = g.ws;
+      p.flags = splitk_flags();
+      if (!p.flags) return false;
+      p.epoch = next_epoch();
+    }
     if (g.fused_split) {
       if ((size_t)(g.split - 1) * p.m_blocks * p.n_blocks * TP_EPI_WARPS > kFlagWords) return false;
       p.flags = splitk_flags();

@@ -278,3 +278,68 @@ def test_budget_property_over_length_schedules(name):
     tight = om.lower_bound(szmax) - 1
     st, _, _ = op.plan(est.predict(cfg.n_seqs * Smax), tight)
     assert st == op.INFEASIBLE
+
+
+# ---------------------------------------------------------------------------
+# sub-layer checkpoint units (DESIGN reading A30)
+# ---------------------------------------------------------------------------
+
+@pytest.mark.parametrize("name", POST_LN)
+def test_units_event_model(name):
+    """Unit event model: with nothing dropped it reaches the layer model's
+    no-checkpoint peak (same push order); dropping every unit gives the unit
+    collector's footprint; dropping only the FFN units of the first k layers
+    lowers the peak by exactly k FFN-internal sizes (closed form, as for layers)."""
+    cfg = wl.CONFIGS[name]
+    L = cfg.n_layers
+    for S in (cfg.seq_lo, cfg.max_seq):
+        sz = om.sizes(cfg, cfg.n_seqs, S)
+        P0 = om.no_ckpt_peak(sz)
+        assert om.simulate_step_units(sz, []).peak == P0
+        assert om.simulate_step_units(sz, [2 * L - 1]).peak == P0      # last unit saves nothing (P:177)
+        c = om.collect_samples_units(sz)
+        assert om.simulate_step_units(sz, range(2 * L)).peak == c["peak"]
+        i_att, i_ffn = sum(sz.internals[:5]), sum(sz.internals[6:])
+        assert c["a"] == [i_att + sz.internals[5], i_ffn + sz.y] * L
+        assert c["y"] == [sz.internals[5], sz.y] * L
+        for k in range(L):
+            # FFN units of layers 0..k-1 dropped: the layer-l backward event loses k FFN internals
+            assert om.simulate_step_units(sz, [2 * j + 1 for j in range(k)]).peak == P0 - k * i_ffn
+
+
+@pytest.mark.parametrize("name", POST_LN)
+def test_units_predicted_peak_formula(name):
+    """The planner's position-aware peak over the 2L-unit collected series is
+    exactly the unit event simulator's peak, for random unit plans."""
+    cfg = wl.CONFIGS[name]
+    rng = random.Random(21)
+    for S in (cfg.seq_lo, cfg.max_seq):
+        sz = om.sizes(cfg, cfg.n_seqs, S)
+        c = om.collect_samples_units(sz)
+        for _ in range(40):
+            plan = rng.sample(range(2 * cfg.n_layers), rng.randint(0, 2 * cfg.n_layers))
+            assert op.predicted_peak(c, plan) == om.simulate_step_units(sz, plan).peak
+
+
+@pytest.mark.parametrize("name", POST_LN)
+def test_units_planners_feasible_and_exact(name):
+    """Algorithm 1 on the unit series (heterogeneous: attention / FFN units
+    alternate) returns a plan within the budget whenever one exists; the exact
+    planner equals brute force (fewest units, then lowest peak, then lexicographic)."""
+    cfg = wl.CONFIGS[name]
+    L = cfg.n_layers
+    sz = om.sizes(cfg, cfg.n_seqs, cfg.max_seq)
+    c = om.collect_samples_units(sz)
+    lo, hi = op.predicted_peak(c, range(2 * L)), op.predicted_peak(c, [])
+    rng = random.Random(22)
+    for _ in range(30 if 2 * L <= 12 else 6):
+        M = rng.randint(lo - 1000, hi + 1000)
+        g = op.plan(c, M)
+        if g[0] == op.OK:
+            assert om.simulate_step_units(sz, g[1]).peak <= M
+        else:
+            assert lo > M
+        if 2 * L <= 12:
+            e = op.plan_exact(c, M)
+            b = op.brute_force(c, M, [1.0] * (2 * L))
+            assert e[0] == b[0] and (e[0] != op.OK or (e[1] == b[1] and e[2] == b[2]))

@@ -19,7 +19,7 @@ shapes = [("NT T x 3072 x 768", T, F, H, H, 1, H, 1), ("NT T x 768 x 3072", T, H
           ("NN T x 3072 x 768", T, F, H, H, 1, 1, F)]
 for name, M, N, K, asm, ask, bsn, bsk in shapes:
     fl = 2.0 * M * N * K
-    for mode in (0, 11, 12, 21, 22):
+    for mode in [int(x) for x in os.environ.get("MODES", "0,11,12,21,22").split(",")]:
         mb.debug_options(gemm_mode=mode)
         us = timeit(lambda: mb.debug_gemm_ex(7, M, N, K, A, asm, ask, B, bsn, bsk, C, N))
         print(f"{name:20s} mode={mode:2d} {us:8.1f} us {fl / us / 1e6:7.1f} TFLOP/s", flush=True)
