@@ -44,6 +44,8 @@ def parse():
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--simt", action="store_true", help="SIMT GEMMs instead of tcgen05")
     ap.add_argument("--gemm-mode", type=int, default=-1, help="tcgen05 GEMM variant (debug_options)")
+    ap.add_argument("--granularity", type=int, default=0, choices=[0, 1],
+                    help="checkpoint units of the headline arm: 0 layers (paper, A14), 1 attention/FFN blocks (A30)")
     ap.add_argument("--planner", default="greedy", choices=["greedy", "exact"],
                     help="Algorithm 1 (default) or the exact fewest-recompute planner (reading A29)")
     return ap.parse_args()
@@ -249,10 +251,10 @@ def main():
         dist.broadcast(t, 0)
         nccl_id = bytes(t.cpu().numpy().tolist())
 
-    def new_ctx(budget, slab_bytes, enforce=1):
+    def new_ctx(budget, slab_bytes, enforce=1, **kw):
         slab = torch.empty(slab_bytes, dtype=torch.uint8, device="cuda")
         ctx = mb.Mimose(cfg, budget, slab=slab, stream=stream, rank=rank, world=world,
-                        nccl_id=nccl_id, enforce_budget=enforce, use_tc=use_tc)
+                        nccl_id=nccl_id, enforce_budget=enforce, use_tc=use_tc, **kw)
         ctx.set_params(wl.pack_params(cfg, wl.init_params(cfg)))
         # AdamW per gradient bucket on a side stream, overlapping the backward
         ctx.set_optimizer(1e-5, fused=True)
@@ -331,7 +333,7 @@ def main():
     samples_per_step = cfg.samples_per_step * world
 
     # ---- Mimose: sheltered phase, then the timed responsive steps ----
-    ctx = new_ctx(M, M)
+    ctx = new_ctx(M, M, granularity=args.granularity)
     t0 = time.perf_counter()
     i = 0
     while ctx.phase == mb.PHASE_SHELTERED:
@@ -405,7 +407,8 @@ def main():
         "e2e": {"value": e2e, "unit": "samples/s", "h2d_bytes_per_step": per_step_h2d, "d2h_bytes_per_step": 4},
         "gpu_launches": launches,
         "clocks": clocks.summary(),
-        "mimose": {"planner": args.planner, "violations": st2["violations"], "peak_bytes_max": st2["max_peak_bytes"],
+        "mimose": {"planner": args.planner, "granularity": "sublayer" if args.granularity else "layer",
+                   "violations": st2["violations"], "peak_bytes_max": st2["max_peak_bytes"],
                    "budget_bytes": M, "mean_layers_dropped": float(np.mean(dropped)),
                    "plan_cache_hits": st2["plan_cache_hits"], "plan_cache_misses": st2["plan_cache_misses"],
                    "planner_us_total": st2["planner_us_total"], "sheltered_iters": st2["collect_steps"],
@@ -444,6 +447,27 @@ def main():
         result["no_ckpt"] = {"value": samples_per_step * args.steps / (ms_n / 1000.0),
                              "ms_per_step": ms_n / args.steps, "peak_bytes": peak_n,
                              "over_budget": peak_n > M}
+        if cfg.arch == wl.ARCH_POST_LN:
+            # sub-layer checkpoint units (reading A30): attention / FFN
+            # blocks planned independently by the same Algorithm 1, same budget
+            ctx = new_ctx(M, M, granularity=1)
+            j = 0
+            while ctx.phase == mb.PHASE_SHELTERED:
+                b = wl.make_batch(cfg, sched[j % len(sched)], seed=wl.batch_seed(cfg, 10**6 + j, rank))
+                ctx.collect(ctx.host_batch(b), want_loss=False)
+                ctx.backward()
+                ctx.step(1e-5)
+                j += 1
+            ms_u, _, _ = timed(ctx, batches, "mimose")
+            stu = ctx.stats()
+            units = [ctx.plan(b.input_size).n_dropped for b in batches[args.warmup:]]
+            ctx.close()
+            del ctx
+            torch.cuda.empty_cache()
+            result["sublayer_units"] = {"value": samples_per_step * args.steps / (ms_u / 1000.0),
+                                        "ms_per_step": ms_u / args.steps, "mean_units_dropped": float(np.mean(units)),
+                                        "units": 2 * cfg.n_layers, "violations": stu["violations"],
+                                        "peak_bytes_max": stu["max_peak_bytes"], "recompute_ratio": ms_u / ms_n}
         result["recompute_ratio"] = ms / ms_n
         result["speedup_vs_static"] = ms_s / ms
         result["paper_context"] = ("V100 (P:227): Mimose ~18.0% faster than Sublinear, ~15.0% than DTR "

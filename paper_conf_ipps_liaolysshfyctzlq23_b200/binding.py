@@ -44,7 +44,8 @@ class Config(C.Structure):
                 ("max_seqs", C.c_int32), ("max_seq_len", C.c_int32),
                 ("arena_base", C.c_void_p), ("arena_bytes", C.c_int64), ("stream", C.c_void_p),
                 ("rank", C.c_int32), ("world", C.c_int32), ("nccl_id", C.c_void_p),
-                ("use_tc", C.c_int32), ("pad_id", C.c_int32), ("reserved", C.c_int32 * 6)]
+                ("use_tc", C.c_int32), ("pad_id", C.c_int32), ("granularity", C.c_int32),
+                ("reserved", C.c_int32 * 5)]
 
 
 class BatchS(C.Structure):
@@ -235,6 +236,8 @@ class Mimose:
         n = C.c_int64()
         _lib.mimose_num_params(self.h, C.byref(n))
         self.n_params = n.value
+        # checkpoint units: layers, or 2L attention / FFN blocks (granularity=1)
+        self.n_units = cfg.n_layers * (2 if c.granularity == 1 else 1)
 
     # -- lifecycle --
     def close(self):
@@ -324,7 +327,7 @@ class Mimose:
     def sample(self, i: int) -> Dict:
         s = SampleS()
         self._chk(_lib.mimose_get_sample(self.h, i, C.byref(s)))
-        return _sample_dict(s, self.cfg.n_layers)
+        return _sample_dict(s, self.n_units)
 
     def dry_run(self, n_seqs: int, seq_len: int, dropped=()) -> int:
         mask = 0
@@ -345,7 +348,7 @@ class Mimose:
     def dry_collect(self, n_seqs: int, seq_len: int) -> Dict:
         s = SampleS()
         self._chk(_lib.mimose_dry_collect(self.h, n_seqs, seq_len, C.byref(s)))
-        return _sample_dict(s, self.cfg.n_layers)
+        return _sample_dict(s, self.n_units)
 
 
 def _sample_dict(s: SampleS, L: int) -> Dict:

@@ -322,6 +322,8 @@ inline int LP(mimose_ctx* c, int l, int k) {
   return layer_base(c) + 12 * l + (c->cfg.arch == 1 ? pre_pos[k] : k);
 }
 inline int HP(mimose_ctx* c, int k) { return layer_base(c) + 12 * c->cfg.n_layers + k; }
+// Checkpoint units: L layers, or 2L sub-layer blocks (granularity 1).
+inline int n_units(const mimose_ctx* c) { return c->cfg.granularity == 1 ? 2 * c->cfg.n_layers : c->cfg.n_layers; }
 
 // ------------------------------------------------------------- probe ------
 void pgemm(mimose_ctx* c, Epi epi, const GemmArgs& g, cudaStream_t st) {
@@ -354,10 +356,13 @@ struct Run {
   cudaStream_t st;
 };
 
-void layer_forward(Run& r, int l, const char* x, LayerBufs& b, char* yout) {
+// Attention block of a post-LN layer: x -> QKV, O, LSE, z1, st1 -> h1 = LN1(z1).
+// h1out == nullptr (sub-layer recompute after h1 was released): the LN1 output
+// store is gated off, the statistics are still written.
+void att_forward(Run& r, int l, const char* x, LayerBufs& b, char* h1out) {
   mimose_ctx* c = r.c;
   if (!r.real) return;
-  const int T = c->T, H = c->cfg.hidden, F = c->cfg.ffn;
+  const int T = c->T, H = c->cfg.hidden;
   GemmArgs g;
   // QKV = x Wqkv^T + b
   g = GemmArgs();
@@ -375,7 +380,15 @@ void layer_forward(Run& r, int l, const char* x, LayerBufs& b, char* yout) {
   g.C = b.z1; g.ldc = H; g.bias = W(c, LP(c, l, L_OB)); g.res = x; g.ldr = H;
   g.drop = make_drop(c, KIND_ATTN_OUT, l);
   pgemm(c, EPI_BIAS_DROP_RES, g, r.st);
-  ln_fwd(c->dt, b.z1, W(c, LP(c, l, L_LN1G)), W(c, LP(c, l, L_LN1B)), b.h1, b.st1, T, H, c->cfg.ln_eps, r.st);
+  ln_fwd(c->dt, b.z1, W(c, LP(c, l, L_LN1G)), W(c, LP(c, l, L_LN1B)), h1out, b.st1, T, H, c->cfg.ln_eps, r.st);
+}
+
+// FFN block: h1 (b.h1) -> u, g, z2, st2 -> y = LN2(z2) (store gated off when yout == nullptr).
+void ffn_forward(Run& r, int l, LayerBufs& b, char* yout) {
+  mimose_ctx* c = r.c;
+  if (!r.real) return;
+  const int T = c->T, H = c->cfg.hidden, F = c->cfg.ffn;
+  GemmArgs g;
   // u = h1 W1^T + b1, g = gelu(u)
   g = GemmArgs();
   g.M = T; g.N = F; g.K = H;
@@ -395,6 +408,11 @@ void layer_forward(Run& r, int l, const char* x, LayerBufs& b, char* yout) {
   ln_fwd(c->dt, b.z2, W(c, LP(c, l, L_LN2G)), W(c, LP(c, l, L_LN2B)), yout, b.st2, T, H, c->cfg.ln_eps, r.st);
 }
 
+void layer_forward(Run& r, int l, const char* x, LayerBufs& b, char* yout) {
+  att_forward(r, l, x, b, b.h1);
+  ffn_forward(r, l, b, yout);
+}
+
 void alloc_internals(Run& r, LayerBufs& b, bool on_stack) {
   Arena& a = r.c->ar;
   auto al = [&](int64_t n) { return on_stack ? a.push(n) : a.talloc(n); };
@@ -408,6 +426,31 @@ void alloc_internals(Run& r, LayerBufs& b, bool on_stack) {
   b.z1 = (float*)al(r.z.z1); b.st1 = (float2*)al(r.z.st1); b.h1 = al(r.z.h1);
   b.u = al(r.z.u); b.g = al(r.z.g); b.z2 = (float*)al(r.z.z2); b.st2 = (float2*)al(r.z.st2);
 }
+// Sub-layer units (granularity 1, post-LN; DESIGN reading A30): the attention
+// block's internals [QKV, O, LSE, z1, st1] and the FFN block's [u, g, z2, st2],
+// in the layer's push order (h1 sits between them).
+void alloc_att(Run& r, LayerBufs& b, bool on_stack) {
+  Arena& a = r.c->ar;
+  auto al = [&](int64_t n) { return on_stack ? a.push(n) : a.talloc(n); };
+  b.qkv = al(r.z.qkv); b.O = al(r.z.O); b.lse = (float*)al(r.z.lse);
+  b.z1 = (float*)al(r.z.z1); b.st1 = (float2*)al(r.z.st1);
+}
+void free_att(Run& r, bool on_stack) {
+  Arena& a = r.c->ar;
+  const int64_t s[5] = {r.z.qkv, r.z.O, r.z.lse, r.z.z1, r.z.st1};
+  for (int i = 4; i >= 0; --i) on_stack ? a.pop(s[i]) : a.tfree(s[i]);
+}
+void alloc_ffn(Run& r, LayerBufs& b, bool on_stack) {
+  Arena& a = r.c->ar;
+  auto al = [&](int64_t n) { return on_stack ? a.push(n) : a.talloc(n); };
+  b.u = al(r.z.u); b.g = al(r.z.g); b.z2 = (float*)al(r.z.z2); b.st2 = (float2*)al(r.z.st2);
+}
+void free_ffn(Run& r, bool on_stack) {
+  Arena& a = r.c->ar;
+  const int64_t s[4] = {r.z.u, r.z.g, r.z.z2, r.z.st2};
+  for (int i = 3; i >= 0; --i) on_stack ? a.pop(s[i]) : a.tfree(s[i]);
+}
+
 void free_internals(Run& r, bool on_stack) {
   Arena& a = r.c->ar;
   const int64_t s0[10] = {r.z.qkv, r.z.O, r.z.lse, r.z.z1, r.z.st1, r.z.h1, r.z.u, r.z.g, r.z.z2, r.z.st2};
@@ -493,14 +536,15 @@ void dgrad(Run& r, Epi epi, const void* dY, int Nout, const void* Wt, int Kin, v
   pgemm(c, epi, g, r.st);
 }
 
-void layer_backward(Run& r, int l, const char* x, LayerBufs& b, float* dy, char* scr) {
+// FFN-block gradients of a post-LN layer: dy -> dz2 -> ... -> dres = dh1;
+// scratch carve: dres (dz / dh1), R2 (du, later dO), R3 (dt2 / dt1, later dQKV).
+void ffn_backward(Run& r, int l, LayerBufs& b, float* dy, char* scr) {
   mimose_ctx* c = r.c;
   if (!r.real) return;
-  const int T = c->T, H = c->cfg.hidden, F = c->cfg.ffn, h = c->cfg.heads;
+  const int T = c->T, H = c->cfg.hidden, F = c->cfg.ffn;
   float* dres = (float*)(scr + r.z.r_dres);
   char* R2 = scr + r.z.r_du;     // du, later dO
   char* R3 = scr + r.z.r_dt;     // dt2 / dt1, later dQKV
-  float* Dbuf = (float*)(scr + r.z.r_dt + a16((int64_t)T * 3 * H * c->e));
   float* pg = c->part;
   float* pb = c->part + (int64_t)NPART * H;
   float* pbias = c->part + 2LL * NPART * H;
@@ -517,6 +561,20 @@ void layer_backward(Run& r, int l, const char* x, LayerBufs& b, float* dy, char*
   wgrad(r, R2, F, b.h1, H, G(c, LP(c, l, L_F1W)));
   colsum(c->dt, R2, T, F, c->part, r.st);
   reduce_partials(c->part, F, F, G(c, LP(c, l, L_F1B)), r.st);
+}
+
+// Attention-block gradients of a post-LN layer (after ffn_backward; dres = dh1).
+void att_backward(Run& r, int l, const char* x, LayerBufs& b, float* dy, char* scr) {
+  mimose_ctx* c = r.c;
+  if (!r.real) return;
+  const int T = c->T, H = c->cfg.hidden, h = c->cfg.heads;
+  float* dres = (float*)(scr + r.z.r_dres);
+  char* R2 = scr + r.z.r_du;
+  char* R3 = scr + r.z.r_dt;
+  float* Dbuf = (float*)(scr + r.z.r_dt + a16((int64_t)T * 3 * H * c->e));
+  float* pg = c->part;
+  float* pb = c->part + (int64_t)NPART * H;
+  float* pbias = c->part + 2LL * NPART * H;
   // LN1 backward + dropout backward -> dz1 (dres, in place), dt1 (R3)
   ln_bwd(c->dt, dres, no_drop(), b.z1, b.st1, W(c, LP(c, l, L_LN1G)), dres, R3, make_drop(c, KIND_ATTN_OUT, l),
          pg, pb, pbias, T, H, r.st);
@@ -532,6 +590,11 @@ void layer_backward(Run& r, int l, const char* x, LayerBufs& b, float* dy, char*
   wgrad(r, R3, 3 * H, x, H, G(c, LP(c, l, L_QKVW)));
   colsum(c->dt, R3, T, 3 * H, c->part, r.st);
   reduce_partials(c->part, 3 * H, 3 * H, G(c, LP(c, l, L_QKVB)), r.st);
+}
+
+void layer_backward(Run& r, int l, const char* x, LayerBufs& b, float* dy, char* scr) {
+  ffn_backward(r, l, b, dy, scr);
+  att_backward(r, l, x, b, dy, scr);
 }
 
 // ---------------------------------------------------------------------------
@@ -773,7 +836,49 @@ void run_forward(Run& r, uint64_t mask, bool collect, Sample* sample) {
   c->lb.assign(L, LayerBufs());
   c->y.assign(L, nullptr);
   const char* x = c->x1;
-  for (int l = 0; l < L; ++l) {
+  for (int l = 0; l < L && c->cfg.granularity == 1; ++l) {   // sub-layer units 2l (attention), 2l+1 (FFN)
+    LayerBufs& b = c->lb[l];
+    const int ua = 2 * l, uf = 2 * l + 1;
+    int64_t b0 = a.live();
+    if (collect && sample) {                  // pass 1 (save mode), timed, discarded
+      LayerBufs tmp;
+      alloc_att(r, tmp, true);
+      char* ht = a.push(r.z.h1);
+      if (r.real) cudaEventRecord(c->ev_t0[ua], r.st);
+      att_forward(r, l, x, tmp, ht);
+      if (r.real) cudaEventRecord(c->ev_t1[ua], r.st);
+      sample->a[ua] = a.live() - b0;
+      a.pop(r.z.h1);
+      free_att(r, true);
+    }
+    const bool da = collect || ((mask >> ua) & 1);
+    alloc_att(r, b, !da);
+    b.h1 = a.push(r.z.h1);
+    att_forward(r, l, x, b, b.h1);
+    if (da) free_att(r, false);
+    if (sample) sample->y[ua] = a.live() - b0;
+    b0 = a.live();
+    if (collect && sample) {
+      LayerBufs tmp;
+      tmp.h1 = b.h1;
+      alloc_ffn(r, tmp, true);
+      char* yt = a.push(r.z.y);
+      if (r.real) cudaEventRecord(c->ev_t0[uf], r.st);
+      ffn_forward(r, l, tmp, yt);
+      if (r.real) cudaEventRecord(c->ev_t1[uf], r.st);
+      sample->a[uf] = a.live() - b0;
+      a.pop(r.z.y);
+      free_ffn(r, true);
+    }
+    const bool df = collect || ((mask >> uf) & 1);
+    alloc_ffn(r, b, !df);
+    c->y[l] = a.push(r.z.y);
+    ffn_forward(r, l, b, c->y[l]);
+    if (df) free_ffn(r, false);
+    if (sample) sample->y[uf] = a.live() - b0;
+    x = c->y[l];
+  }
+  for (int l = 0; l < L && c->cfg.granularity == 0; ++l) {
     const int64_t b0 = a.live();
     if (collect && sample) {
       // pass 1: normal forward (save mode), timed; output and activations discarded
@@ -867,7 +972,31 @@ mimose_status run_backward(Run& r, Sample* sample) {
   a.pop(r.z.y);                                       // y_L
   // ---- layers ----
   a.top_phase_peak = a.top;
-  for (int l = L - 1; l >= 0; --l) {
+  for (int l = L - 1; l >= 0 && c->cfg.granularity == 1; --l) {   // sub-layer units
+    LayerBufs& b = c->lb[l];
+    const char* x = l > 0 ? c->y[l - 1] : c->x1;
+    if ((c->drop_mask >> (2 * l + 1)) & 1) {          // recompute the FFN block from h1
+      alloc_ffn(r, b, true);
+      ffn_forward(r, l, b, nullptr);
+    }
+    char* scr = a.talloc(r.z.layer_scr);
+    ffn_backward(r, l, b, dy, scr);
+    free_ffn(r, true);
+    a.pop(r.z.h1);                                    // h1: dead after the FFN1 wgrad
+    if ((c->drop_mask >> (2 * l)) & 1) {              // recompute the attention block from y_{l-1}
+      alloc_att(r, b, true);
+      att_forward(r, l, x, b, nullptr);
+    }
+    att_backward(r, l, x, b, dy, scr);
+    a.tfree(r.z.layer_scr);
+    if (r.real) {
+      mimose_status s = allreduce_bucket(c, layer_base(c) + 12 * l, layer_base(c) + 12 * l + 11, l);
+      if (s) return s;
+    }
+    free_att(r, true);
+    if (l > 0) a.pop(r.z.y);                          // y_{l-1}: input of layer l
+  }
+  for (int l = L - 1; l >= 0 && c->cfg.granularity == 0; --l) {
     const bool dropped = (c->drop_mask >> l) & 1;
     const char* x = l > 0 ? c->y[l - 1] : c->x1;
     if (dropped) {                                    // recompute right before the gradients
@@ -968,7 +1097,7 @@ void resolve_times(mimose_ctx* c) {
   if (!c->pending_times || !c->device) return;
   cudaStreamSynchronize(c->st);
   Sample& s = c->samples.back();
-  for (int l = 0; l < c->cfg.n_layers; ++l) {
+  for (int l = 0; l < n_units(c); ++l) {
     float ms = 0.f;
     cudaEventElapsedTime(&ms, c->ev_t0[l], c->ev_t1[l]);
     s.t_ms[l] = ms;
@@ -1040,7 +1169,8 @@ mimose_status mimose_init(const mimose_config* cfgp, mimose_ctx** out) {
       k.max_seqs < 1 || k.max_seq_len < 1 || (int64_t)k.max_seqs * k.max_seq_len > 32768 || k.max_pos < 1 ||
       (k.head == MIMOSE_HEAD_MC && k.n_choices < 1) ||
       (k.head == MIMOSE_HEAD_SEQCLS && (k.n_labels < 1 || k.n_labels > 32)) || k.world < 1 || k.rank < 0 ||
-      k.rank >= k.world || k.bucket_den <= 0 || k.degree < 0 || k.degree > 2) {
+      k.rank >= k.world || k.bucket_den <= 0 || k.degree < 0 || k.degree > 2 || k.granularity < 0 ||
+      k.granularity > 1 || (k.granularity == 1 && (k.arch != MIMOSE_ARCH_POST_LN || 2 * k.n_layers > 64))) {
     mimose_status s = bad("invalid model / sizing config");
     *out = c;   // returned so mimose_last_error works; caller destroys
     return s;
@@ -1095,9 +1225,10 @@ mimose_status mimose_init(const mimose_config* cfgp, mimose_ctx** out) {
   if (c->device) {
     c->st = (cudaStream_t)k.stream;
     const int L = k.n_layers;
-    c->ev_t0.resize(L);
-    c->ev_t1.resize(L);
-    for (int l = 0; l < L; ++l) {
+    const int U = n_units(c);
+    c->ev_t0.resize(U);
+    c->ev_t1.resize(U);
+    for (int l = 0; l < U; ++l) {
       CK(cudaEventCreate(&c->ev_t0[l]));
       CK(cudaEventCreate(&c->ev_t1[l]));
     }
@@ -1226,8 +1357,8 @@ mimose_status mimose_collect(mimose_ctx* c, const mimose_batch* bt, float* loss_
   auto t0 = std::chrono::steady_clock::now();
   c->collecting = unseen;
   Sample smp;
-  const int L = c->cfg.n_layers;
-  smp.a.assign(L, 0); smp.y.assign(L, 0); smp.t_ms.assign(L, 0.f);
+  const int U = n_units(c);
+  smp.a.assign(U, 0); smp.y.assign(U, 0); smp.t_ms.assign(U, 0.f);
   mimose_status s = begin_step(c, bt, ~0ull, true, unseen ? &smp : nullptr);
   if (s) return s;
   if (unseen) {
@@ -1504,7 +1635,7 @@ mimose_status mimose_dry_collect(mimose_ctx* c, int32_t n_seqs, int32_t seq_len,
   if (!c || !out) return MIMOSE_E_INVALID;
   mimose_batch bt{nullptr, nullptr, nullptr, nullptr, n_seqs, seq_len, 1};
   if (mimose_status s = check_batch(c, &bt)) return s;
-  const int L = c->cfg.n_layers;
+  const int L = n_units(c);
   Sample smp;
   smp.a.assign(L, 0); smp.y.assign(L, 0); smp.t_ms.assign(L, 0.f);
   int64_t peak;

@@ -14,8 +14,10 @@ import pytest
 torch = pytest.importorskip("torch")
 pytestmark = pytest.mark.gpu
 
+from oracle import estimator as oe
 from oracle import memsim as om
 from oracle import model as omodel
+from oracle import planner as op
 from paper_conf_ipps_liaolysshfyctzlq23_b200 import workload as wl
 
 
@@ -231,3 +233,94 @@ def test_fused_optimizer_bitwise_equal(case):
         out.append(ctx.get_params())
         ctx.close()
     assert np.array_equal(out[0], out[1])
+
+
+# ---------------------------------------------------------------------------
+# sub-layer checkpoint units (granularity=1, DESIGN reading A30)
+# ---------------------------------------------------------------------------
+
+@pytest.mark.parametrize("case", ["toy-fp32", "mc-bf16", "qa-bf16-long"])
+def test_units_recompute_replay_bitwise(case):
+    """Unit plans (attention / FFN blocks dropped independently) replay the
+    forward bit for bit: loss and gradients equal the layer-granularity
+    no-checkpoint step exactly, for every unit plan."""
+    cfg = CASES[case]
+    params = wl.init_params(cfg, parity=True, seed=3)
+    L = cfg.n_layers
+    rng = np.random.default_rng(2)
+    plans = [[], [0], [1], list(range(2 * L)), [2 * L - 1], [2 * l + 1 for l in range(L)],
+             [2 * l for l in range(L)], sorted(rng.choice(2 * L, L, replace=False).tolist())]
+    b = wl.make_batch(cfg, cfg.seq_hi - 1, seed=7)
+    ctx = make_ctx(cfg)
+    ctx.set_params(wl.pack_params(cfg, params))
+    ref = run_step(ctx, cfg, b, [])
+    ctx.close()
+    for plan in plans:
+        ctx = make_ctx(cfg, granularity=1)
+        ctx.set_params(wl.pack_params(cfg, params))
+        loss, g = run_step(ctx, cfg, b, plan)
+        assert loss == ref[0], plan
+        assert np.array_equal(g, ref[1]), plan
+        st = ctx.stats()
+        assert st["peak_bytes"] == om.simulate_step_units(om.sizes(cfg, cfg.n_seqs, b.seq_len), plan).peak
+        ctx.close()
+
+
+def test_units_step_parity_against_oracle():
+    """A unit plan's loss and gradients against the fp64 oracle (the plain step:
+    checkpointing is exact) within the bf16 tolerance."""
+    cfg = CASES["mc-bf16"]
+    params = wl.init_params(cfg, parity=True, seed=11)
+    W = rounded_params(cfg, params)
+    ctx = make_ctx(cfg, granularity=1)
+    ctx.set_params(wl.pack_params(cfg, params))
+    b = wl.make_batch(cfg, cfg.seq_hi, seed=100)
+    loss, g = run_step(ctx, cfg, b, [0, 3, 4])
+    ref_loss, G = omodel.train_step_grads(cfg, W, b, wl.dropout_seed(cfg), ctx.stats()["steps"])
+    assert abs(loss - ref_loss) <= TOL2["bf16"] * max(1.0, abs(ref_loss))
+    gd = grads_dict(cfg, g)
+    floor2 = 1e-3 * max(float(np.linalg.norm(v)) for v in G.values())
+    for k in G:
+        assert rel2(gd[k], G[k], floor2) <= TOL2["bf16"], (k, rel2(gd[k], G[k], floor2))
+
+
+def test_units_collector_plans_and_budget_on_gpu():
+    """Sheltered phase at unit granularity on the GPU: samples == the unit event
+    model, plans == the oracle planner on the oracle's samples, arena peak ==
+    simulated peak <= M on every step, 0 violations."""
+    cfg = CASES["mc-bf16"]
+    sz = om.sizes(cfg, cfg.n_seqs, cfg.max_seq)
+    M = max(sz.C + int(0.6 * (om.no_ckpt_peak(sz) - sz.C)), om.lower_bound(sz))
+    ctx = make_ctx(cfg, budget=M, granularity=1)
+    ctx.set_params(wl.pack_params(cfg, wl.init_params(cfg)))
+    sched = wl.length_schedule(cfg, 50)
+    i, samples = 0, []
+    while ctx.phase == mb().PHASE_SHELTERED:
+        b = wl.make_batch(cfg, sched[i], seed=i)
+        ctx.collect(device_batch(ctx, b))
+        ctx.backward()
+        ctx.step(1e-4)
+        i += 1
+    for j in range(ctx.stats()["n_samples"]):
+        s = ctx.sample(j)
+        want = om.collect_samples_units(om.sizes(cfg, cfg.n_seqs, s["x"] // cfg.n_seqs))
+        for k in ("C", "E", "Hd", "Th", "Tb", "Te", "a", "y"):
+            assert s[k] == want[k]
+        assert all(t > 0 for t in s["t_ms"][:2 * cfg.n_layers])
+        want["x"] = s["x"]
+        samples.append(want)
+    est = oe.Estimator(samples)
+    for L_t in sched[i:]:
+        b = wl.make_batch(cfg, L_t, seed=1000 + i)
+        p = ctx.plan(b.input_size)
+        ost, odropped, _ = op.plan(est.predict(b.input_size), M)
+        assert p.dropped == list(odropped)
+        loss = ctx.forward(device_batch(ctx, b), p)
+        ctx.backward()
+        ctx.step(1e-4)
+        st = ctx.stats()
+        assert st["peak_bytes"] <= M
+        assert st["peak_bytes"] == om.simulate_step_units(om.sizes(cfg, cfg.n_seqs, b.seq_len), p.dropped).peak
+        assert np.isfinite(loss)
+        i += 1
+    assert ctx.stats()["violations"] == 0

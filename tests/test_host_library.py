@@ -223,3 +223,75 @@ def test_exact_planner_on_config_series(name):
         if st == mb.OK:
             assert pk <= M and pk == op.predicted_peak(p, dropped) and len(dropped) <= len(gdropped)
     assert worst < 0.5, worst
+
+
+# ---------------------------------------------------------------------------
+# sub-layer checkpoint units (granularity=1, DESIGN reading A30)
+# ---------------------------------------------------------------------------
+UNIT_CFGS = ["toy", "bert-base", "bert-large", "roberta-large"]
+
+
+@pytest.mark.parametrize("name", UNIT_CFGS)
+def test_units_dry_run_and_collector_match_event_model(name):
+    """Host-only ctx at granularity 1: the arena's dry-run peak of random unit
+    plans and the unit collector's samples equal oracle/memsim's unit model."""
+    cfg = wl.CONFIGS[name]
+    ctx = mb.Mimose(cfg, budget_for(cfg), granularity=1)
+    assert ctx.n_units == 2 * cfg.n_layers
+    rng = random.Random(15)
+    for S in sorted({cfg.pad, cfg.seq_lo, cfg.max_seq}):
+        sz = om.sizes(cfg, cfg.n_seqs, S)
+        for _ in range(6):
+            plan = rng.sample(range(2 * cfg.n_layers), rng.randint(0, 2 * cfg.n_layers))
+            assert ctx.dry_run(cfg.n_seqs, S, plan) == om.simulate_step_units(sz, plan).peak
+        got = ctx.dry_collect(cfg.n_seqs, S)
+        want = om.collect_samples_units(sz)
+        for k in ("C", "E", "Hd", "Th", "Tb", "Te", "a", "y"):
+            assert got[k] == want[k], (k, S)
+
+
+@pytest.mark.parametrize("name,planner", [(n, "greedy") for n in UNIT_CFGS] + [("toy", "exact")])
+def test_units_pipeline_matches_oracle(name, planner):
+    """Sheltered phase -> estimator -> Algorithm 1 (or the exact planner, whose
+    oracle is brute force: toy only) over the 2L units: every plan equals the
+    oracle's, and its simulated peak is within the budget."""
+    cfg = wl.CONFIGS[name]
+    M = budget_for(cfg)
+    ctx = mb.Mimose(cfg, M, granularity=1)
+    if planner == "exact":
+        ctx.set_planner(1)
+    sched = wl.length_schedule(cfg, 120)
+    samples, seen, i = [], set(), 0
+    while ctx.phase == mb.PHASE_SHELTERED:
+        b = wl.make_batch(cfg, sched[i], seed=i)
+        ctx.collect(ctx.host_batch(b))
+        ctx.backward()
+        if b.input_size not in seen:
+            seen.add(b.input_size)
+            s = om.collect_samples_units(om.sizes(cfg, cfg.n_seqs, b.seq_len))
+            s["x"] = b.input_size
+            samples.append(s)
+        i += 1
+    for j, s in enumerate(samples):
+        got = ctx.sample(j)
+        for k in ("x", "C", "E", "Hd", "Th", "Tb", "Te", "a", "y"):
+            assert got[k] == s[k]
+    est = oe.Estimator(samples)
+    fn = op.plan if planner == "greedy" else op.plan_exact
+    for L_t in sched[i:i + 40]:
+        S = wl.roundup(L_t, cfg.pad)
+        x = cfg.n_seqs * S
+        p = ctx.plan(x)
+        ost, odropped, opk = fn(est.predict(x), M)
+        assert p.status == mb.OK and ost == op.OK
+        assert p.dropped == list(odropped) and p.predicted_peak == opk
+        assert ctx.dry_run(cfg.n_seqs, S, p.dropped) == om.simulate_step_units(
+            om.sizes(cfg, cfg.n_seqs, S), p.dropped).peak <= M
+
+
+def test_units_config_validation():
+    """granularity 1 is post-LN only (GPT-2's pre-LN blocks are not split)."""
+    with pytest.raises(mb.MimoseError):
+        mb.Mimose(wl.CONFIGS["gpt2-medium"], 1 << 40, granularity=1)
+    with pytest.raises(mb.MimoseError):
+        mb.Mimose(wl.CONFIGS["toy"], 1 << 40, granularity=2)
