@@ -272,10 +272,22 @@ mimose_status mimose_debug_gemm_ex(int32_t epi, int32_t M, int32_t N, int32_t K,
                                    void* C2, const void* bias, const void* res, int64_t ldr, const void* aux,
                                    int64_t ldx, int32_t split, int32_t use_tc, void* stream);
 
+/* Test hook: two fp32-output bf16 GEMMs (as mimose_debug_gemm with epi 6, split 1)
+   in ONE grouped persistent tcgen05 launch, 128 x 256 tiles (the grouped wgrad of
+   the FFN block).  Returns MIMOSE_E_INVALID if the pair cannot be grouped (N % 256,
+   more tiles than SMs). */
+mimose_status mimose_debug_gemm_grouped(int32_t M1, int32_t N1, int32_t K1, const void* A1, int64_t a_sm1,
+                                        int64_t a_sk1, const void* B1, int64_t b_sn1, int64_t b_sk1, void* C1,
+                                        int32_t M2, int32_t N2, int32_t K2, const void* A2, int64_t a_sm2,
+                                        int64_t a_sk2, const void* B2, int64_t b_sn2, int64_t b_sk2, void* C2,
+                                        void* stream);
+
 /* Test hook: process-wide kernel options. gemm_mode 0 = one 128x128 tile per CTA,
-   1 = persistent double-buffered single-CTA tcgen05 GEMM, 2 = persistent CTA-pair
-   (cta_group::2, 256-row tiles; default); attn_tc 0/1 routes bf16
-   attention with S <= 128 to the SIMT / tcgen05 kernels.  Negative = unchanged. */
+   1 = persistent double-buffered single-CTA tcgen05 GEMM (default), 2 = persistent
+   CTA-pair (cta_group::2, 256-row tiles), 11 / 12 / 13 = persistent with tile
+   width 128 / 256 / 64, 14 = persistent deterministic stream-K; attn_tc 0/1
+   routes bf16 attention with S <= 128 to the SIMT / tcgen05 kernels.
+   Negative = unchanged. */
 void mimose_debug_options(int32_t gemm_mode, int32_t attn_tc);
 
 /* 1 if this build routes bf16 GEMMs to the tcgen05/TMEM/TMA kernels. */

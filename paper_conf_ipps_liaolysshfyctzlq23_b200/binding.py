@@ -149,6 +149,21 @@ def debug_gemm(epi, M, N, K, A, a_sm, a_sk, B, b_sn, b_sk, Cm, ldc, bias=None, s
         raise MimoseError(st, "debug_gemm")
 
 
+_lib.mimose_debug_gemm_grouped.argtypes = ([C.c_int32, C.c_int32, C.c_int32, _P, C.c_int64, C.c_int64, _P,
+                                             C.c_int64, C.c_int64, _P] * 2 + [_P])
+EXPORTED.append("mimose_debug_gemm_grouped")
+
+
+def debug_gemm_grouped(op1, C1, op2, C2, stream=0):
+    """Test hook: two fp32 GEMMs (M, N, K, A, a_sm, a_sk, B, b_sn, b_sk) in one grouped launch."""
+    args = []
+    for (M, N, K, A, a_sm, a_sk, B, b_sn, b_sk), Cm in ((op1, C1), (op2, C2)):
+        args += [M, N, K, A.data_ptr(), a_sm, a_sk, B.data_ptr(), b_sn, b_sk, Cm.data_ptr()]
+    st = _lib.mimose_debug_gemm_grouped(*args, stream)
+    if st != OK:
+        raise MimoseError(st, "debug_gemm_grouped")
+
+
 _lib.mimose_debug_gemm_ex.argtypes = [C.c_int32, C.c_int32, C.c_int32, C.c_int32, _P, C.c_int64, C.c_int64,
                                       _P, C.c_int64, C.c_int64, _P, C.c_int64, _P, _P, _P, C.c_int64, _P, C.c_int64,
                                       C.c_int32, C.c_int32, _P]

@@ -524,6 +524,53 @@ void wgrad(Run& r, const void* dY, int N, const void* X, int K, float* out) {
   }
 }
 
+// dW1 = dY1^T X1 and dW2 = dY2^T X2 (both deterministic, fp32 out): one grouped
+// tcgen05 launch with 128 x 256 tiles when the two fit one wave of SMs (the FFN
+// pair of BERT-base: 72 + 72 tiles), else two wgrad() calls.
+void wgrad2(Run& r, const void* dY1, int N1, const void* X1, int K1, float* out1, const void* dY2, int N2,
+            const void* X2, int K2, float* out2) {
+  mimose_ctx* c = r.c;
+  const int T = c->T;
+  if (c->dt == DT_BF16 && c->cfg.use_tc && K1 % 256 == 0 && K2 % 256 == 0) {
+    GemmArgs g[2];
+    const void* dY[2] = {dY1, dY2};
+    const void* X[2] = {X1, X2};
+    const int N[2] = {N1, N2}, K[2] = {K1, K2};
+    float* out[2] = {out1, out2};
+    for (int i = 0; i < 2; ++i) {
+      g[i].M = N[i]; g[i].N = K[i]; g[i].K = T;
+      g[i].A = dY[i]; g[i].a_sm = 1; g[i].a_sk = N[i];
+      g[i].B = X[i]; g[i].b_sn = 1; g[i].b_sk = K[i];
+      g[i].C = out[i]; g[i].ldc = K[i];
+    }
+    const bool on = c->probe == 1 && c->device;
+    if (on) {
+      if (c->probe_used + 2 > c->probe_ev.size()) {
+        for (int i = 0; i < 256; ++i) {
+          cudaEvent_t e;
+          cudaEventCreate(&e);
+          c->probe_ev.push_back(e);
+        }
+      }
+      cudaEventRecord(c->probe_ev[c->probe_used], r.st);
+    }
+    const bool done = gemm_tc_grouped(g[0], g[1], 256, r.st);
+    if (on) {
+      cudaEventRecord(c->probe_ev[c->probe_used + 1], r.st);
+      if (done) {
+        c->probe_used += 2;
+        c->probe_flops += 2.0 * T * ((double)N1 * K1 + (double)N2 * K2);
+      }
+    }
+    if (done) {
+      note_launch(1);
+      return;
+    }
+  }
+  wgrad(r, dY1, N1, X1, K1, out1);
+  wgrad(r, dY2, N2, X2, K2, out2);
+}
+
 void dgrad(Run& r, Epi epi, const void* dY, int Nout, const void* Wt, int Kin, void* out, const void* res_or_aux) {
   mimose_ctx* c = r.c;
   GemmArgs g;
@@ -553,12 +600,13 @@ void ffn_backward(Run& r, int l, LayerBufs& b, float* dy, char* scr) {
          pg, pb, pbias, T, H, r.st);
   reduce_rows3(pg, G(c, LP(c, l, L_LN2G)), pb, G(c, LP(c, l, L_LN2B)), pbias, G(c, LP(c, l, L_F2B)), NPART, H, H,
                r.st);
-  // FFN2: du = (dt2 W2) * gelu'(u); dW2 = dt2^T g
+  // FFN2: du = (dt2 W2) * gelu'(u)
   dgrad(r, EPI_GELU_BWD, R3, H, W(c, LP(c, l, L_F2W)), F, R2, b.u);
-  wgrad(r, R3, H, b.g, F, G(c, LP(c, l, L_F2W)));
-  // FFN1: dh1 = du W1 + dz2 (in place in dres); dW1 = du^T h1; db1 = colsum du
+  // FFN1: dh1 = du W1 + dz2 (in place in dres)
   dgrad(r, EPI_ACC_RES_F32, R2, F, W(c, LP(c, l, L_F1W)), H, dres, dres);
-  wgrad(r, R2, F, b.h1, H, G(c, LP(c, l, L_F1W)));
+  // dW2 = dt2^T g and dW1 = du^T h1 together (dt2 in R3 lives until LN1 backward)
+  wgrad2(r, R3, H, b.g, F, G(c, LP(c, l, L_F2W)), R2, F, b.h1, H, G(c, LP(c, l, L_F1W)));
+  // db1 = colsum du
   colsum(c->dt, R2, T, F, c->part, r.st);
   reduce_partials(c->part, F, F, G(c, LP(c, l, L_F1B)), r.st);
 }
@@ -1536,6 +1584,20 @@ mimose_status mimose_debug_gemm_ex(int32_t epi, int32_t M, int32_t N, int32_t K,
   g.drop.enabled = 1; g.drop.seed_lo = 7; g.drop.seed_hi = 0; g.drop.site = 0; g.drop.step = 1;
   g.drop.thresh = 3865470566u; g.drop.scale = (float)(1.0 / 0.9);
   gemm(DT_BF16, (Epi)epi, g, (cudaStream_t)stream, use_tc != 0);
+  return cudaGetLastError() == cudaSuccess ? MIMOSE_OK : MIMOSE_E_CUDA;
+}
+
+mimose_status mimose_debug_gemm_grouped(int32_t M1, int32_t N1, int32_t K1, const void* A1, int64_t a_sm1,
+                                        int64_t a_sk1, const void* B1, int64_t b_sn1, int64_t b_sk1, void* C1,
+                                        int32_t M2, int32_t N2, int32_t K2, const void* A2, int64_t a_sm2,
+                                        int64_t a_sk2, const void* B2, int64_t b_sn2, int64_t b_sk2, void* C2,
+                                        void* stream) {
+  GemmArgs g1, g2;
+  g1.M = M1; g1.N = N1; g1.K = K1; g1.A = A1; g1.a_sm = a_sm1; g1.a_sk = a_sk1;
+  g1.B = B1; g1.b_sn = b_sn1; g1.b_sk = b_sk1; g1.C = C1; g1.ldc = N1;
+  g2.M = M2; g2.N = N2; g2.K = K2; g2.A = A2; g2.a_sm = a_sm2; g2.a_sk = a_sk2;
+  g2.B = B2; g2.b_sn = b_sn2; g2.b_sk = b_sk2; g2.C = C2; g2.ldc = N2;
+  if (!gemm_tc_grouped(g1, g2, 256, (cudaStream_t)stream)) return MIMOSE_E_INVALID;
   return cudaGetLastError() == cudaSuccess ? MIMOSE_OK : MIMOSE_E_CUDA;
 }
 

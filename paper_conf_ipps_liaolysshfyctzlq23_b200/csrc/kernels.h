@@ -54,6 +54,10 @@ struct GemmArgs {
 };
 void gemm(DType dt, Epi epi, const GemmArgs& g, cudaStream_t st, bool use_tc);
 bool tc_available();
+// Two independent fp32-output (EPI_F32, split 1) bf16 GEMMs in one persistent
+// tcgen05 launch with tile width bn (128 or 256; N % bn == 0).  Returns false
+// (nothing launched) when the shapes / mode do not allow it.
+bool gemm_tc_grouped(const GemmArgs& g1, const GemmArgs& g2, int bn, cudaStream_t st);
 // 0: one tile per CTA; 1: persistent double-buffered (default).
 void set_gemm_mode(int m);
 // Deterministic split-K reduction: out[i] = sum_s part[s*n + i] (fixed order).

@@ -549,7 +549,7 @@ struct TpArgs {
 //   in that fixed order and runs the epilogue.  Producers compute their
 //   partial first and heads wait last, so the waits cannot deadlock with
 //   all CTAs resident (grid <= #SMs, one CTA per SM).
-struct Seg { int r, z, kb0, kb1; };
+struct Seg { int r, z, kb0, kb1, p = 0; };
 MDEV int64_t sk_u0(int cta, int64_t W) { return (int64_t)cta * W / gridDim.x; }
 template <bool SK>
 MDEV bool seg_of(const TpArgs& a, int i, Seg& s) {
@@ -574,6 +574,23 @@ MDEV bool seg_of(const TpArgs& a, int i, Seg& s) {
   s.kb1 = min(ta.kb_total, s.kb0 + ta.kb_per_split);
   return true;
 }
+// Grouped launch of two independent problems (same epilogue, no split): tiles
+// of problem 0 first, then problem 1, one round-robin order over both.
+template <bool SK, bool G2>
+MDEV bool seg_of2(const TpArgs& a, const TpArgs& a2, int i, Seg& s) {
+  if constexpr (!G2) {
+    return seg_of<SK>(a, i, s);
+  } else {
+    const int tile = blockIdx.x + i * gridDim.x;
+    if (tile >= a.n_tiles + a2.n_tiles) return false;
+    s.p = tile >= a.n_tiles;
+    s.r = s.p ? tile - a.n_tiles : tile;
+    s.z = 0;
+    s.kb0 = 0;
+    s.kb1 = (s.p ? a2 : a).t.kb_total;
+    return true;
+  }
+}
 MDEV uint32_t ld_acquire_u32(const uint32_t* p) {
   uint32_t v;
   asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
@@ -588,9 +605,11 @@ MDEV float4 ld_cg_f4(const float* p) {
   return v;
 }
 
-template <int BN, int EPI, bool SK>
+template <int BN, int EPI, bool SK, bool G2>
 __global__ void __launch_bounds__(TP_THREADS, 1)
-    k_gemm_tcp(const __grid_constant__ CUtensorMap tma_a, const __grid_constant__ CUtensorMap tma_b, const TpArgs args) {
+    k_gemm_tcp(const __grid_constant__ CUtensorMap tma_a, const __grid_constant__ CUtensorMap tma_b, const TpArgs args,
+               const __grid_constant__ CUtensorMap tma_a2, const __grid_constant__ CUtensorMap tma_b2,
+               const TpArgs args2) {
   pdl_trigger();
   using Cf = TpCfg<BN>;
   extern __shared__ uint8_t smem_raw[];
@@ -610,6 +629,10 @@ __global__ void __launch_bounds__(TP_THREADS, 1)
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
     asm volatile("prefetch.tensormap [%0];" ::"l"(&tma_a) : "memory");
     asm volatile("prefetch.tensormap [%0];" ::"l"(&tma_b) : "memory");
+    if (G2) {
+      asm volatile("prefetch.tensormap [%0];" ::"l"(&tma_a2) : "memory");
+      asm volatile("prefetch.tensormap [%0];" ::"l"(&tma_b2) : "memory");
+    }
   }
   if (warp == 1) {
     asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(smem_u32(tmem_slot)),
@@ -627,9 +650,13 @@ __global__ void __launch_bounds__(TP_THREADS, 1)
     if (lane == 0) {                                   // ---------------- TMA producer
       int it = 0;
       Seg sg;
-      for (int si = 0; seg_of<SK>(args, si, sg); ++si) {
+      for (int si = 0; seg_of2<SK, G2>(args, args2, si, sg); ++si) {
+        const TpArgs& A = (G2 && sg.p) ? args2 : args;
+        const TcArgs& ta = A.t;
+        const CUtensorMap* map_a = (G2 && sg.p) ? &tma_a2 : &tma_a;
+        const CUtensorMap* map_b = (G2 && sg.p) ? &tma_b2 : &tma_b;
         const int r = sg.r;
-        const int m0 = (r / args.n_blocks) * TBM, n0 = (r % args.n_blocks) * BN;
+        const int m0 = (r / A.n_blocks) * TBM, n0 = (r % A.n_blocks) * BN;
         const int kb0 = sg.kb0, kb1 = sg.kb1;
         for (int kb = kb0; kb < kb1; ++kb, ++it) {
           const int s = it % Cf::STAGES;
@@ -639,28 +666,29 @@ __global__ void __launch_bounds__(TP_THREADS, 1)
           const int k = kb * TBK;
           mbar_expect_tx(&full[s], Cf::STAGE_BYTES);
           if (ta.a_mn) {
-            tma_load_2d(&tma_a, &full[s], sa, m0, k);
-            tma_load_2d(&tma_a, &full[s], sa + 8192, m0 + 64, k);
+            tma_load_2d(map_a, &full[s], sa, m0, k);
+            tma_load_2d(map_a, &full[s], sa + 8192, m0 + 64, k);
           } else {
-            tma_load_2d(&tma_a, &full[s], sa, k, m0);
+            tma_load_2d(map_a, &full[s], sa, k, m0);
           }
           if (ta.b_mn) {
 #pragma unroll
-            for (int j = 0; j < BN / 64; ++j) tma_load_2d(&tma_b, &full[s], sb + 8192 * j, n0 + 64 * j, k);
+            for (int j = 0; j < BN / 64; ++j) tma_load_2d(map_b, &full[s], sb + 8192 * j, n0 + 64 * j, k);
           } else {
 #pragma unroll
             for (int j = 0; j < (BN + 255) / 256; ++j)      // box rows <= 256
-              tma_load_2d(&tma_b, &full[s], sb + j * 256 * 128, k, n0 + 256 * j);
+              tma_load_2d(map_b, &full[s], sb + j * 256 * 128, k, n0 + 256 * j);
           }
         }
       }
     }
   } else if (warp == 1) {
     if (lane == 0) {                                   // ---------------- MMA issuer
-      const uint32_t idesc = idesc_bf16(TBM, BN, ta.a_mn, ta.b_mn);
       int it = 0, local = 0;
       Seg sg;
-      for (; seg_of<SK>(args, local, sg); ++local) {
+      for (; seg_of2<SK, G2>(args, args2, local, sg); ++local) {
+        const TcArgs& ta = ((G2 && sg.p) ? args2 : args).t;
+        const uint32_t idesc = idesc_bf16(TBM, BN, ta.a_mn, ta.b_mn);
         const int kb0 = sg.kb0, kb1 = sg.kb1;
         const int acc = local & 1;
         if (local >= 2) mbar_wait(&tempty[acc], ((local >> 1) - 1) & 1);
@@ -687,12 +715,13 @@ __global__ void __launch_bounds__(TP_THREADS, 1)
     const int e = warp - 2;
     const int q = warp & 3;                            // TMEM lane quarter of this warp
     const int grp = e >> 2, ngrp = TP_EPI_WARPS / 4;  // column group of this warp
-    const GemmArgs& g = ta.g;
     int local = 0;
     Seg sg;
-    for (; seg_of<SK>(args, local, sg); ++local) {
+    for (; seg_of2<SK, G2>(args, args2, local, sg); ++local) {
+      const TpArgs& A = (G2 && sg.p) ? args2 : args;
+      const GemmArgs& g = A.t.g;
       const int z = sg.z, r = sg.r;
-      const int m0 = (r / args.n_blocks) * TBM, n0 = (r % args.n_blocks) * BN;
+      const int m0 = (r / A.n_blocks) * TBM, n0 = (r % A.n_blocks) * BN;
       const int kb0 = sg.kb0, kb1 = sg.kb1;
       const int acc = local & 1;
       const int m = m0 + 32 * q + lane;
@@ -1090,6 +1119,8 @@ bool tc_map_bf16(CUtensorMap* out, const void* ptr, uint64_t inner, uint64_t out
   return make_map(out, ptr, inner, outer, stride_elems, box_inner, box_outer);
 }
 
+static int num_sms();
+
 template <int BN, int EPI>
 static void launch_tc(const CUtensorMap& ma, const CUtensorMap& mb, const TcArgs& a, dim3 grid, cudaStream_t st) {
   static bool attr = false;
@@ -1104,8 +1135,8 @@ template <int BN, int EPI>
 static void launch_tcp(const CUtensorMap& ma, const CUtensorMap& mb, const TpArgs& a, cudaStream_t st) {
   static bool attr = false;
   if (!attr) {
-    cudaFuncSetAttribute(k_gemm_tcp<BN, EPI, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, TpCfg<BN>::SMEM);
-    cudaFuncSetAttribute(k_gemm_tcp<BN, EPI, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, TpCfg<BN>::SMEM);
+    cudaFuncSetAttribute(k_gemm_tcp<BN, EPI, false, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, TpCfg<BN>::SMEM);
+    cudaFuncSetAttribute(k_gemm_tcp<BN, EPI, true, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, TpCfg<BN>::SMEM);
     attr = true;
   }
   static int nsm = 0;
@@ -1116,9 +1147,25 @@ static void launch_tcp(const CUtensorMap& ma, const CUtensorMap& mb, const TpArg
   }
   const int64_t units = a.sk ? (int64_t)a.n_tiles * a.t.kb_total : a.n_tiles;
   if (a.sk)
-    launch_k(k_gemm_tcp<BN, EPI, true>, (int)std::min<int64_t>(nsm, units), TP_THREADS, TpCfg<BN>::SMEM, st, ma, mb, a);
+    launch_k(k_gemm_tcp<BN, EPI, true, false>, (int)std::min<int64_t>(nsm, units), TP_THREADS, TpCfg<BN>::SMEM, st,
+             ma, mb, a, ma, mb, a);
   else
-    launch_k(k_gemm_tcp<BN, EPI, false>, (int)std::min<int64_t>(nsm, units), TP_THREADS, TpCfg<BN>::SMEM, st, ma, mb, a);
+    launch_k(k_gemm_tcp<BN, EPI, false, false>, (int)std::min<int64_t>(nsm, units), TP_THREADS, TpCfg<BN>::SMEM, st,
+             ma, mb, a, ma, mb, a);
+}
+
+// Two independent EPI_F32 problems in one persistent launch (grouped wgrad).
+template <int BN>
+static void launch_tcp_g2(const CUtensorMap& ma, const CUtensorMap& mb, const TpArgs& a, const CUtensorMap& ma2,
+                          const CUtensorMap& mb2, const TpArgs& a2, cudaStream_t st) {
+  static bool attr = false;
+  if (!attr) {
+    cudaFuncSetAttribute(k_gemm_tcp<BN, EPI_F32, false, true>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                         TpCfg<BN>::SMEM);
+    attr = true;
+  }
+  launch_k(k_gemm_tcp<BN, EPI_F32, false, true>, std::min(num_sms(), a.n_tiles + a2.n_tiles), TP_THREADS,
+           TpCfg<BN>::SMEM, st, ma, mb, a, ma2, mb2, a2);
 }
 
 template <int BN>
@@ -1363,6 +1410,45 @@ bool gemm_tc(Epi epi, const GemmArgs& g, cudaStream_t st) {
     case EPI_ACC_F32: launch_tc<BN1, EPI_ACC_F32>(ma, mb, a, grid, st); break;
     default: launch_tc<BN1, EPI_F32>(ma, mb, a, grid, st); break;
   }
+  return true;
+}
+
+// Grouped EPI_F32 GEMM: two independent problems (split 1, both operand majors
+// as in gemm_tc) in one persistent launch -- tiles of g1 then g2 -- so two
+// weight gradients with few output tiles each fill the SMs together (only when
+// all tiles fit one wave; otherwise false and the caller launches them apart).  Each
+// tile's K loop is the same as in a single launch, so results are bitwise
+// equal to two separate launches with the same tile width.
+bool gemm_tc_grouped(const GemmArgs& g1, const GemmArgs& g2, int bn, cudaStream_t st) {
+  if (g_gemm_mode != 1 || g1.split != 1 || g2.split != 1 || g1.fused_split || g2.fused_split) return false;
+  if (bn != 128 && bn != 256) return false;
+  TpArgs p[2];
+  CUtensorMap ma[2], mb[2];
+  const GemmArgs* gs[2] = {&g1, &g2};
+  for (int i = 0; i < 2; ++i) {
+    const GemmArgs& g = *gs[i];
+    TcArgs a;
+    a.g = g;
+    if (g.a_sk == 1 && g.a_sm % 8 == 0) a.a_mn = 0;
+    else if (g.a_sm == 1 && g.a_sk % 8 == 0) a.a_mn = 1;
+    else return false;
+    if (g.b_sk == 1 && g.b_sn % 8 == 0) a.b_mn = 0;
+    else if (g.b_sn == 1 && g.b_sk % 8 == 0) a.b_mn = 1;
+    else return false;
+    if ((((uintptr_t)g.A | (uintptr_t)g.B) & 15) || g.ldc % 8 || g.N % bn) return false;
+    a.kb_total = (g.K + TBK - 1) / TBK;
+    a.kb_per_split = a.kb_total;
+    bool ok = a.a_mn ? make_map(&ma[i], g.A, g.M, g.K, g.a_sk, 64, 64) : make_map(&ma[i], g.A, g.K, g.M, g.a_sm, 64, TBM);
+    if (ok) ok = a.b_mn ? make_map(&mb[i], g.B, g.N, g.K, g.b_sk, 64, 64) : make_map(&mb[i], g.B, g.K, g.N, g.b_sn, 64, bn);
+    if (!ok) return false;
+    p[i].t = a;
+    p[i].m_blocks = (g.M + TBM - 1) / TBM;
+    p[i].n_blocks = g.N / bn;
+    p[i].n_tiles = p[i].m_blocks * p[i].n_blocks;
+  }
+  if (p[0].n_tiles + p[1].n_tiles > num_sms()) return false;   // grouping pays only within one wave
+  if (bn == 256) launch_tcp_g2<256>(ma[0], mb[0], p[0], ma[1], mb[1], p[1], st);
+  else launch_tcp_g2<128>(ma[0], mb[0], p[0], ma[1], mb[1], p[1], st);
   return true;
 }
 

@@ -181,3 +181,30 @@ def test_gemm_stream_k(shape, epi):
     if epi == 2:
         assert ((a2 - ref2).abs().max() / ref2.abs().max()).item() < 2e-2
         assert torch.equal(a2, b2)
+
+
+@pytest.mark.parametrize("pair", [((768, 3072, 5120), (3072, 768, 5120)), ((768, 3072, 1000), (3072, 768, 1000)),
+                                  ((296, 512, 136), (1000, 256, 136))])
+def test_gemm_grouped_wgrad(pair):
+    """Two wgrad-shaped (TN) fp32 GEMMs in one grouped launch are bitwise equal
+    to the same problems launched alone with the same 128 x 256 tiles."""
+    outs, refs = [], []
+    ops = []
+    for i, (M, N, K) in enumerate(pair):
+        A, B, As, Bs, a_sm, a_sk, b_sn, b_sk = operands(M, N, K, 1, 1, seed=20 + i)
+        ops.append((M, N, K, As, a_sm, a_sk, Bs, b_sn, b_sk))
+        refs.append(A.float() @ B.float().t())
+    C = [torch.full((o[0], o[1]), float("nan"), device="cuda") for o in ops]
+    mb().debug_gemm_grouped(ops[0], C[0], ops[1], C[1])
+    torch.cuda.synchronize()
+    mb().debug_options(gemm_mode=12)          # separate persistent launches, 256-wide tiles
+    try:
+        for o, ref, c in zip(ops, refs, C):
+            M, N, K, As, a_sm, a_sk, Bs, b_sn, b_sk = o
+            alone = torch.full((M, N), float("nan"), device="cuda")
+            mb().debug_gemm(6, M, N, K, As, a_sm, a_sk, Bs, b_sn, b_sk, alone, N)
+            torch.cuda.synchronize()
+            assert torch.equal(c, alone)
+            assert ((c - ref).abs().max() / ref.abs().max()).item() < 1e-5
+    finally:
+        mb().debug_options(gemm_mode=1)
