@@ -525,13 +525,14 @@ void wgrad(Run& r, const void* dY, int N, const void* X, int K, float* out) {
 }
 
 // dW1 = dY1^T X1 and dW2 = dY2^T X2 (both deterministic, fp32 out): one grouped
-// tcgen05 launch with 128 x 256 tiles when the two fit one wave of SMs (the FFN
-// pair of BERT-base: 72 + 72 tiles), else two wgrad() calls.
+// tcgen05 launch with 128 x bn tiles when the two fit one wave of SMs (BERT-base:
+// the FFN pair 72 + 72 tiles at bn 256, the attention pair 36 + 108 at bn 128),
+// else two wgrad() calls.
 void wgrad2(Run& r, const void* dY1, int N1, const void* X1, int K1, float* out1, const void* dY2, int N2,
-            const void* X2, int K2, float* out2) {
+            const void* X2, int K2, float* out2, int bn = 256) {
   mimose_ctx* c = r.c;
   const int T = c->T;
-  if (c->dt == DT_BF16 && c->cfg.use_tc && K1 % 256 == 0 && K2 % 256 == 0) {
+  if (c->dt == DT_BF16 && c->cfg.use_tc && K1 % bn == 0 && K2 % bn == 0) {
     GemmArgs g[2];
     const void* dY[2] = {dY1, dY2};
     const void* X[2] = {X1, X2};
@@ -554,7 +555,7 @@ void wgrad2(Run& r, const void* dY1, int N1, const void* X1, int K1, float* out1
       }
       cudaEventRecord(c->probe_ev[c->probe_used], r.st);
     }
-    const bool done = gemm_tc_grouped(g[0], g[1], 256, r.st);
+    const bool done = gemm_tc_grouped(g[0], g[1], bn, r.st);
     if (on) {
       cudaEventRecord(c->probe_ev[c->probe_used + 1], r.st);
       if (done) {
@@ -623,19 +624,27 @@ void att_backward(Run& r, int l, const char* x, LayerBufs& b, float* dy, char* s
   float* pg = c->part;
   float* pb = c->part + (int64_t)NPART * H;
   float* pbias = c->part + 2LL * NPART * H;
-  // LN1 backward + dropout backward -> dz1 (dres, in place), dt1 (R3)
-  ln_bwd(c->dt, dres, no_drop(), b.z1, b.st1, W(c, LP(c, l, L_LN1G)), dres, R3, make_drop(c, KIND_ATTN_OUT, l),
+  // dt1 goes to the spare tail of R2 (R2 holds T x F, dO uses its first T x H) so
+  // that it outlives the attention backward and dWo can be grouped with dWqkv
+  const bool spare = c->cfg.ffn >= 2 * H;
+  char* DT1 = spare ? R2 + a16((int64_t)T * H * c->e) : R3;
+  // LN1 backward + dropout backward -> dz1 (dres, in place), dt1 (DT1)
+  ln_bwd(c->dt, dres, no_drop(), b.z1, b.st1, W(c, LP(c, l, L_LN1G)), dres, DT1, make_drop(c, KIND_ATTN_OUT, l),
          pg, pb, pbias, T, H, r.st);
   reduce_rows3(pg, G(c, LP(c, l, L_LN1G)), pb, G(c, LP(c, l, L_LN1B)), pbias, G(c, LP(c, l, L_OB)), NPART, H, H,
                r.st);
-  // out-proj: dO = dt1 Wo (R2); dWo = dt1^T O
-  dgrad(r, EPI_STORE, R3, H, W(c, LP(c, l, L_OW)), H, R2, nullptr);
-  wgrad(r, R3, H, b.O, H, G(c, LP(c, l, L_OW)));
+  // out-proj: dO = dt1 Wo (R2)
+  dgrad(r, EPI_STORE, DT1, H, W(c, LP(c, l, L_OW)), H, R2, nullptr);
+  if (!spare) wgrad(r, DT1, H, b.O, H, G(c, LP(c, l, L_OW)));     // dWo = dt1^T O before R3 is reused
   // attention backward -> dQKV (R3)
   attn_bwd(c->dt, b.qkv, b.O, R2, b.lse, c->lens, Dbuf, R3, c->B, c->S, H, h, make_drop(c, KIND_ATTN_PROBS, l), r.st);
-  // QKV: dx = dQKV Wqkv + dz1 -> dy buffer; dWqkv = dQKV^T x; dbqkv = colsum dQKV
+  // QKV: dx = dQKV Wqkv + dz1 -> dy buffer
   dgrad(r, EPI_ACC_RES_F32, R3, 3 * H, W(c, LP(c, l, L_QKVW)), H, dy, dres);
-  wgrad(r, R3, 3 * H, x, H, G(c, LP(c, l, L_QKVW)));
+  // dWo = dt1^T O and dWqkv = dQKV^T x; dbqkv = colsum dQKV
+  if (spare)
+    wgrad2(r, DT1, H, b.O, H, G(c, LP(c, l, L_OW)), R3, 3 * H, x, H, G(c, LP(c, l, L_QKVW)), 128);
+  else
+    wgrad(r, R3, 3 * H, x, H, G(c, LP(c, l, L_QKVW)));
   colsum(c->dt, R3, T, 3 * H, c->part, r.st);
   reduce_partials(c->part, 3 * H, 3 * H, G(c, LP(c, l, L_QKVB)), r.st);
 }
