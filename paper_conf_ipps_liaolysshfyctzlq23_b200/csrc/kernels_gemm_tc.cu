@@ -244,6 +244,27 @@ struct EpiIn {
   uint4 b[4];   // bias (bf16 x 32)
   uint4 x[8];   // aux or residual: bf16 x 32 uses x[0..3], fp32 x 32 uses x[0..7]
 };
+
+// Dropout keep bits of the 32 consecutive elements e0..e0+31 (e0 % 4 == 0): bit i
+// = word(e0 + i) < thresh, the same Philox words and rule as drop_factor4.  The
+// persistent GEMM computes them before its accumulator is ready, so the Philox
+// work of a tile overlaps that tile's MMAs instead of extending its epilogue.
+MDEV uint32_t drop_bits32(const Drop& d, uint64_t e0) {
+  if (!d.enabled) return 0xFFFFFFFFu;
+  uint32_t bits = 0;
+#pragma unroll
+  for (int q = 0; q < 8; ++q) {
+    const uint4 w = drop_words(d, (e0 >> 2) + q);
+    bits |= ((uint32_t)(w.x < d.thresh) | ((uint32_t)(w.y < d.thresh) << 1) | ((uint32_t)(w.z < d.thresh) << 2) |
+             ((uint32_t)(w.w < d.thresh) << 3)) << (4 * q);
+  }
+  return bits;
+}
+MDEV float4 drop_from_bits(const Drop& d, uint32_t bits, int q) {
+  const float s = d.enabled ? d.scale : 1.0f;
+  return make_float4((bits >> (4 * q)) & 1 ? s : 0.f, (bits >> (4 * q + 1)) & 1 ? s : 0.f,
+                     (bits >> (4 * q + 2)) & 1 ? s : 0.f, (bits >> (4 * q + 3)) & 1 ? s : 0.f);
+}
 template <int EPI>
 MDEV void epi_load(const GemmArgs& g, int m, int n, bool live, EpiIn& in) {
   if constexpr (EPI == EPI_BIAS || EPI == EPI_BIAS_GELU || EPI == EPI_BIAS_DROP_RES || EPI == EPI_BIAS_GELUT ||
@@ -274,7 +295,7 @@ MDEV void epi_load(const GemmArgs& g, int m, int n, bool live, EpiIn& in) {
 
 template <int EPI>
 MDEV void epi_frag32_in(const GemmArgs& g, int m_base, int n, float (&v)[32], int z, uint8_t* stg, int lane,
-                        const EpiIn& in) {
+                        const EpiIn& in, uint32_t keep) {
   using E = __nv_bfloat16;
   const int m = m_base + lane;
   const int rows_valid = g.M - m_base;
@@ -307,10 +328,9 @@ MDEV void epi_frag32_in(const GemmArgs& g, int m_base, int n, float (&v)[32], in
       float r[32];
 #pragma unroll
       for (int i = 0; i < 4; ++i) unpack8(in.x[i], r + 8 * i);
-      const int64_t o = (int64_t)m * g.ldc + n;
 #pragma unroll
       for (int q = 0; q < 8; ++q) {
-        const float4 f = live ? drop_factor4(g.drop, (uint64_t)(o + 4 * q) >> 2) : make_float4(0.f, 0.f, 0.f, 0.f);
+        const float4 f = live ? drop_from_bits(g.drop, keep, q) : make_float4(0.f, 0.f, 0.f, 0.f);
         v[4 * q + 0] = (live ? r[4 * q + 0] : 0.f) + v[4 * q + 0] * f.x;
         v[4 * q + 1] = (live ? r[4 * q + 1] : 0.f) + v[4 * q + 1] * f.y;
         v[4 * q + 2] = (live ? r[4 * q + 2] : 0.f) + v[4 * q + 2] * f.z;
@@ -352,10 +372,9 @@ MDEV void epi_frag32_in(const GemmArgs& g, int m_base, int n, float (&v)[32], in
       stage_store_bf16(stg, v, (E*)g.C2 + (int64_t)m_base * g.ldc + n, g.ldc, rows_valid, lane);
     } else {
       const float* r = (const float*)in.x;
-      const int64_t o = (int64_t)m * g.ldc + n;
 #pragma unroll
       for (int q = 0; q < 8; ++q) {
-        const float4 f = live ? drop_factor4(g.drop, (uint64_t)(o + 4 * q) >> 2) : make_float4(0.f, 0.f, 0.f, 0.f);
+        const float4 f = live ? drop_from_bits(g.drop, keep, q) : make_float4(0.f, 0.f, 0.f, 0.f);
         v[4 * q + 0] = (live ? r[4 * q + 0] : 0.f) + v[4 * q + 0] * f.x;
         v[4 * q + 1] = (live ? r[4 * q + 1] : 0.f) + v[4 * q + 1] * f.y;
         v[4 * q + 2] = (live ? r[4 * q + 2] : 0.f) + v[4 * q + 2] * f.z;
@@ -762,14 +781,29 @@ __global__ void __launch_bounds__(TP_THREADS, 1)
           __syncwarp();
         }
       }
+      // dropout keep bits of this warp's chunks, computed while the MMAs run
+      constexpr int NCH = BN / 32 / (TP_EPI_WARPS / 4);
+      uint32_t kbits[NCH];
+      constexpr bool DROP_EPI = EPI == EPI_BIAS_DROP_RES || EPI == EPI_BIAS_DROP_RESF32;
+#pragma unroll
+      for (int i = 0; i < NCH; ++i) {
+        kbits[i] = 0u;
+        if constexpr (DROP_EPI) {
+          const int n = n0 + 32 * (c_beg + i);
+          if (m < g.M && n + 32 <= g.N && !(SK && sk_part)) kbits[i] = drop_bits32(g.drop, (uint64_t)m * g.ldc + n);
+        }
+      }
+      EpiIn nxt;   // the first chunk's epilogue inputs are in flight while the MMAs finish
+      if (n0 + 32 * c_beg + 32 <= g.N) epi_load<EPI>(g, m, n0 + 32 * c_beg, m < g.M, nxt);
       mbar_wait(&tfull[acc], (local >> 1) & 1);
       __syncwarp();
       tc_fence_after();
-      EpiIn nxt;
-      if (n0 + 32 * c_beg + 32 <= g.N) epi_load<EPI>(g, m, n0 + 32 * c_beg, m < g.M, nxt);
 #pragma unroll 1
       for (int c = c_beg; c < c_end; ++c) {
         const EpiIn cur = nxt;
+        const uint32_t keep = kbits[0];
+#pragma unroll
+        for (int i = 0; i + 1 < NCH; ++i) kbits[i] = kbits[i + 1];   // register rotation, no local memory
         const int n = n0 + 32 * c;
         if (c + 1 < c_end && n + 64 <= g.N) epi_load<EPI>(g, m, n + 32, m < g.M, nxt);
         float v[32];
@@ -816,7 +850,7 @@ __global__ void __launch_bounds__(TP_THREADS, 1)
             stage_store_f32(stg_base + e * 4096, v, dst + (int64_t)mb * g.ldc + n, g.ldc, g.M - mb, lane);
           }
         } else if (n + 32 <= g.N) {
-          if (m0 + 32 * q < g.M) epi_frag32_in<EPI>(g, m0 + 32 * q, n, v, z, stg_base + e * 4096, lane, cur);
+          if (m0 + 32 * q < g.M) epi_frag32_in<EPI>(g, m0 + 32 * q, n, v, z, stg_base + e * 4096, lane, cur, keep);
         } else if (m < g.M) {
 #pragma unroll
           for (int i = 0; i < 32; ++i)
