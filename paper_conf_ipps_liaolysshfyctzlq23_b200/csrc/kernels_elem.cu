@@ -110,11 +110,12 @@ void ln_fwd(DType dt, const float* z, const void* g, const void* b, void* y, flo
 // NPART CTAs x 4 warps; warp w of CTA p owns rows r = p*4 + w + k*NPART*4 (fixed).
 // Per-lane register partials of dgamma, dbeta, dbias over the warp's rows, then a
 // fixed-order reduction over the 4 warps through shared memory.  KCH = 8-column
-// chunks per lane (ceil(H / 256)); gamma is read from shared memory.  ~140
-// registers x 128 threads: 3 CTAs / SM, so all NPART CTAs are resident at once.
+// chunks per lane (ceil(H / 256)); gamma is read from shared memory.  For
+// H <= 768 the next row's loads are issued before the current row is processed.
+// <= 255 registers x 128 threads: 2 CTAs / SM, so all NPART CTAs are resident at once.
 constexpr int LNB_WARPS = 4;
 template <typename E, int KCH>
-__global__ void __launch_bounds__(32 * LNB_WARPS, 3) k_ln_bwd(const float* dy, Drop premask,
+__global__ void __launch_bounds__(32 * LNB_WARPS, 2) k_ln_bwd(const float* dy, Drop premask,
                                                               const float* __restrict__ z,
                                                               const float2* __restrict__ st, const E* __restrict__ g,
                                                               float* dz, E* __restrict__ dtout, Drop mask,
@@ -134,18 +135,34 @@ __global__ void __launch_bounds__(32 * LNB_WARPS, 3) k_ln_bwd(const float* dy, D
   for (int k = 0; k < KCH; ++k)
 #pragma unroll
     for (int i = 0; i < 8; ++i) { ag[k][i] = 0.f; ab[k][i] = 0.f; at[k][i] = 0.f; }
-  for (int row = blockIdx.x * LNB_WARPS + warp; row < T; row += NPART * LNB_WARPS) {
-    const float2 ms = st[row];
-    float dyv[KCH][8], xh[KCH][8];
-    float s1 = 0.f, s2 = 0.f;
+  // software pipeline: the next row's dy, z and statistics are loaded before the
+  // current row is processed (two rows of loads in flight per warp)
+  constexpr int STRIDE = NPART * LNB_WARPS;
+  float dyn[KCH][8], xn[KCH][8];
+  float2 msn = make_float2(0.f, 0.f);
+  auto load_row = [&](int rr) {
+    msn = st[rr];
 #pragma unroll
     for (int k = 0; k < KCH; ++k) {
       const int j = lane + 32 * k;
       if (j < nch) {
-        ld8(dy + (int64_t)row * H + 8 * j, dyv[k]);
-        ld8(z + (int64_t)row * H + 8 * j, xh[k]);
+        ld8(dy + (int64_t)rr * H + 8 * j, dyn[k]);
+        ld8(z + (int64_t)rr * H + 8 * j, xn[k]);
       }
     }
+  };
+  constexpr bool PF = KCH <= 3;        // H <= 768: registers allow the prefetch without spills
+  if (PF && blockIdx.x * LNB_WARPS + warp < T) load_row(blockIdx.x * LNB_WARPS + warp);
+  for (int row = blockIdx.x * LNB_WARPS + warp; row < T; row += STRIDE) {
+    if (!PF) load_row(row);
+    const float2 ms = msn;
+    float dyv[KCH][8], xh[KCH][8];
+#pragma unroll
+    for (int k = 0; k < KCH; ++k)
+#pragma unroll
+      for (int i = 0; i < 8; ++i) { dyv[k][i] = dyn[k][i]; xh[k][i] = xn[k][i]; }
+    if (PF && row + STRIDE < T) load_row(row + STRIDE);
+    float s1 = 0.f, s2 = 0.f;
 #pragma unroll
     for (int k = 0; k < KCH; ++k) {
       const int j = lane + 32 * k;
