@@ -282,7 +282,14 @@ __global__ void __launch_bounds__(1024) k_reduce_rows(RedJobs jobs, int rows, in
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const int c = blockIdx.x * 32 + lane;
   float acc = 0.f;
-  if (c < n) {
+  if (c < n && rows <= 320) {            // NPART rows: all <= 10 loads of a lane in flight at once
+    float v[10];
+#pragma unroll
+    for (int i = 0; i < 10; ++i) v[i] = warp + 32 * i < rows ? jb.part[(int64_t)(warp + 32 * i) * ld + c] : 0.f;
+#pragma unroll
+    for (int i = 0; i < 10; ++i)
+      if (warp + 32 * i < rows) acc += v[i];   // row order, as below
+  } else if (c < n) {
     int p = warp;
     for (; p + 96 < rows; p += 128) {     // 4 independent loads in flight, added in row order
       const float v0 = jb.part[(int64_t)p * ld + c], v1 = jb.part[(int64_t)(p + 32) * ld + c];
