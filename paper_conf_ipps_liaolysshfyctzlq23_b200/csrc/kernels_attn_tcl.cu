@@ -112,8 +112,9 @@ __global__ void __launch_bounds__(LTH, 2) k_attn_fwd_tcl(const __grid_constant__
   uint8_t* sK = sm + LT;
   uint8_t* sV = sm + 2 * LT;
   uint8_t* sP = sm + 3 * LT;
-  uint64_t* bar = (uint64_t*)(sP + LPT);        // [0] Q, [1] K/V, [2] MMA S, [3] MMA O
-  uint32_t* tslot = (uint32_t*)(bar + 4);
+  // [0] Q, [1] K buffer sK, [2] MMA S, [3] MMA O, [4] K buffer sV (pass 1), [5] V (pass 2)
+  uint64_t* bar = (uint64_t*)(sP + LPT);
+  uint32_t* tslot = (uint32_t*)(bar + 6);
   float* red = (float*)(bar + 8);               // [2][128] x 2
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const int hf = warp >> 2, t = 32 * (warp & 3) + lane;
@@ -124,7 +125,7 @@ __global__ void __launch_bounds__(LTH, 2) k_attn_fwd_tcl(const __grid_constant__
   const int kl_tile = a.causal ? min(len, q0 + LQ) : len;
   const int nkt = (kl_tile + LQ - 1) / LQ;
   if (threadIdx.x == 0) {
-    for (int i = 0; i < 4; ++i) mbar_init(&bar[i], 1);
+    for (int i = 0; i < 6; ++i) mbar_init(&bar[i], 1);
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
   }
   if (warp == 0) tmem_alloc(tslot, 256);
@@ -133,24 +134,33 @@ __global__ void __launch_bounds__(LTH, 2) k_attn_fwd_tcl(const __grid_constant__
   const uint32_t trow = tmem + ((uint32_t)(32 * (warp & 3)) << 16);
   const int row0 = b * S;
   const float sl2 = a.scale * 1.4426950408889634f;
+  // TMA prefetch (thread 0 only; its phase bits): pass 1 double-buffers K in sK / sV
+  // (V is not needed yet); pass 2 reloads K as soon as S = Q K_j is done and V as
+  // soon as O += P~ V_j is done, so each tile's loads overlap the previous tile.
+  uint32_t ph_k0 = 0, ph_k1 = 0, ph_v = 0;
   if (threadIdx.x == 0 && nkt > 0) {
     mbar_expect_tx(&bar[0], LT);
     tma_load_2d(&tq, &bar[0], sQ, hd * LD, row0 + q0);
+    mbar_expect_tx(&bar[1], LT);
+    tma_load_2d(&tq, &bar[1], sK, a.H + hd * LD, row0);
   }
-  int ph_kv = 0, ph_s = 0, ph_o = 0;
+  int ph_s = 0, ph_o = 0;
   // ---- pass 1: exact row max and sum (log2 domain) ----
   float m = -INFINITY, l = 0.f;
   for (int j = 0; j < nkt; ++j) {
     if (threadIdx.x == 0) {
-      mbar_expect_tx(&bar[1], LT);
-      tma_load_2d(&tq, &bar[1], sK, a.H + hd * LD, row0 + j * LQ);
+      const int bf = j & 1;
+      if (j + 1 < nkt) {                        // buffer !bf held K_{j-1}: its MMA is done
+        mbar_expect_tx(&bar[bf ? 1 : 4], LT);
+        tma_load_2d(&tq, &bar[bf ? 1 : 4], bf ? sK : sV, a.H + hd * LD, row0 + (j + 1) * LQ);
+      }
       if (j == 0) mbar_wait(&bar[0], 0);
-      mbar_wait(&bar[1], ph_kv);
+      if (bf) { mbar_wait(&bar[4], ph_k1); ph_k1 ^= 1; }
+      else { mbar_wait(&bar[1], ph_k0); ph_k0 ^= 1; }
       tc_fence_after();
-      mma_nt64(tmem, smem_u32(sQ), smem_u32(sK));
+      mma_nt64(tmem, smem_u32(sQ), smem_u32(bf ? sV : sK));
       mma_commit(&bar[2]);
     }
-    ph_kv ^= 1;
     mbar_wait(&bar[2], ph_s);
     ph_s ^= 1;
     __syncwarp();
@@ -180,21 +190,28 @@ __global__ void __launch_bounds__(LTH, 2) k_attn_fwd_tcl(const __grid_constant__
   const float L2 = M + __log2f(lt);             // log2-domain LSE of s * scale
   const uint64_t ebase = (((uint64_t)b * a.h + hd) * S + (uint64_t)q) * S;
   // ---- pass 2: P~ = exp(S - LSE) * dropout, O += P~ V ----
+  if (threadIdx.x == 0 && nkt > 0) {            // every pass-1 MMA is done (bar[2] waited)
+    mbar_expect_tx(&bar[1], LT);
+    tma_load_2d(&tq, &bar[1], sK, a.H + hd * LD, row0);
+    mbar_expect_tx(&bar[5], LT);
+    tma_load_2d(&tq, &bar[5], sV, 2 * a.H + hd * LD, row0);
+  }
   for (int j = 0; j < nkt; ++j) {
     if (threadIdx.x == 0) {
-      mbar_expect_tx(&bar[1], 2 * LT);
-      tma_load_2d(&tq, &bar[1], sK, a.H + hd * LD, row0 + j * LQ);
-      tma_load_2d(&tq, &bar[1], sV, 2 * a.H + hd * LD, row0 + j * LQ);
-      mbar_wait(&bar[1], ph_kv);
+      mbar_wait(&bar[1], ph_k0);
+      ph_k0 ^= 1;
       tc_fence_after();
       mma_nt64(tmem, smem_u32(sQ), smem_u32(sK));
       mma_commit(&bar[2]);
     }
-    ph_kv ^= 1;
     mbar_wait(&bar[2], ph_s);
     ph_s ^= 1;
     __syncwarp();
     tc_fence_after();
+    if (threadIdx.x == 0 && j + 1 < nkt) {      // sK is free once S = Q K_j is in TMEM
+      mbar_expect_tx(&bar[1], LT);
+      tma_load_2d(&tq, &bar[1], sK, a.H + hd * LD, row0 + (j + 1) * LQ);
+    }
 #pragma unroll
     for (int c = 0; c < 4; ++c) {
       float v[16];
@@ -219,13 +236,20 @@ __global__ void __launch_bounds__(LTH, 2) k_attn_fwd_tcl(const __grid_constant__
     fence_async_smem();
     bar_sync_all();
     if (threadIdx.x == 0) {
+      mbar_wait(&bar[5], ph_v);
+      ph_v ^= 1;
+      tc_fence_after();
       mma_pv(tmem + 128, smem_u32(sP), smem_u32(sV), j > 0);
       mma_commit(&bar[3]);
     }
-    mbar_wait(&bar[3], ph_o);                   // P~, K, V and S free for the next tile
+    mbar_wait(&bar[3], ph_o);                   // P~, V and S free for the next tile
     ph_o ^= 1;
     __syncwarp();
     tc_fence_after();
+    if (threadIdx.x == 0 && j + 1 < nkt) {
+      mbar_expect_tx(&bar[5], LT);
+      tma_load_2d(&tq, &bar[5], sV, 2 * a.H + hd * LD, row0 + (j + 1) * LQ);
+    }
   }
   {  // epilogue: half hf stores dims [32hf, 32hf + 32) of row q
     float v[32];
