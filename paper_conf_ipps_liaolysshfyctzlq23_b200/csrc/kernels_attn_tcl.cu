@@ -272,7 +272,7 @@ __global__ void __launch_bounds__(LTH, 2) k_attn_fwd_tcl(const __grid_constant__
 }
 
 // ------------------------------------------------------------ backward dQ --
-constexpr int LQ_SMEM = 4 * LT + LPT + 1024 + 2048;   // Q, dO, K, V, dS
+constexpr int LQ_SMEM = 6 * LT + LPT + 1024 + 2048;   // Q, dO, K[2], V[2], dS
 
 __global__ void __launch_bounds__(LTH, 1) k_attn_bwd_dq_tcl(const __grid_constant__ CUtensorMap tq,
                                                             const __grid_constant__ CUtensorMap tdo, const LArgs a) {
@@ -281,11 +281,13 @@ __global__ void __launch_bounds__(LTH, 1) k_attn_bwd_dq_tcl(const __grid_constan
   uint8_t* sm = (uint8_t*)(((uintptr_t)smraw + 1023) & ~(uintptr_t)1023);
   uint8_t* sQ = sm;
   uint8_t* sdO = sm + LT;
-  uint8_t* sK = sm + 2 * LT;
-  uint8_t* sV = sm + 3 * LT;
-  uint8_t* sdS = sm + 4 * LT;
-  uint64_t* bar = (uint64_t*)(sdS + LPT);       // [0] Q/dO, [1] K/V, [2] MMA S/dP, [3] MMA dQ
-  uint32_t* tslot = (uint32_t*)(bar + 4);
+  // K_j / V_j in buffer j & 1 (K at 2LT + 2LT*buf, V right after): tile j+1 loads
+  // while tile j is processed
+  auto sKb = [&](int bf) { return sm + 2 * LT + 2 * LT * bf; };
+  auto sVb = [&](int bf) { return sm + 3 * LT + 2 * LT * bf; };
+  uint8_t* sdS = sm + 6 * LT;
+  uint64_t* bar = (uint64_t*)(sdS + LPT);       // [0] Q/dO, [1] K/V buf 0, [2] MMA S/dP, [3] MMA dQ, [4] K/V buf 1
+  uint32_t* tslot = (uint32_t*)(bar + 6);
   float* red = (float*)(bar + 8);
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const int hf = warp >> 2, t = 32 * (warp & 3) + lane;
@@ -297,7 +299,7 @@ __global__ void __launch_bounds__(LTH, 1) k_attn_bwd_dq_tcl(const __grid_constan
   const int kl_tile = a.causal ? min(len, q0 + LQ) : len;
   const int nkt = q0 < len ? (kl_tile + LQ - 1) / LQ : 0;
   if (threadIdx.x == 0) {
-    for (int i = 0; i < 4; ++i) mbar_init(&bar[i], 1);
+    for (int i = 0; i < 5; ++i) mbar_init(&bar[i], 1);
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
   }
   if (warp == 0) tmem_alloc(tslot, 512);
@@ -309,6 +311,9 @@ __global__ void __launch_bounds__(LTH, 1) k_attn_bwd_dq_tcl(const __grid_constan
     mbar_expect_tx(&bar[0], 2 * LT);
     tma_load_2d(&tq, &bar[0], sQ, hd * LD, row0 + q0);
     tma_load_2d(&tdo, &bar[0], sdO, hd * LD, row0 + q0);
+    mbar_expect_tx(&bar[1], 2 * LT);
+    tma_load_2d(&tq, &bar[1], sKb(0), a.H + hd * LD, row0);
+    tma_load_2d(&tq, &bar[1], sVb(0), 2 * a.H + hd * LD, row0);
   }
   // D_q = rowsum(dO * O): half hf sums dims [32hf, 32hf + 32); D = half 0 + half 1
   float Dh = 0.f, Lt = 0.f;
@@ -326,20 +331,26 @@ __global__ void __launch_bounds__(LTH, 1) k_attn_bwd_dq_tcl(const __grid_constan
   if (hf == 0 && q < S) a.Dbuf[((int64_t)b * a.h + hd) * S + q] = Dt;
   const float sl2 = a.scale * 1.4426950408889634f, Ll2 = Lt * 1.4426950408889634f;
   const uint64_t ebase = (((uint64_t)b * a.h + hd) * S + (uint64_t)q) * S;
-  int ph_kv = 0, ph_s = 0, ph_o = 0;
+  uint32_t ph_kv0 = 0, ph_kv1 = 0;
+  int ph_s = 0, ph_o = 0;
   for (int j = 0; j < nkt; ++j) {
+    const int bf = j & 1;
+    uint8_t* sK = sKb(bf);
+    uint8_t* sV = sVb(bf);
     if (threadIdx.x == 0) {
-      mbar_expect_tx(&bar[1], 2 * LT);
-      tma_load_2d(&tq, &bar[1], sK, a.H + hd * LD, row0 + j * LQ);
-      tma_load_2d(&tq, &bar[1], sV, 2 * a.H + hd * LD, row0 + j * LQ);
+      if (j + 1 < nkt) {                        // buffer !bf held tile j-1: its MMAs are done
+        mbar_expect_tx(&bar[bf ? 1 : 4], 2 * LT);
+        tma_load_2d(&tq, &bar[bf ? 1 : 4], sKb(bf ^ 1), a.H + hd * LD, row0 + (j + 1) * LQ);
+        tma_load_2d(&tq, &bar[bf ? 1 : 4], sVb(bf ^ 1), 2 * a.H + hd * LD, row0 + (j + 1) * LQ);
+      }
       if (j == 0) mbar_wait(&bar[0], 0);
-      mbar_wait(&bar[1], ph_kv);
+      if (bf) { mbar_wait(&bar[4], ph_kv1); ph_kv1 ^= 1; }
+      else { mbar_wait(&bar[1], ph_kv0); ph_kv0 ^= 1; }
       tc_fence_after();
       mma_nt64(tmem, smem_u32(sQ), smem_u32(sK));          // S = Q K^T
       mma_nt64(tmem + 128, smem_u32(sdO), smem_u32(sV));   // dP~ = dO V^T
       mma_commit(&bar[2]);
     }
-    ph_kv ^= 1;
     mbar_wait(&bar[2], ph_s);
     ph_s ^= 1;
     __syncwarp();
@@ -397,7 +408,7 @@ __global__ void __launch_bounds__(LTH, 1) k_attn_bwd_dq_tcl(const __grid_constan
 }
 
 // --------------------------------------------------------- backward dK, dV --
-constexpr int LKV_SMEM = 4 * LT + 2 * LPT + 1024 + 2048;   // K, V, Q, dO, P~, dS
+constexpr int LKV_SMEM = 6 * LT + 2 * LPT + 1024 + 2048;   // K, V, Q[2], dO[2], P~, dS
 
 __global__ void __launch_bounds__(LTH, 1) k_attn_bwd_dkv_tcl(const __grid_constant__ CUtensorMap tq,
                                                              const __grid_constant__ CUtensorMap tdo, const LArgs a) {
@@ -406,12 +417,13 @@ __global__ void __launch_bounds__(LTH, 1) k_attn_bwd_dkv_tcl(const __grid_consta
   uint8_t* sm = (uint8_t*)(((uintptr_t)smraw + 1023) & ~(uintptr_t)1023);
   uint8_t* sK = sm;
   uint8_t* sV = sm + LT;
-  uint8_t* sQ = sm + 2 * LT;
-  uint8_t* sdO = sm + 3 * LT;
-  uint8_t* sP = sm + 4 * LT;
+  // Q_i / dO_i in buffer (i - i0) & 1: tile i+1 loads while tile i is processed
+  auto sQb = [&](int bf) { return sm + 2 * LT + 2 * LT * bf; };
+  auto sdOb = [&](int bf) { return sm + 3 * LT + 2 * LT * bf; };
+  uint8_t* sP = sm + 6 * LT;
   uint8_t* sdS = sP + LPT;
-  uint64_t* bar = (uint64_t*)(sdS + LPT);       // [0] K/V, [1] Q/dO, [2] MMA S/dP, [3] MMA dV/dK
-  uint32_t* tslot = (uint32_t*)(bar + 4);
+  uint64_t* bar = (uint64_t*)(sdS + LPT);       // [0] K/V, [1] Q/dO buf 0, [2] MMA S/dP, [3] MMA dV/dK, [4] Q/dO buf 1
+  uint32_t* tslot = (uint32_t*)(bar + 6);
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const int hf = warp >> 2, t = 32 * (warp & 3) + lane;
   const int k0 = blockIdx.x * LQ, bh = blockIdx.y, b = bh / a.h, hd = bh % a.h;
@@ -420,7 +432,7 @@ __global__ void __launch_bounds__(LTH, 1) k_attn_bwd_dkv_tcl(const __grid_consta
   const int i0 = a.causal ? k0 / LQ : 0;
   const int i1 = k0 < len ? (len + LQ - 1) / LQ : 0;
   if (threadIdx.x == 0) {
-    for (int i = 0; i < 4; ++i) mbar_init(&bar[i], 1);
+    for (int i = 0; i < 5; ++i) mbar_init(&bar[i], 1);
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
   }
   if (warp == 0) tmem_alloc(tslot, 512);
@@ -432,22 +444,31 @@ __global__ void __launch_bounds__(LTH, 1) k_attn_bwd_dkv_tcl(const __grid_consta
     mbar_expect_tx(&bar[0], 2 * LT);
     tma_load_2d(&tq, &bar[0], sK, a.H + hd * LD, row0 + k0);
     tma_load_2d(&tq, &bar[0], sV, 2 * a.H + hd * LD, row0 + k0);
+    mbar_expect_tx(&bar[1], 2 * LT);
+    tma_load_2d(&tq, &bar[1], sQb(0), hd * LD, row0 + i0 * LQ);
+    tma_load_2d(&tdo, &bar[1], sdOb(0), hd * LD, row0 + i0 * LQ);
   }
   const float sl2 = a.scale * 1.4426950408889634f;
-  int ph_q = 0, ph_s = 0, ph_o = 0;
+  uint32_t ph_q0 = 0, ph_q1 = 0;
+  int ph_s = 0, ph_o = 0;
   for (int i = i0; i < i1; ++i) {
+    const int bf = (i - i0) & 1;
+    uint8_t* sQ = sQb(bf);
+    uint8_t* sdO = sdOb(bf);
     if (threadIdx.x == 0) {
-      mbar_expect_tx(&bar[1], 2 * LT);
-      tma_load_2d(&tq, &bar[1], sQ, hd * LD, row0 + i * LQ);
-      tma_load_2d(&tdo, &bar[1], sdO, hd * LD, row0 + i * LQ);
+      if (i + 1 < i1) {                         // buffer !bf held tile i-1: its MMAs are done
+        mbar_expect_tx(&bar[bf ? 1 : 4], 2 * LT);
+        tma_load_2d(&tq, &bar[bf ? 1 : 4], sQb(bf ^ 1), hd * LD, row0 + (i + 1) * LQ);
+        tma_load_2d(&tdo, &bar[bf ? 1 : 4], sdOb(bf ^ 1), hd * LD, row0 + (i + 1) * LQ);
+      }
       if (i == i0) mbar_wait(&bar[0], 0);
-      mbar_wait(&bar[1], ph_q);
+      if (bf) { mbar_wait(&bar[4], ph_q1); ph_q1 ^= 1; }
+      else { mbar_wait(&bar[1], ph_q0); ph_q0 ^= 1; }
       tc_fence_after();
       mma_nt64(tmem, smem_u32(sQ), smem_u32(sK));          // S_i = Q_i K^T (rows = queries)
       mma_nt64(tmem + 128, smem_u32(sdO), smem_u32(sV));   // dP~_i = dO_i V^T
       mma_commit(&bar[2]);
     }
-    ph_q ^= 1;
     const int q = i * LQ + t;
     const bool live = q < len;
     const int kl = a.causal ? min(len, q + 1) : len;
