@@ -28,7 +28,7 @@ from typing import Dict, List, Optional, Sequence
 from paper_conf_ipps_liaolysshfyctzlq23_b200.workload import (
     ARCH_PRE_LN, HEAD_LM, HEAD_QA, ModelConfig, param_spec)
 
-LM_CHUNK = 512     # tokens per LM-head chunk (logits never exceed LM_CHUNK x Vpad)
+LM_CHUNK = 2048     # tokens per LM-head chunk (logits never exceed LM_CHUNK x Vpad)
 
 
 def vpad(v: int) -> int:

@@ -37,7 +37,7 @@ struct ParamInfo {
 };
 
 // The documented parameter order (DESIGN "Parameter layout").
-constexpr int LM_CHUNK = 512;   // tokens per LM-head chunk (DESIGN "Memory model")
+constexpr int LM_CHUNK = 2048;   // tokens per LM-head chunk (DESIGN "Memory model")
 inline int64_t vpad(int64_t v) { return (v + 7) / 8 * 8; }
 
 std::vector<ParamInfo> build_layout(const mimose_config& c, int64_t* npad) {
