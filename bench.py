@@ -447,27 +447,26 @@ def main():
         result["no_ckpt"] = {"value": samples_per_step * args.steps / (ms_n / 1000.0),
                              "ms_per_step": ms_n / args.steps, "peak_bytes": peak_n,
                              "over_budget": peak_n > M}
-        if cfg.arch == wl.ARCH_POST_LN:
-            # sub-layer checkpoint units (reading A30): attention / FFN
-            # blocks planned independently by the same Algorithm 1, same budget
-            ctx = new_ctx(M, M, granularity=1)
-            j = 0
-            while ctx.phase == mb.PHASE_SHELTERED:
-                b = wl.make_batch(cfg, sched[j % len(sched)], seed=wl.batch_seed(cfg, 10**6 + j, rank))
-                ctx.collect(ctx.host_batch(b), want_loss=False)
-                ctx.backward()
-                ctx.step(1e-5)
-                j += 1
-            ms_u, _, _ = timed(ctx, batches, "mimose")
-            stu = ctx.stats()
-            units = [ctx.plan(b.input_size).n_dropped for b in batches[args.warmup:]]
-            ctx.close()
-            del ctx
-            torch.cuda.empty_cache()
-            result["sublayer_units"] = {"value": samples_per_step * args.steps / (ms_u / 1000.0),
-                                        "ms_per_step": ms_u / args.steps, "mean_units_dropped": float(np.mean(units)),
-                                        "units": 2 * cfg.n_layers, "violations": stu["violations"],
-                                        "peak_bytes_max": stu["max_peak_bytes"], "recompute_ratio": ms_u / ms_n}
+        # sub-layer checkpoint units (reading A30): attention / FFN
+        # blocks planned independently by the same Algorithm 1, same budget
+        ctx = new_ctx(M, M, granularity=1)
+        j = 0
+        while ctx.phase == mb.PHASE_SHELTERED:
+            b = wl.make_batch(cfg, sched[j % len(sched)], seed=wl.batch_seed(cfg, 10**6 + j, rank))
+            ctx.collect(ctx.host_batch(b), want_loss=False)
+            ctx.backward()
+            ctx.step(1e-5)
+            j += 1
+        ms_u, _, _ = timed(ctx, batches, "mimose")
+        stu = ctx.stats()
+        units = [ctx.plan(b.input_size).n_dropped for b in batches[args.warmup:]]
+        ctx.close()
+        del ctx
+        torch.cuda.empty_cache()
+        result["sublayer_units"] = {"value": samples_per_step * args.steps / (ms_u / 1000.0),
+                                    "ms_per_step": ms_u / args.steps, "mean_units_dropped": float(np.mean(units)),
+                                    "units": 2 * cfg.n_layers, "violations": stu["violations"],
+                                    "peak_bytes_max": stu["max_peak_bytes"], "recompute_ratio": ms_u / ms_n}
         result["recompute_ratio"] = ms / ms_n
         result["speedup_vs_static"] = ms_s / ms
         result["paper_context"] = ("V100 (P:227): Mimose ~18.0% faster than Sublinear, ~15.0% than DTR "

@@ -95,12 +95,13 @@ typedef struct {
   int32_t use_tc;        /* 1: tcgen05 GEMMs in bf16 mode (default); 0: SIMT GEMMs  */
   int32_t pad_id;        /* padding token id: its embedding row gets no gradient (HF
                             padding_idx semantics, reading A24); -1 = none           */
-  int32_t granularity;   /* checkpoint unit: 0 = encoder layer (default, A14); 1 = sub-layer
-                            (post-LN only): unit 2l = attention block of layer l (internals
-                            QKV, O, LSE, z1, st1; output h1), unit 2l+1 = its FFN block
-                            (internals u, g, z2, st2; output y), so 2L <= 64 units
-                            ("attention block"; reading A30).
-                            Samples, series and drop masks are then indexed by unit.  */
+  int32_t granularity;   /* checkpoint unit: 0 = encoder layer (default, A14); 1 = sub-layer:
+                            unit 2l = attention block of layer l (post-LN internals QKV, O,
+                            LSE, z1, st1, output h1; pre-LN a, st1, QKV, O, LSE, output r1),
+                            unit 2l+1 = its FFN block (post-LN u, g, z2, st2; pre-LN st2, m,
+                            u, g; output y), so 2L <= 64 units (SURVEY f1, P:125/P:140
+                            "attention block"; reading A30).  Samples, series and drop
+                            masks are then indexed by unit.                              */
   int32_t reserved[5];
 } mimose_config;
 

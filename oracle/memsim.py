@@ -332,14 +332,14 @@ def collect_samples(sz: Sizes) -> Dict[str, object]:
 # --------------------------------------------------------------------------
 # P:125 and P:140 name the "attention block" as a unit Mimose can checkpoint
 # ("the output ... of the attention block"), P:170 lets a stage be any
-# user-code structure.  With granularity 1 each post-LN layer l is two units:
-#   unit 2l   attention block  internals QKV, O, LSE, z1, st1   output h1
-#   unit 2l+1 FFN block        internals u, g, z2, st2          output y
+# user-code structure.  With granularity 1 each layer l is two units:
+#   unit 2l   attention block  post-LN: QKV, O, LSE, z1, st1 -> h1; pre-LN: a, st1, QKV, O, LSE -> r1
+#   unit 2l+1 FFN block        post-LN: u, g, z2, st2 -> y;     pre-LN: st2, m, u, g -> y
 # Forward: a kept unit pushes its internals then its output; a dropped unit
 # places its internals in the top region, pushes its output, frees them.
 # Backward of layer l (after y_l is gone):
-#   FFN dropped -> push its internals (recompute from h1)
-#   talloc layer scratch; FFN-block gradients; pop FFN internals; pop h1
+#   FFN dropped -> push its internals (recompute from h1 / r1)
+#   talloc layer scratch; FFN-block gradients; pop FFN internals; pop h1 / r1
 #   attention dropped -> push its internals (recompute from y_{l-1})
 #   attention-block gradients; tfree scratch; pop attention internals; pop y_{l-1}
 # With nothing dropped the event sequence reaches the same peak as the layer
@@ -347,8 +347,9 @@ def collect_samples(sz: Sizes) -> Dict[str, object]:
 # unchanged to the 2L-unit series.
 
 def unit_list(sz: Sizes) -> List[tuple]:
-    """[(internals, output)] for the 2L units of a post-LN stack."""
-    assert len(sz.internals) == 10, "sub-layer units are defined for the post-LN layer"
+    """[(internals, output)] for the 2L units of a stack (both layer types keep
+    10 internals whose 6th is the block boundary h1 / r1)."""
+    assert len(sz.internals) == 10
     att, h1, ffn = sz.internals[:5], sz.internals[5], sz.internals[6:]
     out = []
     for _ in range(sz.n_layers):

@@ -429,25 +429,39 @@ void alloc_internals(Run& r, LayerBufs& b, bool on_stack) {
 // Sub-layer units (granularity 1, post-LN; DESIGN reading A30): the attention
 // block's internals [QKV, O, LSE, z1, st1] and the FFN block's [u, g, z2, st2],
 // in the layer's push order (h1 sits between them).
+// Pre-LN (GPT-2): attention [a, st1, QKV, O, LSE] -> r1, FFN [st2, m, u, g] -> y.
 void alloc_att(Run& r, LayerBufs& b, bool on_stack) {
   Arena& a = r.c->ar;
   auto al = [&](int64_t n) { return on_stack ? a.push(n) : a.talloc(n); };
+  if (r.c->cfg.arch == 1) {
+    b.a = al(r.z.a); b.st1 = (float2*)al(r.z.st1); b.qkv = al(r.z.qkv); b.O = al(r.z.O);
+    b.lse = (float*)al(r.z.lse);
+    return;
+  }
   b.qkv = al(r.z.qkv); b.O = al(r.z.O); b.lse = (float*)al(r.z.lse);
   b.z1 = (float*)al(r.z.z1); b.st1 = (float2*)al(r.z.st1);
 }
 void free_att(Run& r, bool on_stack) {
   Arena& a = r.c->ar;
-  const int64_t s[5] = {r.z.qkv, r.z.O, r.z.lse, r.z.z1, r.z.st1};
+  const int64_t s0[5] = {r.z.qkv, r.z.O, r.z.lse, r.z.z1, r.z.st1};
+  const int64_t s1[5] = {r.z.a, r.z.st1, r.z.qkv, r.z.O, r.z.lse};
+  const int64_t* s = r.c->cfg.arch == 1 ? s1 : s0;
   for (int i = 4; i >= 0; --i) on_stack ? a.pop(s[i]) : a.tfree(s[i]);
 }
 void alloc_ffn(Run& r, LayerBufs& b, bool on_stack) {
   Arena& a = r.c->ar;
   auto al = [&](int64_t n) { return on_stack ? a.push(n) : a.talloc(n); };
+  if (r.c->cfg.arch == 1) {
+    b.st2 = (float2*)al(r.z.st2); b.m = al(r.z.m); b.u = al(r.z.u); b.g = al(r.z.g);
+    return;
+  }
   b.u = al(r.z.u); b.g = al(r.z.g); b.z2 = (float*)al(r.z.z2); b.st2 = (float2*)al(r.z.st2);
 }
 void free_ffn(Run& r, bool on_stack) {
   Arena& a = r.c->ar;
-  const int64_t s[4] = {r.z.u, r.z.g, r.z.z2, r.z.st2};
+  const int64_t s0[4] = {r.z.u, r.z.g, r.z.z2, r.z.st2};
+  const int64_t s1[4] = {r.z.st2, r.z.m, r.z.u, r.z.g};
+  const int64_t* s = r.c->cfg.arch == 1 ? s1 : s0;
   for (int i = 3; i >= 0; --i) on_stack ? a.pop(s[i]) : a.tfree(s[i]);
 }
 
@@ -659,10 +673,12 @@ void layer_backward(Run& r, int l, const char* x, LayerBufs& b, float* dy, char*
 // m = LN2(r1); y = r1 + drop(gelu_tanh(m W1 + b1) W2 + b2).  x, r1, y fp32.
 // In recompute (yout == nullptr) the FFN2 GEMM is skipped: y is not needed.
 // ---------------------------------------------------------------------------
-void layer_forward_pre(Run& r, int l, const float* x, LayerBufs& b, float* yout) {
+// Attention block of a pre-LN layer: x -> a = LN1(x), QKV, O, LSE -> r1 = x + drop(O Wo^T + bo).
+// r1out == nullptr (sub-layer recompute after r1 was released): the out-proj GEMM is skipped.
+void att_forward_pre(Run& r, int l, const float* x, LayerBufs& b, float* r1out) {
   mimose_ctx* c = r.c;
   if (!r.real) return;
-  const int T = c->T, H = c->cfg.hidden, F = c->cfg.ffn;
+  const int T = c->T, H = c->cfg.hidden;
   ln_fwd(c->dt, x, W(c, LP(c, l, L_LN1G)), W(c, LP(c, l, L_LN1B)), b.a, b.st1, T, H, c->cfg.ln_eps, r.st);
   GemmArgs g;
   g.M = T; g.N = 3 * H; g.K = H;
@@ -672,13 +688,23 @@ void layer_forward_pre(Run& r, int l, const float* x, LayerBufs& b, float* yout)
   pgemm(c, EPI_BIAS, g, r.st);
   attn_fwd(c->dt, b.qkv, c->lens, b.O, b.lse, c->B, c->S, H, c->cfg.heads, make_drop(c, KIND_ATTN_PROBS, l), r.st,
            true);
+  if (!r1out) return;
   g = GemmArgs();
   g.M = T; g.N = H; g.K = H;
   g.A = b.O; g.a_sm = H; g.a_sk = 1;
   g.B = W(c, LP(c, l, L_OW)); g.b_sn = H; g.b_sk = 1;
-  g.C = b.r1; g.ldc = H; g.bias = W(c, LP(c, l, L_OB)); g.res = x; g.ldr = H;
+  g.C = r1out; g.ldc = H; g.bias = W(c, LP(c, l, L_OB)); g.res = x; g.ldr = H;
   g.drop = make_drop(c, KIND_ATTN_OUT, l);
   pgemm(c, EPI_BIAS_DROP_RESF32, g, r.st);
+}
+
+// FFN block of a pre-LN layer: r1 (b.r1) -> m = LN2(r1), u, g -> y = r1 + drop(g W2^T + b2);
+// yout == nullptr (recompute): the FFN2 GEMM is skipped, y is not needed.
+void ffn_forward_pre(Run& r, int l, LayerBufs& b, float* yout) {
+  mimose_ctx* c = r.c;
+  if (!r.real) return;
+  const int T = c->T, H = c->cfg.hidden, F = c->cfg.ffn;
+  GemmArgs g;
   ln_fwd(c->dt, b.r1, W(c, LP(c, l, L_LN2G)), W(c, LP(c, l, L_LN2B)), b.m, b.st2, T, H, c->cfg.ln_eps, r.st);
   g = GemmArgs();
   g.M = T; g.N = F; g.K = H;
@@ -696,10 +722,16 @@ void layer_forward_pre(Run& r, int l, const float* x, LayerBufs& b, float* yout)
   pgemm(c, EPI_BIAS_DROP_RESF32, g, r.st);
 }
 
-void layer_backward_pre(Run& r, int l, const float* x, LayerBufs& b, float* dy, char* scr) {
+void layer_forward_pre(Run& r, int l, const float* x, LayerBufs& b, float* yout) {
+  att_forward_pre(r, l, x, b, b.r1);
+  ffn_forward_pre(r, l, b, yout);
+}
+
+// FFN-block gradients of a pre-LN layer, through LN2: dy -> dr1 (in place), dt1 (R3).
+void ffn_backward_pre(Run& r, int l, LayerBufs& b, float* dy, char* scr) {
   mimose_ctx* c = r.c;
   if (!r.real) return;
-  const int T = c->T, H = c->cfg.hidden, F = c->cfg.ffn, h = c->cfg.heads;
+  const int T = c->T, H = c->cfg.hidden, F = c->cfg.ffn;
   float* dres = (float*)(scr + r.z.r_dres);
   char* R2 = scr + r.z.r_du;     // du, later dO
   char* R3 = scr + r.z.r_dt;     // dt2 / dt1, later dQKV
@@ -730,6 +762,19 @@ void layer_backward_pre(Run& r, int l, const float* x, LayerBufs& b, float* dy, 
          pg, pb, pbias, T, H, r.st, dy);
   reduce_rows3(pg, G(c, LP(c, l, L_LN2G)), pb, G(c, LP(c, l, L_LN2B)), pbias, G(c, LP(c, l, L_OB)), NPART, H, H,
                r.st);
+}
+
+// Attention-block gradients of a pre-LN layer (after ffn_backward_pre: dy = dr1, R3 = dt1).
+void att_backward_pre(Run& r, int l, const float* x, LayerBufs& b, float* dy, char* scr) {
+  mimose_ctx* c = r.c;
+  if (!r.real) return;
+  const int T = c->T, H = c->cfg.hidden, h = c->cfg.heads;
+  float* dres = (float*)(scr + r.z.r_dres);
+  char* R2 = scr + r.z.r_du;
+  char* R3 = scr + r.z.r_dt;
+  float* Dbuf = (float*)(scr + r.z.r_dt + a16((int64_t)T * 3 * H * c->e));
+  float* pg = c->part;
+  float* pb = c->part + (int64_t)NPART * H;
   // out-proj: dO = dt1 Wo (R2); dWo = dt1^T O
   dgrad(r, EPI_STORE, R3, H, W(c, LP(c, l, L_OW)), H, R2, nullptr);
   wgrad(r, R3, H, b.O, H, G(c, LP(c, l, L_OW)));
@@ -744,6 +789,11 @@ void layer_backward_pre(Run& r, int l, const float* x, LayerBufs& b, float* dy, 
   ln_bwd(c->dt, dres, no_drop(), x, b.st1, W(c, LP(c, l, L_LN1G)), dy, nullptr, no_drop(), pg, pb, nullptr, T, H,
          r.st, dy);
   reduce_rows3(pg, G(c, LP(c, l, L_LN1G)), pb, G(c, LP(c, l, L_LN1B)), nullptr, nullptr, NPART, H, H, r.st);
+}
+
+void layer_backward_pre(Run& r, int l, const float* x, LayerBufs& b, float* dy, char* scr) {
+  ffn_backward_pre(r, l, b, dy, scr);
+  att_backward_pre(r, l, x, b, dy, scr);
 }
 
 // LM head (GPT-2): hf = LNf(y); chunks of LM_CHUNK tokens: logits = hf W_e^T (fp32),
@@ -865,6 +915,31 @@ void layer_bwd_any(Run& r, int l, const char* x, LayerBufs& b, float* dy, char* 
   else layer_backward(r, l, x, b, dy, scr);
 }
 
+// Sub-layer unit steps for either architecture; the unit boundary tensor ("mid")
+// is h1 = LN1(z1) (post-LN) or r1 = x + drop(attn) (pre-LN).
+int64_t mid_size(const Run& r) { return r.c->cfg.arch == 1 ? r.z.r1 : r.z.h1; }
+char* mid_of(const Run& r, const LayerBufs& b) { return r.c->cfg.arch == 1 ? (char*)b.r1 : b.h1; }
+void set_mid(const Run& r, LayerBufs& b, char* p) {
+  if (r.c->cfg.arch == 1) b.r1 = (float*)p;
+  else b.h1 = p;
+}
+void att_fwd_u(Run& r, int l, const char* x, LayerBufs& b, char* mid_out) {
+  if (r.c->cfg.arch == 1) att_forward_pre(r, l, (const float*)x, b, (float*)mid_out);
+  else att_forward(r, l, x, b, mid_out);
+}
+void ffn_fwd_u(Run& r, int l, LayerBufs& b, char* yout) {
+  if (r.c->cfg.arch == 1) ffn_forward_pre(r, l, b, (float*)yout);
+  else ffn_forward(r, l, b, yout);
+}
+void ffn_bwd_u(Run& r, int l, LayerBufs& b, float* dy, char* scr) {
+  if (r.c->cfg.arch == 1) ffn_backward_pre(r, l, b, dy, scr);
+  else ffn_backward(r, l, b, dy, scr);
+}
+void att_bwd_u(Run& r, int l, const char* x, LayerBufs& b, float* dy, char* scr) {
+  if (r.c->cfg.arch == 1) att_backward_pre(r, l, (const float*)x, b, dy, scr);
+  else att_backward(r, l, x, b, dy, scr);
+}
+
 // Forward of one step.  mode 0: plan-driven; mode 1: shuttling collector.
 // When `sample` is non-null the collector deltas are recorded.
 void run_forward(Run& r, uint64_t mask, bool collect, Sample* sample) {
@@ -900,28 +975,29 @@ void run_forward(Run& r, uint64_t mask, bool collect, Sample* sample) {
     if (collect && sample) {                  // pass 1 (save mode), timed, discarded
       LayerBufs tmp;
       alloc_att(r, tmp, true);
-      char* ht = a.push(r.z.h1);
+      char* ht = a.push(mid_size(r));
+      set_mid(r, tmp, ht);
       if (r.real) cudaEventRecord(c->ev_t0[ua], r.st);
-      att_forward(r, l, x, tmp, ht);
+      att_fwd_u(r, l, x, tmp, ht);
       if (r.real) cudaEventRecord(c->ev_t1[ua], r.st);
       sample->a[ua] = a.live() - b0;
-      a.pop(r.z.h1);
+      a.pop(mid_size(r));
       free_att(r, true);
     }
     const bool da = collect || ((mask >> ua) & 1);
     alloc_att(r, b, !da);
-    b.h1 = a.push(r.z.h1);
-    att_forward(r, l, x, b, b.h1);
+    set_mid(r, b, a.push(mid_size(r)));
+    att_fwd_u(r, l, x, b, mid_of(r, b));
     if (da) free_att(r, false);
     if (sample) sample->y[ua] = a.live() - b0;
     b0 = a.live();
     if (collect && sample) {
       LayerBufs tmp;
-      tmp.h1 = b.h1;
+      set_mid(r, tmp, mid_of(r, b));
       alloc_ffn(r, tmp, true);
       char* yt = a.push(r.z.y);
       if (r.real) cudaEventRecord(c->ev_t0[uf], r.st);
-      ffn_forward(r, l, tmp, yt);
+      ffn_fwd_u(r, l, tmp, yt);
       if (r.real) cudaEventRecord(c->ev_t1[uf], r.st);
       sample->a[uf] = a.live() - b0;
       a.pop(r.z.y);
@@ -930,7 +1006,7 @@ void run_forward(Run& r, uint64_t mask, bool collect, Sample* sample) {
     const bool df = collect || ((mask >> uf) & 1);
     alloc_ffn(r, b, !df);
     c->y[l] = a.push(r.z.y);
-    ffn_forward(r, l, b, c->y[l]);
+    ffn_fwd_u(r, l, b, c->y[l]);
     if (df) free_ffn(r, false);
     if (sample) sample->y[uf] = a.live() - b0;
     x = c->y[l];
@@ -1032,19 +1108,19 @@ mimose_status run_backward(Run& r, Sample* sample) {
   for (int l = L - 1; l >= 0 && c->cfg.granularity == 1; --l) {   // sub-layer units
     LayerBufs& b = c->lb[l];
     const char* x = l > 0 ? c->y[l - 1] : c->x1;
-    if ((c->drop_mask >> (2 * l + 1)) & 1) {          // recompute the FFN block from h1
+    if ((c->drop_mask >> (2 * l + 1)) & 1) {          // recompute the FFN block from h1 / r1
       alloc_ffn(r, b, true);
-      ffn_forward(r, l, b, nullptr);
+      ffn_fwd_u(r, l, b, nullptr);
     }
     char* scr = a.talloc(r.z.layer_scr);
-    ffn_backward(r, l, b, dy, scr);
+    ffn_bwd_u(r, l, b, dy, scr);
     free_ffn(r, true);
-    a.pop(r.z.h1);                                    // h1: dead after the FFN1 wgrad
+    a.pop(mid_size(r));                               // h1 / r1: dead after the FFN block's gradients
     if ((c->drop_mask >> (2 * l)) & 1) {              // recompute the attention block from y_{l-1}
       alloc_att(r, b, true);
-      att_forward(r, l, x, b, nullptr);
+      att_fwd_u(r, l, x, b, nullptr);
     }
-    att_backward(r, l, x, b, dy, scr);
+    att_bwd_u(r, l, x, b, dy, scr);
     a.tfree(r.z.layer_scr);
     if (r.real) {
       mimose_status s = allreduce_bucket(c, layer_base(c) + 12 * l, layer_base(c) + 12 * l + 11, l);
@@ -1227,7 +1303,7 @@ mimose_status mimose_init(const mimose_config* cfgp, mimose_ctx** out) {
       (k.head == MIMOSE_HEAD_MC && k.n_choices < 1) ||
       (k.head == MIMOSE_HEAD_SEQCLS && (k.n_labels < 1 || k.n_labels > 32)) || k.world < 1 || k.rank < 0 ||
       k.rank >= k.world || k.bucket_den <= 0 || k.degree < 0 || k.degree > 2 || k.granularity < 0 ||
-      k.granularity > 1 || (k.granularity == 1 && (k.arch != MIMOSE_ARCH_POST_LN || 2 * k.n_layers > 64))) {
+      k.granularity > 1 || (k.granularity == 1 && 2 * k.n_layers > 64)) {
     mimose_status s = bad("invalid model / sizing config");
     *out = c;   // returned so mimose_last_error works; caller destroys
     return s;

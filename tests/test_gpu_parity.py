@@ -239,7 +239,8 @@ def test_fused_optimizer_bitwise_equal(case):
 # sub-layer checkpoint units (granularity=1, DESIGN reading A30)
 # ---------------------------------------------------------------------------
 
-@pytest.mark.parametrize("case", ["toy-fp32", "mc-bf16", "qa-bf16-long"])
+@pytest.mark.parametrize("case", ["toy-fp32", "mc-bf16", "qa-bf16-long", "lm-gpt2-bf16", "lm-gpt2-bf16-long",
+                                  "lm-gpt2-fp32"])
 def test_units_recompute_replay_bitwise(case):
     """Unit plans (attention / FFN blocks dropped independently) replay the
     forward bit for bit: loss and gradients equal the layer-granularity

@@ -228,7 +228,7 @@ def test_exact_planner_on_config_series(name):
 # ---------------------------------------------------------------------------
 # sub-layer checkpoint units (granularity=1, DESIGN reading A30)
 # ---------------------------------------------------------------------------
-UNIT_CFGS = ["toy", "bert-base", "bert-large", "roberta-large"]
+UNIT_CFGS = ["toy", "bert-base", "bert-large", "roberta-large", "gpt2-medium"]
 
 
 @pytest.mark.parametrize("name", UNIT_CFGS)
@@ -290,8 +290,8 @@ def test_units_pipeline_matches_oracle(name, planner):
 
 
 def test_units_config_validation():
-    """granularity 1 is post-LN only (GPT-2's pre-LN blocks are not split)."""
-    with pytest.raises(mb.MimoseError):
-        mb.Mimose(wl.CONFIGS["gpt2-medium"], 1 << 40, granularity=1)
+    """granularity is 0 or 1, and 2L units must fit the 64-bit drop mask."""
     with pytest.raises(mb.MimoseError):
         mb.Mimose(wl.CONFIGS["toy"], 1 << 40, granularity=2)
+    with pytest.raises(mb.MimoseError):
+        mb.Mimose(wl.small_config("bert-base", n_layers=33), 1 << 40, granularity=1)

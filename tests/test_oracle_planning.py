@@ -307,7 +307,7 @@ def test_units_event_model(name):
             assert om.simulate_step_units(sz, [2 * j + 1 for j in range(k)]).peak == P0 - k * i_ffn
 
 
-@pytest.mark.parametrize("name", POST_LN)
+@pytest.mark.parametrize("name", CFGS)
 def test_units_predicted_peak_formula(name):
     """The planner's position-aware peak over the 2L-unit collected series is
     exactly the unit event simulator's peak, for random unit plans."""
@@ -321,7 +321,7 @@ def test_units_predicted_peak_formula(name):
             assert op.predicted_peak(c, plan) == om.simulate_step_units(sz, plan).peak
 
 
-@pytest.mark.parametrize("name", POST_LN)
+@pytest.mark.parametrize("name", CFGS)
 def test_units_planners_feasible_and_exact(name):
     """Algorithm 1 on the unit series (heterogeneous: attention / FFN units
     alternate) returns a plan within the budget whenever one exists; the exact
