@@ -342,7 +342,17 @@ __global__ void __launch_bounds__(256) k_colsum(const E* __restrict__ X, int T, 
   const int c = blockIdx.x * 2048 + threadIdx.x * 8;
   if (c >= N) return;
   float acc[8] = {0.f, 0.f, 0.f, 0.f, 0.f, 0.f, 0.f, 0.f};
-  for (int r = blockIdx.y; r < T; r += NPART) {
+  int r = blockIdx.y;
+  for (; r + 3 * NPART < T; r += 4 * NPART) {   // 4 rows of loads in flight, added in row order
+    float v[4][8];
+#pragma unroll
+    for (int k = 0; k < 4; ++k) ld8(X + (int64_t)(r + k * NPART) * N + c, v[k]);
+#pragma unroll
+    for (int k = 0; k < 4; ++k)
+#pragma unroll
+      for (int i = 0; i < 8; ++i) acc[i] += v[k][i];
+  }
+  for (; r < T; r += NPART) {
     float v[8];
     ld8(X + (int64_t)r * N + c, v);
 #pragma unroll

@@ -24,7 +24,7 @@ def main(src, dst):
         names[k] = r["Kernel Name"]
         v = float(r["Metric Value"].replace(",", "")) * UNIT.get(r["Metric Unit"], 1.0)
         per[k][r["Metric Name"]] = v
-    launches = [m for m in per.values() if "dram__bytes_read.sum" in m]
+    launches = [m for k, m in per.items() if "dram__bytes_read.sum" in m and "k_gemm_tc" in names[k]]
     rd = sum(m["dram__bytes_read.sum"] for m in launches)
     wr = sum(m.get("dram__bytes_write.sum", 0.0) for m in launches)
     t = sum(m.get("gpu__time_duration.sum", 0.0) for m in launches)
@@ -33,7 +33,8 @@ def main(src, dst):
            "dram_read_bytes_per_launch": rd / max(n, 1), "dram_write_bytes_per_launch": wr / max(n, 1),
            "mean_duration_us": 1e6 * t / max(n, 1),
            "how": "ncu --metrics dram__bytes_read.sum,dram__bytes_write.sum over every k_gemm_tc* launch of "
-                  "`bench.py --steps 3 --warmup 3` (cold cache per launch, ncu default cache control)",
+                  "`bench.py --steps 2 --warmup 3 --no-baselines --no-cpu-baseline` (cold cache per launch, "
+                  "ncu default cache control)",
            "source": src}
     json.dump(out, open(dst, "w"), indent=1)
     print(json.dumps(out))
