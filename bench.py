@@ -157,11 +157,18 @@ def dist_env():
 # reference arm: the fp64 CPU oracle (DESIGN "Measurement")
 # ---------------------------------------------------------------------------
 
-def oracle_sample_step(cfg, S_longest, n_q, step):
-    """One oracle training step on a bounded sample: n_q questions of the workload."""
+def oracle_sample_step(cfg, S_longest, n_q, step, n_layers=None):
+    """One oracle training step (forward, backward, AdamW) on a bounded sample:
+    n_q questions of the workload through a model of n_layers encoder layers
+    (default: all) whose word-embedding table shrinks in the same proportion,
+    so every part of the step (layers, embedding, AdamW over the parameters)
+    scales by n_layers / L.  Returns (seconds, samples processed)."""
     from oracle import model as om
-    sub = wl.small_config(cfg.name, n_seqs=n_q * (cfg.n_choices if cfg.head == wl.HEAD_MC else 1))
-    params = ORACLE_PARAMS.setdefault(cfg.name, wl.init_params(cfg))
+    L = cfg.n_layers if n_layers is None else n_layers
+    V = cfg.vocab if L == cfg.n_layers else max(1024, cfg.vocab * L // cfg.n_layers)
+    sub = wl.small_config(cfg.name, n_seqs=n_q * (cfg.n_choices if cfg.head == wl.HEAD_MC else 1), n_layers=L,
+                          vocab=V)
+    params = ORACLE_PARAMS.setdefault((cfg.name, L), wl.init_params(sub))
     b = wl.make_batch(sub, S_longest, seed=wl.batch_seed(cfg, step))
     t0 = time.perf_counter()
     loss, G = om.train_step_grads(sub, params, b, wl.dropout_seed(cfg), step + 1)
@@ -187,22 +194,39 @@ def cpu_baseline(cfg, n_steps=2, n_q=2):
                       f"({cfg.name}, full width/depth), {tot_t:.1f} s"}
 
 
+REF_BUDGET_S = 150.0   # the reference arm's whole --steps K --warmup W run
+
+
 def run_reference(args):
+    """--impl reference: the fp64 oracle as it stands, on the host cores, on a
+    bounded sample per step.  A step is one question (MC) / sequence through the
+    full model when K + W such steps fit REF_BUDGET_S; otherwise through a
+    model with L_s of the L encoder layers and an L_s / L word-embedding table
+    (every part of the step then scales by f = L_s / L: the L identical layers,
+    the embedding and the AdamW sweep), L_s the largest that fits, counted as
+    f of a sample."""
     world, rank, _ = dist_env()
     if rank != 0:
         return
     cfg = wl.CONFIGS[args.config]
-    sched = wl.length_schedule(cfg, args.warmup + args.steps)
+    sched = wl.length_schedule(cfg, args.warmup + args.steps + 1)
     n_q = 1
+    L = cfg.n_layers
+    t_cal, _ = oracle_sample_step(cfg, sched[0], n_q, 0)           # calibration: one full-model step
+    n = args.warmup + args.steps
+    L_s = L if n * t_cal <= REF_BUDGET_S else max(1, int(L * REF_BUDGET_S / (n * t_cal)))
     for i in range(args.warmup):
-        oracle_sample_step(cfg, sched[i], n_q, i)
-    tot_t, tot_s = 0.0, 0
+        oracle_sample_step(cfg, sched[1 + i], n_q, 1 + i, L_s)
+    tot_t, tot_s = 0.0, 0.0
     for i in range(args.steps):
-        t, s = oracle_sample_step(cfg, sched[args.warmup + i], n_q, args.warmup + i)
+        t, s_ = oracle_sample_step(cfg, sched[1 + args.warmup + i], n_q, 1 + args.warmup + i, L_s)
         tot_t += t
-        tot_s += s
+        tot_s += s_ * L_s / L
     v = tot_s / tot_t
-    sample = f"per step {n_q} questions of the {cfg.name} workload at the schedule's S_t (fp64 numpy)"
+    sample = (f"per step {n_q} question(s) of the {cfg.name} workload at the schedule's S_t through "
+              f"{L_s} of {L} encoder layers with a {L_s}/{L} word-embedding table (+ head, AdamW), counted as "
+              f"{L_s}/{L} of a sample; "
+              f"fp64 numpy; calibration full-model step {t_cal:.2f} s")
     line = {"impl": "reference", "metric": METRIC, "value": v, "unit": "samples/s", "n_gpus": args.gpus,
             "steps": args.steps, "warmup": args.warmup, "ms_per_step": 1000 * tot_t / args.steps,
             "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "f64",
