@@ -540,12 +540,22 @@ void wgrad(Run& r, const void* dY, int N, const void* X, int K, float* out) {
 
 // dW1 = dY1^T X1 and dW2 = dY2^T X2 (both deterministic, fp32 out): one grouped
 // tcgen05 launch with 128 x bn tiles when the two fit one wave of SMs (BERT-base:
-// the FFN pair 72 + 72 tiles at bn 256, the attention pair 36 + 108 at bn 128),
-// else two wgrad() calls.
+// the FFN pair 72 + 72 tiles at bn 256, the attention pair 36 + 108 at bn 128;
+// H = 1024: the attention pair 32 + 96 at bn 256), else two wgrad() calls.
 void wgrad2(Run& r, const void* dY1, int N1, const void* X1, int K1, float* out1, const void* dY2, int N2,
-            const void* X2, int K2, float* out2, int bn = 256) {
+            const void* X2, int K2, float* out2, int bn = 0) {
   mimose_ctx* c = r.c;
   const int T = c->T;
+  if (bn == 0) {
+    // tile width: the one whose single wave keeps more SMs busy, weighting a
+    // 128-wide tile at 0.58 of a 256-wide one (its measured mainloop rate);
+    // more tiles than SMs cannot be grouped (-> two launches)
+    auto tiles = [&](int w) {
+      return (K1 % w || K2 % w) ? 1 << 30 : ((N1 + 127) / 128) * (K1 / w) + ((N2 + 127) / 128) * (K2 / w);
+    };
+    const double e256 = tiles(256) <= 148 ? tiles(256) : 0.0, e128 = tiles(128) <= 148 ? 0.58 * tiles(128) : 0.0;
+    bn = e256 >= e128 ? 256 : 128;
+  }
   if (c->dt == DT_BF16 && c->cfg.use_tc && K1 % bn == 0 && K2 % bn == 0) {
     GemmArgs g[2];
     const void* dY[2] = {dY1, dY2};
@@ -656,7 +666,7 @@ void att_backward(Run& r, int l, const char* x, LayerBufs& b, float* dy, char* s
   dgrad(r, EPI_ACC_RES_F32, R3, 3 * H, W(c, LP(c, l, L_QKVW)), H, dy, dres);
   // dWo = dt1^T O and dWqkv = dQKV^T x; dbqkv = colsum dQKV
   if (spare)
-    wgrad2(r, DT1, H, b.O, H, G(c, LP(c, l, L_OW)), R3, 3 * H, x, H, G(c, LP(c, l, L_QKVW)), 128);
+    wgrad2(r, DT1, H, b.O, H, G(c, LP(c, l, L_OW)), R3, 3 * H, x, H, G(c, LP(c, l, L_QKVW)));
   else
     wgrad(r, R3, 3 * H, x, H, G(c, LP(c, l, L_QKVW)));
   colsum(c->dt, R3, T, 3 * H, c->part, r.st);
@@ -757,8 +767,10 @@ void ffn_backward_pre(Run& r, int l, LayerBufs& b, float* dy, char* scr) {
   wgrad(r, R2, F, b.m, H, G(c, LP(c, l, L_F1W)));
   colsum(c->dt, R2, T, F, c->part, r.st);
   reduce_partials(c->part, F, F, G(c, LP(c, l, L_F1B)), r.st);
-  // LN2 backward + residual: dr1 = dy + LN2'(dm) (in place in dy); dt1 = dr1 * mask (R3)
-  ln_bwd(c->dt, dres, no_drop(), b.r1, b.st2, W(c, LP(c, l, L_LN2G)), dy, R3, make_drop(c, KIND_ATTN_OUT, l),
+  // LN2 backward + residual: dr1 = dy + LN2'(dm) (in place in dy); dt1 = dr1 * mask (DT1: the
+  // spare tail of R2 when F >= 2H, so it outlives the dQKV write into R3, else R3)
+  char* DT1 = F >= 2 * H ? R2 + a16((int64_t)T * H * c->e) : R3;
+  ln_bwd(c->dt, dres, no_drop(), b.r1, b.st2, W(c, LP(c, l, L_LN2G)), dy, DT1, make_drop(c, KIND_ATTN_OUT, l),
          pg, pb, pbias, T, H, r.st, dy);
   reduce_rows3(pg, G(c, LP(c, l, L_LN2G)), pb, G(c, LP(c, l, L_LN2B)), pbias, G(c, LP(c, l, L_OB)), NPART, H, H,
                r.st);
@@ -775,14 +787,19 @@ void att_backward_pre(Run& r, int l, const float* x, LayerBufs& b, float* dy, ch
   float* Dbuf = (float*)(scr + r.z.r_dt + a16((int64_t)T * 3 * H * c->e));
   float* pg = c->part;
   float* pb = c->part + (int64_t)NPART * H;
-  // out-proj: dO = dt1 Wo (R2); dWo = dt1^T O
-  dgrad(r, EPI_STORE, R3, H, W(c, LP(c, l, L_OW)), H, R2, nullptr);
-  wgrad(r, R3, H, b.O, H, G(c, LP(c, l, L_OW)));
+  const bool spare = c->cfg.ffn >= 2 * H;          // dt1 in the spare tail of R2 (ffn_backward_pre)
+  char* DT1 = spare ? R2 + a16((int64_t)T * H * c->e) : R3;
+  // out-proj: dO = dt1 Wo (R2)
+  dgrad(r, EPI_STORE, DT1, H, W(c, LP(c, l, L_OW)), H, R2, nullptr);
+  if (!spare) wgrad(r, DT1, H, b.O, H, G(c, LP(c, l, L_OW)));
   attn_bwd(c->dt, b.qkv, b.O, R2, b.lse, c->lens, Dbuf, R3, c->B, c->S, H, h, make_drop(c, KIND_ATTN_PROBS, l),
            r.st, true);
-  // QKV: da = dQKV Wqkv (fp32, dres); dWqkv = dQKV^T a; dbqkv
+  // QKV: da = dQKV Wqkv (fp32, dres); dWo = dt1^T O with dWqkv = dQKV^T a (grouped); dbqkv
   dgrad(r, EPI_F32, R3, 3 * H, W(c, LP(c, l, L_QKVW)), H, dres, nullptr);
-  wgrad(r, R3, 3 * H, b.a, H, G(c, LP(c, l, L_QKVW)));
+  if (spare)
+    wgrad2(r, DT1, H, b.O, H, G(c, LP(c, l, L_OW)), R3, 3 * H, b.a, H, G(c, LP(c, l, L_QKVW)));
+  else
+    wgrad(r, R3, 3 * H, b.a, H, G(c, LP(c, l, L_QKVW)));
   colsum(c->dt, R3, T, 3 * H, c->part, r.st);
   reduce_partials(c->part, 3 * H, 3 * H, G(c, LP(c, l, L_QKVB)), r.st);
   // LN1 backward + residual: dx = dr1 + LN1'(da) (in place in dy)
