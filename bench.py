@@ -267,18 +267,21 @@ def main():
     M = max(C0 + int(cfg.budget_frac * (P0 - C0)), LB)
     probe_ctx.close()
 
-    nccl_id = None
-    if world > 1:
+    def fresh_nccl_id():
+        # one ncclUniqueId per communicator: every library context (one per arm)
+        # bootstraps its own, so rank 0 draws a new id and broadcasts it each time
+        if world == 1:
+            return None
         t = torch.zeros(128, dtype=torch.uint8, device="cuda")
         if rank == 0:
             t.copy_(torch.frombuffer(bytearray(mb.nccl_unique_id()), dtype=torch.uint8))
         dist.broadcast(t, 0)
-        nccl_id = bytes(t.cpu().numpy().tolist())
+        return bytes(t.cpu().numpy().tolist())
 
     def new_ctx(budget, slab_bytes, enforce=1, **kw):
         slab = torch.empty(slab_bytes, dtype=torch.uint8, device="cuda")
         ctx = mb.Mimose(cfg, budget, slab=slab, stream=stream, rank=rank, world=world,
-                        nccl_id=nccl_id, enforce_budget=enforce, use_tc=use_tc, **kw)
+                        nccl_id=fresh_nccl_id(), enforce_budget=enforce, use_tc=use_tc, **kw)
         ctx.set_params(wl.pack_params(cfg, wl.init_params(cfg)))
         # AdamW per gradient bucket on a side stream, overlapping the backward
         ctx.set_optimizer(1e-5, fused=True)
