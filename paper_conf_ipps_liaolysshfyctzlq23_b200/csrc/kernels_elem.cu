@@ -1162,8 +1162,13 @@ __global__ void __launch_bounds__(256) k_adamw(E* __restrict__ w, float* __restr
     *(float4*)(m + i) = make_float4(mm[0], mm[1], mm[2], mm[3]);
     *(float4*)(v + i) = make_float4(vv[0], vv[1], vv[2], vv[3]);
     if (master) *(float4*)(master + i) = make_float4(p[0], p[1], p[2], p[3]);
+    if constexpr (std::is_same<E, __nv_bfloat16>::value) {   // one 8-B store of the 4 bf16 weights
+      __nv_bfloat162 lo = __floats2bfloat162_rn(p[0], p[1]), hi = __floats2bfloat162_rn(p[2], p[3]);
+      *(uint2*)(w + i) = make_uint2(*(uint32_t*)&lo, *(uint32_t*)&hi);
+    } else {
 #pragma unroll
-    for (int k = 0; k < 4; ++k) stf(w + i + k, p[k]);
+      for (int k = 0; k < 4; ++k) stf(w + i + k, p[k]);
+    }
   }
 }
 
