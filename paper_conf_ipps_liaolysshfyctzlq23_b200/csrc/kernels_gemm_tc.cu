@@ -1346,11 +1346,15 @@ bool gemm_tc(Epi epi, const GemmArgs& g, cudaStream_t st) {
       return true;
     }
   }
-  // BN = 256 when N is a multiple of 256 and the 128x256 tiles still fill most
-  // of the 148 SMs; BN = 128 otherwise (measured per shape, tools/bench_gemm.py:
-  // BN = 64 loses on every step shape -- the per-tile fixed cost dominates).
+  // BN = 256 when N is a multiple of 256 and the 128x256 tiles fill at least half
+  // of the SMs; BN = 128 otherwise (measured per shape, tools/one_gemm.py; BN = 64
+  // loses on every step shape -- the per-tile fixed cost dominates).
   auto tiles = [&](int bn) { return m_blocks * ((g.N + bn - 1) / bn) * g.split; };
-  int BN = (g.N % 256 == 0 && tiles(256) >= 100) ? 256 : 128;
+  // 128-wide tiles run at ~0.58 of the 256-wide mainloop rate (half the work at
+  // ~1.15x the time): 256-wide wins as soon as its tiles occupy half the SMs
+  // (measured: T = 3584 x 768 x 3072 dropout-residual 29.1 us at 256 vs 39.5 at
+  // 128; T = 2560: 27.6 vs 23.8).
+  int BN = (g.N % 256 == 0 && 2 * tiles(256) >= num_sms()) ? 256 : 128;
   // Stream-K (split == 1, workspace given): cost model in 128 x 256 x 64
   // k-block times -- data-parallel = rounds x k-blocks per tile; stream-K =
   // the balanced share + ~4 blocks for the partial exchange; a 128-wide tile's
