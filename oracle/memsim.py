@@ -18,7 +18,17 @@ the GPU arena is an independent implementation of the same spec and must
 report the same integers.
 
 Pinned by: closed forms P(empty)=C+E+(L-1)a+i+Tb, LB, peak({L})=peak(empty),
-peak(first k)=P(empty)-k*i, monotonicity in x (tests/test_oracle_planning.py).
+peak(first k)=P(empty)-k*i, monotonicity in x (tests/test_oracle_planning.py);
+the event-list closed forms of both layer types incl. GPT-2's LM-head event,
+and C written from DESIGN.md §3 with the parameter count pinned to HF
+transformers' own model classes (tests/test_oracle_pins.py).
+
+Allocation-spec constants.  The byte sizes below name allocation choices of
+the DESIGN.md §3 spec that the product's arena also follows: NPART reduction
+partials, the 4H^2 fp32 split-K workspace, the radix-sort digit histograms
+(256 x int32 per 1024-token tile) and LM_CHUNK tokens per LM-head chunk.
+They define WHICH buffers a step allocates, not any arithmetic; a change to
+one of them is a change of DESIGN.md §3 and its commit cites that passage.
 """
 from __future__ import annotations
 

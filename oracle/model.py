@@ -405,9 +405,3 @@ def adamw(params, grads, m, v, t, lr, beta1=0.9, beta2=0.999, eps=1e-8, wd=0.0):
         out_p[k] = pk - (lr / bc1) * mk / denom
         out_m[k], out_v[k] = mk, vk
     return out_p, out_m, out_v
-
-
-def dp_mean_grads(grads_per_rank):
-    """Data-parallel semantics (c-J): gradient = mean over ranks."""
-    n = len(grads_per_rank)
-    return {k: sum(g[k] for g in grads_per_rank) / n for k in grads_per_rank[0]}

@@ -25,7 +25,8 @@ Readings (DESIGN.md register, numbered as SURVEY §8(c)-R):
 All byte arithmetic is in Python integers.
 
 Pinned by: hand traces (tests/golden/alg1_traces.txt), brute force over all
-subsets on <=10-layer stacks, budget property tests.  Optimality on
+subsets on <=10-layer stacks evaluated with the event simulator
+(brute_force_sim; tests/test_oracle_pins.py), budget property tests.  Optimality on
 heterogeneous stacks is "parity unpinned" (the paper claims near-optimal only).
 """
 from __future__ import annotations
@@ -153,6 +154,25 @@ def brute_force(p: Dict, budget: int, cost: Sequence[float], reserve: int = 0):
     for k in range(L + 1):
         for sub in itertools.combinations(range(L), k):
             pk = predicted_peak(p, sub)
+            if pk > budget - reserve:
+                continue
+            key = (sum(cost[l] for l in sub), pk, sub)
+            if best is None or key < best:
+                best = key
+    if best is None:
+        return INFEASIBLE, None, None
+    return OK, list(best[2]), best[1]
+
+
+def brute_force_sim(peak_of, n_units: int, budget: int, cost: Sequence[float], reserve: int = 0):
+    """SURVEY c-G's brute-force pin: all 2^n drop sets evaluated with the EVENT
+    SIMULATOR (``peak_of(dropped)``, e.g. memsim.simulate_step on the true
+    Sizes), not with the planner's own predicted-peak formula.  Feasible with
+    minimum sum(cost), then minimum peak, then lexicographically smallest."""
+    best = None
+    for k in range(n_units + 1):
+        for sub in itertools.combinations(range(n_units), k):
+            pk = peak_of(sub)
             if pk > budget - reserve:
                 continue
             key = (sum(cost[l] for l in sub), pk, sub)

@@ -35,8 +35,9 @@ def sources():
 
 
 def headers():
-    return sorted(glob.glob(os.path.join(CSRC, "**", "*.h"), recursive=True) +
-                  [os.path.join(ROOT, "include", "mimose.h")])
+    pats = ("*.h", "*.cuh", "*.hpp")
+    return sorted([f for p in pats for f in glob.glob(os.path.join(CSRC, "**", p), recursive=True)] +
+                  glob.glob(os.path.join(ROOT, "include", "*.h")))
 
 
 def compile_one(src: str, nccl: str, verbose: bool) -> str:
