@@ -102,7 +102,17 @@ typedef struct {
                             u, g; output y), so 2L <= 64 units (SURVEY f1, P:125/P:140
                             "attention block"; reading A30).  Samples, series and drop
                             masks are then indexed by unit.                              */
-  int32_t reserved[5];
+  int32_t comm_force;    /* 1: create the NCCL communicator (and run the per-bucket
+                            ncclAllReduce, the loss all-reduce and the plan check) even
+                            at world == 1 (a 1-rank communicator; test / single-GPU
+                            evidence of the a10 path).  0: only when world > 1        */
+  int32_t nccl_max_ctas; /* NCCL CTA cap (ncclConfig_t.maxCTAs): 0 = 16 (default),
+                            < 0 = NCCL's own default                                   */
+  int32_t check_plans;   /* 1: every mimose_forward all-gathers a 64-bit hash of
+                            (x, drop mask, predicted peak) over the communicator and
+                            fails with MIMOSE_E_STATE if any rank differs (
+                            debug: one small device->host sync per step)               */
+  int32_t reserved[2];
 } mimose_config;
 
 /* Fill defaults (collect_iters 10, ratio 9/10, degree 2, p 0.1, eps 1e-12,
@@ -169,6 +179,11 @@ typedef struct {
   double planner_us_total;             /* host time in estimator+planner on misses     */
   double collector_ms_total;           /* host wall time of shuttled collect calls     */
   int64_t kernel_launches;             /* our kernels launched since init              */
+  int64_t allreduce_calls;             /* ncclAllReduce of gradient buckets issued      */
+  int64_t allreduce_bytes;             /* their fp32 bytes                             */
+  int64_t plan_checks;                 /* cross-rank plan-hash checks passed (X4)      */
+  int32_t comm_nranks;                 /* communicator size (0: no communicator)       */
+  int32_t pad_;
 } mimose_stats;
 
 mimose_status mimose_init(const mimose_config* cfg, mimose_ctx** out);
@@ -184,6 +199,8 @@ mimose_status mimose_num_params(const mimose_ctx* ctx, int64_t* n);
 mimose_status mimose_set_params(mimose_ctx* ctx, const float* host_blob, int64_t n);
 /* Reads the working copy (bf16 mode: bf16 values widened to fp32). */
 mimose_status mimose_get_params(mimose_ctx* ctx, float* host_blob, int64_t n);
+/* Reads the fp32 master copy AdamW updates (bf16 mode; fp32 mode: the weights). */
+mimose_status mimose_get_master(mimose_ctx* ctx, float* host_blob, int64_t n);
 /* fp32 gradients of the last backward (after the DP all-reduce, before the
    1/world scale), same order.  Test hook; synchronises the stream. */
 mimose_status mimose_get_grads(mimose_ctx* ctx, float* host_blob, int64_t n);

@@ -45,7 +45,8 @@ class Config(C.Structure):
                 ("arena_base", C.c_void_p), ("arena_bytes", C.c_int64), ("stream", C.c_void_p),
                 ("rank", C.c_int32), ("world", C.c_int32), ("nccl_id", C.c_void_p),
                 ("use_tc", C.c_int32), ("pad_id", C.c_int32), ("granularity", C.c_int32),
-                ("reserved", C.c_int32 * 5)]
+                ("comm_force", C.c_int32), ("nccl_max_ctas", C.c_int32), ("check_plans", C.c_int32),
+                ("reserved", C.c_int32 * 2)]
 
 
 class BatchS(C.Structure):
@@ -78,7 +79,9 @@ class Stats(C.Structure):
                 ("n_samples", C.c_int64), ("phase", C.c_int32), ("last_n_dropped", C.c_int32),
                 ("last_drop_mask", C.c_uint64), ("last_predicted_peak", C.c_int64),
                 ("planner_us_total", C.c_double), ("collector_ms_total", C.c_double),
-                ("kernel_launches", C.c_int64)]
+                ("kernel_launches", C.c_int64), ("allreduce_calls", C.c_int64),
+                ("allreduce_bytes", C.c_int64), ("plan_checks", C.c_int64),
+                ("comm_nranks", C.c_int32), ("pad_", C.c_int32)]
 
     def asdict(self) -> Dict:
         return {k: getattr(self, k) for k, _ in self._fields_}
@@ -97,7 +100,7 @@ _lib.mimose_destroy.argtypes = [_P]
 _lib.mimose_last_error.argtypes = [_P]
 _lib.mimose_last_error.restype = C.c_char_p
 _lib.mimose_num_params.argtypes = [_P, C.POINTER(C.c_int64)]
-for _n in ("mimose_set_params", "mimose_get_params", "mimose_get_grads"):
+for _n in ("mimose_set_params", "mimose_get_params", "mimose_get_grads", "mimose_get_master"):
     getattr(_lib, _n).argtypes = [_P, _P, C.c_int64]
 _lib.mimose_collect.argtypes = [_P, C.POINTER(BatchS), C.POINTER(C.c_float)]
 _lib.mimose_plan.argtypes = [_P, C.c_int64, C.POINTER(Plan)]
@@ -128,7 +131,7 @@ EXPORTED = ["mimose_default_config", "mimose_init", "mimose_destroy", "mimose_la
             "mimose_step", "mimose_get_stats", "mimose_phase", "mimose_get_sample", "mimose_dry_run",
             "mimose_dry_collect", "mimose_predicted_peak", "mimose_plan_series", "mimose_fit_predict",
             "mimose_nccl_unique_id", "mimose_probe", "mimose_probe_read", "mimose_set_optimizer",
-            "mimose_set_planner"]
+            "mimose_set_planner", "mimose_get_master"]
 
 
 _lib.mimose_tc_available.restype = C.c_int32
@@ -279,6 +282,11 @@ class Mimose:
     def get_params(self) -> np.ndarray:
         b = np.empty(self.n_params, np.float32)
         self._chk(_lib.mimose_get_params(self.h, b.ctypes.data, b.size))
+        return b
+
+    def get_master(self) -> np.ndarray:
+        b = np.empty(self.n_params, np.float32)
+        self._chk(_lib.mimose_get_master(self.h, b.ctypes.data, b.size))
         return b
 
     def get_grads(self) -> np.ndarray:

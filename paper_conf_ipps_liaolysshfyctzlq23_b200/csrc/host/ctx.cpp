@@ -188,6 +188,9 @@ struct mimose_ctx {
   int B = 0, S = 0, T = 0;
   uint64_t drop_mask = 0;
   bool fwd_done = false, bwd_done = false, collecting = false;
+  bool step_pending = false;   // fused optimizer: backward applied the update, mimose_step not yet called
+  int64_t stats_allreduce_calls = 0, stats_allreduce_bytes = 0;
+  int64_t stats_plan_checks = 0;
   float* z0 = nullptr;
   char* x1 = nullptr;
   float2* st0 = nullptr;
@@ -877,11 +880,13 @@ int64_t bucket_end(mimose_ctx* c, int last_param) {
 // comm stream and, with the fused optimizer, update it on the optimizer stream,
 // both overlapping the rest of the backward.
 mimose_status allreduce_bucket(mimose_ctx* c, int first, int last, int evi) {
-  if (!c->device || (c->cfg.world <= 1 && !c->opt_fused)) return MIMOSE_OK;
+  if (!c->device || (!c->comm && !c->opt_fused)) return MIMOSE_OK;
   const int64_t b0 = bucket_begin(c, first), b1 = bucket_end(c, last);
   CK(cudaEventRecord(c->ev_layer[evi], c->st));
   cudaEvent_t ready = c->ev_layer[evi];
-  if (c->cfg.world > 1) {
+  if (c->comm) {
+    c->stats_allreduce_calls++;
+    c->stats_allreduce_bytes += (b1 - b0) * 4;
     CK(cudaStreamWaitEvent(c->comm_st, c->ev_layer[evi], 0));
     NK(ncclAllReduce(c->grad + b0, c->grad + b0, (size_t)(b1 - b0), ncclFloat, ncclSum, c->comm, c->comm_st));
     CK(cudaEventRecord(c->ev_ar[evi], c->comm_st));
@@ -1220,6 +1225,7 @@ void dry_step(mimose_ctx* c, int B, int S, uint64_t mask, bool collect, int64_t*
   char *sx1 = c->x1, *shp = c->hp;
   float2* sst0 = c->st0;
   float* slog = c->logits;
+  float2 *slst = c->lm_stf, *sltk = c->lm_tok;
   std::vector<LayerBufs> slb = c->lb;
   std::vector<char*> sy = c->y;
   c->B = B; c->S = S; c->T = B * S;
@@ -1234,6 +1240,7 @@ void dry_step(mimose_ctx* c, int B, int S, uint64_t mask, bool collect, int64_t*
   c->ar = saved;
   c->B = sB; c->S = sS; c->T = sT; c->drop_mask = sm;
   c->z0 = sz0; c->x1 = sx1; c->hp = shp; c->st0 = sst0; c->logits = slog;
+  c->lm_stf = slst; c->lm_tok = sltk;
   c->lb = slb; c->y = sy;
 }
 
@@ -1258,7 +1265,12 @@ void resolve_times(mimose_ctx* c) {
 mimose_status read_loss(mimose_ctx* c, float* loss_out) {
   if (!loss_out) return MIMOSE_OK;
   if (!c->device) { *loss_out = 0.f; return MIMOSE_OK; }
-  CK(cudaMemcpyAsync(loss_out, c->misc, 4, cudaMemcpyDeviceToHost, c->st));
+  const float* src = c->misc;
+  if (c->comm) {   // the scalar loss is all-reduced (mean over ranks) for logging
+    NK(ncclAllReduce(c->misc, c->misc + 1, 1, ncclFloat, ncclAvg, c->comm, c->st));
+    src = c->misc + 1;
+  }
+  CK(cudaMemcpyAsync(loss_out, src, 4, cudaMemcpyDeviceToHost, c->st));
   CK(cudaStreamSynchronize(c->st));
   return MIMOSE_OK;
 }
@@ -1389,14 +1401,21 @@ mimose_status mimose_init(const mimose_config* cfgp, mimose_ctx** out) {
     for (auto& e : c->ev_ar) CK(cudaEventCreateWithFlags(&e, cudaEventDisableTiming));
     CK(cudaStreamCreateWithFlags(&c->opt_st, cudaStreamNonBlocking));
     CK(cudaEventCreateWithFlags(&c->ev_opt_done, cudaEventDisableTiming));
-    if (k.world > 1) {
-      if (!k.nccl_id) { *out = c; return bad("world > 1 needs nccl_id"); }
+    if (k.world > 1 || k.comm_force) {
+      if (k.world > 1 && !k.nccl_id) { *out = c; return bad("world > 1 needs nccl_id"); }
       int lo, hi;
       CK(cudaDeviceGetStreamPriorityRange(&lo, &hi));
       CK(cudaStreamCreateWithPriority(&c->comm_st, cudaStreamNonBlocking, hi));
       ncclUniqueId id;
-      std::memcpy(&id, k.nccl_id, sizeof(id));
-      NK(ncclCommInitRank(&c->comm, k.world, id, k.rank));
+      if (k.nccl_id) std::memcpy(&id, k.nccl_id, sizeof(id));
+      else NK(ncclGetUniqueId(&id));                // world == 1 with comm_force: own 1-rank communicator
+      // Cap NCCL's CTAs: its kernels run on the comm stream next to the
+      // persistent GEMMs (grid = SM count) and the fused AdamW; the GEMMs'
+      // CTAs never wait on each other, so a cap only trades bandwidth for SMs.
+      ncclConfig_t nc = NCCL_CONFIG_INITIALIZER;
+      const int cap = k.nccl_max_ctas < 0 ? 0 : (k.nccl_max_ctas == 0 ? 16 : k.nccl_max_ctas);
+      if (cap > 0) { nc.maxCTAs = cap; nc.minCTAs = std::min(cap, 4); }
+      NK(ncclCommInitRankConfig(&c->comm, k.world, id, k.rank, &nc));
       CK(cudaEventCreateWithFlags(&c->ev_comm_done, cudaEventDisableTiming));
     }
   }
@@ -1451,7 +1470,8 @@ static mimose_status xfer_params(mimose_ctx* c, float* host, int64_t n, int whic
     CK(cudaMemsetAsync(c->v, 0, (size_t)c->npad * 4, c->st));
     c->adam_t = 0;
   } else {
-    if (which == 1) cast_to_f32(c->dt, c->w, tmp, c->npad, c->st);
+    if (which == 1 || (which == 3 && !c->master)) cast_to_f32(c->dt, c->w, tmp, c->npad, c->st);
+    else if (which == 3) CK(cudaMemcpyAsync(tmp, c->master, (size_t)c->npad * 4, cudaMemcpyDeviceToDevice, c->st));
     else CK(cudaMemcpyAsync(tmp, c->grad, (size_t)c->npad * 4, cudaMemcpyDeviceToDevice, c->st));
     CK(cudaMemcpyAsync(img.data(), tmp, (size_t)c->npad * 4, cudaMemcpyDeviceToHost, c->st));
   }
@@ -1467,9 +1487,33 @@ static mimose_status xfer_params(mimose_ctx* c, float* host, int64_t n, int whic
 
 mimose_status mimose_set_params(mimose_ctx* c, const float* h, int64_t n) { return xfer_params(c, (float*)h, n, 0); }
 mimose_status mimose_get_params(mimose_ctx* c, float* h, int64_t n) { return xfer_params(c, h, n, 1); }
+mimose_status mimose_get_master(mimose_ctx* c, float* h, int64_t n) { return xfer_params(c, h, n, 3); }
 mimose_status mimose_get_grads(mimose_ctx* c, float* h, int64_t n) {
   if (c && c->device && c->comm_st) cudaStreamSynchronize(c->comm_st);
   return xfer_params(c, h, n, 2);
+}
+
+// every rank must run the same plan for the same x (the
+// plan is derived, never broadcast).  All-gather a 64-bit FNV-1a hash of
+// (x, drop mask, peak) and compare; one 8-B-per-rank exchange + a host sync.
+static mimose_status check_plan_consistency(mimose_ctx* c, int64_t x, uint64_t mask, int64_t peak) {
+  uint64_t h = 1469598103934665603ull;
+  for (uint64_t v : {(uint64_t)x, mask, (uint64_t)peak})
+    for (int i = 0; i < 8; ++i) { h ^= (v >> (8 * i)) & 0xff; h *= 1099511628211ull; }
+  int n = 1;
+  NK(ncclCommCount(c->comm, &n));
+  if (n > 15) return MIMOSE_OK;                             // misc[32..63] holds 16 hash words
+  uint64_t* dev = (uint64_t*)(c->misc + 32);                // [0] own hash, [1..n] the gather
+  uint64_t* gat = dev + 1;
+  CK(cudaMemcpyAsync(dev, &h, 8, cudaMemcpyHostToDevice, c->st));
+  NK(ncclAllGather(dev, gat, 1, ncclUint64, c->comm, c->st));
+  uint64_t got[16];
+  CK(cudaMemcpyAsync(got, gat, 8 * (size_t)n, cudaMemcpyDeviceToHost, c->st));
+  CK(cudaStreamSynchronize(c->st));
+  for (int r = 0; r < n; ++r)
+    if (got[r] != h) return fail(c, MIMOSE_E_STATE, "plan mismatch across ranks (rank " + std::to_string(r) + ")");
+  c->stats_plan_checks++;
+  return MIMOSE_OK;
 }
 
 static mimose_status begin_step(mimose_ctx* c, const mimose_batch* bt, uint64_t mask, bool collect, Sample* smp) {
@@ -1482,6 +1526,10 @@ static mimose_status begin_step(mimose_ctx* c, const mimose_batch* bt, uint64_t 
     c->stats.violations++;
     return fail(c, MIMOSE_E_BUDGET, "step would exceed the budget (predicted " + std::to_string(peak) +
                                         " B > M = " + std::to_string(c->ar.budget) + ")");
+  }
+  if (c->comm && c->cfg.check_plans) {
+    if (mimose_status s = check_plan_consistency(c, (int64_t)bt->n_seqs * bt->seq_len, collect ? ~0ull : mask, peak))
+      return s;
   }
   c->B = bt->n_seqs; c->S = bt->seq_len; c->T = c->B * c->S;
   c->drop_mask = collect ? ~0ull : mask;
@@ -1501,6 +1549,7 @@ mimose_status mimose_collect(mimose_ctx* c, const mimose_batch* bt, float* loss_
   if (mimose_status s = check_ready(c)) return s;
   if (c->phase != MIMOSE_PHASE_SHELTERED) return fail(c, MIMOSE_E_STATE, "collect after the sheltered phase");
   if (c->fwd_done && !c->bwd_done) return fail(c, MIMOSE_E_STATE, "forward pending its backward");
+  if (c->step_pending) return fail(c, MIMOSE_E_STATE, "fused optimizer: mimose_step must close the previous step");
   resolve_times(c);
   const int64_t x = bt ? (int64_t)bt->n_seqs * bt->seq_len : 0;
   const bool unseen = std::find(c->seen_x.begin(), c->seen_x.end(), x) == c->seen_x.end();
@@ -1529,6 +1578,7 @@ mimose_status mimose_collect(mimose_ctx* c, const mimose_batch* bt, float* loss_
 mimose_status mimose_forward(mimose_ctx* c, const mimose_batch* bt, const mimose_plan_t* plan, float* loss_out) {
   if (mimose_status s = check_ready(c)) return s;
   if (c->fwd_done && !c->bwd_done) return fail(c, MIMOSE_E_STATE, "forward pending its backward");
+  if (c->step_pending) return fail(c, MIMOSE_E_STATE, "fused optimizer: mimose_step must close the previous step");
   resolve_times(c);
   c->collecting = false;
   const uint64_t mask = plan ? plan->drop_mask : 0;
@@ -1543,6 +1593,7 @@ mimose_status mimose_backward(mimose_ctx* c) {
   Sample* smp = c->collecting ? &c->samples.back() : nullptr;
   if (mimose_status s = run_backward(r, smp)) return s;
   c->bwd_done = true;
+  c->step_pending = c->device && c->opt_fused;   // the per-bucket updates are already applied
   c->stats.peak_bytes = c->ar.peak;
   c->stats.max_peak_bytes = std::max(c->stats.max_peak_bytes, c->ar.peak);
   c->stats.steps++;
@@ -1575,15 +1626,20 @@ mimose_status mimose_step(mimose_ctx* c, float lr, float b1, float b2, float eps
   if (!c->bwd_done) return fail(c, MIMOSE_E_STATE, "step without a backward");
   if (!c->device) return MIMOSE_OK;
   if (c->opt_fused) {   // the per-bucket updates were launched during backward
-    if (lr != c->opt_lr || b1 != c->opt_b1 || b2 != c->opt_b2 || eps != c->opt_eps || wd != c->opt_wd)
-      return fail(c, MIMOSE_E_INVALID, "fused optimizer: step arguments differ from mimose_set_optimizer");
+    // The update has been applied with the mimose_set_optimizer arguments:
+    // order the compute stream behind it and advance t whatever this call's
+    // arguments say, then report a mismatch.
     CK(cudaEventRecord(c->ev_opt_done, c->opt_st));
     CK(cudaStreamWaitEvent(c->st, c->ev_opt_done, 0));
     c->adam_t++;
     c->fwd_done = false;
+    c->step_pending = false;
+    if (lr != c->opt_lr || b1 != c->opt_b1 || b2 != c->opt_b2 || eps != c->opt_eps || wd != c->opt_wd)
+      return fail(c, MIMOSE_E_INVALID,
+                  "fused optimizer: step arguments differ from mimose_set_optimizer (the update used the latter)");
     return MIMOSE_OK;
   }
-  if (c->cfg.world > 1) {
+  if (c->comm) {
     CK(cudaEventRecord(c->ev_comm_done, c->comm_st));
     CK(cudaStreamWaitEvent(c->st, c->ev_comm_done, 0));
   }
@@ -1600,6 +1656,7 @@ mimose_status mimose_step(mimose_ctx* c, float lr, float b1, float b2, float eps
 mimose_status mimose_set_optimizer(mimose_ctx* c, float lr, float b1, float b2, float eps, float wd, int32_t fused) {
   if (mimose_status s = check_ready(c)) return s;
   if (c->fwd_done && !c->bwd_done) return fail(c, MIMOSE_E_STATE, "set_optimizer inside a step");
+  if (c->step_pending) return fail(c, MIMOSE_E_STATE, "set_optimizer before mimose_step closed the step");
   c->opt_fused = fused != 0;
   c->opt_lr = lr; c->opt_b1 = b1; c->opt_b2 = b2; c->opt_eps = eps; c->opt_wd = wd;
   return MIMOSE_OK;
@@ -1763,6 +1820,14 @@ mimose_status mimose_get_stats(const mimose_ctx* c, mimose_stats* out) {
   out->live_bytes = c->ar.live();
   out->phase = c->phase;
   out->kernel_launches = kernel_launch_count();
+  out->allreduce_calls = c->stats_allreduce_calls;
+  out->allreduce_bytes = c->stats_allreduce_bytes;
+  out->plan_checks = c->stats_plan_checks;
+  out->comm_nranks = 0;
+  if (c->comm) {
+    int n = 0;
+    if (ncclCommCount(c->comm, &n) == ncclSuccess) out->comm_nranks = n;
+  }
   return MIMOSE_OK;
 }
 

@@ -1,0 +1,78 @@
+"""TEST INFRASTRUCTURE: SURVEY c-K's parity metric for the GPU-vs-oracle tests.
+
+* metric: per-tensor normwise inf-norm error  max|g - g_ref| / max|g_ref|,
+  over the loss and every gradient tensor;
+* bound: 2e-2 (bf16) / 1e-4 (fp32).  A bf16 tensor may exceed 2e-2 only where
+  the bf16-storage emulation (tests/bf16_emulation.py: the fp64 oracle with
+  exactly the CUDA path's bf16 storage points rounded) shows the excess is
+  inherent: then the bound is 1.5x the emulated error of that tensor.  The
+  relative 2-norm error stays <= 2e-2 for every tensor regardless;
+* provably zero tensors (no relative error exists): the MC classifier bias
+  (CE over a question's choices is shift invariant), the QA bias and the last
+  layer's LN2 shift (the start/end CE gradients sum to zero over positions,
+  and every token's dy is dlogits W_qa) -- their absolute value must be
+  fp32 round-off: <= 1e-6 of the largest gradient.
+Every check writes its per-tensor table to gpurun_out/parity/<name>.json.
+"""
+from __future__ import annotations
+
+import json
+import os
+
+import numpy as np
+
+from paper_conf_ipps_liaolysshfyctzlq23_b200 import workload as wl
+
+TOL = {"fp32": 1e-4, "bf16": 2e-2}
+EMU_FACTOR = 1.5
+
+
+def zero_tensors(cfg):
+    if cfg.head == wl.HEAD_MC:
+        return {"cls.b"}
+    if cfg.head == wl.HEAD_QA:
+        return {"qa.b", f"layer{cfg.n_layers - 1}.ln2.b"}
+    return set()
+
+
+def inf_err(a, b):
+    a, b = np.asarray(a, np.float64), np.asarray(b, np.float64)
+    return float(np.abs(a - b).max() / max(float(np.abs(b).max()), 1e-300))
+
+
+def rel2_err(a, b):
+    a, b = np.asarray(a, np.float64), np.asarray(b, np.float64)
+    return float(np.linalg.norm(a - b) / max(float(np.linalg.norm(b)), 1e-300))
+
+
+def check(name, cfg, gd, G, loss, ref_loss, emulate=None):
+    """Assert c-K parity; ``emulate()`` -> (loss, grads) of the bf16-storage
+    emulation on the same inputs (called only if some tensor exceeds 2e-2)."""
+    tol = TOL[cfg.dtype]
+    zeros = zero_tensors(cfg)
+    gmax = max(float(np.abs(v).max()) for v in G.values())
+    rows = {k: dict(name=k, inf=inf_err(gd[k], G[k]), rel2=rel2_err(gd[k], G[k]),
+                    max_ref=float(np.abs(G[k]).max()), zero=k in zeros) for k in G}
+    over = [k for k, r in rows.items() if not r["zero"] and r["inf"] > tol]
+    emu = None
+    if over and cfg.dtype == "bf16" and emulate is not None:
+        _, E = emulate()
+        emu = {k: inf_err(E[k], G[k]) for k in over}
+        for k in over:
+            rows[k]["emulated_inf"] = emu[k]
+    rec = dict(case=name, dtype=cfg.dtype, hidden=cfg.hidden, n_layers=cfg.n_layers, loss=loss,
+               ref_loss=ref_loss, loss_rel=abs(loss - ref_loss) / max(1.0, abs(ref_loss)),
+               grads=sorted(rows.values(), key=lambda r: -r["inf"] if not r["zero"] else 0))
+    out = os.path.join(os.environ.get("GRAFT_REPO_ROOT", os.getcwd()), "gpurun_out", "parity")
+    os.makedirs(out, exist_ok=True)
+    with open(os.path.join(out, name + ".json"), "w") as f:
+        json.dump(rec, f, indent=1)
+    assert rec["loss_rel"] <= tol, (name, loss, ref_loss)
+    for k, r in rows.items():
+        if r["zero"]:
+            assert float(np.abs(gd[k]).max()) <= 1e-6 * gmax, (name, k)
+            continue
+        assert r["rel2"] <= tol, (name, k, r)
+        bound = tol if emu is None or k not in emu else max(tol, EMU_FACTOR * emu[k])
+        assert r["inf"] <= bound, (name, k, r, "emulated", None if emu is None else emu.get(k))
+    return rec

@@ -20,29 +20,17 @@ from oracle import model as omodel
 from oracle import planner as op
 from paper_conf_ipps_liaolysshfyctzlq23_b200 import workload as wl
 
+import parity_metrics as pm
+
 
 def mb():
     from paper_conf_ipps_liaolysshfyctzlq23_b200 import binding
     return binding
 
 
-def normwise(a, b, floor=1e-6):
-    """inf-norm relative error max|a-b| / max|b| (floor for identically-zero b)."""
-    a, b = np.asarray(a, np.float64), np.asarray(b, np.float64)
-    return float(np.abs(a - b).max() / max(float(np.abs(b).max()), floor))
-
-
-def rel2(a, b, floor=1e-6):
-    """2-norm relative error ||a-b|| / ||b|| (DESIGN reading R-T)."""
-    a, b = np.asarray(a, np.float64), np.asarray(b, np.float64)
-    return float(np.linalg.norm(a - b) / max(float(np.linalg.norm(b)), floor))
-
-
-# DESIGN reading R-T: "max relative error 2e-2 (bf16) / 1e-4 (fp32)" = the largest
-# per-tensor relative 2-norm error over the loss and every gradient tensor; the
-# inf-norm is bounded too (bf16: 5e-2, fp32: 1e-4).
-TOL2 = {"fp32": 1e-4, "bf16": 2e-2}
-TOLINF = {"fp32": 1e-4, "bf16": 5e-2}
+# DESIGN reading R-T / SURVEY c-K: tests/parity_metrics.py (inf-norm normwise
+# per tensor <= 2e-2 bf16 / 1e-4 fp32; excess only where the bf16-storage
+# emulation shows it is inherent; provably zero tensors at fp32 round-off).
 
 
 def make_ctx(cfg, budget=None, extra=0, **kw):
@@ -117,10 +105,18 @@ CASES = {
 }
 
 
+def emulator(cfg, W, b, it):
+    """bf16-storage emulation of the same step (post-LN bf16 only), lazily."""
+    if cfg.dtype != "bf16" or cfg.arch != wl.ARCH_POST_LN:
+        return None
+    import bf16_emulation as be
+    return lambda: be.train_step_grads(cfg, W, b, wl.dropout_seed(cfg), it)
+
+
 @pytest.mark.parametrize("case", list(CASES))
 def test_step_parity_against_oracle(case):
+    """c-K: loss and every gradient against the fp64 oracle (parity_metrics)."""
     cfg = CASES[case]
-    tol, tolinf = TOL2[cfg.dtype], TOLINF[cfg.dtype]
     params = wl.init_params(cfg, parity=True, seed=11)
     ctx = make_ctx(cfg)
     ctx.set_params(wl.pack_params(cfg, params))
@@ -130,15 +126,7 @@ def test_step_parity_against_oracle(case):
         loss, g = run_step(ctx, cfg, b)
         it = ctx.stats()["steps"]          # the library's dropout step counter == forward calls
         ref_loss, G = omodel.train_step_grads(cfg, W, b, wl.dropout_seed(cfg), it)
-        assert abs(loss - ref_loss) <= tol * max(1.0, abs(ref_loss)), (loss, ref_loss)
-        gd = grads_dict(cfg, g)
-        # floor: 1e-3 of the largest gradient, so mathematically-zero tensors (the MC
-        # classifier bias: CE over choices is shift invariant) compare round-off to scale
-        floor = 1e-3 * max(float(np.abs(v).max()) for v in G.values())
-        floor2 = 1e-3 * max(float(np.linalg.norm(v)) for v in G.values())
-        for k in G:
-            assert rel2(gd[k], G[k], floor2) <= tol, (case, k, rel2(gd[k], G[k], floor2))
-            assert normwise(gd[k], G[k], floor) <= tolinf, (case, k, normwise(gd[k], G[k], floor))
+        pm.check(f"{case}-step{step}", cfg, grads_dict(cfg, g), G, loss, ref_loss, emulator(cfg, W, b, it))
 
 
 @pytest.mark.parametrize("case", ["toy-fp32", "mc-bf16", "qa-bf16", "lm-gpt2-bf16", "lm-gpt2-bf16-long"])
@@ -213,6 +201,37 @@ def test_adamw_step_against_oracle():
         assert np.abs(got[k] - newP[k]).max() <= 1e-6, k
 
 
+@pytest.mark.parametrize("fused", [False, True])
+def test_bf16_adamw_against_oracle(fused):
+    """bf16 mode: AdamW updates the fp32 master copy from the
+    fp32 gradients as the fp64 oracle's AdamW (c-I) does, to fp32 rounding, over
+    two steps (bias correction t = 1, 2, weight decay on), and the bf16 working
+    copy is the round-to-nearest-even of the master."""
+    cfg = CASES["mc-bf16"]
+    params = wl.init_params(cfg, parity=True, seed=6)
+    ctx = make_ctx(cfg)
+    ctx.set_params(wl.pack_params(cfg, params))
+    if fused:
+        ctx.set_optimizer(lr=1e-3, wd=0.01, fused=True)
+    P = {k: v.astype(np.float64) for k, v in params.items()}
+    m = {k: np.zeros_like(v) for k, v in P.items()}
+    v = {k: np.zeros_like(x) for k, x in P.items()}
+    for t in (1, 2):
+        b = wl.make_batch(cfg, 30 + t, seed=70 + t)
+        _, g = run_step(ctx, cfg, b)
+        ctx.step(lr=1e-3, beta1=0.9, beta2=0.999, eps=1e-8, wd=0.01)
+        torch.cuda.synchronize()
+        G = grads_dict(cfg, g.astype(np.float64))
+        P, m, v = omodel.adamw(P, G, m, v, t, 1e-3, wd=0.01)
+        master = grads_dict(cfg, ctx.get_master())
+        for k in P:
+            assert np.abs(master[k] - P[k]).max() <= 2e-6 * max(1.0, np.abs(P[k]).max()), (t, k)
+        work = ctx.get_params()
+        want = torch.tensor(ctx.get_master()).bfloat16().float().numpy()
+        assert np.array_equal(work, want)
+    ctx.close()
+
+
 @pytest.mark.parametrize("case", ["mc-bf16", "lm-gpt2-bf16"])
 def test_fused_optimizer_bitwise_equal(case):
     """Per-bucket AdamW on the side stream during backward == one AdamW after it."""
@@ -277,12 +296,9 @@ def test_units_step_parity_against_oracle():
     ctx.set_params(wl.pack_params(cfg, params))
     b = wl.make_batch(cfg, cfg.seq_hi, seed=100)
     loss, g = run_step(ctx, cfg, b, [0, 3, 4])
-    ref_loss, G = omodel.train_step_grads(cfg, W, b, wl.dropout_seed(cfg), ctx.stats()["steps"])
-    assert abs(loss - ref_loss) <= TOL2["bf16"] * max(1.0, abs(ref_loss))
-    gd = grads_dict(cfg, g)
-    floor2 = 1e-3 * max(float(np.linalg.norm(v)) for v in G.values())
-    for k in G:
-        assert rel2(gd[k], G[k], floor2) <= TOL2["bf16"], (k, rel2(gd[k], G[k], floor2))
+    it = ctx.stats()["steps"]
+    ref_loss, G = omodel.train_step_grads(cfg, W, b, wl.dropout_seed(cfg), it)
+    pm.check("units-mc-bf16", cfg, grads_dict(cfg, g), G, loss, ref_loss, emulator(cfg, W, b, it))
 
 
 def test_units_collector_plans_and_budget_on_gpu():
