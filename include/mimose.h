@@ -220,13 +220,17 @@ mimose_status mimose_collect(mimose_ctx* ctx, const mimose_batch* batch, float* 
    the deepest plan predicts a peak above M - reserve (out->status set too). */
 mimose_status mimose_plan(mimose_ctx* ctx, int64_t input_size, mimose_plan_t* out);
 
-/* Selects the scheduler behind mimose_plan (PAPER.md P:207: Mimose "reserves a
+/* Selects the scheduler behind mimose_plan (PAPER.md P:179: Mimose "reserves a
    flexible interface for users to experiment with other scheduling algorithms,
    such as the Knapsack optimization").  kind 0 = Algorithm 1 greedy (default);
    kind 1 = exact: the fewest recomputed layers whose position-aware predicted
    peak fits M - reserve, then the lowest peak, then the lexicographically
-   smallest layer list (reading A29).  Clears the plan cache when the
-   kind changes.  MIMOSE_E_INVALID for an unknown kind; host only. */
+   smallest layer list (reading A29); kind 2 = time-weighted exact
+   (the Knapsack): the least total recompute cost, cost_l(x) = the collector's
+   forward time t_l regressed on x (integer ns, >= 1; averaged over the
+   ranks before the fit when a communicator exists), then the lowest peak, then
+   lexicographic (reading A31).  Clears the plan cache when the kind changes.
+   MIMOSE_E_INVALID for an unknown kind; host only. */
 mimose_status mimose_set_planner(mimose_ctx* ctx, int32_t kind);
 
 /* Responsive forward under plan (NULL -> no layer dropped).  Dropped layers
@@ -326,6 +330,10 @@ mimose_status mimose_plan_series(const mimose_series* s, int64_t budget, int64_t
                                  int32_t bucket_num, int32_t bucket_den,
                                  uint64_t* drop_mask, int64_t* predicted_peak);
 /* (bucket_num == 0 selects the exact planner of mimose_set_planner kind 1.) */
+/* The time-weighted exact planner (kind 2) on given predictions and per-layer
+   integer costs cost[0..n_layers) (each clamped to >= 1). */
+mimose_status mimose_plan_series_cost(const mimose_series* s, const int64_t* cost, int64_t budget,
+                                      int64_t reserve, uint64_t* drop_mask, int64_t* predicted_peak);
 /* Quadratic least squares (reading A18): fit ys(xs), predict at x_eval[i]. */
 mimose_status mimose_fit_predict(const int64_t* xs, const int64_t* ys, int32_t n, int32_t degree,
                                  const int64_t* x_eval, int32_t n_eval, int64_t* out);

@@ -17,7 +17,10 @@ Readings (DESIGN.md register, numbered as SURVEY §8(c)-R):
          last resort before INFEASIBLE
   A13    when the linear accounting says excess <= 0, re-check with the
          position-aware predicted peak P(L',x) and continue if still over
-  A29    the exact alternative planner (P:207: "a flexible interface for ...
+  A31    the time-weighted exact planner (the Knapsack of P:179): minimum
+         total integer recompute cost, then peak, then lexicographic
+         = brute_force(cost) (plan_exact_cost)
+  A29    the exact alternative planner (P:179: "a flexible interface for ...
          other scheduling algorithms, such as the Knapsack optimization"):
          fewest recomputed layers (unit cost: homogeneous encoder layers)
          with predicted_peak <= M - reserve, then the lowest peak, then the
@@ -189,6 +192,19 @@ def plan_exact(p: Dict, budget: int, reserve: int = 0):
     An infeasible budget returns (INFEASIBLE, all layers, their peak)."""
     L = len(p["a"])
     st, dropped, pk = brute_force(p, budget, [1] * L, reserve)
+    if st != OK:
+        return INFEASIBLE, list(range(L)), predicted_peak(p, range(L))
+    return OK, dropped, pk
+
+
+def plan_exact_cost(p: Dict, budget: int, cost: Sequence[int], reserve: int = 0):
+    """Reading A31 ("Knapsack"): the time-weighted exact planner is, by
+    definition, the brute-force minimum over all 2^L drop sets of the total
+    integer recompute cost (each cost clamped to >= 1), then the lowest peak,
+    then the lexicographically smallest sorted layer list.  Infeasible ->
+    (INFEASIBLE, all layers, their peak)."""
+    L = len(p["a"])
+    st, dropped, pk = brute_force(p, budget, [max(1, int(c)) for c in cost], reserve)
     if st != OK:
         return INFEASIBLE, list(range(L)), predicted_peak(p, range(L))
     return OK, dropped, pk

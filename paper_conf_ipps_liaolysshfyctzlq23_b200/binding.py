@@ -392,7 +392,7 @@ def predicted_peak(p: Dict, dropped=()) -> int:
     return _lib.mimose_predicted_peak(C.byref(s), C.c_uint64(mask))
 
 
-PLANNER_GREEDY, PLANNER_EXACT = 0, 1
+PLANNER_GREEDY, PLANNER_EXACT, PLANNER_EXACT_TIME = 0, 1, 2
 
 
 def plan_series(p: Dict, budget: int, reserve: int = 0, num: int = 9, den: int = 10, planner: int = PLANNER_GREEDY):
@@ -403,6 +403,22 @@ def plan_series(p: Dict, budget: int, reserve: int = 0, num: int = 9, den: int =
     mask = C.c_uint64()
     pk = C.c_int64()
     st = _lib.mimose_plan_series(C.byref(s), budget, reserve, num, den, C.byref(mask), C.byref(pk))
+    return st, [l for l in range(64) if (mask.value >> l) & 1], pk.value
+
+
+_lib.mimose_plan_series_cost.argtypes = [C.POINTER(Series), C.POINTER(C.c_int64), C.c_int64, C.c_int64,
+                                         C.POINTER(C.c_uint64), C.POINTER(C.c_int64)]
+EXPORTED.append("mimose_plan_series_cost")
+
+
+def plan_series_cost(p: Dict, cost, budget: int, reserve: int = 0):
+    """The library's time-weighted exact planner on explicit series and costs (test hook)."""
+    s, keep = _series(p)
+    L = len(p["a"])
+    cst = (C.c_int64 * L)(*[int(v) for v in cost])
+    mask = C.c_uint64()
+    pk = C.c_int64()
+    st = _lib.mimose_plan_series_cost(C.byref(s), cst, budget, reserve, C.byref(mask), C.byref(pk))
     return st, [l for l in range(64) if (mask.value >> l) & 1], pk.value
 
 

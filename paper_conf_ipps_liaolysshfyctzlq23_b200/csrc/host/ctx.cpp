@@ -1262,6 +1262,30 @@ void resolve_times(mimose_ctx* c) {
   c->pending_times = false;
 }
 
+// Data parallel: every rank must derive the same plans, but the
+// collector's forward times are per-rank measurements.  Before the estimator
+// is fitted, the ranks average their time samples (same x sequence on every
+// rank: the length schedule is shared), so the time-weighted planner's costs
+// agree bit for bit.  Memory samples are exact integers and already agree.
+mimose_status agree_times(mimose_ctx* c) {
+  if (!c->comm || c->samples.empty()) return MIMOSE_OK;
+  const int U = n_units(c);
+  const size_t n = c->samples.size() * (size_t)U;
+  std::vector<float> h(n);
+  for (size_t i = 0; i < c->samples.size(); ++i)
+    for (int l = 0; l < U; ++l) h[i * U + l] = c->samples[i].t_ms[l];
+  float* d = nullptr;
+  CK(cudaMallocAsync((void**)&d, n * 4, c->st));
+  CK(cudaMemcpyAsync(d, h.data(), n * 4, cudaMemcpyHostToDevice, c->st));
+  NK(ncclAllReduce(d, d, n, ncclFloat, ncclAvg, c->comm, c->st));
+  CK(cudaMemcpyAsync(h.data(), d, n * 4, cudaMemcpyDeviceToHost, c->st));
+  CK(cudaFreeAsync(d, c->st));
+  CK(cudaStreamSynchronize(c->st));
+  for (size_t i = 0; i < c->samples.size(); ++i)
+    for (int l = 0; l < U; ++l) c->samples[i].t_ms[l] = h[i * U + l];
+  return MIMOSE_OK;
+}
+
 mimose_status read_loss(mimose_ctx* c, float* loss_out) {
   if (!loss_out) return MIMOSE_OK;
   if (!c->device) { *loss_out = 0.f; return MIMOSE_OK; }
@@ -1609,6 +1633,7 @@ mimose_status mimose_backward(mimose_ctx* c) {
     const int64_t n = c->stats.collect_steps;
     if (!c->samples.empty() && ((n >= c->cfg.collect_iters && distinct >= 3) || n >= 30)) {
       resolve_times(c);
+      if (mimose_status s2 = agree_times(c)) return s2;
       auto t0 = std::chrono::steady_clock::now();
       c->est.fit(c->samples, c->cfg.degree);
       c->stats.planner_us_total +=
@@ -1664,7 +1689,8 @@ mimose_status mimose_set_optimizer(mimose_ctx* c, float lr, float b1, float b2, 
 
 mimose_status mimose_set_planner(mimose_ctx* c, int32_t kind) {
   if (mimose_status s = check_ready(c)) return s;
-  if (kind != PLANNER_GREEDY && kind != PLANNER_EXACT) return fail(c, MIMOSE_E_INVALID, "unknown planner");
+  if (kind != PLANNER_GREEDY && kind != PLANNER_EXACT && kind != PLANNER_EXACT_TIME)
+    return fail(c, MIMOSE_E_INVALID, "unknown planner");
   if (kind != c->planner) c->cache.clear();      // cached plans belong to the previous planner
   c->planner = kind;
   return MIMOSE_OK;
@@ -1684,9 +1710,11 @@ mimose_status mimose_plan(mimose_ctx* c, int64_t x, mimose_plan_t* out) {
     c->stats.plan_cache_misses++;
     auto t0 = std::chrono::steady_clock::now();
     const Series s = c->est.predict(x);
-    const PlanResult pr = c->planner == PLANNER_EXACT
-                              ? plan_exact(s, c->ar.budget, c->cfg.reserve_bytes)
-                              : plan_greedy(s, c->ar.budget, c->cfg.reserve_bytes, c->cfg.bucket_num, c->cfg.bucket_den);
+    const PlanResult pr =
+        c->planner == PLANNER_EXACT ? plan_exact(s, c->ar.budget, c->cfg.reserve_bytes)
+        : c->planner == PLANNER_EXACT_TIME
+            ? plan_exact_cost(s, c->est.predict_cost(x), c->ar.budget, c->cfg.reserve_bytes)
+            : plan_greedy(s, c->ar.budget, c->cfg.reserve_bytes, c->cfg.bucket_num, c->cfg.bucket_den);
     c->stats.planner_us_total +=
         std::chrono::duration<double, std::micro>(std::chrono::steady_clock::now() - t0).count();
     mimose_plan_t p{};
@@ -1894,6 +1922,16 @@ mimose_status mimose_plan_series(const mimose_series* s, int64_t budget, int64_t
                                  uint64_t* mask, int64_t* peak) {
   if (!s || !mask || !peak || s->n_layers < 1 || s->n_layers > 64 || bd <= 0) return MIMOSE_E_INVALID;
   const PlanResult r = bn == 0 ? plan_exact(to_series(s), budget, reserve) : plan_greedy(to_series(s), budget, reserve, bn, bd);
+  *mask = r.drop_mask;
+  *peak = r.peak;
+  return r.feasible ? MIMOSE_OK : MIMOSE_E_INFEASIBLE;
+}
+
+mimose_status mimose_plan_series_cost(const mimose_series* s, const int64_t* cost, int64_t budget, int64_t reserve,
+                                      uint64_t* mask, int64_t* peak) {
+  if (!s || !cost || !mask || !peak || s->n_layers < 1 || s->n_layers > 64) return MIMOSE_E_INVALID;
+  const PlanResult r =
+      plan_exact_cost(to_series(s), std::vector<int64_t>(cost, cost + s->n_layers), budget, reserve);
   *mask = r.drop_mask;
   *peak = r.peak;
   return r.feasible ? MIMOSE_OK : MIMOSE_E_INFEASIBLE;

@@ -130,62 +130,81 @@ PlanResult plan_greedy(const Series& s, int64_t budget, int64_t reserve, int bnu
 }
 
 namespace {
-struct ExactSearch {
-  const Series& s;
-  int L;
-  int64_t R;           // limit - (C + E): room for stack + transients
-  int k;               // drops to place
-  std::vector<int64_t> need;   // per-layer transient on top of its prefix
-  std::vector<int64_t> suf_a, suf_dmax;   // sum a_j and max (a_j - y_j) over j >= l
-  bool found = false;
-  int64_t best_pk = 0;
-  uint64_t best_mask = 0;
-  // Layers [l, L) remain; `left` drops still to place; prefix = stack bytes
-  // below layer l; runmax = max over the constraints of layers < l.
-  void dfs(int l, int left, int64_t prefix, int64_t runmax, uint64_t mask) {
-    if (found && runmax >= best_pk) return;             // cannot beat the best peak
-    if (l == L) {
-      if (left) return;
-      const int64_t pk = std::max(runmax, prefix + s.Hd + s.Th);
-      if (pk > R) return;
-      if (!found || pk < best_pk) { found = true; best_pk = pk; best_mask = mask; }
-      return;
+// Least total recompute cost of layers [l0, L) given `S0` stack bytes below l0,
+// such that every remaining event fits R (relative to C + E): layer l's
+// forward / backward events S_l + max(a_l, a_l - y_l + Tb) and the head event
+// S_L + Hd + Th.  Forward DP over layers with the 2-D Pareto front of
+// (stack bytes, cost): a state with no more bytes and no more cost than
+// another makes every completion at least as cheap and as feasible.
+int64_t min_cost_from(const Series& s, const std::vector<int64_t>& cost, const std::vector<int64_t>& suf_y,
+                      int l0, int64_t S0, int64_t R) {
+  const int L = (int)s.a.size();
+  std::vector<std::pair<int64_t, int64_t>> cur{{S0, 0}}, nxt;
+  for (int l = l0; l < L && !cur.empty(); ++l) {
+    const int64_t need = std::max(s.a[l], s.a[l] - s.y[l] + s.Tb);
+    nxt.clear();
+    for (auto& [S, c] : cur) {
+      if (S + need > R) continue;
+      if (S + s.y[l] + suf_y[l + 1] + s.Hd + s.Th <= R) nxt.push_back({S + s.y[l], c + cost[l]});
+      if (S + s.a[l] + suf_y[l + 1] + s.Hd + s.Th <= R) nxt.push_back({S + s.a[l], c});
     }
-    if (L - l < left) return;
-    // even the `left` largest savings below cannot bring the head event under R
-    if (prefix + suf_a[l] - (int64_t)left * suf_dmax[l] + s.Hd + s.Th > R) return;
-    const int64_t here = prefix + need[l];              // layer l's forward / backward events
-    if (here > R) return;                               // fixed by the choices below l
-    const int64_t rm = std::max(runmax, here);
-    if (left > 0) dfs(l + 1, left - 1, prefix + s.y[l], rm, mask | (1ull << l));   // drop first: lex order
-    dfs(l + 1, left, prefix + s.a[l], rm, mask);
+    std::sort(nxt.begin(), nxt.end());
+    cur.clear();
+    int64_t best = INT64_MAX;
+    for (auto& st : nxt)
+      if (st.second < best) { cur.push_back(st); best = st.second; }
   }
-};
+  int64_t best = INT64_MAX;
+  for (auto& [S, c] : cur)
+    if (S + s.Hd + s.Th <= R) best = std::min(best, c);
+  return best;
+}
 }  // namespace
 
-PlanResult plan_exact(const Series& s, int64_t budget, int64_t reserve) {
+PlanResult plan_exact_cost(const Series& s, const std::vector<int64_t>& cost_in, int64_t budget, int64_t reserve) {
   const int L = (int)s.a.size();
   const int64_t base = s.C + s.E;
-  ExactSearch x{s, L, budget - reserve - base, 0, {}};
-  x.need.resize(L);
-  for (int l = 0; l < L; ++l) x.need[l] = std::max(s.a[l], s.a[l] - s.y[l] + s.Tb);
-  x.suf_a.assign(L + 1, 0);
-  x.suf_dmax.assign(L + 1, 0);
-  for (int l = L - 1; l >= 0; --l) {
-    x.suf_a[l] = x.suf_a[l + 1] + s.a[l];
-    x.suf_dmax[l] = std::max(x.suf_dmax[l + 1], s.a[l] - s.y[l]);
+  const int64_t R = budget - reserve - base;
+  const uint64_t all = L >= 64 ? ~0ull : ((1ull << L) - 1);
+  std::vector<int64_t> cost(L), suf_y(L + 1, 0);
+  for (int l = 0; l < L; ++l) cost[l] = std::max<int64_t>(1, cost_in[l]);
+  for (int l = L - 1; l >= 0; --l) suf_y[l] = suf_y[l + 1] + s.y[l];
+  auto mc = [&](int l0, int64_t S0, int64_t lim) {
+    return s.Te <= lim ? min_cost_from(s, cost, suf_y, l0, S0, lim) : INT64_MAX;
+  };
+  // 1. the least total cost
+  const int64_t cstar = mc(0, 0, R);
+  if (cstar == INT64_MAX) return {false, all, predicted_peak(s, all)};
+  // 2. the lowest peak among least-cost sets: the smallest limit P <= R under
+  //    which the least cost is still cstar (it only rises as P falls)
+  int64_t lo = 0, hi = R;
+  while (lo < hi) {
+    const int64_t mid = lo + (hi - lo) / 2;
+    if (mc(0, 0, mid) == cstar) hi = mid; else lo = mid + 1;
   }
-  if (s.Te <= x.R) {
-    for (int k = 0; k <= L && !x.found; ++k) {
-      x.k = k;
-      x.dfs(0, k, 0, s.Te, 0);
+  const int64_t P = hi;
+  // 3. the lexicographically smallest sorted layer list among them: drop each
+  //    layer in order whenever a completion with total cost cstar under P exists
+  //    (all costs >= 1, so no least-cost list is a proper prefix of another)
+  uint64_t mask = 0;
+  int64_t S = 0, c = 0;
+  for (int l = 0; l < L; ++l) {
+    const int64_t rest = mc(l + 1, S + s.y[l], P);
+    if (rest != INT64_MAX && c + cost[l] + rest == cstar) {
+      mask |= 1ull << l;
+      S += s.y[l];
+      c += cost[l];
+    } else {
+      S += s.a[l];
     }
   }
-  if (!x.found) {
-    const uint64_t all = L >= 64 ? ~0ull : ((1ull << L) - 1);
-    return {false, all, predicted_peak(s, all)};
-  }
-  return {true, x.best_mask, base + x.best_pk};
+  return {true, mask, base + P};
+}
+
+// Unit recompute cost: the same least-cost search with every cost 1 (fewest
+// recomputed layers, then lowest peak, then lexicographic; reading A29).
+PlanResult plan_exact(const Series& s, int64_t budget, int64_t reserve) {
+  return plan_exact_cost(s, std::vector<int64_t>(s.a.size(), 1), budget, reserve);
 }
 
 void Estimator::fit(const std::vector<Sample>& smp, int degree) {
@@ -209,7 +228,16 @@ void Estimator::fit(const std::vector<Sample>& smp, int degree) {
   fTh.fit(xs, series([](const Sample& s) { return s.Th; }), degree);
   fTb.fit(xs, series([](const Sample& s) { return s.Tb; }), degree);
   fTe.fit(xs, series([](const Sample& s) { return s.Te; }), degree);
+  ft.assign(L, Poly());
+  for (int l = 0; l < L; ++l)
+    ft[l].fit(xs, series([&](const Sample& s) { return (int64_t)std::llround((double)s.t_ms[l] * 1e6); }), degree);
   fitted = true;
+}
+
+std::vector<int64_t> Estimator::predict_cost(int64_t x) const {
+  std::vector<int64_t> c(ft.size());
+  for (size_t l = 0; l < ft.size(); ++l) c[l] = std::max<int64_t>(1, (int64_t)std::nearbyint(ft[l].eval(x)));
+  return c;
 }
 
 Series Estimator::predict(int64_t x) const {

@@ -38,15 +38,24 @@ struct PlanResult {
 // Algorithm 1 (A1-A11) + last-layer exclusion (A12) + verify (A13).
 PlanResult plan_greedy(const Series& s, int64_t budget, int64_t reserve, int bucket_num, int bucket_den);
 
-// The exact alternative behind the same (M, x, L) -> L' interface (P:207: "a
+// The exact alternative behind the same (M, x, L) -> L' interface (P:179: "a
 // flexible interface ... such as the Knapsack optimization"): among all drop
 // sets whose position-aware predicted peak is <= budget - reserve, the one with
 // the fewest recomputed layers (unit recompute cost: the encoder layers are
 // homogeneous), then the lowest peak, then the lexicographically smallest
-// sorted layer list.  Depth-first over layers in order with the exact prefix
-// constraints of predicted_peak as pruning (reading A29).
+// sorted layer list (reading A29): plan_exact_cost with every cost 1.
 PlanResult plan_exact(const Series& s, int64_t budget, int64_t reserve);
-enum PlannerKind : int { PLANNER_GREEDY = 0, PLANNER_EXACT = 1 };
+
+// The recompute-time-weighted exact planner ("Knapsack", reading
+// A31): among all feasible drop sets, the minimum total recompute cost
+// sum cost[l] (integers, each >= 1), then the lowest peak, then the
+// lexicographically smallest sorted layer list.  Three exact phases, each a
+// forward dynamic program over the layers with the 2-D Pareto front of
+// (stack bytes, cost): the least cost; the lowest peak among least-cost sets
+// (binary search on the event limit); then the lexicographic choice layer by
+// layer.  Milliseconds at 48 units.
+PlanResult plan_exact_cost(const Series& s, const std::vector<int64_t>& cost, int64_t budget, int64_t reserve);
+enum PlannerKind : int { PLANNER_GREEDY = 0, PLANNER_EXACT = 1, PLANNER_EXACT_TIME = 2 };
 
 // One collected sheltered-iteration sample (arena deltas).
 struct Sample {
@@ -60,8 +69,11 @@ struct Estimator {
   int64_t C = 0;
   std::vector<Poly> fa, fy;
   Poly fE, fHd, fTh, fTb, fTe;
+  std::vector<Poly> ft;   // per-layer forward time, integer ns (the collector's t_l(x))
   void fit(const std::vector<Sample>& samples, int degree);
   Series predict(int64_t x) const;
+  // Recompute cost per layer at x: the fitted forward time in ns, at least 1.
+  std::vector<int64_t> predict_cost(int64_t x) const;
 };
 
 }  // namespace mimose

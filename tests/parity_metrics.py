@@ -67,6 +67,9 @@ def check(name, cfg, gd, G, loss, ref_loss, emulate=None):
     os.makedirs(out, exist_ok=True)
     with open(os.path.join(out, name + ".json"), "w") as f:
         json.dump(rec, f, indent=1)
+    if os.environ.get("MIMOSE_PARITY_DUMP"):          # GPU gradients of the worst tensors, for offline study
+        for r in rec["grads"][:3]:
+            np.save(os.path.join(out, f"{name}__{r['name']}.npy"), np.asarray(gd[r["name"]], np.float32))
     assert rec["loss_rel"] <= tol, (name, loss, ref_loss)
     for k, r in rows.items():
         if r["zero"]:

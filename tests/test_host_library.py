@@ -225,6 +225,55 @@ def test_exact_planner_on_config_series(name):
     assert worst < 0.5, worst
 
 
+def test_time_weighted_planner_matches_brute_force():
+    """Reading A31: the library's cost-weighted exact planner (kind 2, a dynamic
+    program with dominance pruning) equals the oracle's brute force (least
+    total integer cost, then lowest peak, then lexicographic) bit for bit, on
+    homogeneous and heterogeneous stacks with random costs, including ties."""
+    rng = random.Random(31)
+    n_ok = 0
+    for it in range(1200):
+        L = rng.randint(1, 11)
+        p = _random_series(rng, L, it % 2 == 0)
+        cost = ([rng.randint(1, 4) for _ in range(L)] if it % 3 == 0 else
+                [rng.randint(0, 10 ** 6) for _ in range(L)])
+        lo, hi = op.predicted_peak(p, range(L)), op.predicted_peak(p, [])
+        M = rng.randint(lo - 5, hi + 5)
+        st, dropped, pk = mb.plan_series_cost(p, cost, M)
+        ost, odropped, opk = op.plan_exact_cost(p, M, cost)
+        assert (st == mb.OK) == (ost == op.OK), (p, cost, M)
+        if ost == op.OK:
+            assert dropped == odropped and pk == opk <= M, (p, cost, M)
+            n_ok += 1
+    assert n_ok > 500
+
+
+@pytest.mark.parametrize("name", CFGS)
+def test_time_weighted_planner_scales_to_units(name):
+    """48-unit series (H = 1024 configs at granularity 1) with attention / FFN
+    recompute costs from the FLOP model: feasible whenever a plan exists, within
+    the budget, never costlier than the unit-count exact plan, and fast."""
+    import time
+    cfg = wl.CONFIGS[name]
+    M = budget_for(cfg)
+    H, F = cfg.hidden, cfg.ffn
+    worst = 0.0
+    for S in range(cfg.pad, cfg.max_seq + 1, max(cfg.pad, cfg.max_seq // 6)):
+        p = om.collect_samples_units(om.sizes(cfg, cfg.n_seqs, S))
+        T = cfg.n_seqs * S
+        cost = [2 * T * 4 * H * H + 4 * cfg.n_seqs * S * S * H, 2 * T * 2 * H * F] * cfg.n_layers
+        cost = [c // 10 ** 6 + 1 for c in cost]
+        t0 = time.perf_counter()
+        st, dropped, pk = mb.plan_series_cost(p, cost, M)
+        worst = max(worst, time.perf_counter() - t0)
+        est, edropped, _ = mb.plan_series(p, M, planner=mb.PLANNER_EXACT)
+        assert (st == mb.OK) == (est == mb.OK)
+        if st == mb.OK:
+            assert pk <= M and pk == op.predicted_peak(p, dropped)
+            assert sum(cost[u] for u in dropped) <= sum(cost[u] for u in edropped)
+    assert worst < 0.5, worst
+
+
 # ---------------------------------------------------------------------------
 # sub-layer checkpoint units (granularity=1; SURVEY f1, DESIGN reading A30)
 # ---------------------------------------------------------------------------
