@@ -9,7 +9,9 @@ Storage points (ctx.cpp schedule; DESIGN §3/§5):
   forward   x_l (layer input), QKV, P~ (attention probabilities after dropout,
             the PV operand), O, h1, u, g, y; z1/z2/LN statistics stay fp32
   backward  dt2 = dz2*mask, du = (dt2 W2) * GELU'(u), dt1, dO, dS (the
-            dQ/dK operand), dQKV; dh1, dz1 and the inter-layer dy stay fp32
+            dQ/dK operand), dQKV; dh1, dz1 and the inter-layer dy stay fp32;
+            the bias gradients of the out-projection and FFN2 sum the stored
+            bf16 dt1 / dt2 rows (as the LN-backward kernel's partials do)
   embedding x1 = drop(LN0(z0));  head: pooled
 The building blocks are the oracle's own (linear, layernorm, gelu, softmax,
 Masks, embed/head); with rnd = identity this function returns the oracle's
@@ -67,7 +69,7 @@ def _attn_bwd(dout, cache, B, S, h, pmask, r):
     return r(np.concatenate([flat(dq), flat(dk), flat(dv)], axis=1))
 
 
-def _layer_fwd(cfg, W, l, x, lengths, B, S, masks, r):
+def _layer_fwd(cfg, W, l, x, lengths, B, S, masks, r, gelu):
     p = f"layer{l}."
     qkv = r(om.linear(x, W[p + "qkv.w"], W[p + "qkv.b"]))
     o, ac = _attn_fwd(qkv, lengths, B, S, cfg.heads, masks.attn_probs(l), r)
@@ -75,26 +77,24 @@ def _layer_fwd(cfg, W, l, x, lengths, B, S, masks, r):
     h1f, ln1 = om.layernorm(z1, W[p + "ln1.g"], W[p + "ln1.b"], cfg.ln_eps)
     h1 = r(h1f)
     uf = om.linear(h1, W[p + "f1.w"], W[p + "f1.b"])
-    u, g = r(uf), r(om.gelu(uf))
+    u, g = r(uf), r(gelu[0](uf))
     z2 = h1 + om.linear(g, W[p + "f2.w"], W[p + "f2.b"]) * masks.ffn_out(l)
     y, ln2 = om.layernorm(z2, W[p + "ln2.g"], W[p + "ln2.b"], cfg.ln_eps)
     return r(y), dict(x=x, qkv=qkv, o=o, ac=ac, ln1=ln1, h1=h1, u=u, g=g, ln2=ln2)
 
 
-def _layer_bwd(cfg, W, l, dy, c, B, S, masks, G, r):
+def _layer_bwd(cfg, W, l, dy, c, B, S, masks, G, r, gelu):
     p = f"layer{l}."
     dz2, G[p + "ln2.g"], G[p + "ln2.b"] = om.layernorm_bwd(dy, c["ln2"], W[p + "ln2.g"])
-    dt2f = dz2 * masks.ffn_out(l)
-    dt2 = r(dt2f)
-    G[p + "f2.b"] = dt2f.sum(axis=0)                    # bias partials from the fp32 LN-backward rows
-    du = r(om.gelu_bwd(dt2 @ W[p + "f2.w"], c["u"]))
+    dt2 = r(dz2 * masks.ffn_out(l))
+    G[p + "f2.b"] = dt2.sum(axis=0)                     # bias partials sum the stored (bf16) rows
+    du = r(gelu[1](dt2 @ W[p + "f2.w"], c["u"]))
     G[p + "f2.w"] = dt2.T @ c["g"]
     dh1, G[p + "f1.w"], G[p + "f1.b"] = om.linear_bwd(du, c["h1"], W[p + "f1.w"])
     dh1 = dh1 + dz2
     dz1, G[p + "ln1.g"], G[p + "ln1.b"] = om.layernorm_bwd(dh1, c["ln1"], W[p + "ln1.g"])
-    dt1f = dz1 * masks.attn_out(l)
-    dt1 = r(dt1f)
-    G[p + "o.b"] = dt1f.sum(axis=0)
+    dt1 = r(dz1 * masks.attn_out(l))
+    G[p + "o.b"] = dt1.sum(axis=0)
     do = r(dt1 @ W[p + "o.w"])
     G[p + "o.w"] = dt1.T @ c["o"]
     dqkv = _attn_bwd(do, c["ac"], B, S, cfg.heads, masks.attn_probs(l), r)
@@ -102,8 +102,12 @@ def _layer_bwd(cfg, W, l, dy, c, B, S, masks, G, r):
     return dx + dz1
 
 
-def train_step_grads(cfg: ModelConfig, params, batch: Batch, seed: int, step: int, rnd=bf16):
-    """Loss and gradients of one plain step with bf16 storage rounding ``rnd``."""
+def train_step_grads(cfg: ModelConfig, params, batch: Batch, seed: int, step: int, rnd=bf16,
+                     gelu: str = "erf"):
+    """Loss and gradients of one plain step with bf16 storage rounding ``rnd``.
+    ``gelu="tanh"``: the tanh-form GELU / GELU' that the bf16 tcgen05 epilogues
+    evaluate for erf-GELU models (DESIGN reading R-G) instead of the exact erf."""
+    gl = (om.gelu, om.gelu_bwd) if gelu == "erf" else (om.gelu_tanh, om.gelu_tanh_bwd)
     assert cfg.arch == ARCH_POST_LN
     W = {k: np.asarray(v, np.float64) for k, v in params.items()}
     B, S = batch.input_ids.shape
@@ -113,10 +117,10 @@ def train_step_grads(cfg: ModelConfig, params, batch: Batch, seed: int, step: in
     x = rnd(x)
     caches = []
     for l in range(cfg.n_layers):
-        x, c = _layer_fwd(cfg, W, l, x, batch.lengths, B, S, masks, rnd)
+        x, c = _layer_fwd(cfg, W, l, x, batch.lengths, B, S, masks, rnd, gl)
         caches.append(c)
     loss, dy = om.head_fwd_bwd(cfg, W, x, batch, masks, G)
     for l in reversed(range(cfg.n_layers)):
-        dy = _layer_bwd(cfg, W, l, dy, caches[l], B, S, masks, G, rnd)
+        dy = _layer_bwd(cfg, W, l, dy, caches[l], B, S, masks, G, rnd, gl)
     om.embed_bwd(cfg, W, dy, ec, masks, G)
     return loss, G

@@ -60,7 +60,7 @@ def emulator(cfg, W, b):
     if cfg.arch != wl.ARCH_POST_LN:
         return None
     import bf16_emulation as be
-    return lambda: be.train_step_grads(cfg, W, b, wl.dropout_seed(cfg), 1)
+    return lambda: be.train_step_grads(cfg, W, b, wl.dropout_seed(cfg), 1, gelu="tanh")
 
 
 def bf16_weights(params):

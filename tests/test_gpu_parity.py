@@ -110,7 +110,7 @@ def emulator(cfg, W, b, it):
     if cfg.dtype != "bf16" or cfg.arch != wl.ARCH_POST_LN:
         return None
     import bf16_emulation as be
-    return lambda: be.train_step_grads(cfg, W, b, wl.dropout_seed(cfg), it)
+    return lambda: be.train_step_grads(cfg, W, b, wl.dropout_seed(cfg), it, gelu="tanh")
 
 
 @pytest.mark.parametrize("case", list(CASES))
