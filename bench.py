@@ -46,6 +46,10 @@ def parse():
     ap.add_argument("--gemm-mode", type=int, default=-1, help="tcgen05 GEMM variant (debug_options)")
     ap.add_argument("--granularity", type=int, default=0, choices=[0, 1],
                     help="checkpoint units of the headline arm: 0 layers (paper, A14), 1 attention/FFN blocks (A30)")
+    ap.add_argument("--zero1", action="store_true",
+                    help="ZeRO-1 optimizer-state sharding (SURVEY f4; needs world > 1 or --comm-force)")
+    ap.add_argument("--comm-force", action="store_true",
+                    help="build the NCCL communicator even at one GPU (a 1-rank communicator)")
     ap.add_argument("--planner", default="greedy", choices=["greedy", "exact", "knapsack"],
                     help="Algorithm 1 (default), the exact fewest-recompute planner (A29) or the "
                          "recompute-time-weighted exact planner (A31)")
@@ -261,7 +265,7 @@ def main():
         mb.debug_options(gemm_mode=args.gemm_mode)
 
     # ---- budget (D2 / reading A21) from the library's own allocation sequence ----
-    probe_ctx = mb.Mimose(cfg, 0)
+    probe_ctx = mb.Mimose(cfg, 0, world=world, zero1=1 if args.zero1 else 0)
     C0 = probe_ctx.stats()["persistent_bytes"]
     P0 = probe_ctx.dry_run(cfg.n_seqs, cfg.max_seq, [])
     LB = probe_ctx.dry_run(cfg.n_seqs, cfg.max_seq, range(cfg.n_layers))
@@ -280,6 +284,8 @@ def main():
         return bytes(t.cpu().numpy().tolist())
 
     def new_ctx(budget, slab_bytes, enforce=1, **kw):
+        kw.setdefault("zero1", 1 if args.zero1 else 0)
+        kw.setdefault("comm_force", 1 if args.comm_force else 0)
         slab = torch.empty(slab_bytes, dtype=torch.uint8, device="cuda")
         ctx = mb.Mimose(cfg, budget, slab=slab, stream=stream, rank=rank, world=world,
                         nccl_id=fresh_nccl_id(), enforce_budget=enforce, use_tc=use_tc, **kw)
@@ -489,10 +495,10 @@ def main():
     del ctx
     torch.cuda.empty_cache()
 
-    def arm(budget, batches_, sched_, granularity=0, planner=None, fixed=None, slab=None, enforce=1):
+    def arm(budget, batches_, sched_, granularity=0, planner=None, fixed=None, slab=None, enforce=1, **kw):
         """One same-run comparison arm: its own context (sheltered phase on
         sched_ unless a fixed plan / none), timed on batches_."""
-        ctx = new_ctx(budget, slab or budget, enforce=enforce, granularity=granularity)
+        ctx = new_ctx(budget, slab or budget, enforce=enforce, granularity=granularity, **kw)
         if planner is not None:
             ctx.set_planner(planner)
         out = {}
@@ -557,6 +563,13 @@ def main():
         nm.update(schedule="truncated normal mu=(lo+hi)/2 sigma=(hi-lo)/4", mean_seq_pad=tokens(nb)[0],
                   no_ckpt_value=nn["value"], recompute_ratio=ms_nm / ms_nn)
         result["normal_schedule"] = nm
+        # the multi-GPU code path on this one GPU: a 1-rank NCCL communicator with
+        # ZeRO-1 (per-bucket reduce-scatter, sharded AdamW, weight all-gather)
+        if world == 1:
+            z, ms_z = arm(M, batches, sched, comm_force=1, zero1=1)
+            z.update(note="comm_force=1, zero1=1 at world 1: the DP/ZeRO-1 collectives run on a 1-rank "
+                          "communicator", overhead_vs_headline=ms_z / ms)
+            result["zero1_nccl_1rank"] = z
         result["recompute_ratio"] = ms / ms_n
         result["speedup_vs_static"] = ms_s / ms
         result["paper_context"] = ("V100 (P:227): Mimose ~18.0% faster than Sublinear, ~15.0% than DTR "

@@ -112,7 +112,15 @@ typedef struct {
                             (x, drop mask, predicted peak) over the communicator and
                             fails with MIMOSE_E_STATE if any rank differs (
                             debug: one small device->host sync per step)               */
-  int32_t reserved[2];
+  int32_t zero1;         /* 1: ZeRO-1: the AdamW state (fp32 master, m, v) is
+                            sharded over the ranks.  Each gradient bucket is padded to
+                            64 x world elements, reduce-scattered (instead of all-reduced),
+                            this rank's shard updated, and the bf16 working weights
+                            all-gathered -- all overlapped with the backward when the
+                            optimizer is fused.  Persistent bytes fall from 18 to
+                            6 + 12 / world B/param.  Needs a communicator (world > 1 or
+                            comm_force); mimose_get_master is then refused for world > 1. */
+  int32_t reserved[1];
 } mimose_config;
 
 /* Fill defaults (collect_iters 10, ratio 9/10, degree 2, p 0.1, eps 1e-12,

@@ -56,15 +56,44 @@ def ebytes(cfg: ModelConfig) -> int:
 NPART = 296   # fixed count of deterministic reduction partials (DESIGN "Memory model")
 
 
-def persistent_bytes(cfg: ModelConfig, max_seqs: int, max_seq_len: int) -> int:
-    """C: weights (e), fp32 grads, fp32 master (bf16 only), AdamW m and v, batch
+def buckets(cfg: ModelConfig) -> List[List[int]]:
+    """Gradient buckets as lists of parameter indices, in layout order: the
+    embedding tensors, one bucket per encoder layer (12 tensors), the head
+    (all-reduced / reduce-scattered as soon as each is final)."""
+    n = len(param_spec(cfg))
+    n_emb = 2 if cfg.arch == ARCH_PRE_LN else 5
+    out = [list(range(n_emb))]
+    for l in range(cfg.n_layers):
+        out.append(list(range(n_emb + 12 * l, n_emb + 12 * (l + 1))))
+    out.append(list(range(n_emb + 12 * cfg.n_layers, n)))
+    return out
+
+
+def padded_numel(cfg: ModelConfig, world: int = 1, zero1: bool = False) -> int:
+    """Elements of the padded flat parameter image: every tensor rounded up to
+    64 elements; with ZeRO-1 every bucket rounded up to 64 x world elements so it
+    splits into world equal shards."""
+    spec = param_spec(cfg)
+    unit = 64 * world if zero1 else 64
+    tot = 0
+    for b in buckets(cfg):
+        nb = sum((int(_prod(spec[i][1])) + 63) // 64 * 64 for i in b)
+        tot += (nb + unit - 1) // unit * unit
+    return tot
+
+
+def persistent_bytes(cfg: ModelConfig, max_seqs: int, max_seq_len: int, world: int = 1,
+                     zero1: bool = False) -> int:
+    """C: weights (e), fp32 grads, fp32 master (bf16 only), AdamW m and v (with
+    ZeRO-1 master, m and v hold this rank's 1/world shard only), batch
     metadata buffers, misc, and the fixed backward workspaces."""
     e = ebytes(cfg)
     H, F = cfg.hidden, cfg.ffn
-    npad = sum((int(_prod(s)) + 63) // 64 * 64 for _, s in param_spec(cfg))
-    c = a16(npad * e) + a16(npad * 4) + a16(npad * 4) + a16(npad * 4)   # w, grad, m, v
+    npad = padded_numel(cfg, world, zero1)
+    nsh = npad // world if zero1 else npad
+    c = a16(npad * e) + a16(npad * 4) + a16(nsh * 4) + a16(nsh * 4)     # w, grad, m, v
     if cfg.dtype != "fp32":
-        c += a16(npad * 4)                                               # master
+        c += a16(nsh * 4)                                                # master
     maxT = max_seqs * max_seq_len
     c += a16(maxT * 4) * 2 + a16(max_seqs * 4) + a16(2 * max_seqs * 4)  # ids, tt, lens, labels
     c += a16(256)                                                        # misc scalars
@@ -113,7 +142,7 @@ class Sizes:
 
 
 def sizes(cfg: ModelConfig, B: int, S: int, max_seqs: Optional[int] = None,
-          max_seq_len: Optional[int] = None) -> Sizes:
+          max_seq_len: Optional[int] = None, world: int = 1, zero1: bool = False) -> Sizes:
     e = ebytes(cfg)
     H, F, h = cfg.hidden, cfg.ffn, cfg.heads
     T = B * S
@@ -155,7 +184,7 @@ def sizes(cfg: ModelConfig, B: int, S: int, max_seqs: Optional[int] = None,
     layer_scr = a16(T * H * 4) + a16(T * F * e) + a16(T * 3 * H * e) + a16(B * h * S * 4)
     ntiles = (ms * mx + 1023) // 1024
     emb_scr = a16(T * H * 4) + a16(16 * T) + a16(4 * 256 * ntiles)   # dz0, 4 int32[T] sort arrays, digit histograms
-    return Sizes(persistent_bytes(cfg, ms, mx), E, internals, y, head, dy, head_scr,
+    return Sizes(persistent_bytes(cfg, ms, mx, world, zero1), E, internals, y, head, dy, head_scr,
                  layer_scr, emb_scr, cfg.n_layers, head_fwd)
 
 

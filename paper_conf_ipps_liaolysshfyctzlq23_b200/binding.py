@@ -46,7 +46,7 @@ class Config(C.Structure):
                 ("rank", C.c_int32), ("world", C.c_int32), ("nccl_id", C.c_void_p),
                 ("use_tc", C.c_int32), ("pad_id", C.c_int32), ("granularity", C.c_int32),
                 ("comm_force", C.c_int32), ("nccl_max_ctas", C.c_int32), ("check_plans", C.c_int32),
-                ("reserved", C.c_int32 * 2)]
+                ("zero1", C.c_int32), ("reserved", C.c_int32 * 1)]
 
 
 class BatchS(C.Structure):

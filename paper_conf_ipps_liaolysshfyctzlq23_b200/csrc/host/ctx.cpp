@@ -40,9 +40,26 @@ struct ParamInfo {
 constexpr int LM_CHUNK = 2048;   // tokens per LM-head chunk (DESIGN "Memory model")
 inline int64_t vpad(int64_t v) { return (v + 7) / 8 * 8; }
 
-std::vector<ParamInfo> build_layout(const mimose_config& c, int64_t* npad) {
+// Every tensor is padded to 64 elements.  The gradient buckets (embedding,
+// one per layer, head; in layout order) end on a multiple of `unit` elements:
+// 64, or 64 x world with ZeRO-1 so that every bucket splits into world equal
+// shards.
+std::vector<ParamInfo> build_layout(const mimose_config& c, int64_t* npad, int64_t unit = 64) {
   std::vector<int64_t> n;
   const int64_t H = c.hidden, F = c.ffn;
+  auto lay = [&](int n_emb) {
+    std::vector<ParamInfo> out;
+    int64_t off = 0;
+    for (size_t i = 0; i < n.size(); ++i) {
+      out.push_back({n[i], off});
+      off += (n[i] + 63) / 64 * 64;
+      const int64_t j = (int64_t)i + 1 - n_emb;          // params completed past the embedding bucket
+      if (j == 0 || (j > 0 && j % 12 == 0 && j <= 12LL * c.n_layers) || i + 1 == n.size())
+        off = (off + unit - 1) / unit * unit;             // bucket end
+    }
+    *npad = off;
+    return out;
+  };
   if (c.arch == 1) {             // GPT-2: wte, wpe, pre-LN layers, lnf
     n.push_back((int64_t)c.vocab * H);
     n.push_back((int64_t)c.max_pos * H);
@@ -52,11 +69,7 @@ std::vector<ParamInfo> build_layout(const mimose_config& c, int64_t* npad) {
     }
     n.push_back(H);
     n.push_back(H);
-    std::vector<ParamInfo> out;
-    int64_t off = 0;
-    for (int64_t x : n) { out.push_back({x, off}); off += (x + 63) / 64 * 64; }
-    *npad = off;
-    return out;
+    return lay(2);
   }
   n.push_back((int64_t)c.vocab * H);
   n.push_back((int64_t)c.max_pos * H);
@@ -77,14 +90,7 @@ std::vector<ParamInfo> build_layout(const mimose_config& c, int64_t* npad) {
     n.push_back(no * H);
     n.push_back(no);
   }
-  std::vector<ParamInfo> out;
-  int64_t off = 0;
-  for (int64_t x : n) {
-    out.push_back({x, off});
-    off += (x + 63) / 64 * 64;
-  }
-  *npad = off;
-  return out;
+  return lay(5);
 }
 
 enum { P_WORD = 0, P_POS, P_TYPE, P_LN0G, P_LN0B, P_LAYER0 };
@@ -189,6 +195,11 @@ struct mimose_ctx {
   uint64_t drop_mask = 0;
   bool fwd_done = false, bwd_done = false, collecting = false;
   bool step_pending = false;   // fused optimizer: backward applied the update, mimose_step not yet called
+  // ZeRO-1: optimizer state (master, m, v) sharded over the ranks
+  bool zero1 = false;
+  int64_t nshard = 0;                        // elements of master / m / v on this rank
+  std::vector<int64_t> bk_b0, bk_b1, bk_sh;  // per bucket (event index): [b0, b1) and shard offset
+  std::vector<cudaEvent_t> ev_upd;           // ZeRO-1: shard update done (opt stream)
   int64_t stats_allreduce_calls = 0, stats_allreduce_bytes = 0;
   int64_t stats_plan_checks = 0;
   float* z0 = nullptr;
@@ -291,8 +302,8 @@ Sz sizes(const mimose_ctx* c, int B, int S) {
 
 int64_t persistent_bytes(const mimose_ctx* c) {
   const int64_t H = c->cfg.hidden, F = c->cfg.ffn;
-  int64_t C = a16(c->npad * c->e) + 3 * a16(c->npad * 4);     // w, grad, m, v
-  if (c->dt != DT_F32) C += a16(c->npad * 4);                  // master
+  int64_t C = a16(c->npad * c->e) + a16(c->npad * 4) + 2 * a16(c->nshard * 4);   // w, grad, m, v
+  if (c->dt != DT_F32) C += a16(c->nshard * 4);                                  // master
   const int64_t maxT = (int64_t)c->cfg.max_seqs * c->cfg.max_seq_len;
   C += 2 * a16(maxT * 4) + a16((int64_t)c->cfg.max_seqs * 4) + a16(2LL * c->cfg.max_seqs * 4);
   C += a16(256);
@@ -879,8 +890,42 @@ int64_t bucket_end(mimose_ctx* c, int last_param) {
 // A gradient bucket (params first..last) is final: all-reduce it (DP) on the
 // comm stream and, with the fused optimizer, update it on the optimizer stream,
 // both overlapping the rest of the backward.
+// ZeRO-1: reduce-scatter the bucket (this rank's shard of the
+// summed gradient lands in its own slice, in place), AdamW on that shard
+// (master, m, v hold shards only), all-gather the updated working weights.
+// `st_rs` runs the collectives, `st_opt` the update; the all-gather waits on it.
+mimose_status zero_bucket(mimose_ctx* c, int evi, cudaStream_t st_rs, cudaStream_t st_opt, bool update) {
+  const int W = c->cfg.world, r = c->cfg.rank;
+  const int64_t b0 = c->bk_b0[evi], cb = (c->bk_b1[evi] - b0) / W, sh = c->bk_sh[evi];
+  float* gsh = c->grad + b0 + r * cb;
+  NK(ncclReduceScatter(c->grad + b0, gsh, (size_t)cb, ncclFloat, ncclSum, c->comm, st_rs));
+  c->stats_allreduce_calls++;
+  c->stats_allreduce_bytes += cb * W * 4;
+  if (!update) return MIMOSE_OK;
+  if (st_opt != st_rs) {
+    CK(cudaEventRecord(c->ev_ar[evi], st_rs));
+    CK(cudaStreamWaitEvent(st_opt, c->ev_ar[evi], 0));
+  }
+  const double t = (double)(c->adam_t + 1);
+  const double bc1 = 1.0 - std::pow((double)c->opt_b1, t), bc2 = 1.0 - std::pow((double)c->opt_b2, t);
+  char* wsh = c->w + (b0 + r * cb) * c->e;
+  adamw(c->dt, wsh, c->master ? c->master + sh : nullptr, gsh, c->m + sh, c->v + sh, cb, c->opt_lr, c->opt_b1,
+        c->opt_b2, c->opt_eps, c->opt_wd, (float)bc1, (float)bc2, 1.0f / (float)W, st_opt);
+  if (st_opt != st_rs) {
+    CK(cudaEventRecord(c->ev_upd[evi], st_opt));
+    CK(cudaStreamWaitEvent(st_rs, c->ev_upd[evi], 0));
+  }
+  NK(ncclAllGather(wsh, c->w + b0 * c->e, (size_t)cb, c->dt == DT_F32 ? ncclFloat : ncclBfloat16, c->comm, st_rs));
+  return MIMOSE_OK;
+}
+
 mimose_status allreduce_bucket(mimose_ctx* c, int first, int last, int evi) {
   if (!c->device || (!c->comm && !c->opt_fused)) return MIMOSE_OK;
+  if (c->zero1) {
+    CK(cudaEventRecord(c->ev_layer[evi], c->st));
+    CK(cudaStreamWaitEvent(c->comm_st, c->ev_layer[evi], 0));
+    return zero_bucket(c, evi, c->comm_st, c->opt_st, c->opt_fused);
+  }
   const int64_t b0 = bucket_begin(c, first), b1 = bucket_end(c, last);
   CK(cudaEventRecord(c->ev_layer[evi], c->st));
   cudaEvent_t ready = c->ev_layer[evi];
@@ -1361,10 +1406,41 @@ mimose_status mimose_init(const mimose_config* cfgp, mimose_ctx** out) {
     *out = c;   // returned so mimose_last_error works; caller destroys
     return s;
   }
+  if (k.zero1 && k.arena_base && k.world == 1 && !k.comm_force) {
+    mimose_status s = bad("zero1 needs a communicator (world > 1 or comm_force)");
+    *out = c;
+    return s;
+  }
   if (c->cfg.collect_iters <= 0) c->cfg.collect_iters = 10;
   c->dt = k.dtype == MIMOSE_FP32 ? DT_F32 : DT_BF16;
   c->e = k.dtype == MIMOSE_FP32 ? 4 : 2;
-  c->layout = build_layout(k, &c->npad);
+  c->zero1 = k.zero1 != 0;
+  c->layout = build_layout(k, &c->npad, c->zero1 ? 64LL * k.world : 64);
+  c->nshard = c->zero1 ? c->npad / k.world : c->npad;
+  {  // gradient buckets by event index: layer l -> l, head -> L, embedding -> L + 1
+    const int L = k.n_layers, lb = k.arch == 1 ? 2 : P_LAYER0;
+    c->bk_b0.assign(L + 2, 0);
+    c->bk_b1.assign(L + 2, 0);
+    c->bk_sh.assign(L + 2, 0);
+    for (int l = 0; l < L; ++l) {
+      c->bk_b0[l] = c->layout[lb + 12 * l].off;
+      c->bk_b1[l] = l + 1 < L ? c->layout[lb + 12 * (l + 1)].off : c->layout[lb + 12 * L].off;
+    }
+    c->bk_b0[L] = c->layout[lb + 12 * L].off;
+    c->bk_b1[L] = c->npad;
+    c->bk_b0[L + 1] = 0;
+    c->bk_b1[L + 1] = c->layout[lb].off;
+    const int W = c->zero1 ? k.world : 1;
+    int64_t sh = 0;
+    for (int i : {L + 1}) { c->bk_sh[i] = sh; sh += (c->bk_b1[i] - c->bk_b0[i]) / W; }
+    for (int l = 0; l < L; ++l) { c->bk_sh[l] = sh; sh += (c->bk_b1[l] - c->bk_b0[l]) / W; }
+    c->bk_sh[L] = sh;
+    sh += (c->bk_b1[L] - c->bk_b0[L]) / W;
+    if (sh != c->nshard) {
+      *out = c;
+      return bad("internal: ZeRO-1 shard layout mismatch");
+    }
+  }
   c->ws_elems = 4LL * k.hidden * k.hidden;   // wgrad split-K partials (oracle/memsim.py)
   c->device = k.arena_base != nullptr;
   Arena& a = c->ar;
@@ -1383,9 +1459,9 @@ mimose_status mimose_init(const mimose_config* cfgp, mimose_ctx** out) {
   auto take = [&](int64_t n) { char* p = a.base + off; off += a16(n); return p; };
   c->w = take(c->npad * c->e);
   c->grad = (float*)take(c->npad * 4);
-  if (c->dt != DT_F32) c->master = (float*)take(c->npad * 4);
-  c->m = (float*)take(c->npad * 4);
-  c->v = (float*)take(c->npad * 4);
+  if (c->dt != DT_F32) c->master = (float*)take(c->nshard * 4);   // ZeRO-1: this rank's shards only
+  c->m = (float*)take(c->nshard * 4);
+  c->v = (float*)take(c->nshard * 4);
   const int64_t maxT = (int64_t)k.max_seqs * k.max_seq_len;
   c->ids = (int32_t*)take(maxT * 4);
   c->tt = (int32_t*)take(maxT * 4);
@@ -1421,6 +1497,8 @@ mimose_status mimose_init(const mimose_config* cfgp, mimose_ctx** out) {
     CK(cudaMemsetAsync(a.base, 0, (size_t)a.C, c->st));
     c->ev_layer.resize(L + 2);
     c->ev_ar.resize(L + 2);
+    c->ev_upd.resize(L + 2);
+    for (auto& e : c->ev_upd) CK(cudaEventCreateWithFlags(&e, cudaEventDisableTiming));
     for (auto& e : c->ev_layer) CK(cudaEventCreateWithFlags(&e, cudaEventDisableTiming));
     for (auto& e : c->ev_ar) CK(cudaEventCreateWithFlags(&e, cudaEventDisableTiming));
     CK(cudaStreamCreateWithFlags(&c->opt_st, cudaStreamNonBlocking));
@@ -1456,6 +1534,7 @@ void mimose_destroy(mimose_ctx* c) {
     if (c->opt_st) cudaStreamSynchronize(c->opt_st);
     for (auto e : c->ev_layer) cudaEventDestroy(e);
     for (auto e : c->ev_ar) cudaEventDestroy(e);
+    for (auto e : c->ev_upd) cudaEventDestroy(e);
     for (auto e : c->probe_ev) cudaEventDestroy(e);
     if (c->ev_opt_done) cudaEventDestroy(c->ev_opt_done);
     if (c->opt_st) cudaStreamDestroy(c->opt_st);
@@ -1480,6 +1559,8 @@ static mimose_status xfer_params(mimose_ctx* c, float* host, int64_t n, int whic
   mimose_num_params(c, &tot);
   if (n != tot || !host) return fail(c, MIMOSE_E_INVALID, "blob size mismatch");
   if (!c->device) return fail(c, MIMOSE_E_NODEVICE, "host-only context");
+  if (which == 3 && c->zero1 && c->cfg.world > 1)
+    return fail(c, MIMOSE_E_INVALID, "ZeRO-1: the master copy is sharded over the ranks");
   if (c->opt_st) CK(cudaStreamSynchronize(c->opt_st));
   float* tmp = nullptr;
   CK(cudaMallocAsync((void**)&tmp, (size_t)c->npad * 4, c->st));
@@ -1489,9 +1570,20 @@ static mimose_status xfer_params(mimose_ctx* c, float* host, int64_t n, int whic
     for (auto& p : c->layout) { std::memcpy(&img[p.off], host + o, p.numel * 4); o += p.numel; }
     CK(cudaMemcpyAsync(tmp, img.data(), (size_t)c->npad * 4, cudaMemcpyHostToDevice, c->st));
     cast_from_f32(c->dt, tmp, c->w, c->npad, c->st);
-    if (c->master) CK(cudaMemcpyAsync(c->master, tmp, (size_t)c->npad * 4, cudaMemcpyDeviceToDevice, c->st));
-    CK(cudaMemsetAsync(c->m, 0, (size_t)c->npad * 4, c->st));
-    CK(cudaMemsetAsync(c->v, 0, (size_t)c->npad * 4, c->st));
+    if (c->master) {
+      if (!c->zero1) {
+        CK(cudaMemcpyAsync(c->master, tmp, (size_t)c->npad * 4, cudaMemcpyDeviceToDevice, c->st));
+      } else {   // this rank's shard of every bucket
+        const int W = c->cfg.world, r = c->cfg.rank;
+        for (size_t i = 0; i < c->bk_b0.size(); ++i) {
+          const int64_t cb = (c->bk_b1[i] - c->bk_b0[i]) / W;
+          CK(cudaMemcpyAsync(c->master + c->bk_sh[i], tmp + c->bk_b0[i] + r * cb, (size_t)cb * 4,
+                             cudaMemcpyDeviceToDevice, c->st));
+        }
+      }
+    }
+    CK(cudaMemsetAsync(c->m, 0, (size_t)c->nshard * 4, c->st));
+    CK(cudaMemsetAsync(c->v, 0, (size_t)c->nshard * 4, c->st));
     c->adam_t = 0;
   } else {
     if (which == 1 || (which == 3 && !c->master)) cast_to_f32(c->dt, c->w, tmp, c->npad, c->st);
@@ -1656,6 +1748,10 @@ mimose_status mimose_step(mimose_ctx* c, float lr, float b1, float b2, float eps
     // arguments say, then report a mismatch.
     CK(cudaEventRecord(c->ev_opt_done, c->opt_st));
     CK(cudaStreamWaitEvent(c->st, c->ev_opt_done, 0));
+    if (c->zero1) {   // the weight all-gathers follow the shard updates on the comm stream
+      CK(cudaEventRecord(c->ev_comm_done, c->comm_st));
+      CK(cudaStreamWaitEvent(c->st, c->ev_comm_done, 0));
+    }
     c->adam_t++;
     c->fwd_done = false;
     c->step_pending = false;
@@ -1667,6 +1763,24 @@ mimose_status mimose_step(mimose_ctx* c, float lr, float b1, float b2, float eps
   if (c->comm) {
     CK(cudaEventRecord(c->ev_comm_done, c->comm_st));
     CK(cudaStreamWaitEvent(c->st, c->ev_comm_done, 0));
+  }
+  if (c->zero1) {   // unfused ZeRO-1: shard updates + all-gathers, bucket by bucket, on the compute stream
+    c->opt_lr = lr; c->opt_b1 = b1; c->opt_b2 = b2; c->opt_eps = eps; c->opt_wd = wd;
+    for (int evi = 0; evi < (int)c->bk_b0.size(); ++evi) {
+      // the reduce-scatter already ran during backward; redo only the update + all-gather
+      const int W = c->cfg.world, r = c->cfg.rank;
+      const int64_t b0 = c->bk_b0[evi], cb = (c->bk_b1[evi] - b0) / W, sh = c->bk_sh[evi];
+      const double t = (double)(c->adam_t + 1);
+      const double bc1 = 1.0 - std::pow((double)b1, t), bc2 = 1.0 - std::pow((double)b2, t);
+      char* wsh = c->w + (b0 + r * cb) * c->e;
+      adamw(c->dt, wsh, c->master ? c->master + sh : nullptr, c->grad + b0 + r * cb, c->m + sh, c->v + sh, cb, lr, b1,
+            b2, eps, wd, (float)bc1, (float)bc2, 1.0f / (float)W, c->st);
+      NK(ncclAllGather(wsh, c->w + b0 * c->e, (size_t)cb, c->dt == DT_F32 ? ncclFloat : ncclBfloat16, c->comm,
+                       c->st));
+    }
+    c->adam_t++;
+    c->fwd_done = false;
+    return MIMOSE_OK;
   }
   c->adam_t++;
   const double bc1 = 1.0 - std::pow((double)b1, (double)c->adam_t);

@@ -62,11 +62,15 @@ def steps(cfg, params, fused, n=3, **kw):
 
 @pytest.mark.parametrize("case", list(CASES))
 @pytest.mark.parametrize("fused", [False, True])
-def test_nccl_allreduce_path_bitwise(case, fused):
+@pytest.mark.parametrize("zero1", [0, 1])
+def test_nccl_allreduce_path_bitwise(case, fused, zero1):
+    """zero1 = 1: the ZeRO-1 path -- per-bucket ncclReduceScatter,
+    AdamW on this rank's shard of master / m / v, ncclAllGather of the bf16
+    weights -- which at one rank must equal the unsharded step bit for bit."""
     cfg = CASES[case]
     params = wl.init_params(cfg, parity=True, seed=4)
     ref = steps(cfg, params, fused)
-    got = steps(cfg, params, fused, comm_force=1, check_plans=1)
+    got = steps(cfg, params, fused, comm_force=1, check_plans=1, zero1=zero1)
     st = got["stats"]
     assert st["comm_nranks"] == 1 and ref["stats"]["comm_nranks"] == 0
     # one bucket per encoder layer + head + embedding, every backward
@@ -119,3 +123,9 @@ def test_plan_check_detects_mismatch_is_noop_single_rank():
     ctx.step()
     assert ctx.stats()["plan_checks"] == 1
     ctx.close()
+
+
+def test_zero1_needs_a_communicator():
+    from paper_conf_ipps_liaolysshfyctzlq23_b200 import binding as mb
+    with pytest.raises(mb.MimoseError):
+        ctx_for(CASES["mc-bf16"], zero1=1)
