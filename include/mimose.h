@@ -121,6 +121,10 @@ typedef struct {
                             6 + 12 / world B/param.  Needs a communicator (world > 1 or
                             comm_force); mimose_get_master is then refused for world > 1. */
   int32_t reserved[1];
+  const int32_t* ffn_layers; /* heterogeneous stages: FFN width of each of the
+                            n_layers layers (multiples of 64, <= ffn; ffn is then the max
+                            and sizes the shared workspaces); NULL = every layer uses ffn.
+                            Read during mimose_init only.                             */
 } mimose_config;
 
 /* Fill defaults (collect_iters 10, ratio 9/10, degree 2, p 0.1, eps 1e-12,

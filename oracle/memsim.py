@@ -123,6 +123,11 @@ class Sizes:
     emb_scratch: int
     n_layers: int
     head_fwd_scratch: int = 0   # transient during the head forward (LM logits chunk)
+    per_layer: Optional[List[List[int]]] = None   # heterogeneous stages: internals of each layer
+
+    def ints(self, l: int) -> List[int]:
+        """Internals of layer l (they differ by stage only in the FFN tensors u, g)."""
+        return self.per_layer[l] if self.per_layer is not None else self.internals
 
     @property
     def i(self) -> int:
@@ -151,23 +156,29 @@ def sizes(cfg: ModelConfig, B: int, S: int, max_seqs: Optional[int] = None,
     # pre-LN sums z0, z1, z2 are fp32 in every mode (reading R-P: bf16 z loses
     # the row mean/spread balance that LayerNorm's backward needs)
     pre = cfg.arch == ARCH_PRE_LN
+    def layer_ints(Fl: int) -> List[int]:
+        if pre:
+            # GPT-2: the residual stream (x1, r1, y) is fp32; LN outputs a, m are the GEMM operands
+            return [a16(T * H * e), a16(T * 8), a16(T * 3 * H * e),          # a, st1, QKV
+                    a16(T * H * e), a16(B * h * S * 4),                       # O, LSE
+                    a16(T * H * 4), a16(T * 8), a16(T * H * e),               # r1, st2, m
+                    a16(T * Fl * e), a16(T * Fl * e)]                         # u, g
+        return [a16(T * 3 * H * e), a16(T * H * e), a16(B * h * S * 4),     # QKV, O, LSE
+                a16(T * H * 4), a16(T * 8), a16(T * H * e),                   # z1, st1, h1
+                a16(T * Fl * e), a16(T * Fl * e),                             # u, g
+                a16(T * H * 4), a16(T * 8)]                                   # z2, st2
+    # (heterogeneous stages: layer l's u, g use its own FFN width;
+    #  the backward layer scratch below is sized for the widest, F = cfg.ffn)
     if pre:
-        # GPT-2: the residual stream (x1, r1, y) is fp32; LN outputs a, m are the GEMM operands
         E = [a16(T * H * 4)]                                                   # x1
-        internals = [a16(T * H * e), a16(T * 8), a16(T * 3 * H * e),          # a, st1, QKV
-                     a16(T * H * e), a16(B * h * S * 4),                       # O, LSE
-                     a16(T * H * 4), a16(T * 8), a16(T * H * e),               # r1, st2, m
-                     a16(T * F * e), a16(T * F * e)]                           # u, g
         y = a16(T * H * 4)
     else:
         # pre-LN sums z0, z1, z2 are fp32 in every mode (reading R-P: bf16 z loses
         # the row mean/spread balance that LayerNorm's backward needs)
         E = [a16(T * H * 4), a16(T * 8), a16(T * H * e)]                       # z0, st0, x1
-        internals = [a16(T * 3 * H * e), a16(T * H * e), a16(B * h * S * 4),   # QKV, O, LSE
-                     a16(T * H * 4), a16(T * 8), a16(T * H * e),               # z1, st1, h1
-                     a16(T * F * e), a16(T * F * e),                           # u, g
-                     a16(T * H * 4), a16(T * 8)]                               # z2, st2
         y = a16(T * H * e)
+    internals = layer_ints(cfg.ffn_of(0))
+    per_layer = [layer_ints(cfg.ffn_of(l)) for l in range(cfg.n_layers)] if cfg.ffn_layers else None
     head_fwd = 0
     if cfg.head == HEAD_LM:
         VP = vpad(cfg.vocab)
@@ -185,7 +196,7 @@ def sizes(cfg: ModelConfig, B: int, S: int, max_seqs: Optional[int] = None,
     ntiles = (ms * mx + 1023) // 1024
     emb_scr = a16(T * H * 4) + a16(16 * T) + a16(4 * 256 * ntiles)   # dz0, 4 int32[T] sort arrays, digit histograms
     return Sizes(persistent_bytes(cfg, ms, mx, world, zero1), E, internals, y, head, dy, head_scr,
-                 layer_scr, emb_scr, cfg.n_layers, head_fwd)
+                 layer_scr, emb_scr, cfg.n_layers, head_fwd, per_layer)
 
 
 # --------------------------------------------------------------------------
@@ -243,13 +254,13 @@ def simulate_step(sz: Sizes, dropped: Sequence[int]) -> Arena:
         A.push(t)
     for l in range(L):                                   # forward
         if l in drop:                                    # no-save: internals transient
-            for t in sz.internals:
+            for t in sz.ints(l):
                 A.talloc(t)
             A.push(sz.y)
-            for t in reversed(sz.internals):
+            for t in reversed(sz.ints(l)):
                 A.tfree(t)
         else:
-            for t in sz.internals:
+            for t in sz.ints(l):
                 A.push(t)
             A.push(sz.y)
     for t in sz.head:
@@ -265,11 +276,11 @@ def simulate_step(sz: Sizes, dropped: Sequence[int]) -> Arena:
     A.pop(sz.y)                                          # y_L
     for l in reversed(range(L)):
         if l in drop:                                    # recompute before gradients
-            for t in sz.internals:
+            for t in sz.ints(l):
                 A.push(t)
         A.talloc(sz.layer_scratch)
         A.tfree(sz.layer_scratch)
-        for t in reversed(sz.internals):
+        for t in reversed(sz.ints(l)):
             A.pop(t)
         if l > 0:
             A.pop(sz.y)                                  # y_{l-1}: input of layer l
@@ -314,19 +325,19 @@ def collect_samples(sz: Sizes) -> Dict[str, object]:
         A.push(t)
     E = A.live - base
     a, y = [], []
-    for _ in range(L):
+    for l in range(L):
         b0 = A.live
-        for t in sz.internals:                           # pass 1: normal forward
+        for t in sz.ints(l):                             # pass 1: normal forward
             A.push(t)
         A.push(sz.y)
         a.append(A.live - b0)
         A.pop(sz.y)
-        for t in reversed(sz.internals):                 # discard output + activations
+        for t in reversed(sz.ints(l)):                   # discard output + activations
             A.pop(t)
-        for t in sz.internals:                           # pass 2: keep only the output
+        for t in sz.ints(l):                             # pass 2: keep only the output
             A.talloc(t)
         A.push(sz.y)
-        for t in reversed(sz.internals):
+        for t in reversed(sz.ints(l)):
             A.tfree(t)
         y.append(A.live - b0)
     b0 = A.live
@@ -347,11 +358,11 @@ def collect_samples(sz: Sizes) -> Dict[str, object]:
     A.pop(sz.y)
     A.top_peak_phase = sum(A.top)
     for l in reversed(range(L)):
-        for t in sz.internals:
+        for t in sz.ints(l):
             A.push(t)
         A.talloc(sz.layer_scratch)
         A.tfree(sz.layer_scratch)
-        for t in reversed(sz.internals):
+        for t in reversed(sz.ints(l)):
             A.pop(t)
         if l > 0:
             A.pop(sz.y)
@@ -389,10 +400,10 @@ def unit_list(sz: Sizes) -> List[tuple]:
     """[(internals, output)] for the 2L units of a stack (both layer types keep
     10 internals whose 6th is the block boundary h1 / r1)."""
     assert len(sz.internals) == 10
-    att, h1, ffn = sz.internals[:5], sz.internals[5], sz.internals[6:]
     out = []
-    for _ in range(sz.n_layers):
-        out += [(att, h1), (ffn, sz.y)]
+    for l in range(sz.n_layers):
+        ints = sz.ints(l)
+        out += [(ints[:5], ints[5]), (ints[6:], sz.y)]
     return out
 
 

@@ -46,7 +46,7 @@ class Config(C.Structure):
                 ("rank", C.c_int32), ("world", C.c_int32), ("nccl_id", C.c_void_p),
                 ("use_tc", C.c_int32), ("pad_id", C.c_int32), ("granularity", C.c_int32),
                 ("comm_force", C.c_int32), ("nccl_max_ctas", C.c_int32), ("check_plans", C.c_int32),
-                ("zero1", C.c_int32), ("reserved", C.c_int32 * 1)]
+                ("zero1", C.c_int32), ("reserved", C.c_int32 * 1), ("ffn_layers", C.c_void_p)]
 
 
 class BatchS(C.Structure):
@@ -217,6 +217,10 @@ def make_config(cfg: wl.ModelConfig, **kw) -> Config:
     c.seed = wl.dropout_seed(cfg)
     c.max_seqs, c.max_seq_len = cfg.n_seqs, cfg.max_seq
     c.pad_id = cfg.pad_id
+    if cfg.ffn_layers:                       # heterogeneous stages: per-layer FFN widths
+        arr = (C.c_int32 * cfg.n_layers)(*cfg.ffn_layers)
+        c._ffn_keep = arr                    # alive until mimose_init has copied it
+        c.ffn_layers = C.cast(arr, C.c_void_p)
     for k, v in kw.items():
         setattr(c, k, v)
     return c

@@ -46,7 +46,8 @@ inline int64_t vpad(int64_t v) { return (v + 7) / 8 * 8; }
 // shards.
 std::vector<ParamInfo> build_layout(const mimose_config& c, int64_t* npad, int64_t unit = 64) {
   std::vector<int64_t> n;
-  const int64_t H = c.hidden, F = c.ffn;
+  const int64_t H = c.hidden;
+  auto Fof = [&](int l) -> int64_t { return c.ffn_layers ? c.ffn_layers[l] : c.ffn; };
   auto lay = [&](int n_emb) {
     std::vector<ParamInfo> out;
     int64_t off = 0;
@@ -64,6 +65,7 @@ std::vector<ParamInfo> build_layout(const mimose_config& c, int64_t* npad, int64
     n.push_back((int64_t)c.vocab * H);
     n.push_back((int64_t)c.max_pos * H);
     for (int l = 0; l < c.n_layers; ++l) {
+      const int64_t F = Fof(l);
       const int64_t v[12] = {H, H, 3 * H * H, 3 * H, H * H, H, H, H, F * H, F, H * F, H};
       for (int64_t x : v) n.push_back(x);
     }
@@ -77,6 +79,7 @@ std::vector<ParamInfo> build_layout(const mimose_config& c, int64_t* npad, int64
   n.push_back(H);
   n.push_back(H);
   for (int l = 0; l < c.n_layers; ++l) {
+    const int64_t F = Fof(l);
     const int64_t v[12] = {3 * H * H, 3 * H, H * H, H, H, H, F * H, F, H * F, H, H, H};
     for (int64_t x : v) n.push_back(x);
   }
@@ -196,6 +199,7 @@ struct mimose_ctx {
   bool fwd_done = false, bwd_done = false, collecting = false;
   bool step_pending = false;   // fused optimizer: backward applied the update, mimose_step not yet called
   // ZeRO-1: optimizer state (master, m, v) sharded over the ranks
+  std::vector<int> ffn_l;                    // per-layer FFN widths (empty: uniform cfg.ffn)
   bool zero1 = false;
   int64_t nshard = 0;                        // elements of master / m / v on this rank
   std::vector<int64_t> bk_b0, bk_b1, bk_sh;  // per bucket (event index): [b0, b1) and shard offset
@@ -327,6 +331,8 @@ Drop make_drop(const mimose_ctx* c, uint32_t kind, uint32_t layer) {
 Drop no_drop() { Drop d{}; d.enabled = 0; return d; }
 
 inline char* W(mimose_ctx* c, int i) { return c->w + c->layout[i].off * c->e; }
+// FFN width of layer l (heterogeneous stages: mimose_config.ffn_layers).
+inline int Fl(const mimose_ctx* c, int l) { return c->ffn_l.empty() ? c->cfg.ffn : c->ffn_l[l]; }
 inline float* G(mimose_ctx* c, int i) { return c->grad + c->layout[i].off; }
 // Parameter index of semantic slot k (L_*) of layer l.  Post-LN order is the
 // L_* enum order; GPT-2 (pre-LN) stores [ln1, qkv, o, ln2, f1, f2].
@@ -401,7 +407,7 @@ void att_forward(Run& r, int l, const char* x, LayerBufs& b, char* h1out) {
 void ffn_forward(Run& r, int l, LayerBufs& b, char* yout) {
   mimose_ctx* c = r.c;
   if (!r.real) return;
-  const int T = c->T, H = c->cfg.hidden, F = c->cfg.ffn;
+  const int T = c->T, H = c->cfg.hidden, F = Fl(c, l);
   GemmArgs g;
   // u = h1 W1^T + b1, g = gelu(u)
   g = GemmArgs();
@@ -477,6 +483,13 @@ void free_ffn(Run& r, bool on_stack) {
   const int64_t s1[4] = {r.z.st2, r.z.m, r.z.u, r.z.g};
   const int64_t* s = r.c->cfg.arch == 1 ? s1 : s0;
   for (int i = 3; i >= 0; --i) on_stack ? a.pop(s[i]) : a.tfree(s[i]);
+}
+
+// Per-layer sizes: only the FFN internals u, g depend on the layer (its FFN
+// width F_l, heterogeneous stages); the layer scratch is sized for max F.
+void set_layer(Run& r, int l) {
+  const int64_t T = (int64_t)r.c->B * r.c->S;
+  r.z.u = r.z.g = a16(T * Fl(r.c, l) * r.c->e);
 }
 
 void free_internals(Run& r, bool on_stack) {
@@ -627,7 +640,7 @@ void dgrad(Run& r, Epi epi, const void* dY, int Nout, const void* Wt, int Kin, v
 void ffn_backward(Run& r, int l, LayerBufs& b, float* dy, char* scr) {
   mimose_ctx* c = r.c;
   if (!r.real) return;
-  const int T = c->T, H = c->cfg.hidden, F = c->cfg.ffn;
+  const int T = c->T, H = c->cfg.hidden, F = Fl(c, l);
   float* dres = (float*)(scr + r.z.r_dres);
   char* R2 = scr + r.z.r_du;     // du, later dO
   char* R3 = scr + r.z.r_dt;     // dt2 / dt1, later dQKV
@@ -727,7 +740,7 @@ void att_forward_pre(Run& r, int l, const float* x, LayerBufs& b, float* r1out) 
 void ffn_forward_pre(Run& r, int l, LayerBufs& b, float* yout) {
   mimose_ctx* c = r.c;
   if (!r.real) return;
-  const int T = c->T, H = c->cfg.hidden, F = c->cfg.ffn;
+  const int T = c->T, H = c->cfg.hidden, F = Fl(c, l);
   GemmArgs g;
   ln_fwd(c->dt, b.r1, W(c, LP(c, l, L_LN2G)), W(c, LP(c, l, L_LN2B)), b.m, b.st2, T, H, c->cfg.ln_eps, r.st);
   g = GemmArgs();
@@ -755,7 +768,7 @@ void layer_forward_pre(Run& r, int l, const float* x, LayerBufs& b, float* yout)
 void ffn_backward_pre(Run& r, int l, LayerBufs& b, float* dy, char* scr) {
   mimose_ctx* c = r.c;
   if (!r.real) return;
-  const int T = c->T, H = c->cfg.hidden, F = c->cfg.ffn;
+  const int T = c->T, H = c->cfg.hidden, F = Fl(c, l);
   float* dres = (float*)(scr + r.z.r_dres);
   char* R2 = scr + r.z.r_du;     // du, later dO
   char* R3 = scr + r.z.r_dt;     // dt2 / dt1, later dQKV
@@ -1036,6 +1049,7 @@ void run_forward(Run& r, uint64_t mask, bool collect, Sample* sample) {
   c->y.assign(L, nullptr);
   const char* x = c->x1;
   for (int l = 0; l < L && c->cfg.granularity == 1; ++l) {   // sub-layer units 2l (attention), 2l+1 (FFN)
+    set_layer(r, l);
     LayerBufs& b = c->lb[l];
     const int ua = 2 * l, uf = 2 * l + 1;
     int64_t b0 = a.live();
@@ -1079,6 +1093,7 @@ void run_forward(Run& r, uint64_t mask, bool collect, Sample* sample) {
     x = c->y[l];
   }
   for (int l = 0; l < L && c->cfg.granularity == 0; ++l) {
+    set_layer(r, l);
     const int64_t b0 = a.live();
     if (collect && sample) {
       // pass 1: normal forward (save mode), timed; output and activations discarded
@@ -1173,6 +1188,7 @@ mimose_status run_backward(Run& r, Sample* sample) {
   // ---- layers ----
   a.top_phase_peak = a.top;
   for (int l = L - 1; l >= 0 && c->cfg.granularity == 1; --l) {   // sub-layer units
+    set_layer(r, l);
     LayerBufs& b = c->lb[l];
     const char* x = l > 0 ? c->y[l - 1] : c->x1;
     if ((c->drop_mask >> (2 * l + 1)) & 1) {          // recompute the FFN block from h1 / r1
@@ -1197,6 +1213,7 @@ mimose_status run_backward(Run& r, Sample* sample) {
     if (l > 0) a.pop(r.z.y);                          // y_{l-1}: input of layer l
   }
   for (int l = L - 1; l >= 0 && c->cfg.granularity == 0; --l) {
+    set_layer(r, l);
     const bool dropped = (c->drop_mask >> l) & 1;
     const char* x = l > 0 ? c->y[l - 1] : c->x1;
     if (dropped) {                                    // recompute right before the gradients
@@ -1414,9 +1431,21 @@ mimose_status mimose_init(const mimose_config* cfgp, mimose_ctx** out) {
   if (c->cfg.collect_iters <= 0) c->cfg.collect_iters = 10;
   c->dt = k.dtype == MIMOSE_FP32 ? DT_F32 : DT_BF16;
   c->e = k.dtype == MIMOSE_FP32 ? 4 : 2;
+  if (k.ffn_layers) {
+    for (int l = 0; l < k.n_layers; ++l) {
+      const int f = k.ffn_layers[l];
+      if (f < 64 || f % 64 || f > k.ffn) {
+        mimose_status s = bad("ffn_layers[l] must be a multiple of 64 in [64, ffn]");
+        *out = c;
+        return s;
+      }
+      c->ffn_l.push_back(f);
+    }
+  }
   c->zero1 = k.zero1 != 0;
   c->layout = build_layout(k, &c->npad, c->zero1 ? 64LL * k.world : 64);
   c->nshard = c->zero1 ? c->npad / k.world : c->npad;
+  c->cfg.ffn_layers = nullptr;   // copied into ffn_l; the caller's array need not outlive init
   {  // gradient buckets by event index: layer l -> l, head -> L, embedding -> L + 1
     const int L = k.n_layers, lb = k.arch == 1 ? 2 : P_LAYER0;
     c->bk_b0.assign(L + 2, 0);

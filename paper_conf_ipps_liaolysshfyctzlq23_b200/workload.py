@@ -57,6 +57,11 @@ class ModelConfig:
     pad_id: int
     first_tok: int
     arch: int = ARCH_POST_LN
+    # heterogeneous stages: FFN width of every layer; () = ffn everywhere
+    ffn_layers: Tuple[int, ...] = ()
+
+    def ffn_of(self, l: int) -> int:
+        return self.ffn_layers[l] if self.ffn_layers else self.ffn
 
     @property
     def causal(self) -> bool:
@@ -122,6 +127,15 @@ CONFIGS: Dict[str, ModelConfig] = {
     "gpt2-medium": ModelConfig("gpt2-medium", 4, 24, 1024, 16, 4096, 50257, 1024, 0, 0,
                                HEAD_LM, 1, 2, "bf16", 1e-5, 0.1, 8, 256, 1024, 8, 0.4,
                                50256, 50256, 50256, 0, ARCH_PRE_LN),
+    # heterogeneous stages.  A synthetic BERT-base-width
+    # encoder whose three 4-layer stages differ in FFN width (4096 / 3072 / 1536),
+    # so the per-layer activation size falls stage by stage (1.15 : 1 : 0.78 per
+    # token) as in Swin or ResNet, whose first stage holds the largest
+    # activations (Fig. 9); SWAG-like MC batches, the BERT-base
+    # length schedule, budget 60%.
+    "hetero": ModelConfig("hetero", 5, 12, 768, 12, 4096, 30522, 512, 2, 0,
+                          HEAD_MC, 4, 2, "bf16", 1e-12, 0.1, 64, 32, 128, 8, 0.6,
+                          101, 102, 0, 103, ARCH_POST_LN, (4096,) * 4 + (3072,) * 4 + (1536,) * 4),
 }
 
 
@@ -142,6 +156,7 @@ def param_spec(cfg: ModelConfig) -> List[Tuple[str, Tuple[int, ...]]]:
         spec = [("emb.word", (V, H)), ("emb.pos", (P, H))]
         for l in range(cfg.n_layers):
             p = f"layer{l}."
+            F = cfg.ffn_of(l)
             spec += [
                 (p + "ln1.g", (H,)), (p + "ln1.b", (H,)),
                 (p + "qkv.w", (3 * H, H)), (p + "qkv.b", (3 * H,)),
@@ -158,6 +173,7 @@ def param_spec(cfg: ModelConfig) -> List[Tuple[str, Tuple[int, ...]]]:
     ]
     for l in range(cfg.n_layers):
         p = f"layer{l}."
+        F = cfg.ffn_of(l)
         spec += [
             (p + "qkv.w", (3 * H, H)), (p + "qkv.b", (3 * H,)),
             (p + "o.w", (H, H)), (p + "o.b", (H,)),

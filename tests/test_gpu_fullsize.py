@@ -35,6 +35,8 @@ FULL = {
     "bl-s512": (wl.small_config("bert-large", n_layers=2), 512, [0]),
     # RoBERTa-large MC, S_max = 512 (16 sequences = 4 questions: bounds the fp64 oracle's RAM)
     "rl-s512": (wl.small_config("roberta-large", n_layers=2, n_seqs=16), 512, [0]),
+    # heterogeneous stages: BERT-base width, one layer per stage, FFN 4096 / 3072 / 1536
+    "hetero-s128": (wl.small_config("hetero", n_layers=3, ffn_layers=(4096, 3072, 1536)), 128, [0, 1]),
     # GPT-2 medium, causal, tied 50257-word LM head, S_max = 1024 (2 sequences)
     "g2-s1024": (wl.small_config("gpt2-medium", n_layers=2, n_seqs=2), 1024, [1]),
 }

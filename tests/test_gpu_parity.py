@@ -99,6 +99,9 @@ CASES = {
     "lm-gpt2-bf16-xlong": wl.small_config("gpt2-medium", n_layers=2, hidden=128, heads=2, ffn=256, vocab=600,
                                           max_pos=640, n_seqs=1, seq_lo=500, seq_hi=632, pad=8, pad_id=599,
                                           cls_id=599, sep_id=599),
+    # heterogeneous stages: per-layer FFN widths 384 / 256 / 128
+    "hetero-bf16": wl.small_config("hetero", n_layers=3, hidden=128, heads=2, ffn=384, ffn_layers=(384, 256, 128),
+                                   vocab=500, max_pos=64, n_seqs=8, seq_lo=8, seq_hi=40, pad=8),
     "lm-gpt2-fp32": wl.small_config("gpt2-medium", n_layers=2, hidden=64, heads=2, ffn=128, vocab=300,
                                     max_pos=64, n_seqs=3, seq_lo=10, seq_hi=50, pad=1, pad_id=299,
                                     cls_id=299, sep_id=299, dtype="fp32"),
@@ -129,7 +132,8 @@ def test_step_parity_against_oracle(case):
         pm.check(f"{case}-step{step}", cfg, grads_dict(cfg, g), G, loss, ref_loss, emulator(cfg, W, b, it))
 
 
-@pytest.mark.parametrize("case", ["toy-fp32", "mc-bf16", "qa-bf16", "lm-gpt2-bf16", "lm-gpt2-bf16-long"])
+@pytest.mark.parametrize("case", ["toy-fp32", "mc-bf16", "qa-bf16", "lm-gpt2-bf16", "lm-gpt2-bf16-long",
+                                  "hetero-bf16"])
 def test_recompute_replay_bitwise(case):
     cfg = CASES[case]
     params = wl.init_params(cfg, parity=True, seed=3)
@@ -149,8 +153,9 @@ def test_recompute_replay_bitwise(case):
         ctx.close()
 
 
-def test_collector_samples_and_budget_on_gpu():
-    cfg = CASES["mc-bf16"]
+@pytest.mark.parametrize("case", ["mc-bf16", "hetero-bf16"])
+def test_collector_samples_and_budget_on_gpu(case):
+    cfg = CASES[case]
     sz = om.sizes(cfg, cfg.n_seqs, cfg.max_seq)
     M = max(sz.C + int(0.6 * (om.no_ckpt_peak(sz) - sz.C)), om.lower_bound(sz))
     ctx = make_ctx(cfg, budget=M)
