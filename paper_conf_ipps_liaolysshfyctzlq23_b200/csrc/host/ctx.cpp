@@ -200,6 +200,11 @@ struct mimose_ctx {
   bool step_pending = false;   // fused optimizer: backward applied the update, mimose_step not yet called
   // ZeRO-1: optimizer state (master, m, v) sharded over the ranks
   std::vector<int> ffn_l;                    // per-layer FFN widths (empty: uniform cfg.ffn)
+  // Side stream for the weight-gradient reductions that nothing on the
+  // backward's critical path reads (LN-partial and bias column sums)
+  cudaStream_t aux_st = nullptr;
+  cudaEvent_t ev_fork = nullptr, ev_join = nullptr;
+  bool aux_pending = false;
   bool zero1 = false;
   int64_t nshard = 0;                        // elements of master / m / v on this rank
   std::vector<int64_t> bk_b0, bk_b1, bk_sh;  // per bucket (event index): [b0, b1) and shard offset
@@ -333,6 +338,37 @@ Drop no_drop() { Drop d{}; d.enabled = 0; return d; }
 inline char* W(mimose_ctx* c, int i) { return c->w + c->layout[i].off * c->e; }
 // FFN width of layer l (heterogeneous stages: mimose_config.ffn_layers).
 inline int Fl(const mimose_ctx* c, int l) { return c->ffn_l.empty() ? c->cfg.ffn : c->ffn_l[l]; }
+
+// Off-critical-path reductions: fork() orders the side stream after the work
+// issued so far on `st` and returns it; join() makes `st` wait for everything
+// issued on the side stream (called before a buffer the side stream reads or
+// writes is reused: the LN partials, the bias-colsum partials, R2 / R3).
+// MIMOSE_AUX=0 keeps every reduction on the compute stream (A/B).
+bool aux_enabled(const mimose_ctx* c) {
+  static const int v = [] {
+    const char* e = std::getenv("MIMOSE_AUX");
+    return e ? std::atoi(e) : 1;
+  }();
+  return v != 0 && c->aux_st != nullptr;
+}
+cudaStream_t fork(mimose_ctx* c, cudaStream_t st) {
+  if (!aux_enabled(c)) return st;
+  cudaEventRecord(c->ev_fork, st);
+  cudaStreamWaitEvent(c->aux_st, c->ev_fork, 0);
+  c->aux_pending = true;
+  return c->aux_st;
+}
+void join(mimose_ctx* c, cudaStream_t st) {
+  if (!c->aux_pending) return;
+  cudaEventRecord(c->ev_join, c->aux_st);
+  cudaStreamWaitEvent(st, c->ev_join, 0);
+  c->aux_pending = false;
+}
+// The LN partials use the first NPART x max(3H, F) floats of c->part, the
+// bias column-sum partials the second.
+inline float* part_cs(const mimose_ctx* c) {
+  return c->part + (int64_t)NPART * std::max<int64_t>(3LL * c->cfg.hidden, (int64_t)c->cfg.ffn);
+}
 inline float* G(mimose_ctx* c, int i) { return c->grad + c->layout[i].off; }
 // Parameter index of semantic slot k (L_*) of layer l.  Post-LN order is the
 // L_* enum order; GPT-2 (pre-LN) stores [ln1, qkv, o, ln2, f1, f2].
@@ -647,20 +683,24 @@ void ffn_backward(Run& r, int l, LayerBufs& b, float* dy, char* scr) {
   float* pg = c->part;
   float* pb = c->part + (int64_t)NPART * H;
   float* pbias = c->part + 2LL * NPART * H;
+  join(c, r.st);                 // the previous layer's side reductions read R3 and the partials
   // LN2 backward + dropout backward -> dz2 (dres), dt2 (R3), partials
   ln_bwd(c->dt, dy, no_drop(), b.z2, b.st2, W(c, LP(c, l, L_LN2G)), dres, R3, make_drop(c, KIND_FFN_OUT, l),
          pg, pb, pbias, T, H, r.st);
   reduce_rows3(pg, G(c, LP(c, l, L_LN2G)), pb, G(c, LP(c, l, L_LN2B)), pbias, G(c, LP(c, l, L_F2B)), NPART, H, H,
-               r.st);
+               fork(c, r.st));
   // FFN2: du = (dt2 W2) * gelu'(u)
   dgrad(r, EPI_GELU_BWD, R3, H, W(c, LP(c, l, L_F2W)), F, R2, b.u);
+  // db1 = colsum du, beside the FFN1 dgrad and the weight gradients
+  {
+    cudaStream_t sa = fork(c, r.st);
+    colsum(c->dt, R2, T, F, part_cs(c), sa);
+    reduce_partials(part_cs(c), F, F, G(c, LP(c, l, L_F1B)), sa);
+  }
   // FFN1: dh1 = du W1 + dz2 (in place in dres)
   dgrad(r, EPI_ACC_RES_F32, R2, F, W(c, LP(c, l, L_F1W)), H, dres, dres);
   // dW2 = dt2^T g and dW1 = du^T h1 together (dt2 in R3 lives until LN1 backward)
   wgrad2(r, R3, H, b.g, F, G(c, LP(c, l, L_F2W)), R2, F, b.h1, H, G(c, LP(c, l, L_F1W)));
-  // db1 = colsum du
-  colsum(c->dt, R2, T, F, c->part, r.st);
-  reduce_partials(c->part, F, F, G(c, LP(c, l, L_F1B)), r.st);
 }
 
 // Attention-block gradients of a post-LN layer (after ffn_backward; dres = dh1).
@@ -679,25 +719,30 @@ void att_backward(Run& r, int l, const char* x, LayerBufs& b, float* dy, char* s
   // that it outlives the attention backward and dWo can be grouped with dWqkv
   const bool spare = c->cfg.ffn >= 2 * H;
   char* DT1 = spare ? R2 + a16((int64_t)T * H * c->e) : R3;
+  join(c, r.st);                 // LN2 partials reduced and du summed before LN1 / dO reuse them
   // LN1 backward + dropout backward -> dz1 (dres, in place), dt1 (DT1)
   ln_bwd(c->dt, dres, no_drop(), b.z1, b.st1, W(c, LP(c, l, L_LN1G)), dres, DT1, make_drop(c, KIND_ATTN_OUT, l),
          pg, pb, pbias, T, H, r.st);
   reduce_rows3(pg, G(c, LP(c, l, L_LN1G)), pb, G(c, LP(c, l, L_LN1B)), pbias, G(c, LP(c, l, L_OB)), NPART, H, H,
-               r.st);
+               fork(c, r.st));
   // out-proj: dO = dt1 Wo (R2)
   dgrad(r, EPI_STORE, DT1, H, W(c, LP(c, l, L_OW)), H, R2, nullptr);
   if (!spare) wgrad(r, DT1, H, b.O, H, G(c, LP(c, l, L_OW)));     // dWo = dt1^T O before R3 is reused
   // attention backward -> dQKV (R3)
   attn_bwd(c->dt, b.qkv, b.O, R2, b.lse, c->lens, Dbuf, R3, c->B, c->S, H, h, make_drop(c, KIND_ATTN_PROBS, l), r.st);
+  // dbqkv = colsum dQKV, beside the QKV dgrad and the weight gradients
+  {
+    cudaStream_t sa = fork(c, r.st);
+    colsum(c->dt, R3, T, 3 * H, part_cs(c), sa);
+    reduce_partials(part_cs(c), 3 * H, 3 * H, G(c, LP(c, l, L_QKVB)), sa);
+  }
   // QKV: dx = dQKV Wqkv + dz1 -> dy buffer
   dgrad(r, EPI_ACC_RES_F32, R3, 3 * H, W(c, LP(c, l, L_QKVW)), H, dy, dres);
-  // dWo = dt1^T O and dWqkv = dQKV^T x; dbqkv = colsum dQKV
+  // dWo = dt1^T O and dWqkv = dQKV^T x
   if (spare)
     wgrad2(r, DT1, H, b.O, H, G(c, LP(c, l, L_OW)), R3, 3 * H, x, H, G(c, LP(c, l, L_QKVW)));
   else
     wgrad(r, R3, 3 * H, x, H, G(c, LP(c, l, L_QKVW)));
-  colsum(c->dt, R3, T, 3 * H, c->part, r.st);
-  reduce_partials(c->part, 3 * H, 3 * H, G(c, LP(c, l, L_QKVB)), r.st);
 }
 
 void layer_backward(Run& r, int l, const char* x, LayerBufs& b, float* dy, char* scr) {
@@ -776,9 +821,10 @@ void ffn_backward_pre(Run& r, int l, LayerBufs& b, float* dy, char* scr) {
   float* pg = c->part;
   float* pb = c->part + (int64_t)NPART * H;
   float* pbias = c->part + 2LL * NPART * H;
+  join(c, r.st);                 // the previous layer's side reductions read R3 and the partials
   // dt2 = dy * mask (bf16), db2 = colsum dt2
   drop_cast_colsum(c->dt, dy, make_drop(c, KIND_FFN_OUT, l), R3, T, H, pbias, r.st);
-  reduce_partials(pbias, H, H, G(c, LP(c, l, L_F2B)), r.st);
+  reduce_partials(pbias, H, H, G(c, LP(c, l, L_F2B)), fork(c, r.st));
   // FFN2: du = (dt2 W2) * gelu_tanh'(u); dW2 = dt2^T g
   {
     GemmArgs g;
@@ -791,16 +837,20 @@ void ffn_backward_pre(Run& r, int l, LayerBufs& b, float* dy, char* scr) {
   wgrad(r, R3, H, b.g, F, G(c, LP(c, l, L_F2W)));
   // FFN1: dm = du W1 (fp32, dres); dW1 = du^T m; db1
   dgrad(r, EPI_F32, R2, F, W(c, LP(c, l, L_F1W)), H, dres, nullptr);
+  {
+    cudaStream_t sa = fork(c, r.st);
+    colsum(c->dt, R2, T, F, part_cs(c), sa);
+    reduce_partials(part_cs(c), F, F, G(c, LP(c, l, L_F1B)), sa);
+  }
   wgrad(r, R2, F, b.m, H, G(c, LP(c, l, L_F1W)));
-  colsum(c->dt, R2, T, F, c->part, r.st);
-  reduce_partials(c->part, F, F, G(c, LP(c, l, L_F1B)), r.st);
+  join(c, r.st);                 // pbias reduced, du summed before LN2 / DT1 reuse them
   // LN2 backward + residual: dr1 = dy + LN2'(dm) (in place in dy); dt1 = dr1 * mask (DT1: the
   // spare tail of R2 when F >= 2H, so it outlives the dQKV write into R3, else R3)
   char* DT1 = F >= 2 * H ? R2 + a16((int64_t)T * H * c->e) : R3;
   ln_bwd(c->dt, dres, no_drop(), b.r1, b.st2, W(c, LP(c, l, L_LN2G)), dy, DT1, make_drop(c, KIND_ATTN_OUT, l),
          pg, pb, pbias, T, H, r.st, dy);
   reduce_rows3(pg, G(c, LP(c, l, L_LN2G)), pb, G(c, LP(c, l, L_LN2B)), pbias, G(c, LP(c, l, L_OB)), NPART, H, H,
-               r.st);
+               fork(c, r.st));
 }
 
 // Attention-block gradients of a pre-LN layer (after ffn_backward_pre: dy = dr1, R3 = dt1).
@@ -821,18 +871,23 @@ void att_backward_pre(Run& r, int l, const float* x, LayerBufs& b, float* dy, ch
   if (!spare) wgrad(r, DT1, H, b.O, H, G(c, LP(c, l, L_OW)));
   attn_bwd(c->dt, b.qkv, b.O, R2, b.lse, c->lens, Dbuf, R3, c->B, c->S, H, h, make_drop(c, KIND_ATTN_PROBS, l),
            r.st, true);
-  // QKV: da = dQKV Wqkv (fp32, dres); dWo = dt1^T O with dWqkv = dQKV^T a (grouped); dbqkv
+  // QKV: da = dQKV Wqkv (fp32, dres); dWo = dt1^T O with dWqkv = dQKV^T a (grouped); dbqkv on the side
+  {
+    cudaStream_t sa = fork(c, r.st);
+    colsum(c->dt, R3, T, 3 * H, part_cs(c), sa);
+    reduce_partials(part_cs(c), 3 * H, 3 * H, G(c, LP(c, l, L_QKVB)), sa);
+  }
   dgrad(r, EPI_F32, R3, 3 * H, W(c, LP(c, l, L_QKVW)), H, dres, nullptr);
   if (spare)
     wgrad2(r, DT1, H, b.O, H, G(c, LP(c, l, L_OW)), R3, 3 * H, b.a, H, G(c, LP(c, l, L_QKVW)));
   else
     wgrad(r, R3, 3 * H, b.a, H, G(c, LP(c, l, L_QKVW)));
-  colsum(c->dt, R3, T, 3 * H, c->part, r.st);
-  reduce_partials(c->part, 3 * H, 3 * H, G(c, LP(c, l, L_QKVB)), r.st);
+  join(c, r.st);                 // LN2 partials reduced before LN1's partials overwrite them
   // LN1 backward + residual: dx = dr1 + LN1'(da) (in place in dy)
   ln_bwd(c->dt, dres, no_drop(), x, b.st1, W(c, LP(c, l, L_LN1G)), dy, nullptr, no_drop(), pg, pb, nullptr, T, H,
          r.st, dy);
-  reduce_rows3(pg, G(c, LP(c, l, L_LN1G)), pb, G(c, LP(c, l, L_LN1B)), nullptr, nullptr, NPART, H, H, r.st);
+  reduce_rows3(pg, G(c, LP(c, l, L_LN1G)), pb, G(c, LP(c, l, L_LN1B)), nullptr, nullptr, NPART, H, H,
+               fork(c, r.st));
 }
 
 void layer_backward_pre(Run& r, int l, const float* x, LayerBufs& b, float* dy, char* scr) {
@@ -934,14 +989,20 @@ mimose_status zero_bucket(mimose_ctx* c, int evi, cudaStream_t st_rs, cudaStream
 
 mimose_status allreduce_bucket(mimose_ctx* c, int first, int last, int evi) {
   if (!c->device || (!c->comm && !c->opt_fused)) return MIMOSE_OK;
+  // the bucket is final once the compute stream AND the side reductions
+  // (its bias / LN gradients) are done
+  const bool side = c->aux_pending;
+  if (side) CK(cudaEventRecord(c->ev_join, c->aux_st));
   if (c->zero1) {
     CK(cudaEventRecord(c->ev_layer[evi], c->st));
     CK(cudaStreamWaitEvent(c->comm_st, c->ev_layer[evi], 0));
+    if (side) CK(cudaStreamWaitEvent(c->comm_st, c->ev_join, 0));
     return zero_bucket(c, evi, c->comm_st, c->opt_st, c->opt_fused);
   }
   const int64_t b0 = bucket_begin(c, first), b1 = bucket_end(c, last);
   CK(cudaEventRecord(c->ev_layer[evi], c->st));
   cudaEvent_t ready = c->ev_layer[evi];
+  if (side) CK(cudaStreamWaitEvent(c->comm ? c->comm_st : c->opt_st, c->ev_join, 0));
   if (c->comm) {
     c->stats_allreduce_calls++;
     c->stats_allreduce_bytes += (b1 - b0) * 4;
@@ -1231,6 +1292,7 @@ mimose_status run_backward(Run& r, Sample* sample) {
     if (l > 0) a.pop(r.z.y);                          // y_{l-1}: input of layer l
   }
   if (sample) sample->Tb = a.top_phase_peak;
+  if (r.real) join(c, r.st);                          // the partials buffer is reused below
   // ---- embedding ----
   a.top_phase_peak = a.top;
   char* es = a.talloc(r.z.emb_scr);
@@ -1531,6 +1593,9 @@ mimose_status mimose_init(const mimose_config* cfgp, mimose_ctx** out) {
     for (auto& e : c->ev_layer) CK(cudaEventCreateWithFlags(&e, cudaEventDisableTiming));
     for (auto& e : c->ev_ar) CK(cudaEventCreateWithFlags(&e, cudaEventDisableTiming));
     CK(cudaStreamCreateWithFlags(&c->opt_st, cudaStreamNonBlocking));
+    CK(cudaStreamCreateWithFlags(&c->aux_st, cudaStreamNonBlocking));
+    CK(cudaEventCreateWithFlags(&c->ev_fork, cudaEventDisableTiming));
+    CK(cudaEventCreateWithFlags(&c->ev_join, cudaEventDisableTiming));
     CK(cudaEventCreateWithFlags(&c->ev_opt_done, cudaEventDisableTiming));
     if (k.world > 1 || k.comm_force) {
       if (k.world > 1 && !k.nccl_id) { *out = c; return bad("world > 1 needs nccl_id"); }
@@ -1567,6 +1632,9 @@ void mimose_destroy(mimose_ctx* c) {
     for (auto e : c->probe_ev) cudaEventDestroy(e);
     if (c->ev_opt_done) cudaEventDestroy(c->ev_opt_done);
     if (c->opt_st) cudaStreamDestroy(c->opt_st);
+    if (c->aux_st) { cudaStreamSynchronize(c->aux_st); cudaStreamDestroy(c->aux_st); }
+    if (c->ev_fork) cudaEventDestroy(c->ev_fork);
+    if (c->ev_join) cudaEventDestroy(c->ev_join);
     if (c->ev_comm_done) cudaEventDestroy(c->ev_comm_done);
     if (c->comm) ncclCommDestroy(c->comm);
     if (c->comm_st) cudaStreamDestroy(c->comm_st);
