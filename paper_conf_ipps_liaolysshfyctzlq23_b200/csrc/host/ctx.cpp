@@ -364,6 +364,15 @@ void join(mimose_ctx* c, cudaStream_t st) {
   cudaStreamWaitEvent(st, c->ev_join, 0);
   c->aux_pending = false;
 }
+// Weight-gradient GEMMs of the post-LN layer on the side stream too, beside the
+// next dgrad (MIMOSE_AUX_WGRAD=0: on the compute stream).
+bool aux_wgrad(const mimose_ctx* c) {
+  static const int v = [] {
+    const char* e = std::getenv("MIMOSE_AUX_WGRAD");
+    return e ? std::atoi(e) : 1;
+  }();
+  return v != 0 && aux_enabled(c) && c->dt == DT_BF16 && c->cfg.use_tc;
+}
 // The LN partials use the first NPART x max(3H, F) floats of c->part, the
 // bias column-sum partials the second.
 inline float* part_cs(const mimose_ctx* c) {
@@ -691,16 +700,21 @@ void ffn_backward(Run& r, int l, LayerBufs& b, float* dy, char* scr) {
                fork(c, r.st));
   // FFN2: du = (dt2 W2) * gelu'(u)
   dgrad(r, EPI_GELU_BWD, R3, H, W(c, LP(c, l, L_F2W)), F, R2, b.u);
-  // db1 = colsum du, beside the FFN1 dgrad and the weight gradients
+  // db1 = colsum du and (aux_wgrad) the weight gradients dW2 = dt2^T g, dW1 = du^T h1
+  // on the side stream, beside the FFN1 dgrad (dt2 in R3 lives until LN1 backward)
   {
     cudaStream_t sa = fork(c, r.st);
     colsum(c->dt, R2, T, F, part_cs(c), sa);
     reduce_partials(part_cs(c), F, F, G(c, LP(c, l, L_F1B)), sa);
+    if (aux_wgrad(c)) {
+      Run ra = r;
+      ra.st = sa;
+      wgrad2(ra, R3, H, b.g, F, G(c, LP(c, l, L_F2W)), R2, F, b.h1, H, G(c, LP(c, l, L_F1W)));
+    }
   }
   // FFN1: dh1 = du W1 + dz2 (in place in dres)
   dgrad(r, EPI_ACC_RES_F32, R2, F, W(c, LP(c, l, L_F1W)), H, dres, dres);
-  // dW2 = dt2^T g and dW1 = du^T h1 together (dt2 in R3 lives until LN1 backward)
-  wgrad2(r, R3, H, b.g, F, G(c, LP(c, l, L_F2W)), R2, F, b.h1, H, G(c, LP(c, l, L_F1W)));
+  if (!aux_wgrad(c)) wgrad2(r, R3, H, b.g, F, G(c, LP(c, l, L_F2W)), R2, F, b.h1, H, G(c, LP(c, l, L_F1W)));
 }
 
 // Attention-block gradients of a post-LN layer (after ffn_backward; dres = dh1).
@@ -730,18 +744,25 @@ void att_backward(Run& r, int l, const char* x, LayerBufs& b, float* dy, char* s
   if (!spare) wgrad(r, DT1, H, b.O, H, G(c, LP(c, l, L_OW)));     // dWo = dt1^T O before R3 is reused
   // attention backward -> dQKV (R3)
   attn_bwd(c->dt, b.qkv, b.O, R2, b.lse, c->lens, Dbuf, R3, c->B, c->S, H, h, make_drop(c, KIND_ATTN_PROBS, l), r.st);
-  // dbqkv = colsum dQKV, beside the QKV dgrad and the weight gradients
+  // dbqkv = colsum dQKV and (aux_wgrad) dWo = dt1^T O with dWqkv = dQKV^T x on the
+  // side stream, beside the QKV dgrad
+  const bool side_w = spare && aux_wgrad(c);
   {
     cudaStream_t sa = fork(c, r.st);
     colsum(c->dt, R3, T, 3 * H, part_cs(c), sa);
     reduce_partials(part_cs(c), 3 * H, 3 * H, G(c, LP(c, l, L_QKVB)), sa);
+    if (side_w) {
+      Run ra = r;
+      ra.st = sa;
+      wgrad2(ra, DT1, H, b.O, H, G(c, LP(c, l, L_OW)), R3, 3 * H, x, H, G(c, LP(c, l, L_QKVW)));
+    }
   }
   // QKV: dx = dQKV Wqkv + dz1 -> dy buffer
   dgrad(r, EPI_ACC_RES_F32, R3, 3 * H, W(c, LP(c, l, L_QKVW)), H, dy, dres);
   // dWo = dt1^T O and dWqkv = dQKV^T x
-  if (spare)
+  if (spare && !side_w)
     wgrad2(r, DT1, H, b.O, H, G(c, LP(c, l, L_OW)), R3, 3 * H, x, H, G(c, LP(c, l, L_QKVW)));
-  else
+  else if (!spare)
     wgrad(r, R3, 3 * H, x, H, G(c, LP(c, l, L_QKVW)));
 }
 
@@ -1253,6 +1274,7 @@ mimose_status run_backward(Run& r, Sample* sample) {
     LayerBufs& b = c->lb[l];
     const char* x = l > 0 ? c->y[l - 1] : c->x1;
     if ((c->drop_mask >> (2 * l + 1)) & 1) {          // recompute the FFN block from h1 / r1
+      if (r.real) join(c, r.st);                      // side-stream readers of the popped region first
       alloc_ffn(r, b, true);
       ffn_fwd_u(r, l, b, nullptr);
     }
@@ -1261,6 +1283,7 @@ mimose_status run_backward(Run& r, Sample* sample) {
     free_ffn(r, true);
     a.pop(mid_size(r));                               // h1 / r1: dead after the FFN block's gradients
     if ((c->drop_mask >> (2 * l)) & 1) {              // recompute the attention block from y_{l-1}
+      if (r.real) join(c, r.st);                      // the FFN block's side wgrad reads g, h1 (popped)
       alloc_att(r, b, true);
       att_fwd_u(r, l, x, b, nullptr);
     }
@@ -1278,6 +1301,7 @@ mimose_status run_backward(Run& r, Sample* sample) {
     const bool dropped = (c->drop_mask >> l) & 1;
     const char* x = l > 0 ? c->y[l - 1] : c->x1;
     if (dropped) {                                    // recompute right before the gradients
+      if (r.real) join(c, r.st);                      // the side wgrads of layer l+1 read x = y_l, O (popped)
       alloc_internals(r, c->lb[l], true);
       layer_fwd_any(r, l, x, c->lb[l], nullptr);
     }
