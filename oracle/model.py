@@ -24,7 +24,7 @@ from typing import Dict, Optional, Sequence
 import numpy as np
 
 from paper_conf_ipps_liaolysshfyctzlq23_b200.workload import (
-    ARCH_PRE_LN, HEAD_LM, HEAD_MC, HEAD_QA, HEAD_SEQCLS, Batch, ModelConfig, param_spec)
+    ARCH_ENCDEC, ARCH_PRE_LN, HEAD_LM, HEAD_MC, HEAD_QA, HEAD_SEQCLS, Batch, ModelConfig, param_spec)
 from . import philox as px
 
 
@@ -229,11 +229,11 @@ def layer_bwd(cfg, W, l, dy, c, B, S, masks: Masks, G):
 # m = LN2(r1); y = r1 + drop(gelu_tanh(m W1 + b1) W2 + b2)
 # --------------------------------------------------------------------------
 
-def layer_fwd_pre(cfg, W, l, x, lengths, B, S, masks: Masks):
+def layer_fwd_pre(cfg, W, l, x, lengths, B, S, masks: Masks, causal: bool = True):
     p = f"layer{l}."
     a, ln1 = layernorm(x, W[p + "ln1.g"], W[p + "ln1.b"], cfg.ln_eps)
     qkv = linear(a, W[p + "qkv.w"], W[p + "qkv.b"])
-    o, acache = attention_fwd(qkv, lengths, B, S, cfg.heads, masks.attn_probs(l), causal=True)
+    o, acache = attention_fwd(qkv, lengths, B, S, cfg.heads, masks.attn_probs(l), causal=causal)
     r1 = x + linear(o, W[p + "o.w"], W[p + "o.b"]) * masks.attn_out(l)
     m, ln2 = layernorm(r1, W[p + "ln2.g"], W[p + "ln2.b"], cfg.ln_eps)
     u = linear(m, W[p + "f1.w"], W[p + "f1.b"])
@@ -367,6 +367,8 @@ def train_step_grads(cfg: ModelConfig, params: Dict[str, np.ndarray], batch: Bat
     ``plan`` = 0-based indices of dropped layers: their caches are discarded
     after forward (only the layer input is kept) and re-created by replaying
     the forward right before their backward."""
+    if cfg.arch == ARCH_ENCDEC:
+        return encdec_step_grads(cfg, params, batch, seed, step, rank, plan, p)
     W = {k: np.asarray(v, np.float64) for k, v in params.items()}
     B, S = batch.input_ids.shape
     masks = Masks(cfg, B, S, seed, step, rank, p, mask_override)
@@ -388,6 +390,183 @@ def train_step_grads(cfg: ModelConfig, params: Dict[str, np.ndarray], batch: Bat
         dy = bwd(cfg, W, l, dy, c, B, S, masks, G)
         caches[l] = None
     embed_bwd(cfg, W, dy, ec, masks, G)
+    return loss, G
+
+
+# --------------------------------------------------------------------------
+# encoder-decoder (Table II TR-T5; reading A32): pre-LN
+# encoder layers (bidirectional) + the encoder's final LN -> enc_out; pre-LN
+# decoder layers: r1 = x + drop(SelfAttn_causal(LN1 x)); r2 = r1 +
+# drop(CrossAttn(LN2 r1, enc_out)); y = r2 + drop(FFN(LN3 r2)); the decoder's
+# final LN -> tied LM head, next-token CE over the target.  Dropout sites
+# (R-B): encoder layers l = 0..Le-1, decoder layers Le + j; the decoder
+# embedding uses layer field DEC_EMB; cross-attention kinds 5 (probabilities,
+# element ((b h + head) S_t + q) S_s + k) and 6 (output hidden).
+# --------------------------------------------------------------------------
+
+DEC_EMB = 0xFFE
+KIND_CROSS_PROBS = 5
+KIND_CROSS_OUT = 6
+
+
+class EncDecMasks:
+    def __init__(self, cfg, B, Ss, St, seed, step, rank=0, p=None):
+        self.cfg, self.B, self.Ss, self.St = cfg, B, Ss, St
+        self.seed, self.step, self.rank = seed, step, rank
+        self.p = cfg.p_drop if p is None else p
+        self.enc = Masks(cfg, B, Ss, seed, step, rank, p)          # encoder layers, encoder embedding
+        self.dec = Masks(cfg, B, St, seed, step, rank, p)          # decoder self-attn / hidden sites
+
+    def _m(self, n, kind, layer, shape):
+        if self.p <= 0.0:
+            return np.ones(shape)
+        keep = px.keep_mask(n, self.p, self.seed, px.site_word(kind, layer, self.rank), self.step)
+        return keep.reshape(shape).astype(np.float64) / (1.0 - self.p)
+
+    def dec_emb(self):
+        T, H = self.B * self.St, self.cfg.hidden
+        return self._m(T * H, px.KIND_EMB, DEC_EMB, (T, H))
+
+    def cross_probs(self, layer):
+        B, h = self.B, self.cfg.heads
+        return self._m(B * h * self.St * self.Ss, KIND_CROSS_PROBS, layer, (B, h, self.St, self.Ss))
+
+    def cross_out(self, layer):
+        T, H = self.B * self.St, self.cfg.hidden
+        return self._m(T * H, KIND_CROSS_OUT, layer, (T, H))
+
+
+def cross_attention_fwd(q, kv, klen, B, St, Ss, h, pmask):
+    """O = drop(softmax(Q K^T / sqrt d + key-pad mask)) V with queries from the
+    decoder [B*St, H] and keys / values from the encoder [B*Ss, 2H]."""
+    H = q.shape[1]
+    d = H // h
+    qh = q.reshape(B, St, h, d).transpose(0, 2, 1, 3)
+    k = kv[:, :H].reshape(B, Ss, h, d).transpose(0, 2, 1, 3)
+    v = kv[:, H:].reshape(B, Ss, h, d).transpose(0, 2, 1, 3)
+    s = qh @ k.transpose(0, 1, 3, 2) / math.sqrt(d)
+    keyvalid = np.arange(Ss)[None, :] < np.asarray(klen)[:, None]
+    s = np.where(np.broadcast_to(keyvalid[:, None, None, :], s.shape), s, -np.inf)
+    p, lse = softmax_lastdim(s)
+    pd = p * pmask
+    o = (pd @ v).transpose(0, 2, 1, 3).reshape(B * St, H)
+    return o, (qh, k, v, p, pd)
+
+
+def cross_attention_bwd(dout, cache, B, St, Ss, h, pmask):
+    """-> dQ [B*St, H], dKV [B*Ss, 2H]."""
+    qh, k, v, p, pd = cache
+    d = qh.shape[-1]
+    H = h * d
+    do = dout.reshape(B, St, h, d).transpose(0, 2, 1, 3)
+    dv = pd.transpose(0, 1, 3, 2) @ do
+    dp = (do @ v.transpose(0, 1, 3, 2)) * pmask
+    ds = p * (dp - (dp * p).sum(axis=-1, keepdims=True))
+    dq = ds @ k / math.sqrt(d)
+    dk = ds.transpose(0, 1, 3, 2) @ qh / math.sqrt(d)
+    flat = lambda t, S: t.transpose(0, 2, 1, 3).reshape(B * S, H)
+    return flat(dq, St), np.concatenate([flat(dk, Ss), flat(dv, Ss)], axis=1)
+
+
+def dec_layer_fwd(cfg, W, j, x, enc_out, tlen, slen, B, St, Ss, mk: EncDecMasks):
+    p, L = f"dec{j}.", cfg.n_layers + j                      # dropout layer field
+    a, ln1 = layernorm(x, W[p + "ln1.g"], W[p + "ln1.b"], cfg.ln_eps)
+    qkv = linear(a, W[p + "qkv.w"], W[p + "qkv.b"])
+    o, ac = attention_fwd(qkv, tlen, B, St, cfg.heads, mk.dec.attn_probs(L), causal=True)
+    r1 = x + linear(o, W[p + "o.w"], W[p + "o.b"]) * mk.dec.attn_out(L)
+    c, ln2 = layernorm(r1, W[p + "ln2.g"], W[p + "ln2.b"], cfg.ln_eps)
+    qc = linear(c, W[p + "cq.w"], W[p + "cq.b"])
+    kvc = linear(enc_out, W[p + "ckv.w"], W[p + "ckv.b"])
+    oc, cc = cross_attention_fwd(qc, kvc, slen, B, St, Ss, cfg.heads, mk.cross_probs(L))
+    r2 = r1 + linear(oc, W[p + "co.w"], W[p + "co.b"]) * mk.cross_out(L)
+    m, ln3 = layernorm(r2, W[p + "ln3.g"], W[p + "ln3.b"], cfg.ln_eps)
+    u = linear(m, W[p + "f1.w"], W[p + "f1.b"])
+    g = gelu_tanh(u)
+    y = r2 + linear(g, W[p + "f2.w"], W[p + "f2.b"]) * mk.dec.ffn_out(L)
+    return y, dict(a=a, ln1=ln1, qkv=qkv, o=o, ac=ac, c=c, ln2=ln2, qc=qc, oc=oc, cc=cc, m=m, ln3=ln3, u=u, g=g)
+
+
+def dec_layer_bwd(cfg, W, j, dy, cch, enc_out, B, St, Ss, mk: EncDecMasks, G):
+    """-> (dx, d enc_out contribution)."""
+    p, L = f"dec{j}.", cfg.n_layers + j
+    dt3 = dy * mk.dec.ffn_out(L)
+    dg, G[p + "f2.w"], G[p + "f2.b"] = linear_bwd(dt3, cch["g"], W[p + "f2.w"])
+    du = gelu_tanh_bwd(dg, cch["u"])
+    dm, G[p + "f1.w"], G[p + "f1.b"] = linear_bwd(du, cch["m"], W[p + "f1.w"])
+    dr2_ln, G[p + "ln3.g"], G[p + "ln3.b"] = layernorm_bwd(dm, cch["ln3"], W[p + "ln3.g"])
+    dr2 = dy + dr2_ln
+    dtc = dr2 * mk.cross_out(L)
+    doc, G[p + "co.w"], G[p + "co.b"] = linear_bwd(dtc, cch["oc"], W[p + "co.w"])
+    dqc, dkvc = cross_attention_bwd(doc, cch["cc"], B, St, Ss, cfg.heads, mk.cross_probs(L))
+    dc, G[p + "cq.w"], G[p + "cq.b"] = linear_bwd(dqc, cch["c"], W[p + "cq.w"])
+    denc, G[p + "ckv.w"], G[p + "ckv.b"] = linear_bwd(dkvc, enc_out, W[p + "ckv.w"])
+    dr1_ln, G[p + "ln2.g"], G[p + "ln2.b"] = layernorm_bwd(dc, cch["ln2"], W[p + "ln2.g"])
+    dr1 = dr2 + dr1_ln
+    dt1 = dr1 * mk.dec.attn_out(L)
+    do, G[p + "o.w"], G[p + "o.b"] = linear_bwd(dt1, cch["o"], W[p + "o.w"])
+    dqkv = attention_bwd(do, cch["ac"], B, St, cfg.heads, mk.dec.attn_probs(L))
+    da, G[p + "qkv.w"], G[p + "qkv.b"] = linear_bwd(dqkv, cch["a"], W[p + "qkv.w"])
+    dx_ln, G[p + "ln1.g"], G[p + "ln1.b"] = layernorm_bwd(da, cch["ln1"], W[p + "ln1.g"])
+    return dr1 + dx_ln, denc
+
+
+def encdec_step_grads(cfg: ModelConfig, params, batch: Batch, seed: int, step: int, rank: int = 0,
+                      plan: Optional[Sequence[int]] = None, p: Optional[float] = None):
+    """Loss and fp64 gradients of one encoder-decoder step; ``plan`` = dropped
+    layers over the Le + Ld units (encoder l, decoder Le + j): discarded
+    caches replayed before their backward (c-C identity)."""
+    W = {k: np.asarray(v, np.float64) for k, v in params.items()}
+    B, Ss = batch.input_ids.shape
+    St = batch.dec_len
+    Le, Ld = cfg.n_layers, cfg.n_dec_layers
+    mk = EncDecMasks(cfg, B, Ss, St, seed, step, rank, p)
+    dropped = set(plan or ())
+    G: Dict[str, np.ndarray] = {}
+    # encoder
+    ids = batch.input_ids.reshape(-1)
+    pos = np.tile(np.arange(Ss) + cfg.pos_offset, B)
+    x = (W["emb.word"][ids] + W["emb.pos"][pos]) * mk.enc.emb()
+    enc_in, enc_c = [], []
+    for l in range(Le):
+        enc_in.append(x)
+        x, c = layer_fwd_pre(cfg, W, l, x, batch.lengths, B, Ss, mk.enc, causal=False)
+        enc_c.append(None if l in dropped else c)
+    enc_out, lne = layernorm(x, W["enc.lnf.g"], W["enc.lnf.b"], cfg.ln_eps)
+    # decoder
+    tids = batch.dec_ids.reshape(-1)
+    tpos = np.tile(np.arange(St) + cfg.pos_offset, B)
+    xd = (W["emb.word"][tids] + W["emb.pos"][tpos]) * mk.dec_emb()
+    dec_in, dec_c = [], []
+    for j in range(Ld):
+        dec_in.append(xd)
+        xd, c = dec_layer_fwd(cfg, W, j, xd, enc_out, batch.dec_lengths, batch.lengths, B, St, Ss, mk)
+        dec_c.append(None if Le + j in dropped else c)
+    # LM head on the decoder (final LN, tied vocabulary projection, next-token CE)
+    tb = Batch(batch.dec_ids, np.zeros_like(batch.dec_ids), batch.dec_lengths, np.zeros(0, np.int32), St)
+    loss, dy = head_fwd_bwd(cfg, W, xd, tb, mk.dec, G)
+    denc = np.zeros_like(enc_out)
+    for j in reversed(range(Ld)):
+        c = dec_c[j]
+        if c is None:
+            _, c = dec_layer_fwd(cfg, W, j, dec_in[j], enc_out, batch.dec_lengths, batch.lengths, B, St, Ss, mk)
+        dy, de = dec_layer_bwd(cfg, W, j, dy, c, enc_out, B, St, Ss, mk, G)
+        denc += de
+    # decoder embedding (tied wte: the LM head's dW_e is in G["emb.word"])
+    dz = dy * mk.dec_emb()
+    np.add.at(G["emb.word"], tids, dz)
+    dpos = np.zeros_like(W["emb.pos"])
+    np.add.at(dpos, tpos, dz)
+    # encoder
+    dx, G["enc.lnf.g"], G["enc.lnf.b"] = layernorm_bwd(denc, lne, W["enc.lnf.g"])
+    for l in reversed(range(Le)):
+        c = enc_c[l]
+        if c is None:
+            _, c = layer_fwd_pre(cfg, W, l, enc_in[l], batch.lengths, B, Ss, mk.enc, causal=False)
+        dx = layer_bwd_pre(cfg, W, l, dx, c, B, Ss, mk.enc, G)
+    dz = dx * mk.enc.emb()
+    np.add.at(G["emb.word"], ids, dz)
+    np.add.at(dpos, pos, dz)
+    G["emb.pos"] = dpos
     return loss, G
 
 

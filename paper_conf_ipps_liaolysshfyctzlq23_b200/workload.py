@@ -16,12 +16,13 @@ from __future__ import annotations
 
 import dataclasses
 import math
-from typing import Dict, List, Tuple
+from typing import Dict, List, Optional, Tuple
 
 import numpy as np
 
 ARCH_POST_LN = 0     # BERT / RoBERTa post-LN encoder
 ARCH_PRE_LN = 1      # GPT-2 pre-LN causal decoder stack
+ARCH_ENCDEC = 2      # T5-like encoder-decoder: pre-LN encoder + pre-LN decoder with cross-attention
 HEAD_SEQCLS = 0      # pooler -> dropout -> linear(n_labels) -> CE
 HEAD_MC = 1          # pooler -> dropout -> linear(1) -> [B_q, n_choices] -> CE
 HEAD_QA = 2          # linear(2) on every token -> start/end CE
@@ -59,6 +60,8 @@ class ModelConfig:
     arch: int = ARCH_POST_LN
     # heterogeneous stages: FFN width of every layer; () = ffn everywhere
     ffn_layers: Tuple[int, ...] = ()
+    # encoder-decoder: decoder layers (n_layers = encoder layers)
+    n_dec_layers: int = 0
 
     def ffn_of(self, l: int) -> int:
         return self.ffn_layers[l] if self.ffn_layers else self.ffn
@@ -66,6 +69,11 @@ class ModelConfig:
     @property
     def causal(self) -> bool:
         return self.arch == ARCH_PRE_LN
+
+    @property
+    def n_units_total(self) -> int:
+        """Checkpointable layers: encoder + decoder layers for ARCH_ENCDEC."""
+        return self.n_layers + self.n_dec_layers
 
     @property
     def head_dim(self) -> int:
@@ -136,6 +144,15 @@ CONFIGS: Dict[str, ModelConfig] = {
     "hetero": ModelConfig("hetero", 5, 12, 768, 12, 4096, 30522, 512, 2, 0,
                           HEAD_MC, 4, 2, "bf16", 1e-12, 0.1, 64, 32, 128, 8, 0.6,
                           101, 102, 0, 103, ARCH_POST_LN, (4096,) * 4 + (3072,) * 4 + (1536,) * 4),
+    # the paper's TR-T5 task (Table II: T5-base on UN_PC, batch 8;
+    # P:73 input sizes 17-460).  T5-base shapes (12 + 12 layers, H 768, 12 heads,
+    # F 3072, 32128-word tied vocabulary) with pre-LN blocks (T5 is pre-norm),
+    # biases and tanh-GELU kept, absolute positions (reading A32); source
+    # lengths 17-128 (the one-tile attention kernels; reading A32), target =
+    # source x U[0.8, 1.2]; budget 50%.
+    "t5-base": ModelConfig("t5-base", 6, 12, 768, 12, 3072, 32128, 512, 0, 0,
+                           HEAD_LM, 1, 2, "bf16", 1e-6, 0.1, 8, 17, 128, 8, 0.5,
+                           1, 1, 0, 3, ARCH_ENCDEC, (), 12),
 }
 
 
@@ -151,6 +168,28 @@ def small_config(base: str, **over) -> ModelConfig:
 def param_spec(cfg: ModelConfig) -> List[Tuple[str, Tuple[int, ...]]]:
     H, F, V = cfg.hidden, cfg.ffn, cfg.vocab
     P = cfg.max_pos
+    if cfg.arch == ARCH_ENCDEC:
+        # shared wte (encoder input, decoder input, tied LM head), wpe; pre-LN
+        # encoder layers, the encoder's final LN; pre-LN decoder layers with a
+        # cross-attention block (LN2 -> Q from the decoder, K/V from the encoder
+        # output); the decoder's final LN
+        spec = [("emb.word", (V, H)), ("emb.pos", (P, H))]
+        for l in range(cfg.n_layers):
+            p = f"layer{l}."
+            spec += [(p + "ln1.g", (H,)), (p + "ln1.b", (H,)), (p + "qkv.w", (3 * H, H)), (p + "qkv.b", (3 * H,)),
+                     (p + "o.w", (H, H)), (p + "o.b", (H,)), (p + "ln2.g", (H,)), (p + "ln2.b", (H,)),
+                     (p + "f1.w", (F, H)), (p + "f1.b", (F,)), (p + "f2.w", (H, F)), (p + "f2.b", (H,))]
+        spec += [("enc.lnf.g", (H,)), ("enc.lnf.b", (H,))]
+        for j in range(cfg.n_dec_layers):
+            p = f"dec{j}."
+            spec += [(p + "ln1.g", (H,)), (p + "ln1.b", (H,)), (p + "qkv.w", (3 * H, H)), (p + "qkv.b", (3 * H,)),
+                     (p + "o.w", (H, H)), (p + "o.b", (H,)),
+                     (p + "ln2.g", (H,)), (p + "ln2.b", (H,)), (p + "cq.w", (H, H)), (p + "cq.b", (H,)),
+                     (p + "ckv.w", (2 * H, H)), (p + "ckv.b", (2 * H,)), (p + "co.w", (H, H)), (p + "co.b", (H,)),
+                     (p + "ln3.g", (H,)), (p + "ln3.b", (H,)),
+                     (p + "f1.w", (F, H)), (p + "f1.b", (F,)), (p + "f2.w", (H, F)), (p + "f2.b", (H,))]
+        spec += [("lnf.g", (H,)), ("lnf.b", (H,))]
+        return spec
     if cfg.arch == ARCH_PRE_LN:
         # GPT-2: wte (tied with the LM head), wpe; pre-LN layers; final LN
         spec = [("emb.word", (V, H)), ("emb.pos", (P, H))]
@@ -239,6 +278,15 @@ class Batch:
     lengths: np.ndarray      # int32 [B]
     labels: np.ndarray       # int32 [n_label_values]
     seq_len: int             # S_pad
+    # encoder-decoder (ARCH_ENCDEC): the decoder's input ids, lengths, padded length
+    dec_ids: Optional[np.ndarray] = None       # int32 [B, S_t_pad]
+    dec_lengths: Optional[np.ndarray] = None   # int32 [B]
+    dec_len: int = 0
+
+    @property
+    def input_size2(self) -> Tuple[int, int]:
+        """The 2-D input size (source, target) of an encoder-decoder batch."""
+        return int(self.input_ids.size), int(self.dec_ids.size) if self.dec_ids is not None else 0
 
     @property
     def n_seqs(self) -> int:
@@ -290,7 +338,7 @@ def make_batch(cfg: ModelConfig, longest: int, seed: int, n_seqs: int | None = N
     tt = np.zeros((B, S), np.int32)
     for b in range(B):
         n = int(lens[b])
-        if cfg.arch == ARCH_PRE_LN:                 # GPT-2: plain text tokens
+        if cfg.arch in (ARCH_PRE_LN, ARCH_ENCDEC):   # GPT-2 / T5 source: plain text tokens
             ids[b, :n] = rng.integers(cfg.first_tok, cfg.vocab - 1, size=n)
             continue
         ids[b, :n] = rng.integers(cfg.first_tok, cfg.vocab, size=n)
@@ -298,6 +346,19 @@ def make_batch(cfg: ModelConfig, longest: int, seed: int, n_seqs: int | None = N
         ids[b, n - 1] = cfg.sep_id
         if cfg.type_vocab > 1:
             tt[b, n // 2:n] = 1
+    if cfg.arch == ARCH_ENCDEC:
+        # target: longest = source longest x U[0.8, 1.2] within [seq_lo/2, seq_hi]
+        # (translation pairs of similar length, UN_PC-like); next-token CE on it
+        Lt = int(np.clip(round(longest * rng.uniform(0.8, 1.2)), max(2, cfg.seq_lo // 2), cfg.seq_hi))
+        St = roundup(Lt, cfg.pad)
+        tl = np.empty(B, np.int32)
+        tl[0] = Lt
+        if B > 1:
+            tl[1:] = rng.integers(max(2, (Lt + 1) // 2), Lt + 1, size=B - 1)
+        did = np.full((B, St), cfg.pad_id, np.int32)
+        for b in range(B):
+            did[b, :int(tl[b])] = rng.integers(cfg.first_tok, cfg.vocab, size=int(tl[b]))
+        return Batch(ids, tt, lens, np.zeros(0, np.int32), S, did, tl, St)
     if cfg.head == HEAD_LM:
         labels = np.zeros(0, np.int32)
     elif cfg.head == HEAD_SEQCLS:
