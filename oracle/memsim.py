@@ -36,7 +36,7 @@ import dataclasses
 from typing import Dict, List, Optional, Sequence
 
 from paper_conf_ipps_liaolysshfyctzlq23_b200.workload import (
-    ARCH_PRE_LN, HEAD_LM, HEAD_QA, ModelConfig, param_spec)
+    ARCH_ENCDEC, ARCH_PRE_LN, HEAD_LM, HEAD_QA, ModelConfig, param_spec)
 
 LM_CHUNK = 2048     # tokens per LM-head chunk (logits never exceed LM_CHUNK x Vpad)
 
@@ -59,8 +59,23 @@ NPART = 296   # fixed count of deterministic reduction partials (DESIGN "Memory 
 def buckets(cfg: ModelConfig) -> List[List[int]]:
     """Gradient buckets as lists of parameter indices, in layout order: the
     embedding tensors, one bucket per encoder layer (12 tensors), the head
-    (all-reduced / reduce-scattered as soon as each is final)."""
+    (all-reduced / reduce-scattered as soon as each is final).
+    Encoder-decoder: embedding, encoder layers, [encoder final LN + decoder
+    layer 0], decoder layers (20 tensors), decoder final LN."""
     n = len(param_spec(cfg))
+    if cfg.arch == ARCH_ENCDEC:
+        out = [[0, 1]]
+        i = 2
+        for _ in range(cfg.n_layers):
+            out.append(list(range(i, i + 12)))
+            i += 12
+        out.append(list(range(i, i + 2 + 20)))          # enc.lnf with decoder layer 0
+        i += 22
+        for _ in range(1, cfg.n_dec_layers):
+            out.append(list(range(i, i + 20)))
+            i += 20
+        out.append(list(range(i, n)))
+        return out
     n_emb = 2 if cfg.arch == ARCH_PRE_LN else 5
     out = [list(range(n_emb))]
     for l in range(cfg.n_layers):
@@ -522,3 +537,196 @@ def collect_samples_units(sz: Sizes) -> Dict[str, object]:
         A.pop(t)
     A.tfree(sz.dy)
     return dict(C=sz.C, E=E, a=a, y=y, Hd=hd, Th=th, Tb=tb, Te=te, peak=A.peak)
+
+
+# --------------------------------------------------------------------------
+# encoder-decoder (reading A32): DESIGN.md §3 "Encoder-decoder"
+# --------------------------------------------------------------------------
+
+@dataclasses.dataclass(frozen=True)
+class EncDecSizes:
+    C: int
+    E: List[int]          # x1_s
+    enc_ints: List[int]
+    enc_y: int
+    bundle: List[int]     # output of the last encoder unit: x_L, enc_out, enc_st, x1_t
+    dec_ints: List[int]
+    dec_y: int
+    head: List[int]
+    head_fwd_scratch: int
+    head_scratch: int
+    dy: int
+    denc: int
+    layer_scratch: int    # uniform over both stacks: decoder + cross + encoder parts
+    emb_scratch: int      # uniform over both embeddings
+    n_enc: int
+    n_dec: int
+
+    def ints(self, u):
+        return self.enc_ints if u < self.n_enc else self.dec_ints
+
+    def outs(self, u):
+        if u < self.n_enc - 1:
+            return [self.enc_y]
+        if u == self.n_enc - 1:
+            return self.bundle
+        return [self.dec_y]
+
+
+def sizes_encdec(cfg: ModelConfig, B: int, Ss: int, St: int, max_seqs: Optional[int] = None,
+                 max_seq_len: Optional[int] = None, world: int = 1, zero1: bool = False) -> EncDecSizes:
+    e = ebytes(cfg)
+    H, F, h = cfg.hidden, cfg.ffn, cfg.heads
+    Ts, Tt = B * Ss, B * St
+    ms = cfg.n_seqs if max_seqs is None else max_seqs
+    mx = cfg.max_seq if max_seq_len is None else max_seq_len
+
+    def pre_ints(T, S):     # a, st1, QKV, O, LSE, r1, st2, m, u, g (GPT-2 layer order)
+        return [a16(T * H * e), a16(T * 8), a16(T * 3 * H * e), a16(T * H * e), a16(B * h * S * 4),
+                a16(T * H * 4), a16(T * 8), a16(T * H * e), a16(T * F * e), a16(T * F * e)]
+
+    dec = [a16(Tt * H * e), a16(Tt * 8), a16(Tt * 3 * H * e), a16(Tt * H * e), a16(B * h * St * 4),  # a st1 QKV O LSE
+           a16(Tt * H * 4), a16(Tt * 8), a16(Tt * H * e), a16(Tt * H * e), a16(Ts * 2 * H * e),    # r1 st2 c Qc KVc
+           a16(Tt * H * e), a16(B * h * St * 4), a16(Tt * H * 4), a16(Tt * 8), a16(Tt * H * e),    # Oc LSEc r2 st3 m
+           a16(Tt * F * e), a16(Tt * F * e)]                                                         # u g
+
+    def lscr(T, S):
+        return a16(T * H * 4) + a16(T * F * e) + a16(T * 3 * H * e) + a16(B * h * S * 4)
+
+    ntiles = (ms * mx + 1023) // 1024
+
+    def escr(T):
+        return a16(T * H * 4) + a16(16 * T) + a16(4 * 256 * ntiles)
+
+    VP = vpad(cfg.vocab)
+    return EncDecSizes(
+        persistent_bytes(cfg, ms, mx, world, zero1), [a16(Ts * H * 4)], pre_ints(Ts, Ss), a16(Ts * H * 4),
+        [a16(Ts * H * 4), a16(Ts * H * e), a16(Ts * 8), a16(Tt * H * 4)], dec, a16(Tt * H * 4),
+        [a16(Tt * H * e), a16(Tt * 8), a16(Tt * 8)], a16(LM_CHUNK * VP * 4),
+        a16(LM_CHUNK * VP * 4) + a16(LM_CHUNK * VP * e), a16(Tt * H * 4), a16(Ts * H * 4),
+        lscr(Tt, St) + a16(Ts * 2 * H * e) + lscr(Ts, Ss), escr(Ts) + escr(Tt),
+        cfg.n_layers, cfg.n_dec_layers)
+
+
+def _encdec_forward(A: Arena, sz: EncDecSizes, drop, collect=False):
+    a_s, y_s = [], []
+    for u in range(sz.n_enc + sz.n_dec):
+        b0 = A.live
+        ints, outs = sz.ints(u), sz.outs(u)
+        if collect:                                           # pass 1: save mode, then discarded
+            for t in ints:
+                A.push(t)
+            for t in outs:
+                A.push(t)
+            a_s.append(A.live - b0)
+            for t in reversed(outs):
+                A.pop(t)
+            for t in reversed(ints):
+                A.pop(t)
+        if collect or u in drop:
+            for t in ints:
+                A.talloc(t)
+            for t in outs:
+                A.push(t)
+            for t in reversed(ints):
+                A.tfree(t)
+        else:
+            for t in ints:
+                A.push(t)
+            for t in outs:
+                A.push(t)
+        y_s.append(A.live - b0)
+    return a_s, y_s
+
+
+def _encdec_backward(A: Arena, sz: EncDecSizes, drop, phases=None):
+    Le, Ld = sz.n_enc, sz.n_dec
+    A.talloc(sz.denc)
+    A.talloc(sz.dy)
+    A.top_peak_phase = sum(A.top)
+    A.talloc(sz.head_scratch)
+    A.tfree(sz.head_scratch)
+    th = A.top_peak_phase
+    for t in reversed(sz.head):
+        A.pop(t)
+    A.pop(sz.dec_y)                                          # the last decoder unit's output
+    A.top_peak_phase = sum(A.top)
+    for j in reversed(range(Ld)):
+        u = Le + j
+        if u in drop:
+            for t in sz.dec_ints:
+                A.push(t)
+        A.talloc(sz.layer_scratch)
+        A.tfree(sz.layer_scratch)
+        for t in reversed(sz.dec_ints):
+            A.pop(t)
+        if j > 0:
+            A.pop(sz.dec_y)
+    tb = A.top_peak_phase
+    A.top_peak_phase = sum(A.top)
+    A.talloc(sz.emb_scratch)                                 # decoder embedding backward
+    A.tfree(sz.emb_scratch)
+    te = A.top_peak_phase
+    x_L, enc_out, enc_st, x1_t = sz.bundle
+    A.pop(x1_t)
+    A.pop(enc_st)                                            # encoder final LN backward (in place, no scratch)
+    A.pop(enc_out)
+    A.pop(x_L)
+    A.top_peak_phase = sum(A.top)
+    for l in reversed(range(Le)):
+        if l in drop:
+            for t in sz.enc_ints:
+                A.push(t)
+        A.talloc(sz.layer_scratch)
+        A.tfree(sz.layer_scratch)
+        for t in reversed(sz.enc_ints):
+            A.pop(t)
+        if l > 0:
+            A.pop(sz.enc_y)
+    tb = max(tb, A.top_peak_phase)
+    A.top_peak_phase = sum(A.top)
+    A.talloc(sz.emb_scratch)                                 # encoder embedding backward
+    A.tfree(sz.emb_scratch)
+    te = max(te, A.top_peak_phase)
+    for t in reversed(sz.E):
+        A.pop(t)
+    A.tfree(sz.dy)
+    A.tfree(sz.denc)
+    if phases is not None:
+        phases.update(Th=th, Tb=tb, Te=te)
+
+
+def simulate_step_encdec(sz: EncDecSizes, dropped: Sequence[int]) -> Arena:
+    """One encoder-decoder step under a plan over the Le + Ld units (encoder l,
+    decoder Le + j)."""
+    drop = set(dropped)
+    A = Arena(sz.C)
+    for t in sz.E:
+        A.push(t)
+    _encdec_forward(A, sz, drop)
+    for t in sz.head:
+        A.push(t)
+    A.talloc(sz.head_fwd_scratch)
+    A.tfree(sz.head_fwd_scratch)
+    _encdec_backward(A, sz, drop)
+    assert A.live == sz.C
+    return A
+
+
+def collect_samples_encdec(sz: EncDecSizes) -> Dict[str, object]:
+    """The shuttling collector over the Le + Ld units (every unit dropped in the
+    sheltered backward)."""
+    A = Arena(sz.C)
+    for t in sz.E:
+        A.push(t)
+    E = A.live - sz.C
+    a, y = _encdec_forward(A, sz, set(), collect=True)
+    b0 = A.live
+    for t in sz.head:
+        A.push(t)
+    hd = A.live - b0
+    A.talloc(sz.head_fwd_scratch)
+    A.tfree(sz.head_fwd_scratch)
+    ph = {}
+    _encdec_backward(A, sz, set(range(sz.n_enc + sz.n_dec)), ph)
+    return dict(C=sz.C, E=E, a=a, y=y, Hd=hd, Th=ph["Th"], Tb=ph["Tb"], Te=ph["Te"], peak=A.peak)
