@@ -50,7 +50,7 @@ typedef enum {
   MIMOSE_E_NODEVICE = 8    /* device call on a host-only ctx (arena_base == NULL)   */
 } mimose_status;
 
-enum { MIMOSE_ARCH_POST_LN = 0, MIMOSE_ARCH_PRE_LN = 1 };
+enum { MIMOSE_ARCH_POST_LN = 0, MIMOSE_ARCH_PRE_LN = 1, MIMOSE_ARCH_ENCDEC = 2 };
 enum { MIMOSE_HEAD_SEQCLS = 0, MIMOSE_HEAD_MC = 1, MIMOSE_HEAD_QA = 2, MIMOSE_HEAD_LM = 3 };
 enum { MIMOSE_FP32 = 0, MIMOSE_BF16 = 1 };
 enum { MIMOSE_PHASE_SHELTERED = 0, MIMOSE_PHASE_RESPONSIVE = 1 };
@@ -120,7 +120,9 @@ typedef struct {
                             optimizer is fused.  Persistent bytes fall from 18 to
                             6 + 12 / world B/param.  Needs a communicator (world > 1 or
                             comm_force); mimose_get_master is then refused for world > 1. */
-  int32_t reserved[1];
+  int32_t n_dec_layers;  /* MIMOSE_ARCH_ENCDEC: decoder layers; n_layers is then
+                            the encoder's.  Checkpoint units: encoder layers 0..n_layers-1,
+                            decoder layers n_layers..n_layers+n_dec_layers-1            */
   const int32_t* ffn_layers; /* heterogeneous stages: FFN width of each of the
                             n_layers layers (multiples of 64, <= ffn; ffn is then the max
                             and sizes the shared workspaces); NULL = every layer uses ffn.
@@ -148,6 +150,15 @@ typedef struct {
   const int32_t* labels;
   int32_t n_seqs, seq_len;
   int32_t on_host;
+  /* encoder-decoder only (MIMOSE_ARCH_ENCDEC): the decoder's input ids
+     [n_seqs, dec_len] (right-padded; the LM targets are these shifted by one
+     inside each sequence) and valid lengths [n_seqs].  input_ids / lengths are
+     then the encoder's source; token_type and labels are unused.  The input
+     size key is 2-D: (n_seqs * seq_len, n_seqs * dec_len). */
+  const int32_t* dec_ids;
+  const int32_t* dec_lengths;
+  int32_t dec_len;
+  int32_t pad_;
 } mimose_batch;
 
 /* Algorithm 1 output L' as a bitmask over layers (bit l = layer l,
@@ -174,6 +185,7 @@ typedef struct {
   int64_t a[64];         /* pass-1 (save mode) delta per layer                       */
   int64_t y[64];         /* pass-2 (no-save mode) delta per layer                    */
   float   t_ms[64];      /* pass-1 forward time per layer (cudaEvent; 0 host-only)   */
+  int64_t xt;            /* encoder-decoder: the target input size (2-D key); else 0  */
 } mimose_sample;
 
 typedef struct {
@@ -231,6 +243,11 @@ mimose_status mimose_collect(mimose_ctx* ctx, const mimose_batch* batch, float* 
    Returns MIMOSE_E_NOT_READY in the sheltered phase; MIMOSE_E_INFEASIBLE if even
    the deepest plan predicts a peak above M - reserve (out->status set too). */
 mimose_status mimose_plan(mimose_ctx* ctx, int64_t input_size, mimose_plan_t* out);
+/* Encoder-decoder (reading A32): the plan for the 2-D input size
+   (x = numel(source ids), x_t = numel(target ids)); the estimator behind it is
+   the bivariate quadratic of the collector's samples (P:162-164 per input
+   tensor).  Same cache / errors as mimose_plan; out->input_size = x. */
+mimose_status mimose_plan2(mimose_ctx* ctx, int64_t x_src, int64_t x_tgt, mimose_plan_t* out);
 
 /* Selects the scheduler behind mimose_plan (Mimose "reserves a
    flexible interface for users to experiment with other scheduling algorithms,
@@ -278,6 +295,11 @@ mimose_status mimose_dry_run(mimose_ctx* ctx, int32_t n_seqs, int32_t seq_len,
    iteration at this shape would record (t_ms = 0). */
 mimose_status mimose_dry_collect(mimose_ctx* ctx, int32_t n_seqs, int32_t seq_len,
                                  mimose_sample* out);
+/* The same two for an encoder-decoder batch shape (source seq_len, target dec_len). */
+mimose_status mimose_dry_run2(mimose_ctx* ctx, int32_t n_seqs, int32_t seq_len, int32_t dec_len,
+                              uint64_t drop_mask, int64_t* peak_out);
+mimose_status mimose_dry_collect2(mimose_ctx* ctx, int32_t n_seqs, int32_t seq_len, int32_t dec_len,
+                                  mimose_sample* out);
 
 /* Writes a fresh 128-byte ncclUniqueId (rank 0 calls it and broadcasts the
    bytes through the caller's process group before mimose_init on every rank). */

@@ -46,13 +46,14 @@ class Config(C.Structure):
                 ("rank", C.c_int32), ("world", C.c_int32), ("nccl_id", C.c_void_p),
                 ("use_tc", C.c_int32), ("pad_id", C.c_int32), ("granularity", C.c_int32),
                 ("comm_force", C.c_int32), ("nccl_max_ctas", C.c_int32), ("check_plans", C.c_int32),
-                ("zero1", C.c_int32), ("reserved", C.c_int32 * 1), ("ffn_layers", C.c_void_p)]
+                ("zero1", C.c_int32), ("n_dec_layers", C.c_int32), ("ffn_layers", C.c_void_p)]
 
 
 class BatchS(C.Structure):
     _fields_ = [("input_ids", C.c_void_p), ("token_type", C.c_void_p), ("lengths", C.c_void_p),
                 ("labels", C.c_void_p), ("n_seqs", C.c_int32), ("seq_len", C.c_int32),
-                ("on_host", C.c_int32)]
+                ("on_host", C.c_int32), ("dec_ids", C.c_void_p), ("dec_lengths", C.c_void_p),
+                ("dec_len", C.c_int32), ("pad_", C.c_int32)]
 
 
 class Plan(C.Structure):
@@ -68,7 +69,7 @@ class Plan(C.Structure):
 class SampleS(C.Structure):
     _fields_ = [("x", C.c_int64), ("C", C.c_int64), ("E", C.c_int64), ("Hd", C.c_int64),
                 ("Th", C.c_int64), ("Tb", C.c_int64), ("Te", C.c_int64),
-                ("a", C.c_int64 * 64), ("y", C.c_int64 * 64), ("t_ms", C.c_float * 64)]
+                ("a", C.c_int64 * 64), ("y", C.c_int64 * 64), ("t_ms", C.c_float * 64), ("xt", C.c_int64)]
 
 
 class Stats(C.Structure):
@@ -112,6 +113,9 @@ _lib.mimose_phase.argtypes = [_P, C.POINTER(C.c_int32)]
 _lib.mimose_get_sample.argtypes = [_P, C.c_int32, C.POINTER(SampleS)]
 _lib.mimose_dry_run.argtypes = [_P, C.c_int32, C.c_int32, C.c_uint64, C.POINTER(C.c_int64)]
 _lib.mimose_dry_collect.argtypes = [_P, C.c_int32, C.c_int32, C.POINTER(SampleS)]
+_lib.mimose_dry_run2.argtypes = [_P, C.c_int32, C.c_int32, C.c_int32, C.c_uint64, C.POINTER(C.c_int64)]
+_lib.mimose_dry_collect2.argtypes = [_P, C.c_int32, C.c_int32, C.c_int32, C.POINTER(SampleS)]
+_lib.mimose_plan2.argtypes = [_P, C.c_int64, C.c_int64, C.POINTER(Plan)]
 _lib.mimose_predicted_peak.argtypes = [C.POINTER(Series), C.c_uint64]
 _lib.mimose_predicted_peak.restype = C.c_int64
 _lib.mimose_plan_series.argtypes = [C.POINTER(Series), C.c_int64, C.c_int64, C.c_int32, C.c_int32,
@@ -131,7 +135,8 @@ EXPORTED = ["mimose_default_config", "mimose_init", "mimose_destroy", "mimose_la
             "mimose_step", "mimose_get_stats", "mimose_phase", "mimose_get_sample", "mimose_dry_run",
             "mimose_dry_collect", "mimose_predicted_peak", "mimose_plan_series", "mimose_fit_predict",
             "mimose_nccl_unique_id", "mimose_probe", "mimose_probe_read", "mimose_set_optimizer",
-            "mimose_set_planner", "mimose_get_master"]
+            "mimose_set_planner", "mimose_get_master", "mimose_plan2", "mimose_dry_run2",
+            "mimose_dry_collect2"]
 
 
 _lib.mimose_tc_available.restype = C.c_int32
@@ -217,6 +222,7 @@ def make_config(cfg: wl.ModelConfig, **kw) -> Config:
     c.seed = wl.dropout_seed(cfg)
     c.max_seqs, c.max_seq_len = cfg.n_seqs, cfg.max_seq
     c.pad_id = cfg.pad_id
+    c.n_dec_layers = cfg.n_dec_layers
     if cfg.ffn_layers:                       # heterogeneous stages: per-layer FFN widths
         arr = (C.c_int32 * cfg.n_layers)(*cfg.ffn_layers)
         c._ffn_keep = arr                    # alive until mimose_init has copied it
@@ -258,8 +264,9 @@ class Mimose:
         n = C.c_int64()
         _lib.mimose_num_params(self.h, C.byref(n))
         self.n_params = n.value
-        # checkpoint units: layers, or 2L attention / FFN blocks (granularity=1)
-        self.n_units = cfg.n_layers * (2 if c.granularity == 1 else 1)
+        # checkpoint units: layers, or 2L attention / FFN blocks (granularity=1);
+        # encoder-decoder: encoder then decoder layers
+        self.n_units = cfg.n_layers * (2 if c.granularity == 1 else 1) + cfg.n_dec_layers
 
     # -- lifecycle --
     def close(self):
@@ -300,13 +307,21 @@ class Mimose:
 
     # -- batches --
     @staticmethod
-    def batch_struct(ids, tt, lens, labels, n_seqs, seq_len, on_host) -> BatchS:
+    def batch_struct(ids, tt, lens, labels, n_seqs, seq_len, on_host, dec_ids=None, dec_lens=None,
+                     dec_len=0) -> BatchS:
         def ptr(a):
+            if a is None:
+                return None
             return a.data_ptr() if hasattr(a, "data_ptr") else a.ctypes.data
-        return BatchS(ptr(ids), ptr(tt), ptr(lens), ptr(labels), n_seqs, seq_len, 1 if on_host else 0)
+        return BatchS(ptr(ids), ptr(tt), ptr(lens), ptr(labels), n_seqs, seq_len, 1 if on_host else 0,
+                      ptr(dec_ids), ptr(dec_lens), dec_len, 0)
 
     def host_batch(self, b: wl.Batch) -> BatchS:
         self._keep = [np.ascontiguousarray(x, np.int32) for x in (b.input_ids, b.token_type, b.lengths, b.labels)]
+        if b.dec_ids is not None:
+            self._keep += [np.ascontiguousarray(b.dec_ids, np.int32), np.ascontiguousarray(b.dec_lengths, np.int32)]
+            return self.batch_struct(*self._keep[:4], b.n_seqs, b.seq_len, True, self._keep[4], self._keep[5],
+                                     b.dec_len)
         return self.batch_struct(*self._keep, b.n_seqs, b.seq_len, True)
 
     # -- the method --
@@ -315,9 +330,13 @@ class Mimose:
         self._chk(_lib.mimose_collect(self.h, C.byref(batch), C.byref(loss) if want_loss else None))
         return loss.value if want_loss else None
 
-    def plan(self, x: int) -> Plan:
+    def plan(self, x: int, xt: Optional[int] = None) -> Plan:
+        """The plan for input size x (or the 2-D key (x, xt) of an encoder-decoder)."""
         p = Plan()
-        self._chk(_lib.mimose_plan(self.h, int(x), C.byref(p)), allow=(E_INFEASIBLE,))
+        if xt is None:
+            self._chk(_lib.mimose_plan(self.h, int(x), C.byref(p)), allow=(E_INFEASIBLE,))
+        else:
+            self._chk(_lib.mimose_plan2(self.h, int(x), int(xt), C.byref(p)), allow=(E_INFEASIBLE,))
         return p
 
     def set_planner(self, kind: int):
@@ -356,12 +375,15 @@ class Mimose:
         self._chk(_lib.mimose_get_sample(self.h, i, C.byref(s)))
         return _sample_dict(s, self.n_units)
 
-    def dry_run(self, n_seqs: int, seq_len: int, dropped=()) -> int:
+    def dry_run(self, n_seqs: int, seq_len: int, dropped=(), dec_len: Optional[int] = None) -> int:
         mask = 0
         for l in dropped:
             mask |= 1 << int(l)
         pk = C.c_int64()
-        self._chk(_lib.mimose_dry_run(self.h, n_seqs, seq_len, C.c_uint64(mask), C.byref(pk)))
+        if dec_len is None:
+            self._chk(_lib.mimose_dry_run(self.h, n_seqs, seq_len, C.c_uint64(mask), C.byref(pk)))
+        else:
+            self._chk(_lib.mimose_dry_run2(self.h, n_seqs, seq_len, dec_len, C.c_uint64(mask), C.byref(pk)))
         return pk.value
 
     def probe(self, kind: int = 1):
@@ -372,14 +394,17 @@ class Mimose:
         self._chk(_lib.mimose_probe_read(self.h, C.byref(ms), C.byref(fl), C.byref(n)))
         return ms.value, fl.value, n.value
 
-    def dry_collect(self, n_seqs: int, seq_len: int) -> Dict:
+    def dry_collect(self, n_seqs: int, seq_len: int, dec_len: Optional[int] = None) -> Dict:
         s = SampleS()
-        self._chk(_lib.mimose_dry_collect(self.h, n_seqs, seq_len, C.byref(s)))
+        if dec_len is None:
+            self._chk(_lib.mimose_dry_collect(self.h, n_seqs, seq_len, C.byref(s)))
+        else:
+            self._chk(_lib.mimose_dry_collect2(self.h, n_seqs, seq_len, dec_len, C.byref(s)))
         return _sample_dict(s, self.n_units)
 
 
 def _sample_dict(s: SampleS, L: int) -> Dict:
-    return dict(x=s.x, C=s.C, E=s.E, Hd=s.Hd, Th=s.Th, Tb=s.Tb, Te=s.Te,
+    return dict(x=s.x, xt=s.xt, C=s.C, E=s.E, Hd=s.Hd, Th=s.Th, Tb=s.Tb, Te=s.Te,
                 a=list(s.a[:L]), y=list(s.y[:L]), t_ms=list(s.t_ms[:L]))
 
 

@@ -61,6 +61,29 @@ std::vector<ParamInfo> build_layout(const mimose_config& c, int64_t* npad, int64
     *npad = off;
     return out;
   };
+  if (c.arch == 2) {             // encoder-decoder: wte, wpe, encoder layers, enc LNf, decoder layers, LNf
+    n.push_back((int64_t)c.vocab * H);
+    n.push_back((int64_t)c.max_pos * H);
+    const int64_t F = c.ffn;
+    for (int l = 0; l < c.n_layers; ++l) {
+      const int64_t v[12] = {H, H, 3 * H * H, 3 * H, H * H, H, H, H, F * H, F, H * F, H};
+      for (int64_t x : v) n.push_back(x);
+    }
+    n.push_back(H);
+    n.push_back(H);
+    for (int j = 0; j < c.n_dec_layers; ++j) {
+      const int64_t v[20] = {H, H, 3 * H * H, 3 * H, H * H, H, H, H, H * H, H, 2 * H * H, 2 * H, H * H, H,
+                             H, H, F * H, F, H * F, H};
+      for (int64_t x : v) n.push_back(x);
+    }
+    n.push_back(H);
+    n.push_back(H);
+    std::vector<ParamInfo> out;
+    int64_t off = 0;
+    for (int64_t x : n) { out.push_back({x, off}); off += (x + 63) / 64 * 64; }
+    *npad = (off + unit - 1) / unit * unit;
+    return out;
+  }
   if (c.arch == 1) {             // GPT-2: wte, wpe, pre-LN layers, lnf
     n.push_back((int64_t)c.vocab * H);
     n.push_back((int64_t)c.max_pos * H);
@@ -154,6 +177,13 @@ struct Arena {
   }
 };
 
+struct DecBufs {
+  char *a = nullptr, *qkv = nullptr, *O = nullptr, *c = nullptr, *qc = nullptr, *kvc = nullptr, *oc = nullptr,
+       *m = nullptr, *u = nullptr, *g = nullptr;
+  float2 *st1 = nullptr, *st2 = nullptr, *st3 = nullptr;
+  float *lse = nullptr, *lsec = nullptr, *r1 = nullptr, *r2 = nullptr;
+};
+
 struct LayerBufs {
   char *qkv = nullptr, *O = nullptr, *h1 = nullptr, *u = nullptr, *g = nullptr;
   float *z1 = nullptr, *z2 = nullptr;   // pre-LN sums, fp32 (reading R-P)
@@ -219,6 +249,12 @@ struct mimose_ctx {
   char* hp = nullptr;         // pooled (cls) or LM: LNf output hf
   float* logits = nullptr;
   float2 *lm_stf = nullptr, *lm_tok = nullptr;   // LM head: LNf stats, per-token (lse, nll)
+  // encoder-decoder: the two stacks' lengths / ids, the encoder output bundle, decoder buffers
+  int Ss = 0, St = 0;
+  int32_t *ids_src = nullptr, *ids_tgt = nullptr, *lens_src = nullptr, *lens_tgt = nullptr;
+  char *enc_out = nullptr, *x1t = nullptr;
+  float2* enc_st = nullptr;
+  std::vector<DecBufs> dlb;
   int64_t it = 0;             // dropout step counter (forward calls)
   int64_t adam_t = 0;
 
@@ -276,7 +312,7 @@ struct Sz {
 Sz sizes(const mimose_ctx* c, int B, int S) {
   const int64_t T = (int64_t)B * S, H = c->cfg.hidden, F = c->cfg.ffn, h = c->cfg.heads, e = c->e;
   Sz z{};
-  const bool pre = c->cfg.arch == 1;
+  const bool pre = c->cfg.arch != 0;
   z.z0 = a16(T * H * 4); z.st0 = a16(T * 8); z.x1 = pre ? a16(T * H * 4) : a16(T * H * e);
   z.a = a16(T * H * e); z.r1 = a16(T * H * 4); z.m = a16(T * H * e);
   z.qkv = a16(T * 3 * H * e); z.O = a16(T * H * e); z.lse = a16((int64_t)B * h * S * 4);
@@ -381,14 +417,19 @@ inline float* part_cs(const mimose_ctx* c) {
 inline float* G(mimose_ctx* c, int i) { return c->grad + c->layout[i].off; }
 // Parameter index of semantic slot k (L_*) of layer l.  Post-LN order is the
 // L_* enum order; GPT-2 (pre-LN) stores [ln1, qkv, o, ln2, f1, f2].
-inline int layer_base(const mimose_ctx* c) { return c->cfg.arch == 1 ? 2 : P_LAYER0; }
+inline int layer_base(const mimose_ctx* c) { return c->cfg.arch != 0 ? 2 : P_LAYER0; }
 inline int LP(mimose_ctx* c, int l, int k) {
   static const int pre_pos[12] = {2, 3, 4, 5, 0, 1, 8, 9, 10, 11, 6, 7};
-  return layer_base(c) + 12 * l + (c->cfg.arch == 1 ? pre_pos[k] : k);
+  return layer_base(c) + 12 * l + (c->cfg.arch != 0 ? pre_pos[k] : k);
 }
-inline int HP(mimose_ctx* c, int k) { return layer_base(c) + 12 * c->cfg.n_layers + k; }
+inline int HP(mimose_ctx* c, int k) {
+  if (c->cfg.arch == 2) return 2 + 12 * c->cfg.n_layers + 2 + 20 * c->cfg.n_dec_layers + k;   // decoder final LN
+  return layer_base(c) + 12 * c->cfg.n_layers + k;
+}
 // Checkpoint units: L layers, or 2L sub-layer blocks (granularity 1).
-inline int n_units(const mimose_ctx* c) { return c->cfg.granularity == 1 ? 2 * c->cfg.n_layers : c->cfg.n_layers; }
+inline int n_units(const mimose_ctx* c) {
+  return (c->cfg.granularity == 1 ? 2 * c->cfg.n_layers : c->cfg.n_layers) + (c->cfg.arch == 2 ? c->cfg.n_dec_layers : 0);
+}
 
 // ------------------------------------------------------------- probe ------
 void pgemm(mimose_ctx* c, Epi epi, const GemmArgs& g, cudaStream_t st) {
@@ -481,7 +522,7 @@ void layer_forward(Run& r, int l, const char* x, LayerBufs& b, char* yout) {
 void alloc_internals(Run& r, LayerBufs& b, bool on_stack) {
   Arena& a = r.c->ar;
   auto al = [&](int64_t n) { return on_stack ? a.push(n) : a.talloc(n); };
-  if (r.c->cfg.arch == 1) {   // [a, st1, QKV, O, LSE, r1, st2, m, u, g]
+  if (r.c->cfg.arch != 0) {   // [a, st1, QKV, O, LSE, r1, st2, m, u, g]
     b.a = al(r.z.a); b.st1 = (float2*)al(r.z.st1); b.qkv = al(r.z.qkv); b.O = al(r.z.O);
     b.lse = (float*)al(r.z.lse); b.r1 = (float*)al(r.z.r1); b.st2 = (float2*)al(r.z.st2); b.m = al(r.z.m);
     b.u = al(r.z.u); b.g = al(r.z.g);
@@ -498,7 +539,7 @@ void alloc_internals(Run& r, LayerBufs& b, bool on_stack) {
 void alloc_att(Run& r, LayerBufs& b, bool on_stack) {
   Arena& a = r.c->ar;
   auto al = [&](int64_t n) { return on_stack ? a.push(n) : a.talloc(n); };
-  if (r.c->cfg.arch == 1) {
+  if (r.c->cfg.arch != 0) {
     b.a = al(r.z.a); b.st1 = (float2*)al(r.z.st1); b.qkv = al(r.z.qkv); b.O = al(r.z.O);
     b.lse = (float*)al(r.z.lse);
     return;
@@ -510,13 +551,13 @@ void free_att(Run& r, bool on_stack) {
   Arena& a = r.c->ar;
   const int64_t s0[5] = {r.z.qkv, r.z.O, r.z.lse, r.z.z1, r.z.st1};
   const int64_t s1[5] = {r.z.a, r.z.st1, r.z.qkv, r.z.O, r.z.lse};
-  const int64_t* s = r.c->cfg.arch == 1 ? s1 : s0;
+  const int64_t* s = r.c->cfg.arch != 0 ? s1 : s0;
   for (int i = 4; i >= 0; --i) on_stack ? a.pop(s[i]) : a.tfree(s[i]);
 }
 void alloc_ffn(Run& r, LayerBufs& b, bool on_stack) {
   Arena& a = r.c->ar;
   auto al = [&](int64_t n) { return on_stack ? a.push(n) : a.talloc(n); };
-  if (r.c->cfg.arch == 1) {
+  if (r.c->cfg.arch != 0) {
     b.st2 = (float2*)al(r.z.st2); b.m = al(r.z.m); b.u = al(r.z.u); b.g = al(r.z.g);
     return;
   }
@@ -526,7 +567,7 @@ void free_ffn(Run& r, bool on_stack) {
   Arena& a = r.c->ar;
   const int64_t s0[4] = {r.z.u, r.z.g, r.z.z2, r.z.st2};
   const int64_t s1[4] = {r.z.st2, r.z.m, r.z.u, r.z.g};
-  const int64_t* s = r.c->cfg.arch == 1 ? s1 : s0;
+  const int64_t* s = r.c->cfg.arch != 0 ? s1 : s0;
   for (int i = 3; i >= 0; --i) on_stack ? a.pop(s[i]) : a.tfree(s[i]);
 }
 
@@ -541,7 +582,7 @@ void free_internals(Run& r, bool on_stack) {
   Arena& a = r.c->ar;
   const int64_t s0[10] = {r.z.qkv, r.z.O, r.z.lse, r.z.z1, r.z.st1, r.z.h1, r.z.u, r.z.g, r.z.z2, r.z.st2};
   const int64_t s1[10] = {r.z.a, r.z.st1, r.z.qkv, r.z.O, r.z.lse, r.z.r1, r.z.st2, r.z.m, r.z.u, r.z.g};
-  const int64_t* s = r.c->cfg.arch == 1 ? s1 : s0;
+  const int64_t* s = r.c->cfg.arch != 0 ? s1 : s0;
   for (int i = 9; i >= 0; --i) on_stack ? a.pop(s[i]) : a.tfree(s[i]);
 }
 
@@ -790,7 +831,7 @@ void att_forward_pre(Run& r, int l, const float* x, LayerBufs& b, float* r1out) 
   g.C = b.qkv; g.ldc = 3 * H; g.bias = W(c, LP(c, l, L_QKVB));
   pgemm(c, EPI_BIAS, g, r.st);
   attn_fwd(c->dt, b.qkv, c->lens, b.O, b.lse, c->B, c->S, H, c->cfg.heads, make_drop(c, KIND_ATTN_PROBS, l), r.st,
-           true);
+           c->cfg.arch == 1);   // GPT-2 causal; the encoder-decoder's encoder is bidirectional
   if (!r1out) return;
   g = GemmArgs();
   g.M = T; g.N = H; g.K = H;
@@ -891,7 +932,7 @@ void att_backward_pre(Run& r, int l, const float* x, LayerBufs& b, float* dy, ch
   dgrad(r, EPI_STORE, DT1, H, W(c, LP(c, l, L_OW)), H, R2, nullptr);
   if (!spare) wgrad(r, DT1, H, b.O, H, G(c, LP(c, l, L_OW)));
   attn_bwd(c->dt, b.qkv, b.O, R2, b.lse, c->lens, Dbuf, R3, c->B, c->S, H, h, make_drop(c, KIND_ATTN_PROBS, l),
-           r.st, true);
+           r.st, c->cfg.arch == 1);
   // QKV: da = dQKV Wqkv (fp32, dres); dWo = dt1^T O with dWqkv = dQKV^T a (grouped); dbqkv on the side
   {
     cudaStream_t sa = fork(c, r.st);
@@ -1051,6 +1092,13 @@ mimose_status copy_batch(mimose_ctx* c, const mimose_batch* bt) {
   else if (c->cfg.head == MIMOSE_HEAD_QA) nl = 2 * bt->n_seqs;
   else if (c->cfg.head == 3) nl = 0;            // LM targets are the next input tokens
   else nl = bt->n_seqs;
+  if (c->cfg.arch == 2) {   // source ids / lengths; decoder ids / lengths in the tt / labels buffers
+    CK(cudaMemcpyAsync(c->ids_src, bt->input_ids, T * 4, k, c->st));
+    CK(cudaMemcpyAsync(c->lens_src, bt->lengths, (int64_t)bt->n_seqs * 4, k, c->st));
+    CK(cudaMemcpyAsync(c->ids_tgt, bt->dec_ids, (int64_t)bt->n_seqs * bt->dec_len * 4, k, c->st));
+    CK(cudaMemcpyAsync(c->lens_tgt, bt->dec_lengths, (int64_t)bt->n_seqs * 4, k, c->st));
+    return MIMOSE_OK;
+  }
   CK(cudaMemcpyAsync(c->ids, bt->input_ids, T * 4, k, c->st));
   CK(cudaMemcpyAsync(c->tt, bt->token_type, T * 4, k, c->st));
   CK(cudaMemcpyAsync(c->lens, bt->lengths, (int64_t)bt->n_seqs * 4, k, c->st));
@@ -1065,47 +1113,497 @@ mimose_status check_batch(mimose_ctx* c, const mimose_batch* bt) {
     return fail(c, MIMOSE_E_INVALID, "MC batch: n_seqs must be a multiple of n_choices");
   if (bt->seq_len + c->cfg.pos_offset > c->cfg.max_pos)
     return fail(c, MIMOSE_E_INVALID, "seq_len + pos_offset exceeds max_pos");
+  if (c->cfg.arch == 2 && (bt->dec_len <= 0 || bt->dec_len > c->cfg.max_seq_len ||
+                           bt->dec_len + c->cfg.pos_offset > c->cfg.max_pos ||
+                           (c->device && bt->input_ids && (!bt->dec_ids || !bt->dec_lengths))))
+    return fail(c, MIMOSE_E_INVALID, "encoder-decoder batch: decoder ids / lengths / dec_len in [1, max_seq_len]");
   return MIMOSE_OK;
 }
 
 void layer_fwd_any(Run& r, int l, const char* x, LayerBufs& b, char* yout) {
-  if (r.c->cfg.arch == 1) layer_forward_pre(r, l, (const float*)x, b, (float*)yout);
+  if (r.c->cfg.arch != 0) layer_forward_pre(r, l, (const float*)x, b, (float*)yout);
   else layer_forward(r, l, x, b, yout);
 }
 void layer_bwd_any(Run& r, int l, const char* x, LayerBufs& b, float* dy, char* scr) {
-  if (r.c->cfg.arch == 1) layer_backward_pre(r, l, (const float*)x, b, dy, scr);
+  if (r.c->cfg.arch != 0) layer_backward_pre(r, l, (const float*)x, b, dy, scr);
   else layer_backward(r, l, x, b, dy, scr);
 }
 
 // Sub-layer unit steps for either architecture; the unit boundary tensor ("mid")
 // is h1 = LN1(z1) (post-LN) or r1 = x + drop(attn) (pre-LN).
-int64_t mid_size(const Run& r) { return r.c->cfg.arch == 1 ? r.z.r1 : r.z.h1; }
-char* mid_of(const Run& r, const LayerBufs& b) { return r.c->cfg.arch == 1 ? (char*)b.r1 : b.h1; }
+int64_t mid_size(const Run& r) { return r.c->cfg.arch != 0 ? r.z.r1 : r.z.h1; }
+char* mid_of(const Run& r, const LayerBufs& b) { return r.c->cfg.arch != 0 ? (char*)b.r1 : b.h1; }
 void set_mid(const Run& r, LayerBufs& b, char* p) {
-  if (r.c->cfg.arch == 1) b.r1 = (float*)p;
+  if (r.c->cfg.arch != 0) b.r1 = (float*)p;
   else b.h1 = p;
 }
 void att_fwd_u(Run& r, int l, const char* x, LayerBufs& b, char* mid_out) {
-  if (r.c->cfg.arch == 1) att_forward_pre(r, l, (const float*)x, b, (float*)mid_out);
+  if (r.c->cfg.arch != 0) att_forward_pre(r, l, (const float*)x, b, (float*)mid_out);
   else att_forward(r, l, x, b, mid_out);
 }
 void ffn_fwd_u(Run& r, int l, LayerBufs& b, char* yout) {
-  if (r.c->cfg.arch == 1) ffn_forward_pre(r, l, b, (float*)yout);
+  if (r.c->cfg.arch != 0) ffn_forward_pre(r, l, b, (float*)yout);
   else ffn_forward(r, l, b, yout);
 }
 void ffn_bwd_u(Run& r, int l, LayerBufs& b, float* dy, char* scr) {
-  if (r.c->cfg.arch == 1) ffn_backward_pre(r, l, b, dy, scr);
+  if (r.c->cfg.arch != 0) ffn_backward_pre(r, l, b, dy, scr);
   else ffn_backward(r, l, b, dy, scr);
 }
 void att_bwd_u(Run& r, int l, const char* x, LayerBufs& b, float* dy, char* scr) {
-  if (r.c->cfg.arch == 1) att_backward_pre(r, l, (const float*)x, b, dy, scr);
+  if (r.c->cfg.arch != 0) att_backward_pre(r, l, (const float*)x, b, dy, scr);
   else att_backward(r, l, x, b, dy, scr);
+}
+
+// ===========================================================================
+// Encoder-decoder (reading A32; DESIGN §3 "Encoder-decoder").
+// Units: encoder layers 0..Le-1 (pre-LN, bidirectional: the GPT-2 layer code
+// with a non-causal mask), decoder layers Le..Le+Ld-1 (pre-LN: causal
+// self-attention, cross-attention on the encoder output, FFN).  The last
+// encoder unit's output bundle is [x_L, enc_out = LN_enc(x_L), enc_st, x1_t].
+// Arena order and sizes follow oracle/memsim.py sizes_encdec exactly.
+// ===========================================================================
+inline int EL(const mimose_ctx* c, int k) { return 2 + 12 * c->cfg.n_layers + k; }   // encoder final LN
+inline int DP(const mimose_ctx* c, int j, int k) { return 2 + 12 * c->cfg.n_layers + 2 + 20 * j + k; }
+enum { D_LN1G = 0, D_LN1B, D_QKVW, D_QKVB, D_OW, D_OB, D_LN2G, D_LN2B, D_CQW, D_CQB, D_CKVW, D_CKVB, D_COW, D_COB,
+       D_LN3G, D_LN3B, D_F1W, D_F1B, D_F2W, D_F2B };
+constexpr uint32_t DEC_EMB_LAYER = 0xFFE;
+constexpr uint32_t KIND_CROSS_PROBS = 5, KIND_CROSS_OUT = 6;
+
+struct SzD {                 // decoder-side and shared sizes of one (B, Ss, St)
+  int64_t a, st, qkv, O, lse, r, c, qc, kvc, m, u, g, y;   // decoder internals (st/r/lse shared shapes)
+  int64_t xL, enc_out, enc_st, x1t;                         // the bundle
+  int64_t head0, head1, head2, head_fwd, head_scr;
+  int64_t dy, denc, U, embU;
+  int64_t scr_enc_off, scr_kv_off;                          // carve offsets inside U
+};
+
+SzD sizes_dec(const mimose_ctx* c, int B, int Ss, int St) {
+  const int64_t Ts = (int64_t)B * Ss, Tt = (int64_t)B * St, H = c->cfg.hidden, F = c->cfg.ffn, h = c->cfg.heads,
+                e = c->e;
+  SzD z{};
+  z.a = a16(Tt * H * e); z.st = a16(Tt * 8); z.qkv = a16(Tt * 3 * H * e); z.O = a16(Tt * H * e);
+  z.lse = a16((int64_t)B * h * St * 4); z.r = a16(Tt * H * 4); z.c = a16(Tt * H * e); z.qc = a16(Tt * H * e);
+  z.kvc = a16(Ts * 2 * H * e); z.m = a16(Tt * H * e); z.u = a16(Tt * F * e); z.g = a16(Tt * F * e);
+  z.y = a16(Tt * H * 4);
+  z.xL = a16(Ts * H * 4); z.enc_out = a16(Ts * H * e); z.enc_st = a16(Ts * 8); z.x1t = a16(Tt * H * 4);
+  const int64_t VP = vpad(c->cfg.vocab);
+  z.head0 = a16(Tt * H * e); z.head1 = a16(Tt * 8); z.head2 = a16(Tt * 8);
+  z.head_fwd = a16((int64_t)LM_CHUNK * VP * 4);
+  z.head_scr = a16((int64_t)LM_CHUNK * VP * 4) + a16((int64_t)LM_CHUNK * VP * e);
+  z.dy = a16(Tt * H * 4); z.denc = a16(Ts * H * 4);
+  auto lscr = [&](int64_t T, int64_t S) {
+    return a16(T * H * 4) + a16(T * F * e) + a16(T * 3 * H * e) + a16((int64_t)B * h * S * 4);
+  };
+  z.scr_kv_off = lscr(Tt, St);
+  z.scr_enc_off = z.scr_kv_off + a16(Ts * 2 * H * e);
+  z.U = z.scr_enc_off + lscr(Ts, Ss);
+  const int64_t maxT = (int64_t)c->cfg.max_seqs * c->cfg.max_seq_len;
+  const int64_t ntiles = (maxT + 1023) / 1024;
+  auto escr = [&](int64_t T) { return a16(T * H * 4) + a16(16 * T) + a16(4 * 256 * ntiles); };
+  z.embU = escr(Ts) + escr(Tt);
+  return z;
+}
+
+
+
+// The decoder internals in the order of oracle/memsim.py sizes_encdec:
+// a st1 QKV O LSE r1 st2 c Qc KVc Oc LSEc r2 st3 m u g
+void dec_sizes_list(const SzD& z, int64_t* s) {
+  const int64_t v[17] = {z.a, z.st, z.qkv, z.O, z.lse, z.r, z.st, z.c, z.qc, z.kvc, z.O, z.lse, z.r, z.st, z.m, z.u, z.g};
+  for (int i = 0; i < 17; ++i) s[i] = v[i];
+}
+void alloc_dec(mimose_ctx* c, const SzD& z, DecBufs& b, bool on_stack) {
+  Arena& a = c->ar;
+  auto al = [&](int64_t n) { return on_stack ? a.push(n) : a.talloc(n); };
+  b.a = al(z.a); b.st1 = (float2*)al(z.st); b.qkv = al(z.qkv); b.O = al(z.O); b.lse = (float*)al(z.lse);
+  b.r1 = (float*)al(z.r); b.st2 = (float2*)al(z.st); b.c = al(z.c); b.qc = al(z.qc); b.kvc = al(z.kvc);
+  b.oc = al(z.O); b.lsec = (float*)al(z.lse); b.r2 = (float*)al(z.r); b.st3 = (float2*)al(z.st); b.m = al(z.m);
+  b.u = al(z.u); b.g = al(z.g);
+}
+void free_dec(mimose_ctx* c, const SzD& z, bool on_stack) {
+  int64_t s[17];
+  dec_sizes_list(z, s);
+  for (int i = 16; i >= 0; --i) on_stack ? c->ar.pop(s[i]) : c->ar.tfree(s[i]);
+}
+
+// Point the step state at one stack: the layer kernels read c->S, c->T and the
+// key/query lengths through c->lens, the LM head the ids through c->ids.
+void use_enc(mimose_ctx* c) {
+  c->S = c->Ss; c->T = c->B * c->Ss;
+  c->lens = c->lens_src; c->ids = c->ids_src;
+}
+void use_dec(mimose_ctx* c) {
+  c->S = c->St; c->T = c->B * c->St;
+  c->lens = c->lens_tgt; c->ids = c->ids_tgt;
+}
+
+void dec_layer_forward(Run& r, const SzD& z, int j, const float* x, DecBufs& b, float* yout) {
+  mimose_ctx* c = r.c;
+  if (!r.real) return;
+  use_dec(c);
+  const int Tt = c->T, Ts = c->B * c->Ss, H = c->cfg.hidden, F = c->cfg.ffn, h = c->cfg.heads;
+  const uint32_t site = (uint32_t)(c->cfg.n_layers + j);
+  ln_fwd(c->dt, x, W(c, DP(c, j, D_LN1G)), W(c, DP(c, j, D_LN1B)), b.a, b.st1, Tt, H, c->cfg.ln_eps, r.st);
+  GemmArgs g;
+  g.M = Tt; g.N = 3 * H; g.K = H;
+  g.A = b.a; g.a_sm = H; g.a_sk = 1;
+  g.B = W(c, DP(c, j, D_QKVW)); g.b_sn = H; g.b_sk = 1;
+  g.C = b.qkv; g.ldc = 3 * H; g.bias = W(c, DP(c, j, D_QKVB));
+  pgemm(c, EPI_BIAS, g, r.st);
+  attn_fwd(c->dt, b.qkv, c->lens_tgt, b.O, b.lse, c->B, c->St, H, h, make_drop(c, KIND_ATTN_PROBS, site), r.st, true);
+  g = GemmArgs();
+  g.M = Tt; g.N = H; g.K = H;
+  g.A = b.O; g.a_sm = H; g.a_sk = 1;
+  g.B = W(c, DP(c, j, D_OW)); g.b_sn = H; g.b_sk = 1;
+  g.C = b.r1; g.ldc = H; g.bias = W(c, DP(c, j, D_OB)); g.res = x; g.ldr = H;
+  g.drop = make_drop(c, KIND_ATTN_OUT, site);
+  pgemm(c, EPI_BIAS_DROP_RESF32, g, r.st);
+  // cross-attention: Q from LN2(r1), K / V from the encoder output
+  ln_fwd(c->dt, b.r1, W(c, DP(c, j, D_LN2G)), W(c, DP(c, j, D_LN2B)), b.c, b.st2, Tt, H, c->cfg.ln_eps, r.st);
+  g = GemmArgs();
+  g.M = Tt; g.N = H; g.K = H;
+  g.A = b.c; g.a_sm = H; g.a_sk = 1;
+  g.B = W(c, DP(c, j, D_CQW)); g.b_sn = H; g.b_sk = 1;
+  g.C = b.qc; g.ldc = H; g.bias = W(c, DP(c, j, D_CQB));
+  pgemm(c, EPI_BIAS, g, r.st);
+  g = GemmArgs();
+  g.M = Ts; g.N = 2 * H; g.K = H;
+  g.A = c->enc_out; g.a_sm = H; g.a_sk = 1;
+  g.B = W(c, DP(c, j, D_CKVW)); g.b_sn = H; g.b_sk = 1;
+  g.C = b.kvc; g.ldc = 2 * H; g.bias = W(c, DP(c, j, D_CKVB));
+  pgemm(c, EPI_BIAS, g, r.st);
+  attn_cross_fwd_tc(b.qc, b.kvc, c->lens_tgt, c->lens_src, b.oc, b.lsec, c->B, c->St, c->Ss, H, h,
+                    make_drop(c, KIND_CROSS_PROBS, site), r.st);
+  note_launch(1);
+  g = GemmArgs();
+  g.M = Tt; g.N = H; g.K = H;
+  g.A = b.oc; g.a_sm = H; g.a_sk = 1;
+  g.B = W(c, DP(c, j, D_COW)); g.b_sn = H; g.b_sk = 1;
+  g.C = b.r2; g.ldc = H; g.bias = W(c, DP(c, j, D_COB)); g.res = b.r1; g.ldr = H;
+  g.drop = make_drop(c, KIND_CROSS_OUT, site);
+  pgemm(c, EPI_BIAS_DROP_RESF32, g, r.st);
+  // FFN
+  ln_fwd(c->dt, b.r2, W(c, DP(c, j, D_LN3G)), W(c, DP(c, j, D_LN3B)), b.m, b.st3, Tt, H, c->cfg.ln_eps, r.st);
+  g = GemmArgs();
+  g.M = Tt; g.N = F; g.K = H;
+  g.A = b.m; g.a_sm = H; g.a_sk = 1;
+  g.B = W(c, DP(c, j, D_F1W)); g.b_sn = H; g.b_sk = 1;
+  g.C = b.u; g.C2 = b.g; g.ldc = F; g.bias = W(c, DP(c, j, D_F1B));
+  pgemm(c, EPI_BIAS_GELUT, g, r.st);
+  if (!yout) return;                            // recompute: y is not needed
+  g = GemmArgs();
+  g.M = Tt; g.N = H; g.K = F;
+  g.A = b.g; g.a_sm = F; g.a_sk = 1;
+  g.B = W(c, DP(c, j, D_F2W)); g.b_sn = F; g.b_sk = 1;
+  g.C = yout; g.ldc = H; g.bias = W(c, DP(c, j, D_F2B)); g.res = b.r2; g.ldr = H;
+  g.drop = make_drop(c, KIND_FFN_OUT, site);
+  pgemm(c, EPI_BIAS_DROP_RESF32, g, r.st);
+}
+
+// Decoder layer backward: dy (fp32 [Tt, H]) in place -> dx; denc (fp32 [Ts, H]) += the
+// cross-attention K / V path.  scr = the uniform layer scratch.
+void dec_layer_backward(Run& r, const SzD& z, int j, const float* x, DecBufs& b, float* dy, float* denc, char* scr) {
+  mimose_ctx* c = r.c;
+  if (!r.real) return;
+  use_dec(c);
+  const int Tt = c->T, Ts = c->B * c->Ss, H = c->cfg.hidden, F = c->cfg.ffn, h = c->cfg.heads;
+  const uint32_t site = (uint32_t)(c->cfg.n_layers + j);
+  const Sz zt = sizes(c, c->B, c->St);
+  float* dres = (float*)(scr + zt.r_dres);
+  char* R2 = scr + zt.r_du;                     // du; then dOc / dO in its head, dtc / dt1 in its tail
+  char* R3 = scr + zt.r_dt;                     // dt3; then dQc; then dQKV
+  float* Dbuf = (float*)(scr + zt.r_dt + a16((int64_t)Tt * 3 * H * c->e));
+  char* dKV = scr + z.scr_kv_off;
+  char* TAIL = R2 + a16((int64_t)Tt * H * c->e);
+  float* pg = c->part;
+  float* pb = c->part + (int64_t)NPART * H;
+  float* pbias = c->part + 2LL * NPART * H;
+  // FFN: dt3 = dy * mask (bf16) with db2; du = (dt3 W2) * gelu_tanh'(u); dW2; dm = du W1; dW1; db1
+  drop_cast_colsum(c->dt, dy, make_drop(c, KIND_FFN_OUT, site), R3, Tt, H, pbias, r.st);
+  reduce_partials(pbias, H, H, G(c, DP(c, j, D_F2B)), r.st);
+  {
+    GemmArgs g;
+    g.M = Tt; g.N = F; g.K = H;
+    g.A = R3; g.a_sm = H; g.a_sk = 1;
+    g.B = W(c, DP(c, j, D_F2W)); g.b_sn = 1; g.b_sk = F;
+    g.C = R2; g.ldc = F; g.aux = b.u; g.ldx = F;
+    pgemm(c, EPI_GELUT_BWD, g, r.st);
+  }
+  wgrad(r, R3, H, b.g, F, G(c, DP(c, j, D_F2W)));
+  dgrad(r, EPI_F32, R2, F, W(c, DP(c, j, D_F1W)), H, dres, nullptr);
+  wgrad(r, R2, F, b.m, H, G(c, DP(c, j, D_F1W)));
+  colsum(c->dt, R2, Tt, F, part_cs(c), r.st);
+  reduce_partials(part_cs(c), F, F, G(c, DP(c, j, D_F1B)), r.st);
+  // LN3 backward + residual: dr2 = dy + LN3'(dm) (in place in dy); dtc = dr2 * mask (TAIL); dbco
+  ln_bwd(c->dt, dres, no_drop(), b.r2, b.st3, W(c, DP(c, j, D_LN3G)), dy, TAIL, make_drop(c, KIND_CROSS_OUT, site),
+         pg, pb, pbias, Tt, H, r.st, dy);
+  reduce_rows3(pg, G(c, DP(c, j, D_LN3G)), pb, G(c, DP(c, j, D_LN3B)), pbias, G(c, DP(c, j, D_COB)), NPART, H, H,
+               r.st);
+  // cross-attention: dOc = dtc Wco (R2 head); dWco; attention backward -> dQc (R3), dKV
+  dgrad(r, EPI_STORE, TAIL, H, W(c, DP(c, j, D_COW)), H, R2, nullptr);
+  wgrad(r, TAIL, H, b.oc, H, G(c, DP(c, j, D_COW)));
+  attn_cross_bwd_tc(b.qc, b.kvc, b.oc, R2, b.lsec, c->lens_tgt, c->lens_src, R3, dKV, c->B, c->St, c->Ss, H, h,
+                    make_drop(c, KIND_CROSS_PROBS, site), r.st);
+  note_launch(1);
+  // dc = dQc Wcq (dres); dWcq; dbcq
+  dgrad(r, EPI_F32, R3, H, W(c, DP(c, j, D_CQW)), H, dres, nullptr);
+  wgrad(r, R3, H, b.c, H, G(c, DP(c, j, D_CQW)));
+  colsum(c->dt, R3, Tt, H, part_cs(c), r.st);
+  reduce_partials(part_cs(c), H, H, G(c, DP(c, j, D_CQB)), r.st);
+  // denc += dKV Wckv (M = Ts); dWckv = dKV^T enc_out; dbckv
+  {
+    GemmArgs g;
+    g.M = Ts; g.N = H; g.K = 2 * H;
+    g.A = dKV; g.a_sm = 2 * H; g.a_sk = 1;
+    g.B = W(c, DP(c, j, D_CKVW)); g.b_sn = 1; g.b_sk = H;
+    g.C = denc; g.ldc = H; g.res = denc; g.ldr = H;
+    pgemm(c, EPI_ACC_RES_F32, g, r.st);
+  }
+  {
+    const int sT = c->T;
+    c->T = Ts;                                   // the weight gradient contracts over the source tokens
+    wgrad(r, dKV, 2 * H, c->enc_out, H, G(c, DP(c, j, D_CKVW)));
+    c->T = sT;
+  }
+  colsum(c->dt, dKV, Ts, 2 * H, part_cs(c), r.st);
+  reduce_partials(part_cs(c), 2 * H, 2 * H, G(c, DP(c, j, D_CKVB)), r.st);
+  // LN2 backward + residual: dr1 = dr2 + LN2'(dc) (in place in dy); dt1 = dr1 * mask (TAIL)
+  ln_bwd(c->dt, dres, no_drop(), b.r1, b.st2, W(c, DP(c, j, D_LN2G)), dy, TAIL, make_drop(c, KIND_ATTN_OUT, site),
+         pg, pb, pbias, Tt, H, r.st, dy);
+  reduce_rows3(pg, G(c, DP(c, j, D_LN2G)), pb, G(c, DP(c, j, D_LN2B)), pbias, G(c, DP(c, j, D_OB)), NPART, H, H,
+               r.st);
+  // self-attention: dO = dt1 Wo (R2 head); dWo; attention backward -> dQKV (R3); da = dQKV Wqkv
+  dgrad(r, EPI_STORE, TAIL, H, W(c, DP(c, j, D_OW)), H, R2, nullptr);
+  wgrad(r, TAIL, H, b.O, H, G(c, DP(c, j, D_OW)));
+  attn_bwd(c->dt, b.qkv, b.O, R2, b.lse, c->lens_tgt, Dbuf, R3, c->B, c->St, H, h, make_drop(c, KIND_ATTN_PROBS, site),
+           r.st, true);
+  dgrad(r, EPI_F32, R3, 3 * H, W(c, DP(c, j, D_QKVW)), H, dres, nullptr);
+  wgrad(r, R3, 3 * H, b.a, H, G(c, DP(c, j, D_QKVW)));
+  colsum(c->dt, R3, Tt, 3 * H, part_cs(c), r.st);
+  reduce_partials(part_cs(c), 3 * H, 3 * H, G(c, DP(c, j, D_QKVB)), r.st);
+  // LN1 backward + residual: dx = dr1 + LN1'(da) (in place in dy)
+  ln_bwd(c->dt, dres, no_drop(), x, b.st1, W(c, DP(c, j, D_LN1G)), dy, nullptr, no_drop(), pg, pb, nullptr, Tt, H,
+         r.st, dy);
+  reduce_rows3(pg, G(c, DP(c, j, D_LN1G)), pb, G(c, DP(c, j, D_LN1B)), nullptr, nullptr, NPART, H, H, r.st);
+}
+
+// The last encoder unit's extra output: enc_out = LN_enc(x_L) and the decoder embedding x1_t.
+void enc_tail_forward(Run& r, const float* xL, char* enc_out, float2* enc_st, float* x1t) {
+  mimose_ctx* c = r.c;
+  if (!r.real) return;
+  const int H = c->cfg.hidden;
+  ln_fwd(c->dt, xL, W(c, EL(c, 0)), W(c, EL(c, 1)), enc_out, enc_st, c->B * c->Ss, H, c->cfg.ln_eps, r.st);
+  embed_fwd_pre(c->dt, c->ids_tgt, W(c, P_WORD), W(c, P_POS), x1t, c->B, c->St, H, c->cfg.pos_offset,
+                make_drop(c, KIND_EMB, DEC_EMB_LAYER), r.st);
+}
+
+void run_forward_ed(Run& r, uint64_t mask, bool collect, Sample* sample) {
+  mimose_ctx* c = r.c;
+  Arena& a = c->ar;
+  const int Le = c->cfg.n_layers, Ld = c->cfg.n_dec_layers, H = c->cfg.hidden;
+  const SzD zd = sizes_dec(c, c->B, c->Ss, c->St);
+  r.z = sizes(c, c->B, c->Ss);                       // encoder-layer sizes (GPT-2 layer list at T_s)
+  const int64_t base = a.live();
+  use_enc(c);
+  c->x1 = a.push(r.z.x1);                            // x1_s
+  if (sample) sample->E = a.live() - base;
+  if (r.real)
+    embed_fwd_pre(c->dt, c->ids_src, W(c, P_WORD), W(c, P_POS), (float*)c->x1, c->B, c->Ss, H, c->cfg.pos_offset,
+                  make_drop(c, KIND_EMB, LAYER_NONE), r.st);
+  c->lb.assign(Le, LayerBufs());
+  c->dlb.assign(Ld, DecBufs());
+  c->y.assign(Le + Ld, nullptr);
+  const char* x = c->x1;
+  for (int l = 0; l < Le; ++l) {
+    use_enc(c);
+    const int64_t b0 = a.live();
+    const bool last = l == Le - 1;
+    if (collect && sample) {                         // pass 1 (save mode), timed, discarded
+      LayerBufs tmp;
+      alloc_internals(r, tmp, true);
+      char* yt = a.push(r.z.y);
+      char *eo = nullptr, *x1t = nullptr;
+      float2* es = nullptr;
+      if (last) { eo = a.push(zd.enc_out); es = (float2*)a.push(zd.enc_st); x1t = a.push(zd.x1t); }
+      if (r.real) cudaEventRecord(c->ev_t0[l], r.st);
+      layer_fwd_any(r, l, x, tmp, yt);
+      if (last) { char* so = c->enc_out; c->enc_out = eo; enc_tail_forward(r, (float*)yt, eo, es, (float*)x1t); c->enc_out = so; }
+      if (r.real) cudaEventRecord(c->ev_t1[l], r.st);
+      sample->a[l] = a.live() - b0;
+      if (last) { a.pop(zd.x1t); a.pop(zd.enc_st); a.pop(zd.enc_out); }
+      a.pop(r.z.y);
+      free_internals(r, true);
+    }
+    const bool dropped = collect || ((mask >> l) & 1);
+    alloc_internals(r, c->lb[l], !dropped);
+    c->y[l] = a.push(r.z.y);
+    if (last) {
+      c->enc_out = a.push(zd.enc_out);
+      c->enc_st = (float2*)a.push(zd.enc_st);
+      c->x1t = a.push(zd.x1t);
+    }
+    layer_fwd_any(r, l, x, c->lb[l], c->y[l]);
+    if (last) enc_tail_forward(r, (float*)c->y[l], c->enc_out, c->enc_st, (float*)c->x1t);
+    if (dropped) free_internals(r, false);
+    if (sample) sample->y[l] = a.live() - b0;
+    x = c->y[l];
+  }
+  x = c->x1t;
+  for (int j = 0; j < Ld; ++j) {
+    const int u = Le + j;
+    const int64_t b0 = a.live();
+    if (collect && sample) {
+      DecBufs tmp;
+      alloc_dec(c, zd, tmp, true);
+      char* yt = a.push(zd.y);
+      if (r.real) cudaEventRecord(c->ev_t0[u], r.st);
+      dec_layer_forward(r, zd, j, (const float*)x, tmp, (float*)yt);
+      if (r.real) cudaEventRecord(c->ev_t1[u], r.st);
+      sample->a[u] = a.live() - b0;
+      a.pop(zd.y);
+      free_dec(c, zd, true);
+    }
+    const bool dropped = collect || ((mask >> u) & 1);
+    alloc_dec(c, zd, c->dlb[j], !dropped);
+    c->y[u] = a.push(zd.y);
+    dec_layer_forward(r, zd, j, (const float*)x, c->dlb[j], (float*)c->y[u]);
+    if (dropped) free_dec(c, zd, false);
+    if (sample) sample->y[u] = a.live() - b0;
+    x = c->y[u];
+  }
+  use_dec(c);
+  const int64_t h0 = a.live();
+  c->hp = a.push(zd.head0);
+  c->lm_stf = (float2*)a.push(zd.head1);
+  c->lm_tok = (float2*)a.push(zd.head2);
+  if (sample) sample->Hd = a.live() - h0;
+  float* lg = (float*)a.talloc(zd.head_fwd);
+  if (r.real) lm_head_forward(r, (float*)c->y[Le + Ld - 1], c->hp, c->lm_stf, c->lm_tok, lg);
+  a.tfree(zd.head_fwd);
+}
+
+mimose_status run_backward_ed(Run& r, Sample* sample) {
+  mimose_ctx* c = r.c;
+  Arena& a = c->ar;
+  const int Le = c->cfg.n_layers, Ld = c->cfg.n_dec_layers, H = c->cfg.hidden;
+  const SzD zd = sizes_dec(c, c->B, c->Ss, c->St);
+  r.z = sizes(c, c->B, c->Ss);
+  const int Ts = c->B * c->Ss, Tt = c->B * c->St;
+  float* denc = (float*)a.talloc(zd.denc);
+  float* dy = (float*)a.talloc(zd.dy);
+  if (r.real) CK(cudaMemsetAsync(denc, 0, (size_t)Ts * H * 4, r.st));
+  // ---- LM head on the decoder ----
+  use_dec(c);
+  a.top_phase_peak = a.top;
+  char* hs = a.talloc(zd.head_scr);
+  if (r.real) {
+    CK(cudaMemsetAsync(G(c, P_WORD), 0, (size_t)c->layout[P_WORD].numel * 4, r.st));
+    lm_head_backward(r, (float*)c->y[Le + Ld - 1], c->hp, c->lm_stf, c->lm_tok, hs, dy);
+  }
+  a.tfree(zd.head_scr);
+  if (sample) sample->Th = a.top_phase_peak;
+  a.pop(zd.head2);
+  a.pop(zd.head1);
+  a.pop(zd.head0);
+  a.pop(zd.y);                                        // the last decoder output
+  // ---- decoder layers ----
+  a.top_phase_peak = a.top;
+  int64_t tb = 0, te = 0;
+  for (int j = Ld - 1; j >= 0; --j) {
+    const int u = Le + j;
+    const float* x = j > 0 ? (const float*)c->y[u - 1] : (const float*)c->x1t;
+    if ((c->drop_mask >> u) & 1) {
+      if (r.real) join(c, r.st);
+      alloc_dec(c, zd, c->dlb[j], true);
+      dec_layer_forward(r, zd, j, x, c->dlb[j], nullptr);
+    }
+    char* scr = a.talloc(zd.U);
+    dec_layer_backward(r, zd, j, x, c->dlb[j], dy, denc, scr);
+    a.tfree(zd.U);
+    free_dec(c, zd, true);
+    if (j > 0) a.pop(zd.y);
+  }
+  tb = a.top_phase_peak;
+  // ---- decoder embedding (tied wte accumulates onto the LM head's dW_e) ----
+  a.top_phase_peak = a.top;
+  char* es = a.talloc(zd.embU);
+  if (r.real) {
+    float* dz0 = (float*)es;
+    int32_t* work = (int32_t*)(es + a16((int64_t)Tt * H * 4));
+    int32_t* hist = (int32_t*)(es + a16((int64_t)Tt * H * 4) + a16(16LL * Tt));
+    drop_f32(dy, make_drop(c, KIND_EMB, DEC_EMB_LAYER), dz0, (int64_t)Tt * H, r.st);
+    pos_grad(dz0, c->B, c->St, H, c->cfg.pos_offset, G(c, P_POS), r.st);    // (writes every row below St)
+    const int64_t maxT = (int64_t)c->cfg.max_seqs * c->cfg.max_seq_len;
+    keyed_rowsum(c->ids_tgt, c->cfg.vocab <= 256 ? 8 : 16, dz0, Tt, H, G(c, P_WORD), work, hist,
+                 (int)((maxT + 1023) / 1024), c->cfg.pad_id, r.st, /*accumulate=*/true);
+  }
+  a.tfree(zd.embU);
+  te = a.top_phase_peak;
+  a.pop(zd.x1t);
+  // ---- encoder final LN (in place in denc) ----
+  use_enc(c);
+  if (r.real) {
+    float* pg = c->part;
+    float* pb = c->part + (int64_t)NPART * H;
+    ln_bwd(c->dt, denc, no_drop(), (const float*)c->y[Le - 1], c->enc_st, W(c, EL(c, 0)), denc, nullptr, no_drop(),
+           pg, pb, nullptr, Ts, H, r.st);
+    reduce_rows3(pg, G(c, EL(c, 0)), pb, G(c, EL(c, 1)), nullptr, nullptr, NPART, H, H, r.st);
+  }
+  a.pop(zd.enc_st);
+  a.pop(zd.enc_out);
+  a.pop(r.z.y);                                       // x_L
+  // ---- encoder layers (GPT-2 layer code, bidirectional) ----
+  a.top_phase_peak = a.top;
+  for (int l = Le - 1; l >= 0; --l) {
+    use_enc(c);
+    const char* x = l > 0 ? c->y[l - 1] : c->x1;
+    if ((c->drop_mask >> l) & 1) {
+      if (r.real) join(c, r.st);
+      alloc_internals(r, c->lb[l], true);
+      layer_fwd_any(r, l, x, c->lb[l], nullptr);
+    }
+    char* scr = a.talloc(zd.U);
+    layer_bwd_any(r, l, x, c->lb[l], denc, scr);
+    a.tfree(zd.U);
+    free_internals(r, true);
+    if (l > 0) a.pop(r.z.y);
+  }
+  tb = std::max(tb, a.top_phase_peak);
+  if (r.real) join(c, r.st);
+  // ---- encoder embedding ----
+  a.top_phase_peak = a.top;
+  es = a.talloc(zd.embU);
+  if (r.real) {
+    float* dz0 = (float*)es;
+    int32_t* work = (int32_t*)(es + a16((int64_t)Ts * H * 4));
+    int32_t* hist = (int32_t*)(es + a16((int64_t)Ts * H * 4) + a16(16LL * Ts));
+    drop_f32(denc, make_drop(c, KIND_EMB, LAYER_NONE), dz0, (int64_t)Ts * H, r.st);
+    if (c->St < c->cfg.max_pos)                      // rows the decoder did not write
+      CK(cudaMemsetAsync(G(c, P_POS) + (int64_t)(c->cfg.pos_offset + c->St) * H, 0,
+                         (size_t)(c->cfg.max_pos - c->cfg.pos_offset - c->St) * H * 4, r.st));
+    pos_grad(dz0, c->B, c->Ss, H, c->cfg.pos_offset, G(c, P_POS), r.st, /*accumulate=*/true);
+    const int64_t maxT = (int64_t)c->cfg.max_seqs * c->cfg.max_seq_len;
+    keyed_rowsum(c->ids_src, c->cfg.vocab <= 256 ? 8 : 16, dz0, Ts, H, G(c, P_WORD), work, hist,
+                 (int)((maxT + 1023) / 1024), c->cfg.pad_id, r.st, /*accumulate=*/true);
+  }
+  a.tfree(zd.embU);
+  te = std::max(te, a.top_phase_peak);
+  if (sample) { sample->Tb = tb; sample->Te = te; }
+  a.pop(r.z.x1);
+  a.tfree(zd.dy);
+  a.tfree(zd.denc);
+  if (r.real) {
+    mimose_status s = allreduce_bucket(c, 0, (int)c->layout.size() - 1, Le + 1);   // one bucket: every tensor
+    if (s) return s;
+  }
+  return MIMOSE_OK;
 }
 
 // Forward of one step.  mode 0: plan-driven; mode 1: shuttling collector.
 // When `sample` is non-null the collector deltas are recorded.
 void run_forward(Run& r, uint64_t mask, bool collect, Sample* sample) {
   mimose_ctx* c = r.c;
+  if (c->cfg.arch == 2) return run_forward_ed(r, mask, collect, sample);
   Arena& a = c->ar;
   const int L = c->cfg.n_layers, H = c->cfg.hidden;
   const int64_t base = a.live();
@@ -1226,6 +1724,7 @@ void run_forward(Run& r, uint64_t mask, bool collect, Sample* sample) {
 
 mimose_status run_backward(Run& r, Sample* sample) {
   mimose_ctx* c = r.c;
+  if (c->cfg.arch == 2) return run_backward_ed(r, sample);
   Arena& a = c->ar;
   const int L = c->cfg.n_layers, H = c->cfg.hidden;
   const int T = c->T;
@@ -1364,9 +1863,14 @@ mimose_status run_backward(Run& r, Sample* sample) {
 }
 
 // Host-only accounting of a full step: peak bytes and breach flag.
-void dry_step(mimose_ctx* c, int B, int S, uint64_t mask, bool collect, int64_t* peak, bool* breach, Sample* smp) {
+void dry_step(mimose_ctx* c, int B, int S, uint64_t mask, bool collect, int64_t* peak, bool* breach, Sample* smp,
+              int St = 0) {
   // Save the ctx step state that the dry run overwrites.
-  const int sB = c->B, sS = c->S, sT = c->T;
+  const int sB = c->B, sS = c->S, sT = c->T, sSs = c->Ss, sSt = c->St;
+  int32_t *sids = c->ids, *slens = c->lens;
+  char *seo = c->enc_out, *sx1t = c->x1t;
+  float2* sest = c->enc_st;
+  std::vector<DecBufs> sdlb = c->dlb;
   const uint64_t sm = c->drop_mask;
   Arena saved = c->ar;
   float* sz0 = c->z0;
@@ -1377,6 +1881,7 @@ void dry_step(mimose_ctx* c, int B, int S, uint64_t mask, bool collect, int64_t*
   std::vector<LayerBufs> slb = c->lb;
   std::vector<char*> sy = c->y;
   c->B = B; c->S = S; c->T = B * S;
+  c->Ss = S; c->St = St;
   c->drop_mask = collect ? ~0ull : mask;
   c->ar.reset_step();
   c->ar.base = nullptr;
@@ -1390,6 +1895,8 @@ void dry_step(mimose_ctx* c, int B, int S, uint64_t mask, bool collect, int64_t*
   c->z0 = sz0; c->x1 = sx1; c->hp = shp; c->st0 = sst0; c->logits = slog;
   c->lm_stf = slst; c->lm_tok = sltk;
   c->lb = slb; c->y = sy;
+  c->Ss = sSs; c->St = sSt; c->ids = sids; c->lens = slens;
+  c->enc_out = seo; c->x1t = sx1t; c->enc_st = sest; c->dlb = sdlb;
 }
 
 mimose_status check_ready(mimose_ctx* c) {
@@ -1496,7 +2003,11 @@ mimose_status mimose_init(const mimose_config* cfgp, mimose_ctx** out) {
   c->cfg = *cfgp;
   const mimose_config& k = c->cfg;
   auto bad = [&](const char* m) { c->err = m; return MIMOSE_E_INVALID; };
-  const bool arch_ok = (k.arch == MIMOSE_ARCH_POST_LN && k.head >= 0 && k.head <= 2) || (k.arch == 1 && k.head == 3);
+  const bool arch_ok = (k.arch == MIMOSE_ARCH_POST_LN && k.head >= 0 && k.head <= 2) || (k.arch == 1 && k.head == 3) ||
+                       (k.arch == 2 && k.head == 3 && k.n_dec_layers >= 1 && k.n_layers + k.n_dec_layers <= 64 &&
+                        k.granularity == 0 && k.zero1 == 0 && !k.ffn_layers && k.max_seq_len <= 128 &&
+                        k.hidden / k.heads == 64 && k.ffn >= 2 * k.hidden &&
+                        (!k.arena_base || (k.dtype == MIMOSE_BF16 && k.use_tc)));
   if (!arch_ok || k.n_layers < 1 || k.n_layers > 64 || k.hidden % 64 || k.heads < 1 ||
       k.hidden % k.heads || (k.hidden / k.heads != 32 && k.hidden / k.heads != 64) || k.ffn % 64 ||
       k.hidden > 1024 || k.ffn > 4096 || k.vocab < 1 || k.vocab > 65536 || (k.arch == 0 && (k.type_vocab < 1 || k.type_vocab > 4)) ||
@@ -1533,7 +2044,7 @@ mimose_status mimose_init(const mimose_config* cfgp, mimose_ctx** out) {
   c->nshard = c->zero1 ? c->npad / k.world : c->npad;
   c->cfg.ffn_layers = nullptr;   // copied into ffn_l; the caller's array need not outlive init
   {  // gradient buckets by event index: layer l -> l, head -> L, embedding -> L + 1
-    const int L = k.n_layers, lb = k.arch == 1 ? 2 : P_LAYER0;
+    const int L = k.n_layers, lb = k.arch != 0 ? 2 : P_LAYER0;
     c->bk_b0.assign(L + 2, 0);
     c->bk_b1.assign(L + 2, 0);
     c->bk_sh.assign(L + 2, 0);
@@ -1582,6 +2093,8 @@ mimose_status mimose_init(const mimose_config* cfgp, mimose_ctx** out) {
   c->tt = (int32_t*)take(maxT * 4);
   c->lens = (int32_t*)take((int64_t)k.max_seqs * 4);
   c->labels = (int32_t*)take(2LL * k.max_seqs * 4);
+  // encoder-decoder: source ids / lengths in ids / lens, decoder ids / lengths in tt / labels
+  c->ids_src = c->ids; c->ids_tgt = c->tt; c->lens_src = c->lens; c->lens_tgt = c->labels;
   c->misc = (float*)take(256);
   c->ws = (float*)take(c->ws_elems * 4);
   c->part = (float*)take((int64_t)NPART * 2 * std::max<int64_t>(3LL * k.hidden, (int64_t)k.ffn) * 4);
@@ -1758,7 +2271,8 @@ static mimose_status begin_step(mimose_ctx* c, const mimose_batch* bt, uint64_t 
   // whole-step accounting first: abandon before any launch on a breach
   int64_t peak;
   bool breach;
-  dry_step(c, bt->n_seqs, bt->seq_len, mask, collect, &peak, &breach, nullptr);
+  const int St = c->cfg.arch == 2 ? bt->dec_len : 0;
+  dry_step(c, bt->n_seqs, bt->seq_len, mask, collect, &peak, &breach, nullptr, St);
   if (breach) {
     c->stats.violations++;
     return fail(c, MIMOSE_E_BUDGET, "step would exceed the budget (predicted " + std::to_string(peak) +
@@ -1769,6 +2283,7 @@ static mimose_status begin_step(mimose_ctx* c, const mimose_batch* bt, uint64_t 
       return s;
   }
   c->B = bt->n_seqs; c->S = bt->seq_len; c->T = c->B * c->S;
+  c->Ss = bt->seq_len; c->St = St;
   c->drop_mask = collect ? ~0ull : mask;
   c->ar.reset_step();
   c->it++;
@@ -1789,7 +2304,9 @@ mimose_status mimose_collect(mimose_ctx* c, const mimose_batch* bt, float* loss_
   if (c->step_pending) return fail(c, MIMOSE_E_STATE, "fused optimizer: mimose_step must close the previous step");
   resolve_times(c);
   const int64_t x = bt ? (int64_t)bt->n_seqs * bt->seq_len : 0;
-  const bool unseen = std::find(c->seen_x.begin(), c->seen_x.end(), x) == c->seen_x.end();
+  const int64_t xt = bt && c->cfg.arch == 2 ? (int64_t)bt->n_seqs * bt->dec_len : 0;
+  const int64_t key = (x << 32) | xt;           // 2-D key of an encoder-decoder (xt = 0 otherwise)
+  const bool unseen = std::find(c->seen_x.begin(), c->seen_x.end(), key) == c->seen_x.end();
   auto t0 = std::chrono::steady_clock::now();
   c->collecting = unseen;
   Sample smp;
@@ -1799,9 +2316,10 @@ mimose_status mimose_collect(mimose_ctx* c, const mimose_batch* bt, float* loss_
   if (s) return s;
   if (unseen) {
     smp.x = x;
+    smp.xt = xt;
     smp.C = c->ar.C;
     c->samples.push_back(smp);     // Th/Tb/Te filled by backward
-    c->seen_x.push_back(x);
+    c->seen_x.push_back(key);
     c->pending_times = c->device;
     c->stats.shuttled_steps++;
   }
@@ -1840,15 +2358,17 @@ mimose_status mimose_backward(mimose_ctx* c) {
   }
   if (c->phase == MIMOSE_PHASE_SHELTERED) {
     std::vector<int64_t> xs;
-    for (auto& s : c->samples) xs.push_back(s.x);
+    for (auto& s : c->samples) xs.push_back((s.x << 32) | s.xt);
     std::sort(xs.begin(), xs.end());
     const int distinct = (int)(std::unique(xs.begin(), xs.end()) - xs.begin());
     const int64_t n = c->stats.collect_steps;
-    if (!c->samples.empty() && ((n >= c->cfg.collect_iters && distinct >= 3) || n >= 30)) {
+    const int need = c->cfg.arch == 2 ? 6 : 3;     // distinct keys for a quadratic (2-D: 6 coefficients)
+    if (!c->samples.empty() && ((n >= c->cfg.collect_iters && distinct >= need) || n >= 30)) {
       resolve_times(c);
       if (mimose_status s2 = agree_times(c)) return s2;
       auto t0 = std::chrono::steady_clock::now();
-      c->est.fit(c->samples, c->cfg.degree);
+      if (c->cfg.arch == 2) c->est.fit2(c->samples, c->cfg.degree);
+      else c->est.fit(c->samples, c->cfg.degree);
       c->stats.planner_us_total +=
           std::chrono::duration<double, std::micro>(std::chrono::steady_clock::now() - t0).count();
       c->phase = MIMOSE_PHASE_RESPONSIVE;
@@ -1931,12 +2451,14 @@ mimose_status mimose_set_planner(mimose_ctx* c, int32_t kind) {
   return MIMOSE_OK;
 }
 
-mimose_status mimose_plan(mimose_ctx* c, int64_t x, mimose_plan_t* out) {
+static mimose_status plan_impl(mimose_ctx* c, int64_t x, int64_t xt, mimose_plan_t* out) {
   if (mimose_status s = check_ready(c)) return s;
-  if (!out || x <= 0) return fail(c, MIMOSE_E_INVALID, "bad plan arguments");
+  if (!out || x <= 0 || (c->cfg.arch == 2 && (xt <= 0 || x >= (1LL << 31) || xt >= (1LL << 31))))
+    return fail(c, MIMOSE_E_INVALID, "bad plan arguments");
   if (c->phase != MIMOSE_PHASE_RESPONSIVE) return fail(c, MIMOSE_E_NOT_READY, "estimator not fitted yet");
   c->stats.plan_calls++;
-  auto it = c->cache.find(x);
+  const int64_t key = c->cfg.arch == 2 ? (x << 32) | xt : x;
+  auto it = c->cache.find(key);
   if (it != c->cache.end()) {
     c->stats.plan_cache_hits++;
     *out = it->second;
@@ -1944,11 +2466,13 @@ mimose_status mimose_plan(mimose_ctx* c, int64_t x, mimose_plan_t* out) {
   } else {
     c->stats.plan_cache_misses++;
     auto t0 = std::chrono::steady_clock::now();
-    const Series s = c->est.predict(x);
+    const bool two = c->cfg.arch == 2;
+    const Series s = two ? c->est.predict2(x, xt) : c->est.predict(x);
     const PlanResult pr =
         c->planner == PLANNER_EXACT ? plan_exact(s, c->ar.budget, c->cfg.reserve_bytes)
         : c->planner == PLANNER_EXACT_TIME
-            ? plan_exact_cost(s, c->est.predict_cost(x), c->ar.budget, c->cfg.reserve_bytes)
+            ? plan_exact_cost(s, two ? c->est.predict_cost2(x, xt) : c->est.predict_cost(x), c->ar.budget,
+                              c->cfg.reserve_bytes)
             : plan_greedy(s, c->ar.budget, c->cfg.reserve_bytes, c->cfg.bucket_num, c->cfg.bucket_den);
     c->stats.planner_us_total +=
         std::chrono::duration<double, std::micro>(std::chrono::steady_clock::now() - t0).count();
@@ -1960,7 +2484,7 @@ mimose_status mimose_plan(mimose_ctx* c, int64_t x, mimose_plan_t* out) {
     p.predicted_peak = pr.peak;
     p.budget = c->ar.budget - c->cfg.reserve_bytes;
     p.status = pr.feasible ? MIMOSE_OK : MIMOSE_E_INFEASIBLE;
-    c->cache[x] = p;
+    c->cache[key] = p;
     *out = p;
   }
   c->stats.last_drop_mask = out->drop_mask;
@@ -1968,6 +2492,16 @@ mimose_status mimose_plan(mimose_ctx* c, int64_t x, mimose_plan_t* out) {
   c->stats.last_predicted_peak = out->predicted_peak;
   if (out->status != MIMOSE_OK) return fail(c, MIMOSE_E_INFEASIBLE, "no plan fits the budget");
   return MIMOSE_OK;
+}
+
+mimose_status mimose_plan(mimose_ctx* c, int64_t x, mimose_plan_t* out) {
+  if (c && c->cfg.arch == 2) return fail(c, MIMOSE_E_INVALID, "encoder-decoder: use mimose_plan2 (2-D key)");
+  return plan_impl(c, x, 0, out);
+}
+
+mimose_status mimose_plan2(mimose_ctx* c, int64_t x, int64_t xt, mimose_plan_t* out) {
+  if (c && c->cfg.arch != 2) return fail(c, MIMOSE_E_INVALID, "mimose_plan2 is for encoder-decoder contexts");
+  return plan_impl(c, x, xt, out);
 }
 
 int32_t mimose_tc_available(void) { return tc_available() ? 1 : 0; }
@@ -2107,25 +2641,30 @@ mimose_status mimose_get_sample(const mimose_ctx* c, int32_t i, mimose_sample* o
   const Sample& s = c->samples[i];
   std::memset(out, 0, sizeof(*out));
   out->x = s.x; out->C = s.C; out->E = s.E; out->Hd = s.Hd; out->Th = s.Th; out->Tb = s.Tb; out->Te = s.Te;
+  out->xt = s.xt;
   for (size_t l = 0; l < s.a.size(); ++l) { out->a[l] = s.a[l]; out->y[l] = s.y[l]; out->t_ms[l] = s.t_ms[l]; }
   return MIMOSE_OK;
 }
 
-mimose_status mimose_dry_run(mimose_ctx* c, int32_t n_seqs, int32_t seq_len, uint64_t mask, int64_t* peak) {
+mimose_status mimose_dry_run2(mimose_ctx* c, int32_t n_seqs, int32_t seq_len, int32_t dec_len, uint64_t mask,
+                              int64_t* peak) {
   if (!c || !peak) return MIMOSE_E_INVALID;
-  mimose_batch bt{nullptr, nullptr, nullptr, nullptr, n_seqs, seq_len, 1};
+  mimose_batch bt{nullptr, nullptr, nullptr, nullptr, n_seqs, seq_len, 1, nullptr, nullptr, dec_len, 0};
   if (mimose_status s = check_batch(c, &bt)) return s;
   bool breach;
   const bool enf = c->ar.enforce;
   c->ar.enforce = false;
-  dry_step(c, n_seqs, seq_len, mask, false, peak, &breach, nullptr);
+  dry_step(c, n_seqs, seq_len, mask, false, peak, &breach, nullptr, c->cfg.arch == 2 ? dec_len : 0);
   c->ar.enforce = enf;
   return MIMOSE_OK;
 }
+mimose_status mimose_dry_run(mimose_ctx* c, int32_t n_seqs, int32_t seq_len, uint64_t mask, int64_t* peak) {
+  return mimose_dry_run2(c, n_seqs, seq_len, c && c->cfg.arch == 2 ? seq_len : 0, mask, peak);
+}
 
-mimose_status mimose_dry_collect(mimose_ctx* c, int32_t n_seqs, int32_t seq_len, mimose_sample* out) {
+mimose_status mimose_dry_collect2(mimose_ctx* c, int32_t n_seqs, int32_t seq_len, int32_t dec_len, mimose_sample* out) {
   if (!c || !out) return MIMOSE_E_INVALID;
-  mimose_batch bt{nullptr, nullptr, nullptr, nullptr, n_seqs, seq_len, 1};
+  mimose_batch bt{nullptr, nullptr, nullptr, nullptr, n_seqs, seq_len, 1, nullptr, nullptr, dec_len, 0};
   if (mimose_status s = check_batch(c, &bt)) return s;
   const int L = n_units(c);
   Sample smp;
@@ -2134,13 +2673,17 @@ mimose_status mimose_dry_collect(mimose_ctx* c, int32_t n_seqs, int32_t seq_len,
   bool breach;
   const bool enf = c->ar.enforce;
   c->ar.enforce = false;
-  dry_step(c, n_seqs, seq_len, ~0ull, true, &peak, &breach, &smp);
+  dry_step(c, n_seqs, seq_len, ~0ull, true, &peak, &breach, &smp, c->cfg.arch == 2 ? dec_len : 0);
   c->ar.enforce = enf;
   std::memset(out, 0, sizeof(*out));
   out->x = (int64_t)n_seqs * seq_len; out->C = c->ar.C;
+  out->xt = c->cfg.arch == 2 ? (int64_t)n_seqs * dec_len : 0;
   out->E = smp.E; out->Hd = smp.Hd; out->Th = smp.Th; out->Tb = smp.Tb; out->Te = smp.Te;
   for (int l = 0; l < L; ++l) { out->a[l] = smp.a[l]; out->y[l] = smp.y[l]; }
   return MIMOSE_OK;
+}
+mimose_status mimose_dry_collect(mimose_ctx* c, int32_t n_seqs, int32_t seq_len, mimose_sample* out) {
+  return mimose_dry_collect2(c, n_seqs, seq_len, c && c->cfg.arch == 2 ? seq_len : 0, out);
 }
 
 static Series to_series(const mimose_series* s) {

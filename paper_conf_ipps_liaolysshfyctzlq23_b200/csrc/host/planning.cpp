@@ -57,6 +57,75 @@ double Poly::eval(int64_t x) const {
 
 int64_t Poly::predict(int64_t x) const { return (int64_t)std::nearbyint(eval(x)) + margin; }
 
+static int solve_normal(double (*A)[7], int n, double* coef) {
+  // Gaussian elimination with partial pivoting in a fixed order; returns 0 if a
+  // pivot vanishes relative to the diagonal scale (rank deficient)
+  double scale = 0.0;
+  for (int r = 0; r < n; ++r) scale = std::max(scale, std::fabs(A[r][r]));
+  for (int col = 0; col < n; ++col) {
+    int piv = col;
+    for (int r = col + 1; r < n; ++r)
+      if (std::fabs(A[r][col]) > std::fabs(A[piv][col])) piv = r;
+    if (!(std::fabs(A[piv][col]) > 1e-10 * scale)) return 0;
+    if (piv != col)
+      for (int c = 0; c <= n; ++c) std::swap(A[col][c], A[piv][c]);
+    for (int r = col + 1; r < n; ++r) {
+      const double f = A[r][col] / A[col][col];
+      for (int c = col; c <= n; ++c) A[r][c] -= f * A[col][c];
+    }
+  }
+  for (int r = n - 1; r >= 0; --r) {
+    double v = A[r][n];
+    for (int c = r + 1; c < n; ++c) v -= A[r][c] * coef[c];
+    coef[r] = v / A[r][r];
+  }
+  return 1;
+}
+
+void Poly2::fit(const std::vector<int64_t>& xs, const std::vector<int64_t>& ts, const std::vector<int64_t>& ys,
+                int max_degree) {
+  std::set<std::pair<int64_t, int64_t>> distinct;
+  for (size_t i = 0; i < xs.size(); ++i) distinct.insert({xs[i], ts[i]});
+  x_ref = t_ref = 1.0;
+  for (size_t i = 0; i < xs.size(); ++i) {
+    x_ref = std::max(x_ref, (double)xs[i]);
+    t_ref = std::max(t_ref, (double)ts[i]);
+  }
+  for (degree = std::min(max_degree, 2); degree >= 0; --degree) {
+    nf = degree == 2 ? 6 : degree == 1 ? 3 : 1;
+    if ((int)distinct.size() < nf) continue;
+    double A[6][7] = {{0}};
+    for (size_t i = 0; i < xs.size(); ++i) {
+      const double s = (double)xs[i] / x_ref, t = (double)ts[i] / t_ref;
+      const double f[6] = {1.0, s, t, s * s, s * t, t * t};
+      for (int r = 0; r < nf; ++r) {
+        for (int c = 0; c < nf; ++c) A[r][c] += f[r] * f[c];
+        A[r][nf] += f[r] * (double)ys[i];
+      }
+    }
+    for (int r = 0; r < 6; ++r) coef[r] = 0.0;
+    if (solve_normal(A, nf, coef)) break;
+  }
+  if (degree < 0) {                          // no pairs at all: constant 0
+    degree = 0;
+    nf = 1;
+    coef[0] = 0.0;
+  }
+  margin = 0;
+  for (size_t i = 0; i < xs.size(); ++i)
+    margin = std::max<int64_t>(margin, ys[i] - (int64_t)std::nearbyint(eval(xs[i], ts[i])));
+}
+
+double Poly2::eval(int64_t x, int64_t xt) const {
+  const double s = (double)x / x_ref, t = (double)xt / t_ref;
+  const double f[6] = {1.0, s, t, s * s, s * t, t * t};
+  double acc = 0.0;
+  for (int k = 0; k < nf; ++k) acc += coef[k] * f[k];
+  return acc;
+}
+
+int64_t Poly2::predict(int64_t x, int64_t xt) const { return (int64_t)std::nearbyint(eval(x, xt)) + margin; }
+
 int64_t predicted_peak(const Series& s, uint64_t mask) {
   const int L = (int)s.a.size();
   const int64_t base = s.C + s.E;
@@ -232,6 +301,55 @@ void Estimator::fit(const std::vector<Sample>& smp, int degree) {
   for (int l = 0; l < L; ++l)
     ft[l].fit(xs, series([&](const Sample& s) { return (int64_t)std::llround((double)s.t_ms[l] * 1e6); }), degree);
   fitted = true;
+}
+
+void Estimator::fit2(const std::vector<Sample>& smp, int degree) {
+  const int L = (int)smp.front().a.size();
+  std::vector<int64_t> xs, ts;
+  for (auto& s : smp) { xs.push_back(s.x); ts.push_back(s.xt); }
+  auto series = [&](auto get) {
+    std::vector<int64_t> v;
+    for (auto& s : smp) v.push_back(get(s));
+    return v;
+  };
+  C = smp.front().C;
+  fa2.assign(L, Poly2());
+  fy2.assign(L, Poly2());
+  ft2.assign(L, Poly2());
+  for (int l = 0; l < L; ++l) {
+    fa2[l].fit(xs, ts, series([&](const Sample& s) { return s.a[l]; }), degree);
+    fy2[l].fit(xs, ts, series([&](const Sample& s) { return s.y[l]; }), degree);
+    ft2[l].fit(xs, ts, series([&](const Sample& s) { return (int64_t)std::llround((double)s.t_ms[l] * 1e6); }),
+               degree);
+  }
+  fE2.fit(xs, ts, series([](const Sample& s) { return s.E; }), degree);
+  fHd2.fit(xs, ts, series([](const Sample& s) { return s.Hd; }), degree);
+  fTh2.fit(xs, ts, series([](const Sample& s) { return s.Th; }), degree);
+  fTb2.fit(xs, ts, series([](const Sample& s) { return s.Tb; }), degree);
+  fTe2.fit(xs, ts, series([](const Sample& s) { return s.Te; }), degree);
+  two_d = true;
+  fitted = true;
+}
+
+Series Estimator::predict2(int64_t x, int64_t xt) const {
+  Series s;
+  s.C = C;
+  s.E = fE2.predict(x, xt);
+  s.Hd = fHd2.predict(x, xt);
+  s.Th = fTh2.predict(x, xt);
+  s.Tb = fTb2.predict(x, xt);
+  s.Te = fTe2.predict(x, xt);
+  for (size_t l = 0; l < fa2.size(); ++l) {
+    s.a.push_back(fa2[l].predict(x, xt));
+    s.y.push_back(fy2[l].predict(x, xt));
+  }
+  return s;
+}
+
+std::vector<int64_t> Estimator::predict_cost2(int64_t x, int64_t xt) const {
+  std::vector<int64_t> c(ft2.size());
+  for (size_t l = 0; l < ft2.size(); ++l) c[l] = std::max<int64_t>(1, (int64_t)std::nearbyint(ft2[l].eval(x, xt)));
+  return c;
 }
 
 std::vector<int64_t> Estimator::predict_cost(int64_t x) const {

@@ -21,6 +21,21 @@ struct Poly {
   int64_t predict(int64_t x) const;
 };
 
+// Bivariate least squares for the 2-D key of an encoder-decoder (reading A32):
+// features [1, s, t, s^2, s t, t^2] (degree 2), [1, s, t] (degree 1) or [1],
+// s = x / x_ref, t = xt / t_ref; the highest degree whose design matrix has
+// full rank on the distinct key pairs; normal equations with partial pivoting.
+struct Poly2 {
+  int degree = 0, nf = 1;
+  double x_ref = 1.0, t_ref = 1.0;
+  double coef[6] = {0, 0, 0, 0, 0, 0};
+  int64_t margin = 0;
+  void fit(const std::vector<int64_t>& xs, const std::vector<int64_t>& ts, const std::vector<int64_t>& ys,
+           int max_degree);
+  double eval(int64_t x, int64_t xt) const;
+  int64_t predict(int64_t x, int64_t xt) const;
+};
+
 // Per-series sizes for one input size x (what the planner reasons about).
 struct Series {
   int64_t C = 0, E = 0, Hd = 0, Th = 0, Tb = 0, Te = 0;
@@ -59,7 +74,7 @@ enum PlannerKind : int { PLANNER_GREEDY = 0, PLANNER_EXACT = 1, PLANNER_EXACT_TI
 
 // One collected sheltered-iteration sample (arena deltas).
 struct Sample {
-  int64_t x = 0, C = 0, E = 0, Hd = 0, Th = 0, Tb = 0, Te = 0;
+  int64_t x = 0, xt = 0, C = 0, E = 0, Hd = 0, Th = 0, Tb = 0, Te = 0;
   std::vector<int64_t> a, y;
   std::vector<float> t_ms;
 };
@@ -70,8 +85,15 @@ struct Estimator {
   std::vector<Poly> fa, fy;
   Poly fE, fHd, fTh, fTb, fTe;
   std::vector<Poly> ft;   // per-layer forward time, integer ns (the collector's t_l(x))
+  // encoder-decoder: the same series on the 2-D key (x, xt)
+  bool two_d = false;
+  std::vector<Poly2> fa2, fy2, ft2;
+  Poly2 fE2, fHd2, fTh2, fTb2, fTe2;
   void fit(const std::vector<Sample>& samples, int degree);
+  void fit2(const std::vector<Sample>& samples, int degree);
   Series predict(int64_t x) const;
+  Series predict2(int64_t x, int64_t xt) const;
+  std::vector<int64_t> predict_cost2(int64_t x, int64_t xt) const;
   // Recompute cost per layer at x: the fitted forward time in ns, at least 1.
   std::vector<int64_t> predict_cost(int64_t x) const;
 };

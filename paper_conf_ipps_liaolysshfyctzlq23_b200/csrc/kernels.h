@@ -75,6 +75,14 @@ void attn_bwd(DType dt, const void* qkv, const void* O, const void* dO, const fl
               const int32_t* lengths, float* Dbuf, void* dqkv, int B, int S, int H, int h,
               Drop drop, cudaStream_t st, bool causal = false);
 
+// Cross-attention (encoder-decoder): q [B*Sq, H], kv [B*Sk, 2H] (k | v); key
+// padding by klens; tcgen05, Sq, Sk <= 128, head dim 64 (false: not launched).
+bool attn_cross_fwd_tc(const void* q, const void* kv, const int32_t* qlens, const int32_t* klens, void* O, float* lse,
+                       int B, int Sq, int Sk, int H, int h, Drop drop, cudaStream_t st);
+bool attn_cross_bwd_tc(const void* q, const void* kv, const void* O, const void* dO, const float* lse,
+                       const int32_t* qlens, const int32_t* klens, void* dq, void* dkv, int B, int Sq, int Sk, int H,
+                       int h, Drop drop, cudaStream_t st);
+
 // ----------------------------------------------------------- layernorm ----
 // y = LN(z) (y may be null: recompute with the output store gated off); st = (mu, rstd).
 // z (pre-LN sum) is fp32 in every mode.
@@ -115,7 +123,8 @@ void drop_f32(const float* dy, Drop mask, float* out, int64_t n, cudaStream_t st
 // dWt[k] = sum over tokens with token_type k of dz0 rows (fixed-order partials)
 void type_grad(const float* dz0, const int32_t* tt, int T, int H, int TV, float* part, float* dWt, cudaStream_t st);
 // dWp[pos_offset + s] = sum_b dz0[b*S + s]
-void pos_grad(const float* dz0, int B, int S, int H, int pos_offset, float* dWp, cudaStream_t st);
+void pos_grad(const float* dz0, int B, int S, int H, int pos_offset, float* dWp, cudaStream_t st,
+              bool accumulate = false);
 
 // ---------------------------------------------------------------- heads ----
 // seq-cls / MC: pooled p [B,H] (E), logits [B,n_out] f32, loss -> misc[0]

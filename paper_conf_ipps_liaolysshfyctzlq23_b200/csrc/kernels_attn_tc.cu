@@ -29,7 +29,14 @@ constexpr int TILE = AQ * AD * 2;        // 16 KB: one [128 x 64] bf16 SW128 til
 constexpr int PT = AQ * AQ * 2;          // 32 KB: one [128 x 128] bf16 tile (2 atoms)
 
 struct AttnArgs {
-  int S, H, h, B;
+  int S, H, h, B;              // S: query rows per sequence
+  int Sk;                      // key rows per sequence (== S for self-attention)
+  int qcol, kcol, vcol;        // column bases of Q (in tq), K and V (in tk): 0, H, 2H for a [T, 3H] qkv
+  int ldo, ocq, ock, ocv;      // backward: dQ row stride, column bases of dQ / dK / dV
+  int ldk;                     // backward: dK / dV row stride (0: ldo)
+  const int32_t* klens;        // key lengths (key padding mask); lengths = query lengths
+  __nv_bfloat16* dq;           // backward: dQ rows (b*S + t); dqkv for self-attention
+  __nv_bfloat16* dkv;          // backward: dK / dV rows (b*Sk + t)
   int causal;                  // GPT-2: key k visible to query q iff k <= q
   float scale;
   Drop drop;
@@ -38,7 +45,6 @@ struct AttnArgs {
   __nv_bfloat16* Oout;
   float* lse;
   const float* lse_in;
-  __nv_bfloat16* dqkv;
   const __nv_bfloat16* dO;
 };
 
@@ -81,7 +87,8 @@ MDEV float ex2f(float x) {
 // Softmax: pass 1 takes the row max, pass 2 writes the unnormalised
 // P~ = exp(s - max) * dropout (bf16) and the row sum l; O = (P~ V) / l in the
 // epilogue, LSE = max + log l (what the backward recomputes P from).
-__global__ void __launch_bounds__(ATT, 3) k_attn_fwd_tc(const __grid_constant__ CUtensorMap tq, const AttnArgs a) {
+__global__ void __launch_bounds__(ATT, 3) k_attn_fwd_tc(const __grid_constant__ CUtensorMap tq,
+                                                     const __grid_constant__ CUtensorMap tk, const AttnArgs a) {
   pdl_enter();
   extern __shared__ __align__(1024) uint8_t sm[];
   uint8_t* sQ = sm;
@@ -94,8 +101,8 @@ __global__ void __launch_bounds__(ATT, 3) k_attn_fwd_tc(const __grid_constant__ 
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const int hf = warp >> 2, t = 32 * (warp & 3) + lane;
   const int bh = blockIdx.x, b = bh / a.h, hd = bh % a.h;
-  const int S = a.S, len = a.lengths[b];
-  const int kmax = (S + 31) & ~31, nch = kmax >> 5, cmid = (nch + 1) >> 1;
+  const int S = a.S, Sk = a.Sk, len = a.klens[b];
+  const int kmax = (Sk + 31) & ~31, nch = kmax >> 5, cmid = (nch + 1) >> 1;
   const int c0 = hf ? cmid : 0, c1 = hf ? nch : cmid;
   if (threadIdx.x == 0) {
     for (int i = 0; i < 3; ++i) mbar_init(&bar[i], 1);
@@ -109,12 +116,12 @@ __global__ void __launch_bounds__(ATT, 3) k_attn_fwd_tc(const __grid_constant__ 
   __syncthreads();
   tc_fence_after();
   const uint32_t tmem = *tslot;
-  const int row0 = b * S;
+  const int row0 = b * S, krow0 = b * Sk;
   if (threadIdx.x == 0) {
     mbar_expect_tx(&bar[0], 3 * TILE);
-    tma_load_2d(&tq, &bar[0], sQ, hd * AD, row0);
-    tma_load_2d(&tq, &bar[0], sK, a.H + hd * AD, row0);
-    tma_load_2d(&tq, &bar[0], sV, 2 * a.H + hd * AD, row0);
+    tma_load_2d(&tq, &bar[0], sQ, a.qcol + hd * AD, row0);
+    tma_load_2d(&tk, &bar[0], sK, a.kcol + hd * AD, krow0);
+    tma_load_2d(&tk, &bar[0], sV, a.vcol + hd * AD, krow0);
     mbar_wait(&bar[0], 0);
     tc_fence_after();
     const uint32_t id = idesc_bf16(AQ, kmax, 0, 0);
@@ -144,7 +151,7 @@ __global__ void __launch_bounds__(ATT, 3) k_attn_fwd_tc(const __grid_constant__ 
   __syncthreads();
   const float sl2 = a.scale * 1.4426950408889634f;               // scale * log2(e)
   const float mrow = fmaxf(red[t], red[128 + t]) * sl2;          // row max of s * scale * log2(e)
-  const uint64_t ebase = (((uint64_t)b * a.h + hd) * S + (uint64_t)t) * S;
+  const uint64_t ebase = (((uint64_t)b * a.h + hd) * S + (uint64_t)t) * Sk;
   // The S MMA has completed (bar[1]), so Q and K are dead: each thread writes its
   // P~ row straight into their space.
   float l = 0.f;
@@ -213,6 +220,7 @@ __global__ void __launch_bounds__(ATT, 3) k_attn_fwd_tc(const __grid_constant__ 
 }
 
 __global__ void __launch_bounds__(ATT, 2) k_attn_bwd_tc(const __grid_constant__ CUtensorMap tq,
+                                                     const __grid_constant__ CUtensorMap tk,
                                                      const __grid_constant__ CUtensorMap tdo, const AttnArgs a) {
   pdl_enter();
   extern __shared__ __align__(1024) uint8_t sm[];
@@ -228,8 +236,9 @@ __global__ void __launch_bounds__(ATT, 2) k_attn_bwd_tc(const __grid_constant__ 
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const int hf = warp >> 2, t = 32 * (warp & 3) + lane;
   const int bh = blockIdx.x, b = bh / a.h, hd = bh % a.h;
-  const int S = a.S, len = a.lengths[b];
-  const int kmax = (S + 31) & ~31, nch = kmax >> 5, cmid = (nch + 1) >> 1;
+  const int S = a.S, Sk = a.Sk, len = a.lengths[b], klen = a.klens[b];
+  const int kmax = (Sk + 31) & ~31, nch = kmax >> 5, cmid = (nch + 1) >> 1;
+  const int qmax = (S + 31) & ~31;                 // contraction range of dV, dK (query rows)
   const int c0 = hf ? cmid : 0, c1 = hf ? nch : cmid;
   if (threadIdx.x == 0) {
     for (int i = 0; i < 3; ++i) mbar_init(&bar[i], 1);
@@ -243,12 +252,12 @@ __global__ void __launch_bounds__(ATT, 2) k_attn_bwd_tc(const __grid_constant__ 
   __syncthreads();
   tc_fence_after();
   const uint32_t tmem = *tslot;
-  const int row0 = b * S;
+  const int row0 = b * S, krow0 = b * Sk;
   if (threadIdx.x == 0) {
     mbar_expect_tx(&bar[0], 4 * TILE);
-    tma_load_2d(&tq, &bar[0], sQ, hd * AD, row0);
-    tma_load_2d(&tq, &bar[0], sK, a.H + hd * AD, row0);
-    tma_load_2d(&tq, &bar[0], sV, 2 * a.H + hd * AD, row0);
+    tma_load_2d(&tq, &bar[0], sQ, a.qcol + hd * AD, row0);
+    tma_load_2d(&tk, &bar[0], sK, a.kcol + hd * AD, krow0);
+    tma_load_2d(&tk, &bar[0], sV, a.vcol + hd * AD, krow0);
     tma_load_2d(&tdo, &bar[0], sdO, hd * AD, row0);
     mbar_wait(&bar[0], 0);
     tc_fence_after();
@@ -262,29 +271,54 @@ __global__ void __launch_bounds__(ATT, 2) k_attn_bwd_tc(const __grid_constant__ 
       mma_bf16(tmem + 128, make_desc(o0 + 32 * kk, 16, 1024), make_desc(v0 + 32 * kk, 16, 1024), id, kk > 0);
     mma_commit(&bar[1]);
   }
-  // D_t = rowsum(dO * O) for query row t: half hf sums dims [32hf, 32hf+32)
-  // (global reads overlap the MMAs); D = half 0 + half 1
-  float Dh = 0.f, Lt = 0.f;
-  if (t < len) {
-    const __nv_bfloat16* orow = a.O + ((int64_t)row0 + t) * a.H + hd * AD + 32 * hf;
-    const __nv_bfloat16* drow = a.dO + ((int64_t)row0 + t) * a.H + hd * AD + 32 * hf;
-    float ov[32], dv[32];
-    ld_bf16x32(orow, ov);
-    ld_bf16x32(drow, dv);
+  // D_t = sum_k P~_tk dP~_tk over this row's keys, in fp32 from the same P~ and
+  // dP~ = dO V^T that dS uses (exactly rowsum(dO * O) in exact arithmetic, but
+  // consistent with dP~ under bf16 storage of O, so dS sums to ~0 per row:
+  // near-uniform attention rows -- e.g. cross-attention -- keep their relative
+  // accuracy).  Pass 1 over the TMEM row: P~, the dropout keep bits (kept in two
+  // registers for pass 2), the D partial of this key half; D = half 0 + half 1.
+  float Lt = 0.f;
+  if (t < len) Lt = a.lse_in[((int64_t)b * a.h + hd) * S + t];
+  mbar_wait(&bar[1], 0);
+  __syncwarp();
+  tc_fence_after();
+  const uint32_t trow = tmem + ((uint32_t)(32 * (warp & 3)) << 16);
+  const uint64_t ebase = (((uint64_t)b * a.h + hd) * S + (uint64_t)t) * Sk;
+  const int kl = a.causal ? min(klen, t + 1) : klen;
+  const float sl2 = a.scale * 1.4426950408889634f, Ll2 = Lt * 1.4426950408889634f;
+  const float keepf = a.drop.enabled ? a.drop.scale : 1.0f;
+  uint32_t kb0 = 0u, kb1 = 0u;             // keep bits of chunks c0 (kb0) and c0 + 1 (kb1) of this half
+  float Dh = 0.f;
+  for (int c = c0; c < c1; ++c)
 #pragma unroll
-    for (int i = 0; i < 32; ++i) Dh += ov[i] * dv[i];
-    Lt = a.lse_in[((int64_t)b * a.h + hd) * S + t];
+  for (int hh = 0; hh < 2; ++hh) {
+    float sv[16], dp[16];
+    tmem_ld16(trow + 32 * c + 16 * hh, sv);
+    tmem_ld16(trow + 128 + 32 * c + 16 * hh, dp);
+    const int kb = 32 * c + 16 * hh;
+    if (t < len && kb < kl) {
+#pragma unroll
+      for (int j = 0; j < 4; ++j) {
+        const int k = kb + 4 * j;
+        const float4 f = (k < kl) ? drop4_or(a.drop, ebase + k) : make_float4(0.f, 0.f, 0.f, 0.f);
+        const float ff[4] = {f.x, f.y, f.z, f.w};
+#pragma unroll
+        for (int i = 0; i < 4; ++i) {
+          const int kk = k + i;
+          const float p = (kk < kl) ? ex2f(fmaf(sv[4 * j + i], sl2, -Ll2)) : 0.f;
+          Dh = fmaf(p * ff[i], dp[4 * j + i], Dh);
+          if (ff[i] != 0.f) {
+            if (c == c0) kb0 |= 1u << (16 * hh + 4 * j + i);
+            else kb1 |= 1u << (16 * hh + 4 * j + i);
+          }
+        }
+      }
+    }
   }
   red[hf * 128 + t] = Dh;
-  mbar_wait(&bar[1], 0);
   __syncthreads();                        // red[] complete; every thread is past the MMAs (V dead)
-  tc_fence_after();
   const float Dt = red[t] + red[128 + t];
   __syncthreads();                        // every D read before dS overwrites red[]
-  const uint32_t trow = tmem + ((uint32_t)(32 * (warp & 3)) << 16);
-  const uint64_t ebase = (((uint64_t)b * a.h + hd) * S + (uint64_t)t) * S;
-  const int kl = a.causal ? min(len, t + 1) : len;
-  const float sl2 = a.scale * 1.4426950408889634f, Ll2 = Lt * 1.4426950408889634f;
   for (int c = c0; c < c1; ++c)
 #pragma unroll
   for (int hh = 0; hh < 2; ++hh) {
@@ -295,17 +329,12 @@ __global__ void __launch_bounds__(ATT, 2) k_attn_bwd_tc(const __grid_constant__ 
     const bool live = t < len && kb < kl;        // padded / foreign query rows contribute 0
     if (live) {
 #pragma unroll
-      for (int j = 0; j < 4; ++j) {
-        const int k = kb + 4 * j;
-        const float4 f = (k < kl) ? drop4_or(a.drop, ebase + k) : make_float4(0.f, 0.f, 0.f, 0.f);
-        const float ff[4] = {f.x, f.y, f.z, f.w};
-#pragma unroll
-        for (int i = 0; i < 4; ++i) {
-          const int kk = k + i;
-          const float p = (kk < kl) ? ex2f(fmaf(sv[4 * j + i], sl2, -Ll2)) : 0.f;
-          sv[4 * j + i] = p * ff[i];                                  // P~
-          dp[4 * j + i] = p * (dp[4 * j + i] * ff[i] - Dt) * a.scale; // dS (scale folded)
-        }
+      for (int q = 0; q < 16; ++q) {
+        const int kk = kb + q;
+        const float p = (kk < kl) ? ex2f(fmaf(sv[q], sl2, -Ll2)) : 0.f;
+        const float fq = (((c == c0 ? kb0 : kb1) >> (16 * hh + q)) & 1u) ? keepf : 0.f;
+        sv[q] = p * fq;                                            // P~
+        dp[q] = p * (dp[q] * fq - Dt) * a.scale;                   // dS (scale folded)
       }
     } else {
 #pragma unroll
@@ -323,32 +352,37 @@ __global__ void __launch_bounds__(ATT, 2) k_attn_bwd_tc(const __grid_constant__ 
     const uint32_t id_q = idesc_bf16(AQ, AD, 0, 1);   // A K-major (queries), B MN-major (d)
     const uint32_t p0 = smem_u32(sP), s0 = smem_u32(sdS);
     const uint32_t q0 = smem_u32(sQ), k0 = smem_u32(sK), o0 = smem_u32(sdO);
-    for (int kk = 0; kk < kmax / 16; ++kk) {    // contraction over queries (dV, dK) / keys (dQ)
-      const uint64_t at_p = make_desc(p0 + 2048 * kk, 16384, 1024);
-      const uint64_t at_s = make_desc(s0 + 2048 * kk, 16384, 1024);
-      const uint64_t bq_do = make_desc(o0 + 2048 * kk, 16384, 1024);
-      const uint64_t bq_q = make_desc(q0 + 2048 * kk, 16384, 1024);
-      mma_bf16(tmem + 0, at_p, bq_do, id_t, kk > 0);          // dV = P~^T dO
-      mma_bf16(tmem + 64, at_s, bq_q, id_t, kk > 0);          // dK = dS^T Q
-      const uint64_t ak_s = make_desc(s0 + (kk >> 2) * (AQ * 128) + 32 * (kk & 3), 16, 1024);
-      const uint64_t bk_k = make_desc(k0 + 2048 * kk, 16384, 1024);
-      mma_bf16(tmem + 128, ak_s, bk_k, id_q, kk > 0);         // dQ = dS K
+    for (int kk = 0; kk < max(kmax, qmax) / 16; ++kk) {   // contraction over queries (dV, dK) / keys (dQ)
+      if (kk < qmax / 16) {
+        const uint64_t at_p = make_desc(p0 + 2048 * kk, 16384, 1024);
+        const uint64_t at_s = make_desc(s0 + 2048 * kk, 16384, 1024);
+        const uint64_t bq_do = make_desc(o0 + 2048 * kk, 16384, 1024);
+        const uint64_t bq_q = make_desc(q0 + 2048 * kk, 16384, 1024);
+        mma_bf16(tmem + 0, at_p, bq_do, id_t, kk > 0);        // dV = P~^T dO
+        mma_bf16(tmem + 64, at_s, bq_q, id_t, kk > 0);        // dK = dS^T Q
+      }
+      if (kk < kmax / 16) {
+        const uint64_t ak_s = make_desc(s0 + (kk >> 2) * (AQ * 128) + 32 * (kk & 3), 16, 1024);
+        const uint64_t bk_k = make_desc(k0 + 2048 * kk, 16384, 1024);
+        mma_bf16(tmem + 128, ak_s, bk_k, id_q, kk > 0);       // dQ = dS K
+      }
     }
     mma_commit(&bar[2]);
   }
   mbar_wait(&bar[2], 0);
   __syncwarp();
   tc_fence_after();
-  {  // every lane loads (.sync.aligned); rows t < S store; half hf stores dims [32hf, 32hf+32)
-    __nv_bfloat16* row = a.dqkv + ((int64_t)row0 + t) * 3 * a.H + hd * AD + 32 * hf;
-    const bool st = t < S;
+  {  // every lane loads (.sync.aligned); query rows t < S store dQ, key rows t < Sk store dK, dV;
+     // half hf stores dims [32hf, 32hf+32)
+    __nv_bfloat16* qrow = a.dq + ((int64_t)row0 + t) * a.ldo + a.ocq + hd * AD + 32 * hf;
+    __nv_bfloat16* krow = a.dkv + ((int64_t)krow0 + t) * (a.ldk ? a.ldk : a.ldo) + hd * AD + 32 * hf;
     float v[32];
     tmem_ld32(trow + 128 + 32 * hf, v);
-    if (st) st_bf16x32(row, v);                              // dQ
+    if (t < S) st_bf16x32(qrow, v);                          // dQ
     tmem_ld32(trow + 64 + 32 * hf, v);
-    if (st) st_bf16x32(row + a.H, v);                        // dK
+    if (t < Sk) st_bf16x32(krow + a.ock, v);                 // dK
     tmem_ld32(trow + 32 * hf, v);
-    if (st) st_bf16x32(row + 2 * a.H, v);                    // dV
+    if (t < Sk) st_bf16x32(krow + a.ocv, v);                 // dV
   }
   tc_fence_before();
   __syncthreads();
@@ -375,10 +409,11 @@ bool attn_fwd_tc(const void* qkv, const int32_t* lengths, void* O, float* lse, i
   static std::once_flag once;
   std::call_once(once, [] { cudaFuncSetAttribute(k_attn_fwd_tc, cudaFuncAttributeMaxDynamicSharedMemorySize, FWD_SMEM); });
   AttnArgs a{};
-  a.S = S; a.H = H; a.h = h; a.B = B;
+  a.S = S; a.Sk = S; a.H = H; a.h = h; a.B = B;
+  a.qcol = 0; a.kcol = H; a.vcol = 2 * H;
   a.scale = 1.0f / sqrtf((float)AD);
-  a.drop = drop; a.lengths = lengths; a.Oout = (__nv_bfloat16*)O; a.lse = lse; a.causal = causal;
-  launch_k(k_attn_fwd_tc, B * h, ATT, FWD_SMEM, st, tq, a);
+  a.drop = drop; a.lengths = lengths; a.klens = lengths; a.Oout = (__nv_bfloat16*)O; a.lse = lse; a.causal = causal;
+  launch_k(k_attn_fwd_tc, B * h, ATT, FWD_SMEM, st, tq, tq, a);
   return true;
 }
 
@@ -391,11 +426,60 @@ bool attn_bwd_tc(const void* qkv, const void* O, const void* dO, const float* ls
   static std::once_flag once;
   std::call_once(once, [] { cudaFuncSetAttribute(k_attn_bwd_tc, cudaFuncAttributeMaxDynamicSharedMemorySize, BWD_SMEM); });
   AttnArgs a{};
-  a.S = S; a.H = H; a.h = h; a.B = B;
+  a.S = S; a.Sk = S; a.H = H; a.h = h; a.B = B;
+  a.qcol = 0; a.kcol = H; a.vcol = 2 * H;
+  a.ldo = 3 * H; a.ocq = 0; a.ock = H; a.ocv = 2 * H;
   a.scale = 1.0f / sqrtf((float)AD);
-  a.drop = drop; a.lengths = lengths; a.O = (const __nv_bfloat16*)O; a.dO = (const __nv_bfloat16*)dO;
-  a.lse_in = lse; a.dqkv = (__nv_bfloat16*)dqkv; a.causal = causal;
-  launch_k(k_attn_bwd_tc, B * h, ATT, BWD_SMEM, st, tq, tdo, a);
+  a.drop = drop; a.lengths = lengths; a.klens = lengths; a.O = (const __nv_bfloat16*)O; a.dO = (const __nv_bfloat16*)dO;
+  a.lse_in = lse; a.dq = (__nv_bfloat16*)dqkv; a.dkv = (__nv_bfloat16*)dqkv; a.causal = causal;
+  launch_k(k_attn_bwd_tc, B * h, ATT, BWD_SMEM, st, tq, tq, tdo, a);
+  return true;
+}
+
+// Cross-attention (encoder-decoder): queries q [B*Sq, H], keys and
+// values kv [B*Sk, 2H] (k | v), key padding by klens, no causal mask; both
+// lengths <= 128.  Dropout element ((b*h + head)*Sq + q)*Sk + k.
+bool attn_cross_ok(int Sq, int Sk, int H, int h) { return Sq <= AQ && Sk <= AQ && H / h == AD && H % 64 == 0; }
+
+bool attn_cross_fwd_tc(const void* q, const void* kv, const int32_t* qlens, const int32_t* klens, void* O, float* lse,
+                       int B, int Sq, int Sk, int H, int h, Drop drop, cudaStream_t st) {
+  if (!attn_cross_ok(Sq, Sk, H, h)) return false;
+  CUtensorMap tq, tk;
+  if (!tc_map_bf16(&tq, q, (uint64_t)H, (uint64_t)B * Sq, (uint64_t)H, 64, AQ)) return false;
+  if (!tc_map_bf16(&tk, kv, 2ull * H, (uint64_t)B * Sk, 2ull * H, 64, AQ)) return false;
+  static std::once_flag once;
+  std::call_once(once, [] { cudaFuncSetAttribute(k_attn_fwd_tc, cudaFuncAttributeMaxDynamicSharedMemorySize, FWD_SMEM); });
+  AttnArgs a{};
+  a.S = Sq; a.Sk = Sk; a.H = H; a.h = h; a.B = B;
+  a.qcol = 0; a.kcol = 0; a.vcol = H;
+  a.scale = 1.0f / sqrtf((float)AD);
+  a.drop = drop; a.lengths = qlens; a.klens = klens; a.Oout = (__nv_bfloat16*)O; a.lse = lse; a.causal = 0;
+  launch_k(k_attn_fwd_tc, B * h, ATT, FWD_SMEM, st, tq, tk, a);
+  return true;
+}
+
+bool attn_cross_bwd_tc(const void* q, const void* kv, const void* O, const void* dO, const float* lse,
+                       const int32_t* qlens, const int32_t* klens, void* dq, void* dkv, int B, int Sq, int Sk, int H,
+                       int h, Drop drop, cudaStream_t st) {
+  if (!attn_cross_ok(Sq, Sk, H, h)) return false;
+  CUtensorMap tq, tk, tdo;
+  if (!tc_map_bf16(&tq, q, (uint64_t)H, (uint64_t)B * Sq, (uint64_t)H, 64, AQ)) return false;
+  if (!tc_map_bf16(&tk, kv, 2ull * H, (uint64_t)B * Sk, 2ull * H, 64, AQ)) return false;
+  if (!tc_map_bf16(&tdo, dO, (uint64_t)H, (uint64_t)B * Sq, (uint64_t)H, 64, AQ)) return false;
+  static std::once_flag once;
+  std::call_once(once, [] { cudaFuncSetAttribute(k_attn_bwd_tc, cudaFuncAttributeMaxDynamicSharedMemorySize, BWD_SMEM); });
+  AttnArgs a{};
+  a.S = Sq; a.Sk = Sk; a.H = H; a.h = h; a.B = B;
+  a.qcol = 0; a.kcol = 0; a.vcol = H;
+  a.scale = 1.0f / sqrtf((float)AD);
+  a.drop = drop; a.lengths = qlens; a.klens = klens; a.O = (const __nv_bfloat16*)O; a.dO = (const __nv_bfloat16*)dO;
+  a.lse_in = lse; a.causal = 0;
+  // dQ [B*Sq, H] and dKV [B*Sk, 2H] have different row strides: two output
+  // pointers, one stride each (ldo for dQ rows, 2H for dK / dV rows)
+  a.dq = (__nv_bfloat16*)dq; a.dkv = (__nv_bfloat16*)dkv;
+  a.ldo = H; a.ocq = 0; a.ock = 0; a.ocv = H;
+  a.ldk = 2 * H;
+  launch_k(k_attn_bwd_tc, B * h, ATT, BWD_SMEM, st, tq, tk, tdo, a);
   return true;
 }
 

@@ -530,18 +530,19 @@ void embed_fwd_pre(DType dt, const int32_t* ids, const void* Ww, const void* Wp,
 }
 
 __global__ void k_pos_grad(const float* __restrict__ dz0, int B, int S, int H, int pos_offset,
-                           float* __restrict__ dWp) {
+                           float* __restrict__ dWp, int accumulate) {
   pdl_enter();
   const int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
   if (i >= (int64_t)S * H) return;
   const int s = (int)(i / H), c = (int)(i % H);
   float acc = 0.f;
   for (int b = 0; b < B; ++b) acc += dz0[((int64_t)b * S + s) * H + c];
-  dWp[(int64_t)(pos_offset + s) * H + c] = acc;
+  float* o = dWp + (int64_t)(pos_offset + s) * H + c;
+  *o = accumulate ? *o + acc : acc;
 }
-void pos_grad(const float* dz0, int B, int S, int H, int pos_offset, float* dWp, cudaStream_t s) {
+void pos_grad(const float* dz0, int B, int S, int H, int pos_offset, float* dWp, cudaStream_t s, bool accumulate) {
   note_launch(1);
-  launch_k(k_pos_grad, cdiv((int64_t)S * H, 256), 256, 0, s, dz0, B, S, H, pos_offset, dWp);
+  launch_k(k_pos_grad, cdiv((int64_t)S * H, 256), 256, 0, s, dz0, B, S, H, pos_offset, dWp, accumulate ? 1 : 0);
 }
 
 // ---- stable LSD radix sort of (key, token) pairs, 8-bit digits, 1024-key tiles ----

@@ -158,3 +158,64 @@ def test_budget_property_over_a_2d_schedule():
     tight = om.simulate_step_encdec(szmax, range(24)).peak - 1
     st, _, _ = op.plan(est.predict(CFG.n_seqs * CFG.max_seq, CFG.n_seqs * CFG.max_seq), tight)
     assert st == op.INFEASIBLE
+
+
+# ---------------------------------------------------------------- library --
+
+def test_library_accounting_matches_oracle():
+    from paper_conf_ipps_liaolysshfyctzlq23_b200 import binding as mb
+    ctx = mb.Mimose(CFG, budget(CFG))
+    assert ctx.n_params == wl.n_params(CFG) and ctx.n_units == 24
+    assert ctx.stats()["persistent_bytes"] == om.persistent_bytes(CFG, CFG.n_seqs, CFG.max_seq)
+    rng = random.Random(8)
+    for Ss, St in [(24, 24), (64, 72), (128, 104), (40, 128), (128, 16)]:
+        sz = om.sizes_encdec(CFG, CFG.n_seqs, Ss, St)
+        for _ in range(10):
+            plan = rng.sample(range(24), rng.randint(0, 24))
+            assert ctx.dry_run(CFG.n_seqs, Ss, plan, dec_len=St) == om.simulate_step_encdec(sz, plan).peak
+        got, want = ctx.dry_collect(CFG.n_seqs, Ss, dec_len=St), om.collect_samples_encdec(sz)
+        assert got["xt"] == CFG.n_seqs * St
+        for k in ("C", "E", "Hd", "Th", "Tb", "Te", "a", "y"):
+            assert got[k] == want[k], k
+
+
+def test_library_pipeline_matches_oracle():
+    """Sheltered phase on 2-D keys -> bivariate fit -> mimose_plan2 (Algorithm
+    1): every plan equals the oracle planner on the oracle's Estimator2D, within
+    the budget.  (The exact planners' oracle is brute force: 3 + 3 layers above.)"""
+    from paper_conf_ipps_liaolysshfyctzlq23_b200 import binding as mb
+    M = budget(CFG)
+    ctx = mb.Mimose(CFG, M)
+    rng = np.random.default_rng(21)
+    samples, seen = [], set()
+    i = 0
+    while ctx.phase == mb.PHASE_SHELTERED:
+        b = wl.make_batch(CFG, int(rng.integers(CFG.seq_lo, CFG.seq_hi + 1)), seed=i)
+        ctx.collect(ctx.host_batch(b))
+        ctx.backward()
+        key = b.input_size2
+        if key not in seen:
+            seen.add(key)
+            s = om.collect_samples_encdec(om.sizes_encdec(CFG, CFG.n_seqs, b.seq_len, b.dec_len))
+            s["x"], s["xt"] = key
+            samples.append(s)
+        i += 1
+    assert len(samples) >= 6
+    for j, s in enumerate(samples):
+        got = ctx.sample(j)
+        for k in ("x", "xt", "C", "E", "Hd", "Th", "Tb", "Te", "a", "y"):
+            assert got[k] == s[k], k
+    est = oe.Estimator2D(samples)
+    fn = op.plan
+    n_drop = 0
+    for Ss, St in pairs(CFG, 60, 22):
+        x, xt = CFG.n_seqs * Ss, CFG.n_seqs * St
+        p = ctx.plan(x, xt)
+        ost, od, opk = fn(est.predict(x, xt), M)
+        assert p.status == mb.OK and ost == op.OK
+        assert p.dropped == list(od) and p.predicted_peak == opk
+        assert ctx.dry_run(CFG.n_seqs, Ss, p.dropped, dec_len=St) <= M
+        n_drop += len(od) > 0
+    assert n_drop > 0
+    with pytest.raises(mb.MimoseError):
+        ctx.plan(CFG.n_seqs * 64)                         # the 1-D call is refused
