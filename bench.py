@@ -139,10 +139,19 @@ class Clocks:
                 "reasons": reasons, "samples": len(self.rows), "source": getattr(self, "source", None)}
 
 
-def step_flops(cfg, n_seqs, S):
+def step_flops(cfg, n_seqs, S, St=0):
     """Algorithmic FLOPs of one step: model = 3 x forward
-    (+ the LM head), and the forward FLOPs of one layer (added per dropped layer)."""
+    (+ the LM head), and the forward FLOPs of one layer (added per dropped layer).
+    Encoder-decoder: encoder layers at T_s, decoder layers (self + cross
+    attention + FFN) at T_t, LM head at T_t; the per-layer figure is the mean."""
     H, F, T = cfg.hidden, cfg.ffn, n_seqs * S
+    if cfg.arch == wl.ARCH_ENCDEC:
+        Tt = n_seqs * St
+        enc = 2.0 * T * (4 * H * H + 2 * H * F) + 4.0 * n_seqs * S * S * H
+        dec = (2.0 * Tt * (4 * H * H + 2 * H * F) + 2.0 * n_seqs * St * St * H          # self (causal)
+               + 2.0 * Tt * 2 * H * H + 2.0 * T * 2 * H * H + 4.0 * n_seqs * St * S * H)  # cross
+        model = 3.0 * (enc * cfg.n_layers + dec * cfg.n_dec_layers + 2.0 * Tt * H * cfg.vocab)
+        return model, (enc * cfg.n_layers + dec * cfg.n_dec_layers) / (cfg.n_layers + cfg.n_dec_layers)
     attn = 4.0 * n_seqs * S * S * H * (0.5 if cfg.arch == wl.ARCH_PRE_LN else 1.0)
     layer = 2.0 * T * (4 * H * H + 2 * H * F) + attn
     model = 3.0 * layer * cfg.n_layers
@@ -267,8 +276,10 @@ def main():
     # ---- budget (D2 / reading A21) from the library's own allocation sequence ----
     probe_ctx = mb.Mimose(cfg, 0, world=world, zero1=1 if args.zero1 else 0)
     C0 = probe_ctx.stats()["persistent_bytes"]
-    P0 = probe_ctx.dry_run(cfg.n_seqs, cfg.max_seq, [])
-    LB = probe_ctx.dry_run(cfg.n_seqs, cfg.max_seq, range(cfg.n_layers))
+    ed = cfg.arch == wl.ARCH_ENCDEC
+    dmax = cfg.max_seq if ed else None
+    P0 = probe_ctx.dry_run(cfg.n_seqs, cfg.max_seq, [], dec_len=dmax)
+    LB = probe_ctx.dry_run(cfg.n_seqs, cfg.max_seq, range(cfg.n_layers + cfg.n_dec_layers), dec_len=dmax)
     M = max(C0 + int(cfg.budget_frac * (P0 - C0)), LB)
     probe_ctx.close()
 
@@ -305,9 +316,15 @@ def main():
         return [wl.make_batch(cfg, sched[offset + i], seed=wl.batch_seed(cfg, offset + i, rank))
                 for i in range(n_total)]
 
+    def arrays(b):
+        xs = [b.input_ids, b.token_type, b.lengths, b.labels]
+        return xs + ([b.dec_ids, b.dec_lengths] if b.dec_ids is not None else [None, None])
+
     def to_dev(b):
-        return [torch.tensor(np.ascontiguousarray(x, np.int32)).cuda() for x in
-                (b.input_ids, b.token_type, b.lengths, b.labels)]
+        return [torch.tensor(np.ascontiguousarray(x, np.int32)).cuda() if x is not None else None for x in arrays(b)]
+
+    def plan_for(ctx, b):
+        return ctx.plan(*b.input_size2) if ed else ctx.plan(b.input_size)
 
     def barrier():
         torch.cuda.synchronize()
@@ -321,16 +338,16 @@ def main():
         if host:
             pinned = []
             for b in batches:
-                ts = [torch.from_numpy(np.ascontiguousarray(x, np.int32)).pin_memory() for x in
-                      (b.input_ids, b.token_type, b.lengths, b.labels)]
+                ts = [torch.from_numpy(np.ascontiguousarray(x, np.int32)).pin_memory() if x is not None else None
+                      for x in arrays(b)]
                 pinned.append(ts)
 
         def one(i):
             b = batches[i]
-            bs = (mb.Mimose.batch_struct(*pinned[i], b.n_seqs, b.seq_len, True) if host else
-                  mb.Mimose.batch_struct(*dev[i], b.n_seqs, b.seq_len, False))
+            t = pinned[i] if host else dev[i]
+            bs = mb.Mimose.batch_struct(*t[:4], b.n_seqs, b.seq_len, host, t[4], t[5], b.dec_len)
             if mode == "mimose":
-                p = ctx.plan(b.input_size)
+                p = plan_for(ctx, b)
             elif mode == "static":
                 p = plan_fixed
             else:
@@ -387,9 +404,11 @@ def main():
         return e0.elapsed_time(e1), n
 
     def tokens(batches):
+        """(mean S_pad, padded tokens, valid tokens); encoder-decoder: source + target."""
         bs = batches[args.warmup:]
-        return (float(np.mean([b.seq_len for b in bs])), int(sum(b.n_seqs * b.seq_len for b in bs)),
-                int(sum(int(b.lengths.sum()) for b in bs)))
+        return (float(np.mean([b.seq_len for b in bs])), int(sum(b.n_seqs * (b.seq_len + b.dec_len) for b in bs)),
+                int(sum(int(b.lengths.sum()) + (int(b.dec_lengths.sum()) if b.dec_lengths is not None else 0)
+                        for b in bs)))
 
     # ---- Mimose: sheltered phase, then the timed responsive steps ----
     ctx = new_ctx(M, M, granularity=args.granularity)
@@ -406,17 +425,17 @@ def main():
     # e2e: host buffers through the public API; H2D + loss D2H inside the timed region
     ms_e2e, _, _ = timed(ctx, batches, "mimose", host=True)
     e2e = samples_per_step * args.steps / (ms_e2e / 1000.0)
-    per_step_h2d = int(np.mean([(b.input_ids.size * 2 + b.lengths.size + b.labels.size) * 4 for b in batches]))
+    per_step_h2d = int(np.mean([sum(x.size for x in arrays(b) if x is not None) * 4 for b in batches]))
     st2 = ctx.stats()
     dropped, pred_err, flops_model, flops_hw = [], [], 0.0, 0.0
     for b in batches[args.warmup:]:
-        p = ctx.plan(b.input_size)
+        p = plan_for(ctx, b)
         dropped.append(p.n_dropped)
         # prediction error as the paper defines it, on the whole-step peak:
         # the estimator's predicted peak for the plan vs the arena's exact peak
-        actual = ctx.dry_run(b.n_seqs, b.seq_len, p.dropped)
+        actual = ctx.dry_run(b.n_seqs, b.seq_len, p.dropped, dec_len=b.dec_len if ed else None)
         pred_err.append(abs(p.predicted_peak - actual) / actual)
-        fm, fr = step_flops(cfg, b.n_seqs, b.seq_len)
+        fm, fr = step_flops(cfg, b.n_seqs, b.seq_len, b.dec_len)
         flops_model += fm
         flops_hw += fm + fr * p.n_dropped
     samples = [ctx.sample(j) for j in range(st["n_samples"])]
@@ -459,8 +478,9 @@ def main():
         "warmup": args.warmup, "ms_per_step": ms_s_step, "higher_is_better": True,
         "scaling": "weak", "vs_baseline": None, "dtype": "bf16" if cfg.dtype == "bf16" else "f32",
         "data": "synthetic",
-        "config": {"workload": cfg.name, "task": {wl.HEAD_MC: "SWAG-like multiple choice", wl.HEAD_QA: "span QA",
-                                                  wl.HEAD_LM: "causal LM"}.get(cfg.head, "seq-cls"),
+        "config": {"workload": cfg.name, "task": "translation-like encoder-decoder (UN_PC-like lengths)" if ed else
+                   {wl.HEAD_MC: "SWAG-like multiple choice", wl.HEAD_QA: "span QA",
+                    wl.HEAD_LM: "causal LM"}.get(cfg.head, "seq-cls"),
                    "batch_per_gpu": cfg.n_seqs, "samples_per_gpu_step": cfg.samples_per_step,
                    "seq_len": f"U[{cfg.seq_lo},{cfg.seq_hi}] pad {cfg.pad}", "budget_frac": cfg.budget_frac,
                    "budget_rule": "A21 (R2): M = max(C + f (P(empty, x_max) - C), LB(x_max))",
@@ -506,7 +526,7 @@ def main():
             sms, sn = sheltered(ctx, sched_, 2 * 10**6)
             out["sheltered_ms"] = sms
         if fixed == "static":
-            p = ctx.plan(cfg.n_seqs * cfg.max_seq)
+            p = ctx.plan(cfg.n_seqs * cfg.max_seq, cfg.n_seqs * cfg.max_seq if ed else None)
             ms_a, _, _ = timed(ctx, batches_, "static", plan_fixed=p)
             out["layers_dropped"] = p.n_dropped
         elif fixed == "all":
@@ -518,7 +538,7 @@ def main():
             ms_a, _, _ = timed(ctx, batches_, "none")
         else:
             ms_a, _, _ = timed(ctx, batches_, "mimose")
-            out["mean_dropped"] = float(np.mean([ctx.plan(b.input_size).n_dropped for b in batches_[args.warmup:]]))
+            out["mean_dropped"] = float(np.mean([plan_for(ctx, b).n_dropped for b in batches_[args.warmup:]]))
         sta = ctx.stats()
         out.update(value=samples_per_step * args.steps / (ms_a / 1000.0), ms_per_step=ms_a / args.steps,
                    violations=sta["violations"], peak_bytes_max=sta["max_peak_bytes"])
@@ -538,14 +558,15 @@ def main():
         result["all_ckpt"]["recompute_ratio"] = ms_a / ms_n
         # sub-layer checkpoint units (reading A30): attention / FFN
         # blocks planned independently by the same Algorithm 1, same budget
-        u, ms_u = arm(M, batches, sched, granularity=1)
-        u.update(units=2 * cfg.n_layers, recompute_ratio=ms_u / ms_n)
-        result["sublayer_units"] = u
+        if not ed:
+            u, ms_u = arm(M, batches, sched, granularity=1)
+            u.update(units=2 * cfg.n_layers, recompute_ratio=ms_u / ms_n)
+            result["sublayer_units"] = u
         # the Knapsack (reading A31): units planned by least total
-        # recompute time (the collector's t_l(x)), same budget
-        k, ms_k = arm(M, batches, sched, granularity=1, planner=mb.PLANNER_EXACT_TIME)
-        k.update(units=2 * cfg.n_layers, recompute_ratio=ms_k / ms_n)
-        result["knapsack_units"] = k
+        # recompute time (the collector's t_l(x)), same budget (encoder-decoder: layers)
+        k, ms_k = arm(M, batches, sched, granularity=0 if ed else 1, planner=mb.PLANNER_EXACT_TIME)
+        k.update(units=cfg.n_layers + cfg.n_dec_layers if ed else 2 * cfg.n_layers, recompute_ratio=ms_k / ms_n)
+        result["knapsack_units" if not ed else "knapsack_layers"] = k
         # the literal "f x no-checkpoint peak" budget, if feasible
         M_lit = int(cfg.budget_frac * P0)
         if M_lit >= LB:
@@ -565,7 +586,7 @@ def main():
         result["normal_schedule"] = nm
         # the multi-GPU code path on this one GPU: a 1-rank NCCL communicator with
         # ZeRO-1 (per-bucket reduce-scatter, sharded AdamW, weight all-gather)
-        if world == 1:
+        if world == 1 and not ed:
             z, ms_z = arm(M, batches, sched, comm_force=1, zero1=1)
             z.update(note="comm_force=1, zero1=1 at world 1: the DP/ZeRO-1 collectives run on a 1-rank "
                           "communicator", overhead_vs_headline=ms_z / ms)
