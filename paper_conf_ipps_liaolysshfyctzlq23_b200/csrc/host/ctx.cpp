@@ -22,6 +22,8 @@
 #include <unordered_map>
 #include <vector>
 
+#include <nvtx3/nvToolsExt.h>
+
 #include "../../../include/mimose.h"
 #include "../kernels.h"
 #include "planning.h"
@@ -31,6 +33,28 @@ using namespace mimose;
 namespace {
 
 inline int64_t a16(int64_t n) { return (n + 15) / 16 * 16; }
+
+// NVTX ranges for Nsight timelines (MIMOSE_NVTX=1): the public calls and every
+// layer / unit forward, recompute and backward.  Header-only NVTX v3; off by default.
+bool nvtx_on() {
+  static const bool v = [] {
+    const char* e = std::getenv("MIMOSE_NVTX");
+    return e && std::atoi(e) != 0;
+  }();
+  return v;
+}
+struct Range {
+  bool on;
+  explicit Range(const char* name) : on(nvtx_on()) { if (on) nvtxRangePushA(name); }
+  Range(const char* what, int idx) : on(nvtx_on()) {
+    if (on) {
+      char buf[64];
+      std::snprintf(buf, sizeof(buf), "%s %d", what, idx);
+      nvtxRangePushA(buf);
+    }
+  }
+  ~Range() { if (on) nvtxRangePop(); }
+};
 
 struct ParamInfo {
   int64_t numel, off;  // off in elements of the padded flat layout
@@ -1121,10 +1145,12 @@ mimose_status check_batch(mimose_ctx* c, const mimose_batch* bt) {
 }
 
 void layer_fwd_any(Run& r, int l, const char* x, LayerBufs& b, char* yout) {
+  Range rg(yout ? "layer fwd" : "layer recompute", l);
   if (r.c->cfg.arch != 0) layer_forward_pre(r, l, (const float*)x, b, (float*)yout);
   else layer_forward(r, l, x, b, yout);
 }
 void layer_bwd_any(Run& r, int l, const char* x, LayerBufs& b, float* dy, char* scr) {
+  Range rg("layer bwd", l);
   if (r.c->cfg.arch != 0) layer_backward_pre(r, l, (const float*)x, b, dy, scr);
   else layer_backward(r, l, x, b, dy, scr);
 }
@@ -2298,6 +2324,7 @@ static mimose_status begin_step(mimose_ctx* c, const mimose_batch* bt, uint64_t 
 }
 
 mimose_status mimose_collect(mimose_ctx* c, const mimose_batch* bt, float* loss_out) {
+  Range rg("mimose_collect");
   if (mimose_status s = check_ready(c)) return s;
   if (c->phase != MIMOSE_PHASE_SHELTERED) return fail(c, MIMOSE_E_STATE, "collect after the sheltered phase");
   if (c->fwd_done && !c->bwd_done) return fail(c, MIMOSE_E_STATE, "forward pending its backward");
@@ -2331,6 +2358,7 @@ mimose_status mimose_collect(mimose_ctx* c, const mimose_batch* bt, float* loss_
 }
 
 mimose_status mimose_forward(mimose_ctx* c, const mimose_batch* bt, const mimose_plan_t* plan, float* loss_out) {
+  Range rg("mimose_forward");
   if (mimose_status s = check_ready(c)) return s;
   if (c->fwd_done && !c->bwd_done) return fail(c, MIMOSE_E_STATE, "forward pending its backward");
   if (c->step_pending) return fail(c, MIMOSE_E_STATE, "fused optimizer: mimose_step must close the previous step");
@@ -2342,6 +2370,7 @@ mimose_status mimose_forward(mimose_ctx* c, const mimose_batch* bt, const mimose
 }
 
 mimose_status mimose_backward(mimose_ctx* c) {
+  Range rg("mimose_backward");
   if (mimose_status s = check_ready(c)) return s;
   if (!c->fwd_done || c->bwd_done) return fail(c, MIMOSE_E_STATE, "backward without a pending forward");
   Run r{c, c->device, sizes(c, c->B, c->S), c->st};
@@ -2380,6 +2409,7 @@ mimose_status mimose_backward(mimose_ctx* c) {
 }
 
 mimose_status mimose_step(mimose_ctx* c, float lr, float b1, float b2, float eps, float wd) {
+  Range rg("mimose_step");
   if (mimose_status s = check_ready(c)) return s;
   if (!c->bwd_done) return fail(c, MIMOSE_E_STATE, "step without a backward");
   if (!c->device) return MIMOSE_OK;
