@@ -219,6 +219,7 @@ __global__ void __launch_bounds__(ATT, 3) k_attn_fwd_tc(const __grid_constant__ 
   }
 }
 
+template <bool DC>   // DC: D = sum_k P~ dP~ (cross-attention); else rowsum(dO * O)
 __global__ void __launch_bounds__(ATT, 2) k_attn_bwd_tc(const __grid_constant__ CUtensorMap tq,
                                                      const __grid_constant__ CUtensorMap tk,
                                                      const __grid_constant__ CUtensorMap tdo, const AttnArgs a) {
@@ -277,8 +278,19 @@ __global__ void __launch_bounds__(ATT, 2) k_attn_bwd_tc(const __grid_constant__ 
   // near-uniform attention rows -- e.g. cross-attention -- keep their relative
   // accuracy).  Pass 1 over the TMEM row: P~, the dropout keep bits (kept in two
   // registers for pass 2), the D partial of this key half; D = half 0 + half 1.
-  float Lt = 0.f;
+  float Lt = 0.f, Dh = 0.f;
   if (t < len) Lt = a.lse_in[((int64_t)b * a.h + hd) * S + t];
+  if (!DC && t < len) {
+    // self-attention: D = rowsum(dO * O), half hf sums dims [32hf, 32hf+32); the
+    // global reads overlap the MMAs
+    const __nv_bfloat16* orow = a.O + ((int64_t)row0 + t) * a.H + hd * AD + 32 * hf;
+    const __nv_bfloat16* drow = a.dO + ((int64_t)row0 + t) * a.H + hd * AD + 32 * hf;
+    float ov[32], dv[32];
+    ld_bf16x32(orow, ov);
+    ld_bf16x32(drow, dv);
+#pragma unroll
+    for (int i = 0; i < 32; ++i) Dh += ov[i] * dv[i];
+  }
   mbar_wait(&bar[1], 0);
   __syncwarp();
   tc_fence_after();
@@ -288,8 +300,7 @@ __global__ void __launch_bounds__(ATT, 2) k_attn_bwd_tc(const __grid_constant__ 
   const float sl2 = a.scale * 1.4426950408889634f, Ll2 = Lt * 1.4426950408889634f;
   const float keepf = a.drop.enabled ? a.drop.scale : 1.0f;
   uint32_t kb0 = 0u, kb1 = 0u;             // keep bits of chunks c0 (kb0) and c0 + 1 (kb1) of this half
-  float Dh = 0.f;
-  for (int c = c0; c < c1; ++c)
+  for (int c = c0; c < c1 && DC; ++c)
 #pragma unroll
   for (int hh = 0; hh < 2; ++hh) {
     float sv[16], dp[16];
@@ -328,11 +339,20 @@ __global__ void __launch_bounds__(ATT, 2) k_attn_bwd_tc(const __grid_constant__ 
     const int kb = 32 * c + 16 * hh;
     const bool live = t < len && kb < kl;        // padded / foreign query rows contribute 0
     if (live) {
+      float fself[16];
+      if (!DC) {                                 // self-attention: the mask from Philox here
+#pragma unroll
+        for (int j = 0; j < 4; ++j) {
+          const int k = kb + 4 * j;
+          const float4 f = (k < kl) ? drop4_or(a.drop, ebase + k) : make_float4(0.f, 0.f, 0.f, 0.f);
+          fself[4 * j] = f.x; fself[4 * j + 1] = f.y; fself[4 * j + 2] = f.z; fself[4 * j + 3] = f.w;
+        }
+      }
 #pragma unroll
       for (int q = 0; q < 16; ++q) {
         const int kk = kb + q;
         const float p = (kk < kl) ? ex2f(fmaf(sv[q], sl2, -Ll2)) : 0.f;
-        const float fq = (((c == c0 ? kb0 : kb1) >> (16 * hh + q)) & 1u) ? keepf : 0.f;
+        const float fq = !DC ? fself[q] : ((((c == c0 ? kb0 : kb1) >> (16 * hh + q)) & 1u) ? keepf : 0.f);
         sv[q] = p * fq;                                            // P~
         dp[q] = p * (dp[q] * fq - Dt) * a.scale;                   // dS (scale folded)
       }
@@ -424,7 +444,9 @@ bool attn_bwd_tc(const void* qkv, const void* O, const void* dO, const float* ls
   if (!tc_map_bf16(&tq, qkv, 3ull * H, (uint64_t)B * S, 3ull * H, 64, AQ)) return false;
   if (!tc_map_bf16(&tdo, dO, (uint64_t)H, (uint64_t)B * S, (uint64_t)H, 64, AQ)) return false;
   static std::once_flag once;
-  std::call_once(once, [] { cudaFuncSetAttribute(k_attn_bwd_tc, cudaFuncAttributeMaxDynamicSharedMemorySize, BWD_SMEM); });
+  std::call_once(once, [] {
+    cudaFuncSetAttribute(k_attn_bwd_tc<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, BWD_SMEM);
+  });
   AttnArgs a{};
   a.S = S; a.Sk = S; a.H = H; a.h = h; a.B = B;
   a.qcol = 0; a.kcol = H; a.vcol = 2 * H;
@@ -432,7 +454,7 @@ bool attn_bwd_tc(const void* qkv, const void* O, const void* dO, const float* ls
   a.scale = 1.0f / sqrtf((float)AD);
   a.drop = drop; a.lengths = lengths; a.klens = lengths; a.O = (const __nv_bfloat16*)O; a.dO = (const __nv_bfloat16*)dO;
   a.lse_in = lse; a.dq = (__nv_bfloat16*)dqkv; a.dkv = (__nv_bfloat16*)dqkv; a.causal = causal;
-  launch_k(k_attn_bwd_tc, B * h, ATT, BWD_SMEM, st, tq, tq, tdo, a);
+  launch_k(k_attn_bwd_tc<false>, B * h, ATT, BWD_SMEM, st, tq, tq, tdo, a);
   return true;
 }
 
@@ -467,7 +489,9 @@ bool attn_cross_bwd_tc(const void* q, const void* kv, const void* O, const void*
   if (!tc_map_bf16(&tk, kv, 2ull * H, (uint64_t)B * Sk, 2ull * H, 64, AQ)) return false;
   if (!tc_map_bf16(&tdo, dO, (uint64_t)H, (uint64_t)B * Sq, (uint64_t)H, 64, AQ)) return false;
   static std::once_flag once;
-  std::call_once(once, [] { cudaFuncSetAttribute(k_attn_bwd_tc, cudaFuncAttributeMaxDynamicSharedMemorySize, BWD_SMEM); });
+  std::call_once(once, [] {
+    cudaFuncSetAttribute(k_attn_bwd_tc<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, BWD_SMEM);
+  });
   AttnArgs a{};
   a.S = Sq; a.Sk = Sk; a.H = H; a.h = h; a.B = B;
   a.qcol = 0; a.kcol = 0; a.vcol = H;
@@ -479,7 +503,7 @@ bool attn_cross_bwd_tc(const void* q, const void* kv, const void* O, const void*
   a.dq = (__nv_bfloat16*)dq; a.dkv = (__nv_bfloat16*)dkv;
   a.ldo = H; a.ocq = 0; a.ock = 0; a.ocv = H;
   a.ldk = 2 * H;
-  launch_k(k_attn_bwd_tc, B * h, ATT, BWD_SMEM, st, tq, tk, tdo, a);
+  launch_k(k_attn_bwd_tc<true>, B * h, ATT, BWD_SMEM, st, tq, tk, tdo, a);
   return true;
 }
 
