@@ -376,7 +376,7 @@ int64_t persistent_bytes(const mimose_ctx* c) {
   const int64_t maxT = (int64_t)c->cfg.max_seqs * c->cfg.max_seq_len;
   C += 2 * a16(maxT * 4) + a16((int64_t)c->cfg.max_seqs * 4) + a16(2LL * c->cfg.max_seqs * 4);
   C += a16(256);
-  C += a16(c->ws_elems * 4);                                   // split-K / stream-K workspace
+  C += a16(c->ws_elems * 4);                                   // wgrad split-K workspace
   C += a16((int64_t)NPART * 2 * std::max(3 * H, F) * 4);
   return C;
 }
@@ -610,51 +610,10 @@ void free_internals(Run& r, bool on_stack) {
   for (int i = 9; i >= 0; --i) on_stack ? a.pop(s[i]) : a.tfree(s[i]);
 }
 
-// MIMOSE_WGRAD_FUSED=1 enables (default off until it wins; see DESIGN) instead of the 128 x 128 / separate-reduction wgrad (A/B).
-static bool wgrad_fused(const mimose_ctx*) {
-  static const int v = [] {
-    const char* e = std::getenv("MIMOSE_WGRAD_FUSED");
-    return e ? std::atoi(e) : 0;
-  }();
-  return v != 0;
-}
-
 void wgrad(Run& r, const void* dY, int N, const void* X, int K, float* out) {
   // dW[N, K] = sum_t dY[t, n] X[t, k]; deterministic split-K over t.
   mimose_ctx* c = r.c;
   const int T = c->T;
-  if (c->dt == DT_BF16 && c->cfg.use_tc && K % 256 == 0 && N % 128 == 0 && wgrad_fused(c)) {
-    // 128 x 256 tiles (N = 256 MMAs; 128 x 128 ones are smem-bound at half
-    // rate) with an in-kernel fused split-K: pick the split s minimising
-    // rounds(s) / s, with the s-1 fp32 partials fitting the workspace; the
-    // 128 x 128 path below is modelled at 0.85 of a 128 x 256 tile-time.
-    const int t256 = (N / 128) * (K / 256);
-    double best = 1e30;
-    int bs = 1;
-    for (int s = 1; s <= 8; ++s) {
-      if ((int64_t)(s - 1) * N * K > c->ws_elems || T / s < 256) break;
-      const double v = (double)((t256 * s + 147) / 148) / s;
-      if (v < best - 1e-9) { best = v; bs = s; }
-    }
-    const int t128 = ((N + 127) / 128) * ((K + 127) / 128);
-    int s_old = std::max(1, std::min(4, 148 / std::max(1, t128)));
-    while (s_old > 1 && (int64_t)s_old * N * K > c->ws_elems) --s_old;
-    const double v_old = 0.85 * (double)((t128 * s_old + 147) / 148) / s_old;
-    if (best <= v_old) {
-      GemmArgs g;
-      g.M = N; g.N = K; g.K = T;
-      g.A = dY; g.a_sm = 1; g.a_sk = N;
-      g.B = X; g.b_sn = 1; g.b_sk = K;
-      g.C = out; g.ldc = K;
-      g.bn = 256;
-      g.split = bs;
-      g.fused_split = bs > 1;
-      g.ws = c->ws;
-      g.split_stride = (int64_t)N * K;
-      pgemm(c, EPI_F32, g, r.st);
-      return;
-    }
-  }
   const int tiles = ((N + 127) / 128) * ((K + 127) / 128);
   int split = std::max(1, std::min(4, 148 / std::max(1, tiles)));
   while (split > 1 && (int64_t)split * N * K > c->ws_elems) --split;
@@ -2536,16 +2495,6 @@ mimose_status mimose_plan2(mimose_ctx* c, int64_t x, int64_t xt, mimose_plan_t* 
 
 int32_t mimose_tc_available(void) { return tc_available() ? 1 : 0; }
 
-// Stream-K partial slots for the GEMM test hooks (outside any arena; tests only).
-static bool debug_sk_ws(GemmArgs& g) {
-  static float* sk_ws = nullptr;
-  const int64_t n = 148LL * 128 * 256;
-  if (!sk_ws && cudaMalloc(&sk_ws, n * 4) != cudaSuccess) return false;
-  g.ws = sk_ws;
-  g.ws_elems = n;
-  return true;
-}
-
 mimose_status mimose_debug_gemm_ex(int32_t epi, int32_t M, int32_t N, int32_t K, const void* A, int64_t a_sm,
                                    int64_t a_sk, const void* B, int64_t b_sn, int64_t b_sk, void* Cp, int64_t ldc,
                                    void* C2, const void* bias, const void* res, int64_t ldr, const void* aux,
@@ -2558,15 +2507,6 @@ mimose_status mimose_debug_gemm_ex(int32_t epi, int32_t M, int32_t N, int32_t K,
   g.C = Cp; g.ldc = ldc; g.C2 = C2; g.bias = bias; g.res = res; g.ldr = ldr; g.aux = aux; g.ldx = ldx;
   g.split = split < 1 ? 1 : split;
   g.split_stride = (int64_t)M * ldc;
-  if (split < 0) {          // fused split-K (EPI_F32, tile width 256): C2 is the partial workspace
-    if (epi != EPI_F32) return MIMOSE_E_INVALID;
-    g.split = -split;
-    g.fused_split = 1;
-    g.bn = 256;
-    g.ws = (float*)C2;
-    g.C2 = nullptr;
-  }
-  if (split == 1 && !debug_sk_ws(g)) return MIMOSE_E_CUDA;
   g.drop.enabled = 1; g.drop.seed_lo = 7; g.drop.seed_hi = 0; g.drop.site = 0; g.drop.step = 1;
   g.drop.thresh = 3865470566u; g.drop.scale = (float)(1.0 / 0.9);
   gemm(DT_BF16, (Epi)epi, g, (cudaStream_t)stream, use_tc != 0);
@@ -2603,7 +2543,6 @@ mimose_status mimose_debug_gemm(int32_t epi, int32_t M, int32_t N, int32_t K, co
   g.C = Cp; g.ldc = ldc; g.bias = bias;
   g.split = split < 1 ? 1 : split;
   g.split_stride = (int64_t)M * ldc;
-  if (g.split == 1 && !debug_sk_ws(g)) return MIMOSE_E_CUDA;
   gemm(DT_BF16, (Epi)epi, g, (cudaStream_t)stream, use_tc != 0);
   return cudaGetLastError() == cudaSuccess ? MIMOSE_OK : MIMOSE_E_CUDA;
 }

@@ -39,18 +39,7 @@ struct GemmArgs {
   const void* aux = nullptr; int64_t ldx = 0;
   Drop drop{};
   int split = 1; int64_t split_stride = 0;
-  // EPI_F32 with fused split-K (tcgen05 persistent kernel only): the units of
-  // split z >= 1 write fp32 partials to ws + (z-1)*split_stride and release a
-  // per-warp flag; the split-0 unit of the same tile waits for them and stores
-  // C = ((acc_0 + p_1) + p_2) + ... in that fixed order (deterministic, no
-  // separate reduction kernel).  bn: forced tile width (0 = heuristic).
-  int fused_split = 0;
-  float* ws = nullptr;
-  // ws_elems: capacity of ws.  With split == 1 and gemm mode 14, the persistent
-  // tcgen05 GEMM runs deterministic stream-K when ws holds one 128 x BN fp32
-  // partial tile per CTA (kernels_gemm_tc.cu seg_of; off by default).
-  int64_t ws_elems = 0;
-  int bn = 0;
+  int bn = 0;              // forced tile width (0 = heuristic)
 };
 void gemm(DType dt, Epi epi, const GemmArgs& g, cudaStream_t st, bool use_tc);
 bool tc_available();

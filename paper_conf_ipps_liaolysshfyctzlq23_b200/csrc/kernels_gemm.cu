@@ -88,14 +88,6 @@ void gemm(DType dt, Epi epi, const GemmArgs& g, cudaStream_t st, bool use_tc) {
   if (g.M <= 0 || g.N <= 0) return;
   note_launch(1);
   if (use_tc && dt == DT_BF16 && gemm_tc(epi, g, st)) return;
-  if (g.fused_split) {          // SIMT: one pass over all of K straight into C
-    GemmArgs g1 = g;
-    g1.fused_split = 0;
-    g1.split = 1;
-    if (dt == DT_F32) launch_simt<float>(epi, g1, st);
-    else launch_simt<__nv_bfloat16>(epi, g1, st);
-    return;
-  }
   if (dt == DT_F32) launch_simt<float>(epi, g, st);
   else launch_simt<__nv_bfloat16>(epi, g, st);
 }

@@ -29,19 +29,6 @@
 namespace mimose {
 
 constexpr int TBM = 128, TBK = 64;
-constexpr int TC_THREADS = 192;
-
-template <int BN>
-struct TcCfg {
-  // 3 stages (96 KB) so two CTAs share an SM: one CTA's epilogue overlaps the
-  // other's TMA/MMA main loop, and 296 tiles are resident per wave
-  static constexpr int STAGES = BN >= 256 ? 3 : 3;
-  static constexpr int A_BYTES = TBM * TBK * 2;
-  static constexpr int B_BYTES = BN * TBK * 2;
-  static constexpr int STAGE_BYTES = A_BYTES + B_BYTES;
-  static constexpr int SMEM = STAGES * STAGE_BYTES + 1024 /*align*/ + 256 /*barriers*/;
-};
-
 struct TcArgs {
   GemmArgs g;
   int a_mn, b_mn;           // 1: operand is MN-major (MN contiguous)
@@ -410,126 +397,6 @@ MDEV void epi_frag32_in(const GemmArgs& g, int m_base, int n, float (&v)[32], in
   }
 }
 
-template <int BN, int EPI>
-__global__ void __launch_bounds__(TC_THREADS, 2)
-    k_gemm_tc(const __grid_constant__ CUtensorMap tma_a, const __grid_constant__ CUtensorMap tma_b, const TcArgs args) {
-  pdl_enter();
-  using Cf = TcCfg<BN>;
-  extern __shared__ uint8_t smem_raw[];
-  uint8_t* smem = (uint8_t*)(((uintptr_t)smem_raw + 1023) & ~(uintptr_t)1023);
-  uint64_t* full = (uint64_t*)(smem + Cf::STAGES * Cf::STAGE_BYTES);
-  uint64_t* empty = full + Cf::STAGES;
-  uint64_t* tfull = empty + Cf::STAGES;
-  uint32_t* tmem_slot = (uint32_t*)(tfull + 1);
-
-  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
-  const int n0 = blockIdx.x * BN, m0 = blockIdx.y * TBM;
-  const int kb0 = blockIdx.z * args.kb_per_split;
-  const int kb1 = min(args.kb_total, kb0 + args.kb_per_split);
-  const int nkb = kb1 - kb0;
-
-  if (warp == 0 && lane == 0) {
-    for (int s = 0; s < Cf::STAGES; ++s) { mbar_init(&full[s], 1); mbar_init(&empty[s], 1); }
-    mbar_init(tfull, 1);
-    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
-    asm volatile("prefetch.tensormap [%0];" ::"l"(&tma_a) : "memory");
-    asm volatile("prefetch.tensormap [%0];" ::"l"(&tma_b) : "memory");
-  }
-  if (warp == 1) {
-    asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(smem_u32(tmem_slot)),
-                 "r"(BN));
-    asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;");
-  }
-  asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
-  __syncthreads();
-  asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
-  const uint32_t tmem = *tmem_slot;
-
-  if (warp == 0) {
-    if (lane == 0) {                                   // ---------------- TMA producer
-      for (int i = 0; i < nkb; ++i) {
-        const int s = i % Cf::STAGES;
-        if (i >= Cf::STAGES) mbar_wait(&empty[s], ((i / Cf::STAGES) - 1) & 1);
-        uint8_t* sa = smem + s * Cf::STAGE_BYTES;
-        uint8_t* sb = sa + Cf::A_BYTES;
-        const int k = (kb0 + i) * TBK;
-        mbar_expect_tx(&full[s], Cf::STAGE_BYTES);
-        if (args.a_mn) {
-          tma_load_2d(&tma_a, &full[s], sa, m0, k);
-          tma_load_2d(&tma_a, &full[s], sa + 8192, m0 + 64, k);
-        } else {
-          tma_load_2d(&tma_a, &full[s], sa, k, m0);
-        }
-        if (args.b_mn) {
-#pragma unroll
-          for (int j = 0; j < BN / 64; ++j) tma_load_2d(&tma_b, &full[s], sb + 8192 * j, n0 + 64 * j, k);
-        } else {
-          tma_load_2d(&tma_b, &full[s], sb, k, n0);
-        }
-      }
-    }
-  } else if (warp == 1) {
-    if (lane == 0) {                                   // ---------------- MMA issuer
-      const uint32_t idesc = (1u << 4) | (1u << 7) | (1u << 10) | ((uint32_t)args.a_mn << 15) |
-                             ((uint32_t)args.b_mn << 16) | ((uint32_t)(BN >> 3) << 17) | ((uint32_t)(TBM >> 4) << 24);
-      for (int i = 0; i < nkb; ++i) {
-        const int s = i % Cf::STAGES;
-        mbar_wait(&full[s], (i / Cf::STAGES) & 1);
-        asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
-        const uint32_t sa = smem_u32(smem + s * Cf::STAGE_BYTES);
-        const uint32_t sb = sa + Cf::A_BYTES;
-#pragma unroll
-        for (int kk = 0; kk < TBK / 16; ++kk) {
-          const uint64_t da = args.a_mn ? make_desc(sa + kk * 2048, 8192, 1024) : make_desc(sa + kk * 32, 16, 1024);
-          const uint64_t db = args.b_mn ? make_desc(sb + kk * 2048, 8192, 1024) : make_desc(sb + kk * 32, 16, 1024);
-          mma_bf16(tmem, da, db, idesc, (i > 0 || kk > 0) ? 1u : 0u);
-        }
-        mma_commit(&empty[s]);
-      }
-      mma_commit(tfull);
-    }
-  } else {                                             // ---------------- epilogue warps 2..5
-    const int q = warp & 3;
-    const int m = m0 + 32 * q + lane;
-    mbar_wait(tfull, 0);
-    asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
-    const GemmArgs& g = args.g;
-#pragma unroll 1
-    for (int c = 0; c < BN / 32; ++c) {
-      float v[32];
-      tmem_ld32(tmem + ((uint32_t)(32 * q) << 16) + 32 * c, v);
-      if (nkb <= 0) {                                  // empty split-K slice: exact zeros
-#pragma unroll
-        for (int i = 0; i < 32; ++i) v[i] = 0.f;
-      }
-      const int n = n0 + 32 * c;
-      if (m < g.M) {
-        if (n + 32 <= g.N) {
-          epi_row32<EPI>(g, m, n, v);
-        } else {
-#pragma unroll
-          for (int i = 0; i < 32; ++i)
-            if (n + i < g.N) epilogue<__nv_bfloat16, EPI>(g, m, n + i, v[i]);
-        }
-      }
-    }
-  }
-  asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
-  __syncthreads();
-  if (warp == 1) {
-    asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
-    asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(tmem), "r"(BN));
-  }
-}
-
-
-// ---------------------------------------------------------------------------
-// Persistent variant: grid = #SMs; each CTA walks tiles t = blockIdx.x + i*gridDim.x
-// (tile = (split, m-block, n-block), n fastest).  Two TMEM accumulators
-// (2 x BN columns) let the epilogue of tile i overlap the MMAs of tile i+1; the
-// smem ring continues across tiles.  8 epilogue warps: warp 2+e handles TMEM
-// lane quarter e%4 and column group e/4 (of TP_EPI_WARPS/4).
-// ---------------------------------------------------------------------------
 constexpr int TP_EPI_WARPS = 8;
 constexpr int TP_THREADS = 64 + 32 * TP_EPI_WARPS;
 
@@ -546,48 +413,17 @@ struct TpCfg {
 struct TpArgs {
   TcArgs t;
   int m_blocks = 0, n_blocks = 0, n_tiles = 0;
-  uint32_t* flags = nullptr;   // fused split-K: [split-1][per_split][TP_EPI_WARPS] release flags
-                               // stream-K: [CTA][TP_EPI_WARPS]
-  uint32_t epoch = 0;          // this launch's flag value (never reused within a process)
-  int sk = 0;                  // 1: deterministic stream-K (split must be 1)
-  float* sk_ws = nullptr;      // stream-K partial slots: [CTA][TBM * BN] fp32
 };
 
 // Work segment i of this CTA: tile r (m-block * n_blocks + n-block), split z
-// and k-block range [kb0, kb1).
-//   default: tile-major round robin, unit = blockIdx.x + i * gridDim.x.  Fused
-//   split-K orders the units z = split-1 first and z = 0 last, so a split-0
-//   unit (which waits for its partials) never runs in an earlier round than
-//   the units it waits on.
-//   stream-K: the n_tiles * kbt (tile, k-block) iterations are cut into
-//   gridDim.x contiguous ranges [u0, u1) (fixed by the shape and grid, so the
-//   split is the same on every launch).  A range starts inside a tile at most
-//   once (its first segment, which then only produces an fp32 partial) and
-//   ends inside a tile at most once (its last segment, the tile's "head",
-//   kb0 = 0): the head CTA adds the partials of CTAs blockIdx.x+1, +2, ...
-//   in that fixed order and runs the epilogue.  Producers compute their
-//   partial first and heads wait last, so the waits cannot deadlock with
-//   all CTAs resident (grid <= #SMs, one CTA per SM).
+// and k-block range [kb0, kb1); tile-major round robin, unit = blockIdx.x + i * gridDim.x.
 struct Seg { int r, z, kb0, kb1, p = 0; };
-MDEV int64_t sk_u0(int cta, int64_t W) { return (int64_t)cta * W / gridDim.x; }
-template <bool SK>
 MDEV bool seg_of(const TpArgs& a, int i, Seg& s) {
   const TcArgs& ta = a.t;
-  if (SK) {
-    const int64_t kbt = ta.kb_total, W = (int64_t)a.n_tiles * kbt;
-    const int64_t u0 = sk_u0(blockIdx.x, W), u1 = sk_u0(blockIdx.x + 1, W);
-    const int64_t t = u0 / kbt + i;
-    const int64_t st = i == 0 ? u0 : t * kbt;
-    if (st >= u1) return false;
-    const int64_t en = u1 < (t + 1) * kbt ? u1 : (t + 1) * kbt;
-    s.r = (int)t; s.z = 0; s.kb0 = (int)(st - t * kbt); s.kb1 = (int)(en - t * kbt);
-    return true;
-  }
   const int tile = blockIdx.x + i * gridDim.x;
   if (tile >= a.n_tiles) return false;
   const int per_split = a.m_blocks * a.n_blocks;
-  const int q = tile / per_split;
-  s.z = ta.g.fused_split ? ta.g.split - 1 - q : q;
+  s.z = tile / per_split;
   s.r = tile % per_split;
   s.kb0 = s.z * ta.kb_per_split;
   s.kb1 = min(ta.kb_total, s.kb0 + ta.kb_per_split);
@@ -595,10 +431,10 @@ MDEV bool seg_of(const TpArgs& a, int i, Seg& s) {
 }
 // Grouped launch of two independent problems (same epilogue, no split): tiles
 // of problem 0 first, then problem 1, one round-robin order over both.
-template <bool SK, bool G2>
+template <bool G2>
 MDEV bool seg_of2(const TpArgs& a, const TpArgs& a2, int i, Seg& s) {
   if constexpr (!G2) {
-    return seg_of<SK>(a, i, s);
+    return seg_of(a, i, s);
   } else {
     const int tile = blockIdx.x + i * gridDim.x;
     if (tile >= a.n_tiles + a2.n_tiles) return false;
@@ -610,21 +446,7 @@ MDEV bool seg_of2(const TpArgs& a, const TpArgs& a2, int i, Seg& s) {
     return true;
   }
 }
-MDEV uint32_t ld_acquire_u32(const uint32_t* p) {
-  uint32_t v;
-  asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
-  return v;
-}
-MDEV void st_release_u32(uint32_t* p, uint32_t v) {
-  asm volatile("st.release.gpu.global.u32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
-}
-MDEV float4 ld_cg_f4(const float* p) {
-  float4 v;
-  asm volatile("ld.global.cg.v4.f32 {%0, %1, %2, %3}, [%4];" : "=f"(v.x), "=f"(v.y), "=f"(v.z), "=f"(v.w) : "l"(p));
-  return v;
-}
-
-template <int BN, int EPI, bool SK, bool G2>
+template <int BN, int EPI, bool G2>
 __global__ void __launch_bounds__(TP_THREADS, 1)
     k_gemm_tcp(const __grid_constant__ CUtensorMap tma_a, const __grid_constant__ CUtensorMap tma_b, const TpArgs args,
                const __grid_constant__ CUtensorMap tma_a2, const __grid_constant__ CUtensorMap tma_b2,
@@ -669,7 +491,7 @@ __global__ void __launch_bounds__(TP_THREADS, 1)
     if (lane == 0) {                                   // ---------------- TMA producer
       int it = 0;
       Seg sg;
-      for (int si = 0; seg_of2<SK, G2>(args, args2, si, sg); ++si) {
+      for (int si = 0; seg_of2<G2>(args, args2, si, sg); ++si) {
         const TpArgs& A = (G2 && sg.p) ? args2 : args;
         const TcArgs& ta = A.t;
         const CUtensorMap* map_a = (G2 && sg.p) ? &tma_a2 : &tma_a;
@@ -705,7 +527,7 @@ __global__ void __launch_bounds__(TP_THREADS, 1)
     if (lane == 0) {                                   // ---------------- MMA issuer
       int it = 0, local = 0;
       Seg sg;
-      for (; seg_of2<SK, G2>(args, args2, local, sg); ++local) {
+      for (; seg_of2<G2>(args, args2, local, sg); ++local) {
         const TcArgs& ta = ((G2 && sg.p) ? args2 : args).t;
         const uint32_t idesc = idesc_bf16(TBM, BN, ta.a_mn, ta.b_mn);
         const int kb0 = sg.kb0, kb1 = sg.kb1;
@@ -736,7 +558,7 @@ __global__ void __launch_bounds__(TP_THREADS, 1)
     const int grp = e >> 2, ngrp = TP_EPI_WARPS / 4;  // column group of this warp
     int local = 0;
     Seg sg;
-    for (; seg_of2<SK, G2>(args, args2, local, sg); ++local) {
+    for (; seg_of2<G2>(args, args2, local, sg); ++local) {
       const TpArgs& A = (G2 && sg.p) ? args2 : args;
       const GemmArgs& g = A.t.g;
       const int z = sg.z, r = sg.r;
@@ -745,19 +567,6 @@ __global__ void __launch_bounds__(TP_THREADS, 1)
       const int acc = local & 1;
       const int m = m0 + 32 * q + lane;
       const int c_beg = grp * (BN / 32) / ngrp, c_end = (grp + 1) * (BN / 32) / ngrp;
-      // stream-K roles of this segment (see seg_of)
-      const bool sk_part = SK && kb0 > 0;                        // partial producer
-      const bool sk_head = SK && kb0 == 0 && kb1 < ta.kb_total;  // adds the partials
-      int sk_n = 0;                                                   // producers of a head
-      if (SK && sk_head) {
-        const int64_t W = (int64_t)args.n_tiles * ta.kb_total, tend = (int64_t)(r + 1) * ta.kb_total;
-        while (blockIdx.x + sk_n + 1 < gridDim.x && sk_u0(blockIdx.x + sk_n + 1, W) < tend) ++sk_n;
-        if (lane == 0)
-          for (int j = 1; j <= sk_n; ++j)
-            while (ld_acquire_u32(args.flags + (size_t)(blockIdx.x + j) * TP_EPI_WARPS + e) != args.epoch)
-              __nanosleep(64);
-        __syncwarp();
-      }
       {  // pull this tile's epilogue inputs into L2 while the MMAs run
         const int nb = n0 + 32 * c_beg;
         if (m < g.M && nb < g.N) {
@@ -771,16 +580,6 @@ __global__ void __launch_bounds__(TP_THREADS, 1)
           for (int o = 0; o < bytes; o += 128) asm volatile("prefetch.global.L2 [%0];" ::"l"(pa + o));
         }
       }
-      if constexpr (EPI == EPI_F32) {
-        if (g.fused_split && z == 0) {   // wait for this warp's partials of splits 1..split-1
-          if (lane == 0)
-            for (int zz = 1; zz < g.split; ++zz) {
-              const uint32_t* f = args.flags + ((size_t)(zz - 1) * per_split + r) * TP_EPI_WARPS + e;
-              while (ld_acquire_u32(f) != args.epoch) __nanosleep(64);
-            }
-          __syncwarp();
-        }
-      }
       // dropout keep bits of this warp's chunks, computed while the MMAs run
       constexpr int NCH = BN / 32 / (TP_EPI_WARPS / 4);
       uint32_t kbits[NCH];
@@ -790,7 +589,7 @@ __global__ void __launch_bounds__(TP_THREADS, 1)
         kbits[i] = 0u;
         if constexpr (DROP_EPI) {
           const int n = n0 + 32 * (c_beg + i);
-          if (m < g.M && n + 32 <= g.N && !(SK && sk_part)) kbits[i] = drop_bits32(g.drop, (uint64_t)m * g.ldc + n);
+          if (m < g.M && n + 32 <= g.N) kbits[i] = drop_bits32(g.drop, (uint64_t)m * g.ldc + n);
         }
       }
       EpiIn nxt;   // the first chunk's epilogue inputs are in flight while the MMAs finish
@@ -812,61 +611,12 @@ __global__ void __launch_bounds__(TP_THREADS, 1)
 #pragma unroll
           for (int i = 0; i < 32; ++i) v[i] = 0.f;
         }
-        if (SK && (sk_part || sk_head)) {   // fragment (q, c): 32 rows x 32 fp32, row = lane, in the CTA's slot
-          const size_t fo = ((size_t)(q * (BN / 32) + c) * 32 + lane) * 32;
-          if (sk_part) {
-            float4* p = (float4*)(args.sk_ws + (size_t)blockIdx.x * (TBM * BN) + fo);
-#pragma unroll
-            for (int j = 0; j < 8; ++j) p[j] = make_float4(v[4 * j], v[4 * j + 1], v[4 * j + 2], v[4 * j + 3]);
-            continue;
-          }
-          for (int jj = 1; jj <= sk_n; ++jj) {
-            const float* p = args.sk_ws + (size_t)(blockIdx.x + jj) * (TBM * BN) + fo;
-#pragma unroll
-            for (int j = 0; j < 8; ++j) {
-              const float4 w = ld_cg_f4(p + 4 * j);
-              v[4 * j] += w.x; v[4 * j + 1] += w.y; v[4 * j + 2] += w.z; v[4 * j + 3] += w.w;
-            }
-          }
-        }
-        if (EPI == EPI_F32 && g.fused_split && n + 32 <= g.N) {
-          const int mb = m0 + 32 * q;
-          if (mb < g.M) {
-            float* dst;
-            if (z > 0) {
-              dst = g.ws + (int64_t)(z - 1) * g.split_stride;
-            } else {
-              dst = (float*)g.C;
-              if (m < g.M)
-                for (int zz = 1; zz < g.split; ++zz) {
-                  const float* p = g.ws + (int64_t)(zz - 1) * g.split_stride + (int64_t)m * g.ldc + n;
-#pragma unroll
-                  for (int j = 0; j < 8; ++j) {
-                    const float4 w = ld_cg_f4(p + 4 * j);
-                    v[4 * j] += w.x; v[4 * j + 1] += w.y; v[4 * j + 2] += w.z; v[4 * j + 3] += w.w;
-                  }
-                }
-            }
-            stage_store_f32(stg_base + e * 4096, v, dst + (int64_t)mb * g.ldc + n, g.ldc, g.M - mb, lane);
-          }
-        } else if (n + 32 <= g.N) {
+        if (n + 32 <= g.N) {
           if (m0 + 32 * q < g.M) epi_frag32_in<EPI>(g, m0 + 32 * q, n, v, z, stg_base + e * 4096, lane, cur, keep);
         } else if (m < g.M) {
 #pragma unroll
           for (int i = 0; i < 32; ++i)
             if (n + i < g.N) epilogue<__nv_bfloat16, EPI>(g, m, n + i, v[i], z);
-        }
-      }
-      if (SK && sk_part) {               // publish this warp's stream-K partial
-        __threadfence();
-        __syncwarp();
-        if (lane == 0) st_release_u32(args.flags + (size_t)blockIdx.x * TP_EPI_WARPS + e, args.epoch);
-      }
-      if constexpr (EPI == EPI_F32) {
-        if (g.fused_split && z > 0) {    // publish this warp's partial rows/columns
-          __threadfence();
-          __syncwarp();
-          if (lane == 0) st_release_u32(args.flags + ((size_t)(z - 1) * per_split + r) * TP_EPI_WARPS + e, args.epoch);
         }
       }
       tc_fence_before();
@@ -883,212 +633,6 @@ __global__ void __launch_bounds__(TP_THREADS, 1)
 }
 
 
-// ---------------------------------------------------------------------------
-// CTA-pair variant (cta_group::2): a cluster of 2 CTAs on one TPC computes a
-// 256 x BN tile.  CTA r TMA-loads rows [128r, 128r+128) of A and rows
-// [BN/2 r, BN/2 (r+1)) of B into its own smem (transaction bytes land on the
-// leader's barrier); the leader's single thread issues tcgen05.mma.cta_group::2
-// (M = 256), which reads both CTAs' smem and writes rows 128r.. of the
-// accumulator into CTA r's TMEM.  Commits are multicast to both CTAs; both
-// CTAs' epilogue warps release an accumulator by arriving on the leader's
-// tmem-empty barrier.  Per SM this halves the B traffic and the smem operand
-// reads per MMA, relative to the single-CTA kernel.
-// ---------------------------------------------------------------------------
-constexpr uint32_t PEER_MASK = 0xFEFFFFFFu;
-
-template <int BN>
-struct T2Cfg {
-  static constexpr int A_BYTES = 128 * TBK * 2;
-  static constexpr int B_BYTES = (BN / 2) * TBK * 2;
-  static constexpr int STAGE_BYTES = A_BYTES + B_BYTES;
-  static constexpr int STAGES = (192 * 1024) / STAGE_BYTES;
-  static constexpr int SMEM = STAGES * STAGE_BYTES + 1024 + 512;
-};
-
-MDEV uint32_t cluster_rank() {
-  uint32_t r;
-  asm volatile("mov.u32 %0, %%cluster_ctarank;" : "=r"(r));
-  return r;
-}
-MDEV void cluster_sync_all() {
-  asm volatile("barrier.cluster.arrive.release.aligned;\nbarrier.cluster.wait.acquire.aligned;" ::: "memory");
-}
-MDEV void tma_load_2d_2sm(const CUtensorMap* map, uint64_t* bar, void* dst, int c0, int c1) {
-  asm volatile(
-      "cp.async.bulk.tensor.2d.cta_group::2.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1, {%3, %4}], [%2];"
-      ::"r"(smem_u32(dst)), "l"(map), "r"(smem_u32(bar) & PEER_MASK), "r"(c0), "r"(c1) : "memory");
-}
-MDEV void mma_bf16_2sm(uint32_t tmem_d, uint64_t da, uint64_t db, uint32_t idesc, uint32_t acc) {
-  asm volatile(
-      "{\n\t.reg .pred p;\n\tsetp.ne.b32 p, %4, 0;\n\t"
-      "tcgen05.mma.cta_group::2.kind::f16 [%0], %1, %2, %3, p;\n\t}"
-      ::"r"(tmem_d), "l"(da), "l"(db), "r"(idesc), "r"(acc));
-}
-MDEV void mma_commit_2sm_mc(uint64_t* bar) {
-  asm volatile("tcgen05.commit.cta_group::2.mbarrier::arrive::one.shared::cluster.multicast::cluster.b64 [%0], %1;"
-               ::"r"(smem_u32(bar)), "h"((uint16_t)3) : "memory");
-}
-MDEV void mbar_arrive_rank(uint64_t* bar, uint32_t rank) {
-  asm volatile("{\n\t.reg .b32 ra;\n\tmapa.shared::cluster.u32 ra, %0, %1;\n\t"
-               "mbarrier.arrive.release.cluster.shared::cluster.b64 _, [ra];\n\t}"
-               ::"r"(smem_u32(bar)), "r"(rank) : "memory");
-}
-
-template <int BN, int EPI>
-__global__ void __launch_bounds__(TP_THREADS, 1)
-    k_gemm_tc2(const __grid_constant__ CUtensorMap tma_a, const __grid_constant__ CUtensorMap tma_b, const TpArgs args) {
-  pdl_enter();
-  using Cf = T2Cfg<BN>;
-  extern __shared__ uint8_t smem_raw[];
-  uint8_t* smem = (uint8_t*)(((uintptr_t)smem_raw + 1023) & ~(uintptr_t)1023);
-  uint64_t* full = (uint64_t*)(smem + Cf::STAGES * Cf::STAGE_BYTES);
-  uint64_t* empty = full + Cf::STAGES;
-  uint64_t* tfull = empty + Cf::STAGES;    // [2]
-  uint64_t* tempty = tfull + 2;            // [2] (the leader's are used)
-  uint32_t* tmem_slot = (uint32_t*)(tempty + 2);
-  const TcArgs& ta = args.t;
-  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
-  const uint32_t rank = cluster_rank();
-  const bool leader = rank == 0;
-  const int cid = blockIdx.x >> 1, ncl = gridDim.x >> 1;
-
-  if (warp == 0 && lane == 0) {
-    for (int s = 0; s < Cf::STAGES; ++s) { mbar_init(&full[s], 1); mbar_init(&empty[s], 1); }
-    for (int a = 0; a < 2; ++a) { mbar_init(&tfull[a], 1); mbar_init(&tempty[a], 2 * TP_EPI_WARPS); }
-    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
-    asm volatile("prefetch.tensormap [%0];" ::"l"(&tma_a) : "memory");
-    asm volatile("prefetch.tensormap [%0];" ::"l"(&tma_b) : "memory");
-  }
-  if (warp == 1) {
-    asm volatile("tcgen05.alloc.cta_group::2.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(smem_u32(tmem_slot)),
-                 "r"(2 * BN));
-    asm volatile("tcgen05.relinquish_alloc_permit.cta_group::2.sync.aligned;");
-  }
-  tc_fence_before();
-  cluster_sync_all();
-  tc_fence_after();
-  const uint32_t tmem = *tmem_slot;
-  const int per_split = args.m_blocks * args.n_blocks;     // m_blocks counts 256-row pairs
-
-  if (warp == 0) {
-    if (lane == 0) {                                   // ---------------- TMA producer (both CTAs)
-      int it = 0;
-      for (int tile = cid; tile < args.n_tiles; tile += ncl) {
-        const int z = tile / per_split, r = tile % per_split;
-        const int m0 = (r / args.n_blocks) * 256 + 128 * rank;
-        const int nb = (r % args.n_blocks) * BN + (BN / 2) * rank;
-        const int kb0 = z * ta.kb_per_split, kb1 = min(ta.kb_total, kb0 + ta.kb_per_split);
-        for (int kb = kb0; kb < kb1; ++kb, ++it) {
-          const int s = it % Cf::STAGES;
-          if (it >= Cf::STAGES) mbar_wait(&empty[s], ((it / Cf::STAGES) - 1) & 1);
-          uint8_t* sa = smem + s * Cf::STAGE_BYTES;
-          uint8_t* sb = sa + Cf::A_BYTES;
-          const int k = kb * TBK;
-          if (leader) mbar_expect_tx(&full[s], 2 * Cf::STAGE_BYTES);
-          if (ta.a_mn) {
-            tma_load_2d_2sm(&tma_a, &full[s], sa, m0, k);
-            tma_load_2d_2sm(&tma_a, &full[s], sa + 8192, m0 + 64, k);
-          } else {
-            tma_load_2d_2sm(&tma_a, &full[s], sa, k, m0);
-          }
-          if (ta.b_mn) {
-#pragma unroll
-            for (int j = 0; j < BN / 128; ++j) tma_load_2d_2sm(&tma_b, &full[s], sb + 8192 * j, nb + 64 * j, k);
-          } else {
-            tma_load_2d_2sm(&tma_b, &full[s], sb, k, nb);
-          }
-        }
-      }
-    }
-  } else if (warp == 1) {
-    if (lane == 0 && leader) {                         // ---------------- MMA issuer (leader)
-      const uint32_t idesc = idesc_bf16(256, BN, ta.a_mn, ta.b_mn);
-      int it = 0, local = 0;
-      for (int tile = cid; tile < args.n_tiles; tile += ncl, ++local) {
-        const int z = tile / per_split;
-        const int kb0 = z * ta.kb_per_split, kb1 = min(ta.kb_total, kb0 + ta.kb_per_split);
-        const int acc = local & 1;
-        if (local >= 2) mbar_wait(&tempty[acc], ((local >> 1) - 1) & 1);
-        tc_fence_after();
-        const uint32_t d = tmem + acc * BN;
-        for (int kb = kb0; kb < kb1; ++kb, ++it) {
-          const int s = it % Cf::STAGES;
-          mbar_wait(&full[s], (it / Cf::STAGES) & 1);
-          tc_fence_after();
-          const uint32_t sa = smem_u32(smem + s * Cf::STAGE_BYTES);
-          const uint32_t sb = sa + Cf::A_BYTES;
-#pragma unroll
-          for (int kk = 0; kk < TBK / 16; ++kk) {
-            const uint64_t da = ta.a_mn ? make_desc(sa + kk * 2048, 8192, 1024) : make_desc(sa + kk * 32, 16, 1024);
-            const uint64_t db = ta.b_mn ? make_desc(sb + kk * 2048, 8192, 1024) : make_desc(sb + kk * 32, 16, 1024);
-            mma_bf16_2sm(d, da, db, idesc, (kb > kb0 || kk > 0) ? 1u : 0u);
-          }
-          mma_commit_2sm_mc(&empty[s]);
-        }
-        mma_commit_2sm_mc(&tfull[acc]);
-      }
-    }
-  } else {                                             // ---------------- epilogue warps (both CTAs)
-    const int e = warp - 2;
-    const int q = warp & 3;
-    const int grp = e >> 2, ngrp = TP_EPI_WARPS / 4;
-    const GemmArgs& g = ta.g;
-    int local = 0;
-    for (int tile = cid; tile < args.n_tiles; tile += ncl, ++local) {
-      const int z = tile / per_split, r = tile % per_split;
-      const int m0 = (r / args.n_blocks) * 256 + 128 * rank;
-      const int n0 = (r % args.n_blocks) * BN;
-      const int kb0 = z * ta.kb_per_split, kb1 = min(ta.kb_total, kb0 + ta.kb_per_split);
-      const int acc = local & 1;
-      const int m = m0 + 32 * q + lane;
-      const int c_beg = grp * (BN / 32) / ngrp, c_end = (grp + 1) * (BN / 32) / ngrp;
-      {
-        const int nbp = n0 + 32 * c_beg, ncol = 32 * (c_end - c_beg);
-        if (m < g.M && nbp < g.N) {
-          const char* pa = nullptr;
-          int bytes = 0;
-          if constexpr (EPI == EPI_GELU_BWD) { pa = (const char*)((const __nv_bfloat16*)g.aux + (int64_t)m * g.ldx + nbp); bytes = 2 * ncol; }
-          if constexpr (EPI == EPI_BIAS_DROP_RES) { pa = (const char*)((const __nv_bfloat16*)g.res + (int64_t)m * g.ldr + nbp); bytes = 2 * ncol; }
-          if constexpr (EPI == EPI_ACC_RES_F32) { pa = (const char*)((const float*)g.res + (int64_t)m * g.ldr + nbp); bytes = 4 * ncol; }
-          for (int o = 0; o < bytes; o += 128) asm volatile("prefetch.global.L2 [%0];" ::"l"(pa + o));
-        }
-      }
-      mbar_wait(&tfull[acc], (local >> 1) & 1);
-      __syncwarp();
-      tc_fence_after();
-#pragma unroll 1
-      for (int c = c_beg; c < c_end; ++c) {
-        float v[32];
-        tmem_ld32(tmem + acc * BN + ((uint32_t)(32 * q) << 16) + 32 * c, v);
-        if (kb1 <= kb0) {
-#pragma unroll
-          for (int i = 0; i < 32; ++i) v[i] = 0.f;
-        }
-        const int n = n0 + 32 * c;
-        if (m < g.M) {
-          if (n + 32 <= g.N) {
-            epi_row32<EPI>(g, m, n, v, z);
-          } else {
-#pragma unroll
-            for (int i = 0; i < 32; ++i)
-              if (n + i < g.N) epilogue<__nv_bfloat16, EPI>(g, m, n + i, v[i], z);
-          }
-        }
-      }
-      tc_fence_before();
-      __syncwarp();
-      if (lane == 0) mbar_arrive_rank(&tempty[acc], 0);
-    }
-  }
-  tc_fence_before();
-  cluster_sync_all();
-  if (warp == 1) {
-    tc_fence_after();
-    asm volatile("tcgen05.dealloc.cta_group::2.sync.aligned.b32 %0, %1;" ::"r"(tmem), "r"(2 * BN));
-  }
-}
-
-// ------------------------------------------------------------------ host --
 typedef CUresult (*EncodeFn)(CUtensorMap*, CUtensorMapDataType, cuuint32_t, void*, const cuuint64_t*,
                              const cuuint64_t*, const cuuint32_t*, const cuuint32_t*, CUtensorMapInterleave,
                              CUtensorMapSwizzle, CUtensorMapL2promotion, CUtensorMapFloatOOBfill);
@@ -1156,21 +700,10 @@ bool tc_map_bf16(CUtensorMap* out, const void* ptr, uint64_t inner, uint64_t out
 static int num_sms();
 
 template <int BN, int EPI>
-static void launch_tc(const CUtensorMap& ma, const CUtensorMap& mb, const TcArgs& a, dim3 grid, cudaStream_t st) {
-  static bool attr = false;
-  if (!attr) {
-    cudaFuncSetAttribute(k_gemm_tc<BN, EPI>, cudaFuncAttributeMaxDynamicSharedMemorySize, TcCfg<BN>::SMEM);
-    attr = true;
-  }
-  launch_k(k_gemm_tc<BN, EPI>, grid, TC_THREADS, TcCfg<BN>::SMEM, st, ma, mb, a);
-}
-
-template <int BN, int EPI>
 static void launch_tcp(const CUtensorMap& ma, const CUtensorMap& mb, const TpArgs& a, cudaStream_t st) {
   static bool attr = false;
   if (!attr) {
-    cudaFuncSetAttribute(k_gemm_tcp<BN, EPI, false, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, TpCfg<BN>::SMEM);
-    cudaFuncSetAttribute(k_gemm_tcp<BN, EPI, true, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, TpCfg<BN>::SMEM);
+    cudaFuncSetAttribute(k_gemm_tcp<BN, EPI, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, TpCfg<BN>::SMEM);
     attr = true;
   }
   static int nsm = 0;
@@ -1179,13 +712,7 @@ static void launch_tcp(const CUtensorMap& ma, const CUtensorMap& mb, const TpArg
     cudaGetDevice(&dev);
     cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, dev);
   }
-  const int64_t units = a.sk ? (int64_t)a.n_tiles * a.t.kb_total : a.n_tiles;
-  if (a.sk)
-    launch_k(k_gemm_tcp<BN, EPI, true, false>, (int)std::min<int64_t>(nsm, units), TP_THREADS, TpCfg<BN>::SMEM, st,
-             ma, mb, a, ma, mb, a);
-  else
-    launch_k(k_gemm_tcp<BN, EPI, false, false>, (int)std::min<int64_t>(nsm, units), TP_THREADS, TpCfg<BN>::SMEM, st,
-             ma, mb, a, ma, mb, a);
+  launch_k(k_gemm_tcp<BN, EPI, false>, std::min(nsm, a.n_tiles), TP_THREADS, TpCfg<BN>::SMEM, st, ma, mb, a, ma, mb, a);
 }
 
 // Two independent EPI_F32 problems in one persistent launch (grouped wgrad).
@@ -1194,11 +721,11 @@ static void launch_tcp_g2(const CUtensorMap& ma, const CUtensorMap& mb, const Tp
                           const CUtensorMap& mb2, const TpArgs& a2, cudaStream_t st) {
   static bool attr = false;
   if (!attr) {
-    cudaFuncSetAttribute(k_gemm_tcp<BN, EPI_F32, false, true>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+    cudaFuncSetAttribute(k_gemm_tcp<BN, EPI_F32, true>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                          TpCfg<BN>::SMEM);
     attr = true;
   }
-  launch_k(k_gemm_tcp<BN, EPI_F32, false, true>, std::min(num_sms(), a.n_tiles + a2.n_tiles), TP_THREADS,
+  launch_k(k_gemm_tcp<BN, EPI_F32, true>, std::min(num_sms(), a.n_tiles + a2.n_tiles), TP_THREADS,
            TpCfg<BN>::SMEM, st, ma, mb, a, ma2, mb2, a2);
 }
 
@@ -1220,79 +747,6 @@ static void dispatch_tcp(Epi epi, const CUtensorMap& ma, const CUtensorMap& mb, 
   }
 }
 
-template <int BN, int EPI>
-static void launch_tc2(const CUtensorMap& ma, const CUtensorMap& mb, const TpArgs& a, cudaStream_t st) {
-  static bool attr = false;
-  if (!attr) {
-    cudaFuncSetAttribute(k_gemm_tc2<BN, EPI>, cudaFuncAttributeMaxDynamicSharedMemorySize, T2Cfg<BN>::SMEM);
-    attr = true;
-  }
-  static int nsm = 0;
-  if (!nsm) {
-    int dev;
-    cudaGetDevice(&dev);
-    cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, dev);
-  }
-  cudaLaunchConfig_t cfg{};
-  cfg.gridDim = dim3(2 * std::min(nsm / 2, a.n_tiles));
-  cfg.blockDim = dim3(TP_THREADS);
-  cfg.dynamicSmemBytes = T2Cfg<BN>::SMEM;
-  cfg.stream = st;
-  cudaLaunchAttribute attr2[1];
-  attr2[0].id = cudaLaunchAttributeClusterDimension;
-  attr2[0].val.clusterDim.x = 2;
-  attr2[0].val.clusterDim.y = 1;
-  attr2[0].val.clusterDim.z = 1;
-  cfg.attrs = attr2;
-  cfg.numAttrs = 1;
-  cudaLaunchKernelEx(&cfg, k_gemm_tc2<BN, EPI>, ma, mb, a);
-}
-
-template <int BN>
-static void dispatch_tc2(Epi epi, const CUtensorMap& ma, const CUtensorMap& mb, const TpArgs& a, cudaStream_t st) {
-  switch (epi) {
-    case EPI_STORE: launch_tc2<BN, EPI_STORE>(ma, mb, a, st); break;
-    case EPI_BIAS: launch_tc2<BN, EPI_BIAS>(ma, mb, a, st); break;
-    case EPI_BIAS_GELU: launch_tc2<BN, EPI_BIAS_GELU>(ma, mb, a, st); break;
-    case EPI_BIAS_DROP_RES: launch_tc2<BN, EPI_BIAS_DROP_RES>(ma, mb, a, st); break;
-    case EPI_GELU_BWD: launch_tc2<BN, EPI_GELU_BWD>(ma, mb, a, st); break;
-    case EPI_ACC_RES_F32: launch_tc2<BN, EPI_ACC_RES_F32>(ma, mb, a, st); break;
-    case EPI_NONE: launch_tc2<BN, EPI_NONE>(ma, mb, a, st); break;
-    case EPI_BIAS_GELUT: launch_tc2<BN, EPI_BIAS_GELUT>(ma, mb, a, st); break;
-    case EPI_GELUT_BWD: launch_tc2<BN, EPI_GELUT_BWD>(ma, mb, a, st); break;
-    case EPI_BIAS_DROP_RESF32: launch_tc2<BN, EPI_BIAS_DROP_RESF32>(ma, mb, a, st); break;
-    case EPI_ACC_F32: launch_tc2<BN, EPI_ACC_F32>(ma, mb, a, st); break;
-    default: launch_tc2<BN, EPI_F32>(ma, mb, a, st); break;
-  }
-}
-
-// Release flags of the fused split-K GEMMs: one zero-initialised buffer per
-// device (outside the arena, like NCCL's buffers: 256 KB), and a process-wide
-// launch epoch, so flags never need resetting.  Fused split-K GEMMs of one
-// device are issued on one stream (the compute stream), never concurrently.
-constexpr size_t kFlagWords = 1 << 16;
-static uint32_t* splitk_flags() {
-  static std::mutex mu;
-  static std::unordered_map<int, uint32_t*> bufs;
-  int dev = 0;
-  cudaGetDevice(&dev);
-  std::lock_guard<std::mutex> lk(mu);
-  auto it = bufs.find(dev);
-  if (it != bufs.end()) return it->second;
-  uint32_t* p = nullptr;
-  if (cudaMalloc(&p, kFlagWords * 4) != cudaSuccess) return nullptr;
-  if (cudaMemset(p, 0, kFlagWords * 4) != cudaSuccess) return nullptr;
-  cudaDeviceSynchronize();
-  bufs[dev] = p;
-  return p;
-}
-static uint32_t next_epoch() {
-  static std::atomic<uint32_t> e{0};
-  uint32_t v = ++e;
-  if (v == 0) v = ++e;
-  return v;
-}
-
 static int num_sms() {
   static int nsm = 0;
   if (!nsm) {
@@ -1304,7 +758,7 @@ static int num_sms() {
   return nsm;
 }
 
-static int g_gemm_mode = 1;   // 0: one tile per CTA (k_gemm_tc); 1: persistent (k_gemm_tcp)
+static int g_gemm_mode = 1;   // 1: default; 12: force 128 x 256 tiles and no grouped launches (test hook)
 void set_gemm_mode(int m) { g_gemm_mode = m; }
 
 bool tc_available() { return encode_fn() != nullptr; }
@@ -1326,75 +780,19 @@ bool gemm_tc(Epi epi, const GemmArgs& g, cudaStream_t st) {
   a.kb_total = (g.K + TBK - 1) / TBK;
   a.kb_per_split = (a.kb_total + g.split - 1) / g.split;
   const int m_blocks = (g.M + TBM - 1) / TBM;
-  if ((g_gemm_mode == 2 || g_gemm_mode == 21 || g_gemm_mode == 22) && g.N % 128 == 0) {   // CTA pairs
-    const int m_pairs = (g.M + 255) / 256;
-    int BN2 = (g.N % 256 == 0 && m_pairs * (g.N / 256) * g.split >= 96) ? 256 : 128;
-    if (g_gemm_mode == 21) BN2 = 128;
-    if (g_gemm_mode == 22 && g.N % 256 == 0) BN2 = 256;
-    CUtensorMap ma2, mb2;
-    bool ok2 = a.a_mn ? make_map(&ma2, g.A, g.M, g.K, g.a_sk, 64, 64) : make_map(&ma2, g.A, g.K, g.M, g.a_sm, 64, 128);
-    if (ok2) ok2 = a.b_mn ? make_map(&mb2, g.B, g.N, g.K, g.b_sk, 64, 64)
-                          : make_map(&mb2, g.B, g.K, g.N, g.b_sn, 64, BN2 / 2);
-    if (ok2) {
-      TpArgs p;
-      p.t = a;
-      p.m_blocks = m_pairs;
-      p.n_blocks = g.N / BN2;
-      p.n_tiles = p.m_blocks * p.n_blocks * g.split;
-      if (BN2 == 256) dispatch_tc2<256>(epi, ma2, mb2, p, st);
-      else dispatch_tc2<128>(epi, ma2, mb2, p, st);
-      return true;
-    }
-  }
   // BN = 256 when N is a multiple of 256 and the 128x256 tiles fill at least half
-  // of the SMs; BN = 128 otherwise (measured per shape, tools/one_gemm.py; BN = 64
-  // loses on every step shape -- the per-tile fixed cost dominates).
-  auto tiles = [&](int bn) { return m_blocks * ((g.N + bn - 1) / bn) * g.split; };
+  // of the SMs; BN = 128 otherwise (measured per shape, tools/one_gemm.py).
   // 128-wide tiles run at ~0.58 of the 256-wide mainloop rate (half the work at
   // ~1.15x the time): 256-wide wins as soon as its tiles occupy half the SMs
   // (measured: T = 3584 x 768 x 3072 dropout-residual 29.1 us at 256 vs 39.5 at
-  // 128; T = 2560: 27.6 vs 23.8).
+  // 128; T = 2560: 27.6 vs 23.8).  Stream-K, CTA pairs, BN = 64, the
+  // one-tile-per-CTA kernel and an in-kernel fused split-K were built in round
+  // 1, measured slower on the step shapes and removed.
+  auto tiles = [&](int bn) { return m_blocks * ((g.N + bn - 1) / bn) * g.split; };
   int BN = (g.N % 256 == 0 && 2 * tiles(256) >= num_sms()) ? 256 : 128;
-  // Stream-K (split == 1, workspace given): cost model in 128 x 256 x 64
-  // k-block times -- data-parallel = rounds x k-blocks per tile; stream-K =
-  // the balanced share + ~4 blocks for the partial exchange; a 128-wide tile's
-  // k-block costs 0.86 (its mainloop runs at ~58% of the 256-wide rate).
-  bool sk = false;
-  const int nsm = num_sms();
-  // Off by default: measured on the BERT-base step shapes (T = 2048..8192),
-  // the balanced schedule runs its mainloop no faster than the data-parallel
-  // one on fewer SMs (e.g. TN 3072 x 768 x 5120: 758 vs 747 TFLOP/s), and the
-  // partial exchange then costs more than the balance gains -- see DESIGN §5.
-  const bool sk_mode = g_gemm_mode == 14;
-  if (sk_mode && g.split == 1 && !g.fused_split && g.ws && g.N % 128 == 0) {
-    const int64_t kbt = a.kb_total;
-    auto dp_cost = [&](int bn) {
-      return (double)((tiles(bn) + nsm - 1) / nsm) * kbt * (bn == 256 ? 1.0 : 0.86);
-    };
-    auto sk_ok = [&](int bn) {
-      const int64_t W = (int64_t)tiles(bn) * kbt;
-      return g.ws_elems >= std::min<int64_t>(nsm, W) * TBM * bn;
-    };
-    const int bn_sk = g.N % 256 == 0 ? 256 : 128;
-    const double sk_cost = (double)(((int64_t)tiles(bn_sk) * kbt + nsm - 1) / nsm) * (bn_sk == 256 ? 1.0 : 0.86) + 4.0;
-    double best = dp_cost(BN);
-    if (g.N % 256 == 0) best = std::min(best, dp_cost(256));
-    if (sk_ok(bn_sk) && (g_gemm_mode == 14 || sk_cost < 0.92 * best)) {
-      sk = true;
-      BN = bn_sk;
-    }
-  }
   if (g.bn == 256 && g.N % 256 == 0) BN = 256;
-  if (g.bn == 128 && !sk) BN = 128;
-  if (g_gemm_mode == 11) BN = 128;
+  if (g.bn == 128) BN = 128;
   if (g_gemm_mode == 12 && g.N % 256 == 0) BN = 256;
-  if (g_gemm_mode == 13) BN = 64;
-  // Modes 0 (and the CTA-pair fallback when N % 128 != 0) run the one-tile-per-CTA
-  // kernel, whose B tile is 128 rows: the tensor-map box must match the kernel.
-  const bool persistent = g_gemm_mode == 1 || g_gemm_mode == 11 || g_gemm_mode == 12 || g_gemm_mode == 13 ||
-                          g_gemm_mode == 2 || g_gemm_mode == 21 || g_gemm_mode == 22;
-  if (!persistent) BN = 128;
-  if (g.fused_split && (!persistent || epi != EPI_F32 || BN == 64)) return false;
   CUtensorMap ma, mb;
   bool ok;
   if (a.a_mn) ok = make_map(&ma, g.A, g.M, g.K, g.a_sk, 64, 64);
@@ -1403,51 +801,13 @@ bool gemm_tc(Epi epi, const GemmArgs& g, cudaStream_t st) {
   if (a.b_mn) ok = make_map(&mb, g.B, g.N, g.K, g.b_sk, 64, 64);
   else ok = make_map(&mb, g.B, g.K, g.N, g.b_sn, 64, std::min(BN, 256));
   if (!ok) return false;
-  if (persistent) {
-    TpArgs p;
-    p.t = a;
-    p.m_blocks = m_blocks;
-    p.n_blocks = (g.N + BN - 1) / BN;
-    p.n_tiles = p.m_blocks * p.n_blocks * g.split;
-    p.flags = nullptr;
-    p.epoch = 0;
-    p.sk = 0;
-    p.sk_ws = nullptr;
-    if (sk) {
-      if ((size_t)nsm * TP_EPI_WARPS > kFlagWords) return false;
-      p.sk = 1;
-      p.sk_ws = g.ws;
-      p.flags = splitk_flags();
-      if (!p.flags) return false;
-      p.epoch = next_epoch();
-    }
-    if (g.fused_split) {
-      if ((size_t)(g.split - 1) * p.m_blocks * p.n_blocks * TP_EPI_WARPS > kFlagWords) return false;
-      p.flags = splitk_flags();
-      if (!p.flags) return false;
-      p.epoch = next_epoch();
-    }
-    if (BN == 256) dispatch_tcp<256>(epi, ma, mb, p, st);
-    else if (BN == 128) dispatch_tcp<128>(epi, ma, mb, p, st);
-    else dispatch_tcp<64>(epi, ma, mb, p, st);
-    return true;
-  }
-  constexpr int BN1 = 128;
-  dim3 grid((g.N + BN1 - 1) / BN1, m_blocks, g.split);
-  switch (epi) {
-    case EPI_STORE: launch_tc<BN1, EPI_STORE>(ma, mb, a, grid, st); break;
-    case EPI_BIAS: launch_tc<BN1, EPI_BIAS>(ma, mb, a, grid, st); break;
-    case EPI_BIAS_GELU: launch_tc<BN1, EPI_BIAS_GELU>(ma, mb, a, grid, st); break;
-    case EPI_BIAS_DROP_RES: launch_tc<BN1, EPI_BIAS_DROP_RES>(ma, mb, a, grid, st); break;
-    case EPI_GELU_BWD: launch_tc<BN1, EPI_GELU_BWD>(ma, mb, a, grid, st); break;
-    case EPI_ACC_RES_F32: launch_tc<BN1, EPI_ACC_RES_F32>(ma, mb, a, grid, st); break;
-    case EPI_NONE: launch_tc<BN1, EPI_NONE>(ma, mb, a, grid, st); break;
-    case EPI_BIAS_GELUT: launch_tc<BN1, EPI_BIAS_GELUT>(ma, mb, a, grid, st); break;
-    case EPI_GELUT_BWD: launch_tc<BN1, EPI_GELUT_BWD>(ma, mb, a, grid, st); break;
-    case EPI_BIAS_DROP_RESF32: launch_tc<BN1, EPI_BIAS_DROP_RESF32>(ma, mb, a, grid, st); break;
-    case EPI_ACC_F32: launch_tc<BN1, EPI_ACC_F32>(ma, mb, a, grid, st); break;
-    default: launch_tc<BN1, EPI_F32>(ma, mb, a, grid, st); break;
-  }
+  TpArgs p;
+  p.t = a;
+  p.m_blocks = m_blocks;
+  p.n_blocks = (g.N + BN - 1) / BN;
+  p.n_tiles = p.m_blocks * p.n_blocks * g.split;
+  if (BN == 256) dispatch_tcp<256>(epi, ma, mb, p, st);
+  else dispatch_tcp<128>(epi, ma, mb, p, st);
   return true;
 }
 
@@ -1458,7 +818,7 @@ bool gemm_tc(Epi epi, const GemmArgs& g, cudaStream_t st) {
 // tile's K loop is the same as in a single launch, so results are bitwise
 // equal to two separate launches with the same tile width.
 bool gemm_tc_grouped(const GemmArgs& g1, const GemmArgs& g2, int bn, cudaStream_t st) {
-  if (g_gemm_mode != 1 || g1.split != 1 || g2.split != 1 || g1.fused_split || g2.fused_split) return false;
+  if (g_gemm_mode != 1 || g1.split != 1 || g2.split != 1) return false;
   if (bn != 128 && bn != 256) return false;
   TpArgs p[2];
   CUtensorMap ma[2], mb[2];
