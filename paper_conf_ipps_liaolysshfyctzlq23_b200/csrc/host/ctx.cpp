@@ -1327,9 +1327,9 @@ void dec_layer_backward(Run& r, const SzD& z, int j, const float* x, DecBufs& b,
   // cross-attention: dOc = dtc Wco (R2 head); dWco; attention backward -> dQc (R3), dKV
   dgrad(r, EPI_STORE, TAIL, H, W(c, DP(c, j, D_COW)), H, R2, nullptr);
   wgrad(r, TAIL, H, b.oc, H, G(c, DP(c, j, D_COW)));
-  attn_cross_bwd_tc(b.qc, b.kvc, b.oc, R2, b.lsec, c->lens_tgt, c->lens_src, R3, dKV, c->B, c->St, c->Ss, H, h,
+  attn_cross_bwd_tc(b.qc, b.kvc, b.oc, R2, b.lsec, c->lens_tgt, c->lens_src, Dbuf, R3, dKV, c->B, c->St, c->Ss, H, h,
                     make_drop(c, KIND_CROSS_PROBS, site), r.st);
-  note_launch(1);
+  note_launch(std::max(c->St, c->Ss) > 128 ? 2 : 1);
   // dc = dQc Wcq (dres); dWcq; dbcq
   dgrad(r, EPI_F32, R3, H, W(c, DP(c, j, D_CQW)), H, dres, nullptr);
   wgrad(r, R3, H, b.c, H, G(c, DP(c, j, D_CQW)));
@@ -1990,7 +1990,7 @@ mimose_status mimose_init(const mimose_config* cfgp, mimose_ctx** out) {
   auto bad = [&](const char* m) { c->err = m; return MIMOSE_E_INVALID; };
   const bool arch_ok = (k.arch == MIMOSE_ARCH_POST_LN && k.head >= 0 && k.head <= 2) || (k.arch == 1 && k.head == 3) ||
                        (k.arch == 2 && k.head == 3 && k.n_dec_layers >= 1 && k.n_layers + k.n_dec_layers <= 64 &&
-                        k.granularity == 0 && k.zero1 == 0 && !k.ffn_layers && k.max_seq_len <= 128 &&
+                        k.granularity == 0 && k.zero1 == 0 && !k.ffn_layers && k.max_seq_len <= 1024 &&
                         k.hidden / k.heads == 64 && k.ffn >= 2 * k.hidden &&
                         (!k.arena_base || (k.dtype == MIMOSE_BF16 && k.use_tc)));
   if (!arch_ok || k.n_layers < 1 || k.n_layers > 64 || k.hidden % 64 || k.heads < 1 ||

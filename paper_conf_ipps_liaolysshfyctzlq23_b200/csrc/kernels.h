@@ -65,12 +65,19 @@ void attn_bwd(DType dt, const void* qkv, const void* O, const void* dO, const fl
               Drop drop, cudaStream_t st, bool causal = false);
 
 // Cross-attention (encoder-decoder): q [B*Sq, H], kv [B*Sk, 2H] (k | v); key
-// padding by klens; tcgen05, Sq, Sk <= 128, head dim 64 (false: not launched).
+// padding by klens; tcgen05, head dim 64: the one-tile kernels when Sq, Sk <=
+// 128, else the tiled ones (<= 1024; Dbuf [B, h, Sq] fp32 scratch for D).
+// false: not launched.
 bool attn_cross_fwd_tc(const void* q, const void* kv, const int32_t* qlens, const int32_t* klens, void* O, float* lse,
                        int B, int Sq, int Sk, int H, int h, Drop drop, cudaStream_t st);
 bool attn_cross_bwd_tc(const void* q, const void* kv, const void* O, const void* dO, const float* lse,
-                       const int32_t* qlens, const int32_t* klens, void* dq, void* dkv, int B, int Sq, int Sk, int H,
-                       int h, Drop drop, cudaStream_t st);
+                       const int32_t* qlens, const int32_t* klens, float* Dbuf, void* dq, void* dkv, int B, int Sq,
+                       int Sk, int H, int h, Drop drop, cudaStream_t st);
+bool attn_cross_fwd_tcl(const void* q, const void* kv, const int32_t* qlens, const int32_t* klens, void* O, float* lse,
+                        int B, int Sq, int Sk, int H, int h, Drop drop, cudaStream_t st);
+bool attn_cross_bwd_tcl(const void* q, const void* kv, const void* O, const void* dO, const float* lse,
+                        const int32_t* qlens, const int32_t* klens, float* Dbuf, void* dq, void* dkv, int B, int Sq,
+                        int Sk, int H, int h, Drop drop, cudaStream_t st);
 
 // ----------------------------------------------------------- layernorm ----
 // y = LN(z) (y may be null: recompute with the output store gated off); st = (mu, rstd).

@@ -465,7 +465,8 @@ bool attn_cross_ok(int Sq, int Sk, int H, int h) { return Sq <= AQ && Sk <= AQ &
 
 bool attn_cross_fwd_tc(const void* q, const void* kv, const int32_t* qlens, const int32_t* klens, void* O, float* lse,
                        int B, int Sq, int Sk, int H, int h, Drop drop, cudaStream_t st) {
-  if (!attn_cross_ok(Sq, Sk, H, h)) return false;
+  if (!attn_cross_ok(Sq, Sk, H, h))        // a length above 128: the tiled kernels
+    return attn_cross_fwd_tcl(q, kv, qlens, klens, O, lse, B, Sq, Sk, H, h, drop, st);
   CUtensorMap tq, tk;
   if (!tc_map_bf16(&tq, q, (uint64_t)H, (uint64_t)B * Sq, (uint64_t)H, 64, AQ)) return false;
   if (!tc_map_bf16(&tk, kv, 2ull * H, (uint64_t)B * Sk, 2ull * H, 64, AQ)) return false;
@@ -481,9 +482,10 @@ bool attn_cross_fwd_tc(const void* q, const void* kv, const int32_t* qlens, cons
 }
 
 bool attn_cross_bwd_tc(const void* q, const void* kv, const void* O, const void* dO, const float* lse,
-                       const int32_t* qlens, const int32_t* klens, void* dq, void* dkv, int B, int Sq, int Sk, int H,
-                       int h, Drop drop, cudaStream_t st) {
-  if (!attn_cross_ok(Sq, Sk, H, h)) return false;
+                       const int32_t* qlens, const int32_t* klens, float* Dbuf, void* dq, void* dkv, int B, int Sq,
+                       int Sk, int H, int h, Drop drop, cudaStream_t st) {
+  if (!attn_cross_ok(Sq, Sk, H, h))
+    return attn_cross_bwd_tcl(q, kv, O, dO, lse, qlens, klens, Dbuf, dq, dkv, B, Sq, Sk, H, h, drop, st);
   CUtensorMap tq, tk, tdo;
   if (!tc_map_bf16(&tq, q, (uint64_t)H, (uint64_t)B * Sq, (uint64_t)H, 64, AQ)) return false;
   if (!tc_map_bf16(&tk, kv, 2ull * H, (uint64_t)B * Sk, 2ull * H, 64, AQ)) return false;

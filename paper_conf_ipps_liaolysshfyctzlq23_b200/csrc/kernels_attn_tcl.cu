@@ -37,7 +37,13 @@ constexpr int LPT = LQ * LQ * 2;         // 32 KB: [128 x 128] bf16 tile (2 atom
 constexpr int LTH = 256;                 // 8 warps
 
 struct LArgs {
-  int S, H, h, B;
+  int S, H, h, B;              // S: query rows per sequence
+  int Sk;                      // key rows per sequence (== S for self-attention)
+  int qcol, kcol, vcol;        // column bases of Q (tq) and K, V (tk)
+  const int32_t* klens;        // key lengths; lengths = query lengths
+  __nv_bfloat16* dq;           // dQ rows b*S + q (row stride ldq, column base ocq)
+  __nv_bfloat16* dkv;          // dK / dV rows b*Sk + k (row stride ldk, column bases ock / ocv)
+  int ldq, ocq, ldk, ock, ocv;
   int causal;
   float scale;
   Drop drop;
@@ -47,7 +53,6 @@ struct LArgs {
   float* lse;
   const float* lse_in;
   float* Dbuf;
-  __nv_bfloat16* dqkv;
   const __nv_bfloat16* dO;
 };
 
@@ -104,7 +109,8 @@ MDEV void mma_ptx(uint32_t d, uint32_t p, uint32_t x, bool acc) {
 // ---------------------------------------------------------------- forward --
 constexpr int LF_SMEM = 3 * LT + LPT + 1024 + 4096;   // Q, K, V, P~ + barriers / row partials + align slack
 
-__global__ void __launch_bounds__(LTH, 2) k_attn_fwd_tcl(const __grid_constant__ CUtensorMap tq, const LArgs a) {
+__global__ void __launch_bounds__(LTH, 2) k_attn_fwd_tcl(const __grid_constant__ CUtensorMap tq,
+                                                       const __grid_constant__ CUtensorMap tk, const LArgs a) {
   pdl_enter();
   extern __shared__ uint8_t smraw[];
   uint8_t* sm = (uint8_t*)(((uintptr_t)smraw + 1023) & ~(uintptr_t)1023);
@@ -119,7 +125,7 @@ __global__ void __launch_bounds__(LTH, 2) k_attn_fwd_tcl(const __grid_constant__
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const int hf = warp >> 2, t = 32 * (warp & 3) + lane;
   const int q0 = blockIdx.x * LQ, bh = blockIdx.y, b = bh / a.h, hd = bh % a.h;
-  const int S = a.S, len = a.lengths[b];
+  const int S = a.S, Sk = a.Sk, len = a.klens[b];
   const int q = q0 + t;
   const int kl = a.causal ? min(len, q + 1) : len;          // keys visible to row q
   const int kl_tile = a.causal ? min(len, q0 + LQ) : len;
@@ -132,7 +138,7 @@ __global__ void __launch_bounds__(LTH, 2) k_attn_fwd_tcl(const __grid_constant__
   bar_sync_all();
   const uint32_t tmem = *tslot;                 // S: cols 0..127, O: cols 128..191
   const uint32_t trow = tmem + ((uint32_t)(32 * (warp & 3)) << 16);
-  const int row0 = b * S;
+  const int row0 = b * S, krow0 = b * Sk;
   const float sl2 = a.scale * 1.4426950408889634f;
   // TMA prefetch (thread 0 only; its phase bits): pass 1 double-buffers K in sK / sV
   // (V is not needed yet); pass 2 reloads K as soon as S = Q K_j is done and V as
@@ -140,9 +146,9 @@ __global__ void __launch_bounds__(LTH, 2) k_attn_fwd_tcl(const __grid_constant__
   uint32_t ph_k0 = 0, ph_k1 = 0, ph_v = 0;
   if (threadIdx.x == 0 && nkt > 0) {
     mbar_expect_tx(&bar[0], LT);
-    tma_load_2d(&tq, &bar[0], sQ, hd * LD, row0 + q0);
+    tma_load_2d(&tq, &bar[0], sQ, a.qcol + hd * LD, row0 + q0);
     mbar_expect_tx(&bar[1], LT);
-    tma_load_2d(&tq, &bar[1], sK, a.H + hd * LD, row0);
+    tma_load_2d(&tk, &bar[1], sK, a.kcol + hd * LD, krow0);
   }
   int ph_s = 0, ph_o = 0;
   // ---- pass 1: exact row max and sum (log2 domain) ----
@@ -152,7 +158,7 @@ __global__ void __launch_bounds__(LTH, 2) k_attn_fwd_tcl(const __grid_constant__
       const int bf = j & 1;
       if (j + 1 < nkt) {                        // buffer !bf held K_{j-1}: its MMA is done
         mbar_expect_tx(&bar[bf ? 1 : 4], LT);
-        tma_load_2d(&tq, &bar[bf ? 1 : 4], bf ? sK : sV, a.H + hd * LD, row0 + (j + 1) * LQ);
+        tma_load_2d(&tk, &bar[bf ? 1 : 4], bf ? sK : sV, a.kcol + hd * LD, krow0 + (j + 1) * LQ);
       }
       if (j == 0) mbar_wait(&bar[0], 0);
       if (bf) { mbar_wait(&bar[4], ph_k1); ph_k1 ^= 1; }
@@ -188,13 +194,13 @@ __global__ void __launch_bounds__(LTH, 2) k_attn_fwd_tcl(const __grid_constant__
   const float lt = (m0 == -INFINITY ? 0.f : red[256 + t] * ex2a(m0 - M)) +
                    (m1 == -INFINITY ? 0.f : red[384 + t] * ex2a(m1 - M));
   const float L2 = M + __log2f(lt);             // log2-domain LSE of s * scale
-  const uint64_t ebase = (((uint64_t)b * a.h + hd) * S + (uint64_t)q) * S;
+  const uint64_t ebase = (((uint64_t)b * a.h + hd) * S + (uint64_t)q) * Sk;
   // ---- pass 2: P~ = exp(S - LSE) * dropout, O += P~ V ----
   if (threadIdx.x == 0 && nkt > 0) {            // every pass-1 MMA is done (bar[2] waited)
     mbar_expect_tx(&bar[1], LT);
-    tma_load_2d(&tq, &bar[1], sK, a.H + hd * LD, row0);
+    tma_load_2d(&tk, &bar[1], sK, a.kcol + hd * LD, krow0);
     mbar_expect_tx(&bar[5], LT);
-    tma_load_2d(&tq, &bar[5], sV, 2 * a.H + hd * LD, row0);
+    tma_load_2d(&tk, &bar[5], sV, a.vcol + hd * LD, krow0);
   }
   for (int j = 0; j < nkt; ++j) {
     if (threadIdx.x == 0) {
@@ -210,7 +216,7 @@ __global__ void __launch_bounds__(LTH, 2) k_attn_fwd_tcl(const __grid_constant__
     tc_fence_after();
     if (threadIdx.x == 0 && j + 1 < nkt) {      // sK is free once S = Q K_j is in TMEM
       mbar_expect_tx(&bar[1], LT);
-      tma_load_2d(&tq, &bar[1], sK, a.H + hd * LD, row0 + (j + 1) * LQ);
+      tma_load_2d(&tk, &bar[1], sK, a.kcol + hd * LD, krow0 + (j + 1) * LQ);
     }
 #pragma unroll
     for (int c = 0; c < 4; ++c) {
@@ -248,7 +254,7 @@ __global__ void __launch_bounds__(LTH, 2) k_attn_fwd_tcl(const __grid_constant__
     tc_fence_after();
     if (threadIdx.x == 0 && j + 1 < nkt) {
       mbar_expect_tx(&bar[5], LT);
-      tma_load_2d(&tq, &bar[5], sV, 2 * a.H + hd * LD, row0 + (j + 1) * LQ);
+      tma_load_2d(&tk, &bar[5], sV, a.vcol + hd * LD, krow0 + (j + 1) * LQ);
     }
   }
   {  // epilogue: half hf stores dims [32hf, 32hf + 32) of row q
@@ -274,7 +280,12 @@ __global__ void __launch_bounds__(LTH, 2) k_attn_fwd_tcl(const __grid_constant__
 // ------------------------------------------------------------ backward dQ --
 constexpr int LQ_SMEM = 6 * LT + LPT + 1024 + 2048;   // Q, dO, K[2], V[2], dS
 
+// DC (cross-attention): D = sum_k P~ dP~ over every key tile, in fp32 from the
+// same P~ and dP~ = dO V^T that dS uses (consistent under bf16 storage of O;
+// kernels_attn_tc.cu), by a first pass over the key tiles; else rowsum(dO * O).
+template <bool DC>
 __global__ void __launch_bounds__(LTH, 1) k_attn_bwd_dq_tcl(const __grid_constant__ CUtensorMap tq,
+                                                            const __grid_constant__ CUtensorMap tk,
                                                             const __grid_constant__ CUtensorMap tdo, const LArgs a) {
   pdl_enter();
   extern __shared__ uint8_t smraw[];
@@ -292,11 +303,11 @@ __global__ void __launch_bounds__(LTH, 1) k_attn_bwd_dq_tcl(const __grid_constan
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const int hf = warp >> 2, t = 32 * (warp & 3) + lane;
   const int q0 = blockIdx.x * LQ, bh = blockIdx.y, b = bh / a.h, hd = bh % a.h;
-  const int S = a.S, len = a.lengths[b];
+  const int S = a.S, Sk = a.Sk, len = a.lengths[b], klen = a.klens[b];
   const int q = q0 + t;
   const bool live = q < len;                    // padded query rows carry zero gradient (A26)
-  const int kl = a.causal ? min(len, q + 1) : len;
-  const int kl_tile = a.causal ? min(len, q0 + LQ) : len;
+  const int kl = a.causal ? min(klen, q + 1) : klen;
+  const int kl_tile = a.causal ? min(klen, q0 + LQ) : klen;
   const int nkt = q0 < len ? (kl_tile + LQ - 1) / LQ : 0;
   if (threadIdx.x == 0) {
     for (int i = 0; i < 5; ++i) mbar_init(&bar[i], 1);
@@ -306,89 +317,100 @@ __global__ void __launch_bounds__(LTH, 1) k_attn_bwd_dq_tcl(const __grid_constan
   bar_sync_all();
   const uint32_t tmem = *tslot;                 // S 0..127, dP 128..255, dQ 256..319
   const uint32_t trow = tmem + ((uint32_t)(32 * (warp & 3)) << 16);
-  const int row0 = b * S;
+  const int row0 = b * S, krow0 = b * Sk;
+  auto load_kv = [&](int j, int bf) {           // thread 0
+    mbar_expect_tx(&bar[bf ? 4 : 1], 2 * LT);
+    tma_load_2d(&tk, &bar[bf ? 4 : 1], sKb(bf), a.kcol + hd * LD, krow0 + j * LQ);
+    tma_load_2d(&tk, &bar[bf ? 4 : 1], sVb(bf), a.vcol + hd * LD, krow0 + j * LQ);
+  };
   if (threadIdx.x == 0 && nkt > 0) {
     mbar_expect_tx(&bar[0], 2 * LT);
-    tma_load_2d(&tq, &bar[0], sQ, hd * LD, row0 + q0);
+    tma_load_2d(&tq, &bar[0], sQ, a.qcol + hd * LD, row0 + q0);
     tma_load_2d(&tdo, &bar[0], sdO, hd * LD, row0 + q0);
-    mbar_expect_tx(&bar[1], 2 * LT);
-    tma_load_2d(&tq, &bar[1], sKb(0), a.H + hd * LD, row0);
-    tma_load_2d(&tq, &bar[1], sVb(0), 2 * a.H + hd * LD, row0);
+    load_kv(0, 0);
   }
-  // D_q = rowsum(dO * O): half hf sums dims [32hf, 32hf + 32); D = half 0 + half 1
   float Dh = 0.f, Lt = 0.f;
-  if (live) {
+  if (live) Lt = a.lse_in[((int64_t)b * a.h + hd) * S + q];
+  if (!DC && live) {   // D_q = rowsum(dO * O): half hf sums dims [32hf, 32hf + 32)
     float ov[32], dv[32];
     ld_bf16x32(a.O + ((int64_t)row0 + q) * a.H + hd * LD + 32 * hf, ov);
     ld_bf16x32(a.dO + ((int64_t)row0 + q) * a.H + hd * LD + 32 * hf, dv);
 #pragma unroll
     for (int i = 0; i < 32; ++i) Dh += ov[i] * dv[i];
-    Lt = a.lse_in[((int64_t)b * a.h + hd) * S + q];
   }
-  red[hf * 128 + t] = Dh;
-  __syncthreads();
-  const float Dt = red[t] + red[128 + t];
-  if (hf == 0 && q < S) a.Dbuf[((int64_t)b * a.h + hd) * S + q] = Dt;
   const float sl2 = a.scale * 1.4426950408889634f, Ll2 = Lt * 1.4426950408889634f;
-  const uint64_t ebase = (((uint64_t)b * a.h + hd) * S + (uint64_t)q) * S;
+  const uint64_t ebase = (((uint64_t)b * a.h + hd) * S + (uint64_t)q) * Sk;
   uint32_t ph_kv0 = 0, ph_kv1 = 0;
   int ph_s = 0, ph_o = 0;
-  for (int j = 0; j < nkt; ++j) {
-    const int bf = j & 1;
-    uint8_t* sK = sKb(bf);
-    uint8_t* sV = sVb(bf);
-    if (threadIdx.x == 0) {
-      if (j + 1 < nkt) {                        // buffer !bf held tile j-1: its MMAs are done
-        mbar_expect_tx(&bar[bf ? 1 : 4], 2 * LT);
-        tma_load_2d(&tq, &bar[bf ? 1 : 4], sKb(bf ^ 1), a.H + hd * LD, row0 + (j + 1) * LQ);
-        tma_load_2d(&tq, &bar[bf ? 1 : 4], sVb(bf ^ 1), 2 * a.H + hd * LD, row0 + (j + 1) * LQ);
+  float Dt = 0.f;
+  // pass 0 (DC only): D over every key tile; pass 1: dS and dQ += dS K
+  for (int pass = DC ? 0 : 1; pass < 2; ++pass) {
+    if (pass == 1) {
+      red[hf * 128 + t] = Dh;
+      __syncthreads();
+      Dt = red[t] + red[128 + t];
+      if (hf == 0 && q < S) a.Dbuf[((int64_t)b * a.h + hd) * S + q] = Dt;
+      __syncthreads();                          // every D read before red[] is reused
+      if (DC && threadIdx.x == 0 && nkt > 0) load_kv(0, 0);   // pass 0's MMAs are done (bar[2] waited)
+    }
+    for (int j = 0; j < nkt; ++j) {
+      const int bf = j & 1;
+      uint8_t* sK = sKb(bf);
+      uint8_t* sV = sVb(bf);
+      if (threadIdx.x == 0) {
+        if (j + 1 < nkt) load_kv(j + 1, bf ^ 1);   // buffer !bf held tile j-1: its MMAs are done
+        if (j == 0 && pass == (DC ? 0 : 1)) mbar_wait(&bar[0], 0);
+        if (bf) { mbar_wait(&bar[4], ph_kv1); ph_kv1 ^= 1; }
+        else { mbar_wait(&bar[1], ph_kv0); ph_kv0 ^= 1; }
+        tc_fence_after();
+        mma_nt64(tmem, smem_u32(sQ), smem_u32(sK));          // S = Q K^T
+        mma_nt64(tmem + 128, smem_u32(sdO), smem_u32(sV));   // dP~ = dO V^T
+        mma_commit(&bar[2]);
       }
-      if (j == 0) mbar_wait(&bar[0], 0);
-      if (bf) { mbar_wait(&bar[4], ph_kv1); ph_kv1 ^= 1; }
-      else { mbar_wait(&bar[1], ph_kv0); ph_kv0 ^= 1; }
+      mbar_wait(&bar[2], ph_s);
+      ph_s ^= 1;
+      __syncwarp();
       tc_fence_after();
-      mma_nt64(tmem, smem_u32(sQ), smem_u32(sK));          // S = Q K^T
-      mma_nt64(tmem + 128, smem_u32(sdO), smem_u32(sV));   // dP~ = dO V^T
-      mma_commit(&bar[2]);
-    }
-    mbar_wait(&bar[2], ph_s);
-    ph_s ^= 1;
-    __syncwarp();
-    tc_fence_after();
 #pragma unroll
-    for (int c = 0; c < 4; ++c) {
-      float sv[16], dp[16];
-      tmem_ld16(trow + 64 * hf + 16 * c, sv);
-      tmem_ld16(trow + 128 + 64 * hf + 16 * c, dp);
-      const int kb = j * LQ + 64 * hf + 16 * c;
-      if (live && kb < kl) {
+      for (int c = 0; c < 4; ++c) {
+        float sv[16], dp[16];
+        tmem_ld16(trow + 64 * hf + 16 * c, sv);
+        tmem_ld16(trow + 128 + 64 * hf + 16 * c, dp);
+        const int kb = j * LQ + 64 * hf + 16 * c;
+        if (live && kb < kl) {
 #pragma unroll
-        for (int g = 0; g < 4; ++g) {
-          const int k = kb + 4 * g;
-          const float4 f = k < kl ? drop4l(a.drop, ebase + k) : make_float4(0.f, 0.f, 0.f, 0.f);
-          const float ff[4] = {f.x, f.y, f.z, f.w};
+          for (int g = 0; g < 4; ++g) {
+            const int k = kb + 4 * g;
+            const float4 f = k < kl ? drop4l(a.drop, ebase + k) : make_float4(0.f, 0.f, 0.f, 0.f);
+            const float ff[4] = {f.x, f.y, f.z, f.w};
 #pragma unroll
-          for (int i = 0; i < 4; ++i) {
-            const float p = (k + i < kl) ? ex2a(fmaf(sv[4 * g + i], sl2, -Ll2)) : 0.f;
-            dp[4 * g + i] = p * (dp[4 * g + i] * ff[i] - Dt) * a.scale;   // dS (scale folded)
+            for (int i = 0; i < 4; ++i) {
+              const float p = (k + i < kl) ? ex2a(fmaf(sv[4 * g + i], sl2, -Ll2)) : 0.f;
+              if (pass == 0) Dh = fmaf(p * ff[i], dp[4 * g + i], Dh);
+              dp[4 * g + i] = p * (dp[4 * g + i] * ff[i] - Dt) * a.scale;   // dS (scale folded)
+            }
           }
-        }
-      } else {
+        } else {
 #pragma unroll
-        for (int i = 0; i < 16; ++i) dp[i] = 0.f;
+          for (int i = 0; i < 16; ++i) dp[i] = 0.f;
+        }
+        if (pass == 1) st_row16(sdS, t, 4 * hf + c, dp);
       }
-      st_row16(sdS, t, 4 * hf + c, dp);
+      if (pass == 0) {
+        bar_sync_all();                          // S / dP read before the next tile's MMAs
+        continue;
+      }
+      fence_async_smem();
+      bar_sync_all();
+      if (threadIdx.x == 0) {
+        mma_pv(tmem + 256, smem_u32(sdS), smem_u32(sK), j > 0);   // dQ += dS K
+        mma_commit(&bar[3]);
+      }
+      mbar_wait(&bar[3], ph_o);
+      ph_o ^= 1;
+      __syncwarp();
+      tc_fence_after();
     }
-    fence_async_smem();
-    bar_sync_all();
-    if (threadIdx.x == 0) {
-      mma_pv(tmem + 256, smem_u32(sdS), smem_u32(sK), j > 0);   // dQ += dS K
-      mma_commit(&bar[3]);
-    }
-    mbar_wait(&bar[3], ph_o);
-    ph_o ^= 1;
-    __syncwarp();
-    tc_fence_after();
   }
   {
     float v[32];
@@ -397,7 +419,7 @@ __global__ void __launch_bounds__(LTH, 1) k_attn_bwd_dq_tcl(const __grid_constan
 #pragma unroll
       for (int i = 0; i < 32; ++i) v[i] = 0.f;
     }
-    if (q < S) st_bf16x32(a.dqkv + ((int64_t)row0 + q) * 3 * a.H + hd * LD + 32 * hf, v);
+    if (q < S) st_bf16x32(a.dq + ((int64_t)row0 + q) * a.ldq + a.ocq + hd * LD + 32 * hf, v);
   }
   tc_fence_before();
   __syncthreads();
@@ -411,6 +433,7 @@ __global__ void __launch_bounds__(LTH, 1) k_attn_bwd_dq_tcl(const __grid_constan
 constexpr int LKV_SMEM = 6 * LT + 2 * LPT + 1024 + 2048;   // K, V, Q[2], dO[2], P~, dS
 
 __global__ void __launch_bounds__(LTH, 1) k_attn_bwd_dkv_tcl(const __grid_constant__ CUtensorMap tq,
+                                                             const __grid_constant__ CUtensorMap tk,
                                                              const __grid_constant__ CUtensorMap tdo, const LArgs a) {
   pdl_enter();
   extern __shared__ uint8_t smraw[];
@@ -427,10 +450,10 @@ __global__ void __launch_bounds__(LTH, 1) k_attn_bwd_dkv_tcl(const __grid_consta
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const int hf = warp >> 2, t = 32 * (warp & 3) + lane;
   const int k0 = blockIdx.x * LQ, bh = blockIdx.y, b = bh / a.h, hd = bh % a.h;
-  const int S = a.S, len = a.lengths[b];
+  const int S = a.S, Sk = a.Sk, len = a.lengths[b], klen = a.klens[b];
   // query tiles that see keys [k0, k0 + 128): causal -> q >= k0; only q < len carry gradient
   const int i0 = a.causal ? k0 / LQ : 0;
-  const int i1 = k0 < len ? (len + LQ - 1) / LQ : 0;
+  const int i1 = k0 < klen ? (len + LQ - 1) / LQ : 0;
   if (threadIdx.x == 0) {
     for (int i = 0; i < 5; ++i) mbar_init(&bar[i], 1);
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
@@ -439,13 +462,13 @@ __global__ void __launch_bounds__(LTH, 1) k_attn_bwd_dkv_tcl(const __grid_consta
   bar_sync_all();
   const uint32_t tmem = *tslot;                 // S 0..127, dP 128..255, dV 256..319, dK 320..383
   const uint32_t trow = tmem + ((uint32_t)(32 * (warp & 3)) << 16);
-  const int row0 = b * S;
+  const int row0 = b * S, krow0 = b * Sk;
   if (threadIdx.x == 0 && i1 > i0) {
     mbar_expect_tx(&bar[0], 2 * LT);
-    tma_load_2d(&tq, &bar[0], sK, a.H + hd * LD, row0 + k0);
-    tma_load_2d(&tq, &bar[0], sV, 2 * a.H + hd * LD, row0 + k0);
+    tma_load_2d(&tk, &bar[0], sK, a.kcol + hd * LD, krow0 + k0);
+    tma_load_2d(&tk, &bar[0], sV, a.vcol + hd * LD, krow0 + k0);
     mbar_expect_tx(&bar[1], 2 * LT);
-    tma_load_2d(&tq, &bar[1], sQb(0), hd * LD, row0 + i0 * LQ);
+    tma_load_2d(&tq, &bar[1], sQb(0), a.qcol + hd * LD, row0 + i0 * LQ);
     tma_load_2d(&tdo, &bar[1], sdOb(0), hd * LD, row0 + i0 * LQ);
   }
   const float sl2 = a.scale * 1.4426950408889634f;
@@ -458,7 +481,7 @@ __global__ void __launch_bounds__(LTH, 1) k_attn_bwd_dkv_tcl(const __grid_consta
     if (threadIdx.x == 0) {
       if (i + 1 < i1) {                         // buffer !bf held tile i-1: its MMAs are done
         mbar_expect_tx(&bar[bf ? 1 : 4], 2 * LT);
-        tma_load_2d(&tq, &bar[bf ? 1 : 4], sQb(bf ^ 1), hd * LD, row0 + (i + 1) * LQ);
+        tma_load_2d(&tq, &bar[bf ? 1 : 4], sQb(bf ^ 1), a.qcol + hd * LD, row0 + (i + 1) * LQ);
         tma_load_2d(&tdo, &bar[bf ? 1 : 4], sdOb(bf ^ 1), hd * LD, row0 + (i + 1) * LQ);
       }
       if (i == i0) mbar_wait(&bar[0], 0);
@@ -471,14 +494,14 @@ __global__ void __launch_bounds__(LTH, 1) k_attn_bwd_dkv_tcl(const __grid_consta
     }
     const int q = i * LQ + t;
     const bool live = q < len;
-    const int kl = a.causal ? min(len, q + 1) : len;
+    const int kl = a.causal ? min(klen, q + 1) : klen;
     float Lt = 0.f, Dt = 0.f;
     if (live) {
       Lt = a.lse_in[((int64_t)b * a.h + hd) * S + q];
       Dt = a.Dbuf[((int64_t)b * a.h + hd) * S + q];
     }
     const float Ll2 = Lt * 1.4426950408889634f;
-    const uint64_t ebase = (((uint64_t)b * a.h + hd) * S + (uint64_t)q) * S;
+    const uint64_t ebase = (((uint64_t)b * a.h + hd) * S + (uint64_t)q) * Sk;
     mbar_wait(&bar[2], ph_s);
     ph_s ^= 1;
     __syncwarp();
@@ -523,20 +546,20 @@ __global__ void __launch_bounds__(LTH, 1) k_attn_bwd_dkv_tcl(const __grid_consta
   }
   {  // TMEM lanes of dV / dK = key rows k0 + t
     const int k = k0 + t;
-    __nv_bfloat16* row = a.dqkv + ((int64_t)row0 + k) * 3 * a.H + hd * LD + 32 * hf;
+    __nv_bfloat16* row = a.dkv + ((int64_t)krow0 + k) * a.ldk + hd * LD + 32 * hf;
     float v[32];
     tmem_ld32(trow + 320 + 32 * hf, v);
     if (i1 <= i0) {
 #pragma unroll
       for (int e = 0; e < 32; ++e) v[e] = 0.f;
     }
-    if (k < S) st_bf16x32(row + a.H, v);                 // dK
+    if (k < Sk) st_bf16x32(row + a.ock, v);              // dK
     tmem_ld32(trow + 256 + 32 * hf, v);
     if (i1 <= i0) {
 #pragma unroll
       for (int e = 0; e < 32; ++e) v[e] = 0.f;
     }
-    if (k < S) st_bf16x32(row + 2 * a.H, v);             // dV
+    if (k < Sk) st_bf16x32(row + a.ocv, v);              // dV
   }
   tc_fence_before();
   __syncthreads();
@@ -554,18 +577,36 @@ bool tc_map_bf16(CUtensorMap* out, const void* ptr, uint64_t inner, uint64_t out
 
 bool attn_tcl_ok(int S, int H, int h) { return S > LQ && S <= 1024 && H / h == LD && H % 64 == 0; }
 
+namespace {
+LArgs self_args(int B, int S, int H, int h, Drop drop, const int32_t* lengths, bool causal) {
+  LArgs a{};
+  a.S = S; a.Sk = S; a.H = H; a.h = h; a.B = B;
+  a.qcol = 0; a.kcol = H; a.vcol = 2 * H;
+  a.scale = 1.0f / sqrtf((float)LD);
+  a.drop = drop; a.lengths = lengths; a.klens = lengths; a.causal = causal;
+  a.ldq = 3 * H; a.ocq = 0; a.ldk = 3 * H; a.ock = H; a.ocv = 2 * H;
+  return a;
+}
+void set_attrs() {
+  static std::once_flag once;
+  std::call_once(once, [] {
+    cudaFuncSetAttribute(k_attn_fwd_tcl, cudaFuncAttributeMaxDynamicSharedMemorySize, LF_SMEM);
+    cudaFuncSetAttribute(k_attn_bwd_dq_tcl<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, LQ_SMEM);
+    cudaFuncSetAttribute(k_attn_bwd_dq_tcl<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, LQ_SMEM);
+    cudaFuncSetAttribute(k_attn_bwd_dkv_tcl, cudaFuncAttributeMaxDynamicSharedMemorySize, LKV_SMEM);
+  });
+}
+}  // namespace
+
 bool attn_fwd_tcl(const void* qkv, const int32_t* lengths, void* O, float* lse, int B, int S, int H, int h,
                   Drop drop, cudaStream_t st, bool causal) {
   if (!attn_tcl_ok(S, H, h)) return false;
   CUtensorMap tq;
   if (!tc_map_bf16(&tq, qkv, 3ull * H, (uint64_t)B * S, 3ull * H, 64, LQ)) return false;
-  static std::once_flag once;
-  std::call_once(once, [] { cudaFuncSetAttribute(k_attn_fwd_tcl, cudaFuncAttributeMaxDynamicSharedMemorySize, LF_SMEM); });
-  LArgs a{};
-  a.S = S; a.H = H; a.h = h; a.B = B;
-  a.scale = 1.0f / sqrtf((float)LD);
-  a.drop = drop; a.lengths = lengths; a.Oout = (__nv_bfloat16*)O; a.lse = lse; a.causal = causal;
-  launch_k(k_attn_fwd_tcl, dim3((S + LQ - 1) / LQ, B * h), LTH, LF_SMEM, st, tq, a);
+  set_attrs();
+  LArgs a = self_args(B, S, H, h, drop, lengths, causal);
+  a.Oout = (__nv_bfloat16*)O; a.lse = lse;
+  launch_k(k_attn_fwd_tcl, dim3((S + LQ - 1) / LQ, B * h), LTH, LF_SMEM, st, tq, tq, a);
   return true;
 }
 
@@ -575,19 +616,53 @@ bool attn_bwd_tcl(const void* qkv, const void* O, const void* dO, const float* l
   CUtensorMap tq, tdo;
   if (!tc_map_bf16(&tq, qkv, 3ull * H, (uint64_t)B * S, 3ull * H, 64, LQ)) return false;
   if (!tc_map_bf16(&tdo, dO, (uint64_t)H, (uint64_t)B * S, (uint64_t)H, 64, LQ)) return false;
-  static std::once_flag once;
-  std::call_once(once, [] {
-    cudaFuncSetAttribute(k_attn_bwd_dq_tcl, cudaFuncAttributeMaxDynamicSharedMemorySize, LQ_SMEM);
-    cudaFuncSetAttribute(k_attn_bwd_dkv_tcl, cudaFuncAttributeMaxDynamicSharedMemorySize, LKV_SMEM);
-  });
-  LArgs a{};
-  a.S = S; a.H = H; a.h = h; a.B = B;
-  a.scale = 1.0f / sqrtf((float)LD);
-  a.drop = drop; a.lengths = lengths; a.O = (const __nv_bfloat16*)O; a.dO = (const __nv_bfloat16*)dO;
-  a.lse_in = lse; a.Dbuf = Dbuf; a.dqkv = (__nv_bfloat16*)dqkv; a.causal = causal;
+  set_attrs();
+  LArgs a = self_args(B, S, H, h, drop, lengths, causal);
+  a.O = (const __nv_bfloat16*)O; a.dO = (const __nv_bfloat16*)dO;
+  a.lse_in = lse; a.Dbuf = Dbuf; a.dq = (__nv_bfloat16*)dqkv; a.dkv = (__nv_bfloat16*)dqkv;
   const dim3 grid((S + LQ - 1) / LQ, B * h);
-  launch_k(k_attn_bwd_dq_tcl, grid, LTH, LQ_SMEM, st, tq, tdo, a);     // also writes D for the dK/dV pass
-  launch_k(k_attn_bwd_dkv_tcl, grid, LTH, LKV_SMEM, st, tq, tdo, a);
+  launch_k(k_attn_bwd_dq_tcl<false>, grid, LTH, LQ_SMEM, st, tq, tq, tdo, a);   // also writes D for the dK/dV pass
+  launch_k(k_attn_bwd_dkv_tcl, grid, LTH, LKV_SMEM, st, tq, tq, tdo, a);
+  return true;
+}
+
+// Cross-attention (encoder-decoder) on the tiled kernels: queries q [B*Sq, H],
+// keys / values kv [B*Sk, 2H]; Sq, Sk <= 1024.  The backward's D is the
+// consistent sum_k P~ dP~ (dQ kernel pass 0), kept in Dbuf [B, h, Sq].
+bool attn_cross_tcl_ok(int Sq, int Sk, int H, int h) {
+  return Sq <= 1024 && Sk <= 1024 && H / h == LD && H % 64 == 0;
+}
+
+bool attn_cross_fwd_tcl(const void* q, const void* kv, const int32_t* qlens, const int32_t* klens, void* O, float* lse,
+                        int B, int Sq, int Sk, int H, int h, Drop drop, cudaStream_t st) {
+  if (!attn_cross_tcl_ok(Sq, Sk, H, h)) return false;
+  CUtensorMap tq, tk;
+  if (!tc_map_bf16(&tq, q, (uint64_t)H, (uint64_t)B * Sq, (uint64_t)H, 64, LQ)) return false;
+  if (!tc_map_bf16(&tk, kv, 2ull * H, (uint64_t)B * Sk, 2ull * H, 64, LQ)) return false;
+  set_attrs();
+  LArgs a = self_args(B, Sq, H, h, drop, qlens, false);
+  a.Sk = Sk; a.klens = klens; a.qcol = 0; a.kcol = 0; a.vcol = H;
+  a.Oout = (__nv_bfloat16*)O; a.lse = lse;
+  launch_k(k_attn_fwd_tcl, dim3((Sq + LQ - 1) / LQ, B * h), LTH, LF_SMEM, st, tq, tk, a);
+  return true;
+}
+
+bool attn_cross_bwd_tcl(const void* q, const void* kv, const void* O, const void* dO, const float* lse,
+                        const int32_t* qlens, const int32_t* klens, float* Dbuf, void* dq, void* dkv, int B, int Sq,
+                        int Sk, int H, int h, Drop drop, cudaStream_t st) {
+  if (!attn_cross_tcl_ok(Sq, Sk, H, h)) return false;
+  CUtensorMap tq, tk, tdo;
+  if (!tc_map_bf16(&tq, q, (uint64_t)H, (uint64_t)B * Sq, (uint64_t)H, 64, LQ)) return false;
+  if (!tc_map_bf16(&tk, kv, 2ull * H, (uint64_t)B * Sk, 2ull * H, 64, LQ)) return false;
+  if (!tc_map_bf16(&tdo, dO, (uint64_t)H, (uint64_t)B * Sq, (uint64_t)H, 64, LQ)) return false;
+  set_attrs();
+  LArgs a = self_args(B, Sq, H, h, drop, qlens, false);
+  a.Sk = Sk; a.klens = klens; a.qcol = 0; a.kcol = 0; a.vcol = H;
+  a.O = (const __nv_bfloat16*)O; a.dO = (const __nv_bfloat16*)dO; a.lse_in = lse; a.Dbuf = Dbuf;
+  a.dq = (__nv_bfloat16*)dq; a.ldq = H; a.ocq = 0;
+  a.dkv = (__nv_bfloat16*)dkv; a.ldk = 2 * H; a.ock = 0; a.ocv = H;
+  launch_k(k_attn_bwd_dq_tcl<true>, dim3((Sq + LQ - 1) / LQ, B * h), LTH, LQ_SMEM, st, tq, tk, tdo, a);
+  launch_k(k_attn_bwd_dkv_tcl, dim3((Sk + LQ - 1) / LQ, B * h), LTH, LKV_SMEM, st, tq, tk, tdo, a);
   return true;
 }
 

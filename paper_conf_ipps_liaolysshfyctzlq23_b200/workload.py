@@ -148,10 +148,9 @@ CONFIGS: Dict[str, ModelConfig] = {
     # P:73 input sizes 17-460).  T5-base shapes (12 + 12 layers, H 768, 12 heads,
     # F 3072, 32128-word tied vocabulary) with pre-LN blocks (T5 is pre-norm),
     # biases and tanh-GELU kept, absolute positions (reading A32); source
-    # lengths 17-128 (the one-tile attention kernels; reading A32), target =
-    # source x U[0.8, 1.2]; budget 50%.
+    # lengths 17-460, target = source x U[0.8, 1.2]; budget 50%.
     "t5-base": ModelConfig("t5-base", 6, 12, 768, 12, 3072, 32128, 512, 0, 0,
-                           HEAD_LM, 1, 2, "bf16", 1e-6, 0.1, 8, 17, 128, 8, 0.5,
+                           HEAD_LM, 1, 2, "bf16", 1e-6, 0.1, 8, 17, 460, 8, 0.5,
                            1, 1, 0, 3, ARCH_ENCDEC, (), 12),
 }
 

@@ -23,6 +23,8 @@ import parity_metrics as pm
 
 SMALL = wl.small_config("t5-base", n_layers=2, n_dec_layers=2, hidden=128, heads=2, ffn=256, vocab=500,
                         max_pos=128, n_seqs=4, seq_lo=17, seq_hi=100, pad=8)
+LONG = wl.small_config("t5-base", n_layers=2, n_dec_layers=2, hidden=128, heads=2, ffn=256, vocab=500,
+                       max_pos=512, n_seqs=3, seq_lo=130, seq_hi=300, pad=8)      # tiled cross-attention
 FULL = wl.small_config("t5-base", n_layers=2, n_dec_layers=2)
 
 
@@ -57,7 +59,8 @@ def bf16(params):
     return {k: torch.tensor(v).bfloat16().double().numpy() for k, v in params.items()}
 
 
-@pytest.mark.parametrize("name,cfg,S", [("t5-small", SMALL, 100), ("t5-s128", FULL, 128)])
+@pytest.mark.parametrize("name,cfg,S", [("t5-small", SMALL, 100), ("t5-long", LONG, 290), ("t5-s128", FULL, 128),
+                                        ("t5-s460", FULL, 460)])
 def test_encdec_parity_against_oracle(name, cfg, S):
     params = wl.init_params(cfg, parity=True, seed=11)
     ctx = make_ctx(cfg)
@@ -69,10 +72,10 @@ def test_encdec_parity_against_oracle(name, cfg, S):
     ctx.close()
 
 
-def test_encdec_recompute_replay_bitwise():
-    cfg = SMALL
+@pytest.mark.parametrize("cfg,S", [(SMALL, 77), (LONG, 250)])
+def test_encdec_recompute_replay_bitwise(cfg, S):
     params = wl.init_params(cfg, parity=True, seed=3)
-    b = wl.make_batch(cfg, 77, seed=7)
+    b = wl.make_batch(cfg, S, seed=7)
     ref = None
     n = cfg.n_layers + cfg.n_dec_layers
     for plan in ([], [0], [2], list(range(n)), [1, 3], [n - 1]):
