@@ -322,7 +322,9 @@ mimose_status mimose_debug_gemm(int32_t epi, int32_t M, int32_t N, int32_t K, co
                                 int64_t a_sk, const void* B, int64_t b_sn, int64_t b_sk, void* C, int64_t ldc,
                                 const void* bias, int32_t split, int32_t use_tc, void* stream);
 /* Same, every epilogue (0 store, 1 bias, 2 bias+GELU -> C, C2, 3 bias+dropout(p=0.1, seed 7)+residual
-   -> fp32 C, 4 GELU' with aux, 5 fp32 C = acc + res, 6 fp32). */
+   -> fp32 C, 4 GELU' with aux, 5 fp32 C = acc + res, 6 fp32, 7 none (benchmark), 8 bias+tanh-GELU
+   -> C, C2, 9 tanh-GELU' with aux, 10 bias+dropout+fp32 residual -> fp32 C, 11 fp32 C += acc);
+   MIMOSE_E_INVALID for any other epi. */
 mimose_status mimose_debug_gemm_ex(int32_t epi, int32_t M, int32_t N, int32_t K, const void* A, int64_t a_sm,
                                    int64_t a_sk, const void* B, int64_t b_sn, int64_t b_sk, void* C, int64_t ldc,
                                    void* C2, const void* bias, const void* res, int64_t ldr, const void* aux,

@@ -2499,7 +2499,7 @@ mimose_status mimose_debug_gemm_ex(int32_t epi, int32_t M, int32_t N, int32_t K,
                                    int64_t a_sk, const void* B, int64_t b_sn, int64_t b_sk, void* Cp, int64_t ldc,
                                    void* C2, const void* bias, const void* res, int64_t ldr, const void* aux,
                                    int64_t ldx, int32_t split, int32_t use_tc, void* stream) {
-  if (epi < 0 || epi > 7) return MIMOSE_E_INVALID;
+  if (epi < 0 || epi > (int)EPI_ACC_F32) return MIMOSE_E_INVALID;
   GemmArgs g;
   g.M = M; g.N = N; g.K = K;
   g.A = A; g.a_sm = a_sm; g.a_sk = a_sk;

@@ -36,72 +36,6 @@ struct TcArgs {
   int kb_total;
 };
 
-// Vectorised epilogue of 32 consecutive columns [n, n+32) of row m (all in range).
-template <int EPI>
-MDEV void epi_row32(const GemmArgs& g, int m, int n, float (&v)[32], int z = -1) {
-  if (z < 0) z = blockIdx.z;
-  using E = __nv_bfloat16;
-  const int64_t o = (int64_t)m * g.ldc + n;
-  if constexpr (EPI == EPI_STORE) {
-    st_bf16x32((E*)g.C + o, v);
-  } else if constexpr (EPI == EPI_BIAS || EPI == EPI_BIAS_GELU || EPI == EPI_BIAS_DROP_RES) {
-    float b[32];
-    ld_bf16x32((const E*)g.bias + n, b);
-#pragma unroll
-    for (int i = 0; i < 32; ++i) v[i] += b[i];
-    if constexpr (EPI == EPI_BIAS) {
-      st_bf16x32((E*)g.C + o, v);
-    } else if constexpr (EPI == EPI_BIAS_GELU) {
-      st_bf16x32((E*)g.C + o, v);
-#pragma unroll
-      for (int i = 0; i < 32; ++i) v[i] = gelu_fast(__bfloat162float(__float2bfloat16_rn(v[i])));
-      st_bf16x32((E*)g.C2 + o, v);
-    } else {
-      float r[32];
-      ld_bf16x32((const E*)g.res + (int64_t)m * g.ldr + n, r);
-      float* out = (float*)g.C + o;
-#pragma unroll
-      for (int q = 0; q < 8; ++q) {
-        const float4 f = drop_factor4(g.drop, (uint64_t)(o + 4 * q) >> 2);
-        float4 w;
-        w.x = r[4 * q + 0] + v[4 * q + 0] * f.x;
-        w.y = r[4 * q + 1] + v[4 * q + 1] * f.y;
-        w.z = r[4 * q + 2] + v[4 * q + 2] * f.z;
-        w.w = r[4 * q + 3] + v[4 * q + 3] * f.w;
-        ((float4*)out)[q] = w;
-      }
-    }
-  } else if constexpr (EPI == EPI_GELU_BWD) {
-    float u[32];
-    ld_bf16x32((const E*)g.aux + (int64_t)m * g.ldx + n, u);
-#pragma unroll
-    for (int i = 0; i < 32; ++i) v[i] *= gelu_grad_fast(u[i]);
-    st_bf16x32((E*)g.C + o, v);
-  } else if constexpr (EPI == EPI_ACC_RES_F32) {
-    const float4* r = (const float4*)((const float*)g.res + (int64_t)m * g.ldr + n);
-    float4* out = (float4*)((float*)g.C + o);
-#pragma unroll
-    for (int q = 0; q < 8; ++q) {
-      const float4 a = r[q];
-      out[q] = make_float4(v[4 * q] + a.x, v[4 * q + 1] + a.y, v[4 * q + 2] + a.z, v[4 * q + 3] + a.w);
-    }
-  } else if constexpr (EPI == EPI_NONE) {
-    float t = 0.f;
-#pragma unroll
-    for (int i = 0; i < 32; ++i) t += v[i];
-    if (t == 1234.5f) ((float*)g.C)[o] = t;
-  } else if constexpr (EPI == EPI_BIAS_GELUT || EPI == EPI_GELUT_BWD || EPI == EPI_BIAS_DROP_RESF32 ||
-                       EPI == EPI_ACC_F32) {
-#pragma unroll
-    for (int i = 0; i < 32; ++i) epilogue<__nv_bfloat16, EPI>(g, m, n + i, v[i], z);
-  } else {
-    float4* out = (float4*)((float*)g.C + (int64_t)z * g.split_stride + o);
-#pragma unroll
-    for (int q = 0; q < 8; ++q) out[q] = make_float4(v[4 * q], v[4 * q + 1], v[4 * q + 2], v[4 * q + 3]);
-  }
-}
-
-
 // ---- coalesced tile stores through a per-warp staging buffer -------------
 // The warp holds a 32 x 32 fragment (lane = row).  It is written to a 32 x 128 B
 // smem buffer with the 16-B chunk index XOR-swizzled by row, then read back so
@@ -158,71 +92,66 @@ MDEV void stage_store_bf16(uint8_t* stg_p, const float (&v)[32], __nv_bfloat16* 
   }
 }
 
-// Epilogue of a 32-row x 32-column fragment (rows m_base + lane, columns n..n+31,
-// all columns in range), stores coalesced through `stg`.
-template <int EPI>
-MDEV void epi_frag32(const GemmArgs& g, int m_base, int n, float (&v)[32], int z, uint8_t* stg, int lane) {
-  using E = __nv_bfloat16;
-  const int m = m_base + lane;
-  const int rows_valid = g.M - m_base;
-  const bool live = m < g.M;
-  if constexpr (EPI == EPI_STORE) {
-    stage_store_bf16(stg, v, (E*)g.C + (int64_t)m_base * g.ldc + n, g.ldc, rows_valid, lane);
-  } else if constexpr (EPI == EPI_BIAS || EPI == EPI_BIAS_GELU || EPI == EPI_BIAS_DROP_RES) {
-    float b[32];
-    ld_bf16x32((const E*)g.bias + n, b);
-#pragma unroll
-    for (int i = 0; i < 32; ++i) v[i] += b[i];
-    if constexpr (EPI == EPI_BIAS) {
-      stage_store_bf16(stg, v, (E*)g.C + (int64_t)m_base * g.ldc + n, g.ldc, rows_valid, lane);
-    } else if constexpr (EPI == EPI_BIAS_GELU) {
-      stage_store_bf16(stg, v, (E*)g.C + (int64_t)m_base * g.ldc + n, g.ldc, rows_valid, lane);
-#pragma unroll
-      for (int i = 0; i < 32; ++i) v[i] = gelu_fast(__bfloat162float(__float2bfloat16_rn(v[i])));
-      stage_store_bf16(stg, v, (E*)g.C2 + (int64_t)m_base * g.ldc + n, g.ldc, rows_valid, lane);
-    } else {
-      float r[32];
-      const int64_t o = (int64_t)m * g.ldc + n;
-      if (live) ld_bf16x32((const E*)g.res + (int64_t)m * g.ldr + n, r);
-#pragma unroll
-      for (int q = 0; q < 8; ++q) {
-        const float4 f = live ? drop_factor4(g.drop, (uint64_t)(o + 4 * q) >> 2) : make_float4(0.f, 0.f, 0.f, 0.f);
-        v[4 * q + 0] = (live ? r[4 * q + 0] : 0.f) + v[4 * q + 0] * f.x;
-        v[4 * q + 1] = (live ? r[4 * q + 1] : 0.f) + v[4 * q + 1] * f.y;
-        v[4 * q + 2] = (live ? r[4 * q + 2] : 0.f) + v[4 * q + 2] * f.z;
-        v[4 * q + 3] = (live ? r[4 * q + 3] : 0.f) + v[4 * q + 3] * f.w;
-      }
-      stage_store_f32(stg, v, (float*)g.C + (int64_t)m_base * g.ldc + n, g.ldc, rows_valid, lane);
-    }
-  } else if constexpr (EPI == EPI_GELU_BWD) {
-    float u[32];
-    if (live) {
-      ld_bf16x32((const E*)g.aux + (int64_t)m * g.ldx + n, u);
-#pragma unroll
-      for (int i = 0; i < 32; ++i) v[i] *= gelu_grad_fast(u[i]);
-    }
-    stage_store_bf16(stg, v, (E*)g.C + (int64_t)m_base * g.ldc + n, g.ldc, rows_valid, lane);
-  } else if constexpr (EPI == EPI_ACC_RES_F32) {
-    if (live) {
-      const float4* r = (const float4*)((const float*)g.res + (int64_t)m * g.ldr + n);
-#pragma unroll
-      for (int q = 0; q < 8; ++q) {
-        const float4 a = r[q];
-        v[4 * q] += a.x; v[4 * q + 1] += a.y; v[4 * q + 2] += a.z; v[4 * q + 3] += a.w;
-      }
-    }
-    stage_store_f32(stg, v, (float*)g.C + (int64_t)m_base * g.ldc + n, g.ldc, rows_valid, lane);
-  } else if constexpr (EPI == EPI_NONE) {
-    float t = 0.f;
-#pragma unroll
-    for (int i = 0; i < 32; ++i) t += v[i];
-    if (t == 1234.5f) ((float*)g.C)[0] = t;
-  } else {
-    stage_store_f32(stg, v, (float*)g.C + (int64_t)z * g.split_stride + (int64_t)m_base * g.ldc + n, g.ldc,
-                    rows_valid, lane);
-  }
-}
 
+// ---- TMA (bulk tensor) stores: the warp writes its 32 x 32 fragment into its
+// staging buffer in the tensor map's swizzled layout and one lane issues
+// cp.async.bulk.tensor (global <- shared); the TMA unit writes whole lines and
+// clips rows >= M, and the warp does not wait for the write.  bf16 fragments
+// (64-B rows, SWIZZLE_64B: 16-B chunk ^= (row / 2) % 4) alternate between the
+// two 2 KB halves of the buffer; fp32 fragments (128-B rows, SWIZZLE_128B:
+// chunk ^= row % 8) use all 4 KB.  Before a half is rewritten, the bulk group
+// that last read it must have finished reading (wait_group.read).
+struct EpiOut {
+  uint8_t* stg;             // this warp's 4 KB staging buffer (1024-B aligned)
+  const CUtensorMap* mc;    // map of C (TMA mode)
+  const CUtensorMap* mc2;   // map of C2 (TMA mode, GELU epilogues)
+  int half;                 // next bf16 half
+};
+template <int N>
+MDEV void bulk_wait_read() { asm volatile("cp.async.bulk.wait_group.read %0;" ::"n"(N) : "memory"); }
+MDEV void bulk_wait_all() { asm volatile("cp.async.bulk.wait_group 0;" ::: "memory"); }
+MDEV void tma_store_2d(const CUtensorMap* map, uint32_t src, int c0, int c1) {
+  asm volatile("cp.async.bulk.tensor.2d.global.shared::cta.bulk_group [%0, {%2, %3}], [%1];"
+               ::"l"(map), "r"(src), "r"(c0), "r"(c1) : "memory");
+  asm volatile("cp.async.bulk.commit_group;" ::: "memory");
+}
+MDEV void tma_out_bf16(EpiOut& o, const float (&v)[32], const CUtensorMap* map, int n, int m_base, int lane) {
+  const uint32_t s = smem_u32(o.stg) + 2048u * (uint32_t)o.half;
+  o.half ^= 1;
+  if (lane == 0) bulk_wait_read<1>();    // the group before last used this half
+  __syncwarp();
+#pragma unroll
+  for (int c = 0; c < 4; ++c) sts128(s + lane * 64 + ((c ^ ((lane >> 1) & 3)) << 4), pack8(v + 8 * c));
+  fence_async_smem();
+  __syncwarp();
+  if (lane == 0) tma_store_2d(map, s, n, m_base);
+}
+MDEV void tma_out_f32(EpiOut& o, const float (&v)[32], const CUtensorMap* map, int n, int m_base, int lane) {
+  const uint32_t s = smem_u32(o.stg);
+  if (lane == 0) bulk_wait_read<0>();
+  __syncwarp();
+#pragma unroll
+  for (int c = 0; c < 8; ++c)
+    sts128(s + lane * 128 + ((c ^ (lane & 7)) << 4),
+           make_uint4(__float_as_uint(v[4 * c]), __float_as_uint(v[4 * c + 1]), __float_as_uint(v[4 * c + 2]),
+                      __float_as_uint(v[4 * c + 3])));
+  fence_async_smem();
+  __syncwarp();
+  if (lane == 0) tma_store_2d(map, s, n, m_base);
+}
+// Output of one fragment: TMA (ST = 1) or LSU stores through the staging buffer (ST = 0).
+template <int ST>
+MDEV void out_bf16(EpiOut& o, const float (&v)[32], __nv_bfloat16* base, int64_t ld, const CUtensorMap* map, int n,
+                   int m_base, int rows_valid, int lane) {
+  if constexpr (ST == 1) tma_out_bf16(o, v, map, n, m_base, lane);
+  else stage_store_bf16(o.stg, v, base + (int64_t)m_base * ld + n, ld, rows_valid, lane);
+}
+template <int ST>
+MDEV void out_f32(EpiOut& o, const float (&v)[32], float* base, int64_t ld, const CUtensorMap* map, int n, int m_base,
+                  int rows_valid, int lane) {
+  if constexpr (ST == 1) tma_out_f32(o, v, map, n, m_base, lane);
+  else stage_store_f32(o.stg, v, base + (int64_t)m_base * ld + n, ld, rows_valid, lane);
+}
 
 // Epilogue inputs of one 32-column chunk, loaded one chunk ahead (software
 // pipelining hides the L2 latency of bias / u / residual behind the previous
@@ -280,15 +209,15 @@ MDEV void epi_load(const GemmArgs& g, int m, int n, bool live, EpiIn& in) {
   }
 }
 
-template <int EPI>
-MDEV void epi_frag32_in(const GemmArgs& g, int m_base, int n, float (&v)[32], int z, uint8_t* stg, int lane,
+template <int EPI, int ST>
+MDEV void epi_frag32_in(const GemmArgs& g, int m_base, int n, float (&v)[32], int z, EpiOut& o, int lane,
                         const EpiIn& in, uint32_t keep) {
   using E = __nv_bfloat16;
   const int m = m_base + lane;
   const int rows_valid = g.M - m_base;
   const bool live = m < g.M;
   if constexpr (EPI == EPI_STORE) {
-    stage_store_bf16(stg, v, (E*)g.C + (int64_t)m_base * g.ldc + n, g.ldc, rows_valid, lane);
+    out_bf16<ST>(o, v, (E*)g.C, g.ldc, o.mc, n, m_base, rows_valid, lane);
   } else if constexpr (EPI == EPI_BIAS || EPI == EPI_BIAS_GELU || EPI == EPI_BIAS_DROP_RES) {
     float b[32];
 #pragma unroll
@@ -300,9 +229,9 @@ MDEV void epi_frag32_in(const GemmArgs& g, int m_base, int n, float (&v)[32], in
       v[i + 1] = r.y;
     }
     if constexpr (EPI == EPI_BIAS) {
-      stage_store_bf16(stg, v, (E*)g.C + (int64_t)m_base * g.ldc + n, g.ldc, rows_valid, lane);
+      out_bf16<ST>(o, v, (E*)g.C, g.ldc, o.mc, n, m_base, rows_valid, lane);
     } else if constexpr (EPI == EPI_BIAS_GELU) {
-      stage_store_bf16(stg, v, (E*)g.C + (int64_t)m_base * g.ldc + n, g.ldc, rows_valid, lane);
+      out_bf16<ST>(o, v, (E*)g.C, g.ldc, o.mc, n, m_base, rows_valid, lane);
 #pragma unroll
       for (int i = 0; i < 32; i += 2) {
         const float2 r = gelu_fast_x2(make_float2(__bfloat162float(__float2bfloat16_rn(v[i])),
@@ -310,7 +239,7 @@ MDEV void epi_frag32_in(const GemmArgs& g, int m_base, int n, float (&v)[32], in
         v[i] = r.x;
         v[i + 1] = r.y;
       }
-      stage_store_bf16(stg, v, (E*)g.C2 + (int64_t)m_base * g.ldc + n, g.ldc, rows_valid, lane);
+      out_bf16<ST>(o, v, (E*)g.C2, g.ldc, o.mc2, n, m_base, rows_valid, lane);
     } else {
       float r[32];
 #pragma unroll
@@ -323,7 +252,7 @@ MDEV void epi_frag32_in(const GemmArgs& g, int m_base, int n, float (&v)[32], in
         v[4 * q + 2] = (live ? r[4 * q + 2] : 0.f) + v[4 * q + 2] * f.z;
         v[4 * q + 3] = (live ? r[4 * q + 3] : 0.f) + v[4 * q + 3] * f.w;
       }
-      stage_store_f32(stg, v, (float*)g.C + (int64_t)m_base * g.ldc + n, g.ldc, rows_valid, lane);
+      out_f32<ST>(o, v, (float*)g.C, g.ldc, o.mc, n, m_base, rows_valid, lane);
     }
   } else if constexpr (EPI == EPI_GELU_BWD) {
     float u[32];
@@ -335,7 +264,7 @@ MDEV void epi_frag32_in(const GemmArgs& g, int m_base, int n, float (&v)[32], in
       v[i] = r.x;
       v[i + 1] = r.y;
     }
-    stage_store_bf16(stg, v, (E*)g.C + (int64_t)m_base * g.ldc + n, g.ldc, rows_valid, lane);
+    out_bf16<ST>(o, v, (E*)g.C, g.ldc, o.mc, n, m_base, rows_valid, lane);
   } else if constexpr (EPI == EPI_ACC_RES_F32) {
     if (live) {
       const float4* r = (const float4*)in.x;
@@ -345,7 +274,7 @@ MDEV void epi_frag32_in(const GemmArgs& g, int m_base, int n, float (&v)[32], in
         v[4 * q] += a.x; v[4 * q + 1] += a.y; v[4 * q + 2] += a.z; v[4 * q + 3] += a.w;
       }
     }
-    stage_store_f32(stg, v, (float*)g.C + (int64_t)m_base * g.ldc + n, g.ldc, rows_valid, lane);
+    out_f32<ST>(o, v, (float*)g.C, g.ldc, o.mc, n, m_base, rows_valid, lane);
   } else if constexpr (EPI == EPI_BIAS_GELUT || EPI == EPI_BIAS_DROP_RESF32) {
     float b[32];
 #pragma unroll
@@ -353,10 +282,10 @@ MDEV void epi_frag32_in(const GemmArgs& g, int m_base, int n, float (&v)[32], in
 #pragma unroll
     for (int i = 0; i < 32; ++i) v[i] += b[i];
     if constexpr (EPI == EPI_BIAS_GELUT) {
-      stage_store_bf16(stg, v, (E*)g.C + (int64_t)m_base * g.ldc + n, g.ldc, rows_valid, lane);
+      out_bf16<ST>(o, v, (E*)g.C, g.ldc, o.mc, n, m_base, rows_valid, lane);
 #pragma unroll
       for (int i = 0; i < 32; ++i) v[i] = gelu_fast(__bfloat162float(__float2bfloat16_rn(v[i])));   // gelu_new == the tanh form
-      stage_store_bf16(stg, v, (E*)g.C2 + (int64_t)m_base * g.ldc + n, g.ldc, rows_valid, lane);
+      out_bf16<ST>(o, v, (E*)g.C2, g.ldc, o.mc2, n, m_base, rows_valid, lane);
     } else {
       const float* r = (const float*)in.x;
 #pragma unroll
@@ -367,7 +296,7 @@ MDEV void epi_frag32_in(const GemmArgs& g, int m_base, int n, float (&v)[32], in
         v[4 * q + 2] = (live ? r[4 * q + 2] : 0.f) + v[4 * q + 2] * f.z;
         v[4 * q + 3] = (live ? r[4 * q + 3] : 0.f) + v[4 * q + 3] * f.w;
       }
-      stage_store_f32(stg, v, (float*)g.C + (int64_t)m_base * g.ldc + n, g.ldc, rows_valid, lane);
+      out_f32<ST>(o, v, (float*)g.C, g.ldc, o.mc, n, m_base, rows_valid, lane);
     }
   } else if constexpr (EPI == EPI_GELUT_BWD) {
     float u[32];
@@ -375,7 +304,7 @@ MDEV void epi_frag32_in(const GemmArgs& g, int m_base, int n, float (&v)[32], in
     for (int i = 0; i < 4; ++i) unpack8(in.x[i], u + 8 * i);
 #pragma unroll
     for (int i = 0; i < 32; ++i) v[i] *= gelu_grad_fast(u[i]);
-    stage_store_bf16(stg, v, (E*)g.C + (int64_t)m_base * g.ldc + n, g.ldc, rows_valid, lane);
+    out_bf16<ST>(o, v, (E*)g.C, g.ldc, o.mc, n, m_base, rows_valid, lane);
   } else if constexpr (EPI == EPI_ACC_F32) {
     if (live) {
       float* out = (float*)g.C + (int64_t)m * g.ldc + n;
@@ -392,21 +321,21 @@ MDEV void epi_frag32_in(const GemmArgs& g, int m_base, int n, float (&v)[32], in
     for (int i = 0; i < 32; ++i) t += v[i];
     if (t == 1234.5f) ((float*)g.C)[0] = t;
   } else {
-    stage_store_f32(stg, v, (float*)g.C + (int64_t)z * g.split_stride + (int64_t)m_base * g.ldc + n, g.ldc,
-                    rows_valid, lane);
+    out_f32<ST>(o, v, (float*)g.C + (int64_t)z * g.split_stride, g.ldc, o.mc, n, m_base, rows_valid, lane);   // TMA: split 1
   }
 }
 
 constexpr int TP_EPI_WARPS = 8;
 constexpr int TP_THREADS = 64 + 32 * TP_EPI_WARPS;
 
-template <int BN>
+template <int BN, int ST>
 struct TpCfg {
   static constexpr int STAGES = BN >= 256 ? 4 : (BN >= 128 ? 6 : 8);
   static constexpr int A_BYTES = TBM * TBK * 2;
   static constexpr int B_BYTES = BN * TBK * 2;
   static constexpr int STAGE_BYTES = A_BYTES + B_BYTES;
-  static constexpr int STG_BYTES = TP_EPI_WARPS * 4096;   // per-warp 32 x 128 B store staging
+  static constexpr int STG_PER = 4096;   // per-warp store staging (1024-B aligned: TMA swizzle atoms)
+  static constexpr int STG_BYTES = TP_EPI_WARPS * STG_PER;
   static constexpr int SMEM = STAGES * STAGE_BYTES + STG_BYTES + 1024 + 256;
 };
 
@@ -446,21 +375,22 @@ MDEV bool seg_of2(const TpArgs& a, const TpArgs& a2, int i, Seg& s) {
     return true;
   }
 }
-template <int BN, int EPI, bool G2>
+template <int BN, int EPI, bool G2, int ST>
 __global__ void __launch_bounds__(TP_THREADS, 1)
     k_gemm_tcp(const __grid_constant__ CUtensorMap tma_a, const __grid_constant__ CUtensorMap tma_b, const TpArgs args,
                const __grid_constant__ CUtensorMap tma_a2, const __grid_constant__ CUtensorMap tma_b2,
-               const TpArgs args2) {
+               const TpArgs args2, const __grid_constant__ CUtensorMap tma_c,
+               const __grid_constant__ CUtensorMap tma_c2) {
   pdl_trigger();
-  using Cf = TpCfg<BN>;
+  using Cf = TpCfg<BN, ST>;
   extern __shared__ uint8_t smem_raw[];
   uint8_t* smem = (uint8_t*)(((uintptr_t)smem_raw + 1023) & ~(uintptr_t)1023);
-  uint64_t* full = (uint64_t*)(smem + Cf::STAGES * Cf::STAGE_BYTES);
+  uint8_t* stg_base = smem + Cf::STAGES * Cf::STAGE_BYTES;
+  uint64_t* full = (uint64_t*)(stg_base + Cf::STG_BYTES);
   uint64_t* empty = full + Cf::STAGES;
   uint64_t* tfull = empty + Cf::STAGES;    // [2]
   uint64_t* tempty = tfull + 2;            // [2]
   uint32_t* tmem_slot = (uint32_t*)(tempty + 2);
-  uint8_t* stg_base = smem + Cf::STAGES * Cf::STAGE_BYTES + 256;
   const TcArgs& ta = args.t;
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
 
@@ -554,6 +484,7 @@ __global__ void __launch_bounds__(TP_THREADS, 1)
     }
   } else {                                             // ---------------- epilogue warps
     const int e = warp - 2;
+    EpiOut eo{stg_base + e * Cf::STG_PER, &tma_c, &tma_c2, 0};
     const int q = warp & 3;                            // TMEM lane quarter of this warp
     const int grp = e >> 2, ngrp = TP_EPI_WARPS / 4;  // column group of this warp
     int local = 0;
@@ -561,6 +492,7 @@ __global__ void __launch_bounds__(TP_THREADS, 1)
     for (; seg_of2<G2>(args, args2, local, sg); ++local) {
       const TpArgs& A = (G2 && sg.p) ? args2 : args;
       const GemmArgs& g = A.t.g;
+      if constexpr (G2) eo.mc = sg.p ? &tma_c2 : &tma_c;
       const int z = sg.z, r = sg.r;
       const int m0 = (r / A.n_blocks) * TBM, n0 = (r % A.n_blocks) * BN;
       const int kb0 = sg.kb0, kb1 = sg.kb1;
@@ -612,7 +544,7 @@ __global__ void __launch_bounds__(TP_THREADS, 1)
           for (int i = 0; i < 32; ++i) v[i] = 0.f;
         }
         if (n + 32 <= g.N) {
-          if (m0 + 32 * q < g.M) epi_frag32_in<EPI>(g, m0 + 32 * q, n, v, z, stg_base + e * 4096, lane, cur, keep);
+          if (m0 + 32 * q < g.M) epi_frag32_in<EPI, ST>(g, m0 + 32 * q, n, v, z, eo, lane, cur, keep);
         } else if (m < g.M) {
 #pragma unroll
           for (int i = 0; i < 32; ++i)
@@ -622,6 +554,9 @@ __global__ void __launch_bounds__(TP_THREADS, 1)
       tc_fence_before();
       __syncwarp();
       if (lane == 0) asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_u32(&tempty[acc])) : "memory");
+    }
+    if constexpr (ST == 1) {
+      if (lane == 0) bulk_wait_all();   // the bulk stores have completed before the CTA exits
     }
   }
   tc_fence_before();
@@ -654,38 +589,42 @@ struct MapKey {
   const void* ptr;
   uint64_t inner, outer, stride;
   uint32_t box_inner, box_outer;
+  int f32, swz;
   bool operator==(const MapKey& o) const {
     return ptr == o.ptr && inner == o.inner && outer == o.outer && stride == o.stride &&
-           box_inner == o.box_inner && box_outer == o.box_outer;
+           box_inner == o.box_inner && box_outer == o.box_outer && f32 == o.f32 && swz == o.swz;
   }
 };
 struct MapKeyHash {
   size_t operator()(const MapKey& k) const {
     size_t h = std::hash<const void*>()(k.ptr);
-    for (uint64_t v : {k.inner, k.outer, k.stride, (uint64_t)k.box_inner << 32 | k.box_outer})
+    for (uint64_t v : {k.inner, k.outer, k.stride, (uint64_t)k.box_inner << 32 | k.box_outer,
+                       (uint64_t)k.f32 << 8 | (uint64_t)k.swz})
       h ^= std::hash<uint64_t>()(v) + 0x9e3779b97f4a7c15ull + (h << 6) + (h >> 2);
     return h;
   }
 };
 
-// 2D bf16 tensor [outer][inner] (inner contiguous), row stride in elements.
+// 2D bf16 (or fp32) tensor [outer][inner] (inner contiguous), row stride in
+// elements; swizzle 128B (operand tiles, fp32 store tiles) or 64B (bf16 store tiles).
 static bool make_map(CUtensorMap* out, const void* ptr, uint64_t inner, uint64_t outer, uint64_t stride_elems,
-                     uint32_t box_inner, uint32_t box_outer) {
+                     uint32_t box_inner, uint32_t box_outer, int f32 = 0, int swz = 128) {
   static std::unordered_map<MapKey, CUtensorMap, MapKeyHash> cache;
   static std::mutex mu;
-  MapKey key{ptr, inner, outer, stride_elems, box_inner, box_outer};
+  MapKey key{ptr, inner, outer, stride_elems, box_inner, box_outer, f32, swz};
   std::lock_guard<std::mutex> lk(mu);
   auto it = cache.find(key);
   if (it != cache.end()) { *out = it->second; return true; }
   EncodeFn fn = encode_fn();
   if (!fn) return false;
   cuuint64_t dims[2] = {inner, outer};
-  cuuint64_t strides[1] = {stride_elems * 2};
+  cuuint64_t strides[1] = {stride_elems * (f32 ? 4 : 2)};
   cuuint32_t box[2] = {box_inner, box_outer};
   cuuint32_t es[2] = {1, 1};
-  CUresult r = fn(out, CU_TENSOR_MAP_DATA_TYPE_BFLOAT16, 2, const_cast<void*>(ptr), dims, strides, box, es,
-                  CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
-                  CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+  CUresult r = fn(out, f32 ? CU_TENSOR_MAP_DATA_TYPE_FLOAT32 : CU_TENSOR_MAP_DATA_TYPE_BFLOAT16, 2,
+                  const_cast<void*>(ptr), dims, strides, box, es, CU_TENSOR_MAP_INTERLEAVE_NONE,
+                  swz == 64 ? CU_TENSOR_MAP_SWIZZLE_64B : CU_TENSOR_MAP_SWIZZLE_128B,
+                  CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
   if (r != CUDA_SUCCESS) return false;
   if (cache.size() > 8192) cache.clear();
   cache.emplace(key, *out);
@@ -699,51 +638,53 @@ bool tc_map_bf16(CUtensorMap* out, const void* ptr, uint64_t inner, uint64_t out
 
 static int num_sms();
 
-template <int BN, int EPI>
-static void launch_tcp(const CUtensorMap& ma, const CUtensorMap& mb, const TpArgs& a, cudaStream_t st) {
+template <int BN, int EPI, int ST>
+static void launch_tcp(const CUtensorMap& ma, const CUtensorMap& mb, const TpArgs& a, const CUtensorMap& mc,
+                       const CUtensorMap& mc2, cudaStream_t st) {
   static bool attr = false;
   if (!attr) {
-    cudaFuncSetAttribute(k_gemm_tcp<BN, EPI, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, TpCfg<BN>::SMEM);
+    cudaFuncSetAttribute(k_gemm_tcp<BN, EPI, false, ST>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                         TpCfg<BN, ST>::SMEM);
     attr = true;
   }
-  static int nsm = 0;
-  if (!nsm) {
-    int dev;
-    cudaGetDevice(&dev);
-    cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, dev);
-  }
-  launch_k(k_gemm_tcp<BN, EPI, false>, std::min(nsm, a.n_tiles), TP_THREADS, TpCfg<BN>::SMEM, st, ma, mb, a, ma, mb, a);
+  launch_k(k_gemm_tcp<BN, EPI, false, ST>, std::min(num_sms(), a.n_tiles), TP_THREADS, TpCfg<BN, ST>::SMEM, st, ma,
+           mb, a, ma, mb, a, mc, mc2);
 }
 
-// Two independent EPI_F32 problems in one persistent launch (grouped wgrad).
-template <int BN>
+// Two independent EPI_F32 problems in one persistent launch (grouped wgrad);
+// mc / mc2: the two problems' C maps (TMA stores).
+template <int BN, int ST>
 static void launch_tcp_g2(const CUtensorMap& ma, const CUtensorMap& mb, const TpArgs& a, const CUtensorMap& ma2,
-                          const CUtensorMap& mb2, const TpArgs& a2, cudaStream_t st) {
+                          const CUtensorMap& mb2, const TpArgs& a2, const CUtensorMap& mc, const CUtensorMap& mc2,
+                          cudaStream_t st) {
   static bool attr = false;
   if (!attr) {
-    cudaFuncSetAttribute(k_gemm_tcp<BN, EPI_F32, true>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                         TpCfg<BN>::SMEM);
+    cudaFuncSetAttribute(k_gemm_tcp<BN, EPI_F32, true, ST>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                         TpCfg<BN, ST>::SMEM);
     attr = true;
   }
-  launch_k(k_gemm_tcp<BN, EPI_F32, true>, std::min(num_sms(), a.n_tiles + a2.n_tiles), TP_THREADS,
-           TpCfg<BN>::SMEM, st, ma, mb, a, ma2, mb2, a2);
+  launch_k(k_gemm_tcp<BN, EPI_F32, true, ST>, std::min(num_sms(), a.n_tiles + a2.n_tiles), TP_THREADS,
+           TpCfg<BN, ST>::SMEM, st, ma, mb, a, ma2, mb2, a2, mc, mc2);
 }
 
-template <int BN>
-static void dispatch_tcp(Epi epi, const CUtensorMap& ma, const CUtensorMap& mb, const TpArgs& a, cudaStream_t st) {
+// ST = 1 (TMA stores) for every epilogue that overwrites its output; the
+// read-modify-write EPI_ACC_F32 and the benchmark EPI_NONE keep LSU stores.
+template <int BN, int ST>
+static void dispatch_tcp(Epi epi, const CUtensorMap& ma, const CUtensorMap& mb, const TpArgs& a,
+                         const CUtensorMap& mc, const CUtensorMap& mc2, cudaStream_t st) {
   switch (epi) {
-    case EPI_STORE: launch_tcp<BN, EPI_STORE>(ma, mb, a, st); break;
-    case EPI_BIAS: launch_tcp<BN, EPI_BIAS>(ma, mb, a, st); break;
-    case EPI_BIAS_GELU: launch_tcp<BN, EPI_BIAS_GELU>(ma, mb, a, st); break;
-    case EPI_BIAS_DROP_RES: launch_tcp<BN, EPI_BIAS_DROP_RES>(ma, mb, a, st); break;
-    case EPI_GELU_BWD: launch_tcp<BN, EPI_GELU_BWD>(ma, mb, a, st); break;
-    case EPI_ACC_RES_F32: launch_tcp<BN, EPI_ACC_RES_F32>(ma, mb, a, st); break;
-    case EPI_NONE: launch_tcp<BN, EPI_NONE>(ma, mb, a, st); break;
-    case EPI_BIAS_GELUT: launch_tcp<BN, EPI_BIAS_GELUT>(ma, mb, a, st); break;
-    case EPI_GELUT_BWD: launch_tcp<BN, EPI_GELUT_BWD>(ma, mb, a, st); break;
-    case EPI_BIAS_DROP_RESF32: launch_tcp<BN, EPI_BIAS_DROP_RESF32>(ma, mb, a, st); break;
-    case EPI_ACC_F32: launch_tcp<BN, EPI_ACC_F32>(ma, mb, a, st); break;
-    default: launch_tcp<BN, EPI_F32>(ma, mb, a, st); break;
+    case EPI_STORE: launch_tcp<BN, EPI_STORE, ST>(ma, mb, a, mc, mc2, st); break;
+    case EPI_BIAS: launch_tcp<BN, EPI_BIAS, ST>(ma, mb, a, mc, mc2, st); break;
+    case EPI_BIAS_GELU: launch_tcp<BN, EPI_BIAS_GELU, ST>(ma, mb, a, mc, mc2, st); break;
+    case EPI_BIAS_DROP_RES: launch_tcp<BN, EPI_BIAS_DROP_RES, ST>(ma, mb, a, mc, mc2, st); break;
+    case EPI_GELU_BWD: launch_tcp<BN, EPI_GELU_BWD, ST>(ma, mb, a, mc, mc2, st); break;
+    case EPI_ACC_RES_F32: launch_tcp<BN, EPI_ACC_RES_F32, ST>(ma, mb, a, mc, mc2, st); break;
+    case EPI_NONE: launch_tcp<BN, EPI_NONE, 0>(ma, mb, a, mc, mc2, st); break;
+    case EPI_BIAS_GELUT: launch_tcp<BN, EPI_BIAS_GELUT, ST>(ma, mb, a, mc, mc2, st); break;
+    case EPI_GELUT_BWD: launch_tcp<BN, EPI_GELUT_BWD, ST>(ma, mb, a, mc, mc2, st); break;
+    case EPI_BIAS_DROP_RESF32: launch_tcp<BN, EPI_BIAS_DROP_RESF32, ST>(ma, mb, a, mc, mc2, st); break;
+    case EPI_ACC_F32: launch_tcp<BN, EPI_ACC_F32, 0>(ma, mb, a, mc, mc2, st); break;
+    default: launch_tcp<BN, EPI_F32, ST>(ma, mb, a, mc, mc2, st); break;
   }
 }
 
@@ -758,10 +699,28 @@ static int num_sms() {
   return nsm;
 }
 
-static int g_gemm_mode = 1;   // 1: default; 12: force 128 x 256 tiles and no grouped launches (test hook)
+static int g_gemm_mode = 1;   // 1: default; 12: force 128 x 256 tiles and no grouped launches; 15: LSU-store epilogues instead of TMA stores (test hooks)
 void set_gemm_mode(int m) { g_gemm_mode = m; }
 
 bool tc_available() { return encode_fn() != nullptr; }
+
+// Output maps of the TMA-store epilogue: 32 x 32 boxes of C / C2 (bf16 with
+// 64-B rows and SWIZZLE_64B, fp32 with 128-B rows and SWIZZLE_128B).
+static bool epi_out_f32(Epi e) {
+  return e == EPI_BIAS_DROP_RES || e == EPI_ACC_RES_F32 || e == EPI_F32 || e == EPI_BIAS_DROP_RESF32;
+}
+static bool out_map(CUtensorMap* m, const void* ptr, int M, int N, int64_t ld, bool f32) {
+  if (!ptr || ((uintptr_t)ptr & 15) || (ld * (f32 ? 4 : 2)) % 16) return false;
+  return make_map(m, ptr, (uint64_t)N, (uint64_t)M, (uint64_t)ld, 32, 32, f32 ? 1 : 0, f32 ? 128 : 64);
+}
+static bool tma_store_ok(Epi epi, const GemmArgs& g, CUtensorMap* mc, CUtensorMap* mc2) {
+  if (g_gemm_mode == 15 || g.split != 1 || epi == EPI_ACC_F32 || epi == EPI_NONE) return false;
+  const bool f32 = epi_out_f32(epi);
+  if (!out_map(mc, g.C, g.M, g.N, g.ldc, f32)) return false;
+  if (epi == EPI_BIAS_GELU || epi == EPI_BIAS_GELUT) return out_map(mc2, g.C2, g.M, g.N, g.ldc, false);
+  *mc2 = *mc;
+  return true;
+}
 
 bool gemm_tc(Epi epi, const GemmArgs& g, cudaStream_t st) {
   TcArgs a;
@@ -806,8 +765,14 @@ bool gemm_tc(Epi epi, const GemmArgs& g, cudaStream_t st) {
   p.m_blocks = m_blocks;
   p.n_blocks = (g.N + BN - 1) / BN;
   p.n_tiles = p.m_blocks * p.n_blocks * g.split;
-  if (BN == 256) dispatch_tcp<256>(epi, ma, mb, p, st);
-  else dispatch_tcp<128>(epi, ma, mb, p, st);
+  CUtensorMap mc, mc2;
+  if (tma_store_ok(epi, g, &mc, &mc2)) {
+    if (BN == 256) dispatch_tcp<256, 1>(epi, ma, mb, p, mc, mc2, st);
+    else dispatch_tcp<128, 1>(epi, ma, mb, p, mc, mc2, st);
+  } else {
+    if (BN == 256) dispatch_tcp<256, 0>(epi, ma, mb, p, ma, ma, st);
+    else dispatch_tcp<128, 0>(epi, ma, mb, p, ma, ma, st);
+  }
   return true;
 }
 
@@ -818,7 +783,7 @@ bool gemm_tc(Epi epi, const GemmArgs& g, cudaStream_t st) {
 // tile's K loop is the same as in a single launch, so results are bitwise
 // equal to two separate launches with the same tile width.
 bool gemm_tc_grouped(const GemmArgs& g1, const GemmArgs& g2, int bn, cudaStream_t st) {
-  if (g_gemm_mode != 1 || g1.split != 1 || g2.split != 1) return false;
+  if ((g_gemm_mode != 1 && g_gemm_mode != 15) || g1.split != 1 || g2.split != 1) return false;
   if (bn != 128 && bn != 256) return false;
   TpArgs p[2];
   CUtensorMap ma[2], mb[2];
@@ -845,8 +810,15 @@ bool gemm_tc_grouped(const GemmArgs& g1, const GemmArgs& g2, int bn, cudaStream_
     p[i].n_tiles = p[i].m_blocks * p[i].n_blocks;
   }
   if (p[0].n_tiles + p[1].n_tiles > num_sms()) return false;   // grouping pays only within one wave
-  if (bn == 256) launch_tcp_g2<256>(ma[0], mb[0], p[0], ma[1], mb[1], p[1], st);
-  else launch_tcp_g2<128>(ma[0], mb[0], p[0], ma[1], mb[1], p[1], st);
+  CUtensorMap mc[2];
+  if (g_gemm_mode != 15 && out_map(&mc[0], g1.C, g1.M, g1.N, g1.ldc, true) &&
+      out_map(&mc[1], g2.C, g2.M, g2.N, g2.ldc, true)) {
+    if (bn == 256) launch_tcp_g2<256, 1>(ma[0], mb[0], p[0], ma[1], mb[1], p[1], mc[0], mc[1], st);
+    else launch_tcp_g2<128, 1>(ma[0], mb[0], p[0], ma[1], mb[1], p[1], mc[0], mc[1], st);
+  } else {
+    if (bn == 256) launch_tcp_g2<256, 0>(ma[0], mb[0], p[0], ma[1], mb[1], p[1], ma[0], ma[0], st);
+    else launch_tcp_g2<128, 0>(ma[0], mb[0], p[0], ma[1], mb[1], p[1], ma[0], ma[0], st);
+  }
   return true;
 }
 

@@ -30,7 +30,7 @@ def operands(M, N, K, a_mn, b_mn, seed=0):
 SHAPES += [(2048, 3072, 768), (512, 768, 3072), (4096, 2304, 768)]   # BN=256 persistent tiles
 
 
-@pytest.fixture(params=[1, 12], ids=["persistent", "persistent-bn256"])
+@pytest.fixture(params=[1, 12, 15], ids=["persistent", "persistent-bn256", "persistent-lsu-store"])
 def gemm_mode(request):
     mb().debug_options(gemm_mode=request.param)
     yield request.param
@@ -108,9 +108,10 @@ def test_gemm_gelu_epilogues(shape, gemm_mode):
     assert err < 1e-2, err
 
 
+@pytest.mark.parametrize("mode", [1, 15])
 @pytest.mark.parametrize("pair", [((768, 3072, 5120), (3072, 768, 5120)), ((768, 3072, 1000), (3072, 768, 1000)),
                                   ((296, 512, 136), (1000, 256, 136))])
-def test_gemm_grouped_wgrad(pair):
+def test_gemm_grouped_wgrad(pair, mode):
     """Two wgrad-shaped (TN) fp32 GEMMs in one grouped launch are bitwise equal
     to the same problems launched alone with the same 128 x 256 tiles."""
     outs, refs = [], []
@@ -120,6 +121,7 @@ def test_gemm_grouped_wgrad(pair):
         ops.append((M, N, K, As, a_sm, a_sk, Bs, b_sn, b_sk))
         refs.append(A.float() @ B.float().t())
     C = [torch.full((o[0], o[1]), float("nan"), device="cuda") for o in ops]
+    mb().debug_options(gemm_mode=mode)
     mb().debug_gemm_grouped(ops[0], C[0], ops[1], C[1])
     torch.cuda.synchronize()
     mb().debug_options(gemm_mode=12)          # separate persistent launches, 256-wide tiles
@@ -133,3 +135,44 @@ def test_gemm_grouped_wgrad(pair):
             assert ((c - ref).abs().max() / ref.abs().max()).item() < 1e-5
     finally:
         mb().debug_options(gemm_mode=1)
+
+
+@pytest.mark.parametrize("epi", [0, 1, 2, 3, 4, 5, 6, 8, 9, 10])
+@pytest.mark.parametrize("shape", [(300, 776, 136), (2100, 3072, 768), (1000, 768, 3072)])
+def test_tma_store_epilogues_bitwise(epi, shape):
+    """The TMA-store epilogue (default: fragments written through swizzled smem
+    by cp.async.bulk.tensor, rows >= M clipped by the unit) stores exactly what
+    the LSU-store epilogue (gemm mode 15) stores, for every epilogue, with ragged M and
+    an N tail (776 = 24 full 32-column chunks + 8 columns on the scalar path)."""
+    M, N, K = shape
+    A, B, As, Bs, a_sm, a_sk, b_sn, b_sk = operands(M, N, K, 0, 0, seed=30 + epi)
+    bf, f32 = torch.bfloat16, torch.float32
+    out_f32 = epi in (3, 5, 6, 10)
+    g = torch.Generator(device="cuda").manual_seed(7)
+    bias = torch.randn(N, device="cuda", generator=g).to(bf)
+    res = torch.randn(M, N, device="cuda", generator=g)
+    aux = torch.randn(M, N, device="cuda", generator=g).to(bf)
+    outs = []
+    for mode in (15, 1):
+        C = torch.full((M, N), float("nan"), device="cuda", dtype=f32 if out_f32 else bf)
+        C2 = torch.full((M, N), float("nan"), device="cuda", dtype=bf)
+        kw = dict(bias=bias)
+        if epi in (2, 8):
+            kw["C2"] = C2
+        if epi == 3:
+            kw.update(res=res.to(bf), ldr=N)
+        if epi in (5, 10):
+            kw.update(res=res, ldr=N)
+        if epi in (4, 9):
+            kw.update(aux=aux, ldx=N)
+        mb().debug_options(gemm_mode=mode)
+        try:
+            mb().debug_gemm_ex(epi, M, N, K, As, a_sm, a_sk, Bs, b_sn, b_sk, C, N, **kw)
+            torch.cuda.synchronize()
+        finally:
+            mb().debug_options(gemm_mode=1)
+        outs.append((C, C2))
+    assert not torch.isnan(outs[0][0].float()).any()
+    assert torch.equal(outs[0][0], outs[1][0])
+    if epi in (2, 8):
+        assert torch.equal(outs[0][1], outs[1][1])

@@ -26,7 +26,7 @@ def timeit(fn, reps=20):
 def main():
     T = int(sys.argv[1]) if len(sys.argv) > 1 else 5120
     only = sys.argv[2] if len(sys.argv) > 2 else ""          # substring filter on the case name
-    modes = [int(m) for m in sys.argv[3].split(",")] if len(sys.argv) > 3 else [1, 11, 12, 13]
+    modes = [int(m) for m in sys.argv[3].split(",")] if len(sys.argv) > 3 else [1, 12]
     H, F = 768, 3072
     dev = "cuda"
     bf = torch.bfloat16
@@ -60,21 +60,12 @@ def main():
         ("wgr FFN1 (F,H,T)", 6, F, H, T, dyF, 1, F, h1, 1, H, {}),
         ("wgr QKV (3H,H,T)", 6, 3 * H, H, T, dy3, 1, 3 * H, x, 1, H, {}),
         ("wgr out  (H,H,T) s4", 6, H, H, T, dyH, 1, H, x, 1, H, dict(split=4)),
-        ("wgr FFN2 fused s2", 6, H, F, T, dyH, 1, H, g, 1, F, dict(fused=2)),
-        ("wgr FFN1 fused s2", 6, F, H, T, dyF, 1, F, h1, 1, H, dict(fused=2)),
-        ("wgr QKV  fused s2", 6, 3 * H, H, T, dy3, 1, 3 * H, x, 1, H, dict(fused=2)),
-        ("wgr out  fused s5", 6, H, H, T, dyH, 1, H, x, 1, H, dict(fused=5)),
-        ("wgr FFN2 fused s1", 6, H, F, T, dyH, 1, H, g, 1, F, dict(fused=1)),
     ]
     for name, epi, M, N, K, A, asm, ask, B, bsn, bsk, ex in cases:
         if only and only not in name:
             continue
         fl = 2.0 * M * N * K
         split = ex.pop("split", 1)
-        fused = ex.pop("fused", 0)
-        if fused:
-            ex = dict(C2=ws)
-            split = -fused
         C = (outf if epi in (3, 5, 6) else outb)
         C_ = ws if split > 1 else C
         for mode in modes:
