@@ -181,37 +181,83 @@ MDEV float4 drop_from_bits(const Drop& d, uint32_t bits, int q) {
   return make_float4((bits >> (4 * q)) & 1 ? s : 0.f, (bits >> (4 * q + 1)) & 1 ? s : 0.f,
                      (bits >> (4 * q + 2)) & 1 ? s : 0.f, (bits >> (4 * q + 3)) & 1 ? s : 0.f);
 }
+// Row-tensor inputs of a chunk (residual / GELU' aux) are loaded COALESCED --
+// consecutive lanes read consecutive 16-B pieces of one row (fp32: 8 lanes per
+// 128-B row, 4 rows per instruction; bf16: 4 lanes per 64-B row, 8 rows) -- and
+// transposed to the lane = row layout of the accumulator fragment through the
+// warp's staging buffer (epi_in_transpose).  One row per lane per instruction
+// would touch 32 lines per load (32 L1 wavefronts instead of 4-8).
 template <int EPI>
-MDEV void epi_load(const GemmArgs& g, int m, int n, bool live, EpiIn& in) {
+constexpr int epi_in_kind() {   // 0 none, 1 bf16 rows, 2 fp32 rows
+  return (EPI == EPI_BIAS_DROP_RES || EPI == EPI_GELU_BWD || EPI == EPI_GELUT_BWD) ? 1
+       : (EPI == EPI_ACC_RES_F32 || EPI == EPI_BIAS_DROP_RESF32) ? 2 : 0;
+}
+template <int EPI>
+MDEV void epi_load(const GemmArgs& g, int m_base, int n, int lane, EpiIn& in) {
   if constexpr (EPI == EPI_BIAS || EPI == EPI_BIAS_GELU || EPI == EPI_BIAS_DROP_RES || EPI == EPI_BIAS_GELUT ||
                 EPI == EPI_BIAS_DROP_RESF32) {
     const uint4* p = (const uint4*)((const __nv_bfloat16*)g.bias + n);
 #pragma unroll
     for (int i = 0; i < 4; ++i) in.b[i] = p[i];
   }
-  if (!live) {   // rows >= M: defined (zero) inputs, results never stored
+  if constexpr (epi_in_kind<EPI>() == 1) {
+    const __nv_bfloat16* base = EPI == EPI_BIAS_DROP_RES ? (const __nv_bfloat16*)g.res : (const __nv_bfloat16*)g.aux;
+    const int64_t ld = EPI == EPI_BIAS_DROP_RES ? g.ldr : g.ldx;
 #pragma unroll
-    for (int i = 0; i < 8; ++i) in.x[i] = make_uint4(0u, 0u, 0u, 0u);
-    return;
+    for (int k = 0; k < 4; ++k) {   // rows >= M: defined (zero) inputs, results never stored
+      const int R = 8 * k + (lane >> 2), c = lane & 3;
+      in.x[k] = m_base + R < g.M ? *(const uint4*)(base + (int64_t)(m_base + R) * ld + n + 8 * c) : make_uint4(0u, 0u, 0u, 0u);
+    }
+  } else if constexpr (epi_in_kind<EPI>() == 2) {
+#pragma unroll
+    for (int k = 0; k < 8; ++k) {
+      const int R = 4 * k + (lane >> 3), c = lane & 7;
+      in.x[k] = m_base + R < g.M ? *(const uint4*)((const float*)g.res + (int64_t)(m_base + R) * g.ldr + n + 4 * c)
+                                 : make_uint4(0u, 0u, 0u, 0u);
+    }
   }
-  if constexpr (EPI == EPI_BIAS_DROP_RES) {
-    const uint4* p = (const uint4*)((const __nv_bfloat16*)g.res + (int64_t)m * g.ldr + n);
+}
+// Coalesced pieces -> lane = row: bf16 x[c] = columns 8c..8c+7 of row `lane`,
+// fp32 x[c] = columns 4c..4c+3 (bf16: 64-B rows, chunk ^= (row / 2) % 4; fp32:
+// 128-B rows, chunk ^= row % 8 -- conflict-free both ways).  The buffer must be
+// free: the previous TMA store has finished reading it (ST = 1), the LSU staging
+// ends with __syncwarp (ST = 0).
+template <int EPI, int ST>
+MDEV void epi_in_transpose(EpiOut& o, EpiIn& in, int lane) {
+  constexpr int kind = epi_in_kind<EPI>();
+  if constexpr (kind != 0) {
+    const uint32_t s = smem_u32(o.stg);
+    if constexpr (ST == 1) {
+      if (lane == 0) bulk_wait_read<0>();
+    }
+    __syncwarp();
+    if constexpr (kind == 1) {
 #pragma unroll
-    for (int i = 0; i < 4; ++i) in.x[i] = p[i];
-  } else if constexpr (EPI == EPI_GELU_BWD || EPI == EPI_GELUT_BWD) {
-    const uint4* p = (const uint4*)((const __nv_bfloat16*)g.aux + (int64_t)m * g.ldx + n);
+      for (int k = 0; k < 4; ++k) {
+        const int R = 8 * k + (lane >> 2), c = lane & 3;
+        sts128(s + R * 64 + ((c ^ ((R >> 1) & 3)) << 4), in.x[k]);
+      }
+      __syncwarp();
 #pragma unroll
-    for (int i = 0; i < 4; ++i) in.x[i] = p[i];
-  } else if constexpr (EPI == EPI_ACC_RES_F32 || EPI == EPI_BIAS_DROP_RESF32) {
-    const uint4* p = (const uint4*)((const float*)g.res + (int64_t)m * g.ldr + n);
+      for (int c = 0; c < 4; ++c) in.x[c] = lds128(s + lane * 64 + ((c ^ ((lane >> 1) & 3)) << 4));
+    } else {
 #pragma unroll
-    for (int i = 0; i < 8; ++i) in.x[i] = p[i];
+      for (int k = 0; k < 8; ++k) {
+        const int R = 4 * k + (lane >> 3), c = lane & 7;
+        sts128(s + R * 128 + ((c ^ (R & 7)) << 4), in.x[k]);
+      }
+      __syncwarp();
+#pragma unroll
+      for (int c = 0; c < 8; ++c) in.x[c] = lds128(s + lane * 128 + ((c ^ (lane & 7)) << 4));
+    }
+    __syncwarp();   // every lane has its row before the buffer takes the output
   }
 }
 
 template <int EPI, int ST>
 MDEV void epi_frag32_in(const GemmArgs& g, int m_base, int n, float (&v)[32], int z, EpiOut& o, int lane,
-                        const EpiIn& in, uint32_t keep) {
+                        EpiIn& in, uint32_t keep) {
+  epi_in_transpose<EPI, ST>(o, in, lane);
   using E = __nv_bfloat16;
   const int m = m_base + lane;
   const int rows_valid = g.M - m_base;
@@ -525,18 +571,18 @@ __global__ void __launch_bounds__(TP_THREADS, 1)
         }
       }
       EpiIn nxt;   // the first chunk's epilogue inputs are in flight while the MMAs finish
-      if (n0 + 32 * c_beg + 32 <= g.N) epi_load<EPI>(g, m, n0 + 32 * c_beg, m < g.M, nxt);
+      if (n0 + 32 * c_beg + 32 <= g.N) epi_load<EPI>(g, m0 + 32 * q, n0 + 32 * c_beg, lane, nxt);
       mbar_wait(&tfull[acc], (local >> 1) & 1);
       __syncwarp();
       tc_fence_after();
 #pragma unroll 1
       for (int c = c_beg; c < c_end; ++c) {
-        const EpiIn cur = nxt;
+        EpiIn cur = nxt;
         const uint32_t keep = kbits[0];
 #pragma unroll
         for (int i = 0; i + 1 < NCH; ++i) kbits[i] = kbits[i + 1];   // register rotation, no local memory
         const int n = n0 + 32 * c;
-        if (c + 1 < c_end && n + 64 <= g.N) epi_load<EPI>(g, m, n + 32, m < g.M, nxt);
+        if (c + 1 < c_end && n + 64 <= g.N) epi_load<EPI>(g, m0 + 32 * q, n + 32, lane, nxt);
         float v[32];
         tmem_ld32(tmem + acc * BN + ((uint32_t)(32 * q) << 16) + 32 * c, v);
         if (kb1 <= kb0) {
