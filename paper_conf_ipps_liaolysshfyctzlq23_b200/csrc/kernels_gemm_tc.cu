@@ -292,11 +292,12 @@ MDEV void epi_frag32_in(const GemmArgs& g, int m_base, int n, float (&v)[32], in
       for (int i = 0; i < 4; ++i) unpack8(in.x[i], r + 8 * i);
 #pragma unroll
       for (int q = 0; q < 8; ++q) {
-        const float4 f = live ? drop_from_bits(g.drop, keep, q) : make_float4(0.f, 0.f, 0.f, 0.f);
-        v[4 * q + 0] = (live ? r[4 * q + 0] : 0.f) + v[4 * q + 0] * f.x;
-        v[4 * q + 1] = (live ? r[4 * q + 1] : 0.f) + v[4 * q + 1] * f.y;
-        v[4 * q + 2] = (live ? r[4 * q + 2] : 0.f) + v[4 * q + 2] * f.z;
-        v[4 * q + 3] = (live ? r[4 * q + 3] : 0.f) + v[4 * q + 3] * f.w;
+        // rows >= M: zero residual and keep bits, never stored
+        const float4 f = drop_from_bits(g.drop, keep, q);
+        v[4 * q + 0] = r[4 * q + 0] + v[4 * q + 0] * f.x;
+        v[4 * q + 1] = r[4 * q + 1] + v[4 * q + 1] * f.y;
+        v[4 * q + 2] = r[4 * q + 2] + v[4 * q + 2] * f.z;
+        v[4 * q + 3] = r[4 * q + 3] + v[4 * q + 3] * f.w;
       }
       out_f32<ST>(o, v, (float*)g.C, g.ldc, o.mc, n, m_base, rows_valid, lane);
     }
@@ -336,11 +337,12 @@ MDEV void epi_frag32_in(const GemmArgs& g, int m_base, int n, float (&v)[32], in
       const float* r = (const float*)in.x;
 #pragma unroll
       for (int q = 0; q < 8; ++q) {
-        const float4 f = live ? drop_from_bits(g.drop, keep, q) : make_float4(0.f, 0.f, 0.f, 0.f);
-        v[4 * q + 0] = (live ? r[4 * q + 0] : 0.f) + v[4 * q + 0] * f.x;
-        v[4 * q + 1] = (live ? r[4 * q + 1] : 0.f) + v[4 * q + 1] * f.y;
-        v[4 * q + 2] = (live ? r[4 * q + 2] : 0.f) + v[4 * q + 2] * f.z;
-        v[4 * q + 3] = (live ? r[4 * q + 3] : 0.f) + v[4 * q + 3] * f.w;
+        // rows >= M: zero residual and keep bits, never stored
+        const float4 f = drop_from_bits(g.drop, keep, q);
+        v[4 * q + 0] = r[4 * q + 0] + v[4 * q + 0] * f.x;
+        v[4 * q + 1] = r[4 * q + 1] + v[4 * q + 1] * f.y;
+        v[4 * q + 2] = r[4 * q + 2] + v[4 * q + 2] * f.z;
+        v[4 * q + 3] = r[4 * q + 3] + v[4 * q + 3] * f.w;
       }
       out_f32<ST>(o, v, (float*)g.C, g.ldc, o.mc, n, m_base, rows_valid, lane);
     }
