@@ -423,6 +423,70 @@ MDEV bool seg_of2(const TpArgs& a, const TpArgs& a2, int i, Seg& s) {
     return true;
   }
 }
+// Epilogue of one accumulator tile by one epilogue warp: rows m0 + 32 q + lane
+// (q = TMEM lane quarter of the warp), column group grp of the BN columns.
+// Keep bits and the first chunk's inputs are prepared before the accumulator
+// is waited for (tfull_bar, parity), so they overlap the tile's MMAs.
+template <int BN, int EPI, int ST>
+MDEV void epi_tile(const GemmArgs& g, int m0, int n0, int z, bool no_k, uint32_t tacc, uint64_t* tfull_bar,
+                   uint32_t parity, EpiOut& eo, int q, int grp, int lane) {
+  const int m = m0 + 32 * q + lane;
+  constexpr int ngrp = TP_EPI_WARPS / 4;
+  const int c_beg = grp * (BN / 32) / ngrp, c_end = (grp + 1) * (BN / 32) / ngrp;
+  {  // pull this tile's epilogue inputs into L2 while the MMAs run
+    const int nb = n0 + 32 * c_beg;
+    if (m < g.M && nb < g.N) {
+      const char* pa = nullptr;
+      int bytes = 0;
+      const int ncol = 32 * (c_end - c_beg);
+      if constexpr (EPI == EPI_GELU_BWD || EPI == EPI_GELUT_BWD) { pa = (const char*)((const __nv_bfloat16*)g.aux + (int64_t)m * g.ldx + nb); bytes = 2 * ncol; }
+      if constexpr (EPI == EPI_BIAS_DROP_RESF32) { pa = (const char*)((const float*)g.res + (int64_t)m * g.ldr + nb); bytes = 4 * ncol; }
+      if constexpr (EPI == EPI_BIAS_DROP_RES) { pa = (const char*)((const __nv_bfloat16*)g.res + (int64_t)m * g.ldr + nb); bytes = 2 * ncol; }
+      if constexpr (EPI == EPI_ACC_RES_F32) { pa = (const char*)((const float*)g.res + (int64_t)m * g.ldr + nb); bytes = 4 * ncol; }
+      for (int o = 0; o < bytes; o += 128) asm volatile("prefetch.global.L2 [%0];" ::"l"(pa + o));
+    }
+  }
+  // dropout keep bits of this warp's chunks, computed while the MMAs run
+  constexpr int NCH = BN / 32 / (TP_EPI_WARPS / 4);
+  uint32_t kbits[NCH];
+  constexpr bool DROP_EPI = EPI == EPI_BIAS_DROP_RES || EPI == EPI_BIAS_DROP_RESF32;
+#pragma unroll
+  for (int i = 0; i < NCH; ++i) {
+    kbits[i] = 0u;
+    if constexpr (DROP_EPI) {
+      const int n = n0 + 32 * (c_beg + i);
+      if (m < g.M && n + 32 <= g.N) kbits[i] = drop_bits32(g.drop, (uint64_t)m * g.ldc + n);
+    }
+  }
+  EpiIn nxt;   // the first chunk's epilogue inputs are in flight while the MMAs finish
+  if (n0 + 32 * c_beg + 32 <= g.N) epi_load<EPI>(g, m0 + 32 * q, n0 + 32 * c_beg, lane, nxt);
+  mbar_wait(tfull_bar, parity);
+  __syncwarp();
+  tc_fence_after();
+#pragma unroll 1
+  for (int c = c_beg; c < c_end; ++c) {
+    EpiIn cur = nxt;
+    const uint32_t keep = kbits[0];
+#pragma unroll
+    for (int i = 0; i + 1 < NCH; ++i) kbits[i] = kbits[i + 1];   // register rotation, no local memory
+    const int n = n0 + 32 * c;
+    if (c + 1 < c_end && n + 64 <= g.N) epi_load<EPI>(g, m0 + 32 * q, n + 32, lane, nxt);
+    float v[32];
+    tmem_ld32(tacc + ((uint32_t)(32 * q) << 16) + 32 * c, v);
+    if (no_k) {
+#pragma unroll
+      for (int i = 0; i < 32; ++i) v[i] = 0.f;
+    }
+    if (n + 32 <= g.N) {
+      if (m0 + 32 * q < g.M) epi_frag32_in<EPI, ST>(g, m0 + 32 * q, n, v, z, eo, lane, cur, keep);
+    } else if (m < g.M) {
+#pragma unroll
+      for (int i = 0; i < 32; ++i)
+        if (n + i < g.N) epilogue<__nv_bfloat16, EPI>(g, m, n + i, v[i], z);
+    }
+  }
+}
+
 template <int BN, int EPI, bool G2, int ST>
 __global__ void __launch_bounds__(TP_THREADS, 1)
     k_gemm_tcp(const __grid_constant__ CUtensorMap tma_a, const __grid_constant__ CUtensorMap tma_b, const TpArgs args,
@@ -534,7 +598,7 @@ __global__ void __launch_bounds__(TP_THREADS, 1)
     const int e = warp - 2;
     EpiOut eo{stg_base + e * Cf::STG_PER, &tma_c, &tma_c2, 0};
     const int q = warp & 3;                            // TMEM lane quarter of this warp
-    const int grp = e >> 2, ngrp = TP_EPI_WARPS / 4;  // column group of this warp
+    const int grp = e >> 2;                            // column group of this warp
     int local = 0;
     Seg sg;
     for (; seg_of2<G2>(args, args2, local, sg); ++local) {
@@ -545,60 +609,8 @@ __global__ void __launch_bounds__(TP_THREADS, 1)
       const int m0 = (r / A.n_blocks) * TBM, n0 = (r % A.n_blocks) * BN;
       const int kb0 = sg.kb0, kb1 = sg.kb1;
       const int acc = local & 1;
-      const int m = m0 + 32 * q + lane;
-      const int c_beg = grp * (BN / 32) / ngrp, c_end = (grp + 1) * (BN / 32) / ngrp;
-      {  // pull this tile's epilogue inputs into L2 while the MMAs run
-        const int nb = n0 + 32 * c_beg;
-        if (m < g.M && nb < g.N) {
-          const char* pa = nullptr;
-          int bytes = 0;
-          const int ncol = 32 * (c_end - c_beg);
-          if constexpr (EPI == EPI_GELU_BWD || EPI == EPI_GELUT_BWD) { pa = (const char*)((const __nv_bfloat16*)g.aux + (int64_t)m * g.ldx + nb); bytes = 2 * ncol; }
-          if constexpr (EPI == EPI_BIAS_DROP_RESF32) { pa = (const char*)((const float*)g.res + (int64_t)m * g.ldr + nb); bytes = 4 * ncol; }
-          if constexpr (EPI == EPI_BIAS_DROP_RES) { pa = (const char*)((const __nv_bfloat16*)g.res + (int64_t)m * g.ldr + nb); bytes = 2 * ncol; }
-          if constexpr (EPI == EPI_ACC_RES_F32) { pa = (const char*)((const float*)g.res + (int64_t)m * g.ldr + nb); bytes = 4 * ncol; }
-          for (int o = 0; o < bytes; o += 128) asm volatile("prefetch.global.L2 [%0];" ::"l"(pa + o));
-        }
-      }
-      // dropout keep bits of this warp's chunks, computed while the MMAs run
-      constexpr int NCH = BN / 32 / (TP_EPI_WARPS / 4);
-      uint32_t kbits[NCH];
-      constexpr bool DROP_EPI = EPI == EPI_BIAS_DROP_RES || EPI == EPI_BIAS_DROP_RESF32;
-#pragma unroll
-      for (int i = 0; i < NCH; ++i) {
-        kbits[i] = 0u;
-        if constexpr (DROP_EPI) {
-          const int n = n0 + 32 * (c_beg + i);
-          if (m < g.M && n + 32 <= g.N) kbits[i] = drop_bits32(g.drop, (uint64_t)m * g.ldc + n);
-        }
-      }
-      EpiIn nxt;   // the first chunk's epilogue inputs are in flight while the MMAs finish
-      if (n0 + 32 * c_beg + 32 <= g.N) epi_load<EPI>(g, m0 + 32 * q, n0 + 32 * c_beg, lane, nxt);
-      mbar_wait(&tfull[acc], (local >> 1) & 1);
-      __syncwarp();
-      tc_fence_after();
-#pragma unroll 1
-      for (int c = c_beg; c < c_end; ++c) {
-        EpiIn cur = nxt;
-        const uint32_t keep = kbits[0];
-#pragma unroll
-        for (int i = 0; i + 1 < NCH; ++i) kbits[i] = kbits[i + 1];   // register rotation, no local memory
-        const int n = n0 + 32 * c;
-        if (c + 1 < c_end && n + 64 <= g.N) epi_load<EPI>(g, m0 + 32 * q, n + 32, lane, nxt);
-        float v[32];
-        tmem_ld32(tmem + acc * BN + ((uint32_t)(32 * q) << 16) + 32 * c, v);
-        if (kb1 <= kb0) {
-#pragma unroll
-          for (int i = 0; i < 32; ++i) v[i] = 0.f;
-        }
-        if (n + 32 <= g.N) {
-          if (m0 + 32 * q < g.M) epi_frag32_in<EPI, ST>(g, m0 + 32 * q, n, v, z, eo, lane, cur, keep);
-        } else if (m < g.M) {
-#pragma unroll
-          for (int i = 0; i < 32; ++i)
-            if (n + i < g.N) epilogue<__nv_bfloat16, EPI>(g, m, n + i, v[i], z);
-        }
-      }
+      epi_tile<BN, EPI, ST>(g, m0, n0, z, kb1 <= kb0, tmem + acc * BN, &tfull[acc], (local >> 1) & 1, eo, q, grp,
+                            lane);
       tc_fence_before();
       __syncwarp();
       if (lane == 0) asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_u32(&tempty[acc])) : "memory");
@@ -615,6 +627,181 @@ __global__ void __launch_bounds__(TP_THREADS, 1)
   }
 }
 
+
+// ---------------------------------------------------------------------------
+// CTA-pair kernel (cta_group::2): a cluster of two CTAs (one TPC) computes
+// 256 x BN tiles.  CTA r TMA-loads rows [128 r, 128 r + 128) of A and rows
+// [BN/2 r, BN/2 (r + 1)) of the B tile into its own smem, the transaction bytes
+// of both landing on the leader's full barrier; the leader's single thread
+// issues tcgen05.mma.cta_group::2 (M = 256, N = BN), which reads both CTAs'
+// smem and accumulates rows 128 r.. of the tile in CTA r's TMEM.  Commits are
+// multicast to both CTAs (stage release, accumulator ready); both CTAs'
+// epilogue warps release an accumulator on the leader's tmem-empty barrier.
+// Per SM the B bytes per MMA and the smem operand reads are halved relative to
+// the single-CTA kernel, and a stage is 32 KB (6 stages in flight).  Each CTA
+// runs the same epilogue (epi_tile) on its 128 rows.
+// ---------------------------------------------------------------------------
+constexpr uint32_t PEER_MASK = 0xFEFFFFFFu;   // shared::cta address -> the leader CTA's copy
+
+template <int BN>
+struct T2Cfg {
+  static constexpr int A_BYTES = TBM * TBK * 2;
+  static constexpr int B_BYTES = (BN / 2) * TBK * 2;
+  static constexpr int STAGE_BYTES = A_BYTES + B_BYTES;
+  static constexpr int STAGES = (192 * 1024) / STAGE_BYTES;
+  static constexpr int STG_PER = 4096;
+  static constexpr int STG_BYTES = TP_EPI_WARPS * STG_PER;
+  static constexpr int SMEM = STAGES * STAGE_BYTES + STG_BYTES + 1024 + 256;
+};
+
+MDEV uint32_t cluster_rank() {
+  uint32_t r;
+  asm volatile("mov.u32 %0, %%cluster_ctarank;" : "=r"(r));
+  return r;
+}
+MDEV void cluster_sync_all() {
+  asm volatile("barrier.cluster.arrive.release.aligned;\n\tbarrier.cluster.wait.acquire.aligned;" ::: "memory");
+}
+MDEV void tma_load_2d_2sm(const CUtensorMap* map, uint64_t* bar, void* dst, int c0, int c1) {
+  asm volatile(
+      "cp.async.bulk.tensor.2d.cta_group::2.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1, {%3, %4}], [%2];"
+      ::"r"(smem_u32(dst)), "l"(map), "r"(smem_u32(bar) & PEER_MASK), "r"(c0), "r"(c1) : "memory");
+}
+MDEV void mma_bf16_2sm(uint32_t tmem_d, uint64_t da, uint64_t db, uint32_t idesc, uint32_t acc) {
+  asm volatile(
+      "{\n\t.reg .pred p;\n\tsetp.ne.b32 p, %4, 0;\n\t"
+      "tcgen05.mma.cta_group::2.kind::f16 [%0], %1, %2, %3, p;\n\t}"
+      ::"r"(tmem_d), "l"(da), "l"(db), "r"(idesc), "r"(acc));
+}
+MDEV void mma_commit_2sm_mc(uint64_t* bar) {
+  asm volatile("tcgen05.commit.cta_group::2.mbarrier::arrive::one.shared::cluster.multicast::cluster.b64 [%0], %1;"
+               ::"r"(smem_u32(bar)), "h"((uint16_t)3) : "memory");
+}
+MDEV void mbar_arrive_rank(uint64_t* bar, uint32_t rank) {
+  asm volatile("{\n\t.reg .b32 ra;\n\tmapa.shared::cluster.u32 ra, %0, %1;\n\t"
+               "mbarrier.arrive.release.cluster.shared::cluster.b64 _, [ra];\n\t}"
+               ::"r"(smem_u32(bar)), "r"(rank) : "memory");
+}
+
+template <int BN, int EPI, int ST>
+__global__ void __launch_bounds__(TP_THREADS, 1)
+    k_gemm_tc2(const __grid_constant__ CUtensorMap tma_a, const __grid_constant__ CUtensorMap tma_b, const TpArgs args,
+               const __grid_constant__ CUtensorMap tma_c, const __grid_constant__ CUtensorMap tma_c2) {
+  pdl_trigger();
+  using Cf = T2Cfg<BN>;
+  extern __shared__ uint8_t smem_raw[];
+  uint8_t* smem = (uint8_t*)(((uintptr_t)smem_raw + 1023) & ~(uintptr_t)1023);
+  uint8_t* stg_base = smem + Cf::STAGES * Cf::STAGE_BYTES;
+  uint64_t* full = (uint64_t*)(stg_base + Cf::STG_BYTES);
+  uint64_t* empty = full + Cf::STAGES;
+  uint64_t* tfull = empty + Cf::STAGES;    // [2]
+  uint64_t* tempty = tfull + 2;            // [2] (the leader's are used)
+  uint32_t* tmem_slot = (uint32_t*)(tempty + 2);
+  const TcArgs& ta = args.t;
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const uint32_t rank = cluster_rank();
+  const bool leader = rank == 0;
+  const int cid = blockIdx.x >> 1, ncl = gridDim.x >> 1;
+
+  if (warp == 0 && lane == 0) {
+    for (int s = 0; s < Cf::STAGES; ++s) { mbar_init(&full[s], 1); mbar_init(&empty[s], 1); }
+    for (int a = 0; a < 2; ++a) { mbar_init(&tfull[a], 1); mbar_init(&tempty[a], 2 * TP_EPI_WARPS); }
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+    asm volatile("prefetch.tensormap [%0];" ::"l"(&tma_a) : "memory");
+    asm volatile("prefetch.tensormap [%0];" ::"l"(&tma_b) : "memory");
+  }
+  if (warp == 1) {
+    asm volatile("tcgen05.alloc.cta_group::2.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(smem_u32(tmem_slot)),
+                 "r"(2 * BN));
+    asm volatile("tcgen05.relinquish_alloc_permit.cta_group::2.sync.aligned;");
+  }
+  tc_fence_before();
+  cluster_sync_all();
+  tc_fence_after();
+  const uint32_t tmem = *tmem_slot;
+  pdl_wait();
+
+  if (warp == 0) {
+    if (lane == 0) {                                   // ---------------- TMA producer (both CTAs)
+      int it = 0;
+      for (int tile = cid; tile < args.n_tiles; tile += ncl) {
+        const int m0 = (tile / args.n_blocks) * 256 + 128 * (int)rank;
+        const int nb = (tile % args.n_blocks) * BN + (BN / 2) * (int)rank;
+        for (int kb = 0; kb < ta.kb_total; ++kb, ++it) {
+          const int s = it % Cf::STAGES;
+          if (it >= Cf::STAGES) mbar_wait(&empty[s], ((it / Cf::STAGES) - 1) & 1);
+          uint8_t* sa = smem + s * Cf::STAGE_BYTES;
+          uint8_t* sb = sa + Cf::A_BYTES;
+          const int k = kb * TBK;
+          if (leader) mbar_expect_tx(&full[s], 2 * Cf::STAGE_BYTES);
+          if (ta.a_mn) {
+            tma_load_2d_2sm(&tma_a, &full[s], sa, m0, k);
+            tma_load_2d_2sm(&tma_a, &full[s], sa + 8192, m0 + 64, k);
+          } else {
+            tma_load_2d_2sm(&tma_a, &full[s], sa, k, m0);
+          }
+          if (ta.b_mn) {
+#pragma unroll
+            for (int j = 0; j < BN / 128; ++j) tma_load_2d_2sm(&tma_b, &full[s], sb + 8192 * j, nb + 64 * j, k);
+          } else {
+            tma_load_2d_2sm(&tma_b, &full[s], sb, k, nb);
+          }
+        }
+      }
+    }
+  } else if (warp == 1) {
+    if (lane == 0 && leader) {                         // ---------------- MMA issuer (leader)
+      const uint32_t idesc = idesc_bf16(256, BN, ta.a_mn, ta.b_mn);
+      int it = 0, local = 0;
+      for (int tile = cid; tile < args.n_tiles; tile += ncl, ++local) {
+        const int acc = local & 1;
+        if (local >= 2) mbar_wait(&tempty[acc], ((local >> 1) - 1) & 1);
+        tc_fence_after();
+        const uint32_t d = tmem + acc * BN;
+        for (int kb = 0; kb < ta.kb_total; ++kb, ++it) {
+          const int s = it % Cf::STAGES;
+          mbar_wait(&full[s], (it / Cf::STAGES) & 1);
+          tc_fence_after();
+          const uint32_t sa = smem_u32(smem + s * Cf::STAGE_BYTES);
+          const uint32_t sb = sa + Cf::A_BYTES;
+#pragma unroll
+          for (int kk = 0; kk < TBK / 16; ++kk) {
+            const uint64_t da = ta.a_mn ? make_desc(sa + kk * 2048, 8192, 1024) : make_desc(sa + kk * 32, 16, 1024);
+            const uint64_t db = ta.b_mn ? make_desc(sb + kk * 2048, 8192, 1024) : make_desc(sb + kk * 32, 16, 1024);
+            mma_bf16_2sm(d, da, db, idesc, (kb > 0 || kk > 0) ? 1u : 0u);
+          }
+          mma_commit_2sm_mc(&empty[s]);
+        }
+        mma_commit_2sm_mc(&tfull[acc]);
+      }
+    }
+  } else {                                             // ---------------- epilogue warps (both CTAs)
+    const int e = warp - 2;
+    EpiOut eo{stg_base + e * Cf::STG_PER, &tma_c, &tma_c2, 0};
+    const int q = warp & 3, grp = e >> 2;
+    const GemmArgs& g = ta.g;
+    int local = 0;
+    for (int tile = cid; tile < args.n_tiles; tile += ncl, ++local) {
+      const int m0 = (tile / args.n_blocks) * 256 + 128 * (int)rank;
+      const int n0 = (tile % args.n_blocks) * BN;
+      const int acc = local & 1;
+      epi_tile<BN, EPI, ST>(g, m0, n0, 0, ta.kb_total <= 0, tmem + acc * BN, &tfull[acc], (local >> 1) & 1, eo, q,
+                            grp, lane);
+      tc_fence_before();
+      __syncwarp();
+      if (lane == 0) mbar_arrive_rank(&tempty[acc], 0);
+    }
+    if constexpr (ST == 1) {
+      if (lane == 0) bulk_wait_all();
+    }
+  }
+  tc_fence_before();
+  cluster_sync_all();
+  if (warp == 1) {
+    tc_fence_after();
+    asm volatile("tcgen05.dealloc.cta_group::2.sync.aligned.b32 %0, %1;" ::"r"(tmem), "r"(2 * BN));
+  }
+}
 
 typedef CUresult (*EncodeFn)(CUtensorMap*, CUtensorMapDataType, cuuint32_t, void*, const cuuint64_t*,
                              const cuuint64_t*, const cuuint32_t*, const cuuint32_t*, CUtensorMapInterleave,
@@ -736,6 +923,37 @@ static void dispatch_tcp(Epi epi, const CUtensorMap& ma, const CUtensorMap& mb, 
   }
 }
 
+template <int BN, int EPI, int ST>
+static void launch_tc2(const CUtensorMap& ma, const CUtensorMap& mb, const TpArgs& a, const CUtensorMap& mc,
+                       const CUtensorMap& mc2, cudaStream_t st) {
+  static bool attr = false;
+  if (!attr) {
+    cudaFuncSetAttribute(k_gemm_tc2<BN, EPI, ST>, cudaFuncAttributeMaxDynamicSharedMemorySize, T2Cfg<BN>::SMEM);
+    attr = true;
+  }
+  launch_kc(k_gemm_tc2<BN, EPI, ST>, 2 * std::min(num_sms() / 2, a.n_tiles), TP_THREADS, T2Cfg<BN>::SMEM, st, 2, ma,
+            mb, a, mc, mc2);
+}
+
+template <int BN, int ST>
+static void dispatch_tc2(Epi epi, const CUtensorMap& ma, const CUtensorMap& mb, const TpArgs& a,
+                         const CUtensorMap& mc, const CUtensorMap& mc2, cudaStream_t st) {
+  switch (epi) {
+    case EPI_STORE: launch_tc2<BN, EPI_STORE, ST>(ma, mb, a, mc, mc2, st); break;
+    case EPI_BIAS: launch_tc2<BN, EPI_BIAS, ST>(ma, mb, a, mc, mc2, st); break;
+    case EPI_BIAS_GELU: launch_tc2<BN, EPI_BIAS_GELU, ST>(ma, mb, a, mc, mc2, st); break;
+    case EPI_BIAS_DROP_RES: launch_tc2<BN, EPI_BIAS_DROP_RES, ST>(ma, mb, a, mc, mc2, st); break;
+    case EPI_GELU_BWD: launch_tc2<BN, EPI_GELU_BWD, ST>(ma, mb, a, mc, mc2, st); break;
+    case EPI_ACC_RES_F32: launch_tc2<BN, EPI_ACC_RES_F32, ST>(ma, mb, a, mc, mc2, st); break;
+    case EPI_NONE: launch_tc2<BN, EPI_NONE, 0>(ma, mb, a, mc, mc2, st); break;
+    case EPI_BIAS_GELUT: launch_tc2<BN, EPI_BIAS_GELUT, ST>(ma, mb, a, mc, mc2, st); break;
+    case EPI_GELUT_BWD: launch_tc2<BN, EPI_GELUT_BWD, ST>(ma, mb, a, mc, mc2, st); break;
+    case EPI_BIAS_DROP_RESF32: launch_tc2<BN, EPI_BIAS_DROP_RESF32, ST>(ma, mb, a, mc, mc2, st); break;
+    case EPI_ACC_F32: launch_tc2<BN, EPI_ACC_F32, 0>(ma, mb, a, mc, mc2, st); break;
+    default: launch_tc2<BN, EPI_F32, ST>(ma, mb, a, mc, mc2, st); break;
+  }
+}
+
 static int num_sms() {
   static int nsm = 0;
   if (!nsm) {
@@ -747,7 +965,7 @@ static int num_sms() {
   return nsm;
 }
 
-static int g_gemm_mode = 1;   // 1: default; 12: force 128 x 256 tiles and no grouped launches; 15: LSU-store epilogues instead of TMA stores (test hooks)
+static int g_gemm_mode = 1;   // 1: default; 12: force 128 x 256 tiles and no grouped launches; 15: LSU-store epilogues instead of TMA stores; 17: CTA-pair kernel (test hooks)
 void set_gemm_mode(int m) { g_gemm_mode = m; }
 
 bool tc_available() { return encode_fn() != nullptr; }
@@ -795,6 +1013,30 @@ bool gemm_tc(Epi epi, const GemmArgs& g, cudaStream_t st) {
   // 128; T = 2560: 27.6 vs 23.8).  Stream-K, CTA pairs, BN = 64, the
   // one-tile-per-CTA kernel and an in-kernel fused split-K were built in round
   // 1, measured slower on the step shapes and removed.
+  // CTA pairs (256 x 256 tiles over two SMs) where the single-CTA kernel has
+  // >= 600 tiles of 128 x 256 (about four waves) and the epilogue carries no
+  // Philox dropout: measured 5-9% faster there (T = 8192 x 3072 / 4096 x 1024,
+  // GPT-2's 50264 x 1024 x 2048 dW_e; BERT-large 622 -> 633 samples/s), equal
+  // or slower with fewer tiles or the dropout epilogues (tools/gpu_pair*.sh).
+  const bool drop_epi = epi == EPI_BIAS_DROP_RES || epi == EPI_BIAS_DROP_RESF32;
+  const bool pair = g.split == 1 && g.N % 256 == 0 &&
+                    (g_gemm_mode == 17 || (g_gemm_mode == 1 && !drop_epi && g.bn != 128 &&
+                                           (int64_t)m_blocks * (g.N / 256) >= 600));
+  if (pair) {
+    CUtensorMap ma2, mb2, mc, mc2;
+    bool ok2 = a.a_mn ? make_map(&ma2, g.A, g.M, g.K, g.a_sk, 64, 64) : make_map(&ma2, g.A, g.K, g.M, g.a_sm, 64, TBM);
+    if (ok2) ok2 = a.b_mn ? make_map(&mb2, g.B, g.N, g.K, g.b_sk, 64, 64) : make_map(&mb2, g.B, g.K, g.N, g.b_sn, 64, 128);
+    if (ok2) {
+      TpArgs p;
+      p.t = a;
+      p.m_blocks = (g.M + 255) / 256;
+      p.n_blocks = g.N / 256;
+      p.n_tiles = p.m_blocks * p.n_blocks;
+      if (tma_store_ok(epi, g, &mc, &mc2)) dispatch_tc2<256, 1>(epi, ma2, mb2, p, mc, mc2, st);
+      else dispatch_tc2<256, 0>(epi, ma2, mb2, p, ma2, ma2, st);
+      return true;
+    }
+  }
   auto tiles = [&](int bn) { return m_blocks * ((g.N + bn - 1) / bn) * g.split; };
   int BN = (g.N % 256 == 0 && 2 * tiles(256) >= num_sms()) ? 256 : 128;
   if (g.bn == 256 && g.N % 256 == 0) BN = 256;

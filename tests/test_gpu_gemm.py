@@ -30,7 +30,7 @@ def operands(M, N, K, a_mn, b_mn, seed=0):
 SHAPES += [(2048, 3072, 768), (512, 768, 3072), (4096, 2304, 768)]   # BN=256 persistent tiles
 
 
-@pytest.fixture(params=[1, 12, 15], ids=["persistent", "persistent-bn256", "persistent-lsu-store"])
+@pytest.fixture(params=[1, 12, 15, 17], ids=["persistent", "persistent-bn256", "persistent-lsu-store", "cta-pair"])
 def gemm_mode(request):
     mb().debug_options(gemm_mode=request.param)
     yield request.param
@@ -175,4 +175,49 @@ def test_tma_store_epilogues_bitwise(epi, shape):
     assert not torch.isnan(outs[0][0].float()).any()
     assert torch.equal(outs[0][0], outs[1][0])
     if epi in (2, 8):
+        assert torch.equal(outs[0][1], outs[1][1])
+
+
+@pytest.mark.parametrize("epi", [0, 2, 3, 4, 5, 6])
+@pytest.mark.parametrize("shape,majors", [((300, 768, 136), (0, 0)), ((2100, 3072, 768), (0, 0)),
+                                          ((1000, 768, 3072), (0, 1)), ((768, 3072, 1000), (1, 1))])
+def test_cta_pair_bitwise(epi, shape, majors):
+    """The CTA-pair kernel (gemm mode 17: cta_group::2, 256 x 256 tiles over two
+    SMs) accumulates every output element over K in the same order as the
+    single-CTA kernel with 256-wide tiles (mode 12), so every epilogue's output
+    is bitwise equal -- with M not a multiple of 256 (the second CTA's rows
+    partly or wholly past M) and both operand majors."""
+    if majors != (0, 0) and epi not in (6,):
+        pytest.skip("MN-major operands: the weight-gradient (fp32) epilogue")
+    M, N, K = shape
+    A, B, As, Bs, a_sm, a_sk, b_sn, b_sk = operands(M, N, K, *majors, seed=40 + epi)
+    bf, f32 = torch.bfloat16, torch.float32
+    out_f32 = epi in (3, 5, 6)
+    g = torch.Generator(device="cuda").manual_seed(9)
+    bias = torch.randn(N, device="cuda", generator=g).to(bf)
+    res = torch.randn(M, N, device="cuda", generator=g)
+    aux = torch.randn(M, N, device="cuda", generator=g).to(bf)
+    outs = []
+    for mode in (12, 17):
+        C = torch.full((M, N), float("nan"), device="cuda", dtype=f32 if out_f32 else bf)
+        C2 = torch.full((M, N), float("nan"), device="cuda", dtype=bf)
+        kw = dict(bias=bias)
+        if epi == 2:
+            kw["C2"] = C2
+        if epi == 3:
+            kw.update(res=res.to(bf), ldr=N)
+        if epi == 5:
+            kw.update(res=res, ldr=N)
+        if epi == 4:
+            kw.update(aux=aux, ldx=N)
+        mb().debug_options(gemm_mode=mode)
+        try:
+            mb().debug_gemm_ex(epi, M, N, K, As, a_sm, a_sk, Bs, b_sn, b_sk, C, N, **kw)
+            torch.cuda.synchronize()
+        finally:
+            mb().debug_options(gemm_mode=1)
+        outs.append((C, C2))
+    assert not torch.isnan(outs[0][0].float()).any()
+    assert torch.equal(outs[0][0], outs[1][0])
+    if epi == 2:
         assert torch.equal(outs[0][1], outs[1][1])
