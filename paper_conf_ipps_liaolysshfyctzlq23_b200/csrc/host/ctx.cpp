@@ -976,12 +976,17 @@ void lm_head_backward(Run& r, float* yL, char* hf, float2* stf, float2* tok, cha
     g.C = logits; g.ldc = VP;
     pgemm(c, EPI_F32, g, r.st);                                  // recompute the chunk's logits
     lm_ce_bwd(c->dt, logits, VP, V, r0, nc, c->ids, c->lens, c->B, c->S, tok, dlog, r.st);
-    g = GemmArgs();                                               // dh = dlog W_e
+    // dh = dlog W_e: K = V but only nc/128 x H/256 output tiles, so the K range is
+    // split in two (fp32 partials in the chunk's logits region, dead once dlog is
+    // written; fixed-order sum): twice the tiles at the 256-wide tile rate.
+    g = GemmArgs();
     g.M = nc; g.N = H; g.K = V;
     g.A = dlog; g.a_sm = VP; g.a_sk = 1;
     g.B = W(c, P_WORD); g.b_sn = 1; g.b_sk = H;
-    g.C = dy + (int64_t)r0 * H; g.ldc = H;
+    g.C = logits; g.ldc = H;
+    g.split = 2; g.split_stride = (int64_t)nc * H;
     pgemm(c, EPI_F32, g, r.st);
+    splitk_reduce(logits, 2, (int64_t)nc * H, dy + (int64_t)r0 * H, r.st);
     g = GemmArgs();                                               // dW_e += dlog^T hf
     g.M = V; g.N = H; g.K = nc;
     g.A = dlog; g.a_sm = 1; g.a_sk = VP;
