@@ -73,10 +73,12 @@ MDEV void stage_store_f32(uint8_t* stg_p, const float (&v)[32], float* out, int6
   }
   __syncwarp();
 }
-MDEV void stage_store_bf16(uint8_t* stg_p, const float (&v)[32], __nv_bfloat16* out, int64_t ld, int rows_valid, int lane) {
+// bf16 fragments travel packed: pk[c] = columns 8c..8c+7 of row `lane` (pack8 order).
+MDEV void stage_store_bf16(uint8_t* stg_p, const uint4 (&pk)[4], __nv_bfloat16* out, int64_t ld, int rows_valid,
+                           int lane) {
   const uint32_t stg = (uint32_t)__cvta_generic_to_shared(stg_p);
 #pragma unroll
-  for (int c = 0; c < 4; ++c) sts128(stg + lane * 128 + ((c ^ (lane & 3)) << 4), pack8(v + 8 * c));
+  for (int c = 0; c < 4; ++c) sts128(stg + lane * 128 + ((c ^ (lane & 3)) << 4), pk[c]);
   __syncwarp();
   uint4 w[4];
 #pragma unroll
@@ -115,13 +117,13 @@ MDEV void tma_store_2d(const CUtensorMap* map, uint32_t src, int c0, int c1) {
                ::"l"(map), "r"(src), "r"(c0), "r"(c1) : "memory");
   asm volatile("cp.async.bulk.commit_group;" ::: "memory");
 }
-MDEV void tma_out_bf16(EpiOut& o, const float (&v)[32], const CUtensorMap* map, int n, int m_base, int lane) {
+MDEV void tma_out_bf16(EpiOut& o, const uint4 (&pk)[4], const CUtensorMap* map, int n, int m_base, int lane) {
   const uint32_t s = smem_u32(o.stg) + 2048u * (uint32_t)o.half;
   o.half ^= 1;
   if (lane == 0) bulk_wait_read<1>();    // the group before last used this half
   __syncwarp();
 #pragma unroll
-  for (int c = 0; c < 4; ++c) sts128(s + lane * 64 + ((c ^ ((lane >> 1) & 3)) << 4), pack8(v + 8 * c));
+  for (int c = 0; c < 4; ++c) sts128(s + lane * 64 + ((c ^ ((lane >> 1) & 3)) << 4), pk[c]);
   fence_async_smem();
   __syncwarp();
   if (lane == 0) tma_store_2d(map, s, n, m_base);
@@ -141,10 +143,42 @@ MDEV void tma_out_f32(EpiOut& o, const float (&v)[32], const CUtensorMap* map, i
 }
 // Output of one fragment: TMA (ST = 1) or LSU stores through the staging buffer (ST = 0).
 template <int ST>
+MDEV void out_bf16p(EpiOut& o, const uint4 (&pk)[4], __nv_bfloat16* base, int64_t ld, const CUtensorMap* map, int n,
+                    int m_base, int rows_valid, int lane) {
+  if constexpr (ST == 1) tma_out_bf16(o, pk, map, n, m_base, lane);
+  else stage_store_bf16(o.stg, pk, base + (int64_t)m_base * ld + n, ld, rows_valid, lane);
+}
+template <int ST>
 MDEV void out_bf16(EpiOut& o, const float (&v)[32], __nv_bfloat16* base, int64_t ld, const CUtensorMap* map, int n,
                    int m_base, int rows_valid, int lane) {
-  if constexpr (ST == 1) tma_out_bf16(o, v, map, n, m_base, lane);
-  else stage_store_bf16(o.stg, v, base + (int64_t)m_base * ld + n, ld, rows_valid, lane);
+  uint4 pk[4];
+#pragma unroll
+  for (int c = 0; c < 4; ++c) pk[c] = pack8(v + 8 * c);
+  out_bf16p<ST>(o, pk, base, ld, map, n, m_base, rows_valid, lane);
+}
+// GELU epilogues: u = acc + bias is stored as bf16 and the GELU reads the STORED
+// u, so u is packed once (F2FP pairs) and unpacked with integer shifts instead of
+// a per-element F2F round trip (which runs on the quarter-rate XU pipe beside the
+// MUFU.TANH of the GELU).
+template <int ST>
+MDEV void out_u_gelu(EpiOut& o, float (&v)[32], __nv_bfloat16* u, __nv_bfloat16* gout, int64_t ld,
+                     const CUtensorMap* mu, const CUtensorMap* mg, int n, int m_base, int rows_valid, int lane) {
+  uint4 pk[4];
+#pragma unroll
+  for (int c = 0; c < 4; ++c) pk[c] = pack8(v + 8 * c);
+  out_bf16p<ST>(o, pk, u, ld, mu, n, m_base, rows_valid, lane);
+#pragma unroll
+  for (int c = 0; c < 4; ++c) {
+    const uint32_t w[4] = {pk[c].x, pk[c].y, pk[c].z, pk[c].w};
+#pragma unroll
+    for (int j = 0; j < 4; ++j) {
+      const float2 uu = make_float2(__uint_as_float(w[j] << 16), __uint_as_float(w[j] & 0xFFFF0000u));
+      const float2 r = gelu_fast_x2(uu);
+      v[8 * c + 2 * j] = r.x;
+      v[8 * c + 2 * j + 1] = r.y;
+    }
+  }
+  out_bf16<ST>(o, v, gout, ld, mg, n, m_base, rows_valid, lane);
 }
 template <int ST>
 MDEV void out_f32(EpiOut& o, const float (&v)[32], float* base, int64_t ld, const CUtensorMap* map, int n, int m_base,
@@ -277,15 +311,7 @@ MDEV void epi_frag32_in(const GemmArgs& g, int m_base, int n, float (&v)[32], in
     if constexpr (EPI == EPI_BIAS) {
       out_bf16<ST>(o, v, (E*)g.C, g.ldc, o.mc, n, m_base, rows_valid, lane);
     } else if constexpr (EPI == EPI_BIAS_GELU) {
-      out_bf16<ST>(o, v, (E*)g.C, g.ldc, o.mc, n, m_base, rows_valid, lane);
-#pragma unroll
-      for (int i = 0; i < 32; i += 2) {
-        const float2 r = gelu_fast_x2(make_float2(__bfloat162float(__float2bfloat16_rn(v[i])),
-                                             __bfloat162float(__float2bfloat16_rn(v[i + 1]))));
-        v[i] = r.x;
-        v[i + 1] = r.y;
-      }
-      out_bf16<ST>(o, v, (E*)g.C2, g.ldc, o.mc2, n, m_base, rows_valid, lane);
+      out_u_gelu<ST>(o, v, (E*)g.C, (E*)g.C2, g.ldc, o.mc, o.mc2, n, m_base, rows_valid, lane);
     } else {
       float r[32];
 #pragma unroll
@@ -328,11 +354,8 @@ MDEV void epi_frag32_in(const GemmArgs& g, int m_base, int n, float (&v)[32], in
     for (int i = 0; i < 4; ++i) unpack8(in.b[i], b + 8 * i);
 #pragma unroll
     for (int i = 0; i < 32; ++i) v[i] += b[i];
-    if constexpr (EPI == EPI_BIAS_GELUT) {
-      out_bf16<ST>(o, v, (E*)g.C, g.ldc, o.mc, n, m_base, rows_valid, lane);
-#pragma unroll
-      for (int i = 0; i < 32; ++i) v[i] = gelu_fast(__bfloat162float(__float2bfloat16_rn(v[i])));   // gelu_new == the tanh form
-      out_bf16<ST>(o, v, (E*)g.C2, g.ldc, o.mc2, n, m_base, rows_valid, lane);
+    if constexpr (EPI == EPI_BIAS_GELUT) {   // gelu_new == the tanh form
+      out_u_gelu<ST>(o, v, (E*)g.C, (E*)g.C2, g.ldc, o.mc, o.mc2, n, m_base, rows_valid, lane);
     } else {
       const float* r = (const float*)in.x;
 #pragma unroll
