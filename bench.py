@@ -16,6 +16,7 @@ Prints ONE JSON line on rank 0.
 from __future__ import annotations
 
 import argparse
+import dataclasses
 import json
 import os
 import subprocess
@@ -53,6 +54,8 @@ def parse():
     ap.add_argument("--planner", default="greedy", choices=["greedy", "exact", "knapsack"],
                     help="Algorithm 1 (default), the exact fewest-recompute planner (A29) or the "
                          "recompute-time-weighted exact planner (A31)")
+    ap.add_argument("--p-drop", type=float, default=None,
+                    help="override the dropout probability (experiments only: the headline keeps the config's)")
     return ap.parse_args()
 
 
@@ -268,6 +271,8 @@ def main():
     if world > 1:
         dist.init_process_group("nccl", device_id=torch.device("cuda", local))
     cfg = wl.CONFIGS[args.config]
+    if args.p_drop is not None:
+        cfg = dataclasses.replace(cfg, p_drop=args.p_drop)
     stream = torch.cuda.current_stream()
     use_tc = 0 if args.simt else 1
     if args.gemm_mode >= 0:

@@ -13,6 +13,7 @@
 #include <nccl.h>
 
 #include <algorithm>
+#include <array>
 #include <chrono>
 #include <cmath>
 #include <cstdio>
@@ -296,6 +297,7 @@ struct mimose_ctx {
   std::vector<cudaEvent_t> probe_ev;
   size_t probe_used = 0;
   double probe_flops = 0.0;
+  std::vector<std::array<int64_t, 4>> probe_shape;   // per probed launch: M, N, K, epi (grouped: -1)
 };
 
 namespace {
@@ -456,7 +458,7 @@ inline int n_units(const mimose_ctx* c) {
 }
 
 // ------------------------------------------------------------- probe ------
-void pgemm(mimose_ctx* c, Epi epi, const GemmArgs& g, cudaStream_t st) {
+bool probe_begin(mimose_ctx* c, cudaStream_t st) {
   const bool on = c->probe == 1 && c->device;
   if (on) {
     if (c->probe_used + 2 > c->probe_ev.size()) {
@@ -468,12 +470,18 @@ void pgemm(mimose_ctx* c, Epi epi, const GemmArgs& g, cudaStream_t st) {
     }
     cudaEventRecord(c->probe_ev[c->probe_used], st);
   }
+  return on;
+}
+void probe_end(mimose_ctx* c, cudaStream_t st, double flops, std::array<int64_t, 4> shape) {
+  cudaEventRecord(c->probe_ev[c->probe_used + 1], st);
+  c->probe_used += 2;
+  c->probe_flops += flops;
+  c->probe_shape.push_back(shape);
+}
+void pgemm(mimose_ctx* c, Epi epi, const GemmArgs& g, cudaStream_t st) {
+  const bool on = probe_begin(c, st);
   gemm(c->dt, epi, g, st, c->cfg.use_tc != 0);
-  if (on) {
-    cudaEventRecord(c->probe_ev[c->probe_used + 1], st);
-    c->probe_used += 2;
-    c->probe_flops += 2.0 * g.M * (double)g.N * g.K;
-  }
+  if (on) probe_end(c, st, 2.0 * g.M * (double)g.N * g.K, {g.M, g.N, g.K, (int64_t)epi});
 }
 
 // ------------------------------------------------------------- schedule ---
@@ -664,24 +672,11 @@ void wgrad2(Run& r, const void* dY1, int N1, const void* X1, int K1, float* out1
       g[i].B = X[i]; g[i].b_sn = 1; g[i].b_sk = K[i];
       g[i].C = out[i]; g[i].ldc = K[i];
     }
-    const bool on = c->probe == 1 && c->device;
-    if (on) {
-      if (c->probe_used + 2 > c->probe_ev.size()) {
-        for (int i = 0; i < 256; ++i) {
-          cudaEvent_t e;
-          cudaEventCreate(&e);
-          c->probe_ev.push_back(e);
-        }
-      }
-      cudaEventRecord(c->probe_ev[c->probe_used], r.st);
-    }
+    const bool on = probe_begin(c, r.st);
     const bool done = gemm_tc_grouped(g[0], g[1], bn, r.st);
     if (on) {
-      cudaEventRecord(c->probe_ev[c->probe_used + 1], r.st);
-      if (done) {
-        c->probe_used += 2;
-        c->probe_flops += 2.0 * T * ((double)N1 * K1 + (double)N2 * K2);
-      }
+      if (done) probe_end(c, r.st, 2.0 * T * ((double)N1 * K1 + (double)N2 * K2), {T, N1 * K1 + N2 * K2, bn, -1});
+      else cudaEventRecord(c->probe_ev[c->probe_used + 1], r.st);
     }
     if (done) {
       note_launch(1);
@@ -2565,6 +2560,7 @@ mimose_status mimose_probe(mimose_ctx* c, int32_t kind) {
   c->probe = kind;
   c->probe_used = 0;
   c->probe_flops = 0.0;
+  c->probe_shape.clear();
   return MIMOSE_OK;
 }
 
@@ -2573,11 +2569,21 @@ mimose_status mimose_probe_read(mimose_ctx* c, double* ms, double* flops, int64_
   double tot = 0.0;
   if (c->device && c->probe_used) {
     CK(cudaStreamSynchronize(c->st));
+    // MIMOSE_PROBE_DUMP=<path>: one CSV line per probed launch (M, N, K, epi, us);
+    // a grouped weight-gradient launch is (T, N1 K1 + N2 K2, tile width, -1)
+    const char* dump = std::getenv("MIMOSE_PROBE_DUMP");
+    FILE* f = dump ? std::fopen(dump, "a") : nullptr;
     for (size_t i = 0; i + 1 < c->probe_used; i += 2) {
       float t = 0.f;
       CK(cudaEventElapsedTime(&t, c->probe_ev[i], c->probe_ev[i + 1]));
       tot += t;
+      if (f && i / 2 < c->probe_shape.size()) {
+        const auto& sh = c->probe_shape[i / 2];
+        std::fprintf(f, "%lld,%lld,%lld,%lld,%.3f\n", (long long)sh[0], (long long)sh[1], (long long)sh[2],
+                     (long long)sh[3], 1000.0 * t);
+      }
     }
+    if (f) std::fclose(f);
   }
   *ms = tot;
   *flops = c->probe_flops;
