@@ -340,11 +340,12 @@ mimose_status mimose_debug_gemm_grouped(int32_t M1, int32_t N1, int32_t K1, cons
                                         int64_t a_sk2, const void* B2, int64_t b_sn2, int64_t b_sk2, void* C2,
                                         void* stream);
 
-/* Test hook: process-wide kernel options. gemm_mode 0 = one 128x128 tile per CTA,
-   1 = persistent double-buffered single-CTA tcgen05 GEMM (default), 2 = persistent
-   CTA-pair (cta_group::2, 256-row tiles), 11 / 12 / 13 = persistent with tile
-   width 128 / 256 / 64, 14 = persistent deterministic stream-K; attn_tc 0/1
-   routes bf16 attention with S <= 128 to the SIMT / tcgen05 kernels.
+/* Test hook: process-wide kernel options. gemm_mode 1 = the default persistent
+   tcgen05 GEMM (tile width and CTA pairs chosen per shape, grouped weight
+   gradients), 12 / 13 = single-CTA tiles of width 256 / 128 for every shape and
+   no grouped launches, 15 = LSU instead of TMA stores in the epilogues, 17 = the
+   CTA-pair kernel (cta_group::2, 256 x 256 tiles) wherever N % 256 == 0; attn_tc
+   0/1 routes bf16 attention with S <= 128 to the SIMT / tcgen05 kernels.
    Negative = unchanged. */
 void mimose_debug_options(int32_t gemm_mode, int32_t attn_tc);
 

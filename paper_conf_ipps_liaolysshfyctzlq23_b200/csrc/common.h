@@ -26,7 +26,17 @@ struct Drop {
   uint32_t thresh;   // keep iff r < thresh; thresh = floor((1-p) 2^32)
   float scale;       // 1/(1-p) rounded to fp32
   int enabled;       // p > 0
+  // Philox round keys (k0 + r W0, k1 + r W1), r = 0..9, from (seed_lo, seed_hi) by
+  // drop_set_keys: kernel-parameter constants, so the 10 rounds of every draw are
+  // 2 IMAD.WIDE + 2 LOP3 each instead of re-deriving the key schedule per draw.
+  uint32_t rk[20];
 };
+inline void drop_set_keys(Drop& d) {
+  for (int r = 0; r < 10; ++r) {
+    d.rk[2 * r] = d.seed_lo + (uint32_t)r * 0x9E3779B9u;
+    d.rk[2 * r + 1] = d.seed_hi + (uint32_t)r * 0xBB67AE85u;
+  }
+}
 
 // Programmatic dependent launch (PDL).  Every kernel of the library is launched
 // with cudaLaunchAttributeProgrammaticStreamSerialization, so the next kernel in
@@ -93,22 +103,21 @@ MDEV void pdl_enter() {
   pdl_wait();
 }
 
-// Philox4x32-10, Salmon et al. SC'11 (same constants as Random123).
-MDEV uint4 philox4x32_10(uint4 c, uint32_t k0, uint32_t k1) {
+// Philox4x32-10, Salmon et al. SC'11 (same constants as Random123), with the
+// key schedule k_r = k + r (0x9E3779B9, 0xBB67AE85) precomputed in Drop::rk.
+MDEV uint4 philox4x32_10_rk(uint4 c, const uint32_t (&rk)[20]) {
 #pragma unroll
   for (int r = 0; r < 10; ++r) {
-    if (r) { k0 += 0x9E3779B9u; k1 += 0xBB67AE85u; }
     uint32_t hi0 = __umulhi(0xD2511F53u, c.x), lo0 = 0xD2511F53u * c.x;
     uint32_t hi1 = __umulhi(0xCD9E8D57u, c.z), lo1 = 0xCD9E8D57u * c.z;
-    c = make_uint4(hi1 ^ c.y ^ k0, lo1, hi0 ^ c.w ^ k1, lo0);
+    c = make_uint4(hi1 ^ c.y ^ rk[2 * r], lo1, hi0 ^ c.w ^ rk[2 * r + 1], lo0);
   }
   return c;
 }
 
 // Four random words for elements 4n..4n+3 of a site.
 MDEV uint4 drop_words(const Drop& d, uint64_t n) {
-  return philox4x32_10(make_uint4((uint32_t)n, (uint32_t)(n >> 32), d.site, d.step),
-                       d.seed_lo, d.seed_hi);
+  return philox4x32_10_rk(make_uint4((uint32_t)n, (uint32_t)(n >> 32), d.site, d.step), d.rk);
 }
 MDEV uint32_t word_of(uint4 w, int lane) {
   return lane == 0 ? w.x : lane == 1 ? w.y : lane == 2 ? w.z : w.w;

@@ -393,6 +393,7 @@ Drop make_drop(const mimose_ctx* c, uint32_t kind, uint32_t layer) {
   d.step = (uint32_t)c->it;
   d.thresh = d.enabled ? (uint32_t)std::floor((1.0 - p) * 4294967296.0) : 0xFFFFFFFFu;
   d.scale = d.enabled ? (float)(1.0 / (1.0 - p)) : 1.0f;
+  drop_set_keys(d);
   return d;
 }
 Drop no_drop() { Drop d{}; d.enabled = 0; return d; }
@@ -2508,6 +2509,7 @@ mimose_status mimose_debug_gemm_ex(int32_t epi, int32_t M, int32_t N, int32_t K,
   g.split = split < 1 ? 1 : split;
   g.split_stride = (int64_t)M * ldc;
   g.drop.enabled = 1; g.drop.seed_lo = 7; g.drop.seed_hi = 0; g.drop.site = 0; g.drop.step = 1;
+  drop_set_keys(g.drop);
   g.drop.thresh = 3865470566u; g.drop.scale = (float)(1.0 / 0.9);
   gemm(DT_BF16, (Epi)epi, g, (cudaStream_t)stream, use_tc != 0);
   return cudaGetLastError() == cudaSuccess ? MIMOSE_OK : MIMOSE_E_CUDA;

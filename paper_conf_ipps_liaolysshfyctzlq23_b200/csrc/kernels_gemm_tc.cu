@@ -988,7 +988,7 @@ static int num_sms() {
   return nsm;
 }
 
-static int g_gemm_mode = 1;   // 1: default; 12: force 128 x 256 tiles and no grouped launches; 15: LSU-store epilogues instead of TMA stores; 17: CTA-pair kernel (test hooks)
+static int g_gemm_mode = 1;   // 1: default; 12 / 13: force 128 x 256 / 128 x 128 tiles and no grouped launches; 15: LSU-store epilogues instead of TMA stores; 17: CTA-pair kernel (test hooks)
 void set_gemm_mode(int m) { g_gemm_mode = m; }
 
 bool tc_available() { return encode_fn() != nullptr; }
@@ -1040,7 +1040,8 @@ bool gemm_tc(Epi epi, const GemmArgs& g, cudaStream_t st) {
   // >= 600 tiles of 128 x 256 (about four waves) and the epilogue carries no
   // Philox dropout: measured 5-9% faster there (T = 8192 x 3072 / 4096 x 1024,
   // GPT-2's 50264 x 1024 x 2048 dW_e; BERT-large 622 -> 633 samples/s), equal
-  // or slower with fewer tiles or the dropout epilogues (tools/gpu_pair*.sh).
+  // or slower with fewer tiles or the dropout epilogues (mode 17 vs 12 in
+  // tools/bench_gemm.py; profiles/r2/gemm_tile_sweep.txt).
   const bool drop_epi = epi == EPI_BIAS_DROP_RES || epi == EPI_BIAS_DROP_RESF32;
   const bool pair = g.split == 1 && g.N % 256 == 0 &&
                     (g_gemm_mode == 17 || (g_gemm_mode == 1 && !drop_epi && g.bn != 128 &&
@@ -1065,6 +1066,7 @@ bool gemm_tc(Epi epi, const GemmArgs& g, cudaStream_t st) {
   if (g.bn == 256 && g.N % 256 == 0) BN = 256;
   if (g.bn == 128) BN = 128;
   if (g_gemm_mode == 12 && g.N % 256 == 0) BN = 256;
+  if (g_gemm_mode == 13) BN = 128;
   CUtensorMap ma, mb;
   bool ok;
   if (a.a_mn) ok = make_map(&ma, g.A, g.M, g.K, g.a_sk, 64, 64);

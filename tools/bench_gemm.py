@@ -56,6 +56,7 @@ def main():
         ("dgr FFN2 gelu'", 4, T, F, H, dyH, H, 1, w2, 1, F, dict(aux=u, ldx=F)),
         ("dgr FFN1 +res", 5, T, H, F, dyF, F, 1, w1, 1, H, dict(res=resf, ldr=H)),
         ("dgr QKV  +res", 5, T, H, 3 * H, dy3, 3 * H, 1, wq, 1, H, dict(res=resf, ldr=H)),
+        ("dgr out  store", 0, T, H, H, dyH, H, 1, wo, 1, H, {}),
         ("wgr FFN2 (H,F,T)", 6, H, F, T, dyH, 1, H, g, 1, F, {}),
         ("wgr FFN1 (F,H,T)", 6, F, H, T, dyF, 1, F, h1, 1, H, {}),
         ("wgr QKV (3H,H,T)", 6, 3 * H, H, T, dy3, 1, 3 * H, x, 1, H, {}),
