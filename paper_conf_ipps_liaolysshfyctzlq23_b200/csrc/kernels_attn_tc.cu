@@ -72,7 +72,8 @@ MDEV float4 drop4_or(const Drop& d, uint64_t e) {
 }
 
 // 8 warps: warp w reads TMEM lane quarter w % 4 (rows 32(w%4)..+31) and
-// handles column half w / 4 of every row: key chunks [0, cmid) or [cmid, nch).
+// handles key half w / 4 of every row: 16-key units [0, umid) or [umid, n16),
+// umid = ceil(n16 / 2) (the halves differ by at most one unit).
 // The two halves of a row combine their max / sum / dot partials through
 // shared memory in a fixed order (half 0 + half 1), so results are
 // deterministic.
@@ -102,8 +103,9 @@ __global__ void __launch_bounds__(ATT, 3) k_attn_fwd_tc(const __grid_constant__ 
   const int hf = warp >> 2, t = 32 * (warp & 3) + lane;
   const int bh = blockIdx.x, b = bh / a.h, hd = bh % a.h;
   const int S = a.S, Sk = a.Sk, len = a.klens[b];
-  const int kmax = (Sk + 31) & ~31, nch = kmax >> 5, cmid = (nch + 1) >> 1;
-  const int c0 = hf ? cmid : 0, c1 = hf ? nch : cmid;
+  // key half hf covers 16-key units [u0, u1): halves differ by at most one unit
+  const int kmax = (Sk + 31) & ~31, n16 = kmax >> 4, umid = (n16 + 1) >> 1;
+  const int u0 = hf ? umid : 0, u1 = hf ? n16 : umid;
   if (threadIdx.x == 0) {
     for (int i = 0; i < 3; ++i) mbar_init(&bar[i], 1);
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
@@ -138,13 +140,13 @@ __global__ void __launch_bounds__(ATT, 3) k_attn_fwd_tc(const __grid_constant__ 
   const uint32_t trow = tmem + ((uint32_t)(32 * (warp & 3)) << 16);
   const int kl = a.causal ? min(len, t + 1) : len;
   float mx = -INFINITY;
-  for (int c = c0; c < c1; ++c) {
-    float v[32];
-    tmem_ld32(trow + 32 * c, v);                // every lane loads (.sync.aligned)
-    if (32 * c < kl) {
+  for (int u = u0; u < u1; ++u) {
+    float v[16];
+    tmem_ld16(trow + 16 * u, v);                // every lane loads (.sync.aligned)
+    if (16 * u < kl) {
 #pragma unroll
-      for (int i = 0; i < 32; ++i)
-        if (32 * c + i < kl) mx = fmaxf(mx, v[i]);
+      for (int i = 0; i < 16; ++i)
+        if (16 * u + i < kl) mx = fmaxf(mx, v[i]);
     }
   }
   red[hf * 128 + t] = mx;
@@ -155,12 +157,12 @@ __global__ void __launch_bounds__(ATT, 3) k_attn_fwd_tc(const __grid_constant__ 
   // The S MMA has completed (bar[1]), so Q and K are dead: each thread writes its
   // P~ row straight into their space.
   float l = 0.f;
-  for (int c = c0; c < c1; ++c) {
-#pragma unroll
-    for (int hh = 0; hh < 2; ++hh) {
+  for (int u = u0; u < u1; ++u) {
+    {
+      const int c = u >> 1, hh = u & 1;
       float v[16];
-      tmem_ld16(trow + 32 * c + 16 * hh, v);
-      const int kb = 32 * c + 16 * hh;
+      tmem_ld16(trow + 16 * u, v);
+      const int kb = 16 * u;
       if (kb < kl && t < S) {
 #pragma unroll
         for (int j = 0; j < 4; ++j) {
@@ -238,9 +240,9 @@ __global__ void __launch_bounds__(ATT, 2) k_attn_bwd_tc(const __grid_constant__ 
   const int hf = warp >> 2, t = 32 * (warp & 3) + lane;
   const int bh = blockIdx.x, b = bh / a.h, hd = bh % a.h;
   const int S = a.S, Sk = a.Sk, len = a.lengths[b], klen = a.klens[b];
-  const int kmax = (Sk + 31) & ~31, nch = kmax >> 5, cmid = (nch + 1) >> 1;
+  const int kmax = (Sk + 31) & ~31, n16 = kmax >> 4, umid = (n16 + 1) >> 1;
   const int qmax = (S + 31) & ~31;                 // contraction range of dV, dK (query rows)
-  const int c0 = hf ? cmid : 0, c1 = hf ? nch : cmid;
+  const int u0 = hf ? umid : 0, u1 = hf ? n16 : umid;   // this half's 16-key units (<= 4)
   if (threadIdx.x == 0) {
     for (int i = 0; i < 3; ++i) mbar_init(&bar[i], 1);
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
@@ -299,14 +301,14 @@ __global__ void __launch_bounds__(ATT, 2) k_attn_bwd_tc(const __grid_constant__ 
   const int kl = a.causal ? min(klen, t + 1) : klen;
   const float sl2 = a.scale * 1.4426950408889634f, Ll2 = Lt * 1.4426950408889634f;
   const float keepf = a.drop.enabled ? a.drop.scale : 1.0f;
-  uint32_t kb0 = 0u, kb1 = 0u;             // keep bits of chunks c0 (kb0) and c0 + 1 (kb1) of this half
-  for (int c = c0; c < c1 && DC; ++c)
-#pragma unroll
-  for (int hh = 0; hh < 2; ++hh) {
+  uint32_t kb0 = 0u, kb1 = 0u;             // keep bits of units u0, u0 + 1 (kb0) and u0 + 2, u0 + 3 (kb1)
+  for (int u = u0; u < u1 && DC; ++u) {
+    const int hh = (u - u0) & 1;
+    const bool lo = u - u0 < 2;
     float sv[16], dp[16];
-    tmem_ld16(trow + 32 * c + 16 * hh, sv);
-    tmem_ld16(trow + 128 + 32 * c + 16 * hh, dp);
-    const int kb = 32 * c + 16 * hh;
+    tmem_ld16(trow + 16 * u, sv);
+    tmem_ld16(trow + 128 + 16 * u, dp);
+    const int kb = 16 * u;
     if (t < len && kb < kl) {
 #pragma unroll
       for (int j = 0; j < 4; ++j) {
@@ -319,7 +321,7 @@ __global__ void __launch_bounds__(ATT, 2) k_attn_bwd_tc(const __grid_constant__ 
           const float p = (kk < kl) ? ex2f(fmaf(sv[4 * j + i], sl2, -Ll2)) : 0.f;
           Dh = fmaf(p * ff[i], dp[4 * j + i], Dh);
           if (ff[i] != 0.f) {
-            if (c == c0) kb0 |= 1u << (16 * hh + 4 * j + i);
+            if (lo) kb0 |= 1u << (16 * hh + 4 * j + i);
             else kb1 |= 1u << (16 * hh + 4 * j + i);
           }
         }
@@ -330,13 +332,14 @@ __global__ void __launch_bounds__(ATT, 2) k_attn_bwd_tc(const __grid_constant__ 
   __syncthreads();                        // red[] complete; every thread is past the MMAs (V dead)
   const float Dt = red[t] + red[128 + t];
   __syncthreads();                        // every D read before dS overwrites red[]
-  for (int c = c0; c < c1; ++c)
-#pragma unroll
-  for (int hh = 0; hh < 2; ++hh) {
+  for (int u = u0; u < u1; ++u) {
+    const int c = u >> 1, hh = u & 1;            // smem tile chunk of the unit
+    const int bh = (u - u0) & 1;                 // bit half of the unit's keep word
+    const bool lo = u - u0 < 2;
     float sv[16], dp[16];
-    tmem_ld16(trow + 32 * c + 16 * hh, sv);
-    tmem_ld16(trow + 128 + 32 * c + 16 * hh, dp);
-    const int kb = 32 * c + 16 * hh;
+    tmem_ld16(trow + 16 * u, sv);
+    tmem_ld16(trow + 128 + 16 * u, dp);
+    const int kb = 16 * u;
     const bool live = t < len && kb < kl;        // padded / foreign query rows contribute 0
     if (live) {
       float fself[16];
@@ -352,7 +355,7 @@ __global__ void __launch_bounds__(ATT, 2) k_attn_bwd_tc(const __grid_constant__ 
       for (int q = 0; q < 16; ++q) {
         const int kk = kb + q;
         const float p = (kk < kl) ? ex2f(fmaf(sv[q], sl2, -Ll2)) : 0.f;
-        const float fq = !DC ? fself[q] : ((((c == c0 ? kb0 : kb1) >> (16 * hh + q)) & 1u) ? keepf : 0.f);
+        const float fq = !DC ? fself[q] : ((((lo ? kb0 : kb1) >> (16 * bh + q)) & 1u) ? keepf : 0.f);
         sv[q] = p * fq;                                            // P~
         dp[q] = p * (dp[q] * fq - Dt) * a.scale;                   // dS (scale folded)
       }

@@ -618,7 +618,9 @@ __global__ void __launch_bounds__(1024) k_rs_scatter(const int32_t* __restrict__
 
 // piece sums: warp per 32 sorted positions; a piece = a run of equal keys inside the chunk.
 // The piece sum overwrites the X row of the piece's first token (read-before-write, same warp).
-// Keys equal to `skip` (the pad id) are ignored.
+// Keys equal to `skip` (the pad id) are ignored.  The rows of 4 consecutive
+// positions are loaded together (4 independent row loads in flight instead of
+// one row per iteration) and then added in position order: the same sums.
 __global__ void __launch_bounds__(256) k_piece_sum(const int32_t* __restrict__ keys, const int32_t* __restrict__ tok,
                                                    float* X, int T, int H, int skip) {
   pdl_enter();
@@ -626,31 +628,42 @@ __global__ void __launch_bounds__(256) k_piece_sum(const int32_t* __restrict__ k
   const int r0 = chunk * 32;
   if (r0 >= T) return;
   const int r1 = min(r0 + 32, T);
-  const int nv = H >> 5;
+  const int nv = H >> 5;              // <= 32
   float acc[32];
 #pragma unroll
   for (int j = 0; j < 32; ++j) acc[j] = 0.f;
   int start = r0;
-  for (int r = r0; r < r1; ++r) {
-    const int key = keys[r];
-    if (key != skip) {
-      const float* xr = X + (int64_t)tok[r] * H;
-      float v[32];
+  for (int rb = r0; rb < r1; rb += 4) {
+    int kq[4];
+    float v[4][32];
 #pragma unroll
-      for (int j = 0; j < 32; ++j) v[j] = j < nv ? xr[lane + 32 * j] : 0.f;
+    for (int u = 0; u < 4; ++u) {
+      const int r = rb + u;
+      kq[u] = r < r1 ? keys[r] : skip;
+      const float* xr = X + (int64_t)(r < r1 ? tok[r] : 0) * H;
 #pragma unroll
-      for (int j = 0; j < 32; ++j) acc[j] += v[j];
+      for (int j = 0; j < 32; ++j) v[u][j] = (kq[u] != skip && j < nv) ? xr[lane + 32 * j] : 0.f;
     }
-    if (r + 1 == r1 || keys[r + 1] != key) {
+#pragma unroll
+    for (int u = 0; u < 4; ++u) {
+      const int r = rb + u;
+      if (r >= r1) break;
+      const int key = kq[u];
       if (key != skip) {
-        float* dst = X + (int64_t)tok[start] * H;
 #pragma unroll
-        for (int j = 0; j < 32; ++j)
-          if (j < nv) dst[lane + 32 * j] = acc[j];
+        for (int j = 0; j < 32; ++j) acc[j] += v[u][j];
       }
+      if (r + 1 == r1 || keys[r + 1] != key) {
+        if (key != skip) {
+          float* dst = X + (int64_t)tok[start] * H;
 #pragma unroll
-      for (int j = 0; j < 32; ++j) acc[j] = 0.f;
-      start = r + 1;
+          for (int j = 0; j < 32; ++j)
+            if (j < nv) dst[lane + 32 * j] = acc[j];
+        }
+#pragma unroll
+        for (int j = 0; j < 32; ++j) acc[j] = 0.f;
+        start = r + 1;
+      }
     }
   }
 }
