@@ -578,6 +578,11 @@ def main():
             lit, ms_l = arm(M_lit, batches, sched)
             lit.update(budget_bytes=M_lit, recompute_ratio=ms_l / ms_n,
                        rule="M = f x P(empty, x_max) (literal north_star reading)")
+            # the same tight budget with attention / FFN units planned by least
+            # recompute time (A30 + A31): what the finer units buy when half the layers must go
+            lk, ms_lk = arm(M_lit, batches, sched, granularity=0 if ed else 1, planner=mb.PLANNER_EXACT_TIME)
+            lk.update(recompute_ratio=ms_lk / ms_n, units=cfg.n_layers + cfg.n_dec_layers if ed else 2 * cfg.n_layers)
+            lit["knapsack_units" if not ed else "knapsack_layers"] = lk
             result["literal_budget"] = lit
         else:
             result["literal_budget"] = {"infeasible": True, "budget_bytes": M_lit, "lower_bound": LB}
