@@ -492,7 +492,8 @@ def main():
                    "budget_bytes": M, "persistent_bytes": C0, "no_ckpt_peak_at_max": P0,
                    "lower_bound_at_max": LB, "parallelism": f"dp{world}",
                    "l2": "no flush: per-step working set (weights+grads+optimizer >= 1.9 GB, activations) >> 126 MB L2",
-                   "gemm": "tcgen05" if tc else "simt"},
+                   "gemm": "tcgen05" if tc else "simt", "p_drop": cfg.p_drop,
+                   **({"p_drop_override": True} if args.p_drop is not None else {})},
         "tokens": {"mean_seq_pad": mean_s, "padded_tokens_per_s": tok_pad * world / (ms / 1000.0),
                    "valid_tokens_per_s": tok_valid * world / (ms / 1000.0),
                    "valid_fraction": tok_valid / tok_pad},
