@@ -3,16 +3,19 @@ CUDA events on the launching stream) by (N, K, epi): launches, share of the
 GEMM time, mean M, achieved TFLOP/s.  Grouped weight-gradient launches are
 (T, N1 K1 + N2 K2, tile width, -1).
 
-usage: python tools/probe_summary.py probe.csv [peak_tflops]
+usage: python tools/probe_summary.py probe.csv [peak_tflops]   (default: MEASURED_PEAKS.json bf16_tflops)
 """
 import collections
+import json
+import os
 import sys
 
 EPI = {0: "store", 1: "bias", 2: "bias+gelu", 3: "bias+drop+res", 4: "gelu'", 5: "acc+res f32", 6: "f32",
        8: "bias+gelu_tanh", 9: "gelu_tanh'", 10: "bias+drop+res f32", 11: "acc f32", -1: "grouped wgrad"}
 
 rows = [tuple(float(x) for x in ln.split(",")) for ln in open(sys.argv[1]) if ln.strip()]
-peak = float(sys.argv[2]) if len(sys.argv) > 2 else 1650.0
+_mp = os.path.join(os.path.dirname(os.path.dirname(os.path.abspath(__file__))), "MEASURED_PEAKS.json")
+peak = float(sys.argv[2]) if len(sys.argv) > 2 else (json.load(open(_mp))["bf16_tflops"] if os.path.exists(_mp) else 1650.0)
 agg = collections.defaultdict(lambda: [0, 0.0, 0.0, 0.0])   # n, us, flops, sum M
 for M, N, K, e, us in rows:
     key = (int(N), int(K), int(e))
