@@ -99,7 +99,12 @@ for s, es in sorted(by_stream.items(), key=lambda x: -len(x[1])):
     print(f"# stream {s}{' (compute)' if s == main else ''}: {len(es) / steps:.0f} kernels/step, "
           f"busy {union(es) / span:.3f} of the span")
 print(f"# all streams: busy {union(ev) / span:.3f} of the span")
-nm = lambda e: re.sub(r"\(.*", "", e["name"]).replace("void mimose::", "").replace("mimose::", "")[:60]
+def nm(e):   # the kernel name without its argument list (names may start with "(anonymous namespace)::")
+    n = e["name"].replace("(anonymous namespace)::", "").replace("void ", "").replace("mimose::", "")
+    return re.sub(r"\(.*", "", n)[:60]
+
+
+
 inc, gap = collections.defaultdict(lambda: [0, 0.0]), collections.defaultdict(lambda: [0, 0.0])
 m = sorted(by_stream[main], key=lambda e: e["ts"])
 front = m[0]["ts"]
