@@ -151,8 +151,8 @@ __global__ void __launch_bounds__(LTH, 2) k_attn_fwd_tcl(const __grid_constant__
     tma_load_2d(&tk, &bar[1], sK, a.kcol + hd * LD, krow0);
   }
   int ph_s = 0, ph_o = 0;
-  // ---- pass 1: exact row max and sum (log2 domain) ----
-  float m = -INFINITY, l = 0.f;
+  // ---- pass 1: exact row max (the sum is taken in pass 2 from the same exponentials) ----
+  float m = -INFINITY;
   for (int j = 0; j < nkt; ++j) {
     if (threadIdx.x == 0) {
       const int bf = j & 1;
@@ -176,26 +176,20 @@ __global__ void __launch_bounds__(LTH, 2) k_attn_fwd_tcl(const __grid_constant__
       float v[16];
       tmem_ld16(trow + 64 * hf + 16 * c, v);
       const int kb = j * LQ + 64 * hf + 16 * c;
+      if (kb < kl) {
 #pragma unroll
-      for (int i = 0; i < 16; ++i) {
-        if (kb + i < kl) {
-          const float s = v[i] * sl2;
-          if (s > m) { l = l * ex2a(m - s) + 1.f; m = s; } else { l += ex2a(s - m); }
-        }
+        for (int i = 0; i < 16; ++i)
+          if (kb + i < kl) m = fmaxf(m, v[i]);
       }
     }
     bar_sync_all();                             // S read before the next MMA overwrites it
   }
   red[hf * 128 + t] = m;
-  red[256 + hf * 128 + t] = l;
   __syncthreads();
-  const float m0 = red[t], m1 = red[128 + t];
-  const float M = fmaxf(m0, m1);
-  const float lt = (m0 == -INFINITY ? 0.f : red[256 + t] * ex2a(m0 - M)) +
-                   (m1 == -INFINITY ? 0.f : red[384 + t] * ex2a(m1 - M));
-  const float L2 = M + __log2f(lt);             // log2-domain LSE of s * scale
+  const float M = fmaxf(red[t], red[128 + t]) * sl2;   // log2-domain row max of s * scale
   const uint64_t ebase = (((uint64_t)b * a.h + hd) * S + (uint64_t)q) * Sk;
-  // ---- pass 2: P~ = exp(S - LSE) * dropout, O += P~ V ----
+  float l = 0.f;                                // this half's sum of exp(s - max), fp32, before dropout
+  // ---- pass 2: P~ = exp(S - max) * dropout (unnormalised), O += P~ V; O / l in the epilogue ----
   if (threadIdx.x == 0 && nkt > 0) {            // every pass-1 MMA is done (bar[2] waited)
     mbar_expect_tx(&bar[1], LT);
     tma_load_2d(&tk, &bar[1], sK, a.kcol + hd * LD, krow0);
@@ -230,8 +224,11 @@ __global__ void __launch_bounds__(LTH, 2) k_attn_fwd_tcl(const __grid_constant__
           const float4 f = k < kl ? drop4l(a.drop, ebase + k) : make_float4(0.f, 0.f, 0.f, 0.f);
           const float ff[4] = {f.x, f.y, f.z, f.w};
 #pragma unroll
-          for (int i = 0; i < 4; ++i)
-            v[4 * g + i] = (k + i < kl) ? ex2a(fmaf(v[4 * g + i], sl2, -L2)) * ff[i] : 0.f;
+          for (int i = 0; i < 4; ++i) {
+            const float p = (k + i < kl) ? ex2a(fmaf(v[4 * g + i], sl2, -M)) : 0.f;
+            l += p;
+            v[4 * g + i] = p * ff[i];
+          }
         }
       } else {
 #pragma unroll
@@ -257,13 +254,16 @@ __global__ void __launch_bounds__(LTH, 2) k_attn_fwd_tcl(const __grid_constant__
       tma_load_2d(&tk, &bar[5], sV, a.vcol + hd * LD, krow0 + (j + 1) * LQ);
     }
   }
-  {  // epilogue: half hf stores dims [32hf, 32hf + 32) of row q
+  red[256 + hf * 128 + t] = l;                 // row sum: half 0 + half 1, fixed order
+  __syncthreads();
+  const float lt = red[256 + t] + red[384 + t];
+  const float L2 = M + __log2f(lt);             // log2-domain LSE of s * scale (what the backward reads)
+  {  // epilogue: half hf stores dims [32hf, 32hf + 32) of row q, O = (P~ V) / l
     float v[32];
     tmem_ld32(trow + 128 + 32 * hf, v);
-    if (nkt == 0) {
+    const float inv = (nkt > 0 && lt > 0.f) ? 1.0f / lt : 0.f;
 #pragma unroll
-      for (int i = 0; i < 32; ++i) v[i] = 0.f;
-    }
+    for (int i = 0; i < 32; ++i) v[i] *= inv;
     if (q < S) {
       st_bf16x32(a.Oout + ((int64_t)row0 + q) * a.H + hd * LD + 32 * hf, v);
       if (hf == 0) a.lse[((int64_t)b * a.h + hd) * S + q] = L2 * 0.69314718055994531f;
